@@ -1,0 +1,382 @@
+"""Synthetic symbolic programs: an Ansor-like GPU multi-level-tiling sketch of a tensor contraction
+and the closed-form feature formulas of the tiled program (SUPPORT for the hot path).
+
+PAPER.md §3.2-3.3 (L522-679): Felix applies a symbolic schedule s* (Tile / Annotation(blockIdx,
+vthread, threadIdx) / CacheRead / Unroll with variable parameters, Fig. 3) to the subgraph
+and extracts 82 feature formulas Feat_k(x) from the symbolic program.  Felix's real extractor needs
+TVM (out of scope); this module builds the same *kind* of formulas for a fixed
+sketch whose concrete loop nest is simple enough that every feature has an independent brute-force
+definition (tests/sim/loopnest.py enumerates the concrete nest and must reproduce each formula
+exactly at every valid integer point — the O-pin-1 check).
+
+Sketch (per spatial axis i with extent E_i, per reduction axis j with extent K_j):
+    blockIdx  b_i in [0, E_i / (V_i T_i I_i))          (fused over i)
+      vthread   v_i in [0, V_i)
+      threadIdx t_i in [0, T_i)
+        for ro_j in [0, K_j / Rt_j)                      # outer reduction, CacheRead tiles per ro
+          for rm_j in [0, RI1_j)          (2-var reduction axes only)
+            for v_i ...                                  # vthread loop (virtual threads)
+              for ri_j in [0, RI2_j | RI_j | K_j)
+                for in_i in [0, I_i)
+                  O[s] += A[...] * B[...]
+    s_i = b_i*(V_i T_i I_i) + v_i*(T_i I_i) + t_i*I_i + in_i
+    r_j = ro_j*Rt_j + rm_j*RI2_j + ri_j            (Rt_j = product of the axis' tile vars, or K_j)
+Per-thread loop list L (outer -> inner): ro_*, rm_*, v_*, ri_*, in_*.
+"""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass, field
+from typing import Dict, List, Optional, Sequence, Tuple
+
+import numpy as np
+
+from .dag import (DagBuilder, Space, Split, Var, VAR_INT, VAR_SPLIT, prune)
+
+N_FEATURES = 82          # "a total of 82 distinct features"
+UNROLL_MAX = 1024        # Unroll(max_step=UNROLL0), Fig. 3 L584 / L599; search range [1, 1024]
+
+
+@dataclass
+class SAxis:
+    name: str
+    extent: int
+    levels: str = "vti"      # which of vthread / thread / inner are schedule variables
+
+
+@dataclass
+class RAxis:
+    name: str
+    extent: int
+    n_vars: int = 1          # 0: fully inner, 1: (outer, RI), 2: (outer, RI1, RI2)
+
+
+@dataclass
+class Buffer:
+    name: str
+    dims: List[List[Tuple[str, int]]]   # each dim: sum of coeff * axis_index
+
+
+@dataclass
+class ProgramSpec:
+    name: str
+    spatial: List[SAxis]
+    reduction: List[RAxis]
+    inputs: List[Buffer]
+    bias: bool = False
+    relu: bool = False
+    gelu: bool = False
+    unroll: bool = True
+    smem_limit: int = 48 * 1024
+    thread_limit: int = 1024
+    local_limit: int = 256
+    vthread_limit: int = 64
+
+    def axis_extent(self, name: str) -> int:
+        for a in self.spatial:
+            if a.name == name:
+                return a.extent
+        for a in self.reduction:
+            if a.name == name:
+                return a.extent
+        raise KeyError(name)
+
+    def is_spatial(self, name: str) -> bool:
+        return any(a.name == name for a in self.spatial)
+
+    def buffer_shape(self, buf: Buffer) -> List[int]:
+        shape = []
+        for dim in buf.dims:
+            shape.append(sum(c * (self.axis_extent(a) - 1) for a, c in dim) + 1 if dim else 1)
+        return shape
+
+
+# ------------------------------------------------------------------------------ variable layout
+def var_layout(spec: ProgramSpec) -> Tuple[List[Var], List[Split], Dict[str, int]]:
+    """Variables in a fixed order: per spatial axis V,T,I (as present), per reduction axis RI1,RI2
+    (or RI), then UNROLL.  Each axis' vars form one divisibility split of its extent (L791-797)."""
+    vars_: List[Var] = []
+    splits: List[Split] = []
+    index: Dict[str, int] = {}
+    for ax in spec.spatial:
+        ids = []
+        for lv, tag in (("v", "V"), ("t", "T"), ("i", "I")):
+            if lv in ax.levels:
+                index[f"{tag}_{ax.name}"] = len(vars_)
+                ids.append(len(vars_))
+                vars_.append(Var(f"{tag}_{ax.name}", VAR_SPLIT, 1, ax.extent))
+        if ids:
+            splits.append(Split(ax.extent, ids))
+    for ax in spec.reduction:
+        ids = []
+        names = [] if ax.n_vars == 0 else ([f"RI_{ax.name}"] if ax.n_vars == 1 else [f"RI1_{ax.name}", f"RI2_{ax.name}"])
+        for nm in names:
+            index[nm] = len(vars_)
+            ids.append(len(vars_))
+            vars_.append(Var(nm, VAR_SPLIT, 1, ax.extent))
+        if ids:
+            splits.append(Split(ax.extent, ids))
+    if spec.unroll:
+        index["UNROLL"] = len(vars_)
+        vars_.append(Var("UNROLL", VAR_INT, 1, UNROLL_MAX))
+    return vars_, splits, index
+
+
+# ------------------------------------------------------------------------------ feature formulas
+class _Ctx:
+    def __init__(self, spec: ProgramSpec, b: DagBuilder, index: Dict[str, int]):
+        self.spec, self.b, self.index = spec, b, index
+
+    def v(self, name: str) -> int:
+        """Node for var `name`, or constant 1 if the level is not a schedule variable."""
+        j = self.index.get(name)
+        return self.b.var(j) if j is not None else self.b.const(1.0)
+
+    # spatial axis quantities
+    def V(self, ax: SAxis) -> int: return self.v(f"V_{ax.name}")
+    def T(self, ax: SAxis) -> int: return self.v(f"T_{ax.name}")
+    def I(self, ax: SAxis) -> int: return self.v(f"I_{ax.name}")
+
+    def Tb(self, ax: SAxis) -> int:
+        return self.b.prod([self.V(ax), self.T(ax), self.I(ax)])
+
+    def Nb(self, ax: SAxis) -> int:
+        return self.b.div(self.b.const(ax.extent), self.Tb(ax))
+
+    # reduction axis quantities
+    def red_levels(self, ax: RAxis) -> Tuple[Optional[int], int]:
+        """(rm extent node or None, ri extent node)."""
+        if ax.n_vars == 0:
+            return None, self.b.const(ax.extent)
+        if ax.n_vars == 1:
+            return None, self.v(f"RI_{ax.name}")
+        return self.v(f"RI1_{ax.name}"), self.v(f"RI2_{ax.name}")
+
+    def Rt(self, ax: RAxis) -> int:
+        rm, ri = self.red_levels(ax)
+        return ri if rm is None else self.b.mul(rm, ri)
+
+    def Ro(self, ax: RAxis) -> int:
+        return self.b.div(self.b.const(ax.extent), self.Rt(ax))
+
+    def loops(self) -> List[Tuple[str, int, str, int]]:
+        """Per-thread loop list L (outer -> inner): (kind, extent node, axis name, step node)."""
+        b, out = self.b, []
+        for ax in self.spec.reduction:
+            out.append(("ro", self.Ro(ax), ax.name, self.Rt(ax)))
+        for ax in self.spec.reduction:
+            rm, ri = self.red_levels(ax)
+            if rm is not None:
+                out.append(("rm", rm, ax.name, ri))
+        for ax in self.spec.spatial:
+            out.append(("v", self.V(ax), ax.name, b.mul(self.T(ax), self.I(ax))))
+        for ax in self.spec.reduction:
+            _, ri = self.red_levels(ax)
+            out.append(("ri", ri, ax.name, b.const(1.0)))
+        for ax in self.spec.spatial:
+            out.append(("in", self.I(ax), ax.name, b.const(1.0)))
+        return out
+
+
+def _dim_footprint(ctx: _Ctx, dim: List[Tuple[str, int]], scope: str) -> int:
+    """Distinct values of one buffer index dim  sum(coeff * axis)  touched by block 0 / thread 0
+    during the first outer-reduction iteration (ro = 0 for every reduction axis)."""
+    b, spec = ctx.b, ctx.spec
+    if not dim:
+        return b.const(1.0)
+    sp = [(a, c) for a, c in dim if spec.is_spatial(a)]
+    rd = [(a, c) for a, c in dim if not spec.is_spatial(a)]
+    assert len(sp) <= 1 and len(rd) <= 1, "index dims combine at most one spatial + one reduction axis"
+    if not sp:
+        (a, c), = rd
+        assert c == 1
+        ax = next(x for x in spec.reduction if x.name == a)
+        return ctx.Rt(ax)
+    (sa, c), = sp
+    ax = next(x for x in spec.spatial if x.name == sa)
+    if not rd:
+        # spatial only: block covers a contiguous run of Tb; thread covers V runs of I (stride T*I)
+        return ctx.Tb(ax) if scope == "block" else b.mul(ctx.V(ax), ctx.I(ax))
+    (ra, rc), = rd
+    rax = next(x for x in spec.reduction if x.name == ra)
+    assert rax.n_vars == 0 and rc == 1, "halo dims use an unsplit reduction axis"
+    R = rax.extent
+    run = ctx.Tb(ax) if scope == "block" else ctx.I(ax)
+    if c > R:   # index c*s + r with r < R < c: all (s, r) pairs distinct, runs never overlap
+        n = run if scope == "block" else b.mul(ctx.V(ax), run)
+        return b.mul(n, b.const(R))
+    # one run of s of length n gives the interval [c*s0, c*(s0+n-1)+R): length c*(n-1)+R
+    L = b.add(b.mul(b.const(c), b.sub(run, b.const(1.0))), b.const(R))
+    if scope == "block":
+        return L
+    # thread: V intervals of length L with stride S = c*T*I; union = V*L - (V-1)*max(0, L-S)
+    S = b.mul(b.const(c), b.mul(ctx.T(ax), ctx.I(ax)))
+    V = ctx.V(ax)
+    overlap = b.max(b.const(0.0), b.sub(L, S))
+    return b.sub(b.mul(V, L), b.mul(b.sub(V, b.const(1.0)), overlap))
+
+
+def _linear_stride(spec: ProgramSpec, buf: Buffer, axis: str) -> int:
+    """Address delta (elements, row-major buffer) when `axis` index increases by 1."""
+    shape = spec.buffer_shape(buf)
+    pitch = [int(np.prod(shape[d + 1:])) for d in range(len(shape))]
+    return sum(pitch[d] * c for d, dim in enumerate(buf.dims) for a, c in dim if a == axis)
+
+
+def build_space(spec: ProgramSpec) -> Space:
+    vars_, splits, index = var_layout(spec)
+    b = DagBuilder()
+    ctx = _Ctx(spec, b, index)
+    feats: List[Tuple[str, int]] = []
+
+    E = [ax.extent for ax in spec.spatial]
+    Kx = [ax.extent for ax in spec.reduction]
+    prodE = float(np.prod(E))
+    nmac = float(np.prod(E) * np.prod(Kx))
+    NB = b.prod([ctx.Nb(ax) for ax in spec.spatial])
+    NT = b.prod([ctx.T(ax) for ax in spec.spatial])
+    NV = b.prod([ctx.V(ax) for ax in spec.spatial])
+    out_per_thread = b.prod([b.mul(ctx.V(ax), ctx.I(ax)) for ax in spec.spatial])
+    stmts_per_thread = b.div(b.const(nmac), b.mul(NB, NT))
+    ro_iters = b.prod([ctx.Ro(ax) for ax in spec.reduction])
+    loops = ctx.loops()
+    nontriv = [b.select(b.gt(ext, b.const(1.0)), b.const(1.0), b.const(0.0)) for _, ext, _, _ in loops]
+    n_nontriv = b.sum(nontriv)
+
+    # -- op counts / GPU mapping / loop structure
+    feats.append(("float_mad", b.const(nmac)))
+    feats.append(("float_addsub", b.const(prodE if spec.bias else 0.0)))
+    feats.append(("float_cmp", b.const(prodE if spec.relu else 0.0)))
+    feats.append(("float_math", b.const(prodE if spec.gelu else 0.0)))
+    feats.append(("blockIdx_len", NB))
+    feats.append(("vthread_len", NV))
+    feats.append(("threadIdx_len", NT))
+    feats.append(("outputs_per_thread", out_per_thread))
+    feats.append(("stmts_per_thread", stmts_per_thread))
+    feats.append(("n_nontrivial_loops", n_nontriv))
+    # paper's example shape: int_add = NMK * select(TILE0 > 1, 5, 2)  (L668-671)
+    feats.append(("int_addsub", b.mul(b.const(nmac), b.add(b.const(2.0), n_nontriv))))
+    n_block_axes = b.sum([b.select(b.gt(ctx.Nb(ax), b.const(1.0)), b.const(1.0), b.const(0.0)) for ax in spec.spatial])
+    feats.append(("int_mul", b.mul(b.const(nmac), n_block_axes)))
+    feats.append(("reduction_outer_iters", ro_iters))
+    per_ro = b.div(stmts_per_thread, ro_iters)
+    if spec.unroll:
+        U = ctx.v("UNROLL")
+        feats.append(("unroll_len", b.min(U, per_ro)))
+        cum, cnt = b.const(1.0), []
+        for _, ext, _, _ in reversed(loops):
+            cum = b.mul(cum, ext)
+            cnt.append(b.select(b.le(cum, U), b.const(1.0), b.const(0.0)))
+        feats.append(("unrolled_loops", b.sum(cnt)))
+    else:
+        feats.append(("unroll_len", b.const(0.0)))
+        feats.append(("unrolled_loops", b.const(0.0)))
+
+    # -- per-input-buffer memory features
+    gbytes = []
+    smem_elems = []
+    stmts_per_block_ro = b.div(b.mul(stmts_per_thread, NT), ro_iters)
+    for buf in spec.inputs:
+        blk = b.prod([_dim_footprint(ctx, d, "block") for d in buf.dims])
+        thr = b.prod([_dim_footprint(ctx, d, "thread") for d in buf.dims])
+        gl = b.mul(b.mul(NB, ro_iters), blk)
+        gb = b.mul(b.const(4.0), gl)
+        gbytes.append(gb)
+        smem_elems.append(blk)
+        # stride along the innermost non-trivial loop of L (0 if every loop is trivial)
+        stride = b.const(0.0)
+        for kind, ext, axn, step in loops:     # outer -> inner: the innermost wins
+            s = _linear_stride(spec, buf, axn)
+            d = b.mul(step, b.const(float(s)))
+            stride = b.select(b.gt(ext, b.const(1.0)), d, stride)
+        feats += [
+            (f"{buf.name}.block_footprint", blk),
+            (f"{buf.name}.global_load_elems", gl),
+            (f"{buf.name}.global_bytes", gb),
+            (f"{buf.name}.coop_loads_per_thread", b.ceildiv(blk, NT)),
+            (f"{buf.name}.thread_footprint", thr),
+            (f"{buf.name}.thread_reuse", b.div(per_ro, thr)),
+            (f"{buf.name}.block_reuse", b.div(stmts_per_block_ro, blk)),
+            (f"{buf.name}.global_reuse", b.div(b.const(nmac), gl)),
+            (f"{buf.name}.innermost_stride", stride),
+            (f"{buf.name}.shared_bytes", b.mul(b.const(4.0), blk)),
+        ]
+    smem_bytes = b.mul(b.const(4.0), b.sum(smem_elems))
+    feats += [
+        ("out.stores", b.const(prodE)),
+        ("shared_bytes_total", smem_bytes),
+        ("local_bytes", b.mul(b.const(4.0), out_per_thread)),
+        ("flops_per_global_byte", b.div(b.const(2.0 * nmac), b.add(b.sum(gbytes), b.const(4.0 * prodE)))),
+        ("flops_per_thread", b.mul(b.const(2.0), stmts_per_thread)),
+        ("global_bytes_per_block", b.div(b.sum(gbytes), NB)),
+    ]
+    assert len(feats) <= N_FEATURES
+    n_used = len(feats)
+    zero = b.const(0.0)
+    for k in range(N_FEATURES - n_used):   # annotation slots this sketch never produces
+        feats.append((f"reserved_{k}", zero))
+
+    # -- user constraints g(x) <= 0, in log form so lambda has a uniform scale (SURVEY O2 reading)
+    cons: List[Tuple[str, int]] = []
+    cons.append(("threads<=limit", b.sub(b.log(NT), b.const(math.log(spec.thread_limit)))))
+    cons.append(("smem<=limit", b.sub(b.log(smem_bytes), b.const(math.log(spec.smem_limit)))))
+    cons.append(("local<=limit", b.sub(b.log(b.mul(b.const(4.0), out_per_thread)), b.const(math.log(spec.local_limit * 4)))))
+    if any("v" in ax.levels for ax in spec.spatial):
+        cons.append(("vthreads<=limit", b.sub(b.log(NV), b.const(math.log(spec.vthread_limit)))))
+
+    nodes = b.nodes()
+    nodes, (froots, croots) = prune(nodes, [np.array([f for _, f in feats], dtype=np.int32),
+                                             np.array([c for _, c in cons], dtype=np.int32)])
+    return Space(spec.name, vars_, splits, nodes, froots, croots,
+                 [n for n, _ in feats], [n for n, _ in cons], spec)
+
+
+# ------------------------------------------------------------------------------ concrete workloads
+def dense_spec(name: str, N: int, M: int, K: int, *, i_levels="ti", j_levels="ti", k_vars=1,
+               bias=True, relu=False, gelu=False, batch: int = 0) -> ProgramSpec:
+    """O[i, j] += A[i, k] * B[k, j]  (Dense / Dense-Add, Fig. 3).  batch > 0 adds a leading
+    spatial axis b (bmm): A[b, i, k], B[b, k, j]."""
+    spatial = [SAxis("i", N, i_levels), SAxis("j", M, j_levels)]
+    a_dims = [[("i", 1)], [("k", 1)]]
+    b_dims = [[("k", 1)], [("j", 1)]]
+    if batch:
+        spatial = [SAxis("b", batch, "t")] + spatial
+        a_dims = [[("b", 1)]] + a_dims
+        b_dims = [[("b", 1)]] + b_dims
+    return ProgramSpec(name, spatial, [RAxis("k", K, k_vars)],
+                       [Buffer("A", a_dims), Buffer("B", b_dims)], bias=bias, relu=relu, gelu=gelu)
+
+
+def conv2d_spec(name: str, C: int, H: int, W: int, K: int, R: int, S: int, stride: int = 1, *,
+                co_levels="vti", h_levels="vti", w_levels="vti", rc_vars=2, bias=True, relu=True) -> ProgramSpec:
+    """O[co, h, w] += In[rc, stride*h + rh, stride*w + rw] * Wt[co, rc, rh, rw] (batch 1, input
+    pre-padded), H, W = output sizes."""
+    spatial = [SAxis("co", K, co_levels), SAxis("h", H, h_levels), SAxis("w", W, w_levels)]
+    red = [RAxis("rc", C, rc_vars), RAxis("rh", R, 0), RAxis("rw", S, 0)]
+    inp = Buffer("In", [[("rc", 1)], [("h", stride), ("rh", 1)], [("w", stride), ("rw", 1)]])
+    wt = Buffer("Wt", [[("co", 1)], [("rc", 1)], [("rh", 1)], [("rw", 1)]])
+    return ProgramSpec(name, spatial, red, [inp, wt], bias=bias, relu=relu)
+
+
+def paper_dense_add_s1(N: int = 64, M: int = 64, K: int = 64) -> Space:
+    """The paper's worked example, symbolic schedule s*_1 of Dense-Add (Fig. 3) with
+    variables TILE0 (tiles both M and K, L579-581) and UNROLL0, and exactly the three feature
+    formulas printed at L668-671:  float_add = N*M*K,  blockIdx_len = N*M/TILE0,
+    int_add = NMK * select(TILE0 > 1, 5, 2);  constraint c11 = (1 <= TILE0 <= K) as the penalty
+    functions g11 = 1 - TILE0, g12 = TILE0 - K (L786-788).  Remaining feature slots are zero."""
+    b = DagBuilder()
+    t = b.var(0)
+    nmk = b.const(float(N * M * K))
+    f_add = nmk
+    f_blk = b.div(b.const(float(N * M)), t)
+    f_int = b.mul(nmk, b.select(b.gt(t, b.const(1.0)), b.const(5.0), b.const(2.0)))
+    zero = b.const(0.0)
+    feats = [f_add, f_blk, f_int] + [zero] * (N_FEATURES - 3)
+    g11 = b.sub(b.const(1.0), t)
+    g12 = b.sub(t, b.const(float(K)))
+    nodes = b.nodes()
+    nodes, (fr, cr) = prune(nodes, [np.array(feats, dtype=np.int32), np.array([g11, g12], dtype=np.int32)])
+    vars_ = [Var("TILE0", VAR_SPLIT, 1, min(M, K)), Var("UNROLL0", VAR_INT, 1, UNROLL_MAX)]
+    splits = [Split(M, [0]), Split(K, [0])]
+    names = ["float_add", "blockIdx_len", "int_add"] + [f"reserved_{k}" for k in range(N_FEATURES - 3)]
+    return Space("paper_dense_add_s1", vars_, splits, nodes, fr, cr, names, ["g11", "g12"], None)
