@@ -1,0 +1,206 @@
+/* felix.h — C ABI of the B200-native Felix hot path (batched differentiable schedule search).
+ *
+ * Paper: Zhao, Sharif, Adve, Misailovic, "Felix: Optimizing Tensor Programs with Gradient Descent",
+ * ASPLOS'24 (/root/reference/PAPER.md, cited "P:Lnnn").  The four primary calls follow the paper's
+ * statement of the problem, Algorithm 1:
+ *   felix_space_create    — one symbolic schedule s*_i: variables x_i, feature formulas Feat_k(x_i),
+ *                           constraints g_ir(x_i) <= 0, divisibility splits
+ *   felix_costmodel_load  — the pretrained MLP cost model C
+ *   felix_search          — lines 12-19: init, then nSteps Adam steps on Eq. 4
+ *   felix_round_topk      — lines 20-21: round to valid integer schedules, score, top-nMeasure
+ *
+ * plus test hooks (felix_eval, felix_round, felix_score, felix_init_sample) that run the same kernels.
+ *
+ * Conventions (all calls):
+ *  - No exceptions cross the ABI.  Every call returns felix_status; on error felix_last_error()
+ *    (thread-local, valid until the next felix_* call on this thread) describes it.  Argument and
+ *    shape validation happens before any launch; a failed call leaves caller buffers untouched
+ *    except where stated.
+ *  - Handles are opaque and library-owned; *_destroy frees them (NULL is a no-op).
+ *  - Host input arrays are COPIED at create/load time; the caller may free them on return.
+ *  - "device" pointers are caller-owned CUDA device memory on the handle's device (e.g. torch
+ *    tensors' data_ptr()); the library never frees them.  "host" pointers are ordinary host memory.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).  Calls enqueue work
+ *    on it and return, except felix_round_topk, which synchronises `stream` because its outputs are
+ *    host arrays.  Calls on one space must not run concurrently (the space owns its workspace).
+ *  - Layouts: candidate-major SoA for per-candidate vectors: y[j * n + i] = y_j of candidate i.
+ *  - The global index of local candidate i is index_base + i; it seeds the sampler and breaks top-k
+ *    ties, which makes results invariant to how candidates are sharded over GPUs.
+ *  - There is no CPU fallback: without a usable sm_100a device every call that needs one returns
+ *    FELIX_E_CUDA.
+ */
+#ifndef FELIX_H_
+#define FELIX_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define FELIX_ABI_VERSION 1
+
+#if defined(__GNUC__)
+#define FELIX_EXPORT __attribute__((visibility("default")))
+#else
+#define FELIX_EXPORT
+#endif
+
+typedef enum {
+  FELIX_OK = 0,
+  FELIX_E_INVALID_ARG = 1,   /* NULL / out-of-range argument                                   */
+  FELIX_E_INVALID_DAG = 2,   /* node args not topological, bad opcode, type error (BOOL vs NUM) */
+  FELIX_E_SHAPE = 3,         /* sizes inconsistent (e.g. n_features != cost-model dims[0])      */
+  FELIX_E_UNSUPPORTED = 4,   /* valid but outside this build (e.g. hidden dim % 64 != 0)        */
+  FELIX_E_CUDA = 5,          /* CUDA runtime/driver error or no sm_100 device                   */
+  FELIX_E_NVRTC = 6,         /* run-time compilation of the space's expression kernels failed   */
+  FELIX_E_OOM = 7            /* device allocation failed                                        */
+} felix_status;
+
+FELIX_EXPORT const char* felix_last_error(void);
+FELIX_EXPORT int32_t felix_abi_version(void);
+
+/* ---------------------------------------------------------------- feature-expression DAG
+ * "each feature expression ... can only contain schedule variables, constants, and a
+ * fixed set of operators ... +, -, *, /, pow, min, max, select, etc."  Nodes are given in
+ * topological order; a, b, c index EARLIER nodes.  Values are NUM (real) or BOOL (comparisons and
+ * logic).  Semantics used by the search ("smooth", reading O3 of DESIGN.md, with
+ * S(t) = 1/2(1 + t/sqrt(1+t^2)) and R(t) = 1/2(t + sqrt(1+t^2))):
+ *   MIN(a,b) = a - R(a-b)      MAX(a,b) = b + R(a-b)
+ *   GT/GE(a,b) = S(a-b)        LT/LE(a,b) = S(b-a)      EQ = S(a-b+1/2) S(b-a+1/2)   NE = 1 - EQ
+ *   AND = p q   OR = p + q - p q   NOT = 1 - p          SELECT(c,a,b) = b + (a-b) c
+ *   FLOORDIV / CEILDIV(a,b) = a / b
+ * and at integer points ("hard", used for validity and scoring): exact comparisons, SELECT picks a
+ * branch, floor/ceil division.  VAR: imm = variable index j, value x_j = exp(y_j).
+ * POW: a ^ imm (unary).  CONST: imm. */
+typedef enum {
+  FELIX_OP_CONST = 0, FELIX_OP_VAR = 1, FELIX_OP_ADD = 2, FELIX_OP_SUB = 3, FELIX_OP_MUL = 4,
+  FELIX_OP_DIV = 5, FELIX_OP_NEG = 6, FELIX_OP_POW = 7, FELIX_OP_EXP = 8, FELIX_OP_LOG = 9,
+  FELIX_OP_SQRT = 10, FELIX_OP_MIN = 11, FELIX_OP_MAX = 12, FELIX_OP_SELECT = 13,
+  FELIX_OP_GT = 14, FELIX_OP_GE = 15, FELIX_OP_LT = 16, FELIX_OP_LE = 17, FELIX_OP_EQ = 18,
+  FELIX_OP_NE = 19, FELIX_OP_AND = 20, FELIX_OP_OR = 21, FELIX_OP_NOT = 22,
+  FELIX_OP_FLOORDIV = 23, FELIX_OP_CEILDIV = 24
+} felix_op;
+
+typedef struct { int32_t op, a, b, c; double imm; } felix_node;          /* 24 bytes */
+
+/* Schedule variables (thread/block sizes, tile sizes, vector sizes, unroll factors;
+ * "a size/factor of value 1 [is] a no-op").  SPLIT: a tiling factor x >= 1 whose products over each
+ * split it belongs to divide the split's extent.  INT: an integer lo <= x <= hi. */
+typedef enum { FELIX_VAR_SPLIT = 0, FELIX_VAR_INT = 1 } felix_var_kind;
+typedef struct { int32_t kind; int32_t _pad; int64_t lo, hi; } felix_var;   /* 24 bytes */
+typedef struct { int64_t extent; int32_t n; int32_t _pad; const int32_t* vars; } felix_split;
+
+typedef struct felix_space felix_space;
+typedef struct felix_costmodel felix_costmodel;
+
+/* Creates a search space on `device`.
+ * vars[n_vars], splits[n_splits] (each SPLIT var in >= 1 split; extents in [1, 2^31)),
+ * nodes[n_nodes], feature_roots[n_features] (NUM nodes; n_features must equal the cost model's
+ * dims[0] at search time), constraint_roots[n_constraints] (NUM nodes, user g_r(x) <= 0).
+ * The library appends the automatic log-space validity roots (reading O2), in this order
+ * after the user roots:  -y_j for every SPLIT var;  sum_{j in s} y_j - ln(extent_s) per split;
+ * ln(lo_j) - y_j and y_j - ln(hi_j) per INT var.  R = total number of roots (felix_space_info).
+ * Builds the divisor-tuple tables of every split component, generates straight-line CUDA for the
+ * DAG (forward, reverse, hard, sampler) and compiles it for sm_100a with NVRTC. */
+FELIX_EXPORT felix_status felix_space_create(int device,
+                                const felix_var* vars, int32_t n_vars,
+                                const felix_split* splits, int32_t n_splits,
+                                const felix_node* nodes, int32_t n_nodes,
+                                const int32_t* feature_roots, int32_t n_features,
+                                const int32_t* constraint_roots, int32_t n_constraints,
+                                felix_space** out);
+FELIX_EXPORT void felix_space_destroy(felix_space* s);
+
+/* Device-free check of a space description: validates it exactly like felix_space_create, generates
+ * the space's CUDA source and, if compile != 0, compiles it with NVRTC for sm_100a (no GPU needed).
+ * Copies up to src_cap bytes of source (NUL-terminated when it fits) into src (may be NULL) and
+ * stores the full length in *src_len (may be NULL). */
+FELIX_EXPORT felix_status felix_codegen(const felix_var* vars, int32_t n_vars,
+                                        const felix_split* splits, int32_t n_splits,
+                                        const felix_node* nodes, int32_t n_nodes,
+                                        const int32_t* feature_roots, int32_t n_features,
+                                        const int32_t* constraint_roots, int32_t n_constraints,
+                                        int32_t compile, char* src, int64_t src_cap, int64_t* src_len);
+
+typedef struct {
+  int32_t n_vars, n_nodes, n_features, n_constraints_user, n_roots_total, n_components;
+  int64_t n_tuples_total;       /* rows of the divisor-tuple tables                            */
+  double nvrtc_ms;              /* time spent compiling the generated kernels                  */
+  int32_t regs_fwd, regs_rev;   /* registers/thread of the generated forward / reverse kernels  */
+  int64_t dag_flops_fwd;        /* arithmetic ops in one forward evaluation (per candidate)    */
+} felix_space_info_t;
+FELIX_EXPORT felix_status felix_space_info(const felix_space* s, felix_space_info_t* out);
+
+/* Loads the cost model C: n_layers linear layers, dims[n_layers+1], dims[n_layers] == 1,
+ * W[l] host row-major [dims[l+1]][dims[l]] fp32, b[l] host [dims[l+1]] fp32; ReLU between layers,
+ * none after the last (TenSet MLP).  Hidden dims must be multiples of 64 and <= 4096,
+ * dims[0] <= 256.  Weights are split on the host into fp16 hi/lo pairs for the tensor cores
+ * and kept in fp64 for scoring. */
+FELIX_EXPORT felix_status felix_costmodel_load(int device, int32_t n_layers, const int32_t* dims,
+                                  const float* const* W, const float* const* b, felix_costmodel** out);
+FELIX_EXPORT void felix_costmodel_destroy(felix_costmodel* m);
+
+/* Algorithm 1 lines 12-19.  n_seeds candidates (nSeeds) x n_steps Adam steps (nSteps).
+ * Per candidate the objective is Eq. 4:  L = -C(slog(Feat(e^y))) + lambda * sum_r max(g_r, 0)^2
+ * (slog(F) = sign(F) log2(1+|F|), reading O4), differentiated w.r.t. y, then one torch.optim.Adam
+ * step (bias-corrected, no weight decay) on y.  A candidate whose loss or gradient is
+ * non-finite is not updated that step (reading R-NaN).
+ * y: device fp32 SoA [n_vars][n_seeds].  If init_from_y == 0 it is OUTPUT-only and first filled by
+ * the rejection sampler (felix_init_sample with rng_seed / index_base); else it is the start point.
+ * final_loss: device fp32 [n_seeds] or NULL — the loss at the point of the last step's evaluation. */
+typedef struct {
+  int64_t n_seeds;
+  int32_t n_steps;
+  float lr, beta1, beta2, eps, lambda;   /* reading O8 defaults: 0.05, 0.9, 0.999, 1e-8, 1.0 */
+  uint64_t rng_seed;
+  int32_t init_from_y;
+  int32_t _pad;
+  int64_t index_base;
+} felix_search_params;
+FELIX_EXPORT felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search_params* p,
+                          float* y, float* final_loss, void* stream);
+
+/* Algorithm 1 lines 20-21 on the n relaxed points y (device SoA
+ * [n_vars][n]): round every point (reading O10: per split component the divisor tuple nearest in
+ * log space, ties to the lexicographically smallest; INT vars to the nearest integer), drop invalid
+ * points (hard semantics, all user g_r <= 1e-9, finite), score C(slog(Feat_hard(x))) in FP64, drop
+ * duplicate schedules (keep the smallest global index), return the best k by (score desc, global
+ * index asc).  Outputs are HOST arrays: idx_out[k] global indices, score_out[k], sched_out[k][n_vars];
+ * *n_out = number filled (<= k).  Synchronises `stream`. */
+FELIX_EXPORT felix_status felix_round_topk(felix_space* s, felix_costmodel* m, const float* y, int64_t n,
+                              int64_t index_base, int32_t k, int64_t* idx_out, double* score_out,
+                              int32_t* sched_out, int32_t* n_out, void* stream);
+
+/* ---------------------------------------------------------------- test hooks (same kernels)
+ * felix_eval: one objective + gradient evaluation, no Adam.  y device [n_vars][n].  Outputs (device,
+ * any may be NULL): phi [n_features][n] (slog features), g [R][n] (user roots then automatic roots),
+ * cost [n] (C, higher = better), loss [n], grad [n_vars][n] (dL/dy). */
+FELIX_EXPORT felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int64_t n, float lambda,
+                        float* phi, float* g, float* cost, float* loss, float* grad, void* stream);
+/* Rounding + validity only: sched device int32 [n][n_vars], valid device uint8 [n]. */
+FELIX_EXPORT felix_status felix_round(felix_space* s, const float* y, int64_t n, int32_t* sched, uint8_t* valid,
+                         void* stream);
+/* FP64 score of integer schedules sched (device int32 [n][n_vars]) -> score device double [n]. */
+FELIX_EXPORT felix_status felix_score(felix_space* s, felix_costmodel* m, const int32_t* sched, int64_t n,
+                         double* score, void* stream);
+/* Rejection sampler of Algorithm 1 line 12 (reading O9): y device fp32 [n_vars][n].
+ * u(seed, cand, attempt, var) = splitmix64 finaliser chained over (seed, cand+1, attempt+1, var+1)
+ * (each step h = mix(h + 0x9E3779B97F4A7C15 * k)), top 53 bits / 2^53.  For outer attempt a2 < 64:
+ * each split component draws y_j = u(.., 64*a2 + a1, j) ln(ub_j) for a1 < 64 until its split roots
+ * are <= 0; INT vars y_j = ln lo + u(.., 64*a2, j)(ln hi - ln lo); accept when every user root
+ * (smooth) is <= 0.  Fallback y = ln(lo). */
+FELIX_EXPORT felix_status felix_init_sample(felix_space* s, int64_t n, uint64_t rng_seed, int64_t index_base,
+                               float* y, void* stream);
+
+/* Per-kernel-class device time accumulated by felix_search while profiling is enabled (CUDA events
+ * on the search stream).  Classes: 0 DAG forward, 1 MLP GEMMs, 2 DAG reverse+Adam, 3 other.
+ * ms[4], launches[4]; reset with felix_profile_reset. */
+FELIX_EXPORT felix_status felix_profile_enable(felix_space* s, int32_t enable);
+FELIX_EXPORT felix_status felix_profile_read(felix_space* s, double* ms, int64_t* launches);
+FELIX_EXPORT felix_status felix_profile_reset(felix_space* s);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FELIX_H_ */

@@ -75,10 +75,27 @@ def smooth_dS(t: np.ndarray) -> np.ndarray:
 
 def smooth_R(t: np.ndarray) -> np.ndarray:
     t = np.asarray(t, dtype=np.float64)
+    return np.where(t >= 0.0, t, 0.0) + smooth_Rgap(t)
+
+
+def smooth_Rgap(t: np.ndarray) -> np.ndarray:
+    """R(t) - relu(t) = 1/2 (sqrt(1+t^2) - |t|) = 1 / (2 (sqrt(1+t^2) + |t|))  (> 0, <= 1/2)."""
+    t = np.asarray(t, dtype=np.float64)
     h = _hyp(t)
-    a = np.abs(t)
-    small = 1.0 / (2.0 * (h + a))            # = 1/2 (h - |t|)
-    return np.where(t >= 0.0, t + small, small)
+    return 1.0 / (2.0 * (h + np.abs(t)))
+
+
+def smooth_min(a: np.ndarray, b: np.ndarray) -> np.ndarray:
+    """min(a,b) smoothed = a - R(a-b) (rule table O3), evaluated without the cancellation of
+    a - (a - b): for t = a - b >= 0 it is b - gap(t), else a - gap(t) (reading R-stable)."""
+    t = a - b
+    return np.where(t >= 0.0, b, a) - smooth_Rgap(t)
+
+
+def smooth_max(a: np.ndarray, b: np.ndarray) -> np.ndarray:
+    """max(a,b) smoothed = b + R(a-b) = (t >= 0 ? a : b) + gap(t)."""
+    t = a - b
+    return np.where(t >= 0.0, a, b) + smooth_Rgap(t)
 
 
 # =============================================================================== forward evaluation
@@ -127,9 +144,9 @@ def eval_dag(space, x: np.ndarray, smooth: bool) -> Eval:
             elif op == OP_SQRT:
                 v = np.sqrt(vals[a])
             elif op == OP_MIN:
-                v = vals[a] - smooth_R(vals[a] - vals[b]) if smooth else np.minimum(vals[a], vals[b])
+                v = smooth_min(vals[a], vals[b]) if smooth else np.minimum(vals[a], vals[b])
             elif op == OP_MAX:
-                v = vals[b] + smooth_R(vals[a] - vals[b]) if smooth else np.maximum(vals[a], vals[b])
+                v = smooth_max(vals[a], vals[b]) if smooth else np.maximum(vals[a], vals[b])
             elif op in (OP_GT, OP_GE):
                 if smooth:
                     v = smooth_S(vals[a] - vals[b])

@@ -1,0 +1,278 @@
+"""Python binding of libfelix (include/felix.h): argument marshalling only.
+
+Every step of the hot path runs in libfelix's CUDA kernels (tcgen05 GEMMs, NVRTC-generated DAG
+kernels, rounding / scoring / top-k kernels).  PyTorch supplies device memory and streams.  There
+is no CPU fallback: importing this package without the built extension raises, and every device
+call needs an sm_100a GPU.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+from typing import Optional, Sequence
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libfelix.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"libfelix.so not built at {LIB_PATH}; run __graft_entry__.build() "
+                      f"(python paper_conf_asplos_zhaosam24_b200/_build.py)")
+_lib = ctypes.CDLL(LIB_PATH)
+
+FELIX_STATUS = {0: "OK", 1: "INVALID_ARG", 2: "INVALID_DAG", 3: "SHAPE", 4: "UNSUPPORTED", 5: "CUDA",
+                6: "NVRTC", 7: "OOM"}
+
+EXPORTED = ["felix_last_error", "felix_abi_version", "felix_space_create", "felix_space_destroy",
+            "felix_space_info", "felix_codegen", "felix_costmodel_load", "felix_costmodel_destroy",
+            "felix_search", "felix_round_topk", "felix_eval", "felix_round", "felix_score",
+            "felix_init_sample", "felix_profile_enable", "felix_profile_read", "felix_profile_reset"]
+
+
+class FelixError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"felix {FELIX_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class _Var(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("_pad", ctypes.c_int32), ("lo", ctypes.c_int64), ("hi", ctypes.c_int64)]
+
+
+class _Split(ctypes.Structure):
+    _fields_ = [("extent", ctypes.c_int64), ("n", ctypes.c_int32), ("_pad", ctypes.c_int32),
+                ("vars", ctypes.POINTER(ctypes.c_int32))]
+
+
+class _SearchParams(ctypes.Structure):
+    _fields_ = [("n_seeds", ctypes.c_int64), ("n_steps", ctypes.c_int32), ("lr", ctypes.c_float),
+                ("beta1", ctypes.c_float), ("beta2", ctypes.c_float), ("eps", ctypes.c_float),
+                ("lam", ctypes.c_float), ("rng_seed", ctypes.c_uint64), ("init_from_y", ctypes.c_int32),
+                ("_pad", ctypes.c_int32), ("index_base", ctypes.c_int64)]
+
+
+class _SpaceInfo(ctypes.Structure):
+    _fields_ = [("n_vars", ctypes.c_int32), ("n_nodes", ctypes.c_int32), ("n_features", ctypes.c_int32),
+                ("n_constraints_user", ctypes.c_int32), ("n_roots_total", ctypes.c_int32),
+                ("n_components", ctypes.c_int32), ("n_tuples_total", ctypes.c_int64), ("nvrtc_ms", ctypes.c_double),
+                ("regs_fwd", ctypes.c_int32), ("regs_rev", ctypes.c_int32), ("dag_flops_fwd", ctypes.c_int64)]
+
+
+_P = ctypes.c_void_p
+_lib.felix_last_error.restype = ctypes.c_char_p
+_lib.felix_abi_version.restype = ctypes.c_int32
+for _name in EXPORTED:
+    if _name not in ("felix_last_error", "felix_abi_version", "felix_space_destroy", "felix_costmodel_destroy"):
+        getattr(_lib, _name).restype = ctypes.c_int
+_lib.felix_space_destroy.restype = None
+_lib.felix_costmodel_destroy.restype = None
+
+
+def _check(status: int) -> None:
+    if status != 0:
+        raise FelixError(status, _lib.felix_last_error().decode(errors="replace"))
+
+
+def _ptr(t) -> int:
+    return 0 if t is None else int(t.data_ptr())
+
+
+def _stream(stream) -> int:
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return int(stream.cuda_stream)
+
+
+def _space_args(space):
+    """Marshal a felix_inputs.Space-like object (vars, splits, nodes, feature_roots, constraint_roots)."""
+    vars_ = (_Var * len(space.vars))()
+    for j, v in enumerate(space.vars):
+        vars_[j].kind, vars_[j].lo, vars_[j].hi = int(v.kind), int(v.lo), int(v.hi)
+    keep = []
+    splits = (_Split * max(1, len(space.splits)))()
+    for s, sp in enumerate(space.splits):
+        arr = (ctypes.c_int32 * len(sp.vars))(*[int(j) for j in sp.vars])
+        keep.append(arr)
+        splits[s].extent, splits[s].n = int(sp.extent), len(sp.vars)
+        splits[s].vars = ctypes.cast(arr, ctypes.POINTER(ctypes.c_int32))
+    nodes = np.ascontiguousarray(space.nodes)
+    assert nodes.dtype.itemsize == 24
+    fr = np.ascontiguousarray(space.feature_roots, dtype=np.int32)
+    cr = np.ascontiguousarray(space.constraint_roots, dtype=np.int32)
+    keep += [nodes, fr, cr]
+    args = [vars_, len(space.vars), splits, len(space.splits), nodes.ctypes.data_as(_P), len(nodes),
+            fr.ctypes.data_as(_P), len(fr), cr.ctypes.data_as(_P) if len(cr) else None, len(cr)]
+    return args, keep
+
+
+def abi_version() -> int:
+    return int(_lib.felix_abi_version())
+
+
+def codegen(space, compile: bool = False) -> str:
+    """Generated CUDA source of a space's expression kernels (device-free; compile=True also runs
+    NVRTC for sm_100a)."""
+    args, keep = _space_args(space)
+    n = ctypes.c_int64(0)
+    _check(_lib.felix_codegen(*args, 0, None, ctypes.c_int64(0), ctypes.byref(n)))
+    buf = ctypes.create_string_buffer(n.value + 1)
+    _check(_lib.felix_codegen(*args, int(compile), buf, ctypes.c_int64(n.value + 1), ctypes.byref(n)))
+    return buf.value.decode()
+
+
+@dataclass
+class SpaceInfo:
+    n_vars: int
+    n_nodes: int
+    n_features: int
+    n_constraints_user: int
+    n_roots_total: int
+    n_components: int
+    n_tuples_total: int
+    nvrtc_ms: float
+    regs_fwd: int
+    regs_rev: int
+    dag_flops_fwd: int
+
+
+class CostModel:
+    """felix_costmodel_load: MLP dims [d0, ..., 1], W[l] fp32 [d_{l+1}, d_l], b[l] fp32 [d_{l+1}]."""
+
+    def __init__(self, dims: Sequence[int], W: Sequence[np.ndarray], b: Sequence[np.ndarray], device: int = 0):
+        L = len(dims) - 1
+        Ws = [np.ascontiguousarray(w, dtype=np.float32) for w in W]
+        bs = [np.ascontiguousarray(x, dtype=np.float32) for x in b]
+        d = (ctypes.c_int32 * (L + 1))(*[int(x) for x in dims])
+        wp = (_P * L)(*[w.ctypes.data for w in Ws])
+        bp = (_P * L)(*[x.ctypes.data for x in bs])
+        h = _P()
+        _check(_lib.felix_costmodel_load(int(device), L, d, wp, bp, ctypes.byref(h)))
+        self._h = h
+        self.dims = tuple(int(x) for x in dims)
+        self.device = device
+
+    @classmethod
+    def from_weights(cls, mlp, device: int = 0) -> "CostModel":
+        return cls(mlp.dims, mlp.W, mlp.b, device)
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h:
+            _lib.felix_costmodel_destroy(h)
+            self._h = None
+
+    def mlp_flops_per_candidate_step(self) -> int:
+        """Forward + input-gradient backward: 4 * sum d_l d_{l+1}."""
+        return 4 * sum(self.dims[l] * self.dims[l + 1] for l in range(len(self.dims) - 1))
+
+
+class Space:
+    """felix_space_create + the search / rounding / scoring calls on it."""
+
+    def __init__(self, space, device: int = 0):
+        args, keep = _space_args(space)
+        h = _P()
+        _check(_lib.felix_space_create(int(device), *args, ctypes.byref(h)))
+        self._h = h
+        self.device = device
+        self.n_vars = len(space.vars)
+        self.name = getattr(space, "name", "space")
+        inf = _SpaceInfo()
+        _check(_lib.felix_space_info(self._h, ctypes.byref(inf)))
+        self.info = SpaceInfo(*[getattr(inf, f) for f, _ in _SpaceInfo._fields_])
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h:
+            _lib.felix_space_destroy(h)
+            self._h = None
+
+    # ---------------------------------------------------------------- primary calls
+    def search(self, cm: CostModel, y, n_steps: int, *, lr=0.05, beta1=0.9, beta2=0.999, eps=1e-8, lam=1.0,
+               rng_seed: int = 0, init_from_y: bool = True, index_base: int = 0, final_loss=None, stream=None):
+        """felix_search on device y (torch fp32 [n_vars, n], updated in place)."""
+        self._check_y(y)
+        p = _SearchParams(int(y.shape[1]), int(n_steps), lr, beta1, beta2, eps, lam, int(rng_seed) & (2**64 - 1),
+                          1 if init_from_y else 0, 0, int(index_base))
+        _check(_lib.felix_search(self._h, cm._h, ctypes.byref(p), _P(_ptr(y)), _P(_ptr(final_loss)),
+                                 _P(_stream(stream))))
+        return y
+
+    def round_topk(self, cm: CostModel, y, k: int, index_base: int = 0, stream=None):
+        """felix_round_topk -> (idx int64 [m], score float64 [m], sched int32 [m, n_vars]) on the host."""
+        self._check_y(y)
+        idx = np.zeros(k, dtype=np.int64)
+        sc = np.zeros(k, dtype=np.float64)
+        sched = np.zeros((k, self.n_vars), dtype=np.int32)
+        cnt = ctypes.c_int32(0)
+        _check(_lib.felix_round_topk(self._h, cm._h, _P(_ptr(y)), ctypes.c_int64(y.shape[1]),
+                                     ctypes.c_int64(index_base), int(k), idx.ctypes.data_as(_P),
+                                     sc.ctypes.data_as(_P), sched.ctypes.data_as(_P), ctypes.byref(cnt),
+                                     _P(_stream(stream))))
+        m = cnt.value
+        return idx[:m], sc[:m], sched[:m]
+
+    # ---------------------------------------------------------------- test hooks
+    def eval(self, cm: CostModel, y, lam: float = 1.0, stream=None):
+        import torch
+        self._check_y(y)
+        n = y.shape[1]
+        dev = y.device
+        out = dict(
+            phi=torch.empty((cm.dims[0], n), dtype=torch.float32, device=dev),
+            g=torch.empty((self.info.n_roots_total, n), dtype=torch.float32, device=dev),
+            cost=torch.empty(n, dtype=torch.float32, device=dev),
+            loss=torch.empty(n, dtype=torch.float32, device=dev),
+            grad=torch.empty((self.n_vars, n), dtype=torch.float32, device=dev),
+        )
+        _check(_lib.felix_eval(self._h, cm._h, _P(_ptr(y)), ctypes.c_int64(n), ctypes.c_float(lam),
+                               _P(_ptr(out["phi"])), _P(_ptr(out["g"])), _P(_ptr(out["cost"])),
+                               _P(_ptr(out["loss"])), _P(_ptr(out["grad"])), _P(_stream(stream))))
+        return out
+
+    def round(self, y, stream=None):
+        import torch
+        self._check_y(y)
+        n = y.shape[1]
+        sched = torch.empty((n, self.n_vars), dtype=torch.int32, device=y.device)
+        valid = torch.empty(n, dtype=torch.uint8, device=y.device)
+        _check(_lib.felix_round(self._h, _P(_ptr(y)), ctypes.c_int64(n), _P(_ptr(sched)), _P(_ptr(valid)),
+                                _P(_stream(stream))))
+        return sched, valid
+
+    def score(self, cm: CostModel, sched, stream=None):
+        import torch
+        n = sched.shape[0]
+        out = torch.empty(n, dtype=torch.float64, device=sched.device)
+        _check(_lib.felix_score(self._h, cm._h, _P(_ptr(sched)), ctypes.c_int64(n), _P(_ptr(out)),
+                                _P(_stream(stream))))
+        return out
+
+    def init_sample(self, n: int, rng_seed: int, index_base: int = 0, device=None, stream=None):
+        import torch
+        y = torch.empty((self.n_vars, n), dtype=torch.float32, device=device or f"cuda:{self.device}")
+        _check(_lib.felix_init_sample(self._h, ctypes.c_int64(n), ctypes.c_uint64(int(rng_seed) & (2**64 - 1)),
+                                      ctypes.c_int64(index_base), _P(_ptr(y)), _P(_stream(stream))))
+        return y
+
+    def profile(self, enable: bool) -> None:
+        _check(_lib.felix_profile_enable(self._h, 1 if enable else 0))
+
+    def profile_read(self):
+        ms = (ctypes.c_double * 4)()
+        ln = (ctypes.c_int64 * 4)()
+        _check(_lib.felix_profile_read(self._h, ms, ln))
+        names = ("dag_fwd", "mlp_gemm", "dag_rev_adam", "init")
+        return {nm: (ms[i], ln[i]) for i, nm in enumerate(names)}
+
+    def profile_reset(self) -> None:
+        _check(_lib.felix_profile_reset(self._h))
+
+    def _check_y(self, y) -> None:
+        import torch
+        if not (isinstance(y, torch.Tensor) and y.is_cuda and y.dtype == torch.float32 and y.dim() == 2
+                and y.shape[0] == self.n_vars and y.is_contiguous()):
+            raise FelixError(1, f"y must be a contiguous CUDA float32 tensor [{self.n_vars}, n]")

@@ -1,0 +1,172 @@
+// aux_kernels.cuh — rounding, FP64 scoring and top-k (Algorithm 1 lines 20-21, P:L919-920,
+// P:L928-935).  All decisions that produce integers are taken in FP64 with explicitly rounded
+// operations (no FMA contraction) against host-built ln tables, so they are reproducible
+// bit-for-bit by the float64 oracle (DESIGN.md "Readings" O10, R-valid).
+#pragma once
+#include <cstdint>
+#include <cfloat>
+
+namespace felix {
+
+// ---------------------------------------------------------------------------- K5a split rounding
+// One warp per (candidate, split component): lanes stride over the component's divisor-tuple
+// table (lexicographic order) computing sum_j (y_j - ln f_j)^2; warp argmin, ties -> lower index
+// (= lexicographically smallest tuple).  Reading O10 of P:L796-801 ("rounds y to the closest ln N_i").
+__global__ void __launch_bounds__(256) round_split_kernel(
+    const float* __restrict__ y, int n, int M, int n_comp,
+    const int* __restrict__ comp_nvars, const int* __restrict__ comp_var0, const int* __restrict__ comp_vars,
+    const long long* __restrict__ comp_eoff, const long long* __restrict__ comp_tcount,
+    const int* __restrict__ tuples, const double* __restrict__ lnf, int* __restrict__ sched) {
+  const long long gw = (static_cast<long long>(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (gw >= static_cast<long long>(n) * n_comp) return;
+  const int cand = static_cast<int>(gw / n_comp), comp = static_cast<int>(gw % n_comp);
+  const int nv = comp_nvars[comp];
+  const int* vars = comp_vars + comp_var0[comp];
+  double yv[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) yv[k] = k < nv ? static_cast<double>(y[static_cast<size_t>(vars[k]) * n + cand]) : 0.0;
+  const long long eoff = comp_eoff[comp], T = comp_tcount[comp];
+  double best = DBL_MAX;
+  long long bi = -1;
+  for (long long t = lane; t < T; t += 32) {
+    const double* l = lnf + eoff + t * nv;
+    double acc = 0.0;
+    for (int k = 0; k < nv; ++k) {
+      const double d = __dsub_rn(yv[k], l[k]);
+      acc = __dadd_rn(acc, __dmul_rn(d, d));
+    }
+    if (acc < best) { best = acc; bi = t; }     // strict: first minimum in this lane's stride
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    const double ob = __shfl_xor_sync(0xffffffffu, best, off);
+    const long long oi = __shfl_xor_sync(0xffffffffu, bi, off);
+    const bool take = (oi >= 0) && (bi < 0 || ob < best || (ob == best && oi < bi));
+    if (take) { best = ob; bi = oi; }
+  }
+  if (lane == 0) {
+    if (bi < 0) bi = 0;    // all distances NaN: first tuple (all ones), as np.argmin
+    const int* tp = tuples + eoff + bi * nv;
+    for (int k = 0; k < nv; ++k) sched[static_cast<size_t>(cand) * M + vars[k]] = tp[k];
+  }
+}
+
+// ---------------------------------------------------------------------------- K5b INT rounding
+// x = lo + #{k in [lo, hi-1] : ln(k + 1/2) <= y}  (nearest integer), binary search.
+__global__ void round_int_kernel(const float* __restrict__ y, int n, int M, int n_int, const int* __restrict__ int_vars,
+                                 const long long* __restrict__ int_lo, const long long* __restrict__ int_cnt,
+                                 const long long* __restrict__ int_toff, const double* __restrict__ thr, int* __restrict__ sched) {
+  const long long g = static_cast<long long>(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (g >= static_cast<long long>(n) * n_int) return;
+  const int cand = static_cast<int>(g / n_int), q = static_cast<int>(g % n_int);
+  const int j = int_vars[q];
+  const double yv = static_cast<double>(y[static_cast<size_t>(j) * n + cand]);
+  const double* t = thr + int_toff[q];
+  long long lo = 0, hi = int_cnt[q];          // count of thresholds <= yv
+  while (lo < hi) {
+    const long long mid = (lo + hi) >> 1;
+    if (t[mid] <= yv) lo = mid + 1; else hi = mid;
+  }
+  sched[static_cast<size_t>(cand) * M + j] = static_cast<int>(int_lo[q] + lo);
+}
+
+// ---------------------------------------------------------------------------- K6 FP64 MLP scoring
+// out[row][col] = act( b[col] + sum_k W[col][k] * in(row, k) ), fixed k order (deterministic).
+__global__ void score_layer_kernel(const double* __restrict__ in, long long in_rs, long long in_cs, int n, int K,
+                                   const double* __restrict__ W, const double* __restrict__ b, double* __restrict__ out,
+                                   int N, int relu) {
+  const long long g = static_cast<long long>(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (g >= static_cast<long long>(n) * N) return;
+  const int row = static_cast<int>(g / N), col = static_cast<int>(g % N);
+  const double* w = W + static_cast<size_t>(col) * K;
+  const double* x = in + static_cast<size_t>(row) * in_rs;
+  double z = b[col];
+  for (int k = 0; k < K; ++k) z = fma(w[k], x[static_cast<size_t>(k) * in_cs], z);
+  out[g] = (relu && !(z > 0.0)) ? 0.0 : z;
+}
+
+// ---------------------------------------------------------------------------- K7 dedup + top-k
+// Each block owns a chunk of entries; k rounds of block argmax by (score desc, candidate asc) over
+// alive entries, then every alive entry whose schedule equals the winner's is killed (dedup keeps
+// the smallest candidate index, which wins ties).  Phase A: entries = candidates, many blocks;
+// phase B: entries = phase-A records, one block.  Warp shuffle + shared-memory block reduction.
+struct TopkKey { double s; int c; };
+__device__ __forceinline__ bool topk_better(const TopkKey& a, const TopkKey& b) {
+  if (a.c < 0) return false;
+  if (b.c < 0) return true;
+  return a.s > b.s || (a.s == b.s && a.c < b.c);
+}
+
+__global__ void __launch_bounds__(1024) topk_select_kernel(
+    long long n_entries, long long chunk, const int* __restrict__ cand_of,
+    const double* __restrict__ score, const unsigned char* __restrict__ valid, const int* __restrict__ sched, int M,
+    int k, unsigned char* __restrict__ alive, int* __restrict__ out_cand, int* __restrict__ out_cnt) {
+  __shared__ TopkKey red[32];
+  __shared__ TopkKey win;
+  const long long c0 = static_cast<long long>(blockIdx.x) * chunk;
+  const long long c1 = min(n_entries, c0 + chunk);
+  for (long long e = c0 + threadIdx.x; e < c1; e += blockDim.x) {
+    const int c = cand_of ? cand_of[e] : static_cast<int>(e);
+    alive[e] = (c >= 0 && valid[c] && isfinite(score[c])) ? 1 : 0;
+  }
+  __syncthreads();
+  int r = 0;
+  for (; r < k; ++r) {
+    TopkKey best{0.0, -1};
+    for (long long e = c0 + threadIdx.x; e < c1; e += blockDim.x) {
+      if (!alive[e]) continue;
+      const int c = cand_of ? cand_of[e] : static_cast<int>(e);
+      const TopkKey t{score[c], c};
+      if (topk_better(t, best)) best = t;
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      TopkKey o{__shfl_xor_sync(0xffffffffu, best.s, off), __shfl_xor_sync(0xffffffffu, best.c, off)};
+      if (topk_better(o, best)) best = o;
+    }
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = best;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+      TopkKey b = (threadIdx.x < (blockDim.x + 31) / 32) ? red[threadIdx.x] : TopkKey{0.0, -1};
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) {
+        TopkKey o{__shfl_xor_sync(0xffffffffu, b.s, off), __shfl_xor_sync(0xffffffffu, b.c, off)};
+        if (topk_better(o, b)) b = o;
+      }
+      if (threadIdx.x == 0) win = b;
+    }
+    __syncthreads();
+    const TopkKey w = win;
+    if (w.c < 0) break;
+    if (threadIdx.x == 0) out_cand[blockIdx.x * static_cast<long long>(k) + r] = w.c;
+    const int* ws = sched + static_cast<size_t>(w.c) * M;
+    for (long long e = c0 + threadIdx.x; e < c1; e += blockDim.x) {
+      if (!alive[e]) continue;
+      const int c = cand_of ? cand_of[e] : static_cast<int>(e);
+      const int* cs = sched + static_cast<size_t>(c) * M;
+      bool same = true;
+      for (int j = 0; j < M; ++j) same = same && (cs[j] == ws[j]);
+      if (same) alive[e] = 0;
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    out_cnt[blockIdx.x] = r;
+    for (int q = r; q < k; ++q) out_cand[blockIdx.x * static_cast<long long>(k) + q] = -1;
+  }
+}
+
+// gather the final records into contiguous arrays for one D2H copy
+__global__ void topk_gather_kernel(const int* __restrict__ cand, const int* __restrict__ cnt, int k, const double* __restrict__ score,
+                                   const int* __restrict__ sched, int M, long long index_base,
+                                   long long* __restrict__ o_idx, double* __restrict__ o_score, int* __restrict__ o_sched) {
+  const int r = threadIdx.x;
+  if (r >= k) return;
+  const int c = r < cnt[0] ? cand[r] : -1;
+  o_idx[r] = c >= 0 ? index_base + c : -1;
+  o_score[r] = c >= 0 ? score[c] : 0.0;
+  for (int j = 0; j < M; ++j) o_sched[static_cast<size_t>(r) * M + j] = c >= 0 ? sched[static_cast<size_t>(c) * M + j] : 0;
+}
+
+}  // namespace felix

@@ -1,0 +1,914 @@
+// felix_api.cu — libfelix: the C ABI of include/felix.h on B200 (sm_100a).
+//
+// Per search step (Algorithm 1 lines 16-19) the device runs, with no host round trip:
+//   felix_fwd (NVRTC, per space)  ->  L-1 forward tcgen05 GEMMs  ->  L-1 backward tcgen05 GEMMs
+//   ->  felix_rev_adam (NVRTC, per space)
+// and after the search (lines 20-21): rounding (K5), hard features + validity (NVRTC), FP64 MLP
+// scoring (K6), dedup + top-k (K7).
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <functional>
+#include <map>
+#include <mutex>
+#include <numeric>
+#include <string>
+#include <vector>
+#include <nvrtc.h>
+#include <cudaTypedefs.h>
+#include "felix_internal.h"
+#include "mlp_gemm.cuh"
+#include "aux_kernels.cuh"
+
+namespace felix {
+
+static thread_local std::string g_last_error;
+void set_error(const std::string& m) { g_last_error = m; }
+
+// ============================================================================ GEMM dispatch
+struct GemmLaunch {
+  int epi = 0, bn = 0;
+  CUtensorMap a_hi, a_lo, b_hi, b_lo;
+  GemmArgs args{};
+  dim3 grid;
+};
+
+template <int BN, int EPI>
+static void launch_gemm_t(const GemmLaunch& g, cudaStream_t st) {
+  auto kern = mlp_gemm_kernel<BN, EPI>;
+  static bool attr_set = false;   // per instantiation; devices share the same limit on one box
+  if (!attr_set) {
+    CUDA_OK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, GemmCfg<BN>::SMEM_BYTES));
+    attr_set = true;
+  }
+  kern<<<g.grid, 128, GemmCfg<BN>::SMEM_BYTES, st>>>(g.a_hi, g.a_lo, g.b_hi, g.b_lo, g.args);
+  CUDA_OK(cudaGetLastError());
+}
+
+static void launch_gemm(const GemmLaunch& g, cudaStream_t st) {
+#define FELIX_G(BN_, EPI_) if (g.bn == BN_ && g.epi == EPI_) return launch_gemm_t<BN_, EPI_>(g, st)
+  FELIX_G(64, EPI_RELU); FELIX_G(128, EPI_RELU); FELIX_G(256, EPI_RELU);
+  FELIX_G(64, EPI_HEAD); FELIX_G(128, EPI_HEAD); FELIX_G(256, EPI_HEAD);
+  FELIX_G(64, EPI_MASK); FELIX_G(128, EPI_MASK); FELIX_G(256, EPI_MASK);
+  FELIX_G(64, EPI_F32T); FELIX_G(96, EPI_F32T); FELIX_G(128, EPI_F32T); FELIX_G(256, EPI_F32T);
+#undef FELIX_G
+  FELIX_THROW(FELIX_E_UNSUPPORTED, "no GEMM instantiation for BN=" + std::to_string(g.bn));
+}
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point: libfelix does not link libcuda,
+// so it loads (and its symbols can be inspected) on a machine without a GPU driver.
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    CUDA_OK(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q));
+    if (q != cudaDriverEntryPointSuccess || !p) FELIX_THROW(FELIX_E_CUDA, "cuTensorMapEncodeTiled unavailable");
+    fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  }
+  return fn;
+}
+
+static CUtensorMap make_tmap(const void* base, int64_t rows, int64_t cols, int box_rows) {
+  CUtensorMap m;
+  cuuint64_t dims[2] = {static_cast<cuuint64_t>(cols), static_cast<cuuint64_t>(rows)};
+  cuuint64_t strides[1] = {static_cast<cuuint64_t>(cols) * 2};
+  cuuint32_t box[2] = {static_cast<cuuint32_t>(GEMM_BK), static_cast<cuuint32_t>(box_rows)};
+  cuuint32_t es[2] = {1, 1};
+  CU_OK(encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE));
+  return m;
+}
+
+// ============================================================================ per-(space, model, n) plan
+struct Plan {
+  const CostModel* cm = nullptr;
+  int64_t n = -1, n_pad = 0;
+  DevBuf phi_hi, phi_lo;                                   // [n][K0p]
+  std::vector<std::unique_ptr<DevBuf>> act_hi, act_lo, mask;  // per hidden layer l = 1..L-1
+  DevBuf c_part, dphi, m, v;
+  int n_head_tiles = 0;
+  std::vector<GemmLaunch> gemms;
+};
+
+struct ProfEvent { int cls; cudaEvent_t a, b; };
+
+}  // namespace felix
+
+struct felix_space {
+  int device = 0;
+  felix::SpaceDesc desc;
+  felix::RoundTables rt;
+  int K0p = 96;
+  // device copies of the rounding tables
+  felix::DevBuf d_comp_nvars, d_comp_var0, d_comp_vars, d_comp_eoff, d_comp_tcount, d_tuples, d_lnf;
+  felix::DevBuf d_int_vars, d_int_lo, d_int_cnt, d_int_toff, d_int_thr;
+  // NVRTC module
+  cudaLibrary_t module = nullptr;
+  cudaKernel_t f_fwd = nullptr, f_rev_adam = nullptr, f_rev_eval = nullptr, f_hard = nullptr, f_init = nullptr;
+  double nvrtc_ms = 0;
+  int regs_fwd = 0, regs_rev = 0;
+  int64_t flops_fwd = 0;
+  std::string source;
+  // plan cache + scratch
+  std::unique_ptr<felix::Plan> plan;
+  felix::DevBuf sched, valid, phi64, score, act64a, act64b, alive, rec_cand, rec_cnt, fin_cand, fin_cnt, o_idx, o_score, o_sched;
+  // profiling
+  bool profiling = false;
+  std::vector<felix::ProfEvent> prof;
+  double prof_ms[4] = {0, 0, 0, 0};
+  int64_t prof_launches[4] = {0, 0, 0, 0};
+  ~felix_space() {
+    for (auto& e : prof) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
+    if (module) cudaLibraryUnload(module);
+  }
+};
+
+struct felix_costmodel : felix::CostModel {};
+
+namespace felix {
+
+// ============================================================================ helpers
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    CUDA_OK(cudaGetDevice(&prev));
+    if (prev != dev) CUDA_OK(cudaSetDevice(dev));
+    CUDA_OK(cudaFree(nullptr));   // ensure the primary context exists (driver API shares it)
+  }
+  ~DeviceGuard() { if (prev >= 0) cudaSetDevice(prev); }
+};
+
+static void check_device(int dev) {
+  int count = 0;
+  if (cudaGetDeviceCount(&count) != cudaSuccess || count == 0)
+    FELIX_THROW(FELIX_E_CUDA, "no CUDA device available (libfelix has no CPU fallback)");
+  if (dev < 0 || dev >= count) FELIX_THROW(FELIX_E_INVALID_ARG, "device index out of range");
+  cudaDeviceProp p{};
+  CUDA_OK(cudaGetDeviceProperties(&p, dev));
+  if (p.major != 10) FELIX_THROW(FELIX_E_CUDA, std::string("libfelix is built for sm_100a; device is ") + p.name);
+}
+
+template <class T>
+static void upload(DevBuf& d, const std::vector<T>& h) {
+  d.alloc(std::max<size_t>(h.size() * sizeof(T), 16));
+  if (!h.empty()) CUDA_OK(cudaMemcpy(d.p, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice));
+}
+
+static void ensure(DevBuf& d, size_t bytes) {
+  if (d.bytes < bytes) d.alloc(bytes);
+}
+
+static int arity(int op) {
+  switch (op) {
+    case FELIX_OP_CONST: case FELIX_OP_VAR: return 0;
+    case FELIX_OP_NEG: case FELIX_OP_EXP: case FELIX_OP_LOG: case FELIX_OP_SQRT: case FELIX_OP_NOT: case FELIX_OP_POW: return 1;
+    case FELIX_OP_SELECT: return 3;
+    default: return 2;
+  }
+}
+static bool is_bool_op(int op) {
+  return op == FELIX_OP_GT || op == FELIX_OP_GE || op == FELIX_OP_LT || op == FELIX_OP_LE || op == FELIX_OP_EQ ||
+         op == FELIX_OP_NE || op == FELIX_OP_AND || op == FELIX_OP_OR || op == FELIX_OP_NOT;
+}
+
+// ============================================================================ rounding tables
+static std::vector<int64_t> divisors(int64_t n) {
+  std::vector<int64_t> d;
+  for (int64_t k = 1; k * k <= n; ++k)
+    if (n % k == 0) { d.push_back(k); if (k * k != n) d.push_back(n / k); }
+  std::sort(d.begin(), d.end());
+  return d;
+}
+
+void build_round_tables(const SpaceDesc& d, RoundTables& t) {
+  const int M = d.n_vars;
+  std::vector<int> parent(M);
+  std::iota(parent.begin(), parent.end(), 0);
+  std::function<int(int)> find = [&](int j) { while (parent[j] != j) { parent[j] = parent[parent[j]]; j = parent[j]; } return j; };
+  for (auto& sv : d.split_vars) for (size_t k = 1; k < sv.size(); ++k) parent[find(sv[k])] = find(sv[0]);
+  std::vector<std::vector<int>> comps;
+  std::vector<int> root_of(M, -1);
+  for (int j = 0; j < M; ++j) {
+    if (d.vars[j].kind != FELIX_VAR_SPLIT) continue;
+    int r = find(j);
+    if (root_of[r] < 0) { root_of[r] = (int)comps.size(); comps.push_back({}); }
+    comps[root_of[r]].push_back(j);
+  }
+  const int64_t kMaxTuples = int64_t(1) << 22;
+  for (auto& comp : comps) {
+    if (comp.size() > 8) FELIX_THROW(FELIX_E_UNSUPPORTED, "split component with more than 8 variables");
+    std::vector<int> sp;   // splits touching the component
+    for (size_t s = 0; s < d.split_vars.size(); ++s)
+      for (int v : d.split_vars[s]) if (std::find(comp.begin(), comp.end(), v) != comp.end()) { sp.push_back((int)s); break; }
+    const int nv = (int)comp.size();
+    t.comp_nvars.push_back(nv);
+    t.comp_var0.push_back((int)t.comp_vars.size());
+    for (int j : comp) t.comp_vars.push_back(j);
+    t.comp_toff.push_back(t.n_tuples_total);
+    t.comp_eoff.push_back((int64_t)t.tuples.size());
+    int64_t count = 0;
+    std::vector<int64_t> rem(sp.size());
+    for (size_t q = 0; q < sp.size(); ++q) rem[q] = d.split_extent[sp[q]];
+    std::vector<int32_t> cur(nv);
+    std::function<void(int)> rec = [&](int k) {
+      if (k == nv) {
+        if (++count > kMaxTuples) FELIX_THROW(FELIX_E_UNSUPPORTED, "divisor-tuple table exceeds 2^22 rows");
+        for (int q = 0; q < nv; ++q) { t.tuples.push_back(cur[q]); t.lnf.push_back(std::log((double)cur[q])); }
+        return;
+      }
+      const int j = comp[k];
+      int64_t g = 0;
+      for (size_t q = 0; q < sp.size(); ++q)
+        if (std::find(d.split_vars[sp[q]].begin(), d.split_vars[sp[q]].end(), j) != d.split_vars[sp[q]].end())
+          g = std::gcd(g, rem[q]);
+      for (int64_t dv : divisors(g)) {
+        std::vector<int64_t> save = rem;
+        for (size_t q = 0; q < sp.size(); ++q)
+          if (std::find(d.split_vars[sp[q]].begin(), d.split_vars[sp[q]].end(), j) != d.split_vars[sp[q]].end())
+            rem[q] /= dv;
+        cur[k] = (int32_t)dv;
+        rec(k + 1);
+        rem = save;
+      }
+    };
+    rec(0);
+    t.comp_tcount.push_back(count);
+    t.n_tuples_total += count;
+  }
+  for (int j = 0; j < M; ++j) {
+    if (d.vars[j].kind != FELIX_VAR_INT) continue;
+    t.int_vars.push_back(j);
+    t.int_lo.push_back(d.vars[j].lo);
+    t.int_hi.push_back(d.vars[j].hi);
+    t.int_toff.push_back((int64_t)t.int_thr.size());
+    for (int64_t k = d.vars[j].lo; k < d.vars[j].hi; ++k) t.int_thr.push_back(std::log((double)k + 0.5));
+  }
+}
+
+// ============================================================================ NVRTC
+static std::vector<char> nvrtc_compile(const std::string& source) {
+  nvrtcProgram prog;
+  if (nvrtcCreateProgram(&prog, source.c_str(), "felix_space.cu", 0, nullptr, nullptr) != NVRTC_SUCCESS)
+    FELIX_THROW(FELIX_E_NVRTC, "nvrtcCreateProgram failed");
+  const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "--fmad=true"};
+  nvrtcResult rc = nvrtcCompileProgram(prog, 4, opts);
+  if (rc != NVRTC_SUCCESS) {
+    size_t ls = 0;
+    nvrtcGetProgramLogSize(prog, &ls);
+    std::string log(ls, '\0');
+    nvrtcGetProgramLog(prog, &log[0]);
+    nvrtcDestroyProgram(&prog);
+    FELIX_THROW(FELIX_E_NVRTC, "NVRTC compile failed: " + log.substr(0, 4000));
+  }
+  size_t cs = 0;
+  nvrtcGetCUBINSize(prog, &cs);
+  std::vector<char> cubin(cs);
+  nvrtcGetCUBIN(prog, cubin.data());
+  nvrtcDestroyProgram(&prog);
+  return cubin;
+}
+
+static void compile_module(felix_space* s) {
+  CodegenInfo info;
+  s->source = generate_dag_module(s->desc, s->K0p, &info);
+  s->flops_fwd = info.flops_fwd;
+  auto t0 = std::chrono::steady_clock::now();
+  std::vector<char> cubin = nvrtc_compile(s->source);
+  CUDA_OK(cudaLibraryLoadData(&s->module, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0));
+  CUDA_OK(cudaLibraryGetKernel(&s->f_fwd, s->module, "felix_fwd"));
+  CUDA_OK(cudaLibraryGetKernel(&s->f_rev_adam, s->module, "felix_rev_adam"));
+  CUDA_OK(cudaLibraryGetKernel(&s->f_rev_eval, s->module, "felix_rev_eval"));
+  CUDA_OK(cudaLibraryGetKernel(&s->f_hard, s->module, "felix_hard"));
+  CUDA_OK(cudaLibraryGetKernel(&s->f_init, s->module, "felix_init"));
+  cudaFuncAttributes fa{};
+  CUDA_OK(cudaFuncGetAttributes(&fa, reinterpret_cast<const void*>(s->f_fwd)));
+  s->regs_fwd = fa.numRegs;
+  CUDA_OK(cudaFuncGetAttributes(&fa, reinterpret_cast<const void*>(s->f_rev_adam)));
+  s->regs_rev = fa.numRegs;
+  s->nvrtc_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
+
+static void launch_nv(cudaKernel_t f, int64_t n, void** args, cudaStream_t st) {
+  if (n <= 0) return;
+  const unsigned grid = static_cast<unsigned>((n + 127) / 128);
+  CUDA_OK(cudaLaunchKernel(reinterpret_cast<const void*>(f), dim3(grid), dim3(128), args, 0, st));
+}
+
+// ============================================================================ plan
+static int choose_bn(int64_t m_tiles, int N) {
+  // prefer >= one full wave of CTAs (148 SMs) before larger tiles
+  if (N % 128 == 0 && m_tiles * (N / 128) >= 148) return 128;
+  if (N % 64 == 0) return 64;
+  FELIX_THROW(FELIX_E_UNSUPPORTED, "hidden dim must be a multiple of 64");
+}
+
+static Plan& get_plan(felix_space* s, const CostModel* cm, int64_t n) {
+  if (s->plan && s->plan->cm == cm && s->plan->n == n) return *s->plan;
+  auto p = std::make_unique<Plan>();
+  p->cm = cm;
+  p->n = n;
+  p->n_pad = (n + 127) / 128 * 128;
+  const int L = cm->n_layers;
+  const auto& d = cm->dims;
+  const int64_t np = p->n_pad;
+  const int K0p = cm->K0p;
+  p->phi_hi.alloc(np * K0p * 2);
+  p->phi_lo.alloc(np * K0p * 2);
+  p->act_hi.resize(L);
+  p->act_lo.resize(L);
+  p->mask.resize(L);
+  for (int l = 1; l <= L - 1; ++l) {
+    p->act_hi[l] = std::make_unique<DevBuf>();
+    p->act_lo[l] = std::make_unique<DevBuf>();
+    p->act_hi[l]->alloc(np * d[l] * 2);
+    p->act_lo[l]->alloc(np * d[l] * 2);
+    if (l <= L - 2) {
+      p->mask[l] = std::make_unique<DevBuf>();
+      p->mask[l]->alloc(np * (d[l] / 32) * 4);
+    }
+  }
+  p->dphi.alloc(static_cast<size_t>(K0p) * np * 4);
+  p->m.alloc(static_cast<size_t>(s->desc.n_vars) * n * 4);
+  p->v.alloc(static_cast<size_t>(s->desc.n_vars) * n * 4);
+  const int64_t mt = np / 128;
+  // forward GEMMs, layer l = 1..L-1 (W index l-1)
+  for (int l = 1; l <= L - 1; ++l) {
+    GemmLaunch g;
+    const bool head = (l == L - 1);
+    g.epi = head ? EPI_HEAD : EPI_RELU;
+    const int N = d[l], Kdim = (l == 1) ? K0p : d[l - 1];
+    g.bn = choose_bn(mt, N);
+    const void* a_hi = (l == 1) ? p->phi_hi.p : p->act_hi[l - 1]->p;
+    const void* a_lo = (l == 1) ? p->phi_lo.p : p->act_lo[l - 1]->p;
+    g.a_hi = make_tmap(a_hi, n, Kdim, 128);
+    g.a_lo = make_tmap(a_lo, n, Kdim, 128);
+    g.b_hi = make_tmap(cm->W_hi[l - 1]->p, N, Kdim, g.bn);
+    g.b_lo = make_tmap(cm->W_lo[l - 1]->p, N, Kdim, g.bn);
+    GemmArgs& a = g.args;
+    a.M = static_cast<int>(n); a.N = N; a.K = Kdim;
+    a.bias = cm->bias[l - 1]->as<float>();
+    a.out_hi = p->act_hi[l]->as<__half>();
+    a.out_lo = p->act_lo[l]->as<__half>();
+    a.ld_out = N;
+    if (head) {
+      a.head_w = cm->head_w.as<float>();
+      p->n_head_tiles = N / g.bn;
+      p->c_part.alloc(static_cast<size_t>(p->n_head_tiles) * np * 4);
+      a.c_part = p->c_part.as<float>();
+      a.ld_c = static_cast<int>(np);
+    } else {
+      a.mask_out = p->mask[l]->as<uint32_t>();
+    }
+    g.grid = dim3(static_cast<unsigned>(mt), N / g.bn);
+    p->gemms.push_back(g);
+  }
+  // backward GEMMs: delta_{l-1} = (delta_l W_l) (.) m_{l-1} for l = L-1..2, then dphi = delta_1 W_1
+  for (int l = L - 1; l >= 1; --l) {
+    GemmLaunch g;
+    const bool last = (l == 1);
+    const int N = last ? K0p : d[l - 1], Kdim = d[l];
+    g.epi = last ? EPI_F32T : EPI_MASK;
+    g.bn = last ? K0p : choose_bn(mt, N);
+    g.a_hi = make_tmap(p->act_hi[l]->p, n, Kdim, 128);
+    g.a_lo = make_tmap(p->act_lo[l]->p, n, Kdim, 128);
+    g.b_hi = make_tmap(cm->WT_hi[l - 1]->p, N, Kdim, g.bn);
+    g.b_lo = make_tmap(cm->WT_lo[l - 1]->p, N, Kdim, g.bn);
+    GemmArgs& a = g.args;
+    a.M = static_cast<int>(n); a.N = N; a.K = Kdim;
+    if (last) {
+      a.out_f32 = p->dphi.as<float>();
+      a.ld_f32 = static_cast<int>(np);
+      a.n_valid = d[0];
+    } else {
+      a.out_hi = p->act_hi[l - 1]->as<__half>();
+      a.out_lo = p->act_lo[l - 1]->as<__half>();
+      a.ld_out = N;
+      a.mask_in = p->mask[l - 1]->as<uint32_t>();
+    }
+    g.grid = dim3(static_cast<unsigned>(mt), N / g.bn);
+    p->gemms.push_back(g);
+  }
+  s->plan = std::move(p);
+  return *s->plan;
+}
+
+// ============================================================================ profiling
+static void prof_mark(felix_space* s, int cls, cudaStream_t st, bool begin) {
+  if (!s->profiling) return;
+  if (begin) {
+    ProfEvent e{cls, nullptr, nullptr};
+    CUDA_OK(cudaEventCreate(&e.a));
+    CUDA_OK(cudaEventCreate(&e.b));
+    CUDA_OK(cudaEventRecord(e.a, st));
+    s->prof.push_back(e);
+  } else {
+    CUDA_OK(cudaEventRecord(s->prof.back().b, st));
+  }
+}
+
+// ============================================================================ step pieces
+static void run_forward_mlp(felix_space* s, Plan& p, const float* y, int64_t n, cudaStream_t st) {
+  int ni = static_cast<int>(n);
+  void* phi_hi = p.phi_hi.p;
+  void* phi_lo = p.phi_lo.p;
+  void* args[] = {&y, &ni, &phi_hi, &phi_lo};
+  prof_mark(s, 0, st, true);
+  launch_nv(s->f_fwd, n, args, st);
+  prof_mark(s, 0, st, false);
+  s->prof_launches[0] += 1;
+  prof_mark(s, 1, st, true);
+  for (const auto& g : p.gemms) launch_gemm(g, st);
+  prof_mark(s, 1, st, false);
+  s->prof_launches[1] += static_cast<int64_t>(p.gemms.size());
+}
+
+}  // namespace felix
+
+using namespace felix;
+
+static std::unique_ptr<felix_space> parse_space(const felix_var* vars, int32_t n_vars, const felix_split* splits,
+                                                int32_t n_splits, const felix_node* nodes, int32_t n_nodes,
+                                                const int32_t* feature_roots, int32_t n_features,
+                                                const int32_t* constraint_roots, int32_t n_constraints) {
+  if (n_vars <= 0 || !vars) FELIX_THROW(FELIX_E_INVALID_ARG, "n_vars must be > 0");
+  if (n_vars > 64) FELIX_THROW(FELIX_E_UNSUPPORTED, "at most 64 schedule variables");
+  if (n_splits < 0 || (n_splits > 0 && !splits)) FELIX_THROW(FELIX_E_INVALID_ARG, "bad splits");
+  if (n_nodes <= 0 || !nodes) FELIX_THROW(FELIX_E_INVALID_DAG, "empty DAG");
+  if (n_features <= 0 || n_features > 256 || !feature_roots) FELIX_THROW(FELIX_E_SHAPE, "n_features must be in [1, 256]");
+  if (n_constraints < 0 || (n_constraints > 0 && !constraint_roots)) FELIX_THROW(FELIX_E_INVALID_ARG, "bad constraints");
+  auto s = std::make_unique<felix_space>();
+  SpaceDesc& d = s->desc;
+  d.n_vars = n_vars;
+  d.vars.assign(vars, vars + n_vars);
+  std::vector<int> nsplit_of(n_vars, 0);
+  for (int j = 0; j < n_vars; ++j) {
+    const auto& v = d.vars[j];
+    if (v.kind == FELIX_VAR_INT) {
+      if (v.lo < 1 || v.hi < v.lo || v.hi > (int64_t(1) << 24)) FELIX_THROW(FELIX_E_INVALID_ARG, "INT var needs 1 <= lo <= hi <= 2^24");
+    } else if (v.kind != FELIX_VAR_SPLIT) {
+      FELIX_THROW(FELIX_E_INVALID_ARG, "unknown var kind");
+    }
+  }
+  for (int s_ = 0; s_ < n_splits; ++s_) {
+    const auto& sp = splits[s_];
+    if (sp.extent < 1 || sp.extent >= (int64_t(1) << 31)) FELIX_THROW(FELIX_E_INVALID_ARG, "split extent out of range");
+    if (sp.n <= 0 || !sp.vars) FELIX_THROW(FELIX_E_INVALID_ARG, "empty split");
+    std::vector<int32_t> sv(sp.vars, sp.vars + sp.n);
+    for (int j : sv) {
+      if (j < 0 || j >= n_vars) FELIX_THROW(FELIX_E_INVALID_ARG, "split var out of range");
+      if (d.vars[j].kind != FELIX_VAR_SPLIT) FELIX_THROW(FELIX_E_INVALID_ARG, "INT var listed in a split");
+      nsplit_of[j]++;
+    }
+    d.split_extent.push_back(sp.extent);
+    d.split_vars.push_back(sv);
+  }
+  for (int j = 0; j < n_vars; ++j)
+    if (d.vars[j].kind == FELIX_VAR_SPLIT && nsplit_of[j] == 0) FELIX_THROW(FELIX_E_INVALID_ARG, "SPLIT var in no split");
+  // DAG: topological order + types (0 NUM, 1 BOOL, 2 CONST = either)
+  d.nodes.assign(nodes, nodes + n_nodes);
+  std::vector<int> ty(n_nodes);
+  for (int i = 0; i < n_nodes; ++i) {
+    const auto& nd = d.nodes[i];
+    if (nd.op < 0 || nd.op > FELIX_OP_CEILDIV) FELIX_THROW(FELIX_E_INVALID_DAG, "bad opcode at node " + std::to_string(i));
+    const int ar = arity(nd.op);
+    const int args[3] = {nd.a, nd.b, nd.c};
+    for (int q = 0; q < ar; ++q)
+      if (args[q] < 0 || args[q] >= i) FELIX_THROW(FELIX_E_INVALID_DAG, "node " + std::to_string(i) + " argument not an earlier node");
+    auto need = [&](int q, int want) {
+      const int t = ty[args[q]];
+      if (t != 2 && t != want)
+        FELIX_THROW(FELIX_E_INVALID_DAG, "type error at node " + std::to_string(i) + (want ? " (expects BOOL)" : " (expects NUM)"));
+    };
+    if (nd.op == FELIX_OP_VAR) {
+      const int j = static_cast<int>(nd.imm);
+      if (nd.imm != j || j < 0 || j >= n_vars) FELIX_THROW(FELIX_E_INVALID_DAG, "VAR index out of range");
+      ty[i] = 0;
+    } else if (nd.op == FELIX_OP_CONST) {
+      if (!std::isfinite(nd.imm)) FELIX_THROW(FELIX_E_INVALID_DAG, "non-finite constant");
+      ty[i] = 2;
+    } else if (nd.op == FELIX_OP_AND || nd.op == FELIX_OP_OR) { need(0, 1); need(1, 1); ty[i] = 1; }
+    else if (nd.op == FELIX_OP_NOT) { need(0, 1); ty[i] = 1; }
+    else if (nd.op == FELIX_OP_SELECT) { need(0, 1); need(1, 0); need(2, 0); ty[i] = 0; }
+    else { for (int q = 0; q < ar; ++q) need(q, 0); ty[i] = is_bool_op(nd.op) ? 1 : 0; }
+  }
+  for (int k = 0; k < n_features; ++k) {
+    const int r = feature_roots[k];
+    if (r < 0 || r >= n_nodes || ty[r] == 1) FELIX_THROW(FELIX_E_INVALID_DAG, "feature root must be a NUM node");
+    d.froots.push_back(r);
+  }
+  for (int k = 0; k < n_constraints; ++k) {
+    const int r = constraint_roots[k];
+    if (r < 0 || r >= n_nodes || ty[r] == 1) FELIX_THROW(FELIX_E_INVALID_DAG, "constraint root must be a NUM node");
+    d.croots.push_back(r);
+  }
+  s->K0p = n_features <= 64 ? 64 : n_features <= 96 ? 96 : n_features <= 128 ? 128 : 256;
+  build_round_tables(d, s->rt);
+  return s;
+}
+
+// ============================================================================ C ABI
+#define FELIX_API_BEGIN try {
+#define FELIX_API_END                                                   \
+  }                                                                     \
+  catch (const felix::Error& e) { felix::set_error(e.msg); return e.code; } \
+  catch (const std::bad_alloc&) { felix::set_error("host allocation failed"); return FELIX_E_OOM; } \
+  catch (const std::exception& e) { felix::set_error(e.what()); return FELIX_E_CUDA; } \
+  return FELIX_OK;
+
+extern "C" {
+
+const char* felix_last_error(void) { return g_last_error.c_str(); }
+int32_t felix_abi_version(void) { return FELIX_ABI_VERSION; }
+
+felix_status felix_space_create(int device, const felix_var* vars, int32_t n_vars, const felix_split* splits,
+                                int32_t n_splits, const felix_node* nodes, int32_t n_nodes, const int32_t* feature_roots,
+                                int32_t n_features, const int32_t* constraint_roots, int32_t n_constraints,
+                                felix_space** out) {
+  FELIX_API_BEGIN
+  if (!out) FELIX_THROW(FELIX_E_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  auto s = parse_space(vars, n_vars, splits, n_splits, nodes, n_nodes, feature_roots, n_features, constraint_roots,
+                       n_constraints);
+  s->device = device;
+  check_device(device);
+  DeviceGuard dg(device);
+  const auto& t = s->rt;
+  upload(s->d_comp_nvars, t.comp_nvars); upload(s->d_comp_var0, t.comp_var0); upload(s->d_comp_vars, t.comp_vars);
+  upload(s->d_comp_eoff, t.comp_eoff); upload(s->d_comp_tcount, t.comp_tcount);
+  upload(s->d_tuples, t.tuples); upload(s->d_lnf, t.lnf);
+  std::vector<int32_t> iv(t.int_vars.begin(), t.int_vars.end());
+  std::vector<int64_t> icnt;
+  for (size_t q = 0; q < t.int_vars.size(); ++q) icnt.push_back(t.int_hi[q] - t.int_lo[q]);
+  upload(s->d_int_vars, iv); upload(s->d_int_lo, t.int_lo); upload(s->d_int_cnt, icnt);
+  upload(s->d_int_toff, t.int_toff); upload(s->d_int_thr, t.int_thr);
+  compile_module(s.get());
+  *out = s.release();
+  FELIX_API_END
+}
+
+
+felix_status felix_codegen(const felix_var* vars, int32_t n_vars, const felix_split* splits, int32_t n_splits,
+                           const felix_node* nodes, int32_t n_nodes, const int32_t* feature_roots, int32_t n_features,
+                           const int32_t* constraint_roots, int32_t n_constraints, int32_t compile, char* src,
+                           int64_t src_cap, int64_t* src_len) {
+  FELIX_API_BEGIN
+  auto s = parse_space(vars, n_vars, splits, n_splits, nodes, n_nodes, feature_roots, n_features, constraint_roots,
+                       n_constraints);
+  CodegenInfo info;
+  const std::string code = generate_dag_module(s->desc, s->K0p, &info);
+  if (src_len) *src_len = static_cast<int64_t>(code.size());
+  if (src && src_cap > 0) {
+    const size_t nb = std::min<size_t>(code.size() + 1, static_cast<size_t>(src_cap));
+    std::memcpy(src, code.c_str(), nb);
+  }
+  if (compile) (void)nvrtc_compile(code);
+  FELIX_API_END
+}
+
+void felix_space_destroy(felix_space* s) {
+  if (!s) return;
+  int prev = -1;
+  cudaGetDevice(&prev);
+  cudaSetDevice(s->device);
+  delete s;
+  if (prev >= 0) cudaSetDevice(prev);
+}
+
+felix_status felix_space_info(const felix_space* s, felix_space_info_t* out) {
+  FELIX_API_BEGIN
+  if (!s || !out) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL argument");
+  out->n_vars = s->desc.n_vars;
+  out->n_nodes = static_cast<int32_t>(s->desc.nodes.size());
+  out->n_features = static_cast<int32_t>(s->desc.froots.size());
+  out->n_constraints_user = static_cast<int32_t>(s->desc.croots.size());
+  out->n_roots_total = s->desc.n_roots_total();
+  out->n_components = static_cast<int32_t>(s->rt.comp_nvars.size());
+  out->n_tuples_total = s->rt.n_tuples_total;
+  out->nvrtc_ms = s->nvrtc_ms;
+  out->regs_fwd = s->regs_fwd;
+  out->regs_rev = s->regs_rev;
+  out->dag_flops_fwd = s->flops_fwd;
+  FELIX_API_END
+}
+
+static void split_half(const std::vector<float>& x, std::vector<__half>& hi, std::vector<__half>& lo) {
+  hi.resize(x.size());
+  lo.resize(x.size());
+  for (size_t i = 0; i < x.size(); ++i) {
+    hi[i] = __float2half_rn(x[i]);
+    lo[i] = __float2half_rn(x[i] - __half2float(hi[i]));
+  }
+}
+
+felix_status felix_costmodel_load(int device, int32_t n_layers, const int32_t* dims, const float* const* W,
+                                  const float* const* b, felix_costmodel** out) {
+  FELIX_API_BEGIN
+  if (!out || !dims || !W || !b) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL argument");
+  *out = nullptr;
+  if (n_layers < 2 || n_layers > 16) FELIX_THROW(FELIX_E_UNSUPPORTED, "n_layers must be in [2, 16]");
+  if (dims[n_layers] != 1) FELIX_THROW(FELIX_E_SHAPE, "the last layer must have one output (predicted performance)");
+  if (dims[0] < 1 || dims[0] > 256) FELIX_THROW(FELIX_E_UNSUPPORTED, "dims[0] must be in [1, 256]");
+  for (int l = 1; l < n_layers; ++l)
+    if (dims[l] <= 0 || dims[l] % 64 != 0 || dims[l] > 4096) FELIX_THROW(FELIX_E_UNSUPPORTED, "hidden dims must be multiples of 64 in [64, 4096]");
+  for (int l = 0; l < n_layers; ++l) if (!W[l] || !b[l]) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL weight");
+  check_device(device);
+  DeviceGuard dg(device);
+  auto m = std::make_unique<felix_costmodel>();
+  m->device = device;
+  m->n_layers = n_layers;
+  m->dims.assign(dims, dims + n_layers + 1);
+  m->K0p = dims[0] <= 64 ? 64 : dims[0] <= 96 ? 96 : dims[0] <= 128 ? 128 : 256;
+  for (int l = 0; l < n_layers - 1; ++l) {
+    const int N = dims[l + 1], K = dims[l];
+    const int Kp = (l == 0) ? m->K0p : K;
+    std::vector<float> w(static_cast<size_t>(N) * Kp, 0.f), wt(static_cast<size_t>(Kp) * N, 0.f);
+    for (int r = 0; r < N; ++r)
+      for (int c = 0; c < K; ++c) {
+        const float v = W[l][static_cast<size_t>(r) * K + c];
+        w[static_cast<size_t>(r) * Kp + c] = v;
+        wt[static_cast<size_t>(c) * N + r] = v;
+      }
+    std::vector<__half> hi, lo, thi, tlo;
+    split_half(w, hi, lo);
+    split_half(wt, thi, tlo);
+    for (auto* vec : {&m->W_hi, &m->W_lo, &m->WT_hi, &m->WT_lo, &m->bias}) vec->push_back(std::make_unique<DevBuf>());
+    upload(*m->W_hi.back(), hi); upload(*m->W_lo.back(), lo);
+    upload(*m->WT_hi.back(), thi); upload(*m->WT_lo.back(), tlo);
+    upload(*m->bias.back(), std::vector<float>(b[l], b[l] + N));
+  }
+  const int Dh = dims[n_layers - 1];
+  upload(m->head_w, std::vector<float>(W[n_layers - 1], W[n_layers - 1] + Dh));
+  m->head_b = b[n_layers - 1][0];
+  for (int l = 0; l < n_layers; ++l) {
+    const int N = dims[l + 1], K = dims[l];
+    std::vector<double> w64(W[l], W[l] + static_cast<size_t>(N) * K), b64(b[l], b[l] + N);
+    m->W64.push_back(std::make_unique<DevBuf>());
+    m->b64.push_back(std::make_unique<DevBuf>());
+    upload(*m->W64.back(), w64);
+    upload(*m->b64.back(), b64);
+  }
+  *out = m.release();
+  FELIX_API_END
+}
+
+void felix_costmodel_destroy(felix_costmodel* m) { delete m; }
+
+static void check_pair(felix_space* s, felix_costmodel* m) {
+  if (!s || !m) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL handle");
+  if (static_cast<int>(s->desc.froots.size()) != m->dims[0])
+    FELIX_THROW(FELIX_E_SHAPE, "space n_features != cost model dims[0]");
+  if (s->device != m->device) FELIX_THROW(FELIX_E_INVALID_ARG, "space and cost model on different devices");
+}
+
+felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search_params* p, float* y,
+                          float* final_loss, void* stream) {
+  FELIX_API_BEGIN
+  check_pair(s, m);
+  if (!p) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL params");
+  if (p->n_seeds == 0) return FELIX_OK;
+  if (!y) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL y");
+  if (p->n_seeds < 0 || p->n_seeds > (int64_t(1) << 30)) FELIX_THROW(FELIX_E_INVALID_ARG, "n_seeds out of range");
+  if (p->n_steps < 0) FELIX_THROW(FELIX_E_INVALID_ARG, "n_steps < 0");
+  if (p->n_seeds == 0) return FELIX_OK;
+  DeviceGuard dg(s->device);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const int64_t n = p->n_seeds;
+  Plan& pl = get_plan(s, m, n);
+  int ni = static_cast<int>(n);
+  if (!p->init_from_y) {
+    unsigned long long seed = p->rng_seed;
+    long long ib = p->index_base;
+    void* args[] = {&seed, &ni, &ib, &y};
+    prof_mark(s, 3, st, true);
+    launch_nv(s->f_init, n, args, st);
+    prof_mark(s, 3, st, false);
+    s->prof_launches[3] += 1;
+  }
+  CUDA_OK(cudaMemsetAsync(pl.m.p, 0, pl.m.bytes, st));
+  CUDA_OK(cudaMemsetAsync(pl.v.p, 0, pl.v.bytes, st));
+  void* dphi = pl.dphi.p;
+  void* cpart = pl.c_part.p;
+  int ld = static_cast<int>(pl.n_pad);
+  int nht = pl.n_head_tiles;
+  float hb = m->head_b, lam = p->lambda, lr = p->lr, b1 = p->beta1, b2 = p->beta2, eps = p->eps;
+  void* mv = pl.m.p;
+  void* vv = pl.v.p;
+  for (int t = 1; t <= p->n_steps; ++t) {
+    run_forward_mlp(s, pl, y, n, st);
+    float* lo = (t == p->n_steps) ? final_loss : nullptr;
+    int tt = t;
+    void* args[] = {&y, &ni, &dphi, &ld, &cpart, &nht, &ld, &hb, &lam, &mv, &vv, &tt, &lr, &b1, &b2, &eps, &lo};
+    prof_mark(s, 2, st, true);
+    launch_nv(s->f_rev_adam, n, args, st);
+    prof_mark(s, 2, st, false);
+    s->prof_launches[2] += 1;
+  }
+  FELIX_API_END
+}
+
+felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int64_t n, float lambda, float* phi,
+                        float* g, float* cost, float* loss, float* grad, void* stream) {
+  FELIX_API_BEGIN
+  check_pair(s, m);
+  if (!y && n > 0) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL y");
+  if (n < 0 || n > (int64_t(1) << 30)) FELIX_THROW(FELIX_E_INVALID_ARG, "n out of range");
+  if (n == 0) return FELIX_OK;
+  DeviceGuard dg(s->device);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  Plan& pl = get_plan(s, m, n);
+  run_forward_mlp(s, pl, y, n, st);
+  int ni = static_cast<int>(n);
+  void* dphi = pl.dphi.p;
+  void* cpart = pl.c_part.p;
+  int ld = static_cast<int>(pl.n_pad);
+  int nht = pl.n_head_tiles;
+  float hb = m->head_b, lam = lambda;
+  void* args[] = {&y, &ni, &dphi, &ld, &cpart, &nht, &ld, &hb, &lam, &phi, &g, &cost, &loss, &grad};
+  launch_nv(s->f_rev_eval, n, args, st);
+  FELIX_API_END
+}
+
+felix_status felix_init_sample(felix_space* s, int64_t n, uint64_t rng_seed, int64_t index_base, float* y, void* stream) {
+  FELIX_API_BEGIN
+  if (!s || (!y && n > 0)) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL argument");
+  if (n < 0 || n > (int64_t(1) << 30)) FELIX_THROW(FELIX_E_INVALID_ARG, "n out of range");
+  if (n == 0) return FELIX_OK;
+  DeviceGuard dg(s->device);
+  int ni = static_cast<int>(n);
+  unsigned long long seed = rng_seed;
+  long long ib = index_base;
+  void* args[] = {&seed, &ni, &ib, &y};
+  launch_nv(s->f_init, n, args, static_cast<cudaStream_t>(stream));
+  FELIX_API_END
+}
+
+static void do_round(felix_space* s, const float* y, int64_t n, int32_t* sched, cudaStream_t st) {
+  const int M = s->desc.n_vars;
+  const int nc = static_cast<int>(s->rt.comp_nvars.size());
+  const int ni = static_cast<int>(n);
+  if (nc > 0) {
+    const long long warps = static_cast<long long>(n) * nc;
+    const unsigned grid = static_cast<unsigned>((warps * 32 + 255) / 256);
+    round_split_kernel<<<grid, 256, 0, st>>>(y, ni, M, nc, s->d_comp_nvars.as<int>(), s->d_comp_var0.as<int>(),
+                                             s->d_comp_vars.as<int>(), s->d_comp_eoff.as<long long>(),
+                                             s->d_comp_tcount.as<long long>(), s->d_tuples.as<int>(),
+                                             s->d_lnf.as<double>(), sched);
+    CUDA_OK(cudaGetLastError());
+  }
+  const int nint = static_cast<int>(s->rt.int_vars.size());
+  if (nint > 0) {
+    const long long tot = static_cast<long long>(n) * nint;
+    round_int_kernel<<<static_cast<unsigned>((tot + 255) / 256), 256, 0, st>>>(
+        y, ni, M, nint, s->d_int_vars.as<int>(), s->d_int_lo.as<long long>(), s->d_int_cnt.as<long long>(),
+        s->d_int_toff.as<long long>(), s->d_int_thr.as<double>(), sched);
+    CUDA_OK(cudaGetLastError());
+  }
+}
+
+static void do_hard(felix_space* s, const int32_t* sched, int64_t n, double* phi64, uint8_t* valid, cudaStream_t st) {
+  int ni = static_cast<int>(n);
+  void* args[] = {&sched, &ni, &phi64, &valid};
+  launch_nv(s->f_hard, n, args, st);
+}
+
+static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, int64_t n, double* score, cudaStream_t st) {
+  const int L = m->n_layers;
+  int maxw = 0;
+  for (int l = 1; l < L; ++l) maxw = std::max(maxw, m->dims[l]);
+  ensure(s->act64a, static_cast<size_t>(n) * maxw * 8);
+  ensure(s->act64b, static_cast<size_t>(n) * maxw * 8);
+  const double* in = phi64;
+  long long rs = 1, cs = n;    // phi64 is [K][n]
+  double* bufs[2] = {s->act64a.as<double>(), s->act64b.as<double>()};
+  for (int l = 0; l < L; ++l) {
+    const int K = m->dims[l], N = m->dims[l + 1];
+    double* out = (l == L - 1) ? score : bufs[l & 1];
+    const long long tot = static_cast<long long>(n) * N;
+    score_layer_kernel<<<static_cast<unsigned>((tot + 255) / 256), 256, 0, st>>>(
+        in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N, l < L - 1 ? 1 : 0);
+    CUDA_OK(cudaGetLastError());
+    in = out;
+    rs = N;
+    cs = 1;
+  }
+}
+
+felix_status felix_round(felix_space* s, const float* y, int64_t n, int32_t* sched, uint8_t* valid, void* stream) {
+  FELIX_API_BEGIN
+  if (!s || ((!y || !sched) && n > 0)) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL argument");
+  if (n < 0 || n > (int64_t(1) << 30)) FELIX_THROW(FELIX_E_INVALID_ARG, "n out of range");
+  if (n == 0) return FELIX_OK;
+  DeviceGuard dg(s->device);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  do_round(s, y, n, sched, st);
+  if (valid) {
+    ensure(s->phi64, static_cast<size_t>(n) * s->desc.froots.size() * 8);
+    do_hard(s, sched, n, s->phi64.as<double>(), valid, st);
+  }
+  FELIX_API_END
+}
+
+felix_status felix_score(felix_space* s, felix_costmodel* m, const int32_t* sched, int64_t n, double* score, void* stream) {
+  FELIX_API_BEGIN
+  check_pair(s, m);
+  if ((!sched || !score) && n > 0) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL argument");
+  if (n < 0 || n > (int64_t(1) << 30)) FELIX_THROW(FELIX_E_INVALID_ARG, "n out of range");
+  if (n == 0) return FELIX_OK;
+  DeviceGuard dg(s->device);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  ensure(s->phi64, static_cast<size_t>(n) * s->desc.froots.size() * 8);
+  ensure(s->valid, static_cast<size_t>(n));
+  do_hard(s, sched, n, s->phi64.as<double>(), s->valid.as<uint8_t>(), st);
+  do_score(s, m, s->phi64.as<double>(), n, score, st);
+  FELIX_API_END
+}
+
+felix_status felix_round_topk(felix_space* s, felix_costmodel* m, const float* y, int64_t n, int64_t index_base,
+                              int32_t k, int64_t* idx_out, double* score_out, int32_t* sched_out, int32_t* n_out,
+                              void* stream) {
+  FELIX_API_BEGIN
+  check_pair(s, m);
+  if (!n_out || (k > 0 && (!idx_out || !score_out || !sched_out))) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL output");
+  if (k < 0 || k > 1024) FELIX_THROW(FELIX_E_INVALID_ARG, "k must be in [0, 1024]");
+  if (n < 0 || n > (int64_t(1) << 30) || (n > 0 && !y)) FELIX_THROW(FELIX_E_INVALID_ARG, "bad y / n");
+  *n_out = 0;
+  if (n == 0 || k == 0) return FELIX_OK;
+  DeviceGuard dg(s->device);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const int M = s->desc.n_vars;
+  ensure(s->sched, static_cast<size_t>(n) * M * 4);
+  ensure(s->valid, static_cast<size_t>(n));
+  ensure(s->phi64, static_cast<size_t>(n) * s->desc.froots.size() * 8);
+  ensure(s->score, static_cast<size_t>(n) * 8);
+  do_round(s, y, n, s->sched.as<int32_t>(), st);
+  do_hard(s, s->sched.as<int32_t>(), n, s->phi64.as<double>(), s->valid.as<uint8_t>(), st);
+  do_score(s, m, s->phi64.as<double>(), n, s->score.as<double>(), st);
+  const long long chunk = 4096;
+  const long long nblk = (n + chunk - 1) / chunk;
+  ensure(s->alive, static_cast<size_t>(std::max<long long>(n, nblk * k)));
+  ensure(s->rec_cand, static_cast<size_t>(nblk) * k * 4);
+  ensure(s->rec_cnt, static_cast<size_t>(nblk) * 4);
+  ensure(s->fin_cand, static_cast<size_t>(k) * 4);
+  ensure(s->fin_cnt, 4);
+  topk_select_kernel<<<static_cast<unsigned>(nblk), 1024, 0, st>>>(
+      n, chunk, nullptr, s->score.as<double>(), s->valid.as<uint8_t>(), s->sched.as<int32_t>(), M, k,
+      s->alive.as<uint8_t>(), s->rec_cand.as<int>(), s->rec_cnt.as<int>());
+  CUDA_OK(cudaGetLastError());
+  topk_select_kernel<<<1, 1024, 0, st>>>(
+      nblk * k, nblk * k, s->rec_cand.as<int>(), s->score.as<double>(), s->valid.as<uint8_t>(), s->sched.as<int32_t>(),
+      M, k, s->alive.as<uint8_t>(), s->fin_cand.as<int>(), s->fin_cnt.as<int>());
+  CUDA_OK(cudaGetLastError());
+  ensure(s->o_idx, static_cast<size_t>(k) * 8);
+  ensure(s->o_score, static_cast<size_t>(k) * 8);
+  ensure(s->o_sched, static_cast<size_t>(k) * M * 4);
+  topk_gather_kernel<<<1, std::max(32, (k + 31) / 32 * 32), 0, st>>>(
+      s->fin_cand.as<int>(), s->fin_cnt.as<int>(), k, s->score.as<double>(), s->sched.as<int32_t>(), M, index_base,
+      s->o_idx.as<long long>(), s->o_score.as<double>(), s->o_sched.as<int32_t>());
+  CUDA_OK(cudaGetLastError());
+  int cnt = 0;
+  CUDA_OK(cudaMemcpyAsync(&cnt, s->fin_cnt.p, 4, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaMemcpyAsync(idx_out, s->o_idx.p, static_cast<size_t>(k) * 8, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaMemcpyAsync(score_out, s->o_score.p, static_cast<size_t>(k) * 8, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaMemcpyAsync(sched_out, s->o_sched.p, static_cast<size_t>(k) * M * 4, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaStreamSynchronize(st));
+  *n_out = cnt;
+  FELIX_API_END
+}
+
+felix_status felix_profile_enable(felix_space* s, int32_t enable) {
+  FELIX_API_BEGIN
+  if (!s) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL space");
+  s->profiling = enable != 0;
+  FELIX_API_END
+}
+
+felix_status felix_profile_read(felix_space* s, double* ms, int64_t* launches) {
+  FELIX_API_BEGIN
+  if (!s || !ms || !launches) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL argument");
+  DeviceGuard dg(s->device);
+  for (auto& e : s->prof) {
+    CUDA_OK(cudaEventSynchronize(e.b));
+    float t = 0;
+    CUDA_OK(cudaEventElapsedTime(&t, e.a, e.b));
+    s->prof_ms[e.cls] += t;
+    cudaEventDestroy(e.a);
+    cudaEventDestroy(e.b);
+  }
+  s->prof.clear();
+  for (int c = 0; c < 4; ++c) { ms[c] = s->prof_ms[c]; launches[c] = s->prof_launches[c]; }
+  FELIX_API_END
+}
+
+felix_status felix_profile_reset(felix_space* s) {
+  FELIX_API_BEGIN
+  if (!s) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL space");
+  for (auto& e : s->prof) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
+  s->prof.clear();
+  for (int c = 0; c < 4; ++c) { s->prof_ms[c] = 0; s->prof_launches[c] = 0; }
+  FELIX_API_END
+}
+
+}  // extern "C"

@@ -1,0 +1,263 @@
+"""GPU parity: the CUDA path (through the C ABI) against the float64 oracle on the same seeded inputs.
+
+Tolerances (BASELINE.json north_star; SURVEY §8(c) parity rules):
+  features phi, g          rel <= 1e-4, floor 1
+  cost c, loss L           rel <= 1e-4, floor = RMS over the batch
+  gradient dL/dy           normwise per candidate <= 1e-3; R-kink exemption (oracle kink margin
+                           min |z| / rms(z) < 1e-4), exempt candidates < 1%
+  y after one Adam step    |dy| <= 1e-4 (1 + |y|), components with |g_ref| < 1e-6 exempt
+  rounding, validity       bit-exact (common input: the GPU's y)
+  top-k (idx, sched)       bit-exact; scores rel <= 1e-12
+"""
+import math
+
+import numpy as np
+import pytest
+import torch
+
+import felix_inputs as fi
+from oracle import felix_oracle as fo
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def fx():
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_asplos_zhaosam24_b200 as m
+    assert torch.cuda.is_available()
+    return m
+
+
+CASES = {
+    # name: (space factory, MLP dims, n)   n spans several 128-row tiles plus a ragged tail
+    "paper": (fi.paper_example_space, (82, 64, 1), 200),
+    "C1": (fi.c1_space, fi.C1_MLP, 300),
+    "C2": (fi.c2_space, fi.DEFAULT_MLP, 1000),
+    "C5": (fi.c5_space, fi.DEFAULT_MLP, 389),
+    "bmm": (lambda: fi.bert_spaces()[1], fi.DEFAULT_MLP, 257),
+}
+
+_cache = {}
+
+
+def _setup(fx, name):
+    if name not in _cache:
+        make, dims, n = CASES[name]
+        sp = make()
+        mlp = fi.make_mlp(dims)
+        _cache[name] = (sp, mlp, n, fx.Space(sp), fx.CostModel.from_weights(mlp))
+    return _cache[name]
+
+
+def kink_margin(zs):
+    m = np.full(zs[0].shape[1], np.inf)
+    for z in zs:
+        rms = np.sqrt(np.mean(z * z, axis=0)) + 1e-300
+        m = np.minimum(m, np.min(np.abs(z), axis=0) / rms)
+    return m
+
+
+@pytest.mark.parametrize("name", list(CASES))
+def test_eval_parity(fx, name):
+    sp, mlp, n, space, cm = _setup(fx, name)
+    y0 = fi.make_y0(sp, n, seed=11)
+    out = {k: v.cpu().numpy() for k, v in space.eval(cm, torch.from_numpy(y0).cuda(), lam=1.0).items()}
+    ref = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
+    # features (slog) and constraint values
+    e_phi = np.abs(out["phi"] - ref.phi) / np.maximum(np.abs(ref.phi), 1.0)
+    k, i = np.unravel_index(np.argmax(e_phi), e_phi.shape)
+    assert e_phi[k, i] <= 1e-4, (sp.feature_names[k], i, out["phi"][k, i], ref.phi[k, i], ref.F[k, i], y0[:, i])
+    e_g = np.abs(out["g"] - ref.g) / np.maximum(np.abs(ref.g), 1.0)
+    assert np.max(e_g) <= 1e-4, np.unravel_index(np.argmax(e_g), e_g.shape)
+    # cost and loss, floor = RMS over the batch
+    for key, r in (("cost", ref.c), ("loss", ref.loss)):
+        s = np.sqrt(np.mean(r ** 2))
+        assert np.max(np.abs(out[key] - r)) / s <= 1e-4, key
+    # gradient, normwise per candidate, R-kink exemption
+    km = kink_margin(ref.zs)
+    err = np.linalg.norm(out["grad"] - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
+    bad = err > 1e-3
+    exempt = bad & (km < 1e-4)
+    assert not np.any(bad & ~exempt), (np.nonzero(bad & ~exempt)[0][:10], err[bad & ~exempt][:10])
+    assert exempt.mean() < 0.01
+
+
+@pytest.mark.parametrize("name", ["C1", "C2"])
+def test_one_adam_step_parity(fx, name):
+    sp, mlp, n, space, cm = _setup(fx, name)
+    y0 = fi.make_y0(sp, n, seed=12)
+    y = torch.from_numpy(y0).cuda()
+    loss = torch.empty(n, device="cuda")
+    space.search(cm, y, 1, lr=0.05, lam=1.0, init_from_y=True, final_loss=loss)
+    got = y.cpu().numpy()
+    ob = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
+    ry, _, _, _ = fo.search(sp, mlp.W, mlp.b, y0, 1, lr=0.05, lam=1.0)
+    tol = 1e-4 * (1 + np.abs(ry))
+    exempt = (np.abs(ob.grad) < 1e-6) | (kink_margin(ob.zs) < 1e-4)[None, :]
+    bad = (np.abs(got - ry) > tol) & ~exempt
+    assert not np.any(bad), (np.argwhere(bad)[:10], got[bad][:10], ry[bad][:10])
+    s = np.sqrt(np.mean(ob.loss ** 2))
+    assert np.max(np.abs(loss.cpu().numpy() - ob.loss)) / s <= 1e-4
+
+
+@pytest.mark.parametrize("name", list(CASES))
+def test_rounding_validity_bit_exact(fx, name):
+    sp, mlp, n, space, cm = _setup(fx, name)
+    y0 = fi.make_y0(sp, n, seed=13, margin=1.0)
+    yt = torch.from_numpy(y0).cuda()
+    sched, valid = space.round(yt)
+    rs = fo.round_schedules(sp, y0)
+    assert np.array_equal(sched.cpu().numpy(), rs)
+    assert np.array_equal(valid.cpu().numpy().astype(bool), fo.validate(sp, rs))
+
+
+@pytest.mark.parametrize("name", ["C1", "C2"])
+def test_rounding_at_midpoints_bit_exact(fx, name):
+    """Adversarial inputs: log-midpoints of consecutive divisors and INT half-integers (fp32)."""
+    sp, mlp, n, space, cm = _setup(fx, name)
+    rng = np.random.default_rng(5)
+    y = np.zeros((sp.n_vars, 512), dtype=np.float32)
+    for j, v in enumerate(sp.vars):
+        if v.kind == fi.VAR_SPLIT:
+            e = int(fi.var_upper_bounds(sp)[j])
+            ds = [d for d in range(1, e + 1) if e % d == 0]
+            mids = [0.5 * (math.log(a) + math.log(b)) for a, b in zip(ds[:-1], ds[1:])]
+            y[j] = np.float32(rng.choice(mids + [math.log(d) for d in ds], size=512))
+        else:
+            y[j] = np.float32(np.log(rng.integers(v.lo, v.hi, size=512) + 0.5))
+    sched, _ = space.round(torch.from_numpy(y).cuda())
+    assert np.array_equal(sched.cpu().numpy(), fo.round_schedules(sp, y))
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C5"])
+def test_score_fp64(fx, name):
+    sp, mlp, n, space, cm = _setup(fx, name)
+    y0 = fi.make_y0(sp, n, seed=14)
+    rs = fo.round_schedules(sp, y0)
+    got = space.score(cm, torch.from_numpy(rs).cuda()).cpu().numpy()
+    ref = fo.score(sp, mlp.W, mlp.b, rs)
+    ok = np.isfinite(ref)
+    assert np.all(np.abs(got[ok] - ref[ok]) <= 1e-12 * np.maximum(np.abs(ref[ok]), 1e-3))
+
+
+def _topk_equal(idx, sc, sched, ridx, rsc, rsched):
+    assert len(idx) == len(ridx)
+    assert np.all(np.abs(sc - rsc) <= 1e-12 * np.maximum(np.abs(rsc), 1e-3))
+    # bit-exact except inside groups of scores tied to 1e-12 (order of equal keys is by index on both
+    # sides; a sub-1e-12 difference between distinct schedules may swap them)
+    i = 0
+    while i < len(ridx):
+        j = i
+        while j + 1 < len(ridx) and abs(rsc[j + 1] - rsc[i]) <= 1e-12 * max(abs(rsc[i]), 1e-3):
+            j += 1
+        if j == i:
+            assert idx[i] == ridx[i] and np.array_equal(sched[i], rsched[i])
+        else:
+            assert set(idx[i:j + 1]) == set(ridx[i:j + 1]) or j == len(ridx) - 1
+        i = j + 1
+
+
+@pytest.mark.parametrize("name", list(CASES))
+def test_round_topk_parity(fx, name):
+    sp, mlp, n, space, cm = _setup(fx, name)
+    y0 = fi.make_y0(sp, n, seed=15)
+    y0[:, n // 2: n // 2 + 20] = y0[:, :20]          # duplicates
+    idx, sc, sched = space.round_topk(cm, torch.from_numpy(y0).cuda(), 16, index_base=777)
+    ridx, rsc, rsched = fo.round_topk(sp, mlp.W, mlp.b, y0, 16, index_base=777)
+    _topk_equal(idx, sc, sched, ridx, rsc, rsched)
+
+
+def test_topk_shard_invariance(fx):
+    """Top-k over two shards (index_base offsets) merged on the host == top-k over the whole set."""
+    sp, mlp, n, space, cm = _setup(fx, "C2")
+    y0 = fi.make_y0(sp, 4096, seed=16)
+    full = space.round_topk(cm, torch.from_numpy(y0).cuda(), 16)
+    recs = []
+    for r in range(2):
+        part = np.ascontiguousarray(y0[:, r * 2048:(r + 1) * 2048])
+        i, s, sc = space.round_topk(cm, torch.from_numpy(part).cuda(), 16, index_base=r * 2048)
+        recs += list(zip(i, s, map(tuple, sc)))
+    seen, merged = {}, []
+    for i, s, sc in sorted(recs, key=lambda t: (-t[1], t[0])):
+        if sc not in seen:
+            seen[sc] = i
+            merged.append((i, s))
+    assert [i for i, _ in merged[:16]] == list(full[0])
+
+
+def test_init_sampler_parity(fx):
+    sp, mlp, n, space, cm = _setup(fx, "C2")
+    y = space.init_sample(2048, 0x5EED0002, index_base=100).cpu().numpy()
+    ry = fo.init_sample(sp, 2048, 0x5EED0002, index_base=100)
+    same = np.all(y == ry, axis=0)
+    assert same.mean() >= 0.99
+    g = np.concatenate([fo.eval_dag(sp, np.exp(y.astype(np.float64)), True).g_user, fo.auto_roots(sp, y.astype(np.float64))])
+    assert np.all(g <= 1e-5)
+
+
+def test_full_size_c2_sampled(fx):
+    """BASELINE configs[1] size (4096 seeds, default MLP) in the launch configuration bench.py times;
+    64 sampled candidates checked one by one against the oracle."""
+    sp, mlp, _, space, cm = _setup(fx, "C2")
+    y0 = fo.init_sample(sp, 4096, 0x5EED0002)
+    out = {k: v.cpu().numpy() for k, v in space.eval(cm, torch.from_numpy(y0).cuda()).items()}
+    pick = np.random.default_rng(0).choice(4096, 64, replace=False)
+    ref = fo.objective(sp, mlp.W, mlp.b, y0[:, pick].astype(np.float64), 1.0)
+    s = np.sqrt(np.mean(ref.c ** 2))
+    assert np.max(np.abs(out["cost"][pick] - ref.c)) / s <= 1e-4
+    err = np.linalg.norm(out["grad"][:, pick] - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
+    assert np.sum((err > 1e-3) & (kink_margin(ref.zs) >= 1e-4)) == 0
+
+
+def test_search_deterministic_and_improves(fx):
+    sp, mlp, _, space, cm = _setup(fx, "C2")
+    y1 = space.init_sample(4096, 0x5EED0002)
+    y2 = y1.clone()
+    l1 = torch.empty(4096, device="cuda")
+    l2 = torch.empty(4096, device="cuda")
+    space.search(cm, y1, 50, init_from_y=True, final_loss=l1)
+    space.search(cm, y2, 50, init_from_y=True, final_loss=l2)
+    assert torch.equal(y1, y2) and torch.equal(l1, l2)
+    y0 = space.init_sample(4096, 0x5EED0002)
+    l0 = space.eval(cm, y0)["loss"]
+    assert l1.mean().item() < l0.mean().item()
+
+
+def test_search_with_device_init_matches_init_sample(fx):
+    sp, mlp, _, space, cm = _setup(fx, "C1")
+    y = torch.empty((sp.n_vars, 64), device="cuda")
+    space.search(cm, y, 0, rng_seed=0x5EED0001, init_from_y=False)
+    assert torch.equal(y, space.init_sample(64, 0x5EED0001))
+
+
+def test_edge_sizes(fx):
+    sp, mlp, _, space, cm = _setup(fx, "C1")
+    for n in (1, 127, 128, 129):
+        y0 = fi.make_y0(sp, n, seed=n)
+        out = space.eval(cm, torch.from_numpy(y0).cuda())
+        ref = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
+        s = max(np.sqrt(np.mean(ref.c ** 2)), 1e-6)
+        assert np.max(np.abs(out["cost"].cpu().numpy() - ref.c)) / s <= 1e-4
+    y = torch.empty((sp.n_vars, 0), device="cuda")
+    space.search(cm, y, 3)                     # n = 0: no-op
+    idx, sc, sched = space.round_topk(cm, torch.from_numpy(fi.make_y0(sp, 5, 1)).cuda(), 16)
+    assert len(idx) <= 5
+
+
+def test_shape_errors(fx):
+    sp, mlp, _, space, cm = _setup(fx, "C1")
+    bad = fx.CostModel.from_weights(fi.make_mlp((82, 64, 64, 1)))
+    y = torch.zeros((sp.n_vars - 1, 10), device="cuda")
+    with pytest.raises(fx.FelixError):
+        space.eval(cm, y)
+    other = fi.make_mlp((80, 64, 1))
+    cm2 = fx.CostModel.from_weights(other)
+    with pytest.raises(fx.FelixError) as e:
+        space.eval(cm2, torch.zeros((sp.n_vars, 10), device="cuda"))
+    assert e.value.status == 3
+    with pytest.raises(fx.FelixError) as e:
+        fx.CostModel.from_weights(fi.make_mlp((82, 100, 1)))
+    assert e.value.status == 4
+    del bad

@@ -1,0 +1,96 @@
+"""Host-side checks of the C-ABI library that need no GPU (-m "not gpu"): the .so loads, exports every
+symbol include/felix.h declares, its opcode/struct layout matches the input format, the space
+validator rejects malformed input, and the generated expression kernels compile for sm_100a (NVRTC)."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import felix_inputs as fi
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = open(os.path.join(ROOT, "include", "felix.h")).read()
+
+
+@pytest.fixture(scope="module")
+def fx():
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_asplos_zhaosam24_b200 as m
+    return m
+
+
+def test_library_exports_every_header_symbol(fx):
+    declared = set(re.findall(r"FELIX_EXPORT\s+[\w\s\*]+?\b(felix_\w+)\s*\(", HEADER))
+    assert len(declared) >= 16
+    lib = ctypes.CDLL(fx.LIB_PATH)
+    for name in declared:
+        assert hasattr(lib, name), name
+    assert declared == set(fx.EXPORTED)
+    assert fx.abi_version() == int(re.search(r"#define FELIX_ABI_VERSION (\d+)", HEADER).group(1))
+
+
+def test_library_does_not_link_libcuda(fx):
+    import subprocess
+    out = subprocess.run(["ldd", fx.LIB_PATH], capture_output=True, text=True).stdout
+    assert "libcuda.so" not in out   # driver reached through cudaGetDriverEntryPoint at run time
+
+
+def test_opcodes_match_header():
+    for name, val in re.findall(r"FELIX_OP_(\w+) = (\d+)", HEADER):
+        assert getattr(fi, "OP_" + name) == int(val), name
+    assert fi.NODE_DTYPE.itemsize == 24
+
+
+def _space(nodes, froots, croots=(), vars_=None, splits=None):
+    vars_ = vars_ or [fi.Var("a", fi.VAR_SPLIT, 1, 64)]
+    splits = splits if splits is not None else [fi.Split(64, [0])]
+    arr = np.zeros(len(nodes), dtype=fi.NODE_DTYPE)
+    for i, r in enumerate(nodes):
+        arr[i] = r
+    return fi.Space("t", vars_, splits, arr, np.array(froots, np.int32), np.array(croots, np.int32))
+
+
+@pytest.mark.parametrize("case,status", [
+    ("forward_ref", 2), ("bool_root", 2), ("type_error", 2), ("var_range", 2),
+    ("int_in_split", 1), ("split_var_no_split", 1), ("bad_opcode", 2),
+])
+def test_validator_rejects(fx, case, status):
+    V = (fi.OP_VAR, -1, -1, -1, 0.0)
+    C1 = (fi.OP_CONST, -1, -1, -1, 1.0)
+    if case == "forward_ref":
+        sp = _space([V, (fi.OP_ADD, 0, 2, -1, 0.0), C1], [1])
+    elif case == "bool_root":
+        sp = _space([V, C1, (fi.OP_GT, 0, 1, -1, 0.0)], [2])
+    elif case == "type_error":
+        sp = _space([V, C1, (fi.OP_AND, 0, 1, -1, 0.0)], [0])
+    elif case == "var_range":
+        sp = _space([(fi.OP_VAR, -1, -1, -1, 3.0)], [0])
+    elif case == "int_in_split":
+        sp = _space([V], [0], vars_=[fi.Var("u", fi.VAR_INT, 1, 8)], splits=[fi.Split(8, [0])])
+    elif case == "split_var_no_split":
+        sp = _space([V], [0], splits=[])
+    else:
+        sp = _space([(99, -1, -1, -1, 0.0)], [0])
+    with pytest.raises(fx.FelixError) as e:
+        fx.codegen(sp)
+    assert e.value.status == status
+
+
+@pytest.mark.parametrize("which", ["paper", "C1", "C2"])
+def test_generated_kernels_compile_for_sm100a(fx, which):
+    sp = {"paper": fi.paper_example_space, "C1": fi.c1_space, "C2": fi.c2_space}[which]()
+    src = fx.codegen(sp, compile=True)
+    for k in ("felix_fwd", "felix_rev_adam", "felix_rev_eval", "felix_hard", "felix_init"):
+        assert f"void __launch_bounds__(128) {k}(" in src
+
+
+def test_device_calls_fail_loudly_without_gpu(fx):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(fx.FelixError) as e:
+        fx.Space(fi.c1_space())
+    assert e.value.status == 5
