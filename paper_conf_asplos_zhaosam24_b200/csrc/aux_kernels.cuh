@@ -72,18 +72,48 @@ __global__ void round_int_kernel(const float* __restrict__ y, int n, int M, int 
 }
 
 // ---------------------------------------------------------------------------- K6 FP64 MLP scoring
-// out[row][col] = act( b[col] + sum_k W[col][k] * in(row, k) ), fixed k order (deterministic).
-__global__ void score_layer_kernel(const double* __restrict__ in, long long in_rs, long long in_cs, int n, int K,
-                                   const double* __restrict__ W, const double* __restrict__ b, double* __restrict__ out,
-                                   int N, int relu) {
-  const long long g = static_cast<long long>(blockIdx.x) * blockDim.x + threadIdx.x;
-  if (g >= static_cast<long long>(n) * N) return;
-  const int row = static_cast<int>(g / N), col = static_cast<int>(g % N);
-  const double* w = W + static_cast<size_t>(col) * K;
-  const double* x = in + static_cast<size_t>(row) * in_rs;
-  double z = b[col];
-  for (int k = 0; k < K; ++k) z = fma(w[k], x[static_cast<size_t>(k) * in_cs], z);
-  out[g] = (relu && !(z > 0.0)) ? 0.0 : z;
+// out[row][col] = act( b[col] + sum_k W[col][k] * in(row, k) ), k ascending (deterministic, so equal
+// schedules get bit-identical scores).  32x32 output tile per 256-thread block, K staged through
+// shared memory in chunks of 32; thread (tx, ty) owns column tx and rows ty*4 .. ty*4+3.
+__global__ void __launch_bounds__(256) score_layer_kernel(const double* __restrict__ in, long long in_rs, long long in_cs,
+                                                          int n, int K, const double* __restrict__ W,
+                                                          const double* __restrict__ b, double* __restrict__ out,
+                                                          int N, int relu) {
+  __shared__ double As[32][33];   // [k][row]
+  __shared__ double Bs[32][33];   // [k][col]
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * 32 + tx;
+  const int row0 = blockIdx.y * 32, col0 = blockIdx.x * 32;
+  const int col = col0 + tx;
+  double acc[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) acc[q] = (col < N) ? b[col] : 0.0;
+  for (int k0 = 0; k0 < K; k0 += 32) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int e = tid + q * 256;           // 1024 elements of each 32x32 tile
+      const int r = e & 31, kk = e >> 5;      // A: consecutive threads -> consecutive rows (SoA input)
+      const int gr = row0 + r, gk = k0 + kk;
+      As[kk][r] = (gr < n && gk < K) ? in[static_cast<size_t>(gr) * in_rs + static_cast<size_t>(gk) * in_cs] : 0.0;
+      const int c = e >> 5, kb = e & 31;      // B: consecutive threads -> consecutive k (row-major W)
+      const int gc = col0 + c, gkb = k0 + kb;
+      Bs[kb][c] = (gc < N && gkb < K) ? W[static_cast<size_t>(gc) * K + gkb] : 0.0;
+    }
+    __syncthreads();
+    const int kmax = min(32, K - k0);
+    for (int kk = 0; kk < kmax; ++kk) {
+      const double w = Bs[kk][tx];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) acc[q] = fma(w, As[kk][ty * 4 + q], acc[q]);
+    }
+    __syncthreads();
+  }
+  if (col < N) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int r = row0 + ty * 4 + q;
+      if (r < n) out[static_cast<size_t>(r) * N + col] = (relu && !(acc[q] > 0.0)) ? 0.0 : acc[q];
+    }
+  }
 }
 
 // ---------------------------------------------------------------------------- K7 dedup + top-k

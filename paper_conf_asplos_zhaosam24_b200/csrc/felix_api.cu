@@ -9,6 +9,7 @@
 #include <chrono>
 #include <cmath>
 #include <cstring>
+#include <cstdlib>
 #include <functional>
 #include <map>
 #include <mutex>
@@ -19,6 +20,7 @@
 #include <cudaTypedefs.h>
 #include "felix_internal.h"
 #include "mlp_gemm.cuh"
+#include "mlp_chain.cuh"
 #include "aux_kernels.cuh"
 
 namespace felix {
@@ -28,22 +30,49 @@ void set_error(const std::string& m) { g_last_error = m; }
 
 // ============================================================================ GEMM dispatch
 struct GemmLaunch {
-  int epi = 0, bn = 0;
-  CUtensorMap a_hi, a_lo, b_hi, b_lo;
+  int epi = 0, bn = 0, stages = 2;
+  CUtensorMap a_hi, a_lo, b_hi, b_lo, c_hi, c_lo;   // c: output tiles (TMA store), = next GEMM's A maps
+  const void* w_hi = nullptr;                         // B operand (weights) base pointers
+  const void* w_lo = nullptr;
   GemmArgs args{};
   dim3 grid;
 };
+
+// Programmatic dependent launch: the kernel's prologue (barrier init, TMEM alloc, descriptor
+// prefetch) overlaps the previous kernel's tail; griddepcontrol.wait orders the data accesses.
+static cudaLaunchAttribute g_pdl_attr = [] {
+  cudaLaunchAttribute a{};
+  a.id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  a.val.programmaticStreamSerializationAllowed = 1;
+  return a;
+}();
 
 template <int BN, int EPI>
 static void launch_gemm_t(const GemmLaunch& g, cudaStream_t st) {
   auto kern = mlp_gemm_kernel<BN, EPI>;
   static bool attr_set = false;   // per instantiation; devices share the same limit on one box
   if (!attr_set) {
-    CUDA_OK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, GemmCfg<BN>::SMEM_BYTES));
+    CUDA_OK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 GemmCfg<BN>::smem_bytes(GemmCfg<BN>::MAX_STAGES)));
     attr_set = true;
   }
-  kern<<<g.grid, 128, GemmCfg<BN>::SMEM_BYTES, st>>>(g.a_hi, g.a_lo, g.b_hi, g.b_lo, g.args);
-  CUDA_OK(cudaGetLastError());
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = g.grid;
+  cfg.blockDim = dim3(128);
+  cfg.dynamicSmemBytes = GemmCfg<BN>::smem_bytes(g.stages);
+  cfg.stream = st;
+  cfg.attrs = &g_pdl_attr;
+  cfg.numAttrs = 1;
+  CUDA_OK(cudaLaunchKernelEx(&cfg, kern, g.a_hi, g.a_lo, g.b_hi, g.b_lo, g.c_hi, g.c_lo, g.args, g.stages));
+}
+
+static int gemm_max_stages(int bn) {
+  switch (bn) {
+    case 64: return GemmCfg<64>::MAX_STAGES;
+    case 96: return GemmCfg<96>::MAX_STAGES;
+    case 128: return GemmCfg<128>::MAX_STAGES;
+    default: return GemmCfg<256>::MAX_STAGES;
+  }
 }
 
 static void launch_gemm(const GemmLaunch& g, cudaStream_t st) {
@@ -88,9 +117,51 @@ struct Plan {
   int64_t n = -1, n_pad = 0;
   DevBuf phi_hi, phi_lo;                                   // [n][K0p]
   std::vector<std::unique_ptr<DevBuf>> act_hi, act_lo, mask;  // per hidden layer l = 1..L-1
-  DevBuf c_part, dphi, m, v;
+  DevBuf c_part, dphi, m, v, step_ctr;
   int n_head_tiles = 0;
-  std::vector<GemmLaunch> gemms;
+  std::vector<GemmLaunch> gemms;           // per-layer kernels (FELIX_MLP=layers)
+  ChainParams chain{};                     // persistent all-layer kernel (default)
+  int chain_grid = 0;
+  DevBuf grid_bar;
+};
+
+static bool use_chain() {
+  const char* e = std::getenv("FELIX_MLP");
+  return !(e && std::string(e) == "layers");
+}
+
+static void launch_chain(const Plan& p, cudaStream_t st) {
+  static bool attr_set = false;
+  if (!attr_set) {
+    CUDA_OK(cudaFuncSetAttribute(mlp_chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES));
+    attr_set = true;
+  }
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(static_cast<unsigned>(p.chain_grid));
+  cfg.blockDim = dim3(CHAIN_THREADS);
+  cfg.dynamicSmemBytes = CHAIN_SMEM_BYTES;
+  cfg.stream = st;
+  cfg.attrs = &g_pdl_attr;
+  cfg.numAttrs = 1;
+  CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_chain_kernel, p.chain));
+}
+
+// The population split into K independent chunks, each with its own workspace (Plan).  One Adam
+// step of all chunks is captured as ONE CUDA graph with K parallel branches (fork/join), so one
+// chunk's tensor-core GEMMs overlap another chunk's latency-bound expression kernels.
+struct Chunks {
+  const CostModel* cm = nullptr;
+  int64_t n = -1;
+  int K = 0;
+  std::vector<int64_t> off, cnt;
+  std::vector<std::unique_ptr<Plan>> plans;
+  std::vector<cudaStream_t> streams;       // capture-time branch streams
+  cudaGraphExec_t graph = nullptr;
+  std::vector<double> graph_key;
+  ~Chunks() {
+    if (graph) cudaGraphExecDestroy(graph);
+    for (auto st : streams) cudaStreamDestroy(st);
+  }
 };
 
 struct ProfEvent { int cls; cudaEvent_t a, b; };
@@ -105,15 +176,19 @@ struct felix_space {
   // device copies of the rounding tables
   felix::DevBuf d_comp_nvars, d_comp_var0, d_comp_vars, d_comp_eoff, d_comp_tcount, d_tuples, d_lnf;
   felix::DevBuf d_int_vars, d_int_lo, d_int_cnt, d_int_toff, d_int_thr;
-  // NVRTC module
-  cudaLibrary_t module = nullptr;
-  cudaKernel_t f_fwd = nullptr, f_rev_adam = nullptr, f_rev_eval = nullptr, f_hard = nullptr, f_init = nullptr;
+  // NVRTC modules, one per cone-partition width P (compiled on first use)
+  struct Module {
+    cudaLibrary_t lib = nullptr;
+    cudaKernel_t f_fwd = nullptr, f_rev_adam = nullptr, f_rev_eval = nullptr, f_hard = nullptr, f_init = nullptr;
+    int P = 1, rev_smem = 0, regs_fwd = 0, regs_rev = 0;
+    std::string source;
+  };
+  std::map<int, Module> modules;
   double nvrtc_ms = 0;
   int regs_fwd = 0, regs_rev = 0;
   int64_t flops_fwd = 0;
-  std::string source;
-  // plan cache + scratch
-  std::unique_ptr<felix::Plan> plan;
+  // workspace caches (search: chunked; eval: one chunk) + scratch
+  std::unique_ptr<felix::Chunks> search_chunks, eval_chunks;
   felix::DevBuf sched, valid, phi64, score, act64a, act64b, alive, rec_cand, rec_cnt, fin_cand, fin_cnt, o_idx, o_score, o_sched;
   // profiling
   bool profiling = false;
@@ -122,7 +197,7 @@ struct felix_space {
   int64_t prof_launches[4] = {0, 0, 0, 0};
   ~felix_space() {
     for (auto& e : prof) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
-    if (module) cudaLibraryUnload(module);
+    for (auto& kv : modules) if (kv.second.lib) cudaLibraryUnload(kv.second.lib);
   }
 };
 
@@ -271,42 +346,73 @@ static std::vector<char> nvrtc_compile(const std::string& source) {
   return cubin;
 }
 
-static void compile_module(felix_space* s) {
+static felix_space::Module& get_module(felix_space* s, int P) {
+  auto it = s->modules.find(P);
+  if (it != s->modules.end()) return it->second;
+  felix_space::Module mod;
+  mod.P = P;
   CodegenInfo info;
-  s->source = generate_dag_module(s->desc, s->K0p, &info);
+  mod.source = generate_dag_module(s->desc, s->K0p, P, &info);
   s->flops_fwd = info.flops_fwd;
+  mod.rev_smem = info.rev_smem_bytes;
   auto t0 = std::chrono::steady_clock::now();
-  std::vector<char> cubin = nvrtc_compile(s->source);
-  CUDA_OK(cudaLibraryLoadData(&s->module, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0));
-  CUDA_OK(cudaLibraryGetKernel(&s->f_fwd, s->module, "felix_fwd"));
-  CUDA_OK(cudaLibraryGetKernel(&s->f_rev_adam, s->module, "felix_rev_adam"));
-  CUDA_OK(cudaLibraryGetKernel(&s->f_rev_eval, s->module, "felix_rev_eval"));
-  CUDA_OK(cudaLibraryGetKernel(&s->f_hard, s->module, "felix_hard"));
-  CUDA_OK(cudaLibraryGetKernel(&s->f_init, s->module, "felix_init"));
+  std::vector<char> cubin = nvrtc_compile(mod.source);
+  CUDA_OK(cudaLibraryLoadData(&mod.lib, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0));
+  CUDA_OK(cudaLibraryGetKernel(&mod.f_fwd, mod.lib, "felix_fwd"));
+  CUDA_OK(cudaLibraryGetKernel(&mod.f_rev_adam, mod.lib, "felix_rev_adam"));
+  CUDA_OK(cudaLibraryGetKernel(&mod.f_rev_eval, mod.lib, "felix_rev_eval"));
+  CUDA_OK(cudaLibraryGetKernel(&mod.f_hard, mod.lib, "felix_hard"));
+  CUDA_OK(cudaLibraryGetKernel(&mod.f_init, mod.lib, "felix_init"));
+  for (cudaKernel_t k : {mod.f_rev_adam, mod.f_rev_eval})
+    CUDA_OK(cudaFuncSetAttribute(reinterpret_cast<const void*>(k), cudaFuncAttributeMaxDynamicSharedMemorySize, mod.rev_smem));
   cudaFuncAttributes fa{};
-  CUDA_OK(cudaFuncGetAttributes(&fa, reinterpret_cast<const void*>(s->f_fwd)));
-  s->regs_fwd = fa.numRegs;
-  CUDA_OK(cudaFuncGetAttributes(&fa, reinterpret_cast<const void*>(s->f_rev_adam)));
-  s->regs_rev = fa.numRegs;
-  s->nvrtc_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  CUDA_OK(cudaFuncGetAttributes(&fa, reinterpret_cast<const void*>(mod.f_fwd)));
+  mod.regs_fwd = fa.numRegs;
+  CUDA_OK(cudaFuncGetAttributes(&fa, reinterpret_cast<const void*>(mod.f_rev_adam)));
+  mod.regs_rev = fa.numRegs;
+  s->nvrtc_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  s->regs_fwd = mod.regs_fwd;
+  s->regs_rev = mod.regs_rev;
+  return s->modules.emplace(P, std::move(mod)).first->second;
 }
 
-static void launch_nv(cudaKernel_t f, int64_t n, void** args, cudaStream_t st) {
+// Cone-partition width: enough warps to give every SM ~8 resident warps of expression work.
+static int choose_P(int64_t n) {
+  const int64_t target = int64_t(148) * 8 * 32;
+  int P = 1;
+  while (P < 8 && n * P < target) P *= 2;
+  return P;
+}
+
+// Launch helpers.  Search kernels: CTA = P warps x 32 candidates (cone partition); hard / sampler
+// kernels: one candidate per thread, 128-thread CTAs.
+static void launch_cfg(const void* f, dim3 grid, dim3 block, size_t smem, void** args, cudaStream_t st, bool pdl) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  if (pdl) { cfg.attrs = &g_pdl_attr; cfg.numAttrs = 1; }
+  CUDA_OK(cudaLaunchKernelExC(&cfg, f, args));
+}
+static void launch_grouped(cudaKernel_t f, int P, int64_t n, size_t smem, void** args, cudaStream_t st, bool pdl) {
   if (n <= 0) return;
-  const unsigned grid = static_cast<unsigned>((n + 127) / 128);
-  CUDA_OK(cudaLaunchKernel(reinterpret_cast<const void*>(f), dim3(grid), dim3(128), args, 0, st));
+  launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((n + 31) / 32)), dim3(32 * P), smem, args, st, pdl);
+}
+static void launch_flat(cudaKernel_t f, int64_t n, void** args, cudaStream_t st) {
+  if (n <= 0) return;
+  launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((n + 127) / 128)), dim3(128), 0, args, st, false);
 }
 
 // ============================================================================ plan
 static int choose_bn(int64_t m_tiles, int N) {
   // prefer >= one full wave of CTAs (148 SMs) before larger tiles
-  if (N % 128 == 0 && m_tiles * (N / 128) >= 148) return 128;
+  if (N % 128 == 0 && m_tiles * (N / 128) >= 2 * 148) return 128;
   if (N % 64 == 0) return 64;
   FELIX_THROW(FELIX_E_UNSUPPORTED, "hidden dim must be a multiple of 64");
 }
 
-static Plan& get_plan(felix_space* s, const CostModel* cm, int64_t n) {
-  if (s->plan && s->plan->cm == cm && s->plan->n == n) return *s->plan;
+static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int64_t n) {
   auto p = std::make_unique<Plan>();
   p->cm = cm;
   p->n = n;
@@ -333,6 +439,7 @@ static Plan& get_plan(felix_space* s, const CostModel* cm, int64_t n) {
   p->dphi.alloc(static_cast<size_t>(K0p) * np * 4);
   p->m.alloc(static_cast<size_t>(s->desc.n_vars) * n * 4);
   p->v.alloc(static_cast<size_t>(s->desc.n_vars) * n * 4);
+  p->step_ctr.alloc(16);
   const int64_t mt = np / 128;
   // forward GEMMs, layer l = 1..L-1 (W index l-1)
   for (int l = 1; l <= L - 1; ++l) {
@@ -345,8 +452,12 @@ static Plan& get_plan(felix_space* s, const CostModel* cm, int64_t n) {
     const void* a_lo = (l == 1) ? p->phi_lo.p : p->act_lo[l - 1]->p;
     g.a_hi = make_tmap(a_hi, n, Kdim, 128);
     g.a_lo = make_tmap(a_lo, n, Kdim, 128);
-    g.b_hi = make_tmap(cm->W_hi[l - 1]->p, N, Kdim, g.bn);
-    g.b_lo = make_tmap(cm->W_lo[l - 1]->p, N, Kdim, g.bn);
+    g.w_hi = cm->W_hi[l - 1]->p;
+    g.w_lo = cm->W_lo[l - 1]->p;
+    g.b_hi = make_tmap(g.w_hi, N, Kdim, g.bn);
+    g.b_lo = make_tmap(g.w_lo, N, Kdim, g.bn);
+    g.c_hi = make_tmap(p->act_hi[l]->p, n, N, 128);
+    g.c_lo = make_tmap(p->act_lo[l]->p, n, N, 128);
     GemmArgs& a = g.args;
     a.M = static_cast<int>(n); a.N = N; a.K = Kdim;
     a.bias = cm->bias[l - 1]->as<float>();
@@ -356,13 +467,14 @@ static Plan& get_plan(felix_space* s, const CostModel* cm, int64_t n) {
     if (head) {
       a.head_w = cm->head_w.as<float>();
       p->n_head_tiles = N / g.bn;
-      p->c_part.alloc(static_cast<size_t>(p->n_head_tiles) * np * 4);
+      p->c_part.alloc(static_cast<size_t>(N / 32) * np * 4);      // room for any partial width >= 32
       a.c_part = p->c_part.as<float>();
       a.ld_c = static_cast<int>(np);
     } else {
       a.mask_out = p->mask[l]->as<uint32_t>();
     }
     g.grid = dim3(static_cast<unsigned>(mt), N / g.bn);
+    g.stages = std::min(gemm_max_stages(g.bn), (Kdim + GEMM_BK - 1) / GEMM_BK);
     p->gemms.push_back(g);
   }
   // backward GEMMs: delta_{l-1} = (delta_l W_l) (.) m_{l-1} for l = L-1..2, then dphi = delta_1 W_1
@@ -374,10 +486,14 @@ static Plan& get_plan(felix_space* s, const CostModel* cm, int64_t n) {
     g.bn = last ? K0p : choose_bn(mt, N);
     g.a_hi = make_tmap(p->act_hi[l]->p, n, Kdim, 128);
     g.a_lo = make_tmap(p->act_lo[l]->p, n, Kdim, 128);
-    g.b_hi = make_tmap(cm->WT_hi[l - 1]->p, N, Kdim, g.bn);
-    g.b_lo = make_tmap(cm->WT_lo[l - 1]->p, N, Kdim, g.bn);
+    g.w_hi = cm->WT_hi[l - 1]->p;
+    g.w_lo = cm->WT_lo[l - 1]->p;
+    g.b_hi = make_tmap(g.w_hi, N, Kdim, g.bn);
+    g.b_lo = make_tmap(g.w_lo, N, Kdim, g.bn);
     GemmArgs& a = g.args;
     a.M = static_cast<int>(n); a.N = N; a.K = Kdim;
+    g.c_hi = last ? g.a_hi : make_tmap(p->act_hi[l - 1]->p, n, N, 128);
+    g.c_lo = last ? g.a_lo : make_tmap(p->act_lo[l - 1]->p, n, N, 128);
     if (last) {
       a.out_f32 = p->dphi.as<float>();
       a.ld_f32 = static_cast<int>(np);
@@ -389,10 +505,68 @@ static Plan& get_plan(felix_space* s, const CostModel* cm, int64_t n) {
       a.mask_in = p->mask[l - 1]->as<uint32_t>();
     }
     g.grid = dim3(static_cast<unsigned>(mt), N / g.bn);
+    g.stages = std::min(gemm_max_stages(g.bn), (Kdim + GEMM_BK - 1) / GEMM_BK);
     p->gemms.push_back(g);
   }
-  s->plan = std::move(p);
-  return *s->plan;
+  // persistent chain: same layers, BN <= 128, one CTA per SM
+  int sms = 148;
+  CUDA_OK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, s->device));
+  if (static_cast<int>(p->gemms.size()) > CHAIN_MAX_LAYERS) FELIX_THROW(FELIX_E_UNSUPPORTED, "too many MLP layers");
+  p->chain.n_layers = static_cast<int>(p->gemms.size());
+  p->chain.m_tiles = static_cast<int>(mt);
+  p->grid_bar.alloc(64);
+  CUDA_OK(cudaMemset(p->grid_bar.p, 0, 64));
+  p->chain.grid_bar = p->grid_bar.as<unsigned int>();
+  int max_tiles = 1;
+  for (size_t i = 0; i < p->gemms.size(); ++i) {
+    const GemmLaunch& g = p->gemms[i];
+    ChainLayer& L = p->chain.layer[i];
+    L.args = g.args;
+    L.epi = g.epi;
+    const int N = g.args.N;
+    int bn = g.bn;
+    if (g.epi == EPI_F32T) bn = g.bn;                                   // K0p (<= 128 required)
+    else bn = (N % 128 == 0 && mt * (N / 128) >= sms * 2 / 3) ? 128 : 64;
+    if (bn > CHAIN_BN_MAX) FELIX_THROW(FELIX_E_UNSUPPORTED, "chain tile N > 128");
+    L.bn = bn;
+    L.n_tiles_n = N / bn;
+    L.n_tiles = static_cast<int>(mt) * L.n_tiles_n;
+    L.idesc = ptx::idesc_f16_f32(GEMM_BM, static_cast<uint32_t>(bn));
+    L.a_hi = g.a_hi; L.a_lo = g.a_lo; L.c_hi = g.c_hi; L.c_lo = g.c_lo;
+    L.b_hi = make_tmap(g.w_hi, N, g.args.K, bn);
+    L.b_lo = make_tmap(g.w_lo, N, g.args.K, bn);
+    if (g.epi == EPI_HEAD && use_chain()) p->n_head_tiles = 2 * (N / bn);   // chain: one partial per column half
+    max_tiles = std::max(max_tiles, L.n_tiles);
+  }
+  p->chain_grid = std::min(sms, max_tiles);
+  return p;
+}
+
+// number of concurrent chunks for a population of n (FELIX_CHUNKS overrides; tuned on B200)
+static int choose_chunks(int64_t n) {
+  if (const char* e = std::getenv("FELIX_CHUNKS")) {
+    const int k = std::atoi(e);
+    if (k >= 1 && k <= 16) return k;
+  }
+  (void)n;   // measured on B200 (C2): 2/4/8 concurrent chunks were 3-14% slower than 1
+  return 1;
+}
+
+static Chunks& get_chunks(felix_space* s, std::unique_ptr<Chunks>& slot, const CostModel* cm, int64_t n, int K) {
+  if (slot && slot->cm == cm && slot->n == n && slot->K == K) return *slot;
+  slot.reset();
+  auto c = std::make_unique<Chunks>();
+  c->cm = cm;
+  c->n = n;
+  const int64_t per = ((n + K - 1) / K + 127) / 128 * 128;
+  for (int64_t o = 0; o < n; o += per) {
+    c->off.push_back(o);
+    c->cnt.push_back(std::min(per, n - o));
+  }
+  c->K = K;
+  for (size_t k = 0; k < c->off.size(); ++k) c->plans.push_back(build_plan(s, cm, c->cnt[k]));
+  slot = std::move(c);
+  return *slot;
 }
 
 // ============================================================================ profiling
@@ -410,19 +584,24 @@ static void prof_mark(felix_space* s, int cls, cudaStream_t st, bool begin) {
 }
 
 // ============================================================================ step pieces
-static void run_forward_mlp(felix_space* s, Plan& p, const float* y, int64_t n, cudaStream_t st) {
-  int ni = static_cast<int>(n);
+static void run_forward_mlp(felix_space* s, Plan& p, const felix_space::Module& mod, const float* y, int64_t n,
+                            int64_t ldy, cudaStream_t st, int* step_ctr) {
+  int ni = static_cast<int>(n), ldi = static_cast<int>(ldy);
   void* phi_hi = p.phi_hi.p;
   void* phi_lo = p.phi_lo.p;
-  void* args[] = {&y, &ni, &phi_hi, &phi_lo};
+  void* args[] = {&y, &ni, &ldi, &phi_hi, &phi_lo, &step_ctr};
   prof_mark(s, 0, st, true);
-  launch_nv(s->f_fwd, n, args, st);
+  launch_grouped(mod.f_fwd, mod.P, n, 0, args, st, true);
   prof_mark(s, 0, st, false);
   s->prof_launches[0] += 1;
   prof_mark(s, 1, st, true);
-  for (const auto& g : p.gemms) launch_gemm(g, st);
+  if (use_chain()) {
+    launch_chain(p, st);
+  } else {
+    for (const auto& g : p.gemms) launch_gemm(g, st);
+  }
   prof_mark(s, 1, st, false);
-  s->prof_launches[1] += static_cast<int64_t>(p.gemms.size());
+  s->prof_launches[1] += use_chain() ? 1 : static_cast<int64_t>(p.gemms.size());
 }
 
 }  // namespace felix
@@ -544,7 +723,7 @@ felix_status felix_space_create(int device, const felix_var* vars, int32_t n_var
   for (size_t q = 0; q < t.int_vars.size(); ++q) icnt.push_back(t.int_hi[q] - t.int_lo[q]);
   upload(s->d_int_vars, iv); upload(s->d_int_lo, t.int_lo); upload(s->d_int_cnt, icnt);
   upload(s->d_int_toff, t.int_toff); upload(s->d_int_thr, t.int_thr);
-  compile_module(s.get());
+  get_module(s.get(), 1);
   *out = s.release();
   FELIX_API_END
 }
@@ -558,7 +737,7 @@ felix_status felix_codegen(const felix_var* vars, int32_t n_vars, const felix_sp
   auto s = parse_space(vars, n_vars, splits, n_splits, nodes, n_nodes, feature_roots, n_features, constraint_roots,
                        n_constraints);
   CodegenInfo info;
-  const std::string code = generate_dag_module(s->desc, s->K0p, &info);
+  const std::string code = generate_dag_module(s->desc, s->K0p, 8, &info);
   if (src_len) *src_len = static_cast<int64_t>(code.size());
   if (src && src_cap > 0) {
     const size_t nb = std::min<size_t>(code.size() + 1, static_cast<size_t>(src_cap));
@@ -676,35 +855,96 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
   DeviceGuard dg(s->device);
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const int64_t n = p->n_seeds;
-  Plan& pl = get_plan(s, m, n);
-  int ni = static_cast<int>(n);
+  Chunks& ch = get_chunks(s, s->search_chunks, m, n, choose_chunks(n));
+  const int nck = static_cast<int>(ch.plans.size());
+  const felix_space::Module& mod = get_module(s, choose_P(ch.cnt[0]));
   if (!p->init_from_y) {
     unsigned long long seed = p->rng_seed;
     long long ib = p->index_base;
+    int ni = static_cast<int>(n);
     void* args[] = {&seed, &ni, &ib, &y};
     prof_mark(s, 3, st, true);
-    launch_nv(s->f_init, n, args, st);
+    launch_flat(mod.f_init, n, args, st);
     prof_mark(s, 3, st, false);
     s->prof_launches[3] += 1;
   }
-  CUDA_OK(cudaMemsetAsync(pl.m.p, 0, pl.m.bytes, st));
-  CUDA_OK(cudaMemsetAsync(pl.v.p, 0, pl.v.bytes, st));
-  void* dphi = pl.dphi.p;
-  void* cpart = pl.c_part.p;
-  int ld = static_cast<int>(pl.n_pad);
-  int nht = pl.n_head_tiles;
-  float hb = m->head_b, lam = p->lambda, lr = p->lr, b1 = p->beta1, b2 = p->beta2, eps = p->eps;
-  void* mv = pl.m.p;
-  void* vv = pl.v.p;
-  for (int t = 1; t <= p->n_steps; ++t) {
-    run_forward_mlp(s, pl, y, n, st);
-    float* lo = (t == p->n_steps) ? final_loss : nullptr;
-    int tt = t;
-    void* args[] = {&y, &ni, &dphi, &ld, &cpart, &nht, &ld, &hb, &lam, &mv, &vv, &tt, &lr, &b1, &b2, &eps, &lo};
-    prof_mark(s, 2, st, true);
-    launch_nv(s->f_rev_adam, n, args, st);
-    prof_mark(s, 2, st, false);
+  for (auto& pl : ch.plans) {
+    CUDA_OK(cudaMemsetAsync(pl->m.p, 0, pl->m.bytes, st));
+    CUDA_OK(cudaMemsetAsync(pl->v.p, 0, pl->v.bytes, st));
+    CUDA_OK(cudaMemsetAsync(pl->step_ctr.p, 0, 4, st));
+  }
+  const float hb = m->head_b, lam0 = p->lambda, lr0 = p->lr, b10 = p->beta1, b20 = p->beta2, eps0 = p->eps;
+  // one Adam step of chunk k (fwd DAG -> GEMMs -> reverse DAG + Adam), PDL-chained on stream cs
+  auto chunk_step = [&](int k, cudaStream_t cs) {
+    Plan& pl = *ch.plans[k];
+    const int64_t o = ch.off[k], cnt = ch.cnt[k];
+    float* yk = y + o;
+    int* ctr = pl.step_ctr.as<int>();
+    run_forward_mlp(s, pl, mod, yk, cnt, n, cs, ctr);
+    int ni = static_cast<int>(cnt), ldy = static_cast<int>(n);
+    void* dphi = pl.dphi.p;
+    void* cpart = pl.c_part.p;
+    int ld = static_cast<int>(pl.n_pad);
+    int nht = pl.n_head_tiles;
+    float hbv = hb, lam = lam0, lr = lr0, b1 = b10, b2 = b20, eps = eps0;
+    void* mv = pl.m.p;
+    void* vv = pl.v.p;
+    float* lo = final_loss ? final_loss + o : nullptr;   // every step writes its loss; the last one stays
+    void* args[] = {&yk, &ni, &ldy, &dphi, &ld, &cpart, &nht, &ld, &hbv, &lam, &mv, &vv, &ctr, &lr, &b1, &b2, &eps, &lo};
+    prof_mark(s, 2, cs, true);
+    launch_grouped(mod.f_rev_adam, mod.P, cnt, mod.rev_smem, args, cs, true);
+    prof_mark(s, 2, cs, false);
     s->prof_launches[2] += 1;
+  };
+  if (s->profiling) {
+    for (int t = 1; t <= p->n_steps; ++t)            // direct launches with per-class events
+      for (int k = 0; k < nck; ++k) chunk_step(k, st);
+  } else if (p->n_steps > 0) {
+    const std::vector<double> key = {static_cast<double>(mod.P), static_cast<double>(reinterpret_cast<uintptr_t>(y)),
+                                     static_cast<double>(reinterpret_cast<uintptr_t>(final_loss)), lam0, lr0, b10, b20, eps0};
+    if (!ch.graph || ch.graph_key != key) {
+      if (ch.graph) { cudaGraphExecDestroy(ch.graph); ch.graph = nullptr; }
+      while (static_cast<int>(ch.streams.size()) < nck) {
+        cudaStream_t b;
+        CUDA_OK(cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking));
+        ch.streams.push_back(b);
+      }
+      cudaGraph_t graph = nullptr;
+      cudaEvent_t fork, join[16];
+      CUDA_OK(cudaEventCreateWithFlags(&fork, cudaEventDisableTiming));
+      for (int k = 0; k < nck; ++k) CUDA_OK(cudaEventCreateWithFlags(&join[k], cudaEventDisableTiming));
+      cudaStream_t cap = ch.streams[0];
+      CUDA_OK(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
+      int64_t saved[4];
+      std::copy(s->prof_launches, s->prof_launches + 4, saved);
+      try {
+        CUDA_OK(cudaEventRecord(fork, cap));
+        for (int k = 1; k < nck; ++k) CUDA_OK(cudaStreamWaitEvent(ch.streams[k], fork, 0));
+        for (int k = 0; k < nck; ++k) chunk_step(k, ch.streams[k]);
+        for (int k = 1; k < nck; ++k) {
+          CUDA_OK(cudaEventRecord(join[k], ch.streams[k]));
+          CUDA_OK(cudaStreamWaitEvent(cap, join[k], 0));
+        }
+        std::copy(saved, saved + 4, s->prof_launches);
+      } catch (...) {
+        cudaStreamEndCapture(cap, &graph);
+        if (graph) cudaGraphDestroy(graph);
+        cudaEventDestroy(fork);
+        for (int k = 0; k < nck; ++k) cudaEventDestroy(join[k]);
+        throw;
+      }
+      CUDA_OK(cudaStreamEndCapture(cap, &graph));
+      cudaError_t ie = cudaGraphInstantiate(&ch.graph, graph, 0);
+      cudaGraphDestroy(graph);
+      cudaEventDestroy(fork);
+      for (int k = 0; k < nck; ++k) cudaEventDestroy(join[k]);
+      CUDA_OK(ie);
+      ch.graph_key = key;
+    }
+    for (int t = 1; t <= p->n_steps; ++t) CUDA_OK(cudaGraphLaunch(ch.graph, st));
+    s->prof_launches[0] += static_cast<int64_t>(p->n_steps) * nck;
+    s->prof_launches[1] += static_cast<int64_t>(p->n_steps) * nck * (use_chain() ? 1 : static_cast<int64_t>(ch.plans[0]->gemms.size()));
+    s->prof_launches[2] += static_cast<int64_t>(p->n_steps) * nck;
   }
   FELIX_API_END
 }
@@ -718,16 +958,17 @@ felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int6
   if (n == 0) return FELIX_OK;
   DeviceGuard dg(s->device);
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  Plan& pl = get_plan(s, m, n);
-  run_forward_mlp(s, pl, y, n, st);
+  Plan& pl = *get_chunks(s, s->eval_chunks, m, n, 1).plans[0];
+  const felix_space::Module& mod = get_module(s, choose_P(n));
+  run_forward_mlp(s, pl, mod, y, n, n, st, nullptr);
   int ni = static_cast<int>(n);
   void* dphi = pl.dphi.p;
   void* cpart = pl.c_part.p;
   int ld = static_cast<int>(pl.n_pad);
   int nht = pl.n_head_tiles;
   float hb = m->head_b, lam = lambda;
-  void* args[] = {&y, &ni, &dphi, &ld, &cpart, &nht, &ld, &hb, &lam, &phi, &g, &cost, &loss, &grad};
-  launch_nv(s->f_rev_eval, n, args, st);
+  void* args[] = {&y, &ni, &ni, &dphi, &ld, &cpart, &nht, &ld, &hb, &lam, &phi, &g, &cost, &loss, &grad};
+  launch_grouped(mod.f_rev_eval, mod.P, n, mod.rev_smem, args, st, false);
   FELIX_API_END
 }
 
@@ -741,7 +982,7 @@ felix_status felix_init_sample(felix_space* s, int64_t n, uint64_t rng_seed, int
   unsigned long long seed = rng_seed;
   long long ib = index_base;
   void* args[] = {&seed, &ni, &ib, &y};
-  launch_nv(s->f_init, n, args, static_cast<cudaStream_t>(stream));
+  launch_flat(get_module(s, 1).f_init, n, args, static_cast<cudaStream_t>(stream));
   FELIX_API_END
 }
 
@@ -771,7 +1012,7 @@ static void do_round(felix_space* s, const float* y, int64_t n, int32_t* sched, 
 static void do_hard(felix_space* s, const int32_t* sched, int64_t n, double* phi64, uint8_t* valid, cudaStream_t st) {
   int ni = static_cast<int>(n);
   void* args[] = {&sched, &ni, &phi64, &valid};
-  launch_nv(s->f_hard, n, args, st);
+  launch_flat(get_module(s, 1).f_hard, n, args, st);
 }
 
 static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, int64_t n, double* score, cudaStream_t st) {
@@ -786,8 +1027,8 @@ static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, in
   for (int l = 0; l < L; ++l) {
     const int K = m->dims[l], N = m->dims[l + 1];
     double* out = (l == L - 1) ? score : bufs[l & 1];
-    const long long tot = static_cast<long long>(n) * N;
-    score_layer_kernel<<<static_cast<unsigned>((tot + 255) / 256), 256, 0, st>>>(
+    const dim3 grid(static_cast<unsigned>((N + 31) / 32), static_cast<unsigned>((n + 31) / 32));
+    score_layer_kernel<<<grid, dim3(32, 8), 0, st>>>(
         in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N, l < L - 1 ? 1 : 0);
     CUDA_OK(cudaGetLastError());
     in = out;

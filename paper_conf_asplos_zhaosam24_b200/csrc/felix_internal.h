@@ -78,8 +78,10 @@ void build_round_tables(const SpaceDesc& d, RoundTables& t);
 // -------------------------------------------------------------------------- codegen
 struct CodegenInfo {
   int64_t flops_fwd = 0;
+  int rev_smem_bytes = 0;
 };
-std::string generate_dag_module(const SpaceDesc& d, int K0p, CodegenInfo* info);
+// P = warps cooperating on one 32-candidate block (cone partition of the roots), 1..8
+std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo* info);
 
 // -------------------------------------------------------------------------- cost model
 struct CostModel {

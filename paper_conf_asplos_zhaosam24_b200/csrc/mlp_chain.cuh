@@ -1,0 +1,309 @@
+// mlp_chain.cuh — the whole cost-model MLP of one Adam step (forward + input-gradient backward,
+// 2(L-1) GEMM layers) in ONE persistent kernel.
+//
+// Why: at the C2 population (4096 candidates) every layer is a few microseconds of tensor work, and
+// separate launches cost ~4 us each at the kernel boundary (launch ramp, prologue, drain) even
+// with PDL + CUDA graphs.  Here one CTA per SM loops over the tiles of every layer; layers are
+// separated by a grid-wide release/acquire barrier.  Per layer the math is the one of
+// mlp_gemm.cuh (split fp16 hi/lo, 3 tcgen05.mma per
+// K step, fp32 TMEM accumulation) and the epilogues are the same (bias/ReLU/mask, head GEMV,
+// -w_L seed, dL/dphi transpose).
+//
+// Warp roles (320 threads): warp 0 = TMA producer, warp 1 = MMA issuer (one elected thread),
+// warps 2..9 = epilogue: warp w drains TMEM lanes 32*(w%4)..+31, warps w and w+4 split every
+// 64-column chunk into two 32-column halves (two warps per SM sub-partition hide the latency of
+// the convert/split chains).  TMEM holds two 128-column accumulators so the epilogue of tile i
+// overlaps the MMAs of tile i+1.
+#pragma once
+#include <cstdint>
+#include <cuda_fp16.h>
+#include "sm100_ptx.cuh"
+#include "mlp_gemm.cuh"
+
+namespace felix {
+
+constexpr int CHAIN_MAX_LAYERS = 14;
+constexpr int CHAIN_BN_MAX = 128;
+constexpr int CHAIN_STAGES = 3;
+constexpr int CHAIN_THREADS = 320;
+constexpr int CHAIN_EPI_WARPS = 8;
+constexpr int CHAIN_A_BYTES = GEMM_BM * GEMM_BK * 2;                 // 16 KB (one of hi / lo)
+constexpr int CHAIN_B_BYTES = CHAIN_BN_MAX * GEMM_BK * 2;            // 16 KB
+constexpr int CHAIN_STAGE_BYTES = 2 * CHAIN_A_BYTES + 2 * CHAIN_B_BYTES;
+constexpr int CHAIN_EPI_BYTES = 2 * GEMM_BM * 64 * 2;                 // hi + lo staging of one 64-col chunk
+constexpr int CHAIN_SMEM_BYTES = 1024 + CHAIN_STAGES * CHAIN_STAGE_BYTES + CHAIN_EPI_BYTES + 256;
+
+struct ChainLayer {
+  CUtensorMap a_hi, a_lo, b_hi, b_lo, c_hi, c_lo;
+  GemmArgs args;
+  int epi, bn, n_tiles_n, n_tiles;     // tiles = m_tiles * n_tiles_n (n fastest)
+  uint32_t idesc;
+  int _pad[3];
+};
+
+struct ChainParams {
+  ChainLayer layer[CHAIN_MAX_LAYERS];
+  int n_layers;
+  int m_tiles;
+  unsigned int* grid_bar;              // monotonic arrival counter (never reset)
+  unsigned long long* trace;           // debug: [grid][layers][8] globaltimer stamps (FELIX_CHAIN_TRACE)
+};
+
+#ifdef FELIX_CHAIN_TRACE
+#define CHAIN_STAMP(l, slot) do { unsigned long long t_; asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t_)); \
+    P.trace[(static_cast<size_t>(blockIdx.x) * CHAIN_MAX_LAYERS + (l)) * 8 + (slot)] = t_; } while (0)
+#else
+#define CHAIN_STAMP(l, slot) do {} while (0)
+#endif
+
+__device__ __forceinline__ void grid_barrier(unsigned int* ctr, unsigned int nblocks) {
+  // arrive (release, after this thread's async-proxy writes are complete) ...
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+  unsigned int old;
+  asm volatile("atom.add.release.gpu.u32 %0, [%1], 1;" : "=r"(old) : "l"(ctr) : "memory");
+  const unsigned int target = (old / nblocks + 1) * nblocks;
+  // ... and wait (acquire)
+  unsigned int cur;
+  do {
+    asm volatile("ld.acquire.gpu.u32 %0, [%1];" : "=r"(cur) : "l"(ctr) : "memory");
+  } while (static_cast<int>(cur - target) < 0);
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+
+__global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __grid_constant__ ChainParams P) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* epi_hi = smem + CHAIN_STAGES * CHAIN_STAGE_BYTES;
+  uint8_t* epi_lo = epi_hi + GEMM_BM * 64 * 2;
+  uint64_t* full_bar = reinterpret_cast<uint64_t*>(epi_hi + CHAIN_EPI_BYTES);
+  uint64_t* empty_bar = full_bar + CHAIN_STAGES;
+  uint64_t* tfull = empty_bar + CHAIN_STAGES;      // [2] accumulator ready
+  uint64_t* tempty = tfull + 2;                    // [2] accumulator drained
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint32_t* gen_slot = tmem_slot + 1;              // layers completed grid-wide (producer handshake)
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const unsigned int G = gridDim.x;
+
+  auto a_hi = [&](int s) { return smem + s * CHAIN_STAGE_BYTES; };
+  auto a_lo = [&](int s) { return smem + s * CHAIN_STAGE_BYTES + CHAIN_A_BYTES; };
+  auto b_hi = [&](int s) { return smem + s * CHAIN_STAGE_BYTES + 2 * CHAIN_A_BYTES; };
+  auto b_lo = [&](int s) { return smem + s * CHAIN_STAGE_BYTES + 2 * CHAIN_A_BYTES + CHAIN_B_BYTES; };
+
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < CHAIN_STAGES; ++s) { ptx::mbar_init(&full_bar[s], 1); ptx::mbar_init(&empty_bar[s], 1); }
+    for (int a = 0; a < 2; ++a) { ptx::mbar_init(&tfull[a], 1); ptx::mbar_init(&tempty[a], CHAIN_EPI_WARPS); }
+    *gen_slot = 0;
+    ptx::fence_barrier_init();
+  }
+  if (warp == 1) ptx::tmem_alloc(tmem_slot, 2 * CHAIN_BN_MAX);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  ptx::pdl_launch_dependents();
+  ptx::pdl_wait();                                  // phi (layer-1 A operand) comes from the DAG kernel
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // ------------------------------------------------------------ TMA producer
+      int it = 0;                                   // running k-block counter (ring position)
+      for (int l = 0; l < P.n_layers; ++l) {
+        const ChainLayer& L = P.layer[l];
+        if (l > 0) {
+          // layer l reads layer l-1's outputs: wait until the epilogue warps of this CTA have
+          // passed the grid barrier (they publish the layer count with st.release.cta)
+          unsigned int g;
+          do {
+            asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(g) : "r"(ptx::smem_u32(gen_slot)) : "memory");
+          } while (g < static_cast<unsigned int>(l));
+          asm volatile("fence.proxy.async.global;" ::: "memory");
+        }
+        CHAIN_STAMP(l, 0);
+        const int nkb = (L.args.K + GEMM_BK - 1) / GEMM_BK;
+        const uint32_t tx = 2 * CHAIN_A_BYTES + 2 * (L.bn * GEMM_BK * 2);
+        for (int tile = blockIdx.x; tile < L.n_tiles; tile += G) {
+          const int m0 = (tile / L.n_tiles_n) * GEMM_BM, n0 = (tile % L.n_tiles_n) * L.bn;
+          for (int kb = 0; kb < nkb; ++kb, ++it) {
+            const int s = it % CHAIN_STAGES;
+            if (it >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], ((it / CHAIN_STAGES) - 1) & 1);
+            ptx::mbar_arrive_expect_tx(&full_bar[s], tx);
+            const int k0 = kb * GEMM_BK;
+            ptx::tma_load_2d(a_hi(s), &L.a_hi, k0, m0, &full_bar[s]);
+            ptx::tma_load_2d(a_lo(s), &L.a_lo, k0, m0, &full_bar[s]);
+            ptx::tma_load_2d(b_hi(s), &L.b_hi, k0, n0, &full_bar[s]);
+            ptx::tma_load_2d(b_lo(s), &L.b_lo, k0, n0, &full_bar[s]);
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // ------------------------------------------------------------ MMA issuer
+      int it = 0, tcount = 0;
+      for (int l = 0; l < P.n_layers; ++l) {
+        const ChainLayer& L = P.layer[l];
+        const int nkb = (L.args.K + GEMM_BK - 1) / GEMM_BK;
+        for (int tile = blockIdx.x; tile < L.n_tiles; tile += G, ++tcount) {
+          const int acc = tcount & 1;
+          if (tcount >= 2) ptx::mbar_wait(&tempty[acc], ((tcount >> 1) - 1) & 1);
+          ptx::tc_fence_after();
+          const uint32_t d = tmem_base + acc * CHAIN_BN_MAX;
+          for (int kb = 0; kb < nkb; ++kb, ++it) {
+            const int s = it % CHAIN_STAGES;
+            ptx::mbar_wait(&full_bar[s], (it / CHAIN_STAGES) & 1);
+            if (kb == 0 && tile == static_cast<int>(blockIdx.x)) CHAIN_STAMP(l, 1);
+            ptx::tc_fence_after();
+            const uint32_t ah = ptx::smem_u32(a_hi(s)), al = ptx::smem_u32(a_lo(s));
+            const uint32_t bh = ptx::smem_u32(b_hi(s)), bl = ptx::smem_u32(b_lo(s));
+#pragma unroll
+            for (int kk = 0; kk < GEMM_BK / GEMM_UMMA_K; ++kk) {
+              const uint32_t off = kk * GEMM_UMMA_K * 2;
+              const uint32_t acc0 = (kb | kk) != 0;
+              ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(al + off), ptx::sdesc_k_sw128(bh + off), L.idesc, acc0);
+              ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bl + off), L.idesc, 1u);
+              ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bh + off), L.idesc, 1u);
+            }
+            ptx::mma_commit(&empty_bar[s]);
+          }
+          ptx::mma_commit(&tfull[acc]);
+          CHAIN_STAMP(l, 2);
+        }
+      }
+    }
+  } else {
+    // ------------------------------------------------------------ epilogue warps 2..9
+    const int q = warp & 3;                          // TMEM lane quadrant this warp may access
+    const int half = (warp - 2) >> 2;                // which 32-column half of each 64-column chunk
+    const int r_tile = q * 32 + lane;
+    const int etid = threadIdx.x - 64;               // 0..255
+    constexpr int NEPI = CHAIN_EPI_WARPS * 32;
+    int tcount = 0;
+    for (int l = 0; l < P.n_layers; ++l) {
+      const ChainLayer& L = P.layer[l];
+      const GemmArgs& args = L.args;
+      for (int tile = blockIdx.x; tile < L.n_tiles; tile += G, ++tcount) {
+        const int acc = tcount & 1;
+        const int m0 = (tile / L.n_tiles_n) * GEMM_BM, n0 = (tile % L.n_tiles_n) * L.bn;
+        const int row = m0 + r_tile;
+        const bool row_ok = row < args.M;
+        ptx::mbar_wait(&tfull[acc], (tcount >> 1) & 1);
+        if (etid == 0 && tile == static_cast<int>(blockIdx.x)) CHAIN_STAMP(l, 3);
+        ptx::tc_fence_after();
+        const uint32_t t_row = tmem_base + acc * CHAIN_BN_MAX + (static_cast<uint32_t>(q * 32) << 16);
+        float head_acc = 0.f;
+        if (L.epi == EPI_F32T) {
+          for (int c = half * 32; c < L.bn; c += 64) {
+            float v[32];
+            {
+              float a[16], b[16];
+              ptx::tmem_ld16(t_row + c, a);
+              ptx::tmem_ld16(t_row + c + 16, b);
+#pragma unroll
+              for (int i = 0; i < 16; ++i) { v[i] = a[i]; v[16 + i] = b[i]; }
+            }
+            const int n = n0 + c;
+            if (row_ok) {
+#pragma unroll
+              for (int i = 0; i < 32; ++i)
+                if (n + i < args.n_valid) args.out_f32[static_cast<size_t>(n + i) * args.ld_f32 + row] = v[i];
+            }
+          }
+        } else {
+          for (int c64 = 0; c64 < L.bn; c64 += 64) {
+            // the staging buffer must be free: previous TMA store finished reading it
+            if (etid == 0) ptx::bulk_wait_read<0>();
+            ptx::named_bar_sync(1, NEPI);
+            {
+              const int c32 = half * 32;
+              const int c = c64 + c32;
+              float v[32];
+              {
+                float a[16], b[16];
+                ptx::tmem_ld16(t_row + c, a);
+                ptx::tmem_ld16(t_row + c + 16, b);
+#pragma unroll
+                for (int i = 0; i < 16; ++i) { v[i] = a[i]; v[16 + i] = b[i]; }
+              }
+              const int n = n0 + c;
+              if (L.epi == EPI_MASK) {
+                // written earlier in this launch by other CTAs: coherent L2 load, not the .nc path
+                const uint32_t bits = row_ok ? __ldcg(&args.mask_in[static_cast<size_t>(row) * (args.N / 32) + n / 32]) : 0u;
+#pragma unroll
+                for (int i = 0; i < 32; ++i) v[i] = ((bits >> i) & 1u) ? v[i] : 0.f;
+              } else {
+                uint32_t bits = 0;
+                const bool head = L.epi == EPI_HEAD;
+#pragma unroll
+                for (int i = 0; i < 32; ++i) {
+                  const float z = v[i] + __ldg(&args.bias[n + i]);
+                  const bool on = z > 0.f;
+                  bits |= (on ? 1u : 0u) << i;
+                  if (!head) {
+                    v[i] = on ? z : 0.f;
+                  } else {
+                    const float w = __ldg(&args.head_w[n + i]);
+                    head_acc += (on ? z : 0.f) * w;
+                    v[i] = on ? -w : 0.f;        // delta_{L-1} = W_L^T (dL/dc = -1) (.) [Z > 0]
+                  }
+                }
+                if (!head && row_ok) args.mask_out[static_cast<size_t>(row) * (args.N / 32) + n / 32] = bits;
+              }
+#pragma unroll
+              for (int qq = 0; qq < 4; ++qq) {
+                // split 8 values into fp16 hi / lo with packed f16x2 converts
+                uint32_t h[4], lo[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                  const float2 f = make_float2(v[qq * 8 + 2 * u], v[qq * 8 + 2 * u + 1]);
+                  const __half2 hh = __float22half2_rn(f);
+                  const float2 back = __half22float2(hh);
+                  const __half2 ll = __float22half2_rn(make_float2(f.x - back.x, f.y - back.y));
+                  h[u] = *reinterpret_cast<const uint32_t*>(&hh);
+                  lo[u] = *reinterpret_cast<const uint32_t*>(&ll);
+                }
+                const int q16 = c32 / 8 + qq;
+                const uint32_t off = r_tile * 128 + ((q16 ^ (r_tile & 7)) << 4);
+                *reinterpret_cast<uint4*>(epi_hi + off) = make_uint4(h[0], h[1], h[2], h[3]);
+                *reinterpret_cast<uint4*>(epi_lo + off) = make_uint4(lo[0], lo[1], lo[2], lo[3]);
+              }
+            }
+            ptx::fence_proxy_async_smem();
+            ptx::named_bar_sync(1, NEPI);
+            if (etid == 0) {
+              ptx::tma_store_2d(&L.c_hi, n0 + c64, m0, epi_hi);
+              ptx::tma_store_2d(&L.c_lo, n0 + c64, m0, epi_lo);
+              ptx::bulk_commit();
+            }
+          }
+        }
+        // head partial per (N tile, column half); the reverse kernel sums all 2 * N / bn partials
+        if (L.epi == EPI_HEAD && row_ok) args.c_part[static_cast<size_t>(2 * (n0 / L.bn) + half) * args.ld_c + row] = head_acc;
+        // accumulator drained: let the MMA warp reuse it
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
+      }
+      // ---- layer end: all of this CTA's outputs complete + visible, then the grid barrier
+      if (etid == 0) CHAIN_STAMP(l, 4);
+      if (l + 1 < P.n_layers) {
+        if (etid == 0) ptx::bulk_wait<0>();
+        __threadfence();
+        ptx::named_bar_sync(1, NEPI);
+        if (etid == 0) {
+          CHAIN_STAMP(l, 5);
+          grid_barrier(P.grid_bar, G);
+          CHAIN_STAMP(l, 6);
+          // publish "layer l done everywhere" to the producer warp of this CTA
+          asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" :: "r"(ptx::smem_u32(gen_slot)), "r"(static_cast<unsigned int>(l + 1)) : "memory");
+        }
+      }
+    }
+    if (etid == 0) ptx::bulk_wait<0>();
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 1) ptx::tmem_dealloc(tmem_base, 2 * CHAIN_BN_MAX);
+}
+
+}  // namespace felix

@@ -84,7 +84,7 @@ def test_generated_kernels_compile_for_sm100a(fx, which):
     sp = {"paper": fi.paper_example_space, "C1": fi.c1_space, "C2": fi.c2_space}[which]()
     src = fx.codegen(sp, compile=True)
     for k in ("felix_fwd", "felix_rev_adam", "felix_rev_eval", "felix_hard", "felix_init"):
-        assert f"void __launch_bounds__(128) {k}(" in src
+        assert re.search(r"__global__ void __launch_bounds__\([^)]*\) " + k + r"\(", src), k
 
 
 def test_device_calls_fail_loudly_without_gpu(fx):
