@@ -38,7 +38,7 @@ UNIT = "cand-steps/s"
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=30)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="felix", choices=["felix", "reference"])
     ap.add_argument("--config", default="C2")
@@ -50,7 +50,7 @@ def parse():
 
 # ------------------------------------------------------------------------------------- clocks
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+    """nvidia-smi clocks / throttle reasons sampled every 50 ms during the timed region."""
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
@@ -64,7 +64,7 @@ class ClockSampler:
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except FileNotFoundError:
             self.proc = None
@@ -270,11 +270,17 @@ def run_felix(args):
     barrier()
     finish_ms = f0.elapsed_time(f1)
 
-    # ---- roofline of the dominant kernel family: the MLP tcgen05 GEMMs (tensor-bound)
+    # ---- roofline of the dominant kernel: the persistent tcgen05 MLP chain (tensor-bound contraction)
     peaks, peak_src = measured_peaks()
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "r01", "roofline_traffic.json")
+    if os.path.exists(tpath):
+        with open(tpath) as f:
+            tj = json.load(f)
+        traffic = tj["dram_bytes_read_per_launch"] + tj["dram_bytes_write_per_launch"]
     gemm_ms, gemm_launches = prof["mlp_gemm"]
     mlp_flops_step = cm.mlp_flops_per_candidate_step() * n           # algorithmic (1-pass) FLOPs per Adam step
-    gemm_per_step_ms = gemm_ms / (K * T)
+    gemm_per_step_ms = gemm_ms / (K * T)         # one chain launch (or 2(L-1) layer launches) per Adam step
     achieved_tflops = mlp_flops_step / (gemm_per_step_ms * 1e-3) / 1e12
     peak = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops")))
     dag_fwd_ms, _ = prof["dag_fwd"]
@@ -321,8 +327,9 @@ def run_felix(args):
         rate, threads, sample, _ = oracle_baseline(cfg, args.cpu_seconds)
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample}
 
-    n_gemm = len(cfg.mlp_dims) * 2 - 4          # (L-1) forward + (L-1) backward GEMMs
-    launches_per_step = 1 + T * (2 + n_gemm) + (6 + len(cfg.mlp_dims) - 1)   # init + steps + finish
+    n_gemm = len(cfg.mlp_dims) * 2 - 4          # (L-1) forward + (L-1) backward GEMM layers
+    mlp_launches = 1 if os.environ.get("FELIX_MLP", "chain") != "layers" else n_gemm
+    launches_per_step = 1 + T * (2 + mlp_launches) + (6 + len(cfg.mlp_dims) - 1)   # init + steps + finish
     ms_per_step = t_max / K
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
@@ -333,8 +340,9 @@ def run_felix(args):
                    "n_seeds_per_gpu": n, "n_steps": T, "topk": k, "parallelism": f"dp{world} (seed shards)",
                    "l2": "flushed (256 MB write) between timed iterations"},
         "roofline": {"bound": "tensor", "achieved": achieved_tflops, "peak": peak, "unit": "TFLOP/s",
-                     "frac": achieved_tflops / peak, "traffic": None,
-                     "kernel": f"mlp_gemm_kernel x{n_gemm} per Adam step (tcgen05 kind::f16, 3-pass hi/lo split)",
+                     "frac": achieved_tflops / peak, "traffic": traffic,
+                     "kernel": f"mlp_chain_kernel (all {n_gemm} MLP layers of one Adam step, tcgen05 kind::f16, 3-pass hi/lo split)",
+                     "traffic_source": "profiles/r01/roofline_traffic.json (ncu --set full, DRAM bytes per launch)",
                      "algorithmic_flops_per_adam_step": mlp_flops_step,
                      "executed_tflops": 3 * achieved_tflops,
                      "peak_source": f"{peak_src} bf16_tflops_sustained (fp16 = bf16 rate)"},
