@@ -199,6 +199,10 @@ FELIX_EXPORT felix_status felix_init_sample(felix_space* s, int64_t n, uint64_t 
 FELIX_EXPORT felix_status felix_profile_enable(felix_space* s, int32_t enable);
 FELIX_EXPORT felix_status felix_profile_read(felix_space* s, double* ms, int64_t* launches);
 FELIX_EXPORT felix_status felix_profile_reset(felix_space* s);
+/* Debug: copy the per-block %globaltimer stamps of the generated kernels (only when the space was
+ * created with the environment variable FELIX_TRACE set): uint64 [2][8192][4] = {fwd, rev} x block x
+ * {start, after griddepcontrol.wait, after compute, end}.  n_words bounds the copy. */
+FELIX_EXPORT felix_status felix_debug_trace(felix_space* s, uint64_t* out, int64_t n_words);
 
 #ifdef __cplusplus
 }

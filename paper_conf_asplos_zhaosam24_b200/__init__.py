@@ -28,7 +28,8 @@ FELIX_STATUS = {0: "OK", 1: "INVALID_ARG", 2: "INVALID_DAG", 3: "SHAPE", 4: "UNS
 EXPORTED = ["felix_last_error", "felix_abi_version", "felix_space_create", "felix_space_destroy",
             "felix_space_info", "felix_codegen", "felix_costmodel_load", "felix_costmodel_destroy",
             "felix_search", "felix_round_topk", "felix_eval", "felix_round", "felix_score",
-            "felix_init_sample", "felix_profile_enable", "felix_profile_read", "felix_profile_reset"]
+            "felix_init_sample", "felix_profile_enable", "felix_profile_read", "felix_profile_reset",
+            "felix_debug_trace"]
 
 
 class FelixError(RuntimeError):
@@ -160,7 +161,7 @@ class CostModel:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h:
+        if h and _lib is not None:
             _lib.felix_costmodel_destroy(h)
             self._h = None
 
@@ -186,7 +187,7 @@ class Space:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h:
+        if h and _lib is not None:
             _lib.felix_space_destroy(h)
             self._h = None
 
@@ -270,6 +271,12 @@ class Space:
 
     def profile_reset(self) -> None:
         _check(_lib.felix_profile_reset(self._h))
+
+    def debug_trace(self) -> np.ndarray:
+        """uint64 [2][8192][4] globaltimer stamps (space created with FELIX_TRACE set)."""
+        out = np.zeros((2, 8192, 4), dtype=np.uint64)
+        _check(_lib.felix_debug_trace(self._h, out.ctypes.data_as(_P), ctypes.c_int64(out.size)))
+        return out
 
     def _check_y(self, y) -> None:
         import torch

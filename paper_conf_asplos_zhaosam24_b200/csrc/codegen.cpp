@@ -23,6 +23,7 @@
 #include <climits>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <functional>
 #include <numeric>
 #include <sstream>
@@ -334,9 +335,15 @@ int SpaceDesc::n_roots_total() const {
 std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo* info) {
   Gen g(d);
   std::ostringstream& o = g.o;
+  const bool trace = std::getenv("FELIX_TRACE") != nullptr;   // debug: per-block phase timestamps
   const int M = d.n_vars, K = (int)d.froots.size(), Ru = (int)d.croots.size();
   const int R = d.n_roots_total(), Ra = R - Ru;
   o << kPrelude;
+  if (trace)
+    o << "__device__ unsigned long long felix_trace[2][8192][4];\n"
+         "#define TSTAMP(k, s) do { if (threadIdx.x == 0 && blockIdx.x < 8192) { unsigned long long t_; asm volatile(\"mov.u64 %0, %globaltimer;\" : \"=l\"(t_)); felix_trace[k][blockIdx.x][s] = t_; } } while (0)\n";
+  else
+    o << "#define TSTAMP(k, s) do {} while (0)\n";
   o << "#define NV " << M << "\n#define NF " << K << "\n#define NRU " << Ru << "\n#define NR " << R
     << "\n#define NRA " << Ra << "\n#define K0P " << K0p << "\n#define PG " << P << "\n";
 
@@ -397,12 +404,16 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
   // shared memory and written out as contiguous 16-byte stores.
   o << "extern \"C\" __global__ void __launch_bounds__(PG * 32) felix_fwd(const float* __restrict__ yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr) {\n"
     << "  __shared__ float sphi[32][K0P + 1];\n"
+    << "  __shared__ double sx[NV][32];   // x = exp(y), computed once per block and shared by the groups\n"
     << "  const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;\n"
     << "  const int c0 = blockIdx.x * 32, c = c0 + lane;\n"
     << "  const int cc = c < n ? c : n - 1;\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
+    << "  TSTAMP(0, 0);\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");   // y is the previous step's output\n"
+    << "  TSTAMP(0, 1);\n"
     << "  if (blockIdx.x == 0 && threadIdx.x == 0 && step_ctr) *step_ctr += 1;\n"
+    << "  for (int e = threadIdx.x; e < NV * 32; e += blockDim.x) { const int l = e & 31; const int cl = c0 + l; sx[e >> 5][l] = exp((double)yv[(size_t)(e >> 5) * ldy + (cl < n ? cl : n - 1)]); }\n"
     << "  for (int k = threadIdx.x; k < 32 * (K0P + 1); k += blockDim.x) (&sphi[0][0])[k] = 0.f;\n"
     << "  __syncthreads();\n";
   for (int q = 0; q < P; ++q) {
@@ -417,14 +428,17 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
         }
     const auto used = vars_in(fcone[q]);
     for (int j = 0; j < M; ++j)
-      if (used[j]) o << "    const double x" << j << " = exp((double)yv[(size_t)" << j << " * ldy + cc]);\n";
+      if (used[j]) o << "    const double x" << j << " = sx[" << j << "][lane];\n";
     g.emit_forward(fcone[q], 0, "x", "    ");
     for (int k : part.feat[q]) o << "    sphi[lane][" << k << "] = slogf_(v" << d.froots[k] << ");\n";
     o << "  }\n";
   }
-  o << "  __syncthreads();\n"
+  o << "  __syncthreads();\n  TSTAMP(0, 2);\n"
     << "  // rows c0 .. c0+31 are contiguous: K0P/8 uint4 per row for hi and for lo\n"
-    << "  for (int e = threadIdx.x; e < 32 * (K0P / 8); e += blockDim.x) {\n"
+    << "#pragma unroll\n"
+    << "  for (int it = 0; it < (32 * (K0P / 8) + PG * 32 - 1) / (PG * 32); ++it) {\n"
+    << "    const int e = threadIdx.x + it * PG * 32;\n"
+    << "    if (e >= 32 * (K0P / 8)) break;\n"
     << "    const int r = e / (K0P / 8), q8 = e % (K0P / 8);\n"
     << "    if (c0 + r >= n) continue;\n"
     << "    u32 h[4], l[4];\n"
@@ -437,7 +451,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "    }\n"
     << "    reinterpret_cast<uint4*>(phi_hi + (size_t)(c0 + r) * K0P)[q8] = make_uint4(h[0], h[1], h[2], h[3]);\n"
     << "    reinterpret_cast<uint4*>(phi_lo + (size_t)(c0 + r) * K0P)[q8] = make_uint4(l[0], l[1], l[2], l[3]);\n"
-    << "  }\n}\n\n";
+    << "  }\n  TSTAMP(0, 3);\n}\n\n";
 
   // ---------------------------------------------------------------- felix_rev (template on mode)
   // smem: partial adjoints of x  spart[PG][NV][32], user-root penalties per group spen[PG][32],
@@ -456,8 +470,25 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "  const bool live = c < n;\n"
     << "  const int cc = live ? c : n - 1;\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
+    << "  if (!EVAL) TSTAMP(1, 0);\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n"
-    << "  const double dlam = (double)lam;\n";
+    << "  if (!EVAL) TSTAMP(1, 1);\n"
+    << "  const double dlam = (double)lam;\n"
+    // everything the epilogue needs from memory is requested now, so its latency overlaps the DAG
+    << "  __shared__ double sx[NV * 32];\n"
+    << "  for (int e = threadIdx.x; e < NV * 32; e += blockDim.x) { const int j = e >> 5, l = e & 31; const int cl = blockIdx.x * 32 + l; const float yy = yin[(size_t)j * ldy + (cl < n ? cl : n - 1)]; sy[e] = yy; sx[e] = exp((double)yy); }\n"
+    << "  __syncthreads();\n"
+    << "  constexpr int NJ = (NV + PG - 1) / PG;   // vars handled by this thread: j = wq + PG * jj\n"
+    << "  float mreg[NJ], vreg[NJ];\n"
+    << "#pragma unroll\n"
+    << "  for (int jj = 0; jj < NJ; ++jj) {\n"
+    << "    const int j = wq + PG * jj;\n"
+    << "    mreg[jj] = 0.f; vreg[jj] = 0.f;\n"
+    << "    if (!EVAL && j < NV) { mreg[jj] = mv[(size_t)j * n + cc]; vreg[jj] = vv[(size_t)j * n + cc]; }\n"
+    << "  }\n"
+    << "  float cst = head_b;\n"
+    << "  if (wq == 0) for (int t = 0; t < n_head_tiles; ++t) cst += c_part[(size_t)t * ld_c + cc];\n"
+    << "  const int tstep = EVAL ? 1 : *step_ctr;\n";
   for (int q = 0; q < P; ++q) {
     o << "  if (wq == " << q << ") {\n";
     if (q == 0) {
@@ -472,7 +503,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     }
     const auto used = vars_in(rcone[q]);
     for (int j = 0; j < M; ++j)
-      if (used[j]) o << "    const double x" << j << " = exp((double)yin[(size_t)" << j << " * ldy + cc]);\n";
+      if (used[j]) o << "    const double x" << j << " = sx[" << j << " * 32 + lane];\n";
     g.emit_forward(rcone[q], 0, "x", "    ");
     // user-root penalties of this group
     o << "    double pen = 0.0;\n";
@@ -499,9 +530,8 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     for (int j = 0; j < M; ++j) o << "    spart[(" << q << " * NV + " << j << ") * 32 + lane] = gx" << j << ";\n";
     o << "  }\n";
   }
-  // y staging + automatic roots (warp 0)
-  o << "  for (int e = threadIdx.x; e < NV * 32; e += blockDim.x) { const int j = e >> 5, l = e & 31; const int cl = blockIdx.x * 32 + l; sy[e] = yin[(size_t)j * ldy + (cl < n ? cl : n - 1)]; }\n"
-    << "  __syncthreads();\n"
+  // automatic roots (warp 0) from the staged y
+  o << "  __syncthreads();\n  if (!EVAL) TSTAMP(1, 2);\n"
     << "  if (wq == 0) {\n";
   for (int j = 0; j < M; ++j) o << "    const double y" << j << " = (double)sy[" << j << " * 32 + lane];\n";
   for (size_t q = 0; q < autos.size(); ++q) {
@@ -512,7 +542,6 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
   // cost + loss (warp 0); the loss is parked in spen[PG-1 .. ] row 0 after the sum
   o << "  __shared__ float sloss[32];\n"
     << "  if (wq == 0) {\n"
-    << "    float cst = head_b;\n    for (int t = 0; t < n_head_tiles; ++t) cst += c_part[(size_t)t * ld_c + cc];\n"
     << "    double pen = 0.0;\n"
     << "    for (int q = 0; q < PG; ++q) pen += spen[q * 32 + lane];\n"
     << "    for (int r = 0; r < NRA; ++r) { const double p = spa[r * 32 + lane]; pen += p * p; }\n"
@@ -521,11 +550,13 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "    if (live) {\n      if (o_loss) o_loss[c] = loss;\n      if (EVAL && o_cost) o_cost[c] = cst;\n    }\n  }\n";
   // gradient per (var, candidate): thread (wq, lane) handles vars j = wq, wq + PG, ...
   o << "  __shared__ float sgrad[NV][32];\n"
-    << "  for (int j = wq; j < NV; j += PG) {\n"
+    << "#pragma unroll\n"
+    << "  for (int jj = 0; jj < NJ; ++jj) {\n"
+    << "    const int j = wq + PG * jj;\n"
+    << "    if (j >= NV) break;\n"
     << "    double gx = 0.0;\n"
     << "    for (int q = 0; q < PG; ++q) gx += spart[(q * NV + j) * 32 + lane];\n"
-    << "    const double y = (double)sy[j * 32 + lane];\n"
-    << "    double gd = exp(y) * gx;\n"
+    << "    double gd = sx[j * 32 + lane] * gx;\n"
     << "    switch (j) {\n";
   for (int j = 0; j < M; ++j) {
     std::string terms;
@@ -545,17 +576,20 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "    bool ok = isfinite(sloss[lane]);\n"
     << "    for (int j = 0; j < NV; ++j) ok = ok && isfinite(sgrad[j][lane]);\n"
     << "    if (ok && live) {\n"
-    << "      const int t = *step_ctr;\n"
-    << "      const float bc1 = 1.f - powf(b1, (float)t), bc2 = 1.f - powf(b2, (float)t);\n"
+    << "      const float bc1 = 1.f - powf(b1, (float)tstep), bc2 = 1.f - powf(b2, (float)tstep);\n"
     << "      const float step = lr / bc1, rb = 1.f / sqrtf(bc2);\n"
-    << "      for (int j = wq; j < NV; j += PG) {\n"
+    << "#pragma unroll\n"
+    << "      for (int jj = 0; jj < NJ; ++jj) {\n"
+    << "        const int j = wq + PG * jj;\n"
+    << "        if (j >= NV) break;\n"
     << "        const float gy = sgrad[j][lane];\n"
     << "        const size_t o_ = (size_t)j * n + c;\n"
-    << "        float m = mv[o_], v = vv[o_];\n"
+    << "        float m = mreg[jj], v = vreg[jj];\n"
     << "        m = b1 * m + (1.f - b1) * gy; v = b2 * v + (1.f - b2) * gy * gy;\n"
     << "        mv[o_] = m; vv[o_] = v; yv[(size_t)j * ldy + c] = sy[j * 32 + lane] - step * m / (sqrtf(v) * rb + eps);\n"
     << "      }\n"
     << "    }\n"
+    << "    TSTAMP(1, 3);\n"
     << "  }\n}\n\n";
   o << "extern \"C\" __global__ void __launch_bounds__(PG * 32) felix_rev_adam(float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
     << "    float* mv, float* vv, const int* step_ctr, float lr, float b1, float b2, float eps, float* o_loss) {\n"

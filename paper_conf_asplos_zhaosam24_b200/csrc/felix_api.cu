@@ -378,9 +378,15 @@ static felix_space::Module& get_module(felix_space* s, int P) {
 
 // Cone-partition width: enough warps to give every SM ~8 resident warps of expression work.
 static int choose_P(int64_t n) {
-  const int64_t target = int64_t(148) * 8 * 32;
+  if (const char* e = std::getenv("FELIX_P")) {   // experiments: force the cone-partition width
+    const int p = std::atoi(e);
+    if (p == 1 || p == 2 || p == 4 || p == 8 || p == 16) return p;
+  }
+  // measured on B200 (C2 space, per-class event timing): P=4 best at 4096 candidates, P=2 at 32768,
+  // P=1 once the population alone fills the SMs
   int P = 1;
-  while (P < 8 && n * P < target) P *= 2;
+  if (n <= 8192) P = 4;
+  else if (n <= 65536) P = 2;
   return P;
 }
 
@@ -1116,6 +1122,25 @@ felix_status felix_round_topk(felix_space* s, felix_costmodel* m, const float* y
   CUDA_OK(cudaMemcpyAsync(sched_out, s->o_sched.p, static_cast<size_t>(k) * M * 4, cudaMemcpyDeviceToHost, st));
   CUDA_OK(cudaStreamSynchronize(st));
   *n_out = cnt;
+  FELIX_API_END
+}
+
+felix_status felix_debug_trace(felix_space* s, uint64_t* out, int64_t n_words) {
+  FELIX_API_BEGIN
+  if (!s || !out) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL argument");
+  DeviceGuard dg(s->device);
+  for (auto it = s->modules.rbegin(); it != s->modules.rend(); ++it) {   // widest P first (the search's)
+    auto& kv = *it;
+    void* ptr = nullptr;
+    size_t bytes = 0;
+    if (cudaLibraryGetGlobal(&ptr, &bytes, kv.second.lib, "felix_trace") != cudaSuccess) {
+      cudaGetLastError();
+      continue;
+    }
+    CUDA_OK(cudaMemcpy(out, ptr, std::min<size_t>(bytes, static_cast<size_t>(n_words) * 8), cudaMemcpyDeviceToHost));
+    return FELIX_OK;
+  }
+  FELIX_THROW(FELIX_E_UNSUPPORTED, "no trace buffer (set FELIX_TRACE before felix_space_create)");
   FELIX_API_END
 }
 
