@@ -134,7 +134,7 @@ FELIX_EXPORT felix_status felix_space_info(const felix_space* s, felix_space_inf
 
 /* Loads the cost model C: n_layers linear layers, dims[n_layers+1], dims[n_layers] == 1,
  * W[l] host row-major [dims[l+1]][dims[l]] fp32, b[l] host [dims[l+1]] fp32; ReLU between layers,
- * none after the last (TenSet MLP).  Hidden dims must be multiples of 64 and <= 4096,
+ * none after the last (TenSet MLP).  Hidden dims must be multiples of 64 and <= 1024,
  * dims[0] <= 256.  Weights are split on the host into fp16 hi/lo pairs for the tensor cores
  * and kept in fp64 for scoring. */
 FELIX_EXPORT felix_status felix_costmodel_load(int device, int32_t n_layers, const int32_t* dims,

@@ -7,7 +7,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libfelix.so")
 SOURCES = ["felix_api.cu", "codegen.cpp"]
-DEPS = SOURCES + ["felix_internal.h", "mlp_gemm.cuh", "sm100_ptx.cuh", "aux_kernels.cuh",
+DEPS = SOURCES + ["felix_internal.h", "mlp_gemm.cuh", "mlp_chain.cuh", "sm100_ptx.cuh", "aux_kernels.cuh",
                   os.path.join("..", "..", "include", "felix.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-shared",
@@ -25,7 +25,8 @@ def up_to_date() -> bool:
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and up_to_date():
         return LIB
-    cmd = [NVCC] + FLAGS + [os.path.join(CSRC, s) for s in SOURCES] + ["-o", LIB + ".tmp"]
+    extra = os.environ.get("FELIX_NVCC_FLAGS", "").split()      # experiments, e.g. -DFELIX_CHAIN_STAGES=3
+    cmd = [NVCC] + FLAGS + extra + [os.path.join(CSRC, s) for s in SOURCES] + ["-o", LIB + ".tmp"]
     if verbose:
         print(" ".join(cmd), file=sys.stderr)
     r = subprocess.run(cmd, capture_output=True, text=True)

@@ -797,7 +797,7 @@ felix_status felix_costmodel_load(int device, int32_t n_layers, const int32_t* d
   if (dims[n_layers] != 1) FELIX_THROW(FELIX_E_SHAPE, "the last layer must have one output (predicted performance)");
   if (dims[0] < 1 || dims[0] > 256) FELIX_THROW(FELIX_E_UNSUPPORTED, "dims[0] must be in [1, 256]");
   for (int l = 1; l < n_layers; ++l)
-    if (dims[l] <= 0 || dims[l] % 64 != 0 || dims[l] > 4096) FELIX_THROW(FELIX_E_UNSUPPORTED, "hidden dims must be multiples of 64 in [64, 4096]");
+    if (dims[l] <= 0 || dims[l] % 64 != 0 || dims[l] > CHAIN_MAX_N) FELIX_THROW(FELIX_E_UNSUPPORTED, "hidden dims must be multiples of 64 in [64, 1024]");
   for (int l = 0; l < n_layers; ++l) if (!W[l] || !b[l]) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL weight");
   check_device(device);
   DeviceGuard dg(device);

@@ -24,14 +24,20 @@ namespace felix {
 
 constexpr int CHAIN_MAX_LAYERS = 14;
 constexpr int CHAIN_BN_MAX = 128;
-constexpr int CHAIN_STAGES = 3;
+#ifndef FELIX_CHAIN_STAGES
+#define FELIX_CHAIN_STAGES 2
+#endif
+constexpr int CHAIN_STAGES = FELIX_CHAIN_STAGES;
+constexpr int CHAIN_EPI_BUFS = CHAIN_STAGES >= 3 ? 1 : 2;   // epilogue staging buffers (double-buffered when smem allows)
 constexpr int CHAIN_THREADS = 320;
 constexpr int CHAIN_EPI_WARPS = 8;
 constexpr int CHAIN_A_BYTES = GEMM_BM * GEMM_BK * 2;                 // 16 KB (one of hi / lo)
 constexpr int CHAIN_B_BYTES = CHAIN_BN_MAX * GEMM_BK * 2;            // 16 KB
 constexpr int CHAIN_STAGE_BYTES = 2 * CHAIN_A_BYTES + 2 * CHAIN_B_BYTES;
-constexpr int CHAIN_EPI_BYTES = 2 * GEMM_BM * 64 * 2;                 // hi + lo staging of one 64-col chunk
-constexpr int CHAIN_SMEM_BYTES = 1024 + CHAIN_STAGES * CHAIN_STAGE_BYTES + CHAIN_EPI_BYTES + 256;
+constexpr int CHAIN_EPI_BYTES = CHAIN_EPI_BUFS * 2 * GEMM_BM * 64 * 2;   // hi + lo staging of 64-col chunks
+constexpr int CHAIN_MAX_N = 1024;                                  // widest layer staged in smem (bias / head row)
+constexpr int CHAIN_PARAM_BYTES = 2 * CHAIN_MAX_N * 4;
+constexpr int CHAIN_SMEM_BYTES = 1024 + CHAIN_STAGES * CHAIN_STAGE_BYTES + CHAIN_EPI_BYTES + CHAIN_PARAM_BYTES + 256;
 
 struct ChainLayer {
   CUtensorMap a_hi, a_lo, b_hi, b_lo, c_hi, c_lo;
@@ -50,10 +56,13 @@ struct ChainParams {
 };
 
 #ifdef FELIX_CHAIN_TRACE
+#define CHAIN_STAMP2(l, slot) do { unsigned long long t_; asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t_)); \
+    P.trace[(static_cast<size_t>(gridDim.x) * CHAIN_MAX_LAYERS + static_cast<size_t>(blockIdx.x) * CHAIN_MAX_LAYERS + (l)) * 8 + (slot)] = t_; } while (0)
 #define CHAIN_STAMP(l, slot) do { unsigned long long t_; asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t_)); \
     P.trace[(static_cast<size_t>(blockIdx.x) * CHAIN_MAX_LAYERS + (l)) * 8 + (slot)] = t_; } while (0)
 #else
 #define CHAIN_STAMP(l, slot) do {} while (0)
+#define CHAIN_STAMP2(l, slot) do {} while (0)
 #endif
 
 __device__ __forceinline__ void grid_barrier(unsigned int* ctr, unsigned int nblocks) {
@@ -73,9 +82,10 @@ __device__ __forceinline__ void grid_barrier(unsigned int* ctr, unsigned int nbl
 __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __grid_constant__ ChainParams P) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t* epi_hi = smem + CHAIN_STAGES * CHAIN_STAGE_BYTES;
-  uint8_t* epi_lo = epi_hi + GEMM_BM * 64 * 2;
-  uint64_t* full_bar = reinterpret_cast<uint64_t*>(epi_hi + CHAIN_EPI_BYTES);
+  uint8_t* epi_base = smem + CHAIN_STAGES * CHAIN_STAGE_BYTES;   // [buf][hi | lo][128 x 64 fp16]
+  float* s_bias = reinterpret_cast<float*>(epi_base + CHAIN_EPI_BYTES);   // [CHAIN_MAX_N] this layer's bias
+  float* s_headw = s_bias + CHAIN_MAX_N;                                   // [CHAIN_MAX_N] head row (HEAD layer)
+  uint64_t* full_bar = reinterpret_cast<uint64_t*>(epi_base + CHAIN_EPI_BYTES + CHAIN_PARAM_BYTES);
   uint64_t* empty_bar = full_bar + CHAIN_STAGES;
   uint64_t* tfull = empty_bar + CHAIN_STAGES;      // [2] accumulator ready
   uint64_t* tempty = tfull + 2;                    // [2] accumulator drained
@@ -177,23 +187,51 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
     const int half = (warp - 2) >> 2;                // which 32-column half of each 64-column chunk
     const int r_tile = q * 32 + lane;
     const int etid = threadIdx.x - 64;               // 0..255
+    int epi_count = 0;                               // 64-column chunks staged so far (buffer parity)
     constexpr int NEPI = CHAIN_EPI_WARPS * 32;
     int tcount = 0;
     for (int l = 0; l < P.n_layers; ++l) {
       const ChainLayer& L = P.layer[l];
-      const GemmArgs& args = L.args;
-      for (int tile = blockIdx.x; tile < L.n_tiles; tile += G, ++tcount) {
+      // per-layer fields in registers once: read through the dynamically indexed param block, the
+      // compiler otherwise re-fetches each pointer (LDC) before every element access
+      const int epi = L.epi, bn = L.bn, ntn = L.n_tiles_n, ntiles = L.n_tiles;
+      const int aM = L.args.M, aN = L.args.N, n_valid = L.args.n_valid, ld_f32 = L.args.ld_f32, ld_c = L.args.ld_c;
+      const float* __restrict__ bias = L.args.bias;
+      const float* __restrict__ head_w = L.args.head_w;
+      uint32_t* __restrict__ mask_out = L.args.mask_out;
+      const uint32_t* mask_in = L.args.mask_in;
+      float* __restrict__ c_part = L.args.c_part;
+      float* __restrict__ out_f32 = L.args.out_f32;
+      const CUtensorMap* tm_c_hi = &L.c_hi;
+      const CUtensorMap* tm_c_lo = &L.c_lo;
+      // stage this layer's bias / head row in smem while the MMA warp works (previous layer's
+      // readers are past the layer-end barrier, so the buffer is free)
+      if (epi == EPI_RELU || epi == EPI_HEAD) {
+        for (int i = etid; i < aN; i += NEPI) {
+          s_bias[i] = __ldg(&bias[i]);
+          if (epi == EPI_HEAD) s_headw[i] = __ldg(&head_w[i]);
+        }
+      }
+      ptx::named_bar_sync(1, NEPI);
+      for (int tile = blockIdx.x; tile < ntiles; tile += G, ++tcount) {
         const int acc = tcount & 1;
-        const int m0 = (tile / L.n_tiles_n) * GEMM_BM, n0 = (tile % L.n_tiles_n) * L.bn;
+        const int m0 = (tile / ntn) * GEMM_BM, n0 = (tile % ntn) * bn;
         const int row = m0 + r_tile;
-        const bool row_ok = row < args.M;
+        const bool row_ok = row < aM;
+        // this thread's mask words for the tile (<= 2 chunks of 64 columns), requested before the wait
+        uint32_t mwords[CHAIN_BN_MAX / 64] = {0u};
+        if (epi == EPI_MASK && row_ok) {
+#pragma unroll
+          for (int q64 = 0; q64 < CHAIN_BN_MAX / 64; ++q64)
+            if (q64 * 64 < bn) mwords[q64] = __ldcg(&mask_in[static_cast<size_t>(row) * (aN / 32) + (n0 + q64 * 64 + half * 32) / 32]);
+        }
         ptx::mbar_wait(&tfull[acc], (tcount >> 1) & 1);
         if (etid == 0 && tile == static_cast<int>(blockIdx.x)) CHAIN_STAMP(l, 3);
         ptx::tc_fence_after();
         const uint32_t t_row = tmem_base + acc * CHAIN_BN_MAX + (static_cast<uint32_t>(q * 32) << 16);
         float head_acc = 0.f;
-        if (L.epi == EPI_F32T) {
-          for (int c = half * 32; c < L.bn; c += 64) {
+        if (epi == EPI_F32T) {
+          for (int c = half * 32; c < bn; c += 64) {
             float v[32];
             {
               float a[16], b[16];
@@ -206,14 +244,21 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             if (row_ok) {
 #pragma unroll
               for (int i = 0; i < 32; ++i)
-                if (n + i < args.n_valid) args.out_f32[static_cast<size_t>(n + i) * args.ld_f32 + row] = v[i];
+                if (n + i < n_valid) out_f32[static_cast<size_t>(n + i) * ld_f32 + row] = v[i];
             }
           }
         } else {
-          for (int c64 = 0; c64 < L.bn; c64 += 64) {
-            // the staging buffer must be free: previous TMA store finished reading it
-            if (etid == 0) ptx::bulk_wait_read<0>();
+          for (int c64 = 0; c64 < bn; c64 += 64) {
+            // the staging buffer must be free: the TMA store that last used it finished reading
+            uint8_t* epi_hi = epi_base + (epi_count % CHAIN_EPI_BUFS) * (2 * GEMM_BM * 64 * 2);
+            uint8_t* epi_lo = epi_hi + GEMM_BM * 64 * 2;
+            ++epi_count;
+            if (etid == 0) {
+              if (CHAIN_EPI_BUFS == 2) ptx::bulk_wait_read<1>(); else ptx::bulk_wait_read<0>();
+            }
             ptx::named_bar_sync(1, NEPI);
+            const bool st0 = etid == 0 && c64 == 0 && tile == static_cast<int>(blockIdx.x);
+            if (st0) CHAIN_STAMP2(l, 0);
             {
               const int c32 = half * 32;
               const int c = c64 + c32;
@@ -225,29 +270,30 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
 #pragma unroll
                 for (int i = 0; i < 16; ++i) { v[i] = a[i]; v[16 + i] = b[i]; }
               }
+              if (st0) CHAIN_STAMP2(l, 1);
               const int n = n0 + c;
-              if (L.epi == EPI_MASK) {
+              if (epi == EPI_MASK) {
                 // written earlier in this launch by other CTAs: coherent L2 load, not the .nc path
-                const uint32_t bits = row_ok ? __ldcg(&args.mask_in[static_cast<size_t>(row) * (args.N / 32) + n / 32]) : 0u;
+                const uint32_t bits = c64 == 0 ? mwords[0] : mwords[CHAIN_BN_MAX / 64 - 1];
 #pragma unroll
                 for (int i = 0; i < 32; ++i) v[i] = ((bits >> i) & 1u) ? v[i] : 0.f;
               } else {
                 uint32_t bits = 0;
-                const bool head = L.epi == EPI_HEAD;
+                const bool head = epi == EPI_HEAD;
 #pragma unroll
                 for (int i = 0; i < 32; ++i) {
-                  const float z = v[i] + __ldg(&args.bias[n + i]);
+                  const float z = v[i] + s_bias[n + i];
                   const bool on = z > 0.f;
                   bits |= (on ? 1u : 0u) << i;
                   if (!head) {
                     v[i] = on ? z : 0.f;
                   } else {
-                    const float w = __ldg(&args.head_w[n + i]);
+                    const float w = s_headw[n + i];
                     head_acc += (on ? z : 0.f) * w;
                     v[i] = on ? -w : 0.f;        // delta_{L-1} = W_L^T (dL/dc = -1) (.) [Z > 0]
                   }
                 }
-                if (!head && row_ok) args.mask_out[static_cast<size_t>(row) * (args.N / 32) + n / 32] = bits;
+                if (!head && row_ok) mask_out[static_cast<size_t>(row) * (aN / 32) + n / 32] = bits;
               }
 #pragma unroll
               for (int qq = 0; qq < 4; ++qq) {
@@ -268,17 +314,19 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
                 *reinterpret_cast<uint4*>(epi_lo + off) = make_uint4(lo[0], lo[1], lo[2], lo[3]);
               }
             }
+            if (st0) CHAIN_STAMP2(l, 2);
             ptx::fence_proxy_async_smem();
             ptx::named_bar_sync(1, NEPI);
+            if (st0) CHAIN_STAMP2(l, 3);
             if (etid == 0) {
-              ptx::tma_store_2d(&L.c_hi, n0 + c64, m0, epi_hi);
-              ptx::tma_store_2d(&L.c_lo, n0 + c64, m0, epi_lo);
+              ptx::tma_store_2d(tm_c_hi, n0 + c64, m0, epi_hi);
+              ptx::tma_store_2d(tm_c_lo, n0 + c64, m0, epi_lo);
               ptx::bulk_commit();
             }
           }
         }
         // head partial per (N tile, column half); the reverse kernel sums all 2 * N / bn partials
-        if (L.epi == EPI_HEAD && row_ok) args.c_part[static_cast<size_t>(2 * (n0 / L.bn) + half) * args.ld_c + row] = head_acc;
+        if (epi == EPI_HEAD && row_ok) c_part[static_cast<size_t>(2 * (n0 / bn) + half) * ld_c + row] = head_acc;
         // accumulator drained: let the MMA warp reuse it
         ptx::tc_fence_before();
         __syncwarp();

@@ -42,7 +42,7 @@ int main(int argc, char** argv) {
   P.n_layers = 6; P.m_tiles = mt;
   P.grid_bar = (unsigned int*)dz(64);
   int grid = std::min(148, mt * 512 / bnA);
-  P.trace = (unsigned long long*)dz((size_t)grid * CHAIN_MAX_LAYERS * 8 * 8);
+  P.trace = (unsigned long long*)dz((size_t)grid * CHAIN_MAX_LAYERS * 8 * 8 * 2);
   cudaFuncSetAttribute(mlp_chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES);
   for (int it = 0; it < 3; ++it) mlp_chain_kernel<<<grid, CHAIN_THREADS, CHAIN_SMEM_BYTES>>>(P);
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
@@ -51,8 +51,9 @@ int main(int argc, char** argv) {
   cudaEventRecord(e1); cudaEventSynchronize(e1);
   float ms; cudaEventElapsedTime(&ms, e0, e1);
   printf("M=%d grid=%d bnA=%d bnB=%d: %.2f us per chain launch (err=%s)\n", M, grid, bnA, bnB, ms * 100, cudaGetErrorString(cudaGetLastError()));
-  std::vector<unsigned long long> h((size_t)grid * CHAIN_MAX_LAYERS * 8);
+  std::vector<unsigned long long> h((size_t)grid * CHAIN_MAX_LAYERS * 8), h2((size_t)grid * CHAIN_MAX_LAYERS * 8);
   cudaMemcpy(h.data(), P.trace, h.size() * 8, cudaMemcpyDeviceToHost);
+  cudaMemcpy(h2.data(), P.trace + h.size(), h2.size() * 8, cudaMemcpyDeviceToHost);
   unsigned long long t0 = ~0ull;
   for (int b = 0; b < grid; ++b) t0 = std::min(t0, h[(size_t)b * CHAIN_MAX_LAYERS * 8 + 0]);
   const char* nm[7] = {"prodStart", "mma1stFull", "mmaLastCommit", "epiStart", "epiEnd", "barArrive", "barLeave"};
@@ -62,6 +63,14 @@ int main(int argc, char** argv) {
       double mn = 1e18, mx = 0, av = 0; int c = 0;
       for (int b = 0; b < grid; ++b) { unsigned long long v = h[((size_t)b * CHAIN_MAX_LAYERS + l) * 8 + sl]; if (!v) continue; double d = (double)(v - t0); mn = std::min(mn, d); mx = std::max(mx, d); av += d; ++c; }
       if (c) printf("  %s %.2f/%.2f/%.2f", nm[sl], mn / 1e3, av / c / 1e3, mx / 1e3);
+    }
+    printf("\n");
+    printf("   epi chunk0 of tile0:");
+    const char* n2[4] = {"bufFree", "tmemLoaded", "smemWritten", "barPassed"};
+    for (int sl = 0; sl < 4; ++sl) {
+      double av = 0; int c = 0;
+      for (int b = 0; b < grid; ++b) { unsigned long long v = h2[((size_t)b * CHAIN_MAX_LAYERS + l) * 8 + sl]; if (!v) continue; av += (double)(v - t0); ++c; }
+      if (c) printf("  %s %.2f", n2[sl], av / c / 1e3);
     }
     printf("\n");
   }
