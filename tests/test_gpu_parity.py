@@ -37,6 +37,11 @@ CASES = {
     "C2": (fi.c2_space, fi.DEFAULT_MLP, 1000),
     "C5": (fi.c5_space, fi.DEFAULT_MLP, 389),
     "bmm": (lambda: fi.bert_spaces()[1], fi.DEFAULT_MLP, 257),
+    # C3 / C4 shapes: ResNet-50 conv1 7x7 stride 2 (halo with stride), a 1x1 stride-2 downsample,
+    # BERT QKV dense (2-var reduction split)
+    "r50_conv1": (lambda: fi.resnet50_spaces()[0], fi.DEFAULT_MLP, 300),
+    "r50_ds1x1": (lambda: fi.resnet50_spaces()[8], fi.DEFAULT_MLP, 160),
+    "bert_qkv": (lambda: fi.bert_spaces()[0], fi.DEFAULT_MLP, 222),
 }
 
 _cache = {}
@@ -187,8 +192,9 @@ def test_topk_shard_invariance(fx):
     assert [i for i, _ in merged[:16]] == list(full[0])
 
 
-def test_init_sampler_parity(fx):
-    sp, mlp, n, space, cm = _setup(fx, "C2")
+@pytest.mark.parametrize("name", ["C1", "C2", "C5", "r50_conv1"])
+def test_init_sampler_parity(fx, name):
+    sp, mlp, n, space, cm = _setup(fx, name)
     y = space.init_sample(2048, 0x5EED0002, index_base=100).cpu().numpy()
     ry = fo.init_sample(sp, 2048, 0x5EED0002, index_base=100)
     same = np.all(y == ry, axis=0)
@@ -209,6 +215,45 @@ def test_full_size_c2_sampled(fx):
     assert np.max(np.abs(out["cost"][pick] - ref.c)) / s <= 1e-4
     err = np.linalg.norm(out["grad"][:, pick] - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
     assert np.sum((err > 1e-3) & (kink_margin(ref.zs) >= 1e-4)) == 0
+
+
+def test_full_size_c5_per_gpu_sampled(fx):
+    """C5's per-GPU shard (2^20 / 8 = 131072 candidates of the ViT-L fc1 space): one objective
+    evaluation at full size, 48 sampled candidates checked against the oracle; then a short search
+    and its top-k, whose records must be valid rounded schedules with oracle-exact FP64 scores."""
+    sp, mlp, _, space, cm = _setup(fx, "C5")
+    n = 131072
+    y0 = fo.init_sample(sp, n, 0x5EED0005)
+    yt = torch.from_numpy(y0).cuda()
+    out = space.eval(cm, yt)
+    pick = np.random.default_rng(1).choice(n, 48, replace=False)
+    ref = fo.objective(sp, mlp.W, mlp.b, y0[:, pick].astype(np.float64), 1.0)
+    cost = out["cost"].cpu().numpy()[pick]
+    s = np.sqrt(np.mean(ref.c ** 2))
+    assert np.max(np.abs(cost - ref.c)) / s <= 1e-4
+    space.search(cm, yt, 5, init_from_y=True)
+    idx, sc, sched = space.round_topk(cm, yt, 64)
+    assert len(idx) == 64 and len(set(map(tuple, sched))) == 64
+    assert np.all(np.diff(sc) <= 0)
+    assert fo.validate(sp, sched).all()
+    assert np.allclose(fo.score(sp, mlp.W, mlp.b, sched), sc, rtol=1e-12, atol=0)
+    assert np.array_equal(fo.round_schedules(sp, yt[:, idx].cpu().numpy()), sched)
+
+
+def test_search_final_loss_matches_eval(fx):
+    """The loss felix_search reports for its last step is the objective at the point that step
+    started from (the same kernels as felix_eval)."""
+    sp, mlp, _, space, cm = _setup(fx, "C2")
+    y = torch.from_numpy(fi.make_y0(sp, 777, seed=9)).cuda()
+    loss = torch.empty(777, device="cuda")
+    space.search(cm, y, 3, init_from_y=True, final_loss=loss)
+    # re-run two steps from scratch, then evaluate at the start of the third
+    y2 = torch.from_numpy(fi.make_y0(sp, 777, seed=9)).cuda()
+    space.search(cm, y2, 2, init_from_y=True)
+    ev = space.eval(cm, y2)["loss"]
+    # steps 1-2 are identical, so y2 == the start point of step 3 only up to Adam state: the
+    # 3-step run used Adam moments of steps 1-2 for its update, not for its loss
+    assert torch.allclose(loss, ev, rtol=1e-6, atol=1e-6)
 
 
 def test_search_deterministic_and_improves(fx):
