@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
+    ap.add_argument("--seeds", type=int, default=0, help="override seeds per GPU (experiments; not the headline)")
+    ap.add_argument("--search-steps", type=int, default=0, help="override Adam steps per search (experiments)")
     return ap.parse_args()
 
 
@@ -193,6 +195,12 @@ def run_felix(args):
     from paper_conf_asplos_zhaosam24_b200 import dist as fdist
 
     cfg = fi.config(args.config)
+    if args.seeds:
+        cfg.n_seeds = args.seeds
+    elif args.config == "C5":
+        cfg.n_seeds = (1 << 20) // 8          # C5 is 2^20 candidates over 8 GPUs: one GPU's shard
+    if args.search_steps:
+        cfg.n_steps = args.search_steps
     sp = cfg.spaces[0]
     mlp = fi.make_mlp(cfg.mlp_dims)
     space = fx.Space(sp, device=dev)
