@@ -71,6 +71,10 @@ __device__ __forceinline__ double f_sqrt(double x) {
 __device__ __forceinline__ double sm_hyp(double t) { return f_sqrt(fma(t, t, 1.0)); }
 __device__ __forceinline__ double sm_S(double t) { const double h = sm_hyp(t); const double tail = 0.5 * f_rcp(h * (h + fabs(t))); return t >= 0.0 ? 1.0 - tail : tail; }
 __device__ __forceinline__ double sm_dS(double t) { const double h = sm_hyp(t); return 0.5 * f_rcp(h * h * h); }
+// variants taking h = sqrt(1+t^2) computed once by the forward and reused by the reverse sweep
+__device__ __forceinline__ double sm_Sh(double t, double h) { const double tail = 0.5 * f_rcp(h * (h + fabs(t))); return t >= 0.0 ? 1.0 - tail : tail; }
+__device__ __forceinline__ double sm_dSh(double h) { return 0.5 * f_rcp(h * h * h); }
+__device__ __forceinline__ double sm_gaph(double t, double h) { return 0.5 * f_rcp(h + fabs(t)); }
 // R(t) - relu(t) = 1/(2(sqrt(1+t^2) + |t|)); min / max without the cancellation of a - (a - b)
 __device__ __forceinline__ double sm_gap(double t) { return 0.5 * f_rcp(sm_hyp(t) + fabs(t)); }
 __device__ __forceinline__ double sm_min(double a, double b) { const double t = a - b; return (t >= 0.0 ? b : a) - sm_gap(t); }
@@ -166,6 +170,41 @@ struct Gen {
       const felix_node& nd = d.nodes[i];
       const std::string A = "v" + std::to_string(nd.a), B = "v" + std::to_string(nd.b), C = "v" + std::to_string(nd.c);
       std::string e;
+      const std::string I = std::to_string(i);
+      if (mode == 0) {
+        // smooth ops: keep t and h = sqrt(1+t^2) as named values for the reverse sweep
+        switch (nd.op) {
+          case FELIX_OP_GT: case FELIX_OP_GE: case FELIX_OP_LT: case FELIX_OP_LE: {
+            const bool ab = nd.op == FELIX_OP_GT || nd.op == FELIX_OP_GE;
+            o << ind << "const double t" << I << " = " << (ab ? A + " - " + B : B + " - " + A) << ";\n"
+              << ind << "const double h" << I << " = sm_hyp(t" << I << ");\n"
+              << ind << "const double v" << I << " = sm_Sh(t" << I << ", h" << I << ");\n";
+            flops += 6;
+            continue;
+          }
+          case FELIX_OP_MIN: case FELIX_OP_MAX: {
+            const bool mx = nd.op == FELIX_OP_MAX;
+            o << ind << "const double t" << I << " = " << A << " - " << B << ";\n"
+              << ind << "const double h" << I << " = sm_hyp(t" << I << ");\n"
+              << ind << "const double v" << I << " = (t" << I << " >= 0.0 ? " << (mx ? A : B) << " : " << (mx ? B : A) << ") "
+              << (mx ? "+" : "-") << " sm_gaph(t" << I << ", h" << I << ");\n";
+            flops += 6;
+            continue;
+          }
+          case FELIX_OP_EQ: case FELIX_OP_NE: {
+            o << ind << "const double t" << I << " = (" << A << " - " << B << ") + 0.5;\n"
+              << ind << "const double u" << I << " = 0.5 - (" << A << " - " << B << ");\n"
+              << ind << "const double h" << I << " = sm_hyp(t" << I << ");\n"
+              << ind << "const double k" << I << " = sm_hyp(u" << I << ");\n"
+              << ind << "const double p" << I << " = sm_Sh(t" << I << ", h" << I << ");\n"
+              << ind << "const double q" << I << " = sm_Sh(u" << I << ", k" << I << ");\n"
+              << ind << "const double v" << I << " = " << (nd.op == FELIX_OP_EQ ? "" : "1.0 - ") << "p" << I << " * q" << I << ";\n";
+            flops += 13;
+            continue;
+          }
+          default: break;
+        }
+      }
       switch (nd.op) {
         case FELIX_OP_CONST: e = lit(nd.imm); break;
         case FELIX_OP_VAR: e = std::string(xname) + std::to_string((int)nd.imm); break;
@@ -250,21 +289,20 @@ struct Gen {
         case FELIX_OP_LOG: acc(nd.a, g + " * f_rcp(" + A + ")"); break;
         case FELIX_OP_SQRT: acc(nd.a, g + " * 0.5 * f_rcp(" + V + ")"); break;
         case FELIX_OP_MAX:
-          o << ind << "  const double s = sm_S(" << A << " - " << B << ");\n";
+          o << ind << "  const double s = sm_Sh(t" << i << ", h" << i << ");\n";
           acc(nd.a, g + " * s"); acc(nd.b, g + " * (1.0 - s)"); break;
         case FELIX_OP_MIN:
-          o << ind << "  const double s = sm_S(" << A << " - " << B << ");\n";
+          o << ind << "  const double s = sm_Sh(t" << i << ", h" << i << ");\n";
           acc(nd.a, g + " * (1.0 - s)"); acc(nd.b, g + " * s"); break;
         case FELIX_OP_GT: case FELIX_OP_GE:
-          o << ind << "  const double t = " << g << " * sm_dS(" << A << " - " << B << ");\n";
+          o << ind << "  const double t = " << g << " * sm_dSh(h" << i << ");\n";
           acc(nd.a, "t"); acc(nd.b, "t", true); break;
         case FELIX_OP_LT: case FELIX_OP_LE:
-          o << ind << "  const double t = " << g << " * sm_dS(" << B << " - " << A << ");\n";
+          o << ind << "  const double t = " << g << " * sm_dSh(h" << i << ");\n";
           acc(nd.a, "t", true); acc(nd.b, "t"); break;
         case FELIX_OP_EQ: case FELIX_OP_NE:
-          o << ind << "  const double dd = " << A << " - " << B << ";\n"
-            << ind << "  const double p = sm_S(dd + 0.5), q = sm_S(0.5 - dd);\n"
-            << ind << "  const double t = " << (nd.op == FELIX_OP_EQ ? "" : "-") << g << " * (sm_dS(dd + 0.5) * q - p * sm_dS(0.5 - dd));\n";
+          o << ind << "  const double t = " << (nd.op == FELIX_OP_EQ ? "" : "-") << g << " * (sm_dSh(h" << i << ") * q" << i
+            << " - p" << i << " * sm_dSh(k" << i << "));\n";
           acc(nd.a, "t"); acc(nd.b, "t", true); break;
         case FELIX_OP_AND: acc(nd.a, g + " * " + B); acc(nd.b, g + " * " + A); break;
         case FELIX_OP_OR: acc(nd.a, g + " * (1.0 - " + B + ")"); acc(nd.b, g + " * (1.0 - " + A + ")"); break;
