@@ -278,11 +278,21 @@ def run_felix(args):
     barrier()
     finish_ms = f0.elapsed_time(f1)
 
-    # ---- roofline of the dominant kernel: the persistent tcgen05 MLP chain (tensor-bound contraction)
+    # ---- roofline of the dominant kernel: the tcgen05 MLP (tensor-bound contraction).  Which MLP kernel
+    # runs follows felix_api.cu mlp_mode(): the tile-local fused kernel from one full wave of 128-row
+    # tiles (TenSet widths), the persistent layer chain below that; FELIX_MLP overrides.
     peaks, peak_src = measured_peaks()
+    sms = torch.cuda.get_device_properties(dev).multi_processor_count
+    env_mode = os.environ.get("FELIX_MLP", "")
+    tile_fits = tuple(cfg.mlp_dims[1:]) == (512, 256, 256, 1)
+    if env_mode in ("chain", "layers"):
+        mlp_kernel = "mlp_chain_kernel" if env_mode == "chain" else "mlp_gemm_kernel"
+    else:
+        mlp_kernel = "mlp_tile_kernel" if tile_fits and (env_mode == "tile" or -(-n // 128) >= sms) else "mlp_chain_kernel"
     traffic = None
-    tpath = os.path.join(ROOT, "profiles", "r01", "roofline_traffic.json")
-    if os.path.exists(tpath):
+    tname = {"mlp_chain_kernel": "roofline_traffic.json", "mlp_tile_kernel": "roofline_traffic_tile.json"}.get(mlp_kernel, "")
+    tpath = os.path.join(ROOT, "profiles", "r01", tname) if tname else ""
+    if tname and os.path.exists(tpath):
         with open(tpath) as f:
             tj = json.load(f)
         traffic = tj["dram_bytes_read_per_launch"] + tj["dram_bytes_write_per_launch"]
@@ -349,8 +359,9 @@ def run_felix(args):
                    "l2": "flushed (256 MB write) between timed iterations"},
         "roofline": {"bound": "tensor", "achieved": achieved_tflops, "peak": peak, "unit": "TFLOP/s",
                      "frac": achieved_tflops / peak, "traffic": traffic,
-                     "kernel": f"mlp_chain_kernel (all {n_gemm} MLP layers of one Adam step, tcgen05 kind::f16, 3-pass hi/lo split)",
-                     "traffic_source": "profiles/r01/roofline_traffic.json (ncu --set full, DRAM bytes per launch)",
+                     "kernel": f"{mlp_kernel} (all {n_gemm} MLP layers of one Adam step, tcgen05 kind::f16, 3-pass hi/lo split)",
+                     "traffic_source": (f"profiles/r01/{tname} (ncu --set full, DRAM bytes per launch)"
+                                        if traffic is not None else None),
                      "algorithmic_flops_per_adam_step": mlp_flops_step,
                      "executed_tflops": 3 * achieved_tflops,
                      "peak_source": f"{peak_src} bf16_tflops_sustained (fp16 = bf16 rate)"},

@@ -7,7 +7,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libfelix.so")
 SOURCES = ["felix_api.cu", "codegen.cpp"]
-DEPS = SOURCES + ["felix_internal.h", "mlp_gemm.cuh", "mlp_chain.cuh", "sm100_ptx.cuh", "aux_kernels.cuh",
+DEPS = SOURCES + ["felix_internal.h", "mlp_gemm.cuh", "mlp_chain.cuh", "mlp_tile.cuh", "sm100_ptx.cuh", "aux_kernels.cuh",
                   os.path.join("..", "..", "include", "felix.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-shared",

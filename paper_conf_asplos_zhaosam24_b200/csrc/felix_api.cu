@@ -21,6 +21,7 @@
 #include "felix_internal.h"
 #include "mlp_gemm.cuh"
 #include "mlp_chain.cuh"
+#include "mlp_tile.cuh"
 #include "aux_kernels.cuh"
 
 namespace felix {
@@ -120,14 +121,59 @@ struct Plan {
   DevBuf c_part, dphi, m, v, step_ctr;
   int n_head_tiles = 0;
   std::vector<GemmLaunch> gemms;           // per-layer kernels (FELIX_MLP=layers)
-  ChainParams chain{};                     // persistent all-layer kernel (default)
+  ChainParams chain{};                     // persistent all-layer kernel
   int chain_grid = 0;
   DevBuf grid_bar;
+  bool tile_ok = false;                    // model has the shape mlp_tile_kernel is specialised for
+  TileParams tile{};                       // tile-local fused MLP (default when tile_ok)
+  int tile_grid = 0;
+  int tile_cg = 1;                         // 1 = one SM per 128-row tile; FELIX_TILE_CG=2: 2-SM cta_group::2 pairs
+  bool tile_full_wave = false;             // >= one 128-row tile per SM
+  int mode = 0;                            // MlpMode, fixed when the plan is built
 };
 
+// MLP execution mode: "tile" (tile-local fused kernel), "chain" (persistent layer-by-layer kernel),
+// "layers" (one kernel per GEMM).  FELIX_MLP overrides.  Default (measured on B200, DESIGN.md
+// "MLP modes"): a tile's serial on-chip pipeline takes ~55 us whatever the population, so the tile
+// kernel wins once there is at least one full wave of 128-row tiles (C5 shard: 364 vs 518 us per
+// Adam step) and the chain, which spreads every layer over all SMs, wins below that (C2: 48 vs 56 us).
+enum MlpMode { MLP_TILE, MLP_CHAIN, MLP_LAYERS };
+static MlpMode mlp_mode(const Plan& p) {
+  const char* e = std::getenv("FELIX_MLP");
+  if (e && std::string(e) == "layers") return MLP_LAYERS;
+  if (e && std::string(e) == "chain") return MLP_CHAIN;
+  if (e && std::string(e) == "tile" && p.tile_ok) return MLP_TILE;
+  return (p.tile_ok && p.tile_full_wave) ? MLP_TILE : MLP_CHAIN;
+}
 static bool use_chain() {
   const char* e = std::getenv("FELIX_MLP");
   return !(e && std::string(e) == "layers");
+}
+
+static void launch_tile(const Plan& p, cudaStream_t st) {
+  static bool attr_set[3] = {false, false, false};
+  const void* fn = p.tile_cg == 2 ? reinterpret_cast<const void*>(mlp_tile_kernel<2>)
+                                  : reinterpret_cast<const void*>(mlp_tile_kernel<1>);
+  if (!attr_set[p.tile_cg]) {
+    CUDA_OK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, tile::SMEM_BYTES));
+    if (p.tile_cg == 2) CUDA_OK(cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 0));
+    attr_set[p.tile_cg] = true;
+  }
+  cudaLaunchAttribute attrs[2];
+  attrs[0] = g_pdl_attr;
+  attrs[1].id = cudaLaunchAttributeClusterDimension;
+  attrs[1].val.clusterDim.x = static_cast<unsigned>(p.tile_cg);
+  attrs[1].val.clusterDim.y = 1;
+  attrs[1].val.clusterDim.z = 1;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(static_cast<unsigned>(p.tile_grid));
+  cfg.blockDim = dim3(tile::THREADS);
+  cfg.dynamicSmemBytes = tile::SMEM_BYTES;
+  cfg.stream = st;
+  cfg.attrs = attrs;
+  cfg.numAttrs = p.tile_cg == 2 ? 2 : 1;
+  if (p.tile_cg == 2) CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_tile_kernel<2>, p.tile));
+  else CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_tile_kernel<1>, p.tile));
 }
 
 static void launch_chain(const Plan& p, cudaStream_t st) {
@@ -545,6 +591,47 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
     max_tiles = std::max(max_tiles, L.n_tiles);
   }
   p->chain_grid = std::min(sms, max_tiles);
+  // tile-local fused MLP: TenSet widths [K0p, 512, 256, 256, 1] only
+  p->tile_ok = L == 4 && d[1] == tile::D1 && d[2] == tile::D2 && d[3] == tile::D3 && K0p <= 128 && K0p % 32 == 0;   // K0p/2 rows: multiple of 16
+  if (p->tile_ok) {
+    if (const char* e = std::getenv("FELIX_TILE_CG")) p->tile_cg = std::atoi(e) == 2 ? 2 : 1;
+    p->tile_full_wave = mt >= sms;
+    const int cg = p->tile_cg;
+    TileParams& t = p->tile;
+    t.phi_hi = make_tmap(p->phi_hi.p, n, K0p, 128);
+    t.phi_lo = make_tmap(p->phi_lo.p, n, K0p, 128);
+    t.w1_hi = make_tmap(cm->W_hi[0]->p, d[1], K0p, 128 / cg);
+    t.w1_lo = make_tmap(cm->W_lo[0]->p, d[1], K0p, 128 / cg);
+    t.w2_hi = make_tmap(cm->W_hi[1]->p, d[2], d[1], 128);
+    t.w2_lo = make_tmap(cm->W_lo[1]->p, d[2], d[1], 128);
+    t.w3_hi = make_tmap(cm->W_hi[2]->p, d[3], d[2], 128);
+    t.w3_lo = make_tmap(cm->W_lo[2]->p, d[3], d[2], 128);
+    t.w3t_hi = make_tmap(cm->WT_hi[2]->p, d[2], d[3], 128);
+    t.w3t_lo = make_tmap(cm->WT_lo[2]->p, d[2], d[3], 128);
+    t.w2t_hi = make_tmap(cm->WT_hi[1]->p, d[1], d[2], 128 / cg);
+    t.w2t_lo = make_tmap(cm->WT_lo[1]->p, d[1], d[2], 128 / cg);
+    t.w1t_hi = make_tmap(cm->WT_hi[0]->p, K0p, d[1], K0p / cg);
+    t.w1t_lo = make_tmap(cm->WT_lo[0]->p, K0p, d[1], K0p / cg);
+    t.b1 = cm->bias[0]->as<float>();
+    t.b2 = cm->bias[1]->as<float>();
+    t.b3 = cm->bias[2]->as<float>();
+    t.w4 = cm->head_w.as<float>();
+    t.c_part = p->c_part.as<float>();
+    t.dphi = p->dphi.as<float>();
+    t.ld = static_cast<int>(np);
+    t.n = static_cast<int>(n);
+    t.n_tiles = static_cast<int>(mt);
+    t.k0p = K0p;
+    t.n_valid = d[0];
+    t.idesc_128 = ptx::idesc_f16_f32(128 * cg, 128);
+    t.idesc_256 = ptx::idesc_f16_f32(128 * cg, 256);
+    t.idesc_k0p = ptx::idesc_f16_f32(128 * cg, static_cast<uint32_t>(K0p));
+    const int64_t units = (mt + cg - 1) / cg;
+    p->tile_grid = static_cast<int>(std::min<int64_t>(sms / cg, units) * cg);
+  }
+  p->mode = mlp_mode(*p);
+  if (p->mode == MLP_TILE) p->n_head_tiles = 2;                           // one partial per column half
+  else if (p->mode == MLP_LAYERS) p->n_head_tiles = p->gemms[L - 2].args.N / p->gemms[L - 2].bn;
   return p;
 }
 
@@ -601,13 +688,16 @@ static void run_forward_mlp(felix_space* s, Plan& p, const felix_space::Module& 
   prof_mark(s, 0, st, false);
   s->prof_launches[0] += 1;
   prof_mark(s, 1, st, true);
-  if (use_chain()) {
+  const MlpMode mode = static_cast<MlpMode>(p.mode);
+  if (mode == MLP_TILE) {
+    launch_tile(p, st);
+  } else if (mode == MLP_CHAIN) {
     launch_chain(p, st);
   } else {
     for (const auto& g : p.gemms) launch_gemm(g, st);
   }
   prof_mark(s, 1, st, false);
-  s->prof_launches[1] += use_chain() ? 1 : static_cast<int64_t>(p.gemms.size());
+  s->prof_launches[1] += mode == MLP_LAYERS ? static_cast<int64_t>(p.gemms.size()) : 1;
 }
 
 }  // namespace felix
@@ -949,7 +1039,8 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     }
     for (int t = 1; t <= p->n_steps; ++t) CUDA_OK(cudaGraphLaunch(ch.graph, st));
     s->prof_launches[0] += static_cast<int64_t>(p->n_steps) * nck;
-    s->prof_launches[1] += static_cast<int64_t>(p->n_steps) * nck * (use_chain() ? 1 : static_cast<int64_t>(ch.plans[0]->gemms.size()));
+    s->prof_launches[1] += static_cast<int64_t>(p->n_steps) * nck *
+                           (ch.plans[0]->mode == MLP_LAYERS ? static_cast<int64_t>(ch.plans[0]->gemms.size()) : 1);
     s->prof_launches[2] += static_cast<int64_t>(p->n_steps) * nck;
   }
   FELIX_API_END

@@ -306,3 +306,47 @@ def test_shape_errors(fx):
         fx.CostModel.from_weights(fi.make_mlp((82, 100, 1)))
     assert e.value.status == 4
     del bad
+
+
+@pytest.mark.parametrize("mode,cg", [("chain", "1"), ("layers", "1"), ("tile", "2")])
+def test_mlp_execution_modes_agree(fx, mode, cg, monkeypatch):
+    """The tile-local fused MLP (1-SM and 2-SM cta_group::2 variants), the persistent chain and the
+    per-layer kernels compute the same split-fp16 products in the same K order: cost and gradient
+    agree to fp32 summation-order noise (the head partial sums are grouped differently)."""
+    sp = fi.c2_space()
+    mlp = fi.make_mlp(fi.DEFAULT_MLP)
+    n = 2000
+    y0 = torch.from_numpy(fi.make_y0(sp, n, seed=5)).cuda()
+    cm = fx.CostModel.from_weights(mlp)
+    monkeypatch.setenv("FELIX_MLP", "tile")
+    monkeypatch.setenv("FELIX_TILE_CG", "1")
+    base = fx.Space(sp).eval(cm, y0, lam=1.0)
+    monkeypatch.setenv("FELIX_MLP", mode)
+    monkeypatch.setenv("FELIX_TILE_CG", cg)
+    other = fx.Space(sp).eval(cm, y0, lam=1.0)
+    for key in ("cost", "grad"):
+        a, b = base[key].cpu().numpy(), other[key].cpu().numpy()
+        s = np.sqrt(np.mean(a.astype(np.float64) ** 2))
+        assert np.max(np.abs(a - b)) / s <= 1e-5, key
+
+
+@pytest.mark.parametrize("cg", ["1", "2"])
+def test_tile_mlp_eval_parity_vs_oracle(fx, cg, monkeypatch):
+    """Tile-local fused MLP (forced; default only from one full wave of tiles) against the oracle on
+    C2 and C5 shapes with a ragged last tile (and, for the 2-SM pairs, an odd tile count)."""
+    monkeypatch.setenv("FELIX_MLP", "tile")
+    monkeypatch.setenv("FELIX_TILE_CG", cg)
+    for name, n in (("C2", 1000), ("C5", 389)):
+        make, dims, _ = CASES[name]
+        sp = make()
+        mlp = fi.make_mlp(dims)
+        y0 = fi.make_y0(sp, n, seed=21)
+        out = {k: v.cpu().numpy() for k, v in fx.Space(sp).eval(fx.CostModel.from_weights(mlp),
+                                                                  torch.from_numpy(y0).cuda(), lam=1.0).items()}
+        ref = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
+        s = np.sqrt(np.mean(ref.c ** 2))
+        assert np.max(np.abs(out["cost"] - ref.c)) / s <= 1e-4, name
+        km = kink_margin(ref.zs)
+        err = np.linalg.norm(out["grad"] - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
+        bad = (err > 1e-3) & ~(km < 1e-4)
+        assert not np.any(bad), (name, np.nonzero(bad)[0][:10], err[bad][:10])
