@@ -38,7 +38,7 @@
 extern "C" {
 #endif
 
-#define FELIX_ABI_VERSION 1
+#define FELIX_ABI_VERSION 2
 
 #if defined(__GNUC__)
 #define FELIX_EXPORT __attribute__((visibility("default")))
@@ -148,14 +148,19 @@ FELIX_EXPORT void felix_costmodel_destroy(felix_costmodel* m);
  * non-finite is not updated that step (reading R-NaN).
  * y: device fp32 SoA [n_vars][n_seeds].  If init_from_y == 0 it is OUTPUT-only and first filled by
  * the rejection sampler (felix_init_sample with rng_seed / index_base); else it is the start point.
- * final_loss: device fp32 [n_seeds] or NULL — the loss at the point of the last step's evaluation. */
+ * final_loss: device fp32 [n_seeds] or NULL — the loss at the point of the last step's evaluation.
+ * history != 0: also record varValuesHistory (Alg. 1 lines 13 and 17): every point at
+ * which the objective is evaluated, sigma_x_i for i = 0 .. n_steps-1, is rounded on the device (same
+ * rounding as felix_round_topk) and each schedule not seen before in this search is kept with its
+ * first (step, global index); read the result with felix_history_topk.  Starting a search clears the
+ * previous history.  Device memory grows with n_seeds x n_steps schedules (worst case). */
 typedef struct {
   int64_t n_seeds;
   int32_t n_steps;
   float lr, beta1, beta2, eps, lambda;   /* reading O8 defaults: 0.05, 0.9, 0.999, 1e-8, 1.0 */
   uint64_t rng_seed;
   int32_t init_from_y;
-  int32_t _pad;
+  int32_t history;                       /* 0: round the final point only (felix_round_topk) */
   int64_t index_base;
 } felix_search_params;
 FELIX_EXPORT felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search_params* p,
@@ -171,6 +176,19 @@ FELIX_EXPORT felix_status felix_search(felix_space* s, felix_costmodel* m, const
 FELIX_EXPORT felix_status felix_round_topk(felix_space* s, felix_costmodel* m, const float* y, int64_t n,
                               int64_t index_base, int32_t k, int64_t* idx_out, double* score_out,
                               int32_t* sched_out, int32_t* n_out, void* stream);
+
+/* Algorithm 1 lines 20-21 over the history of the last felix_search run with history != 0 (paper-
+ * faithful Alg. 1: "takes all the variable values traversed in the optimization process, rounds them
+ * to integers ... and removes invalid rounded schedules"): every distinct rounded schedule
+ * visited at steps 0 .. n_steps-1 is validated (hard semantics) and scored in FP64 as in
+ * felix_round_topk; the best k by (score desc, step asc, global index asc) are returned, each with the
+ * first (step, global index) at which it was visited.  Outputs are HOST arrays: idx_out[k] global
+ * indices, step_out[k], score_out[k], sched_out[k][n_vars]; *n_out = number filled (<= k);
+ * *n_unique_out (may be NULL) = distinct schedules visited (valid or not).  Synchronises `stream`.
+ * FELIX_E_INVALID_ARG if the last search did not record a history. */
+FELIX_EXPORT felix_status felix_history_topk(felix_space* s, felix_costmodel* m, int32_t k, int64_t* idx_out,
+                                int32_t* step_out, double* score_out, int32_t* sched_out, int32_t* n_out,
+                                int64_t* n_unique_out, void* stream);
 
 /* ---------------------------------------------------------------- test hooks (same kernels)
  * felix_eval: one objective + gradient evaluation, no Adam.  y device [n_vars][n].  Outputs (device,

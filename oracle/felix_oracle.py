@@ -626,3 +626,32 @@ def round_topk(space, W, b, y: np.ndarray, k: int, index_base: int = 0):
     order = sorted(uniq.tolist(), key=lambda i: (-sc[i], gidx[i]))
     sel = np.array(order[:k], dtype=np.int64)
     return gidx[sel], sc[sel], sched[sel]
+
+
+def round_topk_history(space, W, b, ys: Sequence[np.ndarray], k: int, index_base: int = 0):
+    """Algorithm 1 lines 20-21 over varValuesHistory (lines 13, 17; "takes all
+    the variable values traversed in the optimization process, rounds them to integers ... removes
+    invalid rounded schedules ... takes the best nMeasure schedules").  ys[i] is sigma_x at which step
+    i's objective was evaluated.  Every point is rounded, validated and scored exactly as round_topk;
+    a schedule visited several times counts once, with its first (step, global index); the best k are
+    returned by (score desc, step asc, global index asc).
+    Returns (idx int64 [m], step int32 [m], score f64 [m], sched int32 [m, M], n_unique)."""
+    first = {}                                   # schedule bytes -> (step, seed, score, valid, sched)
+    for i, y in enumerate(ys):
+        sched = round_schedules(space, y)
+        valid = validate(space, sched)
+        sc = score(space, W, b, sched)
+        for s in range(sched.shape[0]):          # ascending (step, seed): the first visit is kept
+            key = sched[s].tobytes()
+            if key not in first:
+                first[key] = (i, s, sc[s], bool(valid[s]) and bool(np.isfinite(sc[s])), sched[s].copy())
+    n_unique = len(first)
+    recs = [r for r in first.values() if r[3]]
+    recs.sort(key=lambda r: (-r[2], r[0], r[1]))
+    recs = recs[:k]
+    M = space.n_vars
+    idx = np.array([index_base + r[1] for r in recs], dtype=np.int64)
+    step = np.array([r[0] for r in recs], dtype=np.int32)
+    scr = np.array([r[2] for r in recs], dtype=np.float64)
+    sch = np.array([r[4] for r in recs], dtype=np.int32).reshape(len(recs), M)
+    return idx, step, scr, sch, n_unique

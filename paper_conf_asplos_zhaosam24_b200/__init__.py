@@ -29,7 +29,7 @@ EXPORTED = ["felix_last_error", "felix_abi_version", "felix_space_create", "feli
             "felix_space_info", "felix_codegen", "felix_costmodel_load", "felix_costmodel_destroy",
             "felix_search", "felix_round_topk", "felix_eval", "felix_round", "felix_score",
             "felix_init_sample", "felix_profile_enable", "felix_profile_read", "felix_profile_reset",
-            "felix_debug_trace"]
+            "felix_debug_trace", "felix_history_topk"]
 
 
 class FelixError(RuntimeError):
@@ -51,7 +51,7 @@ class _SearchParams(ctypes.Structure):
     _fields_ = [("n_seeds", ctypes.c_int64), ("n_steps", ctypes.c_int32), ("lr", ctypes.c_float),
                 ("beta1", ctypes.c_float), ("beta2", ctypes.c_float), ("eps", ctypes.c_float),
                 ("lam", ctypes.c_float), ("rng_seed", ctypes.c_uint64), ("init_from_y", ctypes.c_int32),
-                ("_pad", ctypes.c_int32), ("index_base", ctypes.c_int64)]
+                ("history", ctypes.c_int32), ("index_base", ctypes.c_int64)]
 
 
 class _SpaceInfo(ctypes.Structure):
@@ -193,11 +193,13 @@ class Space:
 
     # ---------------------------------------------------------------- primary calls
     def search(self, cm: CostModel, y, n_steps: int, *, lr=0.05, beta1=0.9, beta2=0.999, eps=1e-8, lam=1.0,
-               rng_seed: int = 0, init_from_y: bool = True, index_base: int = 0, final_loss=None, stream=None):
-        """felix_search on device y (torch fp32 [n_vars, n], updated in place)."""
+               rng_seed: int = 0, init_from_y: bool = True, index_base: int = 0, final_loss=None, history=False,
+               stream=None):
+        """felix_search on device y (torch fp32 [n_vars, n], updated in place).  history=True also records
+        varValuesHistory (Alg. 1 l.13/17) for history_topk."""
         self._check_y(y)
         p = _SearchParams(int(y.shape[1]), int(n_steps), lr, beta1, beta2, eps, lam, int(rng_seed) & (2**64 - 1),
-                          1 if init_from_y else 0, 0, int(index_base))
+                          1 if init_from_y else 0, 1 if history else 0, int(index_base))
         _check(_lib.felix_search(self._h, cm._h, ctypes.byref(p), _P(_ptr(y)), _P(_ptr(final_loss)),
                                  _P(_stream(stream))))
         return y
@@ -215,6 +217,21 @@ class Space:
                                      _P(_stream(stream))))
         m = cnt.value
         return idx[:m], sc[:m], sched[:m]
+
+    def history_topk(self, cm: CostModel, k: int, stream=None):
+        """felix_history_topk over the last search(history=True) -> (idx int64 [m], step int32 [m],
+        score float64 [m], sched int32 [m, n_vars], n_unique) on the host."""
+        idx = np.zeros(k, dtype=np.int64)
+        step = np.zeros(k, dtype=np.int32)
+        sc = np.zeros(k, dtype=np.float64)
+        sched = np.zeros((k, self.n_vars), dtype=np.int32)
+        cnt = ctypes.c_int32(0)
+        nu = ctypes.c_int64(0)
+        _check(_lib.felix_history_topk(self._h, cm._h, int(k), idx.ctypes.data_as(_P), step.ctypes.data_as(_P),
+                                       sc.ctypes.data_as(_P), sched.ctypes.data_as(_P), ctypes.byref(cnt),
+                                       ctypes.byref(nu), _P(_stream(stream))))
+        m = cnt.value
+        return idx[:m], step[:m], sc[:m], sched[:m], int(nu.value)
 
     # ---------------------------------------------------------------- test hooks
     def eval(self, cm: CostModel, y, lam: float = 1.0, stream=None):

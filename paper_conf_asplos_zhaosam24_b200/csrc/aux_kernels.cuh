@@ -117,19 +117,24 @@ __global__ void __launch_bounds__(256) score_layer_kernel(const double* __restri
 }
 
 // ---------------------------------------------------------------------------- K7 dedup + top-k
-// Each block owns a chunk of entries; k rounds of block argmax by (score desc, candidate asc) over
+// Each block owns a chunk of entries; k rounds of block argmax by (score desc, order key asc) over
 // alive entries, then every alive entry whose schedule equals the winner's is killed (dedup keeps
-// the smallest candidate index, which wins ties).  Phase A: entries = candidates, many blocks;
-// phase B: entries = phase-A records, one block.  Warp shuffle + shared-memory block reduction.
-struct TopkKey { double s; int c; };
+// the smallest order key, which wins ties).  The order key is the candidate index (final-step
+// rounding) or the packed (step, seed) of a history record.  Phase A: entries = candidates, many
+// blocks; phase B: entries = phase-A records, one block.  Warp shuffle + shared-memory block reduction.
+struct TopkKey { double s; long long o; int c; };
 __device__ __forceinline__ bool topk_better(const TopkKey& a, const TopkKey& b) {
   if (a.c < 0) return false;
   if (b.c < 0) return true;
-  return a.s > b.s || (a.s == b.s && a.c < b.c);
+  return a.s > b.s || (a.s == b.s && a.o < b.o);
+}
+__device__ __forceinline__ TopkKey topk_shfl(const TopkKey& k, int off) {
+  return TopkKey{__shfl_xor_sync(0xffffffffu, k.s, off), __shfl_xor_sync(0xffffffffu, k.o, off),
+                 __shfl_xor_sync(0xffffffffu, k.c, off)};
 }
 
 __global__ void __launch_bounds__(1024) topk_select_kernel(
-    long long n_entries, long long chunk, const int* __restrict__ cand_of,
+    long long n_entries, long long chunk, const int* __restrict__ cand_of, const long long* __restrict__ okey,
     const double* __restrict__ score, const unsigned char* __restrict__ valid, const int* __restrict__ sched, int M,
     int k, unsigned char* __restrict__ alive, int* __restrict__ out_cand, int* __restrict__ out_cnt) {
   __shared__ TopkKey red[32];
@@ -143,25 +148,25 @@ __global__ void __launch_bounds__(1024) topk_select_kernel(
   __syncthreads();
   int r = 0;
   for (; r < k; ++r) {
-    TopkKey best{0.0, -1};
+    TopkKey best{0.0, 0, -1};
     for (long long e = c0 + threadIdx.x; e < c1; e += blockDim.x) {
       if (!alive[e]) continue;
       const int c = cand_of ? cand_of[e] : static_cast<int>(e);
-      const TopkKey t{score[c], c};
+      const TopkKey t{score[c], okey ? okey[c] : static_cast<long long>(c), c};
       if (topk_better(t, best)) best = t;
     }
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) {
-      TopkKey o{__shfl_xor_sync(0xffffffffu, best.s, off), __shfl_xor_sync(0xffffffffu, best.c, off)};
+      const TopkKey o = topk_shfl(best, off);
       if (topk_better(o, best)) best = o;
     }
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = best;
     __syncthreads();
     if (threadIdx.x < 32) {
-      TopkKey b = (threadIdx.x < (blockDim.x + 31) / 32) ? red[threadIdx.x] : TopkKey{0.0, -1};
+      TopkKey b = (threadIdx.x < (blockDim.x + 31) / 32) ? red[threadIdx.x] : TopkKey{0.0, 0, -1};
 #pragma unroll
       for (int off = 16; off > 0; off >>= 1) {
-        TopkKey o{__shfl_xor_sync(0xffffffffu, b.s, off), __shfl_xor_sync(0xffffffffu, b.c, off)};
+        const TopkKey o = topk_shfl(b, off);
         if (topk_better(o, b)) b = o;
       }
       if (threadIdx.x == 0) win = b;
@@ -185,6 +190,86 @@ __global__ void __launch_bounds__(1024) topk_select_kernel(
     out_cnt[blockIdx.x] = r;
     for (int q = r; q < k; ++q) out_cand[blockIdx.x * static_cast<long long>(k) + q] = -1;
   }
+}
+
+// ---------------------------------------------------------------------------- K8 history (Alg. 1 l.13/17/20)
+// One thread per seed, run on the rounded point sigma_x_i at which step i's objective is evaluated
+// (before the fwd kernel bumps step_ctr to i+1).  A seed whose rounded schedule equals its previous
+// step's is skipped; otherwise the schedule is inserted into an open-addressing hash set keyed by the
+// full tuple (64-bit hash for the probe, exact tuple compare on a hash match, so distinct schedules are
+// never merged).  A new schedule is appended to the pool with key (step << 32 | seed); a repeat lowers
+// the stored key with atomicMin, so each pool record ends up with its first (step, seed) occurrence.
+__device__ __forceinline__ unsigned long long hist_hash(const int* t, int M) {
+  unsigned long long h = 0x9E3779B97F4A7C15ull;
+  for (int j = 0; j < M; ++j) {
+    h ^= static_cast<unsigned int>(t[j]);
+    h *= 0xBF58476D1CE4E5B9ull;
+    h ^= h >> 31;
+  }
+  return h | 1ull;                        // 0 marks an empty slot
+}
+
+__global__ void hist_insert_kernel(const int* __restrict__ sched, int n, int M, const int* __restrict__ step_ctr,
+                                   int* __restrict__ last, unsigned long long* slot_h, int* slot_i,
+                                   unsigned long long slot_mask, int* pool_sched, long long* pool_key, int* pool_cnt,
+                                   int pool_cap, int* overflow) {
+  const int s = blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= n) return;
+  const int step = *step_ctr;
+  const int* cur = sched + static_cast<size_t>(s) * M;
+  int* lst = last + static_cast<size_t>(s) * M;
+  bool changed = (step == 0);
+  for (int j = 0; j < M; ++j) changed = changed || (cur[j] != lst[j]);
+  if (!changed) return;
+  for (int j = 0; j < M; ++j) lst[j] = cur[j];
+  const unsigned long long h = hist_hash(cur, M);
+  const long long key = (static_cast<long long>(step) << 32) | static_cast<long long>(s);
+  unsigned long long p = h & slot_mask;
+  for (;;) {
+    const unsigned long long prev = atomicCAS(&slot_h[p], 0ull, h);
+    if (prev == 0ull) {                                       // claimed: publish a new pool record
+      const int idx = atomicAdd(pool_cnt, 1);
+      if (idx >= pool_cap) {
+        atomicExch(overflow, 1);
+        atomicExch(&slot_i[p], -2);
+        return;
+      }
+      for (int j = 0; j < M; ++j) pool_sched[static_cast<size_t>(idx) * M + j] = cur[j];
+      pool_key[idx] = key;
+      __threadfence();
+      atomicExch(&slot_i[p], idx);
+      return;
+    }
+    if (prev == h) {                                          // same hash: wait for the record, compare
+      int idx;
+      while ((idx = atomicAdd(&slot_i[p], 0)) == -1) {}
+      if (idx == -2) return;
+      __threadfence();
+      const int* ps = pool_sched + static_cast<size_t>(idx) * M;
+      bool same = true;
+      for (int j = 0; j < M; ++j) same = same && (ps[j] == cur[j]);
+      if (same) {
+        atomicMin(&pool_key[idx], key);
+        return;
+      }
+    }
+    p = (p + 1) & slot_mask;
+  }
+}
+
+// history records -> host arrays: global index = index_base + seed, step
+__global__ void hist_gather_kernel(const int* __restrict__ cand, const int* __restrict__ cnt, int k,
+                                   const double* __restrict__ score, const int* __restrict__ sched,
+                                   const long long* __restrict__ key, int M, long long index_base,
+                                   long long* __restrict__ o_idx, int* __restrict__ o_step, double* __restrict__ o_score,
+                                   int* __restrict__ o_sched) {
+  const int r = threadIdx.x;
+  if (r >= k) return;
+  const int c = r < cnt[0] ? cand[r] : -1;
+  o_idx[r] = c >= 0 ? index_base + (key[c] & 0xffffffffll) : -1;
+  o_step[r] = c >= 0 ? static_cast<int>(key[c] >> 32) : -1;
+  o_score[r] = c >= 0 ? score[c] : 0.0;
+  for (int j = 0; j < M; ++j) o_sched[static_cast<size_t>(r) * M + j] = c >= 0 ? sched[static_cast<size_t>(c) * M + j] : 0;
 }
 
 // gather the final records into contiguous arrays for one D2H copy

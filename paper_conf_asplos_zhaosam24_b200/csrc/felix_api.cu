@@ -236,6 +236,12 @@ struct felix_space {
   // workspace caches (search: chunked; eval: one chunk) + scratch
   std::unique_ptr<felix::Chunks> search_chunks, eval_chunks;
   felix::DevBuf sched, valid, phi64, score, act64a, act64b, alive, rec_cand, rec_cnt, fin_cand, fin_cnt, o_idx, o_score, o_sched;
+  // varValuesHistory (Alg. 1 l.13/17) of the last search run with history != 0: per-step rounded points,
+  // each seed's previous schedule, the schedule hash set and the pool of distinct schedules
+  felix::DevBuf h_sched, h_last, h_slot_h, h_slot_i, h_pool_sched, h_pool_key, h_cnt, o_step;   // h_cnt: count, overflow
+  bool h_valid = false;
+  int64_t h_n = 0, h_cap = 0, h_index_base = 0;
+  uint64_t h_mask = 0;
   // profiling
   bool profiling = false;
   std::vector<felix::ProfEvent> prof;
@@ -938,6 +944,8 @@ static void check_pair(felix_space* s, felix_costmodel* m) {
   if (s->device != m->device) FELIX_THROW(FELIX_E_INVALID_ARG, "space and cost model on different devices");
 }
 
+static void do_round(felix_space* s, const float* y, int64_t n, int32_t* sched, cudaStream_t st);
+
 felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search_params* p, float* y,
                           float* final_loss, void* stream) {
   FELIX_API_BEGIN
@@ -969,6 +977,38 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     CUDA_OK(cudaMemsetAsync(pl->v.p, 0, pl->v.bytes, st));
     CUDA_OK(cudaMemsetAsync(pl->step_ctr.p, 0, 4, st));
   }
+  // varValuesHistory: a fresh pool for this search (worst case: every seed at every step is new)
+  const int M = s->desc.n_vars;
+  s->h_valid = p->history != 0;
+  if (s->h_valid) {
+    const int64_t cap = n * std::max(1, p->n_steps);
+    if (cap > INT32_MAX - 1) FELIX_THROW(FELIX_E_UNSUPPORTED, "history: n_seeds x n_steps exceeds 2^31 schedules");
+    uint64_t slots = 1024;
+    while (slots < static_cast<uint64_t>(cap) * 2) slots <<= 1;
+    ensure(s->h_sched, static_cast<size_t>(n) * M * 4);
+    ensure(s->h_last, static_cast<size_t>(n) * M * 4);
+    ensure(s->h_slot_h, slots * 8);
+    ensure(s->h_slot_i, slots * 4);
+    ensure(s->h_pool_sched, static_cast<size_t>(cap) * M * 4);
+    ensure(s->h_pool_key, static_cast<size_t>(cap) * 8);
+    ensure(s->h_cnt, 8);
+    CUDA_OK(cudaMemsetAsync(s->h_slot_h.p, 0, slots * 8, st));
+    CUDA_OK(cudaMemsetAsync(s->h_slot_i.p, 0xFF, slots * 4, st));
+    CUDA_OK(cudaMemsetAsync(s->h_cnt.p, 0, 8, st));
+    s->h_n = n;
+    s->h_cap = cap;
+    s->h_mask = slots - 1;
+    s->h_index_base = p->index_base;
+  }
+  // round sigma_x_i (before this step's fwd kernel bumps step_ctr) and insert new schedules
+  auto history_step = [&](cudaStream_t cs) {
+    do_round(s, y, n, s->h_sched.as<int32_t>(), cs);
+    hist_insert_kernel<<<static_cast<unsigned>((n + 255) / 256), 256, 0, cs>>>(
+        s->h_sched.as<int32_t>(), static_cast<int>(n), M, ch.plans[0]->step_ctr.as<int>(), s->h_last.as<int32_t>(),
+        s->h_slot_h.as<unsigned long long>(), s->h_slot_i.as<int>(), s->h_mask, s->h_pool_sched.as<int32_t>(),
+        s->h_pool_key.as<long long>(), s->h_cnt.as<int>(), static_cast<int>(s->h_cap), s->h_cnt.as<int>() + 1);
+    CUDA_OK(cudaGetLastError());
+  };
   const float hb = m->head_b, lam0 = p->lambda, lr0 = p->lr, b10 = p->beta1, b20 = p->beta2, eps0 = p->eps;
   // one Adam step of chunk k (fwd DAG -> GEMMs -> reverse DAG + Adam), PDL-chained on stream cs
   auto chunk_step = [&](int k, cudaStream_t cs) {
@@ -993,11 +1033,20 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     s->prof_launches[2] += 1;
   };
   if (s->profiling) {
-    for (int t = 1; t <= p->n_steps; ++t)            // direct launches with per-class events
+    for (int t = 1; t <= p->n_steps; ++t) {          // direct launches with per-class events
+      if (s->h_valid) {
+        prof_mark(s, 3, st, true);
+        history_step(st);
+        prof_mark(s, 3, st, false);
+      }
       for (int k = 0; k < nck; ++k) chunk_step(k, st);
+    }
   } else if (p->n_steps > 0) {
-    const std::vector<double> key = {static_cast<double>(mod.P), static_cast<double>(reinterpret_cast<uintptr_t>(y)),
-                                     static_cast<double>(reinterpret_cast<uintptr_t>(final_loss)), lam0, lr0, b10, b20, eps0};
+    auto ptr = [](const void* q) { return static_cast<double>(reinterpret_cast<uintptr_t>(q)); };
+    const std::vector<double> key = {static_cast<double>(mod.P), ptr(y), ptr(final_loss), lam0, lr0, b10, b20, eps0,
+                                     static_cast<double>(s->h_valid), ptr(s->h_sched.p), ptr(s->h_last.p),
+                                     ptr(s->h_slot_h.p), ptr(s->h_pool_sched.p), ptr(s->h_pool_key.p),
+                                     static_cast<double>(s->h_mask), static_cast<double>(s->h_cap)};
     if (!ch.graph || ch.graph_key != key) {
       if (ch.graph) { cudaGraphExecDestroy(ch.graph); ch.graph = nullptr; }
       while (static_cast<int>(ch.streams.size()) < nck) {
@@ -1014,6 +1063,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
       int64_t saved[4];
       std::copy(s->prof_launches, s->prof_launches + 4, saved);
       try {
+        if (s->h_valid) history_step(cap);
         CUDA_OK(cudaEventRecord(fork, cap));
         for (int k = 1; k < nck; ++k) CUDA_OK(cudaStreamWaitEvent(ch.streams[k], fork, 0));
         for (int k = 0; k < nck; ++k) chunk_step(k, ch.streams[k]);
@@ -1192,11 +1242,11 @@ felix_status felix_round_topk(felix_space* s, felix_costmodel* m, const float* y
   ensure(s->fin_cand, static_cast<size_t>(k) * 4);
   ensure(s->fin_cnt, 4);
   topk_select_kernel<<<static_cast<unsigned>(nblk), 1024, 0, st>>>(
-      n, chunk, nullptr, s->score.as<double>(), s->valid.as<uint8_t>(), s->sched.as<int32_t>(), M, k,
+      n, chunk, nullptr, nullptr, s->score.as<double>(), s->valid.as<uint8_t>(), s->sched.as<int32_t>(), M, k,
       s->alive.as<uint8_t>(), s->rec_cand.as<int>(), s->rec_cnt.as<int>());
   CUDA_OK(cudaGetLastError());
   topk_select_kernel<<<1, 1024, 0, st>>>(
-      nblk * k, nblk * k, s->rec_cand.as<int>(), s->score.as<double>(), s->valid.as<uint8_t>(), s->sched.as<int32_t>(),
+      nblk * k, nblk * k, s->rec_cand.as<int>(), nullptr, s->score.as<double>(), s->valid.as<uint8_t>(), s->sched.as<int32_t>(),
       M, k, s->alive.as<uint8_t>(), s->fin_cand.as<int>(), s->fin_cnt.as<int>());
   CUDA_OK(cudaGetLastError());
   ensure(s->o_idx, static_cast<size_t>(k) * 8);
@@ -1209,6 +1259,66 @@ felix_status felix_round_topk(felix_space* s, felix_costmodel* m, const float* y
   int cnt = 0;
   CUDA_OK(cudaMemcpyAsync(&cnt, s->fin_cnt.p, 4, cudaMemcpyDeviceToHost, st));
   CUDA_OK(cudaMemcpyAsync(idx_out, s->o_idx.p, static_cast<size_t>(k) * 8, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaMemcpyAsync(score_out, s->o_score.p, static_cast<size_t>(k) * 8, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaMemcpyAsync(sched_out, s->o_sched.p, static_cast<size_t>(k) * M * 4, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaStreamSynchronize(st));
+  *n_out = cnt;
+  FELIX_API_END
+}
+
+felix_status felix_history_topk(felix_space* s, felix_costmodel* m, int32_t k, int64_t* idx_out, int32_t* step_out,
+                                double* score_out, int32_t* sched_out, int32_t* n_out, int64_t* n_unique_out,
+                                void* stream) {
+  FELIX_API_BEGIN
+  check_pair(s, m);
+  if (!n_out || (k > 0 && (!idx_out || !step_out || !score_out || !sched_out))) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL output");
+  if (k < 0 || k > 1024) FELIX_THROW(FELIX_E_INVALID_ARG, "k must be in [0, 1024]");
+  if (!s->h_valid) FELIX_THROW(FELIX_E_INVALID_ARG, "the last felix_search did not record a history (history = 0)");
+  *n_out = 0;
+  DeviceGuard dg(s->device);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const int M = s->desc.n_vars;
+  int hc[2] = {0, 0};
+  CUDA_OK(cudaMemcpyAsync(hc, s->h_cnt.p, 8, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaStreamSynchronize(st));
+  if (hc[1]) FELIX_THROW(FELIX_E_UNSUPPORTED, "history pool overflow");
+  const int64_t n = std::min<int64_t>(hc[0], s->h_cap);
+  if (n_unique_out) *n_unique_out = n;
+  if (n == 0 || k == 0) return FELIX_OK;
+  const int32_t* sched = s->h_pool_sched.as<int32_t>();
+  ensure(s->valid, static_cast<size_t>(n));
+  ensure(s->phi64, static_cast<size_t>(n) * s->desc.froots.size() * 8);
+  ensure(s->score, static_cast<size_t>(n) * 8);
+  do_hard(s, sched, n, s->phi64.as<double>(), s->valid.as<uint8_t>(), st);
+  do_score(s, m, s->phi64.as<double>(), n, s->score.as<double>(), st);
+  const long long chunk = 4096;
+  const long long nblk = (n + chunk - 1) / chunk;
+  ensure(s->alive, static_cast<size_t>(std::max<long long>(n, nblk * k)));
+  ensure(s->rec_cand, static_cast<size_t>(nblk) * k * 4);
+  ensure(s->rec_cnt, static_cast<size_t>(nblk) * 4);
+  ensure(s->fin_cand, static_cast<size_t>(k) * 4);
+  ensure(s->fin_cnt, 4);
+  const long long* key = s->h_pool_key.as<long long>();
+  topk_select_kernel<<<static_cast<unsigned>(nblk), 1024, 0, st>>>(
+      n, chunk, nullptr, key, s->score.as<double>(), s->valid.as<uint8_t>(), sched, M, k,
+      s->alive.as<uint8_t>(), s->rec_cand.as<int>(), s->rec_cnt.as<int>());
+  CUDA_OK(cudaGetLastError());
+  topk_select_kernel<<<1, 1024, 0, st>>>(
+      nblk * k, nblk * k, s->rec_cand.as<int>(), key, s->score.as<double>(), s->valid.as<uint8_t>(), sched,
+      M, k, s->alive.as<uint8_t>(), s->fin_cand.as<int>(), s->fin_cnt.as<int>());
+  CUDA_OK(cudaGetLastError());
+  ensure(s->o_idx, static_cast<size_t>(k) * 8);
+  ensure(s->o_step, static_cast<size_t>(k) * 4);
+  ensure(s->o_score, static_cast<size_t>(k) * 8);
+  ensure(s->o_sched, static_cast<size_t>(k) * M * 4);
+  hist_gather_kernel<<<1, std::max(32, (k + 31) / 32 * 32), 0, st>>>(
+      s->fin_cand.as<int>(), s->fin_cnt.as<int>(), k, s->score.as<double>(), sched, key, M, s->h_index_base,
+      s->o_idx.as<long long>(), s->o_step.as<int>(), s->o_score.as<double>(), s->o_sched.as<int32_t>());
+  CUDA_OK(cudaGetLastError());
+  int cnt = 0;
+  CUDA_OK(cudaMemcpyAsync(&cnt, s->fin_cnt.p, 4, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaMemcpyAsync(idx_out, s->o_idx.p, static_cast<size_t>(k) * 8, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaMemcpyAsync(step_out, s->o_step.p, static_cast<size_t>(k) * 4, cudaMemcpyDeviceToHost, st));
   CUDA_OK(cudaMemcpyAsync(score_out, s->o_score.p, static_cast<size_t>(k) * 8, cudaMemcpyDeviceToHost, st));
   CUDA_OK(cudaMemcpyAsync(sched_out, s->o_sched.p, static_cast<size_t>(k) * M * 4, cudaMemcpyDeviceToHost, st));
   CUDA_OK(cudaStreamSynchronize(st));

@@ -350,3 +350,63 @@ def test_tile_mlp_eval_parity_vs_oracle(fx, cg, monkeypatch):
         err = np.linalg.norm(out["grad"] - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
         bad = (err > 1e-3) & ~(km < 1e-4)
         assert not np.any(bad), (name, np.nonzero(bad)[0][:10], err[bad][:10])
+
+
+def _gpu_trajectory(space, cm, y0, T, **kw):
+    """sigma_x_i, i = 0..T-1, as the GPU computes them: search(i steps) from y0 is deterministic and
+    identical to the first i steps of a longer search (Adam state starts fresh every call)."""
+    ys = [y0.copy()]
+    for i in range(1, T):
+        y = torch.from_numpy(y0).cuda()
+        space.search(cm, y, i, init_from_y=True, **kw)
+        ys.append(y.cpu().numpy())
+    return ys
+
+
+@pytest.mark.parametrize("name,T", [("C1", 5), ("C2", 4), ("bert_qkv", 4)])
+def test_history_topk_parity(fx, name, T):
+    """History rounding (Alg. 1 l.13/17/20-21): the device pool (per-step rounding, per-seed change
+    filter, hash-set dedup with first (step, seed), FP64 scoring, ordered top-k) against the oracle on
+    the GPU's own trajectory: idx / step / schedules bit-exact, scores rel <= 1e-12."""
+    sp, mlp, n, space, cm = _setup(fx, name)
+    y0 = fi.make_y0(sp, n, seed=31)
+    y = torch.from_numpy(y0).cuda()
+    space.search(cm, y, T, init_from_y=True, index_base=7000, history=True)
+    idx, step, sc, sched, n_unique = space.history_topk(cm, 64)
+    ys = _gpu_trajectory(space, cm, y0, T, index_base=7000)
+    ridx, rstep, rsc, rsched, rn = fo.round_topk_history(sp, mlp.W, mlp.b, ys, 64, index_base=7000)
+    assert n_unique == rn
+    assert np.array_equal(idx, ridx) and np.array_equal(step, rstep) and np.array_equal(sched, rsched)
+    assert np.max(np.abs(sc - rsc) / np.maximum(np.abs(rsc), 1e-300)) <= 1e-12
+
+
+def test_history_full_size_c2_properties(fx):
+    """Bench-size history (C2, 4096 seeds x 200 steps): records are valid, distinct, ordered, their
+    scores equal felix_score of their schedules, steps/indices are in range, and the history's best is
+    at least the best of the last evaluated point sigma_x_199 (which it contains)."""
+    cfg = fi.config("C2")
+    sp = cfg.spaces[0]
+    mlp = fi.make_mlp(cfg.mlp_dims)
+    space, cm = fx.Space(sp), fx.CostModel.from_weights(mlp)
+    n, T = cfg.n_seeds, 200
+    y = torch.empty((sp.n_vars, n), device="cuda")
+    space.search(cm, y, T, rng_seed=cfg.rng_seed, init_from_y=False, history=True)
+    idx, step, sc, sched, n_unique = space.history_topk(cm, 256)
+    assert len(idx) == 256 and n_unique >= 256
+    assert np.all((idx >= 0) & (idx < n)) and np.all((step >= 0) & (step < T))
+    assert len({s.tobytes() for s in sched}) == len(sched)
+    assert np.all(np.diff(sc) <= 0)
+    rescored = space.score(cm, torch.from_numpy(sched).cuda()).cpu().numpy()
+    assert np.array_equal(rescored, sc)
+    y199 = torch.empty_like(y)
+    space.search(cm, y199, T - 1, rng_seed=cfg.rng_seed, init_from_y=False)
+    _, lsc, _ = space.round_topk(cm, y199, 1)
+    assert sc[0] >= lsc[0]
+
+
+def test_history_requires_recording(fx):
+    sp, mlp, n, space, cm = _setup(fx, "C1")
+    y = torch.from_numpy(fi.make_y0(sp, n, seed=3)).cuda()
+    space.search(cm, y, 2, init_from_y=True)
+    with pytest.raises(fx.FelixError):
+        space.history_topk(cm, 8)

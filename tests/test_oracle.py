@@ -368,3 +368,45 @@ def test_search_decreases_loss_and_beats_random():
     yr = fo.init_sample(sp, 1600, 99)
     _, scr, _ = fo.round_topk(sp, mlp.W, mlp.b, yr, 1)
     assert sc[0] >= scr[0] - 1e-9
+
+
+def _history_setup(n=60, steps=6):
+    c = fi.config("C1")
+    sp = c.spaces[0]
+    mlp = fi.make_mlp(c.mlp_dims)
+    y0 = fo.init_sample(sp, n, c.rng_seed)
+    _, _, _, hist = fo.search(sp, mlp.W, mlp.b, y0, steps, c.lr, c.lam, history=True)
+    return sp, mlp, [h[0].astype(np.float32) for h in hist]
+
+
+def test_history_topk_single_step_is_round_topk():
+    """Alg. 1 l.20-21 over a one-entry history = final-point rounding of that entry (round_topk)."""
+    sp, mlp, ys = _history_setup()
+    idx, step, sc, sched, _ = fo.round_topk_history(sp, mlp.W, mlp.b, ys[:1], 16, index_base=500)
+    ridx, rsc, rsched = fo.round_topk(sp, mlp.W, mlp.b, ys[0], 16, index_base=500)
+    assert np.all(step == 0)
+    assert np.array_equal(idx, ridx) and np.array_equal(sc, rsc) and np.array_equal(sched, rsched)
+
+
+def test_history_topk_equals_round_topk_of_concatenated_points():
+    """The history as one population: point (step i, seed s) -> column i*n + s.  Ordering by
+    (step, seed) is ordering by that column index, so dedup (first visit) and the (score, index)
+    order coincide with round_topk on the concatenation."""
+    sp, mlp, ys = _history_setup()
+    n = ys[0].shape[1]
+    idx, step, sc, sched, n_unique = fo.round_topk_history(sp, mlp.W, mlp.b, ys, 32)
+    cat = np.concatenate(ys, axis=1)
+    cidx, csc, csched = fo.round_topk(sp, mlp.W, mlp.b, cat, 32)
+    assert np.array_equal(idx, cidx % n) and np.array_equal(step, cidx // n)
+    assert np.array_equal(sc, csc) and np.array_equal(sched, csched)
+    assert n_unique == len({r.tobytes() for r in fo.round_schedules(sp, cat)})
+
+
+def test_history_topk_monotone_and_revisits_add_nothing():
+    sp, mlp, ys = _history_setup()
+    best = [fo.round_topk_history(sp, mlp.W, mlp.b, ys[:t], 1)[2][0] for t in range(1, len(ys) + 1)]
+    assert all(b1 >= b0 for b0, b1 in zip(best, best[1:]))              # more history never hurts
+    perm = ys[0][:, ::-1].copy()                                        # same points, other seeds, later step
+    a = fo.round_topk_history(sp, mlp.W, mlp.b, ys[:1], 16)
+    b = fo.round_topk_history(sp, mlp.W, mlp.b, ys[:1] + [perm], 16)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1]) and a[4] == b[4]
