@@ -47,6 +47,9 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
     ap.add_argument("--seeds", type=int, default=0, help="override seeds per GPU (experiments; not the headline)")
     ap.add_argument("--search-steps", type=int, default=0, help="override Adam steps per search (experiments)")
+    ap.add_argument("--history", action="store_true",
+                    help="paper-faithful Alg. 1: round every visited point (varValuesHistory, l.13/17/20) "
+                         "instead of the final point only (SURVEY 8(f) row 1; not the headline)")
     return ap.parse_args()
 
 
@@ -114,7 +117,7 @@ def dist_env():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
 
 
-def oracle_baseline(cfg, seconds: float):
+def oracle_baseline(cfg, seconds: float, history: bool = False):
     """The float64 oracle as it stands, timed on this host's cores on a bounded sample of the same
     workload: the first min(n_seeds, 4096) seeds of the same space/model/starting points, as many Adam
     steps as fit in ~`seconds`, then its rounding + top-k.  Returns (cand-steps/s, threads, sample)."""
@@ -134,17 +137,24 @@ def oracle_baseline(cfg, seconds: float):
     fo.search(sp, mlp.W, mlp.b, y0, 1, cfg.lr, cfg.lam)
     one = time.perf_counter() - t0
     steps = int(max(2, min(cfg.n_steps, seconds / max(one, 1e-6))))
+    if history:
+        steps = max(2, steps // 3)
     t0 = time.perf_counter()
-    y, _, _, _ = fo.search(sp, mlp.W, mlp.b, y0, steps, cfg.lr, cfg.lam)
+    y, _, _, hist = fo.search(sp, mlp.W, mlp.b, y0, steps, cfg.lr, cfg.lam, history=history)
     t_search = time.perf_counter() - t0
     t0 = time.perf_counter()
-    fo.round_topk(sp, mlp.W, mlp.b, y.astype(np.float32), cfg.topk)
+    if history:
+        fo.round_topk_history(sp, mlp.W, mlp.b, [h[0].astype(np.float32) for h in hist], cfg.topk)
+    else:
+        fo.round_topk(sp, mlp.W, mlp.b, y.astype(np.float32), cfg.topk)
     t_fin = time.perf_counter() - t0
-    # whole-job rate: the full search is n_steps steps + one finish; scale the measured parts
+    # whole-job rate: the full search is n_steps steps + one finish; scale the measured parts (the history
+    # finish grows with the steps recorded, so it is scaled with them)
     per_step = t_search / steps
-    t_job = per_step * cfg.n_steps + t_fin
+    t_job = per_step * cfg.n_steps + (t_fin * cfg.n_steps / steps if history else t_fin)
     rate = n * cfg.n_steps / t_job
-    sample = (f"{n} seeds x {steps} Adam steps of {sp.name} (of {cfg.n_steps}) + round/top-k, "
+    what = "history round/validate/score/top-k of every visited point" if history else "round/top-k"
+    sample = (f"{n} seeds x {steps} Adam steps of {sp.name} (of {cfg.n_steps}) + {what}, "
               f"extrapolated linearly to {cfg.n_steps} steps; numpy float64")
     return rate, threads, sample, t_search + t_fin
 
@@ -162,7 +172,7 @@ def run_reference(args):
     tot = 0.0
     for it in range(W + K):
         secs = max(2.0, args.cpu_seconds / max(1, (W + K)))
-        rate, threads, sample, t = oracle_baseline(cfg, secs)
+        rate, threads, sample, t = oracle_baseline(cfg, secs, args.history)
         if it >= W:
             rates.append(rate)
             tot += t
@@ -212,11 +222,21 @@ def run_felix(args):
     loss = torch.empty(n, dtype=torch.float32, device=dev)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # > 126 MB L2
 
+    hist = args.history
+
+    def finish(yv):
+        if not hist:
+            return space.round_topk(cm, yv, k, index_base=base, stream=stream)
+        idx, step, sc, sched, _ = space.history_topk(cm, k, stream=stream)
+        # merge key for the multi-GPU top-k: (step, global index) packed so that its order is the
+        # history order (score desc, step asc, global index asc)
+        return (step.astype(np.int64) << 40) | idx, sc, sched
+
     def bench_step():
         # Algorithm 1: init (device sampler) -> T Adam steps -> round / validate / score / top-k
         space.search(cm, y, T, lr=cfg.lr, lam=cfg.lam, rng_seed=cfg.rng_seed, init_from_y=False,
-                     index_base=base, final_loss=loss, stream=stream)
-        return space.round_topk(cm, y, k, index_base=base, stream=stream)
+                     index_base=base, final_loss=loss, history=hist, stream=stream)
+        return finish(y)
 
     def barrier():
         if world > 1:
@@ -264,7 +284,7 @@ def run_felix(args):
     e0.record(stream)
     for i in range(K):
         space.search(cm, y, T, lr=cfg.lr, lam=cfg.lam, rng_seed=cfg.rng_seed, init_from_y=False, index_base=base,
-                     final_loss=loss, stream=stream)
+                     final_loss=loss, history=hist, stream=stream)
     e1.record(stream)
     barrier()
     space.profile(False)
@@ -273,7 +293,7 @@ def run_felix(args):
     # finish (round/top-k) alone
     f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     f0.record(stream)
-    space.round_topk(cm, y, k, index_base=base, stream=stream)
+    finish(y)
     f1.record(stream)
     barrier()
     finish_ms = f0.elapsed_time(f1)
@@ -315,9 +335,9 @@ def run_felix(args):
         def e2e_step():
             y_dev.copy_(y0_host, non_blocking=True)                          # H2D: starting points
             space.search(cm, y_dev, T, lr=cfg.lr, lam=cfg.lam, init_from_y=True, index_base=base,
-                         final_loss=loss, stream=stream)
+                         final_loss=loss, history=hist, stream=stream)
             loss_host.copy_(loss, non_blocking=True)                         # D2H: final losses
-            return space.round_topk(cm, y_dev, k, index_base=base, stream=stream)   # D2H: top-k records
+            return finish(y_dev)                                             # D2H: top-k records
         for _ in range(2):
             e2e_step()
         barrier()
@@ -342,7 +362,7 @@ def run_felix(args):
 
     cpu = None
     if not args.no_cpu_baseline and world == 1:
-        rate, threads, sample, _ = oracle_baseline(cfg, args.cpu_seconds)
+        rate, threads, sample, _ = oracle_baseline(cfg, args.cpu_seconds, hist)
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample}
 
     n_gemm = len(cfg.mlp_dims) * 2 - 4          # (L-1) forward + (L-1) backward GEMM layers
@@ -354,7 +374,8 @@ def run_felix(args):
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "fp16x3 split (fp32-accurate) MLP, f64 DAG, f32 Adam", "data": "synthetic",
         "config": {"workload": f"{cfg.name}: {sp.name}, {sp.n_vars} vars, {n} seeds x {T} steps per GPU, "
-                               f"MLP {list(cfg.mlp_dims)}, top-{k}",
+                               f"MLP {list(cfg.mlp_dims)}, top-{k}" + (", history rounding (Alg. 1 l.20 over all "
+                                                                       "visited points)" if hist else ""),
                    "n_seeds_per_gpu": n, "n_steps": T, "topk": k, "parallelism": f"dp{world} (seed shards)",
                    "l2": "flushed (256 MB write) between timed iterations"},
         "roofline": {"bound": "tensor", "achieved": achieved_tflops, "peak": peak, "unit": "TFLOP/s",
@@ -371,7 +392,9 @@ def run_felix(args):
         "finish_ms": finish_ms,
         "gpu_launches": launches_per_step * K,
         "clocks": clocks.summary(),
-        "top1": {"global_idx": int(gidx[0]) if len(gidx) else None, "score": float(gsc[0]) if len(gsc) else None},
+        "top1": ({"global_idx": int(gidx[0]) & ((1 << 40) - 1), "step": int(gidx[0]) >> 40, "score": float(gsc[0])}
+                 if hist and len(gidx) else
+                 {"global_idx": int(gidx[0]) if len(gidx) else None, "score": float(gsc[0]) if len(gsc) else None}),
     }
     if e2e is not None:
         line["e2e"] = e2e
