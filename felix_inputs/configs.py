@@ -111,6 +111,19 @@ def c2_space() -> Space:
     return build_space(conv2d_spec("resnet50_conv3x3_56x56x64", 64, 56, 56, 64, 3, 3, 1))
 
 
+def c2_sketches() -> List[Space]:
+    """Several symbolic programs p*_i of the C2 subgraph (Eq. 3): the multi-level-tiling
+    sketch with 3-level spatial tiling and a 2-way reduction split (= c2_space), with a 1-way
+    reduction split, and with 2-level spatial tiling (no virtual threads)."""
+    C, H, W, K, R, S = 64, 56, 56, 64, 3, 3
+    return [
+        build_space(conv2d_spec("resnet50_conv3x3_56x56x64", C, H, W, K, R, S, 1)),
+        build_space(conv2d_spec("resnet50_conv3x3_56x56x64_rc1", C, H, W, K, R, S, 1, rc_vars=1)),
+        build_space(conv2d_spec("resnet50_conv3x3_56x56x64_ti", C, H, W, K, R, S, 1,
+                                co_levels="ti", h_levels="ti", w_levels="ti", rc_vars=2)),
+    ]
+
+
 def c5_space() -> Space:
     return build_space(dense_spec("vitl16_fc1_197x4096x1024", 197, 4096, 1024, i_levels="vti", j_levels="vti",
                                   k_vars=2, bias=True, gelu=True))

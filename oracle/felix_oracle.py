@@ -628,6 +628,19 @@ def round_topk(space, W, b, y: np.ndarray, k: int, index_base: int = 0):
     return gidx[sel], sc[sel], sched[sel]
 
 
+def subgraph_topk(per_sketch, k: int):
+    """Eq. 3: the best schedules of a subgraph are the best over all its symbolic programs
+    p*_i.  per_sketch[i] = (idx, score, sched) = round_topk of sketch i (distinct schedules of one
+    program).  Schedules of different programs are different programs, so there is no cross-sketch
+    dedup, and the global top-k lies in the union of the per-sketch top-k lists.  Order: (score desc,
+    sketch asc, global index asc).  Returns a list of (sketch, idx, score, sched)."""
+    recs = []
+    for i, (idx, sc, sched) in enumerate(per_sketch):
+        recs += [(i, int(idx[r]), float(sc[r]), np.asarray(sched[r])) for r in range(len(idx))]
+    recs.sort(key=lambda r: (-r[2], r[0], r[1]))
+    return recs[:k]
+
+
 def round_topk_history(space, W, b, ys: Sequence[np.ndarray], k: int, index_base: int = 0):
     """Algorithm 1 lines 20-21 over varValuesHistory (lines 13, 17; "takes all
     the variable values traversed in the optimization process, rounds them to integers ... removes

@@ -123,6 +123,7 @@ struct Plan {
   std::vector<GemmLaunch> gemms;           // per-layer kernels (FELIX_MLP=layers)
   ChainParams chain{};                     // persistent all-layer kernel
   int chain_grid = 0;
+  int chain_cs = 1;                        // 4: cluster chain (one 4-CTA cluster per row block, cluster barriers)
   DevBuf grid_bar;
   bool tile_ok = false;                    // model has the shape mlp_tile_kernel is specialised for
   TileParams tile{};                       // tile-local fused MLP (default when tile_ok)
@@ -177,19 +178,33 @@ static void launch_tile(const Plan& p, cudaStream_t st) {
 }
 
 static void launch_chain(const Plan& p, cudaStream_t st) {
-  static bool attr_set = false;
-  if (!attr_set) {
-    CUDA_OK(cudaFuncSetAttribute(mlp_chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES));
-    attr_set = true;
+  static bool attr_set[2] = {false, false};
+  const int ci = p.chain_cs == 4 ? 1 : 0;
+  if (!attr_set[ci]) {
+    if (ci) CUDA_OK(cudaFuncSetAttribute(mlp_chain_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES));
+    else CUDA_OK(cudaFuncSetAttribute(mlp_chain_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES));
+    attr_set[ci] = true;
+  }
+  cudaLaunchAttribute attrs[2];
+  attrs[0] = g_pdl_attr;
+  if (ci) {
+    attrs[1].id = cudaLaunchAttributeClusterDimension;
+    attrs[1].val.clusterDim.x = static_cast<unsigned>(p.chain_cs);
+    attrs[1].val.clusterDim.y = 1;
+    attrs[1].val.clusterDim.z = 1;
+  } else {
+    attrs[1].id = cudaLaunchAttributeCooperative;   // the grid barrier needs every CTA resident
+    attrs[1].val.cooperative = 1;
   }
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(static_cast<unsigned>(p.chain_grid));
   cfg.blockDim = dim3(CHAIN_THREADS);
   cfg.dynamicSmemBytes = CHAIN_SMEM_BYTES;
   cfg.stream = st;
-  cfg.attrs = &g_pdl_attr;
-  cfg.numAttrs = 1;
-  CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_chain_kernel, p.chain));
+  cfg.attrs = attrs;
+  cfg.numAttrs = 2;
+  if (ci) CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_chain_kernel<4>, p.chain));
+  else CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_chain_kernel<1>, p.chain));
 }
 
 // The population split into K independent chunks, each with its own workspace (Plan).  One Adam
@@ -201,11 +216,18 @@ struct Chunks {
   int K = 0;
   std::vector<int64_t> off, cnt;
   std::vector<std::unique_ptr<Plan>> plans;
-  std::vector<cudaStream_t> streams;       // capture-time branch streams
+  std::vector<cudaStream_t> streams;       // capture-time branch streams / per-chunk launch streams
   cudaGraphExec_t graph = nullptr;
   std::vector<double> graph_key;
+  std::vector<cudaGraphExec_t> chunk_graphs;   // independent per-chunk step graphs (no per-step join)
+  std::vector<double> chunk_key;
+  cudaEvent_t ev_fork = nullptr;
+  std::vector<cudaEvent_t> ev_join;
   ~Chunks() {
     if (graph) cudaGraphExecDestroy(graph);
+    for (auto g : chunk_graphs) if (g) cudaGraphExecDestroy(g);
+    if (ev_fork) cudaEventDestroy(ev_fork);
+    for (auto e : ev_join) cudaEventDestroy(e);
     for (auto st : streams) cudaStreamDestroy(st);
   }
 };
@@ -597,6 +619,14 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
     max_tiles = std::max(max_tiles, L.n_tiles);
   }
   p->chain_grid = std::min(sms, max_tiles);
+  // Cluster chain (one 4-CTA cluster per row block, cluster barriers) when every row block gets its own
+  // cluster: same speed as the grid chain at C2 (47.3 vs 47.1 us; the per-layer cost is the L2 round trip
+  // of the activations, not the barrier) but it only needs each cluster co-scheduled, so concurrent
+  // searches on different streams cannot deadlock.  Above 37 row blocks the grid chain is faster
+  // (n=8192: 64 vs 90 us) and is launched cooperatively (all CTAs gang-scheduled).  FELIX_CHAIN_CS=1|4.
+  p->chain_cs = mt <= sms / 4 ? 4 : 1;
+  if (const char* e = std::getenv("FELIX_CHAIN_CS")) p->chain_cs = std::atoi(e) == 4 ? 4 : 1;
+  if (p->chain_cs == 4) p->chain_grid = static_cast<int>(std::min<int64_t>(sms / 4, mt)) * 4;
   // tile-local fused MLP: TenSet widths [K0p, 512, 256, 256, 1] only
   p->tile_ok = L == 4 && d[1] == tile::D1 && d[2] == tile::D2 && d[3] == tile::D3 && K0p <= 128 && K0p % 32 == 0;   // K0p/2 rows: multiple of 16
   if (p->tile_ok) {
@@ -1041,6 +1071,59 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
       }
       for (int k = 0; k < nck; ++k) chunk_step(k, st);
     }
+  } else if (p->n_steps > 0 && nck > 1 && !s->h_valid) {
+    // The chunks are independent candidates: each gets its own one-step graph on its own stream,
+    // launched n_steps times with no per-step join, so one chunk's MLP overlaps another's DAG kernels
+    // (a per-step fork/join would re-synchronise them every step).  Joined once at the end.
+    auto ptr = [](const void* q) { return static_cast<double>(reinterpret_cast<uintptr_t>(q)); };
+    const std::vector<double> key = {static_cast<double>(mod.P), ptr(y), ptr(final_loss), lam0, lr0, b10, b20, eps0};
+    while (static_cast<int>(ch.streams.size()) < nck) {
+      cudaStream_t b;
+      CUDA_OK(cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking));
+      ch.streams.push_back(b);
+    }
+    if (!ch.ev_fork) CUDA_OK(cudaEventCreateWithFlags(&ch.ev_fork, cudaEventDisableTiming));
+    while (static_cast<int>(ch.ev_join.size()) < nck) {
+      cudaEvent_t e;
+      CUDA_OK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+      ch.ev_join.push_back(e);
+    }
+    if (static_cast<int>(ch.chunk_graphs.size()) != nck || ch.chunk_key != key) {
+      for (auto g : ch.chunk_graphs) if (g) cudaGraphExecDestroy(g);
+      ch.chunk_graphs.assign(nck, nullptr);
+      int64_t saved[4];
+      std::copy(s->prof_launches, s->prof_launches + 4, saved);
+      for (int k = 0; k < nck; ++k) {
+        cudaGraph_t graph = nullptr;
+        cudaStream_t cs = ch.streams[k];
+        CUDA_OK(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
+        try {
+          chunk_step(k, cs);
+        } catch (...) {
+          cudaStreamEndCapture(cs, &graph);
+          if (graph) cudaGraphDestroy(graph);
+          throw;
+        }
+        CUDA_OK(cudaStreamEndCapture(cs, &graph));
+        cudaError_t ie = cudaGraphInstantiate(&ch.chunk_graphs[k], graph, 0);
+        cudaGraphDestroy(graph);
+        CUDA_OK(ie);
+      }
+      std::copy(saved, saved + 4, s->prof_launches);
+      ch.chunk_key = key;
+    }
+    CUDA_OK(cudaEventRecord(ch.ev_fork, st));
+    for (int k = 0; k < nck; ++k) CUDA_OK(cudaStreamWaitEvent(ch.streams[k], ch.ev_fork, 0));
+    for (int t = 1; t <= p->n_steps; ++t)
+      for (int k = 0; k < nck; ++k) CUDA_OK(cudaGraphLaunch(ch.chunk_graphs[k], ch.streams[k]));
+    for (int k = 0; k < nck; ++k) {
+      CUDA_OK(cudaEventRecord(ch.ev_join[k], ch.streams[k]));
+      CUDA_OK(cudaStreamWaitEvent(st, ch.ev_join[k], 0));
+    }
+    s->prof_launches[0] += static_cast<int64_t>(p->n_steps) * nck;
+    s->prof_launches[1] += static_cast<int64_t>(p->n_steps) * nck *
+                           (ch.plans[0]->mode == MLP_LAYERS ? static_cast<int64_t>(ch.plans[0]->gemms.size()) : 1);
+    s->prof_launches[2] += static_cast<int64_t>(p->n_steps) * nck;
   } else if (p->n_steps > 0) {
     auto ptr = [](const void* q) { return static_cast<double>(reinterpret_cast<uintptr_t>(q)); };
     const std::vector<double> key = {static_cast<double>(mod.P), ptr(y), ptr(final_loss), lam0, lr0, b10, b20, eps0,

@@ -79,6 +79,46 @@ __device__ __forceinline__ void grid_barrier(unsigned int* ctr, unsigned int nbl
   asm volatile("fence.proxy.async.global;" ::: "memory");
 }
 
+// Tiles of one layer owned by this CTA.  CS == 1: tile = blockIdx.x, +gridDim.x, ... over all
+// (row block, N tile) pairs, layers separated by a grid-wide barrier.  CS > 1 (cluster chain): CTA rank
+// r of cluster c computes N tiles r, r+CS, ... of row blocks c, c+#clusters, ..., so every dependency
+// between consecutive layers stays inside the cluster and the layer barrier is a cluster barrier.
+template <int CS>
+struct ChainTiles {
+  int t0, tstep, m, mstep, nt0, nt, ntn, mt;
+  __device__ ChainTiles(int n_tiles_n, int m_tiles) : ntn(n_tiles_n), mt(m_tiles) {
+    if (CS == 1) { t0 = blockIdx.x; tstep = gridDim.x; }
+    else { m = blockIdx.x / CS; mstep = gridDim.x / CS; nt0 = blockIdx.x % CS; nt = nt0; }
+  }
+  // first tile (or -1), then next(tile)
+  __device__ int first() {
+    if (CS == 1) return t0 < ntn * mt ? t0 : -1;
+    nt = nt0;
+    return (m < mt && nt < ntn) ? m * ntn + nt : -1;
+  }
+  __device__ int next(int tile) {
+    if (CS == 1) { tile += tstep; return tile < ntn * mt ? tile : -1; }
+    int mm = tile / ntn;
+    nt += CS;
+    if (nt >= ntn) { nt = nt0; mm += mstep; }
+    return (mm < mt && nt < ntn) ? mm * ntn + nt : -1;
+  }
+};
+
+// cluster barrier for one thread per CTA: arrive (release, cluster scope) on every CTA's layer
+// barrier, then wait on this CTA's (acquire, cluster scope); global writes of the async proxy
+// (TMA stores, completed by bulk_wait) are ordered around it with fence.proxy.async.global
+template <int CS>
+__device__ __forceinline__ void cluster_layer_barrier(uint64_t* bar, uint32_t phase) {
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+  const uint32_t a = ptx::smem_u32(bar);
+#pragma unroll
+  for (int r = 0; r < CS; ++r) ptx::mbar_arrive_cluster(ptx::mapa_shared(a, r));
+  ptx::mbar_wait_cluster(bar, phase & 1u);
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+
+template <int CS>
 __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __grid_constant__ ChainParams P) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -91,6 +131,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
   uint64_t* tempty = tfull + 2;                    // [2] accumulator drained
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
   uint32_t* gen_slot = tmem_slot + 1;              // layers completed grid-wide (producer handshake)
+  uint64_t* cl_bar = tempty + 3;                   // cluster layer barrier (CS > 1), 8-byte aligned
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned int G = gridDim.x;
@@ -103,12 +144,14 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < CHAIN_STAGES; ++s) { ptx::mbar_init(&full_bar[s], 1); ptx::mbar_init(&empty_bar[s], 1); }
     for (int a = 0; a < 2; ++a) { ptx::mbar_init(&tfull[a], 1); ptx::mbar_init(&tempty[a], CHAIN_EPI_WARPS); }
+    if (CS > 1) ptx::mbar_init(cl_bar, CS);
     *gen_slot = 0;
     ptx::fence_barrier_init();
   }
   if (warp == 1) ptx::tmem_alloc(tmem_slot, 2 * CHAIN_BN_MAX);
   ptx::tc_fence_before();
-  __syncthreads();
+  if constexpr (CS > 1) ptx::cluster_sync();
+  else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
   ptx::pdl_launch_dependents();
@@ -132,7 +175,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         CHAIN_STAMP(l, 0);
         const int nkb = (L.args.K + GEMM_BK - 1) / GEMM_BK;
         const uint32_t tx = 2 * CHAIN_A_BYTES + 2 * (L.bn * GEMM_BK * 2);
-        for (int tile = blockIdx.x; tile < L.n_tiles; tile += G) {
+        ChainTiles<CS> tiles(L.n_tiles_n, P.m_tiles);
+        for (int tile = tiles.first(); tile >= 0; tile = tiles.next(tile)) {
           const int m0 = (tile / L.n_tiles_n) * GEMM_BM, n0 = (tile % L.n_tiles_n) * L.bn;
           for (int kb = 0; kb < nkb; ++kb, ++it) {
             const int s = it % CHAIN_STAGES;
@@ -154,7 +198,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       for (int l = 0; l < P.n_layers; ++l) {
         const ChainLayer& L = P.layer[l];
         const int nkb = (L.args.K + GEMM_BK - 1) / GEMM_BK;
-        for (int tile = blockIdx.x; tile < L.n_tiles; tile += G, ++tcount) {
+        ChainTiles<CS> tiles(L.n_tiles_n, P.m_tiles);
+        for (int tile = tiles.first(); tile >= 0; tile = tiles.next(tile), ++tcount) {
           const int acc = tcount & 1;
           if (tcount >= 2) ptx::mbar_wait(&tempty[acc], ((tcount >> 1) - 1) & 1);
           ptx::tc_fence_after();
@@ -162,7 +207,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
           for (int kb = 0; kb < nkb; ++kb, ++it) {
             const int s = it % CHAIN_STAGES;
             ptx::mbar_wait(&full_bar[s], (it / CHAIN_STAGES) & 1);
-            if (kb == 0 && tile == static_cast<int>(blockIdx.x)) CHAIN_STAMP(l, 1);
+            if (kb == 0 && tcount == 0) CHAIN_STAMP(l, 1);
             ptx::tc_fence_after();
             const uint32_t ah = ptx::smem_u32(a_hi(s)), al = ptx::smem_u32(a_lo(s));
             const uint32_t bh = ptx::smem_u32(b_hi(s)), bl = ptx::smem_u32(b_lo(s));
@@ -213,7 +258,9 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         }
       }
       ptx::named_bar_sync(1, NEPI);
-      for (int tile = blockIdx.x; tile < ntiles; tile += G, ++tcount) {
+      ChainTiles<CS> tiles(ntn, P.m_tiles);
+      int first_tile = tiles.first();
+      for (int tile = first_tile; tile >= 0; tile = tiles.next(tile), ++tcount) {
         const int acc = tcount & 1;
         const int m0 = (tile / ntn) * GEMM_BM, n0 = (tile % ntn) * bn;
         const int row = m0 + r_tile;
@@ -226,7 +273,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             if (q64 * 64 < bn) mwords[q64] = __ldcg(&mask_in[static_cast<size_t>(row) * (aN / 32) + (n0 + q64 * 64 + half * 32) / 32]);
         }
         ptx::mbar_wait(&tfull[acc], (tcount >> 1) & 1);
-        if (etid == 0 && tile == static_cast<int>(blockIdx.x)) CHAIN_STAMP(l, 3);
+        if (etid == 0 && tile == first_tile) CHAIN_STAMP(l, 3);
         ptx::tc_fence_after();
         const uint32_t t_row = tmem_base + acc * CHAIN_BN_MAX + (static_cast<uint32_t>(q * 32) << 16);
         float head_acc = 0.f;
@@ -257,7 +304,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
               if (CHAIN_EPI_BUFS == 2) ptx::bulk_wait_read<1>(); else ptx::bulk_wait_read<0>();
             }
             ptx::named_bar_sync(1, NEPI);
-            const bool st0 = etid == 0 && c64 == 0 && tile == static_cast<int>(blockIdx.x);
+            const bool st0 = etid == 0 && c64 == 0 && tile == first_tile;
             if (st0) CHAIN_STAMP2(l, 0);
             {
               const int c32 = half * 32;
@@ -340,7 +387,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         ptx::named_bar_sync(1, NEPI);
         if (etid == 0) {
           CHAIN_STAMP(l, 5);
-          grid_barrier(P.grid_bar, G);
+          if constexpr (CS > 1) cluster_layer_barrier<CS>(cl_bar, static_cast<uint32_t>(l));
+          else grid_barrier(P.grid_bar, G);
           CHAIN_STAMP(l, 6);
           // publish "layer l done everywhere" to the producer warp of this CTA
           asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" :: "r"(ptx::smem_u32(gen_slot)), "r"(static_cast<unsigned int>(l + 1)) : "memory");
@@ -350,7 +398,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
     if (etid == 0) ptx::bulk_wait<0>();
   }
   ptx::tc_fence_before();
-  __syncthreads();
+  if constexpr (CS > 1) ptx::cluster_sync();
+  else __syncthreads();
   if (warp == 1) ptx::tmem_dealloc(tmem_base, 2 * CHAIN_BN_MAX);
 }
 

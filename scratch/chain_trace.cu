@@ -43,14 +43,24 @@ int main(int argc, char** argv) {
   P.grid_bar = (unsigned int*)dz(64);
   int grid = std::min(148, mt * 512 / bnA);
   P.trace = (unsigned long long*)dz((size_t)grid * CHAIN_MAX_LAYERS * 8 * 8 * 2);
-  cudaFuncSetAttribute(mlp_chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES);
-  for (int it = 0; it < 3; ++it) mlp_chain_kernel<<<grid, CHAIN_THREADS, CHAIN_SMEM_BYTES>>>(P);
+  const int CS = argc > 4 ? atoi(argv[4]) : 1;
+  if (CS == 4) grid = std::min(148 / 4, mt) * 4;
+  cudaFuncSetAttribute(mlp_chain_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES);
+  cudaFuncSetAttribute(mlp_chain_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES);
+  auto launch = [&]() {
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension; at[0].val.clusterDim.x = CS; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+    cudaLaunchConfig_t cfg{}; cfg.gridDim = dim3(grid); cfg.blockDim = dim3(CHAIN_THREADS); cfg.dynamicSmemBytes = CHAIN_SMEM_BYTES;
+    cfg.attrs = at; cfg.numAttrs = 1;
+    if (CS == 4) cudaLaunchKernelEx(&cfg, mlp_chain_kernel<4>, P); else cudaLaunchKernelEx(&cfg, mlp_chain_kernel<1>, P);
+  };
+  for (int it = 0; it < 3; ++it) launch();
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
   cudaEventRecord(e0);
-  for (int it = 0; it < 10; ++it) mlp_chain_kernel<<<grid, CHAIN_THREADS, CHAIN_SMEM_BYTES>>>(P);
+  for (int it = 0; it < 10; ++it) launch();
   cudaEventRecord(e1); cudaEventSynchronize(e1);
   float ms; cudaEventElapsedTime(&ms, e0, e1);
-  printf("M=%d grid=%d bnA=%d bnB=%d: %.2f us per chain launch (err=%s)\n", M, grid, bnA, bnB, ms * 100, cudaGetErrorString(cudaGetLastError()));
+  printf("CS=%d M=%d grid=%d bnA=%d bnB=%d: %.2f us per chain launch (err=%s)\n", CS, M, grid, bnA, bnB, ms * 100, cudaGetErrorString(cudaGetLastError()));
   std::vector<unsigned long long> h((size_t)grid * CHAIN_MAX_LAYERS * 8), h2((size_t)grid * CHAIN_MAX_LAYERS * 8);
   cudaMemcpy(h.data(), P.trace, h.size() * 8, cudaMemcpyDeviceToHost);
   cudaMemcpy(h2.data(), P.trace + h.size(), h2.size() * 8, cudaMemcpyDeviceToHost);

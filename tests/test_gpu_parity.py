@@ -308,7 +308,7 @@ def test_shape_errors(fx):
     del bad
 
 
-@pytest.mark.parametrize("mode,cg", [("chain", "1"), ("layers", "1"), ("tile", "2")])
+@pytest.mark.parametrize("mode,cg", [("chain", "1"), ("chain-cluster", "1"), ("layers", "1"), ("tile", "2")])
 def test_mlp_execution_modes_agree(fx, mode, cg, monkeypatch):
     """The tile-local fused MLP (1-SM and 2-SM cta_group::2 variants), the persistent chain and the
     per-layer kernels compute the same split-fp16 products in the same K order: cost and gradient
@@ -321,8 +321,9 @@ def test_mlp_execution_modes_agree(fx, mode, cg, monkeypatch):
     monkeypatch.setenv("FELIX_MLP", "tile")
     monkeypatch.setenv("FELIX_TILE_CG", "1")
     base = fx.Space(sp).eval(cm, y0, lam=1.0)
-    monkeypatch.setenv("FELIX_MLP", mode)
+    monkeypatch.setenv("FELIX_MLP", mode.split("-")[0])
     monkeypatch.setenv("FELIX_TILE_CG", cg)
+    monkeypatch.setenv("FELIX_CHAIN_CS", "4" if mode == "chain-cluster" else "1")
     other = fx.Space(sp).eval(cm, y0, lam=1.0)
     for key in ("cost", "grad"):
         a, b = base[key].cpu().numpy(), other[key].cpu().numpy()
@@ -410,3 +411,29 @@ def test_history_requires_recording(fx):
     space.search(cm, y, 2, init_from_y=True)
     with pytest.raises(fx.FelixError):
         space.history_topk(cm, 8)
+
+
+@pytest.mark.parametrize("n", [1000, 8192])
+@pytest.mark.timeout(300)
+def test_subgraph_concurrent_sketches(fx, n):
+    """Eq. 3 over the C2 subgraph's three symbolic programs, searched concurrently on three streams
+    (n=1000: cluster chains; n=8192: cooperative grid chains, which must not deadlock each other):
+    the merged records equal the sequential run bit for bit and the oracle's merge of the per-program
+    top-k lists."""
+    from paper_conf_asplos_zhaosam24_b200.subgraph import SubgraphSearch
+    mlp = fi.make_mlp(fi.DEFAULT_MLP)
+    cm = fx.CostModel.from_weights(mlp)
+    sks = fi.c2_sketches()
+    drv = SubgraphSearch(sks, cm)
+    T = 12 if n == 1000 else 4
+    conc = drv.run(n, T, 16, rng_seed=77, concurrent=True)
+    seq = drv.run(n, T, 16, rng_seed=77, concurrent=False)
+    assert [(r.sketch, r.idx, r.score) for r in conc] == [(r.sketch, r.idx, r.score) for r in seq]
+    assert all(np.array_equal(a.sched, b.sched) for a, b in zip(conc, seq))
+    per = []
+    for sp in drv.spaces:
+        y = torch.empty((sp.n_vars, n), device="cuda")
+        sp.search(cm, y, T, rng_seed=77, init_from_y=False)
+        per.append(sp.round_topk(cm, y, 16))
+    ref = fo.subgraph_topk(per, 16)
+    assert [(r.sketch, r.idx, r.score) for r in conc] == [(a, b, c) for a, b, c, _ in ref]

@@ -410,3 +410,26 @@ def test_history_topk_monotone_and_revisits_add_nothing():
     a = fo.round_topk_history(sp, mlp.W, mlp.b, ys[:1], 16)
     b = fo.round_topk_history(sp, mlp.W, mlp.b, ys[:1] + [perm], 16)
     assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1]) and a[4] == b[4]
+
+
+def test_subgraph_topk_equals_bruteforce_over_all_sketches():
+    """Eq. 3's max over programs: merging the per-sketch top-k lists equals ranking every valid
+    rounded point of every sketch (dedup within a sketch only) in one sort."""
+    mlp = fi.make_mlp(fi.DEFAULT_MLP)
+    sks = fi.c2_sketches()
+    ys = [fi.make_y0(sp, 120, seed=40 + i) for i, sp in enumerate(sks)]
+    per = [fo.round_topk(sp, mlp.W, mlp.b, y, 8) for sp, y in zip(sks, ys)]
+    got = fo.subgraph_topk(per, 8)
+    allrec = []
+    for i, (sp, y) in enumerate(zip(sks, ys)):
+        sched = fo.round_schedules(sp, y)
+        ok = fo.validate(sp, sched)
+        sc = fo.score(sp, mlp.W, mlp.b, sched)
+        seen = set()
+        for s in range(y.shape[1]):
+            if ok[s] and np.isfinite(sc[s]) and sched[s].tobytes() not in seen:
+                seen.add(sched[s].tobytes())
+                allrec.append((i, s, sc[s]))
+    allrec.sort(key=lambda r: (-r[2], r[0], r[1]))
+    assert [(r[0], r[1]) for r in got] == [(r[0], r[1]) for r in allrec[:8]]
+    assert [r[2] for r in got] == [r[2] for r in allrec[:8]]
