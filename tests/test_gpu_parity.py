@@ -437,3 +437,27 @@ def test_subgraph_concurrent_sketches(fx, n):
         per.append(sp.round_topk(cm, y, 16))
     ref = fo.subgraph_topk(per, 16)
     assert [(r.sketch, r.idx, r.score) for r in conc] == [(a, b, c) for a, b, c, _ in ref]
+
+
+def test_search_quality_curves(fx):
+    """Fig. 8-style diagnostic (tools/search_quality.py): on C1 the history best / 64th-best are
+    non-decreasing in the schedules searched, and the s-step history top-k equals the oracle's on
+    the GPU trajectory for a short prefix."""
+    import importlib.util, os
+    spec = importlib.util.spec_from_file_location("sq", os.path.join(os.path.dirname(__file__), "..", "tools", "search_quality.py"))
+    sq = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(sq)
+    cfg = fi.config("C1")
+    sp = cfg.spaces[0]
+    mlp = fi.make_mlp(cfg.mlp_dims)
+    space, cm = fx.Space(sp), fx.CostModel.from_weights(mlp)
+    res = sq.curves(space, cm, cfg.n_seeds, [1, 2, 5, 10, 20], cfg.rng_seed, cfg.lr, cfg.lam, kq=16)
+    best = [r["best"] for r in res]
+    q = [r["top16"] for r in res]
+    assert all(b1 >= b0 for b0, b1 in zip(best, best[1:]))
+    assert all(b1 >= b0 for b0, b1 in zip(q, q[1:]))
+    y0 = space.init_sample(cfg.n_seeds, cfg.rng_seed).cpu().numpy()
+    ys = _gpu_trajectory(space, cm, y0, 5, lr=cfg.lr, lam=cfg.lam)
+    ref = fo.round_topk_history(sp, mlp.W, mlp.b, ys, 16)
+    assert abs(res[2]["best"] - ref[2][0]) <= 1e-12 * abs(ref[2][0])            # FP64 scores: rel <= 1e-12
+    assert abs(res[2]["top16"] - ref[2][15]) <= 1e-12 * abs(ref[2][15])
