@@ -261,14 +261,18 @@ struct Gen {
 
   void emit_adj_decls(const std::vector<bool>& need, const char* ind) {
     for (int i = 0; i < n; ++i)
-      if (need[i] && d.nodes[i].op != FELIX_OP_VAR) o << ind << "double a" << i << " = 0.0;\n";
+      if (need[i] && d.nodes[i].op != FELIX_OP_VAR) o << ind << "ADJ_T a" << i << " = 0;\n";
   }
 
+  // Reverse sweep.  Adjoints are ADJ_T (double by default; float with FELIX_ADJ=f32);
+  // every local partial derivative is evaluated in FP64 from the FP64 forward values and rounded to
+  // ADJ_T once, via J(...), before it multiplies the adjoint.
   void emit_reverse_body(const std::vector<bool>& need, const char* ind) {
     auto acc = [&](int tgt, const std::string& expr, bool neg = false) {
       if (!depvar[tgt]) return;
       o << ind << "  " << adj(tgt) << (neg ? " -= " : " += ") << expr << ";\n";
     };
+    auto J = [](const std::string& e) { return "(ADJ_T)(" + e + ")"; };
     for (int i = n - 1; i >= 0; --i) {
       const felix_node& nd = d.nodes[i];
       if (!need[i] || nd.op == FELIX_OP_VAR || nd.op == FELIX_OP_CONST) continue;
@@ -279,36 +283,38 @@ struct Gen {
       switch (nd.op) {
         case FELIX_OP_ADD: acc(nd.a, g); acc(nd.b, g); break;
         case FELIX_OP_SUB: acc(nd.a, g); acc(nd.b, g, true); break;
-        case FELIX_OP_MUL: acc(nd.a, g + " * " + B); acc(nd.b, g + " * " + A); break;
+        case FELIX_OP_MUL: acc(nd.a, g + " * " + J(B)); acc(nd.b, g + " * " + J(A)); break;
         case FELIX_OP_DIV: case FELIX_OP_FLOORDIV: case FELIX_OP_CEILDIV:
-          o << ind << "  const double t = " << g << " * f_rcp(" << B << ");\n";
-          acc(nd.a, "t"); acc(nd.b, "t * " + V, true); break;
+          o << ind << "  const ADJ_T t = " << g << " * " << J("f_rcp(" + B + ")") << ";\n";
+          acc(nd.a, "t"); acc(nd.b, "t * " + J(V), true); break;
         case FELIX_OP_NEG: acc(nd.a, g, true); break;
-        case FELIX_OP_POW: acc(nd.a, g + " * " + lit(nd.imm) + " * pow(" + A + ", " + lit(nd.imm - 1.0) + ")"); break;
-        case FELIX_OP_EXP: acc(nd.a, g + " * " + V); break;
-        case FELIX_OP_LOG: acc(nd.a, g + " * f_rcp(" + A + ")"); break;
-        case FELIX_OP_SQRT: acc(nd.a, g + " * 0.5 * f_rcp(" + V + ")"); break;
+        case FELIX_OP_POW: acc(nd.a, g + " * " + J(lit(nd.imm) + " * pow(" + A + ", " + lit(nd.imm - 1.0) + ")")); break;
+        case FELIX_OP_EXP: acc(nd.a, g + " * " + J(V)); break;
+        case FELIX_OP_LOG: acc(nd.a, g + " * " + J("f_rcp(" + A + ")")); break;
+        case FELIX_OP_SQRT: acc(nd.a, g + " * " + J("0.5 * f_rcp(" + V + ")")); break;
         case FELIX_OP_MAX:
-          o << ind << "  const double s = sm_Sh(t" << i << ", h" << i << ");\n";
-          acc(nd.a, g + " * s"); acc(nd.b, g + " * (1.0 - s)"); break;
+          o << ind << "  const ADJ_T s = " << J("sm_Sh(t" + std::to_string(i) + ", h" + std::to_string(i) + ")") << ";\n";
+          acc(nd.a, g + " * s"); acc(nd.b, g + " * ((ADJ_T)1 - s)"); break;
         case FELIX_OP_MIN:
-          o << ind << "  const double s = sm_Sh(t" << i << ", h" << i << ");\n";
-          acc(nd.a, g + " * (1.0 - s)"); acc(nd.b, g + " * s"); break;
+          o << ind << "  const ADJ_T s = " << J("sm_Sh(t" + std::to_string(i) + ", h" + std::to_string(i) + ")") << ";\n";
+          acc(nd.a, g + " * ((ADJ_T)1 - s)"); acc(nd.b, g + " * s"); break;
         case FELIX_OP_GT: case FELIX_OP_GE:
-          o << ind << "  const double t = " << g << " * sm_dSh(h" << i << ");\n";
+          o << ind << "  const ADJ_T t = " << g << " * " << J("sm_dSh(h" + std::to_string(i) + ")") << ";\n";
           acc(nd.a, "t"); acc(nd.b, "t", true); break;
         case FELIX_OP_LT: case FELIX_OP_LE:
-          o << ind << "  const double t = " << g << " * sm_dSh(h" << i << ");\n";
+          o << ind << "  const ADJ_T t = " << g << " * " << J("sm_dSh(h" + std::to_string(i) + ")") << ";\n";
           acc(nd.a, "t", true); acc(nd.b, "t"); break;
-        case FELIX_OP_EQ: case FELIX_OP_NE:
-          o << ind << "  const double t = " << (nd.op == FELIX_OP_EQ ? "" : "-") << g << " * (sm_dSh(h" << i << ") * q" << i
-            << " - p" << i << " * sm_dSh(k" << i << "));\n";
+        case FELIX_OP_EQ: case FELIX_OP_NE: {
+          const std::string I = std::to_string(i);
+          o << ind << "  const ADJ_T t = " << (nd.op == FELIX_OP_EQ ? "" : "-") << g << " * "
+            << J("sm_dSh(h" + I + ") * q" + I + " - p" + I + " * sm_dSh(k" + I + ")") << ";\n";
           acc(nd.a, "t"); acc(nd.b, "t", true); break;
-        case FELIX_OP_AND: acc(nd.a, g + " * " + B); acc(nd.b, g + " * " + A); break;
-        case FELIX_OP_OR: acc(nd.a, g + " * (1.0 - " + B + ")"); acc(nd.b, g + " * (1.0 - " + A + ")"); break;
+        }
+        case FELIX_OP_AND: acc(nd.a, g + " * " + J(B)); acc(nd.b, g + " * " + J(A)); break;
+        case FELIX_OP_OR: acc(nd.a, g + " * " + J("1.0 - " + B)); acc(nd.b, g + " * " + J("1.0 - " + A)); break;
         case FELIX_OP_NOT: acc(nd.a, g, true); break;
         case FELIX_OP_SELECT:
-          acc(nd.a, g + " * (" + B + " - " + C + ")"); acc(nd.b, g + " * " + A); acc(nd.c, g + " * (1.0 - " + A + ")"); break;
+          acc(nd.a, g + " * " + J(B + " - " + C)); acc(nd.b, g + " * " + J(A)); acc(nd.c, g + " * " + J("1.0 - " + A)); break;
         default: break;
       }
       o << ind << "}\n";
@@ -382,6 +388,11 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
          "#define TSTAMP(k, s) do { if (threadIdx.x == 0 && blockIdx.x < 8192) { unsigned long long t_; asm volatile(\"mov.u64 %0, %globaltimer;\" : \"=l\"(t_)); felix_trace[k][blockIdx.x][s] = t_; } } while (0)\n";
   else
     o << "#define TSTAMP(k, s) do {} while (0)\n";
+  // reverse-sweep adjoint type: double by default; FELIX_ADJ=f32 uses float adjoints (parity-green,
+  // measured no faster: C2 reverse kernel 16.7 us either way, C5 -2 %)
+  const char* adj_env = std::getenv("FELIX_ADJ");
+  const bool adj64 = !(adj_env && std::string(adj_env) == "f32");
+  o << "#define ADJ_T " << (adj64 ? "double" : "float") << "\n";
   o << "#define NV " << M << "\n#define NF " << K << "\n#define NRU " << Ru << "\n#define NR " << R
     << "\n#define NRA " << Ra << "\n#define K0P " << K0p << "\n#define PG " << P << "\n";
 
@@ -555,17 +566,17 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     o << "    }\n";
     const auto need = g.rev_live(rcone[q], rroots_g[q]);
     g.emit_adj_decls(need, "    ");
-    for (int j = 0; j < M; ++j) o << "    double gx" << j << " = 0.0;\n";
+    for (int j = 0; j < M; ++j) o << "    ADJ_T gx" << j << " = 0;\n";
     for (int k : part.feat[q]) {
       const int r = d.froots[k];
-      o << "    " << g.adj(r) << " += (double)dphi[(size_t)" << k << " * ld_dphi + cc] * slogp_(v" << r << ");\n";
+      o << "    " << g.adj(r) << " += (ADJ_T)((double)dphi[(size_t)" << k << " * ld_dphi + cc] * slogp_(v" << r << "));\n";
     }
     for (int r : part.cons[q]) {
       const int nd = d.croots[r];
-      if (g.depvar[nd]) o << "    " << g.adj(nd) << " += 2.0 * dlam * p" << r << ";\n";
+      if (g.depvar[nd]) o << "    " << g.adj(nd) << " += (ADJ_T)(2.0 * dlam * p" << r << ");\n";
     }
     g.emit_reverse_body(need, "    ");
-    for (int j = 0; j < M; ++j) o << "    spart[(" << q << " * NV + " << j << ") * 32 + lane] = gx" << j << ";\n";
+    for (int j = 0; j < M; ++j) o << "    spart[(" << q << " * NV + " << j << ") * 32 + lane] = (double)gx" << j << ";\n";
     o << "  }\n";
   }
   // automatic roots (warp 0) from the staged y
