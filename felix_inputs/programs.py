@@ -22,6 +22,15 @@ Sketch (per spatial axis i with extent E_i, per reduction axis j with extent K_j
     s_i = b_i*(V_i T_i I_i) + v_i*(T_i I_i) + t_i*I_i + in_i
     r_j = ro_j*Rt_j + rm_j*RI2_j + ri_j            (Rt_j = product of the axis' tile vars, or K_j)
 Per-thread loop list L (outer -> inner): ro_*, rm_*, v_*, ri_*, in_*.
+
+With statements=2 (TenSet-style per-statement features; the paper's feature
+examples count one statement), the fused bias / activation epilogue is a statement of its
+own, run by the same threads after the reduction:
+            for v_i in [0, V_i):
+              for in_i in [0, I_i):
+                O[s] = act(O[s] + Bias[s_c])           (s_c = the spatial axis `bias_axis`)
+Its epilogue loop list L_E is v_*, in_*; its read buffers are [Bias] (if any).  Both statements use
+the same 82 feature definitions; the main statement then carries no epilogue op counts.
 """
 from __future__ import annotations
 
@@ -67,6 +76,7 @@ class ProgramSpec:
     relu: bool = False
     gelu: bool = False
     unroll: bool = True
+    bias_axis: str = ""        # spatial axis indexing the bias vector (epilogue statement's read buffer)
     smem_limit: int = 48 * 1024
     thread_limit: int = 1024
     local_limit: int = 256
@@ -223,7 +233,83 @@ def _linear_stride(spec: ProgramSpec, buf: Buffer, axis: str) -> int:
     return sum(pitch[d] * c for d, dim in enumerate(buf.dims) for a, c in dim if a == axis)
 
 
-def build_space(spec: ProgramSpec) -> Space:
+def _epilogue_feats(spec: ProgramSpec, ctx: "_Ctx") -> List[Tuple[str, int]]:
+    """Feature formulas of the epilogue statement (module docstring), same names / order / definitions
+    as the main statement's."""
+    b = ctx.b
+    E = float(np.prod([ax.extent for ax in spec.spatial]))
+    NB = b.prod([ctx.Nb(ax) for ax in spec.spatial])
+    NT = b.prod([ctx.T(ax) for ax in spec.spatial])
+    NV = b.prod([ctx.V(ax) for ax in spec.spatial])
+    opt = b.prod([b.mul(ctx.V(ax), ctx.I(ax)) for ax in spec.spatial])      # instances = outputs per thread
+    loops = [("v", ctx.V(ax), ax.name, b.mul(ctx.T(ax), ctx.I(ax))) for ax in spec.spatial] + \
+            [("in", ctx.I(ax), ax.name, b.const(1.0)) for ax in spec.spatial]
+    nontriv = b.sum([b.select(b.gt(ext, b.const(1.0)), b.const(1.0), b.const(0.0)) for _, ext, _, _ in loops])
+    n_ops = float(spec.bias) + float(spec.relu) + float(spec.gelu)
+    f: List[Tuple[str, int]] = []
+    f.append(("float_mad", b.const(0.0)))
+    f.append(("float_addsub", b.const(E if spec.bias else 0.0)))
+    f.append(("float_cmp", b.const(E if spec.relu else 0.0)))
+    f.append(("float_math", b.const(E if spec.gelu else 0.0)))
+    f.append(("blockIdx_len", NB))
+    f.append(("vthread_len", NV))
+    f.append(("threadIdx_len", NT))
+    f.append(("outputs_per_thread", opt))
+    f.append(("stmts_per_thread", opt))
+    f.append(("n_nontrivial_loops", nontriv))
+    f.append(("int_addsub", b.mul(b.const(E), b.add(b.const(2.0), nontriv))))
+    n_block_axes = b.sum([b.select(b.gt(ctx.Nb(ax), b.const(1.0)), b.const(1.0), b.const(0.0)) for ax in spec.spatial])
+    f.append(("int_mul", b.mul(b.const(E), n_block_axes)))
+    f.append(("reduction_outer_iters", b.const(1.0)))
+    if spec.unroll:
+        U = ctx.v("UNROLL")
+        f.append(("unroll_len", b.min(U, opt)))
+        cum, cnt = b.const(1.0), []
+        for _, ext, _, _ in reversed(loops):
+            cum = b.mul(cum, ext)
+            cnt.append(b.select(b.le(cum, U), b.const(1.0), b.const(0.0)))
+        f.append(("unrolled_loops", b.sum(cnt)))
+    else:
+        f.append(("unroll_len", b.const(0.0)))
+        f.append(("unrolled_loops", b.const(0.0)))
+    gbytes, smem = [], []
+    bufs = [Buffer("Bias", [[(spec.bias_axis, 1)]])] if spec.bias else []
+    for slot in range(len(spec.inputs)):
+        if slot < len(bufs):
+            buf = bufs[slot]
+            blk = _dim_footprint(ctx, buf.dims[0], "block")
+            thr = _dim_footprint(ctx, buf.dims[0], "thread")
+            gl = b.mul(NB, blk)
+            gb = b.mul(b.const(4.0), gl)
+            gbytes.append(gb)
+            smem.append(blk)
+            stride = b.const(0.0)
+            for kind, ext, axn, step in loops:
+                d = b.mul(step, b.const(float(_linear_stride(spec, buf, axn))))
+                stride = b.select(b.gt(ext, b.const(1.0)), d, stride)
+            vals = [blk, gl, gb, b.ceildiv(blk, NT), thr, b.div(opt, thr), b.div(b.mul(opt, NT), blk),
+                    b.div(b.const(E), gl), stride, b.mul(b.const(4.0), blk)]
+        else:
+            vals = [b.const(0.0)] * 10
+        names = ["block_footprint", "global_load_elems", "global_bytes", "coop_loads_per_thread", "thread_footprint",
+                 "thread_reuse", "block_reuse", "global_reuse", "innermost_stride", "shared_bytes"]
+        f += [(f"in{slot}.{nm}", v) for nm, v in zip(names, vals)]
+    gsum = b.sum(gbytes) if gbytes else b.const(0.0)
+    f += [
+        ("out.stores", b.const(E)),
+        ("shared_bytes_total", b.mul(b.const(4.0), b.sum(smem)) if smem else b.const(0.0)),
+        ("local_bytes", b.mul(b.const(4.0), opt)),
+        ("flops_per_global_byte", b.div(b.const(n_ops * E), b.add(gsum, b.const(4.0 * E)))),
+        ("flops_per_thread", b.mul(b.const(n_ops), opt)),
+        ("global_bytes_per_block", b.div(gsum, NB)),
+    ]
+    return f
+
+
+def build_space(spec: ProgramSpec, statements: int = 1) -> Space:
+    """statements=1: one feature vector (the main statement, epilogue ops folded in); statements=2:
+    [main statement | epilogue statement], 82 features each, statement-major (TenSet segment sum)."""
+    assert statements in (1, 2)
     vars_, splits, index = var_layout(spec)
     b = DagBuilder()
     ctx = _Ctx(spec, b, index)
@@ -244,10 +330,11 @@ def build_space(spec: ProgramSpec) -> Space:
     n_nontriv = b.sum(nontriv)
 
     # -- op counts / GPU mapping / loop structure
+    epi_in_main = statements == 1
     feats.append(("float_mad", b.const(nmac)))
-    feats.append(("float_addsub", b.const(prodE if spec.bias else 0.0)))
-    feats.append(("float_cmp", b.const(prodE if spec.relu else 0.0)))
-    feats.append(("float_math", b.const(prodE if spec.gelu else 0.0)))
+    feats.append(("float_addsub", b.const(prodE if spec.bias and epi_in_main else 0.0)))
+    feats.append(("float_cmp", b.const(prodE if spec.relu and epi_in_main else 0.0)))
+    feats.append(("float_math", b.const(prodE if spec.gelu and epi_in_main else 0.0)))
     feats.append(("blockIdx_len", NB))
     feats.append(("vthread_len", NV))
     feats.append(("threadIdx_len", NT))
@@ -315,6 +402,11 @@ def build_space(spec: ProgramSpec) -> Space:
     zero = b.const(0.0)
     for k in range(N_FEATURES - n_used):   # annotation slots this sketch never produces
         feats.append((f"reserved_{k}", zero))
+    if statements == 2:
+        ef = _epilogue_feats(spec, ctx)
+        assert len(ef) == n_used
+        feats = [(f"S0.{nm}", v) for nm, v in feats] + [(f"S1.{nm}", v) for nm, v in ef] + \
+                [(f"S1.reserved_{k}", zero) for k in range(N_FEATURES - n_used)]
 
     # -- user constraints g(x) <= 0, in log form so lambda has a uniform scale (SURVEY O2 reading)
     cons: List[Tuple[str, int]] = []
@@ -344,7 +436,7 @@ def dense_spec(name: str, N: int, M: int, K: int, *, i_levels="ti", j_levels="ti
         a_dims = [[("b", 1)]] + a_dims
         b_dims = [[("b", 1)]] + b_dims
     return ProgramSpec(name, spatial, [RAxis("k", K, k_vars)],
-                       [Buffer("A", a_dims), Buffer("B", b_dims)], bias=bias, relu=relu, gelu=gelu)
+                       [Buffer("A", a_dims), Buffer("B", b_dims)], bias=bias, relu=relu, gelu=gelu, bias_axis="j")
 
 
 def conv2d_spec(name: str, C: int, H: int, W: int, K: int, R: int, S: int, stride: int = 1, *,
@@ -355,7 +447,7 @@ def conv2d_spec(name: str, C: int, H: int, W: int, K: int, R: int, S: int, strid
     red = [RAxis("rc", C, rc_vars), RAxis("rh", R, 0), RAxis("rw", S, 0)]
     inp = Buffer("In", [[("rc", 1)], [("h", stride), ("rh", 1)], [("w", stride), ("rw", 1)]])
     wt = Buffer("Wt", [[("co", 1)], [("rc", 1)], [("rh", 1)], [("rw", 1)]])
-    return ProgramSpec(name, spatial, red, [inp, wt], bias=bias, relu=relu)
+    return ProgramSpec(name, spatial, red, [inp, wt], bias=bias, relu=relu, bias_axis="co")
 
 
 def paper_dense_add_s1(N: int = 64, M: int = 64, K: int = 64) -> Space:

@@ -260,6 +260,26 @@ def mlp_input_grad(W: Sequence[np.ndarray], zs: Sequence[np.ndarray], dc: np.nda
     return delta
 
 
+def segment_sum_forward(W: Sequence[np.ndarray], b: Sequence[np.ndarray], phi: np.ndarray):
+    """TenSet-style cost over per-statement feature vectors (per-statement feature
+    examples P:L668-671): phi [S*K0, B] statement-major, C = sum_s MLP(phi_s).  S = 1 is mlp_forward.
+    Returns c [B] and the per-statement pre-activation lists."""
+    K0 = np.asarray(W[0]).shape[1]
+    S = phi.shape[0] // K0
+    assert S * K0 == phi.shape[0]
+    c, zs_all = None, []
+    for s in range(S):
+        cs, zs = mlp_forward(W, b, phi[s * K0:(s + 1) * K0])
+        c = cs if c is None else c + cs
+        zs_all.append(zs)
+    return c, zs_all
+
+
+def segment_sum_input_grad(W: Sequence[np.ndarray], zs_all, dc: np.ndarray) -> np.ndarray:
+    """dC/dphi of segment_sum_forward: each statement's MLP input gradient (dC/dc_s = dC/dc)."""
+    return np.concatenate([mlp_input_grad(W, zs, dc) for zs in zs_all], axis=0)
+
+
 # =============================================================================== O6/O7 objective + grad
 @dataclass
 class Objective:
@@ -285,13 +305,14 @@ def objective(space, W, b, y: np.ndarray, lam: float, with_grad: bool = True) ->
     ev = eval_dag(space, x, smooth=True)
     g = np.concatenate([ev.g_user, auto_roots(space, y)], axis=0)
     phi = slog(ev.F)
-    c, zs = mlp_forward(W, b, phi)
+    c, zs_all = segment_sum_forward(W, b, phi)                # one statement unless the space has S of them
+    zs = [z for zst in zs_all for z in zst]
     with np.errstate(all="ignore"):
         pen = np.maximum(g, 0.0)
         loss = -c + lam * np.sum(pen * pen, axis=0)
     if not with_grad:
         return Objective(x, ev.F, phi, g, c, loss, None, zs, None)
-    dphi = mlp_input_grad(W, zs, -np.ones_like(c))            # dL/dc = -1
+    dphi = segment_sum_input_grad(W, zs_all, -np.ones_like(c))   # dL/dc = -1
     with np.errstate(all="ignore"):
         seedF = dphi * slog_prime(ev.F)
         seedG = 2.0 * lam * pen
@@ -602,7 +623,7 @@ def score(space, W, b, sched: np.ndarray) -> np.ndarray:
     (TopNSchedulesByPredPerf, Alg. 1 line 21)."""
     x = sched.T.astype(np.float64)
     ev = eval_dag(space, x, smooth=False)
-    c, _ = mlp_forward(W, b, slog(ev.F))
+    c, _ = segment_sum_forward(W, b, slog(ev.F))
     return c
 
 

@@ -220,3 +220,99 @@ def enumerate_valid(space) -> List[Dict[str, int]]:
                 del cur[j]
     rec(0, {})
     return [{names[j]: v for j, v in a.items()} for a in out]
+
+
+def simulate_epilogue(spec, x: Dict[str, int]) -> Dict[str, float]:
+    """The fused bias / activation epilogue statement (felix_inputs/programs.py docstring), counted from
+    its enumerated instances (block, thread, v_*, in_*): one instance per output element."""
+    sp, _ = _levels(spec, x)
+    L = [("v", s["name"], s["V"]) for s in sp] + [("in", s["name"], s["I"]) for s in sp]
+    blk_ranges = [range(s["Nb"]) for s in sp]
+    thr_ranges = [range(s["T"]) for s in sp]
+    rows = []
+    for bi, bt in enumerate(itertools.product(*blk_ranges)):
+        for ti, tt in enumerate(itertools.product(*thr_ranges)):
+            for li in itertools.product(*[range(e) for _, _, e in L]):
+                rows.append((bi, ti) + tuple(bt) + tuple(tt) + tuple(li))
+    arr = np.array(rows, dtype=np.int64)
+    ns = len(sp)
+    blk, thr = arr[:, 0], arr[:, 1]
+    bvec, tvec, lvec = arr[:, 2:2 + ns], arr[:, 2 + ns:2 + 2 * ns], arr[:, 2 + 2 * ns:]
+    li = {(k, a): lvec[:, n] for n, (k, a, _) in enumerate(L)}
+    idx = {}
+    for i, s in enumerate(sp):
+        idx[s["name"]] = (bvec[:, i] * (s["V"] * s["T"] * s["I"]) + li[("v", s["name"])] * (s["T"] * s["I"])
+                          + tvec[:, i] * s["I"] + li[("in", s["name"])])
+    n = len(blk)
+    E = int(np.prod([s["E"] for s in sp]))
+    assert n == E
+    f: Dict[str, float] = {}
+    f["float_mad"] = 0
+    f["float_addsub"] = E if spec.bias else 0
+    f["float_cmp"] = E if spec.relu else 0
+    f["float_math"] = E if spec.gelu else 0
+    NB, NT = len(np.unique(blk)), len(np.unique(thr))
+    f["blockIdx_len"] = NB
+    f["vthread_len"] = int(np.prod([s["V"] for s in sp]))
+    f["threadIdx_len"] = NT
+    t0 = (blk == 0) & (thr == 0)
+    f["outputs_per_thread"] = int(t0.sum())
+    f["stmts_per_thread"] = int(t0.sum())
+    nontriv = sum(1 for _, _, e in L if e > 1)
+    f["n_nontrivial_loops"] = nontriv
+    f["int_addsub"] = n * (2 + nontriv)
+    f["int_mul"] = n * sum(1 for s in sp if s["Nb"] > 1)
+    f["reduction_outer_iters"] = 1
+    per_thread = int(t0.sum())
+    if spec.unroll:
+        U = x["UNROLL"]
+        f["unroll_len"] = min(U, per_thread)
+        cum, cnt = 1, 0
+        for _, _, e in reversed(L):
+            cum *= e
+            if cum <= U:
+                cnt += 1
+        f["unrolled_loops"] = cnt
+    else:
+        f["unroll_len"] = 0
+        f["unrolled_loops"] = 0
+    inner = None
+    for pos in range(len(L) - 1, -1, -1):
+        if L[pos][2] > 1:
+            inner = pos
+            break
+    names = ["block_footprint", "global_load_elems", "global_bytes", "coop_loads_per_thread", "thread_footprint",
+             "thread_reuse", "block_reuse", "global_reuse", "innermost_stride", "shared_bytes"]
+    gsum = smem = 0
+    for slot in range(len(spec.inputs)):
+        if slot == 0 and spec.bias:
+            lin = idx[spec.bias_axis]                       # Bias[s_c], a vector
+            b0 = blk == 0
+            blk_fp = len(np.unique(lin[b0]))
+            gl = int(sum(len(np.unique(lin[blk == bb])) for bb in range(NB)))
+            thr_fp = len(np.unique(lin[t0]))
+            pt = np.bincount(np.arange(blk_fp) % NT, minlength=NT)
+            if inner is None:
+                stride = 0
+            else:
+                sel0 = t0 & np.all(lvec == 0, axis=1)
+                one = np.zeros(len(L), dtype=np.int64)
+                one[inner] = 1
+                sel1 = t0 & np.all(lvec == one[None, :], axis=1)
+                stride = int(lin[sel1][0] - lin[sel0][0])
+            vals = [blk_fp, gl, 4 * gl, int(pt.max()), thr_fp, per_thread / thr_fp, int(b0.sum()) / blk_fp, n / gl,
+                    stride, 4 * blk_fp]
+            gsum += 4 * gl
+            smem += 4 * blk_fp
+        else:
+            vals = [0] * 10
+        for nm, v in zip(names, vals):
+            f[f"in{slot}.{nm}"] = v
+    n_ops = int(spec.bias) + int(spec.relu) + int(spec.gelu)
+    f["out.stores"] = E
+    f["shared_bytes_total"] = smem
+    f["local_bytes"] = 4 * f["outputs_per_thread"]
+    f["flops_per_global_byte"] = n_ops * E / (gsum + 4 * E)
+    f["flops_per_thread"] = n_ops * per_thread
+    f["global_bytes_per_block"] = gsum / NB
+    return f

@@ -14,7 +14,7 @@ import torch
 import felix_inputs as fi
 from felix_inputs.programs import build_space, conv2d_spec, dense_spec
 from oracle import felix_oracle as fo
-from tests.sim.loopnest import enumerate_valid, simulate
+from tests.sim.loopnest import enumerate_valid, simulate, simulate_epilogue
 
 GOLD = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "paper_dense_add_s1.json")))
 
@@ -28,6 +28,33 @@ TINY_SPECS = [
 
 
 # ----------------------------------------------------------------------------- O-pin-1
+@pytest.mark.parametrize("spec", TINY_SPECS, ids=lambda s: s.name)
+def test_two_statement_features_equal_bruteforce(spec):
+    """Per-statement features (statements=2, TenSet segment-sum layout): the main statement equals the
+    brute-force count without the epilogue ops, the epilogue statement equals its own enumeration."""
+    sp = build_space(spec, statements=2)
+    assert len(sp.feature_roots) == 2 * 82
+    pts = enumerate_valid(sp)
+    rng = np.random.default_rng(11)
+    for i in rng.choice(len(pts), min(40, len(pts)), replace=False):
+        p = dict(pts[i])
+        if spec.unroll:
+            p["UNROLL"] = int(rng.choice([1, 2, 4, 16, 1024]))
+        x = np.array([[p[v.name]] for v in sp.vars], dtype=float)
+        F = fo.eval_dag(sp, x, smooth=False).F[:, 0]
+        main, epi = simulate(spec, p), simulate_epilogue(spec, p)
+        for k, nm in enumerate(sp.feature_names):
+            st, base = nm.split(".", 1)
+            if base.startswith("reserved"):
+                assert F[k] == 0.0
+                continue
+            if st == "S0":
+                exp = 0.0 if base in ("float_addsub", "float_cmp", "float_math") else main[base]
+            else:
+                exp = epi[base]
+            assert abs(F[k] - exp) <= 1e-12 * max(1.0, abs(exp)), (spec.name, nm, p, F[k], exp)
+
+
 @pytest.mark.parametrize("spec", TINY_SPECS, ids=lambda s: s.name)
 def test_hard_features_equal_bruteforce_loop_nest(spec):
     """Hard-semantics DAG at every sampled valid integer point == brute-force enumeration of the
@@ -433,3 +460,33 @@ def test_subgraph_topk_equals_bruteforce_over_all_sketches():
     allrec.sort(key=lambda r: (-r[2], r[0], r[1]))
     assert [(r[0], r[1]) for r in got] == [(r[0], r[1]) for r in allrec[:8]]
     assert [r[2] for r in got] == [r[2] for r in allrec[:8]]
+
+
+def test_segment_sum_cost_and_gradient():
+    """Two-statement C2 space: C = MLP(phi_S0) + MLP(phi_S1) checked against the plain MLP on each
+    block and against the torch float64 MLP on the summed outputs; the search gradient of the
+    two-statement objective against central finite differences."""
+    sp = build_space(conv2d_spec("c2_two_stmt", 64, 56, 56, 64, 3, 3, 1), statements=2)
+    mlp = fi.make_mlp(fi.DEFAULT_MLP)
+    y = fi.make_y0(sp, 6, seed=3).astype(np.float64)
+    ob = fo.objective(sp, mlp.W, mlp.b, y, 1.0)
+    c0, _ = fo.mlp_forward(mlp.W, mlp.b, ob.phi[:82])
+    c1, _ = fo.mlp_forward(mlp.W, mlp.b, ob.phi[82:])
+    assert np.allclose(ob.c, c0 + c1, rtol=0, atol=1e-12)
+    net = torch.nn.Sequential(*[m for l in range(len(mlp.W)) for m in
+                                ([torch.nn.Linear(mlp.W[l].shape[1], mlp.W[l].shape[0]).double()] +
+                                 ([torch.nn.ReLU()] if l < len(mlp.W) - 1 else []))])
+    with torch.no_grad():
+        for l, lin in enumerate([m for m in net if isinstance(m, torch.nn.Linear)]):
+            lin.weight.copy_(torch.from_numpy(mlp.W[l].astype(np.float64)))
+            lin.bias.copy_(torch.from_numpy(mlp.b[l].astype(np.float64)))
+        ref = (net(torch.from_numpy(ob.phi[:82].T.copy())) + net(torch.from_numpy(ob.phi[82:].T.copy()))).numpy()[:, 0]
+    assert np.allclose(ob.c, ref, rtol=1e-12, atol=1e-12)
+    h = 1e-6
+    for j in range(sp.n_vars):
+        yp, ym = y.copy(), y.copy()
+        yp[j] += h
+        ym[j] -= h
+        fd = (fo.objective(sp, mlp.W, mlp.b, yp, 1.0, with_grad=False).loss
+              - fo.objective(sp, mlp.W, mlp.b, ym, 1.0, with_grad=False).loss) / (2 * h)
+        assert np.allclose(ob.grad[j], fd, rtol=1e-4, atol=1e-6 * np.max(np.abs(fd)) + 1e-8), (j, ob.grad[j], fd)
