@@ -47,6 +47,9 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
     ap.add_argument("--seeds", type=int, default=0, help="override seeds per GPU (experiments; not the headline)")
     ap.add_argument("--search-steps", type=int, default=0, help="override Adam steps per search (experiments)")
+    ap.add_argument("--two-statements", action="store_true",
+                    help="C2 with TenSet-style per-statement features [reduction | epilogue], C = sum_s MLP "
+                         "(SURVEY 8(f) row 3; not the headline)")
     ap.add_argument("--history", action="store_true",
                     help="paper-faithful Alg. 1: round every visited point (varValuesHistory, l.13/17/20) "
                          "instead of the final point only (SURVEY 8(f) row 1; not the headline)")
@@ -166,6 +169,8 @@ def run_reference(args):
         return 0
     import felix_inputs as fi
     cfg = fi.config(args.config)
+    if args.two_statements:
+        cfg.spaces = [fi.c2_space_two_statements()]
     W = max(args.warmup, 0)
     K = max(args.steps, 1)
     rates = []
@@ -211,6 +216,9 @@ def run_felix(args):
         cfg.n_seeds = (1 << 20) // 8          # C5 is 2^20 candidates over 8 GPUs: one GPU's shard
     if args.search_steps:
         cfg.n_steps = args.search_steps
+    if args.two_statements:
+        assert args.config == "C2", "--two-statements is defined for C2"
+        cfg.spaces = [fi.c2_space_two_statements()]
     sp = cfg.spaces[0]
     mlp = fi.make_mlp(cfg.mlp_dims)
     space = fx.Space(sp, device=dev)
@@ -305,10 +313,11 @@ def run_felix(args):
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
     env_mode = os.environ.get("FELIX_MLP", "")
     tile_fits = tuple(cfg.mlp_dims[1:]) == (512, 256, 256, 1)
+    n_rows = n * sp.n_statements
     if env_mode in ("chain", "layers"):
         mlp_kernel = "mlp_chain_kernel" if env_mode == "chain" else "mlp_gemm_kernel"
     else:
-        mlp_kernel = "mlp_tile_kernel" if tile_fits and (env_mode == "tile" or -(-n // 128) >= sms) else "mlp_chain_kernel"
+        mlp_kernel = "mlp_tile_kernel" if tile_fits and (env_mode == "tile" or -(-n_rows // 128) >= sms) else "mlp_chain_kernel"
     traffic = None
     tname = {"mlp_chain_kernel": "roofline_traffic.json", "mlp_tile_kernel": "roofline_traffic_tile.json"}.get(mlp_kernel, "")
     tpath = os.path.join(ROOT, "profiles", "r01", tname) if tname else ""
@@ -317,7 +326,7 @@ def run_felix(args):
             tj = json.load(f)
         traffic = tj["dram_bytes_read_per_launch"] + tj["dram_bytes_write_per_launch"]
     gemm_ms, gemm_launches = prof["mlp_gemm"]
-    mlp_flops_step = cm.mlp_flops_per_candidate_step() * n           # algorithmic (1-pass) FLOPs per Adam step
+    mlp_flops_step = cm.mlp_flops_per_candidate_step() * n * sp.n_statements   # algorithmic (1-pass) FLOPs / Adam step
     gemm_per_step_ms = gemm_ms / (K * T)         # one chain launch (or 2(L-1) layer launches) per Adam step
     achieved_tflops = mlp_flops_step / (gemm_per_step_ms * 1e-3) / 1e12
     peak = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops")))
@@ -374,7 +383,9 @@ def run_felix(args):
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "fp16x3 split (fp32-accurate) MLP, f64 DAG, f32 Adam", "data": "synthetic",
         "config": {"workload": f"{cfg.name}: {sp.name}, {sp.n_vars} vars, {n} seeds x {T} steps per GPU, "
-                               f"MLP {list(cfg.mlp_dims)}, top-{k}" + (", history rounding (Alg. 1 l.20 over all "
+                               f"MLP {list(cfg.mlp_dims)}, top-{k}" + (f", {sp.n_statements} statements (segment sum)"
+                                                                       if sp.n_statements > 1 else "")
+                               + (", history rounding (Alg. 1 l.20 over all "
                                                                        "visited points)" if hist else ""),
                    "n_seeds_per_gpu": n, "n_steps": T, "topk": k, "parallelism": f"dp{world} (seed shards)",
                    "l2": "flushed (256 MB write) between timed iterations"},

@@ -111,6 +111,12 @@ def c2_space() -> Space:
     return build_space(conv2d_spec("resnet50_conv3x3_56x56x64", 64, 56, 56, 64, 3, 3, 1))
 
 
+def c2_space_two_statements() -> Space:
+    """C2 with TenSet-style per-statement features: [reduction statement | fused bias+ReLU epilogue],
+    82 features each."""
+    return build_space(conv2d_spec("resnet50_conv3x3_56x56x64_2stmt", 64, 56, 56, 64, 3, 3, 1), statements=2)
+
+
 def c2_sketches() -> List[Space]:
     """Several symbolic programs p*_i of the C2 subgraph (Eq. 3): the multi-level-tiling
     sketch with 3-level spatial tiling and a 2-way reduction split (= c2_space), with a 1-way

@@ -66,6 +66,7 @@ class Space:
     feature_names: List[str] = field(default_factory=list)
     constraint_names: List[str] = field(default_factory=list)
     program: Optional[object] = None  # ProgramSpec for the brute-force simulator (tests)
+    n_statements: int = 1            # feature_roots = n_statements per-statement vectors (statement-major)
 
     @property
     def n_vars(self) -> int:

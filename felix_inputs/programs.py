@@ -420,7 +420,7 @@ def build_space(spec: ProgramSpec, statements: int = 1) -> Space:
     nodes, (froots, croots) = prune(nodes, [np.array([f for _, f in feats], dtype=np.int32),
                                              np.array([c for _, c in cons], dtype=np.int32)])
     return Space(spec.name, vars_, splits, nodes, froots, croots,
-                 [n for n, _ in feats], [n for n, _ in cons], spec)
+                 [n for n, _ in feats], [n for n, _ in cons], spec, n_statements=statements)
 
 
 # ------------------------------------------------------------------------------ concrete workloads

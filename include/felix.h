@@ -38,7 +38,7 @@
 extern "C" {
 #endif
 
-#define FELIX_ABI_VERSION 2
+#define FELIX_ABI_VERSION 3
 
 #if defined(__GNUC__)
 #define FELIX_EXPORT __attribute__((visibility("default")))
@@ -97,7 +97,8 @@ typedef struct felix_costmodel felix_costmodel;
 /* Creates a search space on `device`.
  * vars[n_vars], splits[n_splits] (each SPLIT var in >= 1 split; extents in [1, 2^31)),
  * nodes[n_nodes], feature_roots[n_features] (NUM nodes; n_features must equal the cost model's
- * dims[0] at search time), constraint_roots[n_constraints] (NUM nodes, user g_r(x) <= 0).
+ * dims[0] at search time, or S * dims[0] after felix_space_set_statements(S)),
+ * constraint_roots[n_constraints] (NUM nodes, user g_r(x) <= 0).
  * The library appends the automatic log-space validity roots (reading O2), in this order
  * after the user roots:  -y_j for every SPLIT var;  sum_{j in s} y_j - ln(extent_s) per split;
  * ln(lo_j) - y_j and y_j - ln(hi_j) per INT var.  R = total number of roots (felix_space_info).
@@ -112,8 +113,18 @@ FELIX_EXPORT felix_status felix_space_create(int device,
                                 felix_space** out);
 FELIX_EXPORT void felix_space_destroy(felix_space* s);
 
+/* Per-statement features (TenSet-style segment sum; the paper's feature formulas are per statement,
+ * P:L668-671): the feature roots are n_statements vectors of n_features /
+ * n_statements features each, statement-major, and the cost is C = sum_s MLP(slog(Feat_s(x))) — every
+ * statement's vector goes through the same MLP (head bias included) and the outputs are summed, for the
+ * search objective (Eq. 4) and for the FP64 scores of rounded schedules alike.  Must be called before
+ * any compute call (it drops the space's compiled kernels and workspaces).  FELIX_E_INVALID_ARG if
+ * n_statements < 1 or does not divide n_features; FELIX_E_UNSUPPORTED if a vector is wider than 128. */
+FELIX_EXPORT felix_status felix_space_set_statements(felix_space* s, int32_t n_statements);
+
 /* Device-free check of a space description: validates it exactly like felix_space_create, generates
- * the space's CUDA source and, if compile != 0, compiles it with NVRTC for sm_100a (no GPU needed).
+ * the space's CUDA source (for n_statements per-statement vectors, as felix_space_set_statements) and,
+ * if compile != 0, compiles it with NVRTC for sm_100a (no GPU needed).
  * Copies up to src_cap bytes of source (NUL-terminated when it fits) into src (may be NULL) and
  * stores the full length in *src_len (may be NULL). */
 FELIX_EXPORT felix_status felix_codegen(const felix_var* vars, int32_t n_vars,
@@ -121,7 +132,8 @@ FELIX_EXPORT felix_status felix_codegen(const felix_var* vars, int32_t n_vars,
                                         const felix_node* nodes, int32_t n_nodes,
                                         const int32_t* feature_roots, int32_t n_features,
                                         const int32_t* constraint_roots, int32_t n_constraints,
-                                        int32_t compile, char* src, int64_t src_cap, int64_t* src_len);
+                                        int32_t n_statements, int32_t compile, char* src, int64_t src_cap,
+                                        int64_t* src_len);
 
 typedef struct {
   int32_t n_vars, n_nodes, n_features, n_constraints_user, n_roots_total, n_components;

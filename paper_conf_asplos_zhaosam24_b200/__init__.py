@@ -29,7 +29,7 @@ EXPORTED = ["felix_last_error", "felix_abi_version", "felix_space_create", "feli
             "felix_space_info", "felix_codegen", "felix_costmodel_load", "felix_costmodel_destroy",
             "felix_search", "felix_round_topk", "felix_eval", "felix_round", "felix_score",
             "felix_init_sample", "felix_profile_enable", "felix_profile_read", "felix_profile_reset",
-            "felix_debug_trace", "felix_history_topk"]
+            "felix_debug_trace", "felix_history_topk", "felix_space_set_statements"]
 
 
 class FelixError(RuntimeError):
@@ -117,10 +117,11 @@ def codegen(space, compile: bool = False) -> str:
     """Generated CUDA source of a space's expression kernels (device-free; compile=True also runs
     NVRTC for sm_100a)."""
     args, keep = _space_args(space)
+    ns = int(getattr(space, "n_statements", 1))
     n = ctypes.c_int64(0)
-    _check(_lib.felix_codegen(*args, 0, None, ctypes.c_int64(0), ctypes.byref(n)))
+    _check(_lib.felix_codegen(*args, ns, 0, None, ctypes.c_int64(0), ctypes.byref(n)))
     buf = ctypes.create_string_buffer(n.value + 1)
-    _check(_lib.felix_codegen(*args, int(compile), buf, ctypes.c_int64(n.value + 1), ctypes.byref(n)))
+    _check(_lib.felix_codegen(*args, ns, int(compile), buf, ctypes.c_int64(n.value + 1), ctypes.byref(n)))
     return buf.value.decode()
 
 
@@ -178,6 +179,9 @@ class Space:
         h = _P()
         _check(_lib.felix_space_create(int(device), *args, ctypes.byref(h)))
         self._h = h
+        self.n_statements = int(getattr(space, "n_statements", 1))
+        if self.n_statements != 1:
+            _check(_lib.felix_space_set_statements(self._h, self.n_statements))
         self.device = device
         self.n_vars = len(space.vars)
         self.name = getattr(space, "name", "space")
@@ -240,7 +244,7 @@ class Space:
         n = y.shape[1]
         dev = y.device
         out = dict(
-            phi=torch.empty((cm.dims[0], n), dtype=torch.float32, device=dev),
+            phi=torch.empty((self.info.n_features, n), dtype=torch.float32, device=dev),
             g=torch.empty((self.info.n_roots_total, n), dtype=torch.float32, device=dev),
             cost=torch.empty(n, dtype=torch.float32, device=dev),
             loss=torch.empty(n, dtype=torch.float32, device=dev),

@@ -73,12 +73,12 @@ __global__ void round_int_kernel(const float* __restrict__ y, int n, int M, int 
 
 // ---------------------------------------------------------------------------- K6 FP64 MLP scoring
 // out[row][col] = act( b[col] + sum_k W[col][k] * in(row, k) ), k ascending (deterministic, so equal
-// schedules get bit-identical scores).  32x32 output tile per 256-thread block, K staged through
+// schedules get bit-identical scores); accumulate != 0 adds to out (segment sum over statements).  32x32 output tile per 256-thread block, K staged through
 // shared memory in chunks of 32; thread (tx, ty) owns column tx and rows ty*4 .. ty*4+3.
 __global__ void __launch_bounds__(256) score_layer_kernel(const double* __restrict__ in, long long in_rs, long long in_cs,
                                                           int n, int K, const double* __restrict__ W,
                                                           const double* __restrict__ b, double* __restrict__ out,
-                                                          int N, int relu) {
+                                                          int N, int relu, int accumulate) {
   __shared__ double As[32][33];   // [k][row]
   __shared__ double Bs[32][33];   // [k][col]
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * 32 + tx;
@@ -111,7 +111,10 @@ __global__ void __launch_bounds__(256) score_layer_kernel(const double* __restri
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
       const int r = row0 + ty * 4 + q;
-      if (r < n) out[static_cast<size_t>(r) * N + col] = (relu && !(acc[q] > 0.0)) ? 0.0 : acc[q];
+      if (r < n) {
+        const double v = (relu && !(acc[q] > 0.0)) ? 0.0 : acc[q];
+        out[static_cast<size_t>(r) * N + col] = accumulate ? out[static_cast<size_t>(r) * N + col] + v : v;
+      }
     }
   }
 }

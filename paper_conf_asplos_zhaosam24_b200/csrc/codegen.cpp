@@ -382,6 +382,10 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
   const bool trace = std::getenv("FELIX_TRACE") != nullptr;   // debug: per-block phase timestamps
   const int M = d.n_vars, K = (int)d.froots.size(), Ru = (int)d.croots.size();
   const int R = d.n_roots_total(), Ra = R - Ru;
+  const int NS = d.n_statements, K0 = K / NS;   // per-statement feature vectors (TenSet segment sum)
+  // feature k -> (statement, index within the statement's vector)
+  auto fs = [&](int k) { return k / K0; };
+  auto fk = [&](int k) { return k % K0; };
   o << kPrelude;
   if (trace)
     o << "__device__ unsigned long long felix_trace[2][8192][4];\n"
@@ -394,7 +398,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
   const bool adj64 = !(adj_env && std::string(adj_env) == "f32");
   o << "#define ADJ_T " << (adj64 ? "double" : "float") << "\n";
   o << "#define NV " << M << "\n#define NF " << K << "\n#define NRU " << Ru << "\n#define NR " << R
-    << "\n#define NRA " << Ra << "\n#define K0P " << K0p << "\n#define PG " << P << "\n";
+    << "\n#define NRA " << Ra << "\n#define K0P " << K0p << "\n#define PG " << P << "\n#define NS " << NS << "\n";
 
   // ---------------------------------------------------------------- automatic validity roots (y space)
   struct Auto { std::string val; std::vector<std::pair<int, int>> terms; };
@@ -450,9 +454,10 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
 
   // ---------------------------------------------------------------- felix_fwd
   // block = PG warps x 32 candidates; warp q evaluates the features of group q; rows are staged in
-  // shared memory and written out as contiguous 16-byte stores.
+  // shared memory and written out as contiguous 16-byte stores.  With NS statements, statement s of
+  // candidate c is MLP row s * n + c.
   o << "extern \"C\" __global__ void __launch_bounds__(PG * 32) felix_fwd(const float* __restrict__ yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr) {\n"
-    << "  __shared__ float sphi[32][K0P + 1];\n"
+    << "  __shared__ float sphi[NS][32][K0P + 1];\n"
     << "  __shared__ double sx[NV][32];   // x = exp(y), computed once per block and shared by the groups\n"
     << "  const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;\n"
     << "  const int c0 = blockIdx.x * 32, c = c0 + lane;\n"
@@ -463,7 +468,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "  TSTAMP(0, 1);\n"
     << "  if (blockIdx.x == 0 && threadIdx.x == 0 && step_ctr) *step_ctr += 1;\n"
     << "  for (int e = threadIdx.x; e < NV * 32; e += blockDim.x) { const int l = e & 31; const int cl = c0 + l; sx[e >> 5][l] = exp((double)yv[(size_t)(e >> 5) * ldy + (cl < n ? cl : n - 1)]); }\n"
-    << "  for (int k = threadIdx.x; k < 32 * (K0P + 1); k += blockDim.x) (&sphi[0][0])[k] = 0.f;\n"
+    << "  for (int k = threadIdx.x; k < NS * 32 * (K0P + 1); k += blockDim.x) (&sphi[0][0][0])[k] = 0.f;\n"
     << "  __syncthreads();\n";
   for (int q = 0; q < P; ++q) {
     o << "  if (wq == " << q << ") {\n";
@@ -473,33 +478,35 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
           // constant feature: value of its (var-free) cone, evaluated here
           o << "    {\n";
           g.emit_forward(g.cone({d.froots[k]}), 0, "x", "      ");
-          o << "      sphi[lane][" << k << "] = slogf_(v" << d.froots[k] << ");\n    }\n";
+          o << "      sphi[" << fs(k) << "][lane][" << fk(k) << "] = slogf_(v" << d.froots[k] << ");\n    }\n";
         }
     const auto used = vars_in(fcone[q]);
     for (int j = 0; j < M; ++j)
       if (used[j]) o << "    const double x" << j << " = sx[" << j << "][lane];\n";
     g.emit_forward(fcone[q], 0, "x", "    ");
-    for (int k : part.feat[q]) o << "    sphi[lane][" << k << "] = slogf_(v" << d.froots[k] << ");\n";
+    for (int k : part.feat[q]) o << "    sphi[" << fs(k) << "][lane][" << fk(k) << "] = slogf_(v" << d.froots[k] << ");\n";
     o << "  }\n";
   }
   o << "  __syncthreads();\n  TSTAMP(0, 2);\n"
-    << "  // rows c0 .. c0+31 are contiguous: K0P/8 uint4 per row for hi and for lo\n"
+    << "  // rows c0 .. c0+31 of each statement are contiguous: K0P/8 uint4 per row for hi and for lo\n"
     << "#pragma unroll\n"
-    << "  for (int it = 0; it < (32 * (K0P / 8) + PG * 32 - 1) / (PG * 32); ++it) {\n"
-    << "    const int e = threadIdx.x + it * PG * 32;\n"
-    << "    if (e >= 32 * (K0P / 8)) break;\n"
+    << "  for (int it = 0; it < (NS * 32 * (K0P / 8) + PG * 32 - 1) / (PG * 32); ++it) {\n"
+    << "    const int e0 = threadIdx.x + it * PG * 32;\n"
+    << "    if (e0 >= NS * 32 * (K0P / 8)) break;\n"
+    << "    const int st = e0 / (32 * (K0P / 8)), e = e0 % (32 * (K0P / 8));\n"
     << "    const int r = e / (K0P / 8), q8 = e % (K0P / 8);\n"
     << "    if (c0 + r >= n) continue;\n"
+    << "    const size_t row = (size_t)st * n + c0 + r;\n"
     << "    u32 h[4], l[4];\n"
     << "#pragma unroll\n"
     << "    for (int u = 0; u < 4; ++u) {\n"
-    << "      const float f0 = sphi[r][q8 * 8 + 2 * u], f1 = sphi[r][q8 * 8 + 2 * u + 1];\n"
+    << "      const float f0 = sphi[st][r][q8 * 8 + 2 * u], f1 = sphi[st][r][q8 * 8 + 2 * u + 1];\n"
     << "      const u16 h0 = f2h(f0), h1 = f2h(f1);\n"
     << "      h[u] = (u32)h0 | ((u32)h1 << 16);\n"
     << "      l[u] = (u32)f2h(f0 - h2f(h0)) | ((u32)f2h(f1 - h2f(h1)) << 16);\n"
     << "    }\n"
-    << "    reinterpret_cast<uint4*>(phi_hi + (size_t)(c0 + r) * K0P)[q8] = make_uint4(h[0], h[1], h[2], h[3]);\n"
-    << "    reinterpret_cast<uint4*>(phi_lo + (size_t)(c0 + r) * K0P)[q8] = make_uint4(l[0], l[1], l[2], l[3]);\n"
+    << "    reinterpret_cast<uint4*>(phi_hi + row * K0P)[q8] = make_uint4(h[0], h[1], h[2], h[3]);\n"
+    << "    reinterpret_cast<uint4*>(phi_lo + row * K0P)[q8] = make_uint4(l[0], l[1], l[2], l[3]);\n"
     << "  }\n  TSTAMP(0, 3);\n}\n\n";
 
   // ---------------------------------------------------------------- felix_rev (template on mode)
@@ -535,8 +542,8 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "    mreg[jj] = 0.f; vreg[jj] = 0.f;\n"
     << "    if (!EVAL && j < NV) { mreg[jj] = mv[(size_t)j * n + cc]; vreg[jj] = vv[(size_t)j * n + cc]; }\n"
     << "  }\n"
-    << "  float cst = head_b;\n"
-    << "  if (wq == 0) for (int t = 0; t < n_head_tiles; ++t) cst += c_part[(size_t)t * ld_c + cc];\n"
+    << "  float cst = head_b * NS;   // segment sum over statements: every statement's MLP adds its head bias\n"
+    << "  if (wq == 0) for (int s = 0; s < NS; ++s) for (int t = 0; t < n_head_tiles; ++t) cst += c_part[(size_t)t * ld_c + (size_t)s * n + cc];\n"
     << "  const int tstep = EVAL ? 1 : *step_ctr;\n";
   for (int q = 0; q < P; ++q) {
     o << "  if (wq == " << q << ") {\n";
@@ -569,7 +576,8 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     for (int j = 0; j < M; ++j) o << "    ADJ_T gx" << j << " = 0;\n";
     for (int k : part.feat[q]) {
       const int r = d.froots[k];
-      o << "    " << g.adj(r) << " += (ADJ_T)((double)dphi[(size_t)" << k << " * ld_dphi + cc] * slogp_(v" << r << "));\n";
+      o << "    " << g.adj(r) << " += (ADJ_T)((double)dphi[(size_t)" << fk(k) << " * ld_dphi + (size_t)" << fs(k)
+        << " * n + cc] * slogp_(v" << r << "));\n";
     }
     for (int r : part.cons[q]) {
       const int nd = d.croots[r];

@@ -492,7 +492,9 @@ static int choose_bn(int64_t m_tiles, int N) {
   FELIX_THROW(FELIX_E_UNSUPPORTED, "hidden dim must be a multiple of 64");
 }
 
-static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int64_t n) {
+static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int64_t n_cand) {
+  // the MLP sees one row per (statement, candidate): row = statement * n_cand + candidate
+  const int64_t n = n_cand * s->desc.n_statements;
   auto p = std::make_unique<Plan>();
   p->cm = cm;
   p->n = n;
@@ -517,8 +519,8 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
     }
   }
   p->dphi.alloc(static_cast<size_t>(K0p) * np * 4);
-  p->m.alloc(static_cast<size_t>(s->desc.n_vars) * n * 4);
-  p->v.alloc(static_cast<size_t>(s->desc.n_vars) * n * 4);
+  p->m.alloc(static_cast<size_t>(s->desc.n_vars) * n_cand * 4);
+  p->v.alloc(static_cast<size_t>(s->desc.n_vars) * n_cand * 4);
   p->step_ctr.alloc(16);
   const int64_t mt = np / 128;
   // forward GEMMs, layer l = 1..L-1 (W index l-1)
@@ -863,11 +865,16 @@ felix_status felix_space_create(int device, const felix_var* vars, int32_t n_var
 
 felix_status felix_codegen(const felix_var* vars, int32_t n_vars, const felix_split* splits, int32_t n_splits,
                            const felix_node* nodes, int32_t n_nodes, const int32_t* feature_roots, int32_t n_features,
-                           const int32_t* constraint_roots, int32_t n_constraints, int32_t compile, char* src,
-                           int64_t src_cap, int64_t* src_len) {
+                           const int32_t* constraint_roots, int32_t n_constraints, int32_t n_statements,
+                           int32_t compile, char* src, int64_t src_cap, int64_t* src_len) {
   FELIX_API_BEGIN
   auto s = parse_space(vars, n_vars, splits, n_splits, nodes, n_nodes, feature_roots, n_features, constraint_roots,
                        n_constraints);
+  if (n_statements < 1 || n_features % n_statements != 0 || n_features / n_statements > 128)
+    FELIX_THROW(FELIX_E_INVALID_ARG, "n_statements must divide n_features into vectors of <= 128");
+  s->desc.n_statements = n_statements;
+  const int K0 = n_features / n_statements;
+  s->K0p = K0 <= 64 ? 64 : K0 <= 96 ? 96 : 128;
   CodegenInfo info;
   const std::string code = generate_dag_module(s->desc, s->K0p, 8, &info);
   if (src_len) *src_len = static_cast<int64_t>(code.size());
@@ -886,6 +893,25 @@ void felix_space_destroy(felix_space* s) {
   cudaSetDevice(s->device);
   delete s;
   if (prev >= 0) cudaSetDevice(prev);
+}
+
+felix_status felix_space_set_statements(felix_space* s, int32_t n_statements) {
+  FELIX_API_BEGIN
+  if (!s) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL space");
+  const int K = static_cast<int>(s->desc.froots.size());
+  if (n_statements < 1 || K % n_statements != 0)
+    FELIX_THROW(FELIX_E_INVALID_ARG, "n_statements must divide n_features");
+  const int K0 = K / n_statements;
+  if (K0 > 128) FELIX_THROW(FELIX_E_UNSUPPORTED, "per-statement feature width > 128");
+  DeviceGuard dg(s->device);
+  CUDA_OK(cudaDeviceSynchronize());
+  s->desc.n_statements = n_statements;
+  s->K0p = K0 <= 64 ? 64 : K0 <= 96 ? 96 : 128;
+  for (auto& kv : s->modules) if (kv.second.lib) cudaLibraryUnload(kv.second.lib);
+  s->modules.clear();
+  s->search_chunks.reset();
+  s->eval_chunks.reset();
+  FELIX_API_END
 }
 
 felix_status felix_space_info(const felix_space* s, felix_space_info_t* out) {
@@ -969,8 +995,8 @@ void felix_costmodel_destroy(felix_costmodel* m) { delete m; }
 
 static void check_pair(felix_space* s, felix_costmodel* m) {
   if (!s || !m) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL handle");
-  if (static_cast<int>(s->desc.froots.size()) != m->dims[0])
-    FELIX_THROW(FELIX_E_SHAPE, "space n_features != cost model dims[0]");
+  if (s->desc.k0() != m->dims[0])
+    FELIX_THROW(FELIX_E_SHAPE, "space per-statement n_features != cost model dims[0]");
   if (s->device != m->device) FELIX_THROW(FELIX_E_INVALID_ARG, "space and cost model on different devices");
 }
 
@@ -1246,24 +1272,29 @@ static void do_hard(felix_space* s, const int32_t* sched, int64_t n, double* phi
 }
 
 static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, int64_t n, double* score, cudaStream_t st) {
+  // TenSet segment sum over statements: score = sum_s MLP(phi_s), phi64 = [S * K0][n] statement-major
   const int L = m->n_layers;
   int maxw = 0;
   for (int l = 1; l < L; ++l) maxw = std::max(maxw, m->dims[l]);
   ensure(s->act64a, static_cast<size_t>(n) * maxw * 8);
   ensure(s->act64b, static_cast<size_t>(n) * maxw * 8);
-  const double* in = phi64;
-  long long rs = 1, cs = n;    // phi64 is [K][n]
   double* bufs[2] = {s->act64a.as<double>(), s->act64b.as<double>()};
-  for (int l = 0; l < L; ++l) {
-    const int K = m->dims[l], N = m->dims[l + 1];
-    double* out = (l == L - 1) ? score : bufs[l & 1];
-    const dim3 grid(static_cast<unsigned>((N + 31) / 32), static_cast<unsigned>((n + 31) / 32));
-    score_layer_kernel<<<grid, dim3(32, 8), 0, st>>>(
-        in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N, l < L - 1 ? 1 : 0);
-    CUDA_OK(cudaGetLastError());
-    in = out;
-    rs = N;
-    cs = 1;
+  for (int st_i = 0; st_i < s->desc.n_statements; ++st_i) {
+    const double* in = phi64 + static_cast<size_t>(st_i) * m->dims[0] * n;
+    long long rs = 1, cs = n;    // phi64 is [K][n]
+    for (int l = 0; l < L; ++l) {
+      const int K = m->dims[l], N = m->dims[l + 1];
+      const bool last = l == L - 1;
+      double* out = last ? score : bufs[l & 1];
+      const dim3 grid(static_cast<unsigned>((N + 31) / 32), static_cast<unsigned>((n + 31) / 32));
+      score_layer_kernel<<<grid, dim3(32, 8), 0, st>>>(
+          in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
+          last ? 0 : 1, last && st_i > 0 ? 1 : 0);
+      CUDA_OK(cudaGetLastError());
+      in = out;
+      rs = N;
+      cs = 1;
+    }
   }
 }
 

@@ -56,6 +56,8 @@ struct SpaceDesc {
   std::vector<std::vector<int32_t>> split_vars;
   std::vector<felix_node> nodes;
   std::vector<int32_t> froots, croots;
+  int n_statements = 1;          // feature roots = n_statements per-statement vectors, statement-major
+  int k0() const { return static_cast<int>(froots.size()) / n_statements; }
   int n_roots_total() const;
 };
 

@@ -42,6 +42,8 @@ CASES = {
     "r50_conv1": (lambda: fi.resnet50_spaces()[0], fi.DEFAULT_MLP, 300),
     "r50_ds1x1": (lambda: fi.resnet50_spaces()[8], fi.DEFAULT_MLP, 160),
     "bert_qkv": (lambda: fi.bert_spaces()[0], fi.DEFAULT_MLP, 222),
+    # TenSet-style per-statement features: [reduction | fused bias+ReLU epilogue], C = sum_s MLP(phi_s)
+    "C2_2stmt": (fi.c2_space_two_statements, fi.DEFAULT_MLP, 700),
 }
 
 _cache = {}
@@ -89,7 +91,7 @@ def test_eval_parity(fx, name):
     assert exempt.mean() < 0.01
 
 
-@pytest.mark.parametrize("name", ["C1", "C2"])
+@pytest.mark.parametrize("name", ["C1", "C2", "C2_2stmt"])
 def test_one_adam_step_parity(fx, name):
     sp, mlp, n, space, cm = _setup(fx, name)
     y0 = fi.make_y0(sp, n, seed=12)
@@ -337,7 +339,7 @@ def test_tile_mlp_eval_parity_vs_oracle(fx, cg, monkeypatch):
     C2 and C5 shapes with a ragged last tile (and, for the 2-SM pairs, an odd tile count)."""
     monkeypatch.setenv("FELIX_MLP", "tile")
     monkeypatch.setenv("FELIX_TILE_CG", cg)
-    for name, n in (("C2", 1000), ("C5", 389)):
+    for name, n in (("C2", 1000), ("C5", 389), ("C2_2stmt", 333)):
         make, dims, _ = CASES[name]
         sp = make()
         mlp = fi.make_mlp(dims)
