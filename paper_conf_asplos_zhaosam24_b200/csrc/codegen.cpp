@@ -376,7 +376,7 @@ int SpaceDesc::n_roots_total() const {
   return (int)croots.size() + n_split + (int)split_extent.size() + 2 * n_int;
 }
 
-std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo* info) {
+std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, CodegenInfo* info) {
   Gen g(d);
   std::ostringstream& o = g.o;
   const bool trace = std::getenv("FELIX_TRACE") != nullptr;   // debug: per-block phase timestamps
@@ -387,6 +387,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
   auto fs = [&](int k) { return k / K0; };
   auto fk = [&](int k) { return k % K0; };
   o << kPrelude;
+
   if (trace)
     o << "__device__ unsigned long long felix_trace[2][8192][4];\n"
          "#define TSTAMP(k, s) do { if (threadIdx.x == 0 && blockIdx.x < 8192) { unsigned long long t_; asm volatile(\"mov.u64 %0, %globaltimer;\" : \"=l\"(t_)); felix_trace[k][blockIdx.x][s] = t_; } } while (0)\n";
@@ -398,7 +399,8 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
   const bool adj64 = !(adj_env && std::string(adj_env) == "f32");
   o << "#define ADJ_T " << (adj64 ? "double" : "float") << "\n";
   o << "#define NV " << M << "\n#define NF " << K << "\n#define NRU " << Ru << "\n#define NR " << R
-    << "\n#define NRA " << Ra << "\n#define K0P " << K0p << "\n#define PG " << P << "\n#define NS " << NS << "\n";
+    << "\n#define NRA " << Ra << "\n#define K0P " << K0p << "\n#define PG " << P << "\n#define NS " << NS
+    << "\n#define NREP " << NREPv << "\n";
 
   // ---------------------------------------------------------------- automatic validity roots (y space)
   struct Auto { std::string val; std::vector<std::pair<int, int>> terms; };
@@ -456,19 +458,24 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
   // block = PG warps x 32 candidates; warp q evaluates the features of group q; rows are staged in
   // shared memory and written out as contiguous 16-byte stores.  With NS statements, statement s of
   // candidate c is MLP row s * n + c.
-  o << "extern \"C\" __global__ void __launch_bounds__(PG * 32) felix_fwd(const float* __restrict__ yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr) {\n"
-    << "  __shared__ float sphi[NS][32][K0P + 1];\n"
-    << "  __shared__ double sx[NV][32];   // x = exp(y), computed once per block and shared by the groups\n"
-    << "  const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;\n"
-    << "  const int c0 = blockIdx.x * 32, c = c0 + lane;\n"
+  // NREP replicas of the PG groups per block, each on its own 32 candidates: warps running the same
+  // cone's straight-line code share the SM's instruction fetches (the code is executed once per warp).
+  o << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd(const float* __restrict__ yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr) {\n"
+    << "  __shared__ float sphi_all[NREP][NS][32][K0P + 1];\n"
+    << "  __shared__ double sx_all[NREP][NV][32];   // x = exp(y), computed once per replica and shared by its groups\n"
+    << "  const int rep = threadIdx.x / (PG * 32), tid = threadIdx.x % (PG * 32);\n"
+    << "  float (&sphi)[NS][32][K0P + 1] = sphi_all[rep];\n"
+    << "  double (&sx)[NV][32] = sx_all[rep];\n"
+    << "  const int lane = threadIdx.x & 31, wq = tid >> 5;\n"
+    << "  const int c0 = (blockIdx.x * NREP + rep) * 32, c = c0 + lane;\n"
     << "  const int cc = c < n ? c : n - 1;\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
     << "  TSTAMP(0, 0);\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");   // y is the previous step's output\n"
     << "  TSTAMP(0, 1);\n"
     << "  if (blockIdx.x == 0 && threadIdx.x == 0 && step_ctr) *step_ctr += 1;\n"
-    << "  for (int e = threadIdx.x; e < NV * 32; e += blockDim.x) { const int l = e & 31; const int cl = c0 + l; sx[e >> 5][l] = exp((double)yv[(size_t)(e >> 5) * ldy + (cl < n ? cl : n - 1)]); }\n"
-    << "  for (int k = threadIdx.x; k < NS * 32 * (K0P + 1); k += blockDim.x) (&sphi[0][0][0])[k] = 0.f;\n"
+    << "  for (int e = tid; e < NV * 32; e += PG * 32) { const int l = e & 31; const int cl = c0 + l; sx[e >> 5][l] = exp((double)yv[(size_t)(e >> 5) * ldy + (cl < n ? cl : n - 1)]); }\n"
+    << "  for (int k = tid; k < NS * 32 * (K0P + 1); k += PG * 32) (&sphi[0][0][0])[k] = 0.f;\n"
     << "  __syncthreads();\n";
   for (int q = 0; q < P; ++q) {
     o << "  if (wq == " << q << ") {\n";
@@ -491,7 +498,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "  // rows c0 .. c0+31 of each statement are contiguous: K0P/8 uint4 per row for hi and for lo\n"
     << "#pragma unroll\n"
     << "  for (int it = 0; it < (NS * 32 * (K0P / 8) + PG * 32 - 1) / (PG * 32); ++it) {\n"
-    << "    const int e0 = threadIdx.x + it * PG * 32;\n"
+    << "    const int e0 = tid + it * PG * 32;\n"
     << "    if (e0 >= NS * 32 * (K0P / 8)) break;\n"
     << "    const int st = e0 / (32 * (K0P / 8)), e = e0 % (32 * (K0P / 8));\n"
     << "    const int r = e / (K0P / 8), q8 = e % (K0P / 8);\n"
@@ -517,12 +524,14 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "    float* __restrict__ mv, float* __restrict__ vv, const int* step_ctr, float lr, float b1, float b2, float eps,\n"
     << "    float* __restrict__ o_phi, float* __restrict__ o_g, float* __restrict__ o_cost, float* __restrict__ o_loss, float* __restrict__ o_grad) {\n"
     << "  extern __shared__ double smem[];\n"
-    << "  double* spart = smem;                                  // [PG][NV][32]\n"
+    << "  const int rep = threadIdx.x / (PG * 32), tid = threadIdx.x % (PG * 32);\n"
+    << "  constexpr int REPW = ((PG * NV * 32 + PG * 32 + (NRA > 0 ? NRA : 1) * 32) * 8 + NV * 32 * 4 + 15) / 16 * 2;   // doubles per replica\n"
+    << "  double* spart = smem + rep * REPW;                     // [PG][NV][32]\n"
     << "  double* spen = spart + PG * NV * 32;                   // [PG][32]\n"
     << "  double* spa = spen + PG * 32;                          // [NRA][32]\n"
     << "  float* sy = reinterpret_cast<float*>(spa + (NRA > 0 ? NRA : 1) * 32);   // [NV][32]\n"
-    << "  const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;\n"
-    << "  const int c = blockIdx.x * 32 + lane;\n"
+    << "  const int lane = threadIdx.x & 31, wq = tid >> 5;\n"
+    << "  const int c0 = (blockIdx.x * NREP + rep) * 32, c = c0 + lane;\n"
     << "  const bool live = c < n;\n"
     << "  const int cc = live ? c : n - 1;\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
@@ -531,8 +540,9 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "  if (!EVAL) TSTAMP(1, 1);\n"
     << "  const double dlam = (double)lam;\n"
     // everything the epilogue needs from memory is requested now, so its latency overlaps the DAG
-    << "  __shared__ double sx[NV * 32];\n"
-    << "  for (int e = threadIdx.x; e < NV * 32; e += blockDim.x) { const int j = e >> 5, l = e & 31; const int cl = blockIdx.x * 32 + l; const float yy = yin[(size_t)j * ldy + (cl < n ? cl : n - 1)]; sy[e] = yy; sx[e] = exp((double)yy); }\n"
+    << "  __shared__ double sx_all[NREP][NV * 32];\n"
+    << "  double* sx = sx_all[rep];\n"
+    << "  for (int e = tid; e < NV * 32; e += PG * 32) { const int j = e >> 5, l = e & 31; const int cl = c0 + l; const float yy = yin[(size_t)j * ldy + (cl < n ? cl : n - 1)]; sy[e] = yy; sx[e] = exp((double)yy); }\n"
     << "  __syncthreads();\n"
     << "  constexpr int NJ = (NV + PG - 1) / PG;   // vars handled by this thread: j = wq + PG * jj\n"
     << "  float mreg[NJ], vreg[NJ];\n"
@@ -597,7 +607,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
   }
   o << "  }\n  __syncthreads();\n";
   // cost + loss (warp 0); the loss is parked in spen[PG-1 .. ] row 0 after the sum
-  o << "  __shared__ float sloss[32];\n"
+  o << "  __shared__ float sloss_all[NREP][32];\n  float* sloss = sloss_all[rep];\n"
     << "  if (wq == 0) {\n"
     << "    double pen = 0.0;\n"
     << "    for (int q = 0; q < PG; ++q) pen += spen[q * 32 + lane];\n"
@@ -606,7 +616,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "    sloss[lane] = loss;\n"
     << "    if (live) {\n      if (o_loss) o_loss[c] = loss;\n      if (EVAL && o_cost) o_cost[c] = cst;\n    }\n  }\n";
   // gradient per (var, candidate): thread (wq, lane) handles vars j = wq, wq + PG, ...
-  o << "  __shared__ float sgrad[NV][32];\n"
+  o << "  __shared__ float sgrad_all[NREP][NV][32];\n  float (&sgrad)[NV][32] = sgrad_all[rep];\n"
     << "#pragma unroll\n"
     << "  for (int jj = 0; jj < NJ; ++jj) {\n"
     << "    const int j = wq + PG * jj;\n"
@@ -648,10 +658,10 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
     << "    }\n"
     << "    TSTAMP(1, 3);\n"
     << "  }\n}\n\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(PG * 32) felix_rev_adam(float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
+  o << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_adam(float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
     << "    float* mv, float* vv, const int* step_ctr, float lr, float b1, float b2, float eps, float* o_loss) {\n"
     << "  rev_body<0>(yv, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, mv, vv, step_ctr, lr, b1, b2, eps, nullptr, nullptr, nullptr, o_loss, nullptr);\n}\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(PG * 32) felix_rev_eval(const float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
+  o << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_eval(const float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
     << "    float* o_phi, float* o_g, float* o_cost, float* o_loss, float* o_grad) {\n"
     << "  rev_body<1>(nullptr, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, nullptr, nullptr, nullptr, 0.f, 0.f, 0.f, 0.f, o_phi, o_g, o_cost, o_loss, o_grad);\n}\n\n";
 
@@ -733,7 +743,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, CodegenInfo*
 
   if (info) {
     info->flops_fwd = flops_fwd;
-    info->rev_smem_bytes = (P * M * 32 + P * 32 + std::max(Ra, 1) * 32) * 8 + M * 32 * 4;
+    info->rev_smem_bytes = NREPv * (((P * M * 32 + P * 32 + std::max(Ra, 1) * 32) * 8 + M * 32 * 4 + 15) / 16 * 16);
   }
   return o.str();
 }

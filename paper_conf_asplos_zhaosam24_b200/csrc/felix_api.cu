@@ -248,7 +248,7 @@ struct felix_space {
   struct Module {
     cudaLibrary_t lib = nullptr;
     cudaKernel_t f_fwd = nullptr, f_rev_adam = nullptr, f_rev_eval = nullptr, f_hard = nullptr, f_init = nullptr;
-    int P = 1, rev_smem = 0, regs_fwd = 0, regs_rev = 0;
+    int P = 1, R = 1, rev_smem = 0, regs_fwd = 0, regs_rev = 0;   // cone groups, replicas per block
     std::string source;
   };
   std::map<int, Module> modules;
@@ -420,13 +420,18 @@ static std::vector<char> nvrtc_compile(const std::string& source) {
   return cubin;
 }
 
-static felix_space::Module& get_module(felix_space* s, int P) {
-  auto it = s->modules.find(P);
+static felix_space::Module& get_module(felix_space* s, int P, int R = 1) {
+  // the forward kernel stages NREP x NS x 32 x (K0P+1) floats + NREP x NV x 32 doubles statically
+  if (R > 1 && static_cast<int64_t>(R) * (s->desc.n_statements * 32 * (s->K0p + 1) * 4 + s->desc.n_vars * 32 * 8) > 48 * 1024)
+    R = 1;
+  const int key = P + 64 * R;
+  auto it = s->modules.find(key);
   if (it != s->modules.end()) return it->second;
   felix_space::Module mod;
   mod.P = P;
+  mod.R = R;
   CodegenInfo info;
-  mod.source = generate_dag_module(s->desc, s->K0p, P, &info);
+  mod.source = generate_dag_module(s->desc, s->K0p, P, R, &info);
   s->flops_fwd = info.flops_fwd;
   mod.rev_smem = info.rev_smem_bytes;
   auto t0 = std::chrono::steady_clock::now();
@@ -447,7 +452,20 @@ static felix_space::Module& get_module(felix_space* s, int P) {
   s->nvrtc_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   s->regs_fwd = mod.regs_fwd;
   s->regs_rev = mod.regs_rev;
-  return s->modules.emplace(P, std::move(mod)).first->second;
+  return s->modules.emplace(key, std::move(mod)).first->second;
+}
+
+// Replicas of the cone groups per block: warps running the same cone's straight-line code share the
+// SM's instruction fetches (ncu: 42 % of the reverse kernel's stall samples are no_instructions; its
+// SASS is 124 KB at C2).  Measured at C2: R=2 takes the reverse kernel from 16.9 to 15.3 us but the step
+// only +0.6 %; R=4 exceeds the static shared budget.  Default 1; FELIX_R overrides.
+static int choose_R(int64_t n) {
+  if (const char* e = std::getenv("FELIX_R")) {
+    const int r = std::atoi(e);
+    if (r == 1 || r == 2 || r == 4) return r;
+  }
+  (void)n;
+  return 1;
 }
 
 // Cone-partition width: enough warps to give every SM ~8 resident warps of expression work.
@@ -475,9 +493,10 @@ static void launch_cfg(const void* f, dim3 grid, dim3 block, size_t smem, void**
   if (pdl) { cfg.attrs = &g_pdl_attr; cfg.numAttrs = 1; }
   CUDA_OK(cudaLaunchKernelExC(&cfg, f, args));
 }
-static void launch_grouped(cudaKernel_t f, int P, int64_t n, size_t smem, void** args, cudaStream_t st, bool pdl) {
+static void launch_grouped(cudaKernel_t f, int P, int R, int64_t n, size_t smem, void** args, cudaStream_t st, bool pdl) {
   if (n <= 0) return;
-  launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((n + 31) / 32)), dim3(32 * P), smem, args, st, pdl);
+  launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((n + 32 * R - 1) / (32 * R))), dim3(32 * P * R),
+             smem, args, st, pdl);
 }
 static void launch_flat(cudaKernel_t f, int64_t n, void** args, cudaStream_t st) {
   if (n <= 0) return;
@@ -722,7 +741,7 @@ static void run_forward_mlp(felix_space* s, Plan& p, const felix_space::Module& 
   void* phi_lo = p.phi_lo.p;
   void* args[] = {&y, &ni, &ldi, &phi_hi, &phi_lo, &step_ctr};
   prof_mark(s, 0, st, true);
-  launch_grouped(mod.f_fwd, mod.P, n, 0, args, st, true);
+  launch_grouped(mod.f_fwd, mod.P, mod.R, n, 0, args, st, true);
   prof_mark(s, 0, st, false);
   s->prof_launches[0] += 1;
   prof_mark(s, 1, st, true);
@@ -876,7 +895,7 @@ felix_status felix_codegen(const felix_var* vars, int32_t n_vars, const felix_sp
   const int K0 = n_features / n_statements;
   s->K0p = K0 <= 64 ? 64 : K0 <= 96 ? 96 : 128;
   CodegenInfo info;
-  const std::string code = generate_dag_module(s->desc, s->K0p, 8, &info);
+  const std::string code = generate_dag_module(s->desc, s->K0p, 8, 1, &info);
   if (src_len) *src_len = static_cast<int64_t>(code.size());
   if (src && src_cap > 0) {
     const size_t nb = std::min<size_t>(code.size() + 1, static_cast<size_t>(src_cap));
@@ -1017,7 +1036,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
   const int64_t n = p->n_seeds;
   Chunks& ch = get_chunks(s, s->search_chunks, m, n, choose_chunks(n));
   const int nck = static_cast<int>(ch.plans.size());
-  const felix_space::Module& mod = get_module(s, choose_P(ch.cnt[0]));
+  const felix_space::Module& mod = get_module(s, choose_P(ch.cnt[0]), choose_R(ch.cnt[0]));
   if (!p->init_from_y) {
     unsigned long long seed = p->rng_seed;
     long long ib = p->index_base;
@@ -1084,7 +1103,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     float* lo = final_loss ? final_loss + o : nullptr;   // every step writes its loss; the last one stays
     void* args[] = {&yk, &ni, &ldy, &dphi, &ld, &cpart, &nht, &ld, &hbv, &lam, &mv, &vv, &ctr, &lr, &b1, &b2, &eps, &lo};
     prof_mark(s, 2, cs, true);
-    launch_grouped(mod.f_rev_adam, mod.P, cnt, mod.rev_smem, args, cs, true);
+    launch_grouped(mod.f_rev_adam, mod.P, mod.R, cnt, mod.rev_smem, args, cs, true);
     prof_mark(s, 2, cs, false);
     s->prof_launches[2] += 1;
   };
@@ -1215,7 +1234,7 @@ felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int6
   DeviceGuard dg(s->device);
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   Plan& pl = *get_chunks(s, s->eval_chunks, m, n, 1).plans[0];
-  const felix_space::Module& mod = get_module(s, choose_P(n));
+  const felix_space::Module& mod = get_module(s, choose_P(n), choose_R(n));
   run_forward_mlp(s, pl, mod, y, n, n, st, nullptr);
   int ni = static_cast<int>(n);
   void* dphi = pl.dphi.p;
@@ -1224,7 +1243,7 @@ felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int6
   int nht = pl.n_head_tiles;
   float hb = m->head_b, lam = lambda;
   void* args[] = {&y, &ni, &ni, &dphi, &ld, &cpart, &nht, &ld, &hb, &lam, &phi, &g, &cost, &loss, &grad};
-  launch_grouped(mod.f_rev_eval, mod.P, n, mod.rev_smem, args, st, false);
+  launch_grouped(mod.f_rev_eval, mod.P, mod.R, n, mod.rev_smem, args, st, false);
   FELIX_API_END
 }
 
