@@ -1051,6 +1051,9 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     CUDA_OK(cudaMemsetAsync(pl->m.p, 0, pl->m.bytes, st));
     CUDA_OK(cudaMemsetAsync(pl->v.p, 0, pl->v.bytes, st));
     CUDA_OK(cudaMemsetAsync(pl->step_ctr.p, 0, 4, st));
+    // the grid-barrier counter's target arithmetic is not wrap-safe (2^32 is not a multiple of the grid):
+    // restart it every search (stream-ordered, no chain kernel in flight on this workspace)
+    CUDA_OK(cudaMemsetAsync(pl->grid_bar.p, 0, pl->grid_bar.bytes, st));
   }
   // varValuesHistory: a fresh pool for this search (worst case: every seed at every step is new)
   const int M = s->desc.n_vars;
@@ -1215,7 +1218,11 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
       CUDA_OK(ie);
       ch.graph_key = key;
     }
-    for (int t = 1; t <= p->n_steps; ++t) CUDA_OK(cudaGraphLaunch(ch.graph, st));
+    for (int t = 1; t <= p->n_steps; ++t) {
+      if (t % 100000 == 0)   // keep the grid-barrier counter far from 2^32 on very long searches
+        for (auto& pl : ch.plans) CUDA_OK(cudaMemsetAsync(pl->grid_bar.p, 0, pl->grid_bar.bytes, st));
+      CUDA_OK(cudaGraphLaunch(ch.graph, st));
+    }
     s->prof_launches[0] += static_cast<int64_t>(p->n_steps) * nck;
     s->prof_launches[1] += static_cast<int64_t>(p->n_steps) * nck *
                            (ch.plans[0]->mode == MLP_LAYERS ? static_cast<int64_t>(ch.plans[0]->gemms.size()) : 1);
@@ -1234,6 +1241,7 @@ felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int6
   DeviceGuard dg(s->device);
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   Plan& pl = *get_chunks(s, s->eval_chunks, m, n, 1).plans[0];
+  CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
   const felix_space::Module& mod = get_module(s, choose_P(n), choose_R(n));
   run_forward_mlp(s, pl, mod, y, n, n, st, nullptr);
   int ni = static_cast<int>(n);
