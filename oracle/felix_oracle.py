@@ -623,7 +623,13 @@ def score(space, W, b, sched: np.ndarray) -> np.ndarray:
     (TopNSchedulesByPredPerf, Alg. 1 line 21)."""
     x = sched.T.astype(np.float64)
     ev = eval_dag(space, x, smooth=False)
-    c, _ = segment_sum_forward(W, b, slog(ev.F))
+    phi = slog(ev.F)
+    # A score is a function of its schedule alone (the top-k order and its shard invariance,
+    # SURVEY §8(e), depend on that): the MLP runs on one candidate column at a time, because a
+    # batched BLAS matmul may sum in a different order for different batch shapes.
+    c = np.empty(phi.shape[1], dtype=np.float64)
+    for i in range(phi.shape[1]):
+        c[i] = segment_sum_forward(W, b, phi[:, i:i + 1])[0][0]
     return c
 
 
