@@ -11,6 +11,10 @@ all-gather over NCCL).
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl {felix,reference}] [--config C2]
 
+`--config C3` (ResNet-50: 21 tasks x 8192 seeds, subgraphs sharded by LPT) and `--config C4` (BERT-base:
+6 tasks x 16384 seeds x 500 steps, every task's seeds sharded) run the multi-task workloads
+(paper_conf_asplos_zhaosam24_b200/tasks.py): strong scaling, one CUDA stream per task.
+
 `--impl reference` times the float64 oracle (oracle/, numpy) on the host cores for the same
 workload on a bounded sample per step (this tier's reference arm: there is no reference code).
 """
@@ -417,11 +421,250 @@ def run_felix(args):
     return 0
 
 
+# ------------------------------------------------------------------------------------- multi-task configs
+def _tasks_module():
+    from paper_conf_asplos_zhaosam24_b200 import tasks
+    return tasks
+
+
+def oracle_baseline_tasks(cfg, seconds: float):
+    """The oracle on a bounded sample of a multi-task workload: the first m seeds of EVERY task (same
+    device-independent starting points), as many Adam steps as fit in ~`seconds` overall, then its
+    round/top-k; extrapolated linearly per task to n_seeds x n_steps + the finish at n_seeds."""
+    from oracle import felix_oracle as fo
+    import felix_inputs as fi
+    try:
+        import threadpoolctl
+        threads = max(i.get("num_threads", 1) for i in threadpoolctl.threadpool_info()) or os.cpu_count()
+    except Exception:
+        threads = os.cpu_count()
+    mlp = fi.make_mlp(cfg.mlp_dims)
+    m = min(cfg.n_seeds, 1024)
+    y0s = [fo.init_sample(sp, m, cfg.rng_seed + t) for t, sp in enumerate(cfg.spaces)]
+    t0 = time.perf_counter()
+    for sp, y0 in zip(cfg.spaces, y0s):
+        fo.search(sp, mlp.W, mlp.b, y0, 1, cfg.lr, cfg.lam)
+    one = time.perf_counter() - t0
+    steps = int(max(2, min(cfg.n_steps, seconds / max(one, 1e-6))))
+    t_job = 0.0
+    t_meas = 0.0
+    for sp, y0 in zip(cfg.spaces, y0s):
+        t0 = time.perf_counter()
+        y, _, _, _ = fo.search(sp, mlp.W, mlp.b, y0, steps, cfg.lr, cfg.lam)
+        t1 = time.perf_counter()
+        fo.round_topk(sp, mlp.W, mlp.b, y.astype(np.float32), cfg.topk)
+        t2 = time.perf_counter()
+        t_meas += t2 - t0
+        t_job += (t1 - t0) * (cfg.n_seeds * cfg.n_steps) / (m * steps) + (t2 - t1) * cfg.n_seeds / m
+    rate = len(cfg.spaces) * cfg.n_seeds * cfg.n_steps / t_job
+    sample = (f"{m} seeds x {steps} Adam steps of each of the {len(cfg.spaces)} tasks (of {cfg.n_seeds} x "
+              f"{cfg.n_steps}) + round/top-k, extrapolated linearly per task; numpy float64")
+    return rate, threads, sample, t_meas
+
+
+def run_felix_tasks(args):
+    """C3 (ResNet-50, 21 tasks sharded by subgraph with LPT) / C4 (BERT-base, every task's seeds
+    sharded): every rank runs its shards concurrently (one stream per task); one bench step = every
+    task's full search + round/top-k; the per-task top-k lists are all-gathered once at the end."""
+    import torch
+    rank, world, local = dist_env()
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.cuda.current_device()
+    import felix_inputs as fi
+    import paper_conf_asplos_zhaosam24_b200 as fx
+    tasks = _tasks_module()
+
+    cfg = fi.config(args.config)
+    if args.seeds:
+        cfg.n_seeds = args.seeds
+    if args.search_steps:
+        cfg.n_steps = args.search_steps
+    mlp = fi.make_mlp(cfg.mlp_dims)
+    cm = fx.CostModel.from_weights(mlp, device=dev)
+    mode = tasks.config_mode(cfg.name)
+    mlp_flops = cm.mlp_flops_per_candidate_step()
+    costs = [tasks.est_cost(cfg.n_seeds, cfg.n_steps, mlp_flops, sp.nodes.shape[0]) for sp in cfg.spaces]
+    shards = tasks.plan(len(cfg.spaces), cfg.n_seeds, world, mode, costs)[rank]
+    runner = tasks.TaskRunner(cfg.spaces, shards, cm, device=dev)
+    T, k = cfg.n_steps, cfg.topk
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+
+    def bench_step(concurrent=True):
+        return runner.run(T, k, rng_seed=cfg.rng_seed, lr=cfg.lr, lam=cfg.lam, concurrent=concurrent)
+
+    def barrier():
+        if world > 1:
+            torch.distributed.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        bench_step()
+    barrier()
+    K = args.steps
+    clocks = ClockSampler(dev if "CUDA_VISIBLE_DEVICES" not in os.environ else
+                          int(os.environ["CUDA_VISIBLE_DEVICES"].split(",")[dev]))
+    clocks.start()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    barrier()
+    last = None
+    for i in range(K):
+        flush.zero_()
+        ev[i][0].record(stream)
+        last = bench_step()
+        ev[i][1].record(stream)
+    barrier()
+    clocks.stop()
+    t_ms = sum(a.elapsed_time(b) for a, b in ev)
+    t_max = t_ms
+    if world > 1:
+        tt = torch.tensor([t_ms], device=dev, dtype=torch.float64)
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        t_max = float(tt.item())
+    total = len(cfg.spaces) * cfg.n_seeds * T                 # candidate-steps of the whole job per bench step
+    value = total * K / (t_max * 1e-3)
+    local_cs = runner.cand_steps(T)
+    n_vars = [sp.n_vars for sp in cfg.spaces]
+    if world > 1:
+        merged = tasks.allgather_task_topk(last, len(cfg.spaces), k, n_vars, device=dev)
+    else:
+        merged = tasks.merge_task_records(tasks.pack_task_records(last, len(cfg.spaces), k, max(n_vars)),
+                                          len(cfg.spaces), k, n_vars)
+
+    # ---- roofline of the MLP kernel: the same shards searched one after another (no overlap, so the
+    # per-class CUDA-event durations are the kernels' own), algorithmic FLOPs / summed MLP time
+    for sp in runner.spaces.values():
+        sp.profile_reset()
+        sp.profile(True)
+    barrier()
+    bench_step(concurrent=False)
+    barrier()
+    gemm_ms = 0.0
+    dag_ms = 0.0
+    for sp in runner.spaces.values():
+        sp.profile(False)
+        pr = sp.profile_read()
+        gemm_ms += pr["mlp_gemm"][0]
+        dag_ms += pr["dag_fwd"][0] + pr["dag_rev_adam"][0]
+    mlp_flops_all = sum(mlp_flops * s.n * runner.spaces[s.task].n_statements * T for s in shards)
+    achieved = mlp_flops_all / (gemm_ms * 1e-3) / 1e12
+    peaks, peak_src = measured_peaks()
+    peak = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops")))
+
+    # ---- end to end through the public API: pinned host starting points in, losses + top-k out
+    e2e = None
+    if not args.no_e2e:
+        y_host = {s.task: torch.from_numpy(fi.make_y0(cfg.spaces[s.task], s.n, seed=1234 + s.task)).pin_memory()
+                  for s in shards}
+        y_dev = {s.task: torch.empty(tuple(y_host[s.task].shape), dtype=torch.float32, device=dev) for s in shards}
+        l_dev = {s.task: torch.empty(s.n, dtype=torch.float32, device=dev) for s in shards}
+        l_host = {s.task: torch.empty(s.n, dtype=torch.float32).pin_memory() for s in shards}
+
+        def e2e_step():
+            for s in shards:
+                y_dev[s.task].copy_(y_host[s.task], non_blocking=True)
+            out = runner.run(T, k, rng_seed=cfg.rng_seed, lr=cfg.lr, lam=cfg.lam, y0=y_dev, loss_out=l_dev)
+            for s in shards:
+                l_host[s.task].copy_(l_dev[s.task], non_blocking=True)
+            torch.cuda.current_stream().synchronize()
+            return out
+        e2e_step()
+        barrier()
+        t0 = time.perf_counter()
+        for _ in range(K):
+            e2e_step()
+        barrier()
+        t_e2e = time.perf_counter() - t0
+        if world > 1:
+            tt = torch.tensor([t_e2e], device=dev, dtype=torch.float64)
+            torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+            t_e2e = float(tt.item())
+        h2d = sum(cfg.spaces[s.task].n_vars * s.n * 4 for s in shards)
+        d2h = sum(s.n * 4 + k * (8 + 8 + 4 * cfg.spaces[s.task].n_vars) + 4 for s in shards)
+        e2e = {"value": total * K / t_e2e, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "timing": "host wall clock incl. pinned H2D of every shard's y0 and D2H of losses + top-k (rank 0's bytes)"}
+
+    if rank != 0:
+        if world > 1:
+            torch.distributed.destroy_process_group()
+        return 0
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        rate, threads, sample, _ = oracle_baseline_tasks(cfg, args.cpu_seconds)
+        cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample}
+    launches = sum(1 + T * 3 + (6 + len(cfg.mlp_dims) - 1) for _ in shards)
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
+        "ms_per_step": t_max / K, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "fp16x3 split (fp32-accurate) MLP, f64 DAG, f32 Adam", "data": "synthetic",
+        "config": {"workload": f"{cfg.name}: {len(cfg.spaces)} tasks x {cfg.n_seeds} seeds x {T} steps, "
+                               f"MLP {list(cfg.mlp_dims)}, top-{k} per task",
+                   "tasks": [sp.name for sp in cfg.spaces], "n_seeds_per_task": cfg.n_seeds, "n_steps": T,
+                   "parallelism": (f"dp{world}: subgraphs by LPT" if mode == "task" else f"dp{world}: seed shards of every task"),
+                   "rank0_tasks": [s.task for s in shards], "rank0_cand_steps_per_bench_step": local_cs,
+                   "concurrency": "one CUDA stream per task", "l2": "flushed (256 MB write) between timed iterations"},
+        "roofline": {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                     "traffic": None, "kernel": "MLP kernels of every task (tasks searched one after another for "
+                                                "this measurement), tcgen05 kind::f16 3-pass split",
+                     "executed_tflops": 3 * achieved,
+                     "peak_source": f"{peak_src} bf16_tflops_sustained (fp16 = bf16 rate)"},
+        "sequential_ms_per_bench_step": {"mlp": gemm_ms, "dag_fwd_rev_adam": dag_ms},
+        "gpu_launches": launches * K,
+        "clocks": clocks.summary(),
+        "top1_per_task": {cfg.spaces[t].name: (float(v[1][0]) if len(v[1]) else None) for t, v in merged.items()},
+    }
+    if e2e is not None:
+        line["e2e"] = e2e
+    if cpu is not None:
+        line["cpu_baseline"] = cpu
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+    return 0
+
+
+def run_reference_tasks(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return 0
+    import felix_inputs as fi
+    cfg = fi.config(args.config)
+    if args.seeds:
+        cfg.n_seeds = args.seeds
+    if args.search_steps:
+        cfg.n_steps = args.search_steps
+    W = max(args.warmup, 0)
+    K = max(args.steps, 1)
+    rates = []
+    for it in range(W + K):
+        secs = max(2.0, args.cpu_seconds / max(1, (W + K)))
+        rate, threads, sample, _ = oracle_baseline_tasks(cfg, secs)
+        if it >= W:
+            rates.append(rate)
+    value = statistics.median(rates)
+    total = len(cfg.spaces) * cfg.n_seeds * cfg.n_steps
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus, "steps": K,
+        "warmup": W, "ms_per_step": total / value * 1e3, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{cfg.name}: {len(cfg.spaces)} tasks x {cfg.n_seeds} seeds x {cfg.n_steps} steps, "
+                               f"MLP {list(cfg.mlp_dims)}, top-{cfg.topk} per task"},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
 def main():
     args = parse()
+    multi = args.config in ("C3", "C4")
     if args.impl == "reference":
-        return run_reference(args)
-    return run_felix(args)
+        return run_reference_tasks(args) if multi else run_reference(args)
+    return run_felix_tasks(args) if multi else run_felix(args)
 
 
 if __name__ == "__main__":

@@ -463,3 +463,71 @@ def test_search_quality_curves(fx):
     ref = fo.round_topk_history(sp, mlp.W, mlp.b, ys, 16)
     assert abs(res[2]["best"] - ref[2][0]) <= 1e-12 * abs(ref[2][0])            # FP64 scores: rel <= 1e-12
     assert abs(res[2]["top16"] - ref[2][15]) <= 1e-12 * abs(ref[2][15])
+
+
+@pytest.mark.parametrize("mode", ["seeds", "task"])
+@pytest.mark.timeout(600)
+def test_multitask_shards_equal_single_rank_and_oracle(fx, mode):
+    """C3/C4-style multi-task workloads (tasks.py): the shards a 2-rank plan gives each
+    rank, run on this GPU one rank at a time with one stream per task and merged as the all-gather
+    merges them, equal the 1-rank run per task; that run's top-k equals the oracle's round/top-k of the
+    GPU's final y of every task."""
+    from paper_conf_asplos_zhaosam24_b200 import tasks
+    mlp = fi.make_mlp(fi.DEFAULT_MLP)
+    cm = fx.CostModel.from_weights(mlp)
+    r50 = fi.resnet50_spaces()
+    spaces = [r50[0], r50[6], r50[-1], fi.bert_spaces()[1]]
+    n, T, k = 700, 6, 16
+    costs = [tasks.est_cost(n, T, cm.mlp_flops_per_candidate_step(), sp.nodes.shape[0]) for sp in spaces]
+    nv = [sp.n_vars for sp in spaces]
+    one = tasks.TaskRunner(spaces, tasks.plan(len(spaces), n, 1, mode, costs)[0], cm)
+    res1 = one.run(T, k, rng_seed=91)
+    rows = []
+    for r in range(2):
+        run = tasks.TaskRunner(spaces, tasks.plan(len(spaces), n, 2, mode, costs)[r], cm)
+        rows.append(tasks.pack_task_records(run.run(T, k, rng_seed=91), len(spaces), k, max(nv)))
+    merged = tasks.merge_task_records(np.concatenate(rows), len(spaces), k, nv)
+    for t in range(len(spaces)):
+        a, b = merged[t], res1[t]
+        assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1]) and np.array_equal(a[2], b[2])
+        yt = one._y[t].cpu().numpy()
+        _topk_equal(*b, *fo.round_topk(spaces[t], mlp.W, mlp.b, yt, k))
+
+
+ALL_TASKS = [("r50", i) for i in range(len(fi.resnet50_spaces()))] + [("bert", i) for i in range(len(fi.bert_spaces()))]
+
+
+@pytest.mark.parametrize("fam,i", ALL_TASKS)
+@pytest.mark.timeout(300)
+def test_every_c3_c4_task_eval_and_rounding_parity(fx, fam, i):
+    """Every ResNet-50 (C3) and BERT-base (C4) task: phi, cost, loss, gradient at y0 within the
+    north-star tolerances, and rounding / validity / top-k bit-exact, vs the oracle (n = 300: three
+    128-row tiles + a ragged tail)."""
+    sp = (fi.resnet50_spaces() if fam == "r50" else fi.bert_spaces())[i]
+    key = f"{fam}{i}"
+    if key not in _cache:
+        mlp = fi.make_mlp(fi.DEFAULT_MLP)
+        _cache[key] = (sp, mlp, 300, fx.Space(sp), fx.CostModel.from_weights(mlp))
+    sp, mlp, n, space, cm = _cache[key]
+    y0 = fi.make_y0(sp, n, seed=50 + i)
+    out = space.eval(cm, torch.from_numpy(y0).cuda(), lam=1.0)
+    ref = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
+    phi = out["phi"].cpu().numpy()
+    assert np.max(np.abs(phi - ref.phi) / np.maximum(np.abs(ref.phi), 1.0)) <= 1e-4
+    rms_c = np.sqrt(np.mean(ref.c ** 2))
+    assert np.max(np.abs(out["cost"].cpu().numpy() - ref.c)) <= 1e-4 * rms_c
+    rms_l = np.sqrt(np.mean(ref.loss ** 2))
+    assert np.max(np.abs(out["loss"].cpu().numpy() - ref.loss)) <= 1e-4 * rms_l
+    e_g = np.abs(out["g"].cpu().numpy() - ref.g) / np.maximum(np.abs(ref.g), 1.0)
+    assert np.max(e_g) <= 1e-4
+    g = out["grad"].cpu().numpy()
+    err = np.linalg.norm(g - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
+    bad = err > 1e-3
+    km = kink_margin(ref.zs)
+    assert not np.any(bad & (km >= 1e-4)) and (bad & (km < 1e-4)).mean() < 0.01
+    sched, valid = space.round(torch.from_numpy(y0).cuda())
+    rs = fo.round_schedules(sp, y0)
+    assert np.array_equal(sched.cpu().numpy(), rs)
+    assert np.array_equal(valid.cpu().numpy().astype(bool), fo.validate(sp, rs))
+    _topk_equal(*space.round_topk(cm, torch.from_numpy(y0).cuda(), 16),
+                *fo.round_topk(sp, mlp.W, mlp.b, y0, 16))
