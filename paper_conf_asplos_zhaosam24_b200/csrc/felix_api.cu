@@ -125,6 +125,7 @@ struct Plan {
   int chain_grid = 0;
   int chain_cs = 1;                        // 4: cluster chain (one 4-CTA cluster per row block, cluster barriers)
   DevBuf grid_bar;
+  DevBuf chain_flags;                      // dataflow chain: per (layer, row block) completion counters
   bool tile_ok = false;                    // model has the shape mlp_tile_kernel is specialised for
   TileParams tile{};                       // tile-local fused MLP (default when tile_ok)
   int tile_grid = 0;
@@ -648,6 +649,16 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
   p->chain_cs = mt <= sms / 4 ? 4 : 1;
   if (const char* e = std::getenv("FELIX_CHAIN_CS")) p->chain_cs = std::atoi(e) == 4 ? 4 : 1;
   if (p->chain_cs == 4) p->chain_grid = static_cast<int>(std::min<int64_t>(sms / 4, mt)) * 4;
+  // grid chain: per-row-block dataflow flags instead of grid barriers between layers (FELIX_CHAIN_FLAGS=0:
+  // grid barriers).  The epoch is the step counter the forward DAG kernel bumps before every chain launch.
+  p->chain_flags.alloc(static_cast<size_t>(p->chain.n_layers) * mt * CHAIN_FLAG_STRIDE * 4);
+  CUDA_OK(cudaMemset(p->chain_flags.p, 0, p->chain_flags.bytes));
+  {
+    const char* e = std::getenv("FELIX_CHAIN_FLAGS");
+    const bool flags = !(e && std::atoi(e) == 0);
+    p->chain.flags = (p->chain_cs == 1 && flags) ? p->chain_flags.as<unsigned int>() : nullptr;
+    p->chain.epoch = p->step_ctr.as<int>();
+  }
   // tile-local fused MLP: TenSet widths [K0p, 512, 256, 256, 1] only
   p->tile_ok = L == 4 && d[1] == tile::D1 && d[2] == tile::D2 && d[3] == tile::D3 && K0p <= 128 && K0p % 32 == 0;   // K0p/2 rows: multiple of 16
   if (p->tile_ok) {
@@ -1054,6 +1065,8 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     // the grid-barrier counter's target arithmetic is not wrap-safe (2^32 is not a multiple of the grid):
     // restart it every search (stream-ordered, no chain kernel in flight on this workspace)
     CUDA_OK(cudaMemsetAsync(pl->grid_bar.p, 0, pl->grid_bar.bytes, st));
+    // dataflow flags count up with step_ctr (reset together; 8 * steps stays far below 2^32)
+    CUDA_OK(cudaMemsetAsync(pl->chain_flags.p, 0, pl->chain_flags.bytes, st));
   }
   // varValuesHistory: a fresh pool for this search (worst case: every seed at every step is new)
   const int M = s->desc.n_vars;
@@ -1242,8 +1255,10 @@ felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int6
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   Plan& pl = *get_chunks(s, s->eval_chunks, m, n, 1).plans[0];
   CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
+  CUDA_OK(cudaMemsetAsync(pl.chain_flags.p, 0, pl.chain_flags.bytes, st));
+  CUDA_OK(cudaMemsetAsync(pl.step_ctr.p, 0, 4, st));     // the forward kernel makes it 1: the chain's epoch
   const felix_space::Module& mod = get_module(s, choose_P(n), choose_R(n));
-  run_forward_mlp(s, pl, mod, y, n, n, st, nullptr);
+  run_forward_mlp(s, pl, mod, y, n, n, st, pl.step_ctr.as<int>());
   int ni = static_cast<int>(n);
   void* dphi = pl.dphi.p;
   void* cpart = pl.c_part.p;

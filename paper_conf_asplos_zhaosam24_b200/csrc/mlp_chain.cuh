@@ -53,7 +53,24 @@ struct ChainParams {
   int m_tiles;
   unsigned int* grid_bar;              // monotonic arrival counter (never reset)
   unsigned long long* trace;           // debug: [grid][layers][8] globaltimer stamps (FELIX_CHAIN_TRACE)
+  // Dataflow mode (CS == 1, flags != nullptr): no grid barrier.  flags[(l * m_tiles + m) * 8] counts the
+  // layer-l tiles of row block m whose outputs are complete (release); a layer-(l+1) tile of row block m
+  // waits (acquire) until it reaches epoch * n_tiles_n(l).  Counters only grow during a search; *epoch
+  // is the launch's 1-based sequence number (the forward DAG kernel's step counter, or 1 after a reset).
+  unsigned int* flags;
+  const int* epoch;
 };
+
+constexpr int CHAIN_FLAG_STRIDE = 8;   // one 32-B sector per counter
+
+__device__ __forceinline__ void flag_wait(const unsigned int* f, unsigned int target) {
+  unsigned int cur;
+  while (true) {
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(cur) : "l"(f) : "memory");
+    if (static_cast<int>(cur - target) >= 0) break;
+    __nanosleep(32);
+  }
+}
 
 #ifdef FELIX_CHAIN_TRACE
 #define CHAIN_STAMP2(l, slot) do { unsigned long long t_; asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t_)); \
@@ -121,7 +138,9 @@ __device__ __forceinline__ void cluster_layer_barrier(uint64_t* bar, uint32_t ph
 template <int CS>
 __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __grid_constant__ ChainParams P) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-B alignment by offsetting the shared array itself (a round trip through uintptr_t would turn
+  // every smem access into a generic LD/ST)
+  uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* epi_base = smem + CHAIN_STAGES * CHAIN_STAGE_BYTES;   // [buf][hi | lo][128 x 64 fp16]
   float* s_bias = reinterpret_cast<float*>(epi_base + CHAIN_EPI_BYTES);   // [CHAIN_MAX_N] this layer's bias
   float* s_headw = s_bias + CHAIN_MAX_N;                                   // [CHAIN_MAX_N] head row (HEAD layer)
@@ -156,6 +175,9 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
   const uint32_t tmem_base = *tmem_slot;
   ptx::pdl_launch_dependents();
   ptx::pdl_wait();                                  // phi (layer-1 A operand) comes from the DAG kernel
+  const bool dataflow = CS == 1 && P.flags != nullptr;
+  const unsigned int epoch = dataflow ? static_cast<unsigned int>(*reinterpret_cast<const volatile int*>(P.epoch)) : 0u;
+  auto flag_of = [&](int l, int m) { return P.flags + (static_cast<size_t>(l) * P.m_tiles + m) * CHAIN_FLAG_STRIDE; };
 
   if (warp == 0) {
     if (lane == 0) {
@@ -163,7 +185,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       int it = 0;                                   // running k-block counter (ring position)
       for (int l = 0; l < P.n_layers; ++l) {
         const ChainLayer& L = P.layer[l];
-        if (l > 0) {
+        if (l > 0 && !dataflow) {
           // layer l reads layer l-1's outputs: wait until the epilogue warps of this CTA have
           // passed the grid barrier (they publish the layer count with st.release.cta)
           unsigned int g;
@@ -178,7 +200,29 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         ChainTiles<CS> tiles(L.n_tiles_n, P.m_tiles);
         for (int tile = tiles.first(); tile >= 0; tile = tiles.next(tile)) {
           const int m0 = (tile / L.n_tiles_n) * GEMM_BM, n0 = (tile % L.n_tiles_n) * L.bn;
-          for (int kb = 0; kb < nkb; ++kb, ++it) {
+          int kb0 = 0;
+          if (dataflow && l > 0) {
+            // weights do not depend on the previous layer: put the first ring stages' B loads in flight,
+            // then wait for this row block of layer l-1 and add the A loads
+            const int pre = nkb < CHAIN_STAGES ? nkb : CHAIN_STAGES;
+            for (int kb = 0; kb < pre; ++kb) {
+              const int s = (it + kb) % CHAIN_STAGES;
+              if (it + kb >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], (((it + kb) / CHAIN_STAGES) - 1) & 1);
+              ptx::mbar_arrive_expect_tx(&full_bar[s], tx);
+              ptx::tma_load_2d(b_hi(s), &L.b_hi, kb * GEMM_BK, n0, &full_bar[s]);
+              ptx::tma_load_2d(b_lo(s), &L.b_lo, kb * GEMM_BK, n0, &full_bar[s]);
+            }
+            flag_wait(flag_of(l - 1, m0 / GEMM_BM), epoch * static_cast<unsigned int>(P.layer[l - 1].n_tiles_n));
+            asm volatile("fence.proxy.async.global;" ::: "memory");
+            for (int kb = 0; kb < pre; ++kb) {
+              const int s = (it + kb) % CHAIN_STAGES;
+              ptx::tma_load_2d(a_hi(s), &L.a_hi, kb * GEMM_BK, m0, &full_bar[s]);
+              ptx::tma_load_2d(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, &full_bar[s]);
+            }
+            kb0 = pre;
+            it += pre;
+          }
+          for (int kb = kb0; kb < nkb; ++kb, ++it) {
             const int s = it % CHAIN_STAGES;
             if (it >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], ((it / CHAIN_STAGES) - 1) & 1);
             ptx::mbar_arrive_expect_tx(&full_bar[s], tx);
@@ -239,7 +283,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       const ChainLayer& L = P.layer[l];
       // per-layer fields in registers once: read through the dynamically indexed param block, the
       // compiler otherwise re-fetches each pointer (LDC) before every element access
-      const int epi = L.epi, bn = L.bn, ntn = L.n_tiles_n, ntiles = L.n_tiles;
+      const int epi = L.epi, bn = L.bn, ntn = L.n_tiles_n;
       const int aM = L.args.M, aN = L.args.N, n_valid = L.args.n_valid, ld_f32 = L.args.ld_f32, ld_c = L.args.ld_c;
       const float* __restrict__ bias = L.args.bias;
       const float* __restrict__ head_w = L.args.head_w;
@@ -267,6 +311,12 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         const bool row_ok = row < aM;
         // this thread's mask words for the tile (<= 2 chunks of 64 columns), requested before the wait
         uint32_t mwords[CHAIN_BN_MAX / 64] = {0u};
+        if (dataflow && epi == EPI_MASK) {
+          // the mask words come from an earlier layer of this row block (other CTAs): acquire the
+          // row block's flag of the previous layer first (the epilogue warps are idle in the mainloop)
+          if (etid == 0) flag_wait(flag_of(l - 1, m0 / GEMM_BM), epoch * static_cast<unsigned int>(P.layer[l - 1].n_tiles_n));
+          ptx::named_bar_sync(1, NEPI);
+        }
         if (epi == EPI_MASK && row_ok) {
 #pragma unroll
           for (int q64 = 0; q64 < CHAIN_BN_MAX / 64; ++q64)
@@ -378,10 +428,20 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
+        if (dataflow && l + 1 < P.n_layers) {
+          // this tile's outputs (TMA stores, mask words) complete and visible, then count it (release)
+          if (etid == 0) ptx::bulk_wait<0>();
+          __threadfence();
+          ptx::named_bar_sync(1, NEPI);
+          if (etid == 0) {
+            asm volatile("fence.proxy.async.global;" ::: "memory");
+            asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(flag_of(l, m0 / GEMM_BM)) : "memory");
+          }
+        }
       }
       // ---- layer end: all of this CTA's outputs complete + visible, then the grid barrier
       if (etid == 0) CHAIN_STAMP(l, 4);
-      if (l + 1 < P.n_layers) {
+      if (l + 1 < P.n_layers && !dataflow) {
         if (etid == 0) ptx::bulk_wait<0>();
         __threadfence();
         ptx::named_bar_sync(1, NEPI);

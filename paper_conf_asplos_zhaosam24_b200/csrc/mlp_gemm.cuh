@@ -96,7 +96,9 @@ mlp_gemm_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constan
                 GemmArgs args, int stages) {
   using Cfg = GemmCfg<BN>;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-B alignment by offsetting the shared array itself (a round trip through uintptr_t would turn
+  // every smem access into a generic LD/ST)
+  uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* full_bar  = reinterpret_cast<uint64_t*>(smem + stages * Cfg::STAGE_BYTES);
   uint64_t* empty_bar = full_bar + Cfg::MAX_STAGES;
   uint64_t* done_bar  = empty_bar + Cfg::MAX_STAGES;

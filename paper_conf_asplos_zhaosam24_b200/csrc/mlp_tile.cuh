@@ -189,7 +189,9 @@ template <int CG>
 __global__ void __launch_bounds__(tile::THREADS, 1) mlp_tile_kernel(const __grid_constant__ TileParams P) {
   using namespace tile;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-B alignment by offsetting the shared array itself (a round trip through uintptr_t would turn
+  // every smem access into a generic LD/ST)
+  uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* R0 = smem;                                  // 4 chunks: phi0 phi1 H0 H1 | delta2_0..3
   uint8_t* RD1 = R0 + R0_BYTES;                        // delta1 chunk
   uint8_t* RING_BASE = RD1 + CHUNK_BYTES;

@@ -44,10 +44,15 @@ int main(int argc, char** argv) {
   int grid = std::min(148, mt * 512 / bnA);
   P.trace = (unsigned long long*)dz((size_t)grid * CHAIN_MAX_LAYERS * 8 * 8 * 2);
   const int CS = argc > 4 ? atoi(argv[4]) : 1;
+  const int FLAGS = argc > 5 ? atoi(argv[5]) : 0;       // 1: dataflow flags (CS == 1)
+  unsigned int* flags = (unsigned int*)dz((size_t)6 * mt * CHAIN_FLAG_STRIDE * 4);
+  int one = 1; int* ep = (int*)dz(4); cudaMemcpy(ep, &one, 4, cudaMemcpyHostToDevice);
+  P.flags = FLAGS ? flags : nullptr; P.epoch = ep;
   if (CS == 4) grid = std::min(148 / 4, mt) * 4;
   cudaFuncSetAttribute(mlp_chain_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES);
   cudaFuncSetAttribute(mlp_chain_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES);
   auto launch = [&]() {
+    if (FLAGS) cudaMemsetAsync(flags, 0, (size_t)6 * mt * CHAIN_FLAG_STRIDE * 4);
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension; at[0].val.clusterDim.x = CS; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
     cudaLaunchConfig_t cfg{}; cfg.gridDim = dim3(grid); cfg.blockDim = dim3(CHAIN_THREADS); cfg.dynamicSmemBytes = CHAIN_SMEM_BYTES;
@@ -60,7 +65,7 @@ int main(int argc, char** argv) {
   for (int it = 0; it < 10; ++it) launch();
   cudaEventRecord(e1); cudaEventSynchronize(e1);
   float ms; cudaEventElapsedTime(&ms, e0, e1);
-  printf("CS=%d M=%d grid=%d bnA=%d bnB=%d: %.2f us per chain launch (err=%s)\n", CS, M, grid, bnA, bnB, ms * 100, cudaGetErrorString(cudaGetLastError()));
+  printf("FLAGS=%d CS=%d M=%d grid=%d bnA=%d bnB=%d: %.2f us per chain launch (err=%s)\n", FLAGS, CS, M, grid, bnA, bnB, ms * 100, cudaGetErrorString(cudaGetLastError()));
   std::vector<unsigned long long> h((size_t)grid * CHAIN_MAX_LAYERS * 8), h2((size_t)grid * CHAIN_MAX_LAYERS * 8);
   cudaMemcpy(h.data(), P.trace, h.size() * 8, cudaMemcpyDeviceToHost);
   cudaMemcpy(h2.data(), P.trace + h.size(), h2.size() * 8, cudaMemcpyDeviceToHost);
