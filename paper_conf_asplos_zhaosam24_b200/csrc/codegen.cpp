@@ -59,6 +59,11 @@ __device__ __forceinline__ double f_rcp(double b) {
   return (r0 == 0.0 || isinf(r0)) ? r0 : r;
 }
 __device__ __forceinline__ double f_div(double a, double b) { return a * f_rcp(b); }
+__device__ __forceinline__ void cp_async4(float* dst, const float* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"((unsigned)__cvta_generic_to_shared(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 __device__ __forceinline__ double f_sqrt(double x) {
   double y; asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
   y = y * fma(-0.5 * x, y * y, 1.5);
@@ -545,15 +550,18 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  for (int e = tid; e < NV * 32; e += PG * 32) { const int j = e >> 5, l = e & 31; const int cl = c0 + l; const float yy = yin[(size_t)j * ldy + (cl < n ? cl : n - 1)]; sy[e] = yy; sx[e] = exp((double)yy); }\n"
     << "  __syncthreads();\n"
     << "  constexpr int NJ = (NV + PG - 1) / PG;   // vars handled by this thread: j = wq + PG * jj\n"
-    << "  float mreg[NJ], vreg[NJ];\n"
-    << "#pragma unroll\n"
-    << "  for (int jj = 0; jj < NJ; ++jj) {\n"
-    << "    const int j = wq + PG * jj;\n"
-    << "    mreg[jj] = 0.f; vreg[jj] = 0.f;\n"
-    << "    if (!EVAL && j < NV) { mreg[jj] = mv[(size_t)j * n + cc]; vreg[jj] = vv[(size_t)j * n + cc]; }\n"
-    << "  }\n"
-    << "  float cst = head_b * NS;   // segment sum over statements: every statement's MLP adds its head bias\n"
-    << "  if (wq == 0) for (int s = 0; s < NS; ++s) for (int t = 0; t < n_head_tiles; ++t) cst += c_part[(size_t)t * ld_c + (size_t)s * n + cc];\n"
+    // Adam state and the head partials go to shared memory with cp.async (no registers held across the
+    // DAG, latency hidden behind it); consumed after the cone groups finish
+    << "  constexpr int HTMAX = 32;\n"
+    << "  __shared__ float smv_all[NREP][2 * NV * 32];\n"
+    << "  __shared__ float scp_all[NREP][HTMAX * 32];\n"
+    << "  float* smv = smv_all[rep];\n"
+    << "  float* scp = scp_all[rep];\n"
+    << "  const int nht_all = NS * n_head_tiles;\n"
+    << "  const bool cp_smem = nht_all <= HTMAX;\n"
+    << "  if (!EVAL) for (int e = tid; e < 2 * NV * 32; e += PG * 32) { const int h = e / (NV * 32), j = (e >> 5) % NV, l = e & 31; const int cl = c0 + l < n ? c0 + l : n - 1; cp_async4(&smv[e], (h ? vv : mv) + (size_t)j * n + cl); }\n"
+    << "  if (cp_smem) for (int e = tid; e < nht_all * 32; e += PG * 32) { const int i = e >> 5, l = e & 31; const int cl = c0 + l < n ? c0 + l : n - 1; cp_async4(&scp[e], c_part + (size_t)(i % n_head_tiles) * ld_c + (size_t)(i / n_head_tiles) * n + cl); }\n"
+    << "  cp_async_commit();\n"
     << "  const int tstep = EVAL ? 1 : *step_ctr;\n";
   for (int q = 0; q < P; ++q) {
     o << "  if (wq == " << q << ") {\n";
@@ -598,7 +606,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     o << "  }\n";
   }
   // automatic roots (warp 0) from the staged y
-  o << "  __syncthreads();\n  if (!EVAL) TSTAMP(1, 2);\n"
+  o << "  cp_async_wait_all();\n  __syncthreads();\n  if (!EVAL) TSTAMP(1, 2);\n"
     << "  if (wq == 0) {\n";
   for (int j = 0; j < M; ++j) o << "    const double y" << j << " = (double)sy[" << j << " * 32 + lane];\n";
   for (size_t q = 0; q < autos.size(); ++q) {
@@ -609,6 +617,9 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
   // cost + loss (warp 0); the loss is parked in spen[PG-1 .. ] row 0 after the sum
   o << "  __shared__ float sloss_all[NREP][32];\n  float* sloss = sloss_all[rep];\n"
     << "  if (wq == 0) {\n"
+    << "    float cst = head_b * NS;   // segment sum over statements: every statement's MLP adds its head bias\n"
+    << "    if (cp_smem) for (int i = 0; i < nht_all; ++i) cst += scp[i * 32 + lane];\n"
+    << "    else for (int s = 0; s < NS; ++s) for (int t = 0; t < n_head_tiles; ++t) cst += c_part[(size_t)t * ld_c + (size_t)s * n + cc];\n"
     << "    double pen = 0.0;\n"
     << "    for (int q = 0; q < PG; ++q) pen += spen[q * 32 + lane];\n"
     << "    for (int r = 0; r < NRA; ++r) { const double p = spa[r * 32 + lane]; pen += p * p; }\n"
@@ -651,7 +662,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "        if (j >= NV) break;\n"
     << "        const float gy = sgrad[j][lane];\n"
     << "        const size_t o_ = (size_t)j * n + c;\n"
-    << "        float m = mreg[jj], v = vreg[jj];\n"
+    << "        float m = smv[j * 32 + lane], v = smv[(NV + j) * 32 + lane];\n"
     << "        m = b1 * m + (1.f - b1) * gy; v = b2 * v + (1.f - b2) * gy * gy;\n"
     << "        mv[o_] = m; vv[o_] = v; yv[(size_t)j * ldy + c] = sy[j * 32 + lane] - step * m / (sqrtf(v) * rb + eps);\n"
     << "      }\n"

@@ -32,7 +32,10 @@ constexpr int CHAIN_EPI_BUFS = CHAIN_STAGES >= 3 ? 1 : 2;   // epilogue staging 
 constexpr int CHAIN_THREADS = 320;
 constexpr int CHAIN_EPI_WARPS = 8;
 constexpr int CHAIN_A_BYTES = GEMM_BM * GEMM_BK * 2;                 // 16 KB (one of hi / lo)
-constexpr int CHAIN_B_BYTES = CHAIN_BN_MAX * GEMM_BK * 2;            // 16 KB
+#ifndef FELIX_CHAIN_STAGE_BN
+#define FELIX_CHAIN_STAGE_BN CHAIN_BN_MAX
+#endif
+constexpr int CHAIN_B_BYTES = FELIX_CHAIN_STAGE_BN * GEMM_BK * 2;     // 16 KB (experiments: widest B tile a stage holds)
 constexpr int CHAIN_STAGE_BYTES = 2 * CHAIN_A_BYTES + 2 * CHAIN_B_BYTES;
 constexpr int CHAIN_EPI_BYTES = CHAIN_EPI_BUFS * 2 * GEMM_BM * 64 * 2;   // hi + lo staging of 64-col chunks
 constexpr int CHAIN_MAX_N = 1024;                                  // widest layer staged in smem (bias / head row)
