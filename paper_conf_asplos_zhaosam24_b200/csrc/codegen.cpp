@@ -391,6 +391,8 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
   // feature k -> (statement, index within the statement's vector)
   auto fs = [&](int k) { return k / K0; };
   auto fk = [&](int k) { return k % K0; };
+  // timing experiment only (FELIX_CPBX=1, wrong results): every warp of a block runs the same cone
+  o << "#define CONE_OF_WARP " << (std::getenv("FELIX_CPBX") ? "((int)(blockIdx.x % PG))" : "wq") << "\n";
   o << kPrelude;
 
   if (trace)
@@ -483,7 +485,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  for (int k = tid; k < NS * 32 * (K0P + 1); k += PG * 32) (&sphi[0][0][0])[k] = 0.f;\n"
     << "  __syncthreads();\n";
   for (int q = 0; q < P; ++q) {
-    o << "  if (wq == " << q << ") {\n";
+    o << "  if (CONE_OF_WARP == " << q << ") {\n";
     if (q == 0)
       for (int k = 0; k < K; ++k)
         if (!g.depvar[d.froots[k]]) {
@@ -564,7 +566,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  cp_async_commit();\n"
     << "  const int tstep = EVAL ? 1 : *step_ctr;\n";
   for (int q = 0; q < P; ++q) {
-    o << "  if (wq == " << q << ") {\n";
+    o << "  if (CONE_OF_WARP == " << q << ") {\n";
     if (q == 0) {
       o << "    if (EVAL && o_phi && live) {\n";
       for (int k = 0; k < K; ++k)

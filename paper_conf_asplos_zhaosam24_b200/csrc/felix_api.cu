@@ -627,7 +627,13 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
     L.epi = g.epi;
     const int N = g.args.N;
     int bn = g.bn;
-    if (g.epi == EPI_F32T) bn = g.bn;                                   // K0p (<= 128 required)
+    if (g.epi == EPI_F32T) {
+      // dL/dphi (K = d1 = 512, N = K0p): its A row block is the largest operand a CTA ingests, and with
+      // one N tile only mt CTAs work; 32-wide N tiles spread it over 3x the CTAs while they fit in one wave
+      bn = g.bn;                                                          // K0p (<= 128 required)
+      if (N % 32 == 0 && mt * (N / 32) <= sms) bn = 32;
+      if (const char* e = std::getenv("FELIX_DPHI_BN")) { const int v = std::atoi(e); if (v > 0 && N % v == 0 && v % 16 == 0) bn = v; }
+    }
     else bn = (N % 128 == 0 && mt * (N / 128) >= sms * 2 / 3) ? 128 : 64;
     if (bn > CHAIN_BN_MAX) FELIX_THROW(FELIX_E_UNSUPPORTED, "chain tile N > 128");
     L.bn = bn;
@@ -641,12 +647,11 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
     max_tiles = std::max(max_tiles, L.n_tiles);
   }
   p->chain_grid = std::min(sms, max_tiles);
-  // Cluster chain (one 4-CTA cluster per row block, cluster barriers) when every row block gets its own
-  // cluster: same speed as the grid chain at C2 (47.3 vs 47.1 us; the per-layer cost is the L2 round trip
-  // of the activations, not the barrier) but it only needs each cluster co-scheduled, so concurrent
-  // searches on different streams cannot deadlock.  Above 37 row blocks the grid chain is faster
-  // (n=8192: 64 vs 90 us) and is launched cooperatively (all CTAs gang-scheduled).  FELIX_CHAIN_CS=1|4.
-  p->chain_cs = mt <= sms / 4 ? 4 : 1;
+  // Grid chain with per-row-block dataflow flags (cooperative launch: every CTA resident) by default: at C2
+  // 44.2 us per Adam step vs 45.7 us for the cluster chain (one 4-CTA cluster per row block, cluster
+  // barriers), and faster above 37 row blocks (n=8192: 56 vs 90 us).  FELIX_CHAIN_CS=4 selects the
+  // cluster chain.
+  p->chain_cs = 1;
   if (const char* e = std::getenv("FELIX_CHAIN_CS")) p->chain_cs = std::atoi(e) == 4 ? 4 : 1;
   if (p->chain_cs == 4) p->chain_grid = static_cast<int>(std::min<int64_t>(sms / 4, mt)) * 4;
   // grid chain: per-row-block dataflow flags instead of grid barriers between layers (FELIX_CHAIN_FLAGS=0:

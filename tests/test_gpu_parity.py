@@ -310,10 +310,11 @@ def test_shape_errors(fx):
     del bad
 
 
-@pytest.mark.parametrize("mode,cg", [("chain", "1"), ("chain-cluster", "1"), ("layers", "1"), ("tile", "2")])
+@pytest.mark.parametrize("mode,cg", [("chain", "1"), ("chain-cluster", "1"), ("chain-barrier", "1"), ("layers", "1"),
+                                     ("tile", "2")])
 def test_mlp_execution_modes_agree(fx, mode, cg, monkeypatch):
-    """The tile-local fused MLP (1-SM and 2-SM cta_group::2 variants), the persistent chain and the
-    per-layer kernels compute the same split-fp16 products in the same K order: cost and gradient
+    """The tile-local fused MLP (1-SM and 2-SM cta_group::2 variants), the persistent chain (dataflow
+    flags, 4-CTA clusters, grid barriers) and the per-layer kernels compute the same split-fp16 products in the same K order: cost and gradient
     agree to fp32 summation-order noise (the head partial sums are grouped differently)."""
     sp = fi.c2_space()
     mlp = fi.make_mlp(fi.DEFAULT_MLP)
@@ -326,6 +327,7 @@ def test_mlp_execution_modes_agree(fx, mode, cg, monkeypatch):
     monkeypatch.setenv("FELIX_MLP", mode.split("-")[0])
     monkeypatch.setenv("FELIX_TILE_CG", cg)
     monkeypatch.setenv("FELIX_CHAIN_CS", "4" if mode == "chain-cluster" else "1")
+    monkeypatch.setenv("FELIX_CHAIN_FLAGS", "0" if mode == "chain-barrier" else "1")
     other = fx.Space(sp).eval(cm, y0, lam=1.0)
     for key in ("cost", "grad"):
         a, b = base[key].cpu().numpy(), other[key].cpu().numpy()

@@ -15,9 +15,10 @@ space.search(cm, y, 10, rng_seed=cfg.rng_seed, init_from_y=False)
 torch.cuda.synchronize()
 tr = space.debug_trace().astype(np.int64)
 nb = (n + 31) // 32
+T0 = tr[0, :nb, 1].min()          # common origin: the forward kernel's first block past griddepcontrol.wait
 for k, name in enumerate(["fwd", "rev"]):
     t = tr[k, :nb]
-    t0 = t[:, 0].min()
+    t0 = T0
     rel = (t - t0) / 1e3
     print(f"{name} P={os.environ.get('FELIX_P','auto')} n={n}: start {rel[:,0].min():.2f}..{rel[:,0].max():.2f} | after-wait {rel[:,1].min():.2f}..{rel[:,1].max():.2f} | "
           f"after-compute {rel[:,2].min():.2f}/{np.median(rel[:,2]):.2f}/{rel[:,2].max():.2f} | end {rel[:,3].min():.2f}/{np.median(rel[:,3]):.2f}/{rel[:,3].max():.2f} us")
