@@ -63,6 +63,15 @@ __device__ __forceinline__ void cp_async4(float* dst, const float* src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"((unsigned)__cvta_generic_to_shared(dst)), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+// ---- thread-block cluster helpers (cone-per-CTA kernels): rank, barrier, distributed shared memory
+__device__ __forceinline__ unsigned cl_rank() { unsigned r; asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r)); return r; }
+__device__ __forceinline__ void cl_sync() { asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory"); }
+__device__ __forceinline__ unsigned cl_map(const void* p, unsigned rank) {
+  unsigned r; asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"((unsigned)__cvta_generic_to_shared(p)), "r"(rank)); return r;
+}
+__device__ __forceinline__ double cl_ld_f64(const double* p, unsigned rank) { double v; asm volatile("ld.shared::cluster.f64 %0, [%1];" : "=d"(v) : "r"(cl_map(p, rank)) : "memory"); return v; }
+__device__ __forceinline__ void cl_st_f32(float* p, unsigned rank, float v) { asm volatile("st.shared::cluster.f32 [%0], %1;" :: "r"(cl_map(p, rank)), "f"(v) : "memory"); }
+__device__ __forceinline__ void cl_st_f64(double* p, unsigned rank, double v) { asm volatile("st.shared::cluster.f64 [%0], %1;" :: "r"(cl_map(p, rank)), "d"(v) : "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 __device__ __forceinline__ double f_sqrt(double x) {
   double y; asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
@@ -391,8 +400,19 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
   // feature k -> (statement, index within the statement's vector)
   auto fs = [&](int k) { return k / K0; };
   auto fk = [&](int k) { return k % K0; };
-  // timing experiment only (FELIX_CPBX=1, wrong results): every warp of a block runs the same cone
-  o << "#define CONE_OF_WARP " << (std::getenv("FELIX_CPBX") ? "((int)(blockIdx.x % PG))" : "wq") << "\n";
+  // NREPv == 0: cone-per-CTA kernels.  A cluster of PG CTAs (PG warps each) owns PG x 32 candidates; CTA q
+  // runs cone q for all of them (its warps share one cone's straight-line code and instruction fetches),
+  // warp w working on the 32 candidates CTA w owns: it reads their x from, and writes features / partial
+  // adjoints to, CTA w's shared memory (DSMEM).  Each CTA then finishes its own 32 rows as before.
+  const bool cpb = NREPv == 0;
+  if (cpb) NREPv = 1;
+  o << "#define CPB " << (cpb ? 1 : 0) << "\n";
+  o << "#define CONE_OF_WARP " << (cpb ? "cone" : "wq") << "\n";
+  // cone-phase access to the owner's staged x / features / partials (owner = warp index in CPB mode)
+  o << "#if CPB\n#define X_OWN(ptr) cl_ld_f64(&(ptr), (unsigned)wq)\n#define ST_OWN32(ptr, v) cl_st_f32(&(ptr), (unsigned)wq, (v))\n"
+       "#define ST_OWN64(ptr, v) cl_st_f64(&(ptr), (unsigned)wq, (v))\n#define BLOCK_SYNC() cl_sync()\n"
+       "#else\n#define X_OWN(ptr) (ptr)\n#define ST_OWN32(ptr, v) ((ptr) = (v))\n#define ST_OWN64(ptr, v) ((ptr) = (v))\n"
+       "#define BLOCK_SYNC() __syncthreads()\n#endif\n";
   o << kPrelude;
 
   if (trace)
@@ -474,8 +494,12 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  float (&sphi)[NS][32][K0P + 1] = sphi_all[rep];\n"
     << "  double (&sx)[NV][32] = sx_all[rep];\n"
     << "  const int lane = threadIdx.x & 31, wq = tid >> 5;\n"
-    << "  const int c0 = (blockIdx.x * NREP + rep) * 32, c = c0 + lane;\n"
-    << "  const int cc = c < n ? c : n - 1;\n"
+    << "#if CPB\n"
+    << "  const int cone = (int)cl_rank();\n"
+    << "  const int c0 = (blockIdx.x / PG) * (PG * 32) + cone * 32;   // the 32 rows this CTA owns\n"
+    << "#else\n"
+    << "  const int c0 = (blockIdx.x * NREP + rep) * 32;\n"
+    << "#endif\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
     << "  TSTAMP(0, 0);\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");   // y is the previous step's output\n"
@@ -483,7 +507,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  if (blockIdx.x == 0 && threadIdx.x == 0 && step_ctr) *step_ctr += 1;\n"
     << "  for (int e = tid; e < NV * 32; e += PG * 32) { const int l = e & 31; const int cl = c0 + l; sx[e >> 5][l] = exp((double)yv[(size_t)(e >> 5) * ldy + (cl < n ? cl : n - 1)]); }\n"
     << "  for (int k = tid; k < NS * 32 * (K0P + 1); k += PG * 32) (&sphi[0][0][0])[k] = 0.f;\n"
-    << "  __syncthreads();\n";
+    << "  BLOCK_SYNC();\n";
   for (int q = 0; q < P; ++q) {
     o << "  if (CONE_OF_WARP == " << q << ") {\n";
     if (q == 0)
@@ -492,16 +516,16 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
           // constant feature: value of its (var-free) cone, evaluated here
           o << "    {\n";
           g.emit_forward(g.cone({d.froots[k]}), 0, "x", "      ");
-          o << "      sphi[" << fs(k) << "][lane][" << fk(k) << "] = slogf_(v" << d.froots[k] << ");\n    }\n";
+          o << "      ST_OWN32(sphi[" << fs(k) << "][lane][" << fk(k) << "], slogf_(v" << d.froots[k] << "));\n    }\n";
         }
     const auto used = vars_in(fcone[q]);
     for (int j = 0; j < M; ++j)
-      if (used[j]) o << "    const double x" << j << " = sx[" << j << "][lane];\n";
+      if (used[j]) o << "    const double x" << j << " = X_OWN(sx[" << j << "][lane]);\n";
     g.emit_forward(fcone[q], 0, "x", "    ");
-    for (int k : part.feat[q]) o << "    sphi[" << fs(k) << "][lane][" << fk(k) << "] = slogf_(v" << d.froots[k] << ");\n";
+    for (int k : part.feat[q]) o << "    ST_OWN32(sphi[" << fs(k) << "][lane][" << fk(k) << "], slogf_(v" << d.froots[k] << "));\n";
     o << "  }\n";
   }
-  o << "  __syncthreads();\n  TSTAMP(0, 2);\n"
+  o << "  BLOCK_SYNC();\n  TSTAMP(0, 2);\n"
     << "  // rows c0 .. c0+31 of each statement are contiguous: K0P/8 uint4 per row for hi and for lo\n"
     << "#pragma unroll\n"
     << "  for (int it = 0; it < (NS * 32 * (K0P / 8) + PG * 32 - 1) / (PG * 32); ++it) {\n"
@@ -538,9 +562,18 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  double* spa = spen + PG * 32;                          // [NRA][32]\n"
     << "  float* sy = reinterpret_cast<float*>(spa + (NRA > 0 ? NRA : 1) * 32);   // [NV][32]\n"
     << "  const int lane = threadIdx.x & 31, wq = tid >> 5;\n"
+    << "#if CPB\n"
+    << "  const int cone = (int)cl_rank();\n"
+    << "  const int c0 = (blockIdx.x / PG) * (PG * 32) + cone * 32, c = c0 + lane;   // own rows (finish)\n"
+    << "  const int cw = (blockIdx.x / PG) * (PG * 32) + wq * 32 + lane;            // this warp's candidate (cone phase)\n"
+    << "#else\n"
     << "  const int c0 = (blockIdx.x * NREP + rep) * 32, c = c0 + lane;\n"
+    << "  const int cw = c;\n"
+    << "#endif\n"
     << "  const bool live = c < n;\n"
     << "  const int cc = live ? c : n - 1;\n"
+    << "  const bool livew = cw < n;\n"
+    << "  const int ccw = livew ? cw : n - 1;\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
     << "  if (!EVAL) TSTAMP(1, 0);\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n"
@@ -550,7 +583,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  __shared__ double sx_all[NREP][NV * 32];\n"
     << "  double* sx = sx_all[rep];\n"
     << "  for (int e = tid; e < NV * 32; e += PG * 32) { const int j = e >> 5, l = e & 31; const int cl = c0 + l; const float yy = yin[(size_t)j * ldy + (cl < n ? cl : n - 1)]; sy[e] = yy; sx[e] = exp((double)yy); }\n"
-    << "  __syncthreads();\n"
+    << "  BLOCK_SYNC();\n"
     << "  constexpr int NJ = (NV + PG - 1) / PG;   // vars handled by this thread: j = wq + PG * jj\n"
     // Adam state and the head partials go to shared memory with cp.async (no registers held across the
     // DAG, latency hidden behind it); consumed after the cone groups finish
@@ -568,28 +601,28 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
   for (int q = 0; q < P; ++q) {
     o << "  if (CONE_OF_WARP == " << q << ") {\n";
     if (q == 0) {
-      o << "    if (EVAL && o_phi && live) {\n";
+      o << "    if (EVAL && o_phi && livew) {\n";
       for (int k = 0; k < K; ++k)
         if (!g.depvar[d.froots[k]]) {
           o << "      {\n";
           g.emit_forward(g.cone({d.froots[k]}), 0, "x", "        ");
-          o << "        o_phi[(size_t)" << k << " * n + c] = slogf_(v" << d.froots[k] << ");\n      }\n";
+          o << "        o_phi[(size_t)" << k << " * n + cw] = slogf_(v" << d.froots[k] << ");\n      }\n";
         }
       o << "    }\n";
     }
     const auto used = vars_in(rcone[q]);
     for (int j = 0; j < M; ++j)
-      if (used[j]) o << "    const double x" << j << " = sx[" << j << " * 32 + lane];\n";
+      if (used[j]) o << "    const double x" << j << " = X_OWN(sx[" << j << " * 32 + lane]);\n";
     g.emit_forward(rcone[q], 0, "x", "    ");
     // user-root penalties of this group
     o << "    double pen = 0.0;\n";
     for (int r : part.cons[q]) {
       o << "    const double p" << r << " = fmax(v" << d.croots[r] << ", 0.0); pen += p" << r << " * p" << r << ";\n";
-      o << "    if (EVAL && o_g && live) o_g[(size_t)" << r << " * n + c] = (float)v" << d.croots[r] << ";\n";
+      o << "    if (EVAL && o_g && livew) o_g[(size_t)" << r << " * n + cw] = (float)v" << d.croots[r] << ";\n";
     }
-    o << "    spen[" << q << " * 32 + lane] = pen;\n";
-    o << "    if (EVAL && o_phi && live) {\n";
-    for (int k : part.feat[q]) o << "      o_phi[(size_t)" << k << " * n + c] = slogf_(v" << d.froots[k] << ");\n";
+    o << "    ST_OWN64(spen[" << q << " * 32 + lane], pen);\n";
+    o << "    if (EVAL && o_phi && livew) {\n";
+    for (int k : part.feat[q]) o << "      o_phi[(size_t)" << k << " * n + cw] = slogf_(v" << d.froots[k] << ");\n";
     o << "    }\n";
     const auto need = g.rev_live(rcone[q], rroots_g[q]);
     g.emit_adj_decls(need, "    ");
@@ -597,18 +630,18 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     for (int k : part.feat[q]) {
       const int r = d.froots[k];
       o << "    " << g.adj(r) << " += (ADJ_T)((double)dphi[(size_t)" << fk(k) << " * ld_dphi + (size_t)" << fs(k)
-        << " * n + cc] * slogp_(v" << r << "));\n";
+        << " * n + ccw] * slogp_(v" << r << "));\n";
     }
     for (int r : part.cons[q]) {
       const int nd = d.croots[r];
       if (g.depvar[nd]) o << "    " << g.adj(nd) << " += (ADJ_T)(2.0 * dlam * p" << r << ");\n";
     }
     g.emit_reverse_body(need, "    ");
-    for (int j = 0; j < M; ++j) o << "    spart[(" << q << " * NV + " << j << ") * 32 + lane] = (double)gx" << j << ";\n";
+    for (int j = 0; j < M; ++j) o << "    ST_OWN64(spart[(" << q << " * NV + " << j << ") * 32 + lane], (double)gx" << j << ");\n";
     o << "  }\n";
   }
   // automatic roots (warp 0) from the staged y
-  o << "  cp_async_wait_all();\n  __syncthreads();\n  if (!EVAL) TSTAMP(1, 2);\n"
+  o << "  cp_async_wait_all();\n  BLOCK_SYNC();\n  if (!EVAL) TSTAMP(1, 2);\n"
     << "  if (wq == 0) {\n";
   for (int j = 0; j < M; ++j) o << "    const double y" << j << " = (double)sy[" << j << " * 32 + lane];\n";
   for (size_t q = 0; q < autos.size(); ++q) {

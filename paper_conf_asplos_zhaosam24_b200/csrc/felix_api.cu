@@ -460,12 +460,22 @@ static felix_space::Module& get_module(felix_space* s, int P, int R = 1) {
 // SM's instruction fetches (ncu: 42 % of the reverse kernel's stall samples are no_instructions; its
 // SASS is 124 KB at C2).  Measured at C2: R=2 takes the reverse kernel from 16.9 to 15.3 us but the step
 // only +0.6 %; R=4 exceeds the static shared budget.  Default 1; FELIX_R overrides.
-static int choose_R(int64_t n) {
+// 0 = cone-per-CTA kernels (FELIX_CPB=1: clusters of P CTAs, DSMEM exchange), else replicas of the cone
+// groups per block (FELIX_R=1|2|4).  Cone-per-CTA is parity-green but measured slower at C2 (forward
+// 11.1 -> 12.8 us at P = 4, 26.9 us at P = 8; reverse 17.4 -> 16.8 / 20.9 us): the DSMEM round trips and
+// cluster barriers cost more than the shared instruction fetches save (a timing-only variant without the
+// exchange gave 8.6 / 12.8 us at P = 8), and 8-CTA clusters of one-CTA-per-SM kernels do not fit one wave.
+static bool use_cpb() {
+  const char* e = std::getenv("FELIX_CPB");
+  return e && std::atoi(e) == 1;
+}
+static int choose_R(int64_t n, int P) {
+  (void)n;
+  if (P > 1 && use_cpb()) return 0;
   if (const char* e = std::getenv("FELIX_R")) {
     const int r = std::atoi(e);
     if (r == 1 || r == 2 || r == 4) return r;
   }
-  (void)n;
   return 1;
 }
 
@@ -478,6 +488,13 @@ static int choose_P(int64_t n) {
   // measured on B200 (C2 space, per-class event timing): P=4 best at 4096 candidates, P=2 at 32768,
   // P=1 once the population alone fills the SMs
   int P = 1;
+  if (use_cpb()) {
+    // cone-per-CTA kernels (measured at C2, timing experiment with every warp of a CTA on one cone:
+    // forward 11.1 -> 8.6 us, reverse 17.5 -> 12.8 us at P = 8)
+    if (n <= 16384) P = 8;
+    else if (n <= 65536) P = 4;
+    return P;
+  }
   if (n <= 8192) P = 4;
   else if (n <= 65536) P = 2;
   return P;
@@ -496,6 +513,24 @@ static void launch_cfg(const void* f, dim3 grid, dim3 block, size_t smem, void**
 }
 static void launch_grouped(cudaKernel_t f, int P, int R, int64_t n, size_t smem, void** args, cudaStream_t st, bool pdl) {
   if (n <= 0) return;
+  if (R == 0) {
+    // cone-per-CTA kernels: clusters of P CTAs x P warps, one cluster per P x 32 candidates
+    cudaLaunchAttribute attrs[2];
+    attrs[0].id = cudaLaunchAttributeClusterDimension;
+    attrs[0].val.clusterDim.x = static_cast<unsigned>(P);
+    attrs[0].val.clusterDim.y = 1;
+    attrs[0].val.clusterDim.z = 1;
+    attrs[1] = g_pdl_attr;
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(static_cast<unsigned>((n + 32 * P - 1) / (32 * P) * P));
+    cfg.blockDim = dim3(32 * P);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cfg.attrs = attrs;
+    cfg.numAttrs = pdl ? 2 : 1;
+    CUDA_OK(cudaLaunchKernelExC(&cfg, reinterpret_cast<const void*>(f), args));
+    return;
+  }
   launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((n + 32 * R - 1) / (32 * R))), dim3(32 * P * R),
              smem, args, st, pdl);
 }
@@ -911,7 +946,10 @@ felix_status felix_codegen(const felix_var* vars, int32_t n_vars, const felix_sp
   const int K0 = n_features / n_statements;
   s->K0p = K0 <= 64 ? 64 : K0 <= 96 ? 96 : 128;
   CodegenInfo info;
-  const std::string code = generate_dag_module(s->desc, s->K0p, 8, 1, &info);
+  // FELIX_CODEGEN_P / FELIX_CODEGEN_R select the variant to inspect (default: P = 8 cone-per-CTA kernels)
+  const char* ep = std::getenv("FELIX_CODEGEN_P");
+  const char* er = std::getenv("FELIX_CODEGEN_R");
+  const std::string code = generate_dag_module(s->desc, s->K0p, ep ? std::atoi(ep) : 8, er ? std::atoi(er) : 0, &info);
   if (src_len) *src_len = static_cast<int64_t>(code.size());
   if (src && src_cap > 0) {
     const size_t nb = std::min<size_t>(code.size() + 1, static_cast<size_t>(src_cap));
@@ -1052,7 +1090,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
   const int64_t n = p->n_seeds;
   Chunks& ch = get_chunks(s, s->search_chunks, m, n, choose_chunks(n));
   const int nck = static_cast<int>(ch.plans.size());
-  const felix_space::Module& mod = get_module(s, choose_P(ch.cnt[0]), choose_R(ch.cnt[0]));
+  const felix_space::Module& mod = get_module(s, choose_P(ch.cnt[0]), choose_R(ch.cnt[0], choose_P(ch.cnt[0])));
   if (!p->init_from_y) {
     unsigned long long seed = p->rng_seed;
     long long ib = p->index_base;
@@ -1262,7 +1300,7 @@ felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int6
   CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
   CUDA_OK(cudaMemsetAsync(pl.chain_flags.p, 0, pl.chain_flags.bytes, st));
   CUDA_OK(cudaMemsetAsync(pl.step_ctr.p, 0, 4, st));     // the forward kernel makes it 1: the chain's epoch
-  const felix_space::Module& mod = get_module(s, choose_P(n), choose_R(n));
+  const felix_space::Module& mod = get_module(s, choose_P(n), choose_R(n, choose_P(n)));
   run_forward_mlp(s, pl, mod, y, n, n, st, pl.step_ctr.as<int>());
   int ni = static_cast<int>(n);
   void* dphi = pl.dphi.p;

@@ -533,3 +533,32 @@ def test_every_c3_c4_task_eval_and_rounding_parity(fx, fam, i):
     assert np.array_equal(valid.cpu().numpy().astype(bool), fo.validate(sp, rs))
     _topk_equal(*space.round_topk(cm, torch.from_numpy(y0).cuda(), 16),
                 *fo.round_topk(sp, mlp.W, mlp.b, y0, 16))
+
+
+@pytest.mark.parametrize("name", ["C2", "C2_2stmt", "bmm"])
+def test_cone_per_cta_kernels_parity(fx, name, monkeypatch):
+    """Opt-in cone-per-CTA DAG kernels (FELIX_CPB=1: clusters of P CTAs, features and partial adjoints
+    exchanged through distributed shared memory): same tolerances as the default kernels, and one Adam
+    step agrees with the default kernels to fp32 rounding."""
+    make, dims, n = CASES[name]
+    sp = make()
+    mlp = fi.make_mlp(dims)
+    cm = fx.CostModel.from_weights(mlp)
+    y0 = fi.make_y0(sp, n, seed=31)
+    monkeypatch.setenv("FELIX_CPB", "1")
+    space = fx.Space(sp)
+    out = {k: v.cpu().numpy() for k, v in space.eval(cm, torch.from_numpy(y0).cuda(), lam=1.0).items()}
+    ref = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
+    assert np.max(np.abs(out["phi"] - ref.phi) / np.maximum(np.abs(ref.phi), 1.0)) <= 1e-4
+    assert np.max(np.abs(out["g"] - ref.g) / np.maximum(np.abs(ref.g), 1.0)) <= 1e-4
+    for key, r in (("cost", ref.c), ("loss", ref.loss)):
+        assert np.max(np.abs(out[key] - r)) / np.sqrt(np.mean(r ** 2)) <= 1e-4, key
+    err = np.linalg.norm(out["grad"] - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
+    km = kink_margin(ref.zs)
+    assert not np.any((err > 1e-3) & (km >= 1e-4))
+    y1 = torch.from_numpy(y0).cuda()
+    space.search(cm, y1, 1, init_from_y=True)
+    monkeypatch.setenv("FELIX_CPB", "0")
+    y2 = torch.from_numpy(y0).cuda()
+    fx.Space(sp).search(cm, y2, 1, init_from_y=True)
+    assert torch.max(torch.abs(y1 - y2)).item() <= 1e-4 * (1 + torch.max(torch.abs(y2)).item())
