@@ -54,6 +54,8 @@ def parse():
     ap.add_argument("--two-statements", action="store_true",
                     help="C2 with TenSet-style per-statement features [reduction | epilogue], C = sum_s MLP "
                          "(SURVEY 8(f) row 3; not the headline)")
+    ap.add_argument("--unbatched", action="store_true",
+                    help="C3/C4: one felix_search per task on its own stream instead of felix_search_group")
     ap.add_argument("--history", action="store_true",
                     help="paper-faithful Alg. 1: round every visited point (varValuesHistory, l.13/17/20) "
                          "instead of the final point only (SURVEY 8(f) row 1; not the headline)")
@@ -493,8 +495,10 @@ def run_felix_tasks(args):
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
 
-    def bench_step(concurrent=True):
-        return runner.run(T, k, rng_seed=cfg.rng_seed, lr=cfg.lr, lam=cfg.lam, concurrent=concurrent)
+    batched = not args.unbatched
+
+    def bench_step():
+        return runner.run(T, k, rng_seed=cfg.rng_seed, lr=cfg.lr, lam=cfg.lam, batched=batched)
 
     def barrier():
         if world > 1:
@@ -534,13 +538,17 @@ def run_felix_tasks(args):
         merged = tasks.merge_task_records(tasks.pack_task_records(last, len(cfg.spaces), k, max(n_vars)),
                                           len(cfg.spaces), k, n_vars)
 
-    # ---- roofline of the MLP kernel: the same shards searched one after another (no overlap, so the
-    # per-class CUDA-event durations are the kernels' own), algorithmic FLOPs / summed MLP time
+    # ---- roofline of the MLP kernel: one profiled bench step (direct launches, CUDA events around every
+    # MLP launch: batched = the one group MLP pass per Adam step over all tasks' rows; unbatched = the
+    # shards searched one after another so the events time the kernels alone), algorithmic FLOPs / MLP time
     for sp in runner.spaces.values():
         sp.profile_reset()
         sp.profile(True)
     barrier()
-    bench_step(concurrent=False)
+    if batched:
+        bench_step()
+    else:
+        runner.run(T, k, rng_seed=cfg.rng_seed, lr=cfg.lr, lam=cfg.lam, batched=False, concurrent=False)
     barrier()
     gemm_ms = 0.0
     dag_ms = 0.0
@@ -566,7 +574,7 @@ def run_felix_tasks(args):
         def e2e_step():
             for s in shards:
                 y_dev[s.task].copy_(y_host[s.task], non_blocking=True)
-            out = runner.run(T, k, rng_seed=cfg.rng_seed, lr=cfg.lr, lam=cfg.lam, y0=y_dev, loss_out=l_dev)
+            out = runner.run(T, k, rng_seed=cfg.rng_seed, lr=cfg.lr, lam=cfg.lam, y0=y_dev, loss_out=l_dev, batched=batched)
             for s in shards:
                 l_host[s.task].copy_(l_dev[s.task], non_blocking=True)
             torch.cuda.current_stream().synchronize()
@@ -605,13 +613,17 @@ def run_felix_tasks(args):
                    "tasks": [sp.name for sp in cfg.spaces], "n_seeds_per_task": cfg.n_seeds, "n_steps": T,
                    "parallelism": (f"dp{world}: subgraphs by LPT" if mode == "task" else f"dp{world}: seed shards of every task"),
                    "rank0_tasks": [s.task for s in shards], "rank0_cand_steps_per_bench_step": local_cs,
-                   "concurrency": "one CUDA stream per task", "l2": "flushed (256 MB write) between timed iterations"},
+                   "batching": ("felix_search_group: per Adam step every task's DAG kernels on its own stream, one "
+                                "tensor-core MLP pass over all tasks' candidates" if batched else
+                                "one felix_search per task, one CUDA stream per task"),
+                   "l2": "flushed (256 MB write) between timed iterations"},
         "roofline": {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
-                     "traffic": None, "kernel": "MLP kernels of every task (tasks searched one after another for "
-                                                "this measurement), tcgen05 kind::f16 3-pass split",
+                     "traffic": None, "kernel": ("group MLP pass over all tasks' rows" if batched else
+                                                 "MLP kernels of every task (searched one after another for this "
+                                                 "measurement)") + ", tcgen05 kind::f16 3-pass split",
                      "executed_tflops": 3 * achieved,
                      "peak_source": f"{peak_src} bf16_tflops_sustained (fp16 = bf16 rate)"},
-        "sequential_ms_per_bench_step": {"mlp": gemm_ms, "dag_fwd_rev_adam": dag_ms},
+        "profiled_mlp_ms_per_bench_step": gemm_ms,
         "gpu_launches": launches * K,
         "clocks": clocks.summary(),
         "top1_per_task": {cfg.spaces[t].name: (float(v[1][0]) if len(v[1]) else None) for t, v in merged.items()},

@@ -178,6 +178,20 @@ typedef struct {
 FELIX_EXPORT felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search_params* p,
                           float* y, float* final_loss, void* stream);
 
+/* Several spaces (the tasks of one DNN, or the symbolic programs of one subgraph,
+ * Eq. 3) searched together with ONE cost model: every Adam step runs each space's DAG
+ * kernels on its own stream, then a single MLP pass (forward + input gradient) over the rows of all
+ * spaces (the cost model is shared, Eq. 4 sums independent per-candidate terms), then each space's
+ * reverse / Adam kernel.  Per space the result is what felix_search computes for it (same formulas,
+ * per-candidate arithmetic; with the same MLP kernel bit for bit).
+ * spaces[n_spaces], params[n_spaces], y[n_spaces] (device SoA [n_vars_i][n_seeds_i]), final_loss
+ * [n_spaces] (NULL, or per-space device [n_seeds_i] / NULL).  All spaces on the cost model's device;
+ * every params[i].n_steps equal; history must be 0 (FELIX_E_UNSUPPORTED otherwise).  The workspace
+ * is cached on spaces[0] for the same (spaces, n_seeds, cost model). */
+FELIX_EXPORT felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, felix_costmodel* m,
+                                             const felix_search_params* params, float* const* y,
+                                             float* const* final_loss, void* stream);
+
 /* Algorithm 1 lines 20-21 on the n relaxed points y (device SoA
  * [n_vars][n]): round every point (reading O10: per split component the divisor tuple nearest in
  * log space, ties to the lexicographically smallest; INT vars to the nearest integer), drop invalid

@@ -29,7 +29,7 @@ EXPORTED = ["felix_last_error", "felix_abi_version", "felix_space_create", "feli
             "felix_space_info", "felix_codegen", "felix_costmodel_load", "felix_costmodel_destroy",
             "felix_search", "felix_round_topk", "felix_eval", "felix_round", "felix_score",
             "felix_init_sample", "felix_profile_enable", "felix_profile_read", "felix_profile_reset",
-            "felix_debug_trace", "felix_history_topk", "felix_space_set_statements"]
+            "felix_debug_trace", "felix_history_topk", "felix_space_set_statements", "felix_search_group"]
 
 
 class FelixError(RuntimeError):
@@ -107,6 +107,29 @@ def _space_args(space):
     args = [vars_, len(space.vars), splits, len(space.splits), nodes.ctypes.data_as(_P), len(nodes),
             fr.ctypes.data_as(_P), len(fr), cr.ctypes.data_as(_P) if len(cr) else None, len(cr)]
     return args, keep
+
+
+def search_group(spaces: Sequence["Space"], cm: "CostModel", ys, n_steps: int, *, lr=0.05, beta1=0.9, beta2=0.999,
+                 eps=1e-8, lam=1.0, rng_seeds: Sequence[int] = None, index_bases: Sequence[int] = None,
+                 init_from_y: bool = True, final_losses=None, stream=None):
+    """felix_search_group: the spaces' searches in lock-step with one MLP pass per Adam step over the
+    candidates of all of them (shared cost model).  ys[i]: device fp32 [n_vars_i, n_i], updated in place."""
+    G = len(spaces)
+    if G == 0:
+        return ys
+    for sp, y in zip(spaces, ys):
+        sp._check_y(y)
+    seeds = list(rng_seeds) if rng_seeds is not None else [0] * G
+    bases = list(index_bases) if index_bases is not None else [0] * G
+    params = (_SearchParams * G)()
+    for i, y in enumerate(ys):
+        params[i] = _SearchParams(int(y.shape[1]), int(n_steps), lr, beta1, beta2, eps, lam, int(seeds[i]) & (2**64 - 1),
+                                  1 if init_from_y else 0, 0, int(bases[i]))
+    hs = (_P * G)(*[sp._h.value for sp in spaces])
+    yp = (_P * G)(*[_ptr(y) for y in ys])
+    lp = (_P * G)(*[_ptr(l) for l in final_losses]) if final_losses is not None else None
+    _check(_lib.felix_search_group(hs, G, cm._h, params, yp, lp, _P(_stream(stream))))
+    return ys
 
 
 def abi_version() -> int:

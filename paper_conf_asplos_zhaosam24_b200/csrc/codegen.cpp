@@ -738,11 +738,15 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
       comps[root_of[r]].push_back(j);
     }
   }
+  // one warp per candidate: lane L evaluates outer attempt a2 = base + L (a pure function of a2), the
+  // first accepted attempt in attempt order wins (ballot) and its y is broadcast: the same starting point
+  // as the serial rejection loop of the spec, with the serial chain of attempts replaced by 32 in flight
   o << "extern \"C\" __global__ void __launch_bounds__(128) felix_init(u64 seed, int n, long long index_base, float* __restrict__ yout) {\n"
-    << "  const int i = blockIdx.x * blockDim.x + threadIdx.x;\n  if (i >= n) return;\n"
+    << "  const int lane = threadIdx.x & 31;\n"
+    << "  const int i = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5);\n  if (i >= n) return;\n"
     << "  const u64 cand = (u64)(index_base + i);\n";
   for (int j = 0; j < M; ++j) o << "  double y" << j << " = 0.0;\n";
-  o << "  bool done = false;\n  for (int a2 = 0; a2 < 64 && !done; ++a2) {\n";
+  o << "  int win = -1;\n  for (int base = 0; base < 64 && win < 0; base += 32) {\n    const int a2 = base + lane;\n";
   for (const auto& comp : comps) {
     o << "    {\n      bool acc = false;\n";
     for (int j : comp) o << "      double c" << j << " = 0.0;\n";
@@ -774,18 +778,21 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     o << "    y" << j << " = __dadd_rn(" << lit(llo) << ", __dmul_rn(cuni(seed, cand, (u64)(a2 * 64), " << j << "ull), "
       << lit(lhi - llo) << "));\n";
   }
-  o << "    {\n";
+  o << "    bool ok = true;\n    {\n";
   for (int j = 0; j < M; ++j) o << "      const double x" << j << " = exp(y" << j << ");\n";
   std::vector<int> cr(d.croots.begin(), d.croots.end());
   g.emit_forward(g.cone(cr), 1, "x", "      ");
-  o << "      bool ok = true;\n";
   for (int r = 0; r < Ru; ++r) o << "      ok = ok && (v" << d.croots[r] << " <= 0.0);\n";
-  o << "      if (ok) done = true;\n    }\n  }\n  if (!done) {\n";
+  o << "    }\n"
+    << "    const unsigned acc_mask = __ballot_sync(0xffffffffu, ok);\n"
+    << "    if (acc_mask) {\n      const int src = __ffs(acc_mask) - 1;\n      win = base + src;\n";
+  for (int j = 0; j < M; ++j) o << "      y" << j << " = __shfl_sync(0xffffffffu, y" << j << ", src);\n";
+  o << "    }\n  }\n  if (win < 0) {\n";
   for (int j = 0; j < M; ++j)
     o << "    y" << j << " = " << (d.vars[j].kind == FELIX_VAR_INT ? lit(std::log((double)d.vars[j].lo)) : "0.0") << ";\n";
   o << "  }\n";
-  for (int j = 0; j < M; ++j) o << "  yout[(size_t)" << j << " * n + i] = (float)y" << j << ";\n";
-  o << "}\n";
+  for (int j = 0; j < M; ++j) o << "  if (lane == " << (j % 32) << ") yout[(size_t)" << j << " * n + i] = (float)y" << j << ";\n";
+  o << "}\n\n";
 
   if (info) {
     info->flops_fwd = flops_fwd;

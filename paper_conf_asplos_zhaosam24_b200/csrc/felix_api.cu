@@ -235,6 +235,23 @@ struct Chunks {
 
 struct ProfEvent { int cls; cudaEvent_t a, b; };
 
+// felix_search_group workspace: one MLP plan over the rows of every member space; per member its Adam
+// state and step counter; a one-step graph (fork: DAG forwards, join: MLP, fork: reverse/Adam, join)
+struct GroupCache {
+  const CostModel* cm = nullptr;
+  std::vector<void*> spaces;
+  std::vector<int64_t> n, row_off;
+  std::unique_ptr<Plan> plan;
+  std::vector<std::unique_ptr<DevBuf>> m, v, step_ctr;
+  std::vector<cudaStream_t> streams;
+  cudaGraphExec_t graph = nullptr;
+  std::vector<double> key;
+  ~GroupCache() {
+    if (graph) cudaGraphExecDestroy(graph);
+    for (auto st : streams) cudaStreamDestroy(st);
+  }
+};
+
 }  // namespace felix
 
 struct felix_space {
@@ -258,6 +275,7 @@ struct felix_space {
   int64_t flops_fwd = 0;
   // workspace caches (search: chunked; eval: one chunk) + scratch
   std::unique_ptr<felix::Chunks> search_chunks, eval_chunks;
+  std::unique_ptr<felix::GroupCache> group_cache;   // felix_search_group with this space first
   felix::DevBuf sched, valid, phi64, score, act64a, act64b, alive, rec_cand, rec_cnt, fin_cand, fin_cnt, o_idx, o_score, o_sched;
   // varValuesHistory (Alg. 1 l.13/17) of the last search run with history != 0: per-step rounded points,
   // each seed's previous schedule, the schedule hash set and the pool of distinct schedules
@@ -534,6 +552,11 @@ static void launch_grouped(cudaKernel_t f, int P, int R, int64_t n, size_t smem,
   launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((n + 32 * R - 1) / (32 * R))), dim3(32 * P * R),
              smem, args, st, pdl);
 }
+// felix_init: one warp per candidate (32 rejection attempts in flight)
+static void launch_warp_per_item(cudaKernel_t f, int64_t n, void** args, cudaStream_t st) {
+  if (n <= 0) return;
+  launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((n * 32 + 127) / 128)), dim3(128), 0, args, st, false);
+}
 static void launch_flat(cudaKernel_t f, int64_t n, void** args, cudaStream_t st) {
   if (n <= 0) return;
   launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((n + 127) / 128)), dim3(128), 0, args, st, false);
@@ -547,9 +570,8 @@ static int choose_bn(int64_t m_tiles, int N) {
   FELIX_THROW(FELIX_E_UNSUPPORTED, "hidden dim must be a multiple of 64");
 }
 
-static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int64_t n_cand) {
-  // the MLP sees one row per (statement, candidate): row = statement * n_cand + candidate
-  const int64_t n = n_cand * s->desc.n_statements;
+// MLP workspace for n MLP rows (and Adam state for n_vars x n_cand when n_cand > 0)
+static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, int64_t n, int n_vars, int64_t n_cand) {
   auto p = std::make_unique<Plan>();
   p->cm = cm;
   p->n = n;
@@ -574,8 +596,8 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
     }
   }
   p->dphi.alloc(static_cast<size_t>(K0p) * np * 4);
-  p->m.alloc(static_cast<size_t>(s->desc.n_vars) * n_cand * 4);
-  p->v.alloc(static_cast<size_t>(s->desc.n_vars) * n_cand * 4);
+  p->m.alloc(static_cast<size_t>(n_vars) * n_cand * 4);
+  p->v.alloc(static_cast<size_t>(n_vars) * n_cand * 4);
   p->step_ctr.alloc(16);
   const int64_t mt = np / 128;
   // forward GEMMs, layer l = 1..L-1 (W index l-1)
@@ -609,6 +631,7 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
       a.ld_c = static_cast<int>(np);
     } else {
       a.mask_out = p->mask[l]->as<uint32_t>();
+      a.ld_mask = static_cast<int>(np);
     }
     g.grid = dim3(static_cast<unsigned>(mt), N / g.bn);
     g.stages = std::min(gemm_max_stages(g.bn), (Kdim + GEMM_BK - 1) / GEMM_BK);
@@ -640,6 +663,7 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
       a.out_lo = p->act_lo[l - 1]->as<__half>();
       a.ld_out = N;
       a.mask_in = p->mask[l - 1]->as<uint32_t>();
+      a.ld_mask = static_cast<int>(np);
     }
     g.grid = dim3(static_cast<unsigned>(mt), N / g.bn);
     g.stages = std::min(gemm_max_stages(g.bn), (Kdim + GEMM_BK - 1) / GEMM_BK);
@@ -647,7 +671,7 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
   }
   // persistent chain: same layers, BN <= 128, one CTA per SM
   int sms = 148;
-  CUDA_OK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, s->device));
+  CUDA_OK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
   if (static_cast<int>(p->gemms.size()) > CHAIN_MAX_LAYERS) FELIX_THROW(FELIX_E_UNSUPPORTED, "too many MLP layers");
   p->chain.n_layers = static_cast<int>(p->gemms.size());
   p->chain.m_tiles = static_cast<int>(mt);
@@ -698,6 +722,19 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
     const bool flags = !(e && std::atoi(e) == 0);
     p->chain.flags = (p->chain_cs == 1 && flags) ? p->chain_flags.as<unsigned int>() : nullptr;
     p->chain.epoch = p->step_ctr.as<int>();
+    // own-chunk reuse (mlp_chain.cuh ChainLayer::reuse) where every CTA keeps its row block between two
+    // layers; FELIX_CHAIN_REUSE=0 disables
+    const char* er = std::getenv("FELIX_CHAIN_REUSE");
+    const bool reuse_ok = p->chain.flags != nullptr && CHAIN_EPI_BUFS == 2 && !(er && std::atoi(er) == 0);
+    for (int i = 0; i < p->chain.n_layers; ++i) {
+      ChainLayer& Li = p->chain.layer[i];
+      Li.reuse = 0;
+      if (!reuse_ok || i == 0) continue;
+      const ChainLayer& Lp = p->chain.layer[i - 1];
+      if (Lp.epi != EPI_F32T && Lp.n_tiles <= p->chain_grid && Li.n_tiles <= p->chain_grid &&
+          Lp.n_tiles_n == Li.n_tiles_n && Lp.bn % GEMM_BK == 0)
+        Li.reuse = 1;
+    }
   }
   // tile-local fused MLP: TenSet widths [K0p, 512, 256, 256, 1] only
   p->tile_ok = L == 4 && d[1] == tile::D1 && d[2] == tile::D2 && d[3] == tile::D3 && K0p <= 128 && K0p % 32 == 0;   // K0p/2 rows: multiple of 16
@@ -741,6 +778,11 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
   if (p->mode == MLP_TILE) p->n_head_tiles = 2;                           // one partial per column half
   else if (p->mode == MLP_LAYERS) p->n_head_tiles = p->gemms[L - 2].args.N / p->gemms[L - 2].bn;
   return p;
+}
+
+static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int64_t n_cand) {
+  // the MLP sees one row per (statement, candidate): row = statement * n_cand + candidate
+  return build_plan_rows(s->device, cm, n_cand * s->desc.n_statements, s->desc.n_vars, n_cand);
 }
 
 // number of concurrent chunks for a population of n (FELIX_CHUNKS overrides; tuned on B200)
@@ -1097,7 +1139,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     int ni = static_cast<int>(n);
     void* args[] = {&seed, &ni, &ib, &y};
     prof_mark(s, 3, st, true);
-    launch_flat(mod.f_init, n, args, st);
+    launch_warp_per_item(mod.f_init, n, args, st);
     prof_mark(s, 3, st, false);
     s->prof_launches[3] += 1;
   }
@@ -1287,6 +1329,178 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
   FELIX_API_END
 }
 
+felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, felix_costmodel* m,
+                                const felix_search_params* params, float* const* y, float* const* final_loss, void* stream) {
+  FELIX_API_BEGIN
+  if (!spaces || !params || !y || n_spaces <= 0 || n_spaces > 256) FELIX_THROW(FELIX_E_INVALID_ARG, "bad group arguments");
+  const int G = n_spaces;
+  int64_t rows = 0;
+  for (int i = 0; i < G; ++i) {
+    check_pair(spaces[i], m);
+    const felix_search_params& p = params[i];
+    if (p.n_steps != params[0].n_steps) FELIX_THROW(FELIX_E_INVALID_ARG, "group members need equal n_steps");
+    if (p.n_steps < 0) FELIX_THROW(FELIX_E_INVALID_ARG, "n_steps < 0");
+    if (p.history) FELIX_THROW(FELIX_E_UNSUPPORTED, "history is not supported in group searches");
+    if (p.n_seeds <= 0 || p.n_seeds > (int64_t(1) << 30)) FELIX_THROW(FELIX_E_INVALID_ARG, "n_seeds out of range");
+    if (!y[i]) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL y");
+    for (int j = 0; j < i; ++j) if (spaces[j] == spaces[i]) FELIX_THROW(FELIX_E_INVALID_ARG, "a space appears twice");
+    rows += p.n_seeds * spaces[i]->desc.n_statements;
+  }
+  if (rows > (int64_t(1) << 30)) FELIX_THROW(FELIX_E_INVALID_ARG, "too many rows");
+  felix_space* s0 = spaces[0];
+  DeviceGuard dg(s0->device);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const int T = params[0].n_steps;
+  // ---- workspace (cached on spaces[0])
+  std::unique_ptr<GroupCache>& slot = s0->group_cache;
+  bool fresh = !slot || slot->cm != m || static_cast<int>(slot->spaces.size()) != G;
+  for (int i = 0; !fresh && i < G; ++i)
+    fresh = slot->spaces[i] != spaces[i] || slot->n[i] != params[i].n_seeds;
+  if (fresh) {
+    slot.reset();
+    auto gc = std::make_unique<GroupCache>();
+    gc->cm = m;
+    int64_t off = 0;
+    for (int i = 0; i < G; ++i) {
+      gc->spaces.push_back(spaces[i]);
+      gc->n.push_back(params[i].n_seeds);
+      gc->row_off.push_back(off);
+      off += params[i].n_seeds * spaces[i]->desc.n_statements;
+      for (auto* vec : {&gc->m, &gc->v}) {
+        vec->push_back(std::make_unique<DevBuf>());
+        vec->back()->alloc(static_cast<size_t>(spaces[i]->desc.n_vars) * params[i].n_seeds * 4);
+      }
+      gc->step_ctr.push_back(std::make_unique<DevBuf>());
+      gc->step_ctr.back()->alloc(16);
+    }
+    gc->plan = build_plan_rows(s0->device, m, rows, 0, 0);
+    gc->plan->chain.epoch = gc->step_ctr[0]->as<int>();   // every member's forward bumps its counter once per step
+    for (int i = 0; i < G; ++i) {
+      cudaStream_t b;
+      CUDA_OK(cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking));
+      gc->streams.push_back(b);
+    }
+    slot = std::move(gc);
+  }
+  GroupCache& gc = *slot;
+  Plan& pl = *gc.plan;
+  // ---- per-search state: starting points, Adam state, counters, dataflow flags
+  std::vector<const felix_space::Module*> mods(G);
+  for (int i = 0; i < G; ++i) {
+    const int64_t n = params[i].n_seeds;
+    mods[i] = &get_module(spaces[i], choose_P(n), choose_R(n, choose_P(n)));
+    if (!params[i].init_from_y) {
+      unsigned long long seed = params[i].rng_seed;
+      long long ib = params[i].index_base;
+      int ni = static_cast<int>(n);
+      float* yi = y[i];
+      void* args[] = {&seed, &ni, &ib, &yi};
+      launch_warp_per_item(mods[i]->f_init, n, args, st);
+    }
+    CUDA_OK(cudaMemsetAsync(gc.m[i]->p, 0, gc.m[i]->bytes, st));
+    CUDA_OK(cudaMemsetAsync(gc.v[i]->p, 0, gc.v[i]->bytes, st));
+    CUDA_OK(cudaMemsetAsync(gc.step_ctr[i]->p, 0, 4, st));
+  }
+  CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
+  CUDA_OK(cudaMemsetAsync(pl.chain_flags.p, 0, pl.chain_flags.bytes, st));
+  if (T == 0) return FELIX_OK;
+  // ---- one Adam step of every member: fork (DAG forwards write their phi rows at their row offsets),
+  // join, one MLP pass over all rows, fork (reverse DAG + Adam per member on its dphi / head-partial
+  // columns), join.  Captured once as a graph; with profiling on (spaces[0]) launched directly with
+  // per-class events, the MLP as class 1.
+  std::vector<cudaEvent_t> ev(2 * G + 2);
+  for (auto& e : ev) CUDA_OK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  struct EvGuard { std::vector<cudaEvent_t>& v; ~EvGuard() { for (auto e : v) cudaEventDestroy(e); } } evg{ev};
+  const int K0p = m->K0p;
+  auto enqueue_step = [&](cudaStream_t main_st) {
+    CUDA_OK(cudaEventRecord(ev[0], main_st));
+    for (int i = 1; i < G; ++i) CUDA_OK(cudaStreamWaitEvent(gc.streams[i], ev[0], 0));
+    for (int i = 0; i < G; ++i) {
+      cudaStream_t si = i == 0 ? main_st : gc.streams[i];
+      int ni = static_cast<int>(params[i].n_seeds), ldi = ni;
+      const float* yi = y[i];
+      void* phi_hi = pl.phi_hi.as<uint16_t>() + gc.row_off[i] * K0p;
+      void* phi_lo = pl.phi_lo.as<uint16_t>() + gc.row_off[i] * K0p;
+      int* ctr = gc.step_ctr[i]->as<int>();
+      void* args[] = {&yi, &ni, &ldi, &phi_hi, &phi_lo, &ctr};
+      launch_grouped(mods[i]->f_fwd, mods[i]->P, mods[i]->R, params[i].n_seeds, 0, args, si, false);
+    }
+    for (int i = 1; i < G; ++i) {
+      CUDA_OK(cudaEventRecord(ev[1 + i], gc.streams[i]));
+      CUDA_OK(cudaStreamWaitEvent(main_st, ev[1 + i], 0));
+    }
+    prof_mark(s0, 1, main_st, true);
+    const MlpMode mode = static_cast<MlpMode>(pl.mode);
+    if (mode == MLP_TILE) launch_tile(pl, main_st);
+    else if (mode == MLP_CHAIN) launch_chain(pl, main_st);
+    else for (const auto& g : pl.gemms) launch_gemm(g, main_st);
+    prof_mark(s0, 1, main_st, false);
+    CUDA_OK(cudaEventRecord(ev[G + 1], main_st));
+    for (int i = 1; i < G; ++i) CUDA_OK(cudaStreamWaitEvent(gc.streams[i], ev[G + 1], 0));
+    for (int i = 0; i < G; ++i) {
+      cudaStream_t si = i == 0 ? main_st : gc.streams[i];
+      const felix_search_params& p = params[i];
+      float* yi = y[i];
+      int ni = static_cast<int>(p.n_seeds), ldy = ni;
+      void* dphi = pl.dphi.as<float>() + gc.row_off[i];
+      void* cpart = pl.c_part.as<float>() + gc.row_off[i];
+      int ld = static_cast<int>(pl.n_pad);
+      int nht = pl.n_head_tiles;
+      float hbv = m->head_b, lam = p.lambda, lr = p.lr, b1 = p.beta1, b2 = p.beta2, eps = p.eps;
+      void* mv = gc.m[i]->p;
+      void* vv = gc.v[i]->p;
+      int* ctr = gc.step_ctr[i]->as<int>();
+      float* lo = final_loss ? final_loss[i] : nullptr;
+      void* args[] = {&yi, &ni, &ldy, &dphi, &ld, &cpart, &nht, &ld, &hbv, &lam, &mv, &vv, &ctr, &lr, &b1, &b2, &eps, &lo};
+      launch_grouped(mods[i]->f_rev_adam, mods[i]->P, mods[i]->R, p.n_seeds, mods[i]->rev_smem, args, si, false);
+    }
+    for (int i = 1; i < G; ++i) {
+      CUDA_OK(cudaEventRecord(ev[G + 1 + i], gc.streams[i]));
+      CUDA_OK(cudaStreamWaitEvent(main_st, ev[G + 1 + i], 0));
+    }
+  };
+  if (s0->profiling) {
+    for (int t = 1; t <= T; ++t) {
+      if (t % 100000 == 0) CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
+      enqueue_step(st);
+      s0->prof_launches[1] += 1;
+    }
+    return FELIX_OK;
+  }
+  auto ptr = [](const void* q) { return static_cast<double>(reinterpret_cast<uintptr_t>(q)); };
+  std::vector<double> key;
+  for (int i = 0; i < G; ++i) {
+    const felix_search_params& p = params[i];
+    key.insert(key.end(), {static_cast<double>(mods[i]->P), static_cast<double>(mods[i]->R), ptr(y[i]),
+                           ptr(final_loss ? final_loss[i] : nullptr), p.lambda, p.lr, p.beta1, p.beta2, p.eps});
+  }
+  if (!gc.graph || gc.key != key) {
+    if (gc.graph) { cudaGraphExecDestroy(gc.graph); gc.graph = nullptr; }
+    cudaGraph_t graph = nullptr;
+    cudaStream_t cap;
+    CUDA_OK(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
+    struct StGuard { cudaStream_t s; ~StGuard() { cudaStreamDestroy(s); } } capg{cap};
+    CUDA_OK(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
+    try {
+      enqueue_step(cap);
+    } catch (...) {
+      cudaStreamEndCapture(cap, &graph);
+      if (graph) cudaGraphDestroy(graph);
+      throw;
+    }
+    CUDA_OK(cudaStreamEndCapture(cap, &graph));
+    cudaError_t ie = cudaGraphInstantiate(&gc.graph, graph, 0);
+    cudaGraphDestroy(graph);
+    CUDA_OK(ie);
+    gc.key = key;
+  }
+  for (int t = 1; t <= T; ++t) {
+    if (t % 100000 == 0) CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
+    CUDA_OK(cudaGraphLaunch(gc.graph, st));
+  }
+  FELIX_API_END
+}
+
 felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int64_t n, float lambda, float* phi,
                         float* g, float* cost, float* loss, float* grad, void* stream) {
   FELIX_API_BEGIN
@@ -1323,7 +1537,7 @@ felix_status felix_init_sample(felix_space* s, int64_t n, uint64_t rng_seed, int
   unsigned long long seed = rng_seed;
   long long ib = index_base;
   void* args[] = {&seed, &ni, &ib, &y};
-  launch_flat(get_module(s, 1).f_init, n, args, static_cast<cudaStream_t>(stream));
+  launch_warp_per_item(get_module(s, 1).f_init, n, args, static_cast<cudaStream_t>(stream));
   FELIX_API_END
 }
 
@@ -1350,6 +1564,16 @@ static void do_round(felix_space* s, const float* y, int64_t n, int32_t* sched, 
   }
 }
 
+// Entries per block in the first top-k phase: every block selects its chunk's best k distinct schedules
+// (k rounds of block argmax + dedup), the second phase merges the blocks' lists.  Enough blocks to run
+// the rounds in parallel (C2: 8 blocks of 512 instead of one of 4096), few enough that the single-block
+// merge stays short.
+static long long topk_chunk(long long n) {
+  long long c = (n + 63) / 64;
+  c = (c + 255) / 256 * 256;
+  return std::max(512LL, std::min(4096LL, c));
+}
+
 static void do_hard(felix_space* s, const int32_t* sched, int64_t n, double* phi64, uint8_t* valid, cudaStream_t st) {
   int ni = static_cast<int>(n);
   void* args[] = {&sched, &ni, &phi64, &valid};
@@ -1371,10 +1595,17 @@ static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, in
       const int K = m->dims[l], N = m->dims[l + 1];
       const bool last = l == L - 1;
       double* out = last ? score : bufs[l & 1];
-      const dim3 grid(static_cast<unsigned>((N + 31) / 32), static_cast<unsigned>((n + 31) / 32));
-      score_layer_kernel<<<grid, dim3(32, 8), 0, st>>>(
-          in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
-          last ? 0 : 1, last && st_i > 0 ? 1 : 0);
+      if (N >= 32) {   // register-blocked 64 x 64 tiles (bit-identical arithmetic)
+        const dim3 grid(static_cast<unsigned>((N + SCORE_T - 1) / SCORE_T), static_cast<unsigned>((n + SCORE_T - 1) / SCORE_T));
+        score_layer_rb_kernel<<<grid, 256, 0, st>>>(
+            in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
+            last ? 0 : 1, last && st_i > 0 ? 1 : 0);
+      } else {
+        const dim3 grid(static_cast<unsigned>((N + 31) / 32), static_cast<unsigned>((n + 31) / 32));
+        score_layer_kernel<<<grid, dim3(32, 8), 0, st>>>(
+            in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
+            last ? 0 : 1, last && st_i > 0 ? 1 : 0);
+      }
       CUDA_OK(cudaGetLastError());
       in = out;
       rs = N;
@@ -1433,7 +1664,7 @@ felix_status felix_round_topk(felix_space* s, felix_costmodel* m, const float* y
   do_round(s, y, n, s->sched.as<int32_t>(), st);
   do_hard(s, s->sched.as<int32_t>(), n, s->phi64.as<double>(), s->valid.as<uint8_t>(), st);
   do_score(s, m, s->phi64.as<double>(), n, s->score.as<double>(), st);
-  const long long chunk = 4096;
+  const long long chunk = topk_chunk(n);
   const long long nblk = (n + chunk - 1) / chunk;
   ensure(s->alive, static_cast<size_t>(std::max<long long>(n, nblk * k)));
   ensure(s->rec_cand, static_cast<size_t>(nblk) * k * 4);
@@ -1490,7 +1721,7 @@ felix_status felix_history_topk(felix_space* s, felix_costmodel* m, int32_t k, i
   ensure(s->score, static_cast<size_t>(n) * 8);
   do_hard(s, sched, n, s->phi64.as<double>(), s->valid.as<uint8_t>(), st);
   do_score(s, m, s->phi64.as<double>(), n, s->score.as<double>(), st);
-  const long long chunk = 4096;
+  const long long chunk = topk_chunk(n);
   const long long nblk = (n + chunk - 1) / chunk;
   ensure(s->alive, static_cast<size_t>(std::max<long long>(n, nblk * k)));
   ensure(s->rec_cand, static_cast<size_t>(nblk) * k * 4);

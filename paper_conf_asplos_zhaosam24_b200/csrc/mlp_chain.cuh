@@ -40,14 +40,22 @@ constexpr int CHAIN_STAGE_BYTES = 2 * CHAIN_A_BYTES + 2 * CHAIN_B_BYTES;
 constexpr int CHAIN_EPI_BYTES = CHAIN_EPI_BUFS * 2 * GEMM_BM * 64 * 2;   // hi + lo staging of 64-col chunks
 constexpr int CHAIN_MAX_N = 1024;                                  // widest layer staged in smem (bias / head row)
 constexpr int CHAIN_PARAM_BYTES = 2 * CHAIN_MAX_N * 4;
-constexpr int CHAIN_SMEM_BYTES = 1024 + CHAIN_STAGES * CHAIN_STAGE_BYTES + CHAIN_EPI_BYTES + CHAIN_PARAM_BYTES + 256;
+// ReLU mask words [buf][half][128 rows] and head partials [half][128 rows], staged for 1-D bulk copies so
+// every global write of a tile goes through the async proxy (one bulk_wait before the row-block flag)
+constexpr int CHAIN_AUX_BYTES = CHAIN_EPI_BUFS * 2 * GEMM_BM * 4 + 2 * GEMM_BM * 4;
+constexpr int CHAIN_SMEM_BYTES = 1024 + CHAIN_STAGES * CHAIN_STAGE_BYTES + CHAIN_EPI_BYTES + CHAIN_PARAM_BYTES + CHAIN_AUX_BYTES + 256;
 
 struct ChainLayer {
   CUtensorMap a_hi, a_lo, b_hi, b_lo, c_hi, c_lo;
   GemmArgs args;
   int epi, bn, n_tiles_n, n_tiles;     // tiles = m_tiles * n_tiles_n (n fastest)
   uint32_t idesc;
-  int _pad[3];
+  // reuse: this layer's A row block is the previous layer's output and every CTA keeps its row block from
+  // one layer to the next (one tile per CTA in both, same N-tile count): the CTA's own previous output
+  // chunks, still in its epilogue staging buffers in the A-operand layout (128-B swizzle, K-major), serve
+  // as those K blocks (no TMA load; no wait for other CTAs), issued first.
+  int reuse;
+  int _pad[2];
 };
 
 struct ChainParams {
@@ -147,13 +155,16 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
   uint8_t* epi_base = smem + CHAIN_STAGES * CHAIN_STAGE_BYTES;   // [buf][hi | lo][128 x 64 fp16]
   float* s_bias = reinterpret_cast<float*>(epi_base + CHAIN_EPI_BYTES);   // [CHAIN_MAX_N] this layer's bias
   float* s_headw = s_bias + CHAIN_MAX_N;                                   // [CHAIN_MAX_N] head row (HEAD layer)
-  uint64_t* full_bar = reinterpret_cast<uint64_t*>(epi_base + CHAIN_EPI_BYTES + CHAIN_PARAM_BYTES);
+  uint32_t* s_mask = reinterpret_cast<uint32_t*>(epi_base + CHAIN_EPI_BYTES + CHAIN_PARAM_BYTES);   // [EPI_BUFS][2][128]
+  float* s_cpart = reinterpret_cast<float*>(s_mask + CHAIN_EPI_BUFS * 2 * GEMM_BM);                  // [2][128]
+  uint64_t* full_bar = reinterpret_cast<uint64_t*>(epi_base + CHAIN_EPI_BYTES + CHAIN_PARAM_BYTES + CHAIN_AUX_BYTES);
   uint64_t* empty_bar = full_bar + CHAIN_STAGES;
   uint64_t* tfull = empty_bar + CHAIN_STAGES;      // [2] accumulator ready
   uint64_t* tempty = tfull + 2;                    // [2] accumulator drained
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
   uint32_t* gen_slot = tmem_slot + 1;              // layers completed grid-wide (producer handshake)
   uint64_t* cl_bar = tempty + 3;                   // cluster layer barrier (CS > 1), 8-byte aligned
+  uint64_t* own_bar = tempty + 4;                  // epilogue -> MMA: a tile's output chunks are staged
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned int G = gridDim.x;
@@ -167,6 +178,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
     for (int s = 0; s < CHAIN_STAGES; ++s) { ptx::mbar_init(&full_bar[s], 1); ptx::mbar_init(&empty_bar[s], 1); }
     for (int a = 0; a < 2; ++a) { ptx::mbar_init(&tfull[a], 1); ptx::mbar_init(&tempty[a], CHAIN_EPI_WARPS); }
     if (CS > 1) ptx::mbar_init(cl_bar, CS);
+    ptx::mbar_init(own_bar, 1);
     *gen_slot = 0;
     ptx::fence_barrier_init();
   }
@@ -204,6 +216,32 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         for (int tile = tiles.first(); tile >= 0; tile = tiles.next(tile)) {
           const int m0 = (tile / L.n_tiles_n) * GEMM_BM, n0 = (tile % L.n_tiles_n) * L.bn;
           int kb0 = 0;
+          if (dataflow && l > 0 && L.reuse) {
+            // own K blocks (B only) first, then the others (B, row-block flag once, A)
+            const ChainLayer& Lp = P.layer[l - 1];
+            const int own0 = (tile % Lp.n_tiles_n) * Lp.bn / GEMM_BK, nown = Lp.bn / GEMM_BK;
+            const uint32_t tx_b = 2 * (L.bn * GEMM_BK * 2);
+            bool flag_ok = false;
+            for (int i = 0; i < nkb; ++i, ++it) {
+              const int kb = i < nown ? own0 + i : (i - nown < own0 ? i - nown : i);
+              const bool own = i < nown;
+              const int s = it % CHAIN_STAGES;
+              if (it >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], ((it / CHAIN_STAGES) - 1) & 1);
+              ptx::mbar_arrive_expect_tx(&full_bar[s], own ? tx_b : tx);
+              ptx::tma_load_2d(b_hi(s), &L.b_hi, kb * GEMM_BK, n0, &full_bar[s]);
+              ptx::tma_load_2d(b_lo(s), &L.b_lo, kb * GEMM_BK, n0, &full_bar[s]);
+              if (!own) {
+                if (!flag_ok) {
+                  flag_wait(flag_of(l - 1, m0 / GEMM_BM), epoch * static_cast<unsigned int>(Lp.n_tiles_n));
+                  asm volatile("fence.proxy.async.global;" ::: "memory");
+                  flag_ok = true;
+                }
+                ptx::tma_load_2d(a_hi(s), &L.a_hi, kb * GEMM_BK, m0, &full_bar[s]);
+                ptx::tma_load_2d(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, &full_bar[s]);
+              }
+            }
+            continue;
+          }
           if (dataflow && l > 0) {
             // weights do not depend on the previous layer: put the first ring stages' B loads in flight,
             // then wait for this row block of layer l-1 and add the A loads
@@ -242,6 +280,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
     if (lane == 0) {
       // ------------------------------------------------------------ MMA issuer
       int it = 0, tcount = 0;
+      int staged_tiles = 0, chunk_count = 0, prev_chunk_base = 0;   // mirror of the epilogue's staging sequence
       for (int l = 0; l < P.n_layers; ++l) {
         const ChainLayer& L = P.layer[l];
         const int nkb = (L.args.K + GEMM_BK - 1) / GEMM_BK;
@@ -251,17 +290,32 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
           if (tcount >= 2) ptx::mbar_wait(&tempty[acc], ((tcount >> 1) - 1) & 1);
           ptx::tc_fence_after();
           const uint32_t d = tmem_base + acc * CHAIN_BN_MAX;
-          for (int kb = 0; kb < nkb; ++kb, ++it) {
+          const bool reuse = dataflow && l > 0 && L.reuse;
+          int own0 = 0, nown = 0;
+          if (reuse) {
+            const ChainLayer& Lp = P.layer[l - 1];
+            own0 = (tile % Lp.n_tiles_n) * Lp.bn / GEMM_BK;
+            nown = Lp.bn / GEMM_BK;
+            // the previous tile's chunks are staged and fenced for the async proxy
+            ptx::mbar_wait(own_bar, (staged_tiles - 1) & 1);
+          }
+          for (int i = 0; i < nkb; ++i, ++it) {
+            const int kb = !reuse ? i : (i < nown ? own0 + i : (i - nown < own0 ? i - nown : i));
             const int s = it % CHAIN_STAGES;
             ptx::mbar_wait(&full_bar[s], (it / CHAIN_STAGES) & 1);
-            if (kb == 0 && tcount == 0) CHAIN_STAMP(l, 1);
+            if (i == 0 && tcount == 0) CHAIN_STAMP(l, 1);
             ptx::tc_fence_after();
-            const uint32_t ah = ptx::smem_u32(a_hi(s)), al = ptx::smem_u32(a_lo(s));
+            uint32_t ah = ptx::smem_u32(a_hi(s)), al = ptx::smem_u32(a_lo(s));
+            if (reuse && i < nown) {
+              const uint8_t* eh = epi_base + ((prev_chunk_base + i) % CHAIN_EPI_BUFS) * (2 * GEMM_BM * 64 * 2);
+              ah = ptx::smem_u32(eh);
+              al = ptx::smem_u32(eh + GEMM_BM * 64 * 2);
+            }
             const uint32_t bh = ptx::smem_u32(b_hi(s)), bl = ptx::smem_u32(b_lo(s));
 #pragma unroll
             for (int kk = 0; kk < GEMM_BK / GEMM_UMMA_K; ++kk) {
               const uint32_t off = kk * GEMM_UMMA_K * 2;
-              const uint32_t acc0 = (kb | kk) != 0;
+              const uint32_t acc0 = (i | kk) != 0;
               ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(al + off), ptx::sdesc_k_sw128(bh + off), L.idesc, acc0);
               ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bl + off), L.idesc, 1u);
               ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bh + off), L.idesc, 1u);
@@ -270,6 +324,11 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
           }
           ptx::mma_commit(&tfull[acc]);
           CHAIN_STAMP(l, 2);
+          if (L.epi != EPI_F32T) {          // the epilogue will stage this tile's bn / 64 chunks
+            prev_chunk_base = chunk_count;
+            chunk_count += L.bn / 64;
+            ++staged_tiles;
+          }
         }
       }
     }
@@ -288,6 +347,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       // compiler otherwise re-fetches each pointer (LDC) before every element access
       const int epi = L.epi, bn = L.bn, ntn = L.n_tiles_n;
       const int aM = L.args.M, aN = L.args.N, n_valid = L.args.n_valid, ld_f32 = L.args.ld_f32, ld_c = L.args.ld_c;
+      const int ld_mask = L.args.ld_mask;
       const float* __restrict__ bias = L.args.bias;
       const float* __restrict__ head_w = L.args.head_w;
       uint32_t* __restrict__ mask_out = L.args.mask_out;
@@ -323,7 +383,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         if (epi == EPI_MASK && row_ok) {
 #pragma unroll
           for (int q64 = 0; q64 < CHAIN_BN_MAX / 64; ++q64)
-            if (q64 * 64 < bn) mwords[q64] = __ldcg(&mask_in[static_cast<size_t>(row) * (aN / 32) + (n0 + q64 * 64 + half * 32) / 32]);
+            if (q64 * 64 < bn) mwords[q64] = __ldcg(&mask_in[static_cast<size_t>((n0 + q64 * 64 + half * 32) / 32) * ld_mask + row]);
         }
         ptx::mbar_wait(&tfull[acc], (tcount >> 1) & 1);
         if (etid == 0 && tile == first_tile) CHAIN_STAMP(l, 3);
@@ -350,7 +410,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         } else {
           for (int c64 = 0; c64 < bn; c64 += 64) {
             // the staging buffer must be free: the TMA store that last used it finished reading
-            uint8_t* epi_hi = epi_base + (epi_count % CHAIN_EPI_BUFS) * (2 * GEMM_BM * 64 * 2);
+            const int ebuf = epi_count % CHAIN_EPI_BUFS;
+            uint8_t* epi_hi = epi_base + ebuf * (2 * GEMM_BM * 64 * 2);
             uint8_t* epi_lo = epi_hi + GEMM_BM * 64 * 2;
             ++epi_count;
             if (etid == 0) {
@@ -393,7 +454,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
                     v[i] = on ? -w : 0.f;        // delta_{L-1} = W_L^T (dL/dc = -1) (.) [Z > 0]
                   }
                 }
-                if (!head && row_ok) mask_out[static_cast<size_t>(row) * (aN / 32) + n / 32] = bits;
+                if (!head) s_mask[(ebuf * 2 + half) * GEMM_BM + r_tile] = bits;
               }
 #pragma unroll
               for (int qq = 0; qq < 4; ++qq) {
@@ -421,25 +482,39 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             if (etid == 0) {
               ptx::tma_store_2d(tm_c_hi, n0 + c64, m0, epi_hi);
               ptx::tma_store_2d(tm_c_lo, n0 + c64, m0, epi_lo);
+              if (epi == EPI_RELU) {   // the chunk's two mask-word columns (rows m0 .. m0+127; ld_mask >= padded rows)
+                ptx::bulk_s2g(mask_out + static_cast<size_t>((n0 + c64) / 32) * ld_mask + m0, s_mask + (ebuf * 2) * GEMM_BM, GEMM_BM * 4);
+                ptx::bulk_s2g(mask_out + static_cast<size_t>((n0 + c64) / 32 + 1) * ld_mask + m0, s_mask + (ebuf * 2 + 1) * GEMM_BM, GEMM_BM * 4);
+              }
               ptx::bulk_commit();
+              if (c64 + 64 >= bn) ptx::mbar_arrive(own_bar);   // all chunks of the tile staged (reuse, next layer)
             }
           }
         }
-        // head partial per (N tile, column half); the reverse kernel sums all 2 * N / bn partials
-        if (epi == EPI_HEAD && row_ok) c_part[static_cast<size_t>(2 * (n0 / bn) + half) * ld_c + row] = head_acc;
+        // head partial per (N tile, column half); the reverse kernel sums all 2 * N / bn partials.  Staged in
+        // shared memory and bulk-copied (rows m0 .. m0+127; c_part has padded rows)
+        if (epi == EPI_HEAD) {
+          if (etid == 0) ptx::bulk_wait_read<0>();          // the previous tile's copy has read s_cpart
+          ptx::named_bar_sync(1, NEPI);
+          s_cpart[half * GEMM_BM + r_tile] = head_acc;
+          ptx::fence_proxy_async_smem();
+          ptx::named_bar_sync(1, NEPI);
+          if (etid == 0) {
+            ptx::bulk_s2g(c_part + static_cast<size_t>(2 * (n0 / bn)) * ld_c + m0, s_cpart, GEMM_BM * 4);
+            ptx::bulk_s2g(c_part + static_cast<size_t>(2 * (n0 / bn) + 1) * ld_c + m0, s_cpart + GEMM_BM, GEMM_BM * 4);
+            ptx::bulk_commit();
+          }
+        }
         // accumulator drained: let the MMA warp reuse it
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
-        if (dataflow && l + 1 < P.n_layers) {
-          // this tile's outputs (TMA stores, mask words) complete and visible, then count it (release)
-          if (etid == 0) ptx::bulk_wait<0>();
-          __threadfence();
-          ptx::named_bar_sync(1, NEPI);
-          if (etid == 0) {
-            asm volatile("fence.proxy.async.global;" ::: "memory");
-            asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(flag_of(l, m0 / GEMM_BM)) : "memory");
-          }
+        if (dataflow && l + 1 < P.n_layers && etid == 0) {
+          // every global write of this tile (activations, mask words, head partials) was a bulk copy issued
+          // by this thread: complete them, then count the tile (release)
+          ptx::bulk_wait<0>();
+          asm volatile("fence.proxy.async.global;" ::: "memory");
+          asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(flag_of(l, m0 / GEMM_BM)) : "memory");
         }
       }
       // ---- layer end: all of this CTA's outputs complete + visible, then the grid barrier

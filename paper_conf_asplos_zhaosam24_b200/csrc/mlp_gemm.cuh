@@ -35,8 +35,9 @@ struct GemmArgs {
   __half* out_hi;             // [M][ld_out]   RELU, HEAD, MASK
   __half* out_lo;
   int ld_out;
-  uint32_t* mask_out;         // [M][N/32]     RELU
-  const uint32_t* mask_in;    // [M][N/32]     MASK
+  uint32_t* mask_out;         // [N/32][ld_mask] RELU: bit i of word (w, row) = [z(row, 32w + i) > 0]
+  const uint32_t* mask_in;    // [N/32][ld_mask] MASK
+  int ld_mask;
   float* c_part;              // [N/BN][ld_c]  HEAD: per-N-tile partial of the head dot product
   int ld_c;
   float* out_f32;             // [n_valid][ld_f32]  F32T
@@ -239,9 +240,9 @@ mlp_gemm_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constan
             }
           }
           if constexpr (EPI == EPI_RELU)
-            if (row_ok) args.mask_out[static_cast<size_t>(row) * (args.N / 32) + n / 32] = bits;
+            if (row_ok) args.mask_out[static_cast<size_t>(n / 32) * args.ld_mask + row] = bits;
         } else {  // EPI_MASK
-          const uint32_t bits = row_ok ? __ldg(&args.mask_in[static_cast<size_t>(row) * (args.N / 32) + n / 32]) : 0u;
+          const uint32_t bits = row_ok ? __ldg(&args.mask_in[static_cast<size_t>(n / 32) * args.ld_mask + row]) : 0u;
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = ((bits >> i) & 1u) ? v[i] : 0.f;
         }

@@ -7,10 +7,14 @@ L513-515), and inside one task Eq. 4 is a sum of per-seed terms with an elementw
 * ``"task"`` (C3, full ResNet-50): whole tasks go to ranks by LPT (longest processing time first)
   on the estimated cost ``n_seeds * n_steps * (mlp_flops + DAG_WEIGHT * n_nodes)``: tasks in
   decreasing cost (ties: lower task index first) each go to the rank with the least assigned cost
-  (ties: lower rank).  Every rank runs its tasks concurrently, one CUDA stream per task.
+  (ties: lower rank).
 * ``"seeds"`` (C4, BERT-base): every task's seeds are cut into ``world`` contiguous ranges,
   rank r searching ``[r*n/world, (r+1)*n/world)`` with ``index_base`` = the range start, so global
   candidate indices (and therefore the top-k tie-breaks) do not depend on the rank count.
+
+On a rank, all its shards are searched as one group (``felix_search_group``): every Adam step runs each
+task's DAG kernels on its own stream and ONE tensor-core MLP pass over the candidates of all tasks (the
+tasks share the cost model), so the small per-task populations fill the GPU like one large population.
 
 The only exchange is at the end: one all-gather of every task's local top-k records, merged per
 task exactly as ``dist.merge_records`` does for one task (dedup by schedule keeping the smallest
@@ -18,7 +22,7 @@ global index, order by (score desc, index asc)).  The merged per-task lists equa
 top-k of every task for any world size.
 
 The planner is plain host logic (no libfelix needed) so it is unit-tested on CPU; the runner calls
-the C ABI only (``Space.search`` / ``Space.round_topk``).
+the C ABI only (``search_group`` / ``Space.search`` / ``Space.round_topk``).
 """
 from __future__ import annotations
 
@@ -141,8 +145,8 @@ def allgather_task_topk(per_task, n_tasks: int, k: int, n_vars: Sequence[int], g
 
 # ----------------------------------------------------------------------------- runner (C ABI only)
 class TaskRunner:
-    """One rank's shards of a multi-task workload: felix_search of every shard on its own CUDA stream
-    (the small searches overlap on the GPU), then felix_round_topk per shard."""
+    """One rank's shards of a multi-task workload: felix_search_group over all shards (or felix_search of
+    every shard on its own CUDA stream), then felix_round_topk per shard."""
 
     def __init__(self, spaces, shards: Sequence[Shard], cm, device: int = 0):
         from . import Space
@@ -152,16 +156,29 @@ class TaskRunner:
         self.spaces = {s.task: Space(spaces[s.task], device=device) for s in self.shards}
 
     def run(self, n_steps: int, k: int, *, rng_seed: int, lr: float = 0.05, lam: float = 1.0,
-            y0: Dict[int, object] = None, loss_out: Dict[int, object] = None, concurrent: bool = True):
+            y0: Dict[int, object] = None, loss_out: Dict[int, object] = None, concurrent: bool = True,
+            batched: bool = True):
         """Search every shard (device init, or from y0[task] if given: a device [n_vars, n] tensor
-        that is overwritten), then round / top-k.  Returns {task: (idx, score, sched)}."""
+        that is overwritten), then round / top-k.  Returns {task: (idx, score, sched)}.
+        batched: one felix_search_group over all shards (each Adam step: every task's DAG kernels on
+        its own stream, ONE tensor-core MLP pass over the candidates of all tasks, since they share the
+        cost model); else one felix_search per shard, on its own stream if `concurrent`."""
         import torch
+        from . import search_group
         dev = torch.device("cuda", self.device)
         main = torch.cuda.current_stream(dev)
         if not hasattr(self, "_streams"):
             self._streams = [torch.cuda.Stream(device=dev) for _ in self.shards]
             self._y = {s.task: torch.empty((self.spaces[s.task].n_vars, s.n), dtype=torch.float32, device=dev)
                        for s in self.shards}
+        if batched and len(self.shards) > 0:
+            ys = [self._y[s.task] if y0 is None else y0[s.task] for s in self.shards]
+            search_group([self.spaces[s.task] for s in self.shards], self.cm, ys, n_steps, lr=lr, lam=lam,
+                         rng_seeds=[rng_seed + s.task for s in self.shards], index_bases=[s.seed_lo for s in self.shards],
+                         init_from_y=y0 is not None,
+                         final_losses=None if loss_out is None else [loss_out[s.task] for s in self.shards], stream=main)
+            return {s.task: self.spaces[s.task].round_topk(self.cm, y, k, index_base=s.seed_lo, stream=main)
+                    for s, y in zip(self.shards, ys)}
         streams = self._streams if concurrent else [main] * len(self.shards)
         for s, st in zip(self.shards, streams):
             st.wait_stream(main)

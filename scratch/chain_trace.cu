@@ -29,7 +29,7 @@ int main(int argc, char** argv) {
     ChainLayer& L = P.layer[i];
     L.a_hi = L.a_lo = mk(a, M, K, 128); L.b_hi = L.b_lo = mk(w, N, K, bn); L.c_hi = L.c_lo = mk(c, M, N, 128);
     GemmArgs& g = L.args; g.M = M; g.N = N; g.K = K; g.bias = bias; g.head_w = hw; g.c_part = cpart; g.ld_c = M;
-    g.out_f32 = dphi; g.ld_f32 = M; g.n_valid = 82; g.mask_out = (uint32_t*)masks[1]; g.mask_in = (const uint32_t*)masks[1];
+    g.out_f32 = dphi; g.ld_f32 = M; g.n_valid = 82; g.ld_mask = (mt * 128); g.mask_out = (uint32_t*)masks[1]; g.mask_in = (const uint32_t*)masks[1];
     L.epi = epi; L.bn = bn; L.n_tiles_n = N / bn; L.n_tiles = mt * L.n_tiles_n; L.idesc = ptx::idesc_f16_f32(128, bn);
   };
   int bnA = argc > 2 ? atoi(argv[2]) : 128, bnB = argc > 3 ? atoi(argv[3]) : 64;
@@ -48,6 +48,9 @@ int main(int argc, char** argv) {
   unsigned int* flags = (unsigned int*)dz((size_t)6 * mt * CHAIN_FLAG_STRIDE * 4);
   int one = 1; int* ep = (int*)dz(4); cudaMemcpy(ep, &one, 4, cudaMemcpyHostToDevice);
   P.flags = FLAGS ? flags : nullptr; P.epoch = ep;
+  const int REUSE = argc > 6 ? atoi(argv[6]) : 0;        // 1: own-chunk reuse where the row block is kept
+  for (int i = 1; i < 6; ++i)
+    P.layer[i].reuse = (FLAGS && REUSE && P.layer[i - 1].epi != EPI_F32T && P.layer[i - 1].n_tiles_n == P.layer[i].n_tiles_n) ? 1 : 0;
   if (CS == 4) grid = std::min(148 / 4, mt) * 4;
   cudaFuncSetAttribute(mlp_chain_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES);
   cudaFuncSetAttribute(mlp_chain_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES);

@@ -562,3 +562,68 @@ def test_cone_per_cta_kernels_parity(fx, name, monkeypatch):
     y2 = torch.from_numpy(y0).cuda()
     fx.Space(sp).search(cm, y2, 1, init_from_y=True)
     assert torch.max(torch.abs(y1 - y2)).item() <= 1e-4 * (1 + torch.max(torch.abs(y2)).item())
+
+
+def _group_spaces():
+    r50 = fi.resnet50_spaces()
+    return [fi.c2_space(), r50[0], fi.bert_spaces()[1]], [700, 400, 513]
+
+
+@pytest.mark.timeout(600)
+def test_search_group_equals_individual_searches(fx, monkeypatch):
+    """felix_search_group (one MLP pass per Adam step over the candidates of several spaces) computes
+    every member's search exactly as felix_search does: with the tile kernel, whose per-row arithmetic
+    does not depend on the row's position, the final y and losses are bit-identical."""
+    monkeypatch.setenv("FELIX_MLP", "tile")
+    mlp = fi.make_mlp(fi.DEFAULT_MLP)
+    cm = fx.CostModel.from_weights(mlp)
+    sps, ns = _group_spaces()
+    spaces = [fx.Space(sp) for sp in sps]
+    T = 6
+    ind, ind_loss = [], []
+    for i, (sp, n) in enumerate(zip(spaces, ns)):
+        y = torch.empty((sp.n_vars, n), device="cuda")
+        l = torch.empty(n, device="cuda")
+        sp.search(cm, y, T, rng_seed=100 + i, init_from_y=False, index_base=7 * i, final_loss=l)
+        ind.append(y)
+        ind_loss.append(l)
+    ys = [torch.empty((sp.n_vars, n), device="cuda") for sp, n in zip(spaces, ns)]
+    ls = [torch.empty(n, device="cuda") for n in ns]
+    fx.search_group(spaces, cm, ys, T, rng_seeds=[100, 101, 102], index_bases=[0, 7, 14], init_from_y=False,
+                    final_losses=ls)
+    for a, b, la, lb in zip(ys, ind, ls, ind_loss):
+        assert torch.equal(a, b) and torch.equal(la, lb)
+    # the workspace is reused on a second call with the same members
+    ys2 = [torch.empty_like(y) for y in ys]
+    fx.search_group(spaces, cm, ys2, T, rng_seeds=[100, 101, 102], index_bases=[0, 7, 14], init_from_y=False)
+    assert all(torch.equal(a, b) for a, b in zip(ys, ys2))
+
+
+@pytest.mark.timeout(600)
+def test_search_group_one_step_vs_oracle(fx):
+    """One group Adam step (default MLP kernel for the group's total rows) against the oracle's one
+    step per member, north-star tolerances; loss per member vs the oracle objective."""
+    mlp = fi.make_mlp(fi.DEFAULT_MLP)
+    cm = fx.CostModel.from_weights(mlp)
+    sps, ns = _group_spaces()
+    spaces = [fx.Space(sp) for sp in sps]
+    y0s = [fi.make_y0(sp, n, seed=60 + i) for i, (sp, n) in enumerate(zip(sps, ns))]
+    ys = [torch.from_numpy(y).cuda() for y in y0s]
+    ls = [torch.empty(n, device="cuda") for n in ns]
+    fx.search_group(spaces, cm, ys, 1, init_from_y=True, final_losses=ls)
+    for sp, y0, y, l in zip(sps, y0s, ys, ls):
+        ob = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
+        ry, _, _, _ = fo.search(sp, mlp.W, mlp.b, y0, 1, lr=0.05, lam=1.0)
+        got = y.cpu().numpy()
+        exempt = (np.abs(ob.grad) < 1e-6) | (kink_margin(ob.zs) < 1e-4)[None, :]
+        assert not np.any((np.abs(got - ry) > 1e-4 * (1 + np.abs(ry))) & ~exempt)
+        assert np.max(np.abs(l.cpu().numpy() - ob.loss)) / np.sqrt(np.mean(ob.loss ** 2)) <= 1e-4
+
+
+def test_search_group_errors(fx):
+    mlp = fi.make_mlp(fi.DEFAULT_MLP)
+    cm = fx.CostModel.from_weights(mlp)
+    sp = fx.Space(fi.c2_space())
+    y = torch.zeros((sp.n_vars, 64), device="cuda")
+    with pytest.raises(fx.FelixError):
+        fx.search_group([sp, sp], cm, [y, y.clone()], 2)          # a space twice
