@@ -382,7 +382,10 @@ def run_felix(args):
 
     n_gemm = len(cfg.mlp_dims) * 2 - 4          # (L-1) forward + (L-1) backward GEMM layers
     mlp_launches = 1 if os.environ.get("FELIX_MLP", "chain") != "layers" else n_gemm
-    launches_per_step = 1 + T * (2 + mlp_launches) + (6 + len(cfg.mlp_dims) - 1)   # init + steps + finish
+    # init + steps + finish; the reverse class counts the split-cone kernels' final Adam launch too
+    rev_launches = int(round(prof["dag_rev_adam"][1] / K))
+    init_launches = max(1, int(round(prof["init"][1] / K)))   # sampler (+ the split-cone counter reset)
+    launches_per_step = init_launches + T * (1 + mlp_launches) + rev_launches + (6 + len(cfg.mlp_dims) - 1)
     ms_per_step = t_max / K
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
@@ -603,7 +606,10 @@ def run_felix_tasks(args):
     if not args.no_cpu_baseline and world == 1:
         rate, threads, sample, _ = oracle_baseline_tasks(cfg, args.cpu_seconds)
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample}
-    launches = sum(1 + T * 3 + (6 + len(cfg.mlp_dims) - 1) for _ in shards)
+    # split-cone kernels (default for these population sizes) add one final Adam launch per task
+    sc_final = 1 if os.environ.get("FELIX_SC", "") == "1" else 0   # groups: split-cone only when forced
+    sc_final *= 2                                                   # counter reset + final Adam
+    launches = sum(1 + T * 3 + sc_final + (6 + len(cfg.mlp_dims) - 1) for _ in shards)
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
         "ms_per_step": t_max / K, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,

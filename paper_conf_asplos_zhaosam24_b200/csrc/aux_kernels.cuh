@@ -199,6 +199,137 @@ __global__ void __launch_bounds__(256) score_layer_kernel(const double* __restri
   }
 }
 
+// ---------------------------------------------------------------------------- K6 FP64 MLP scoring (v2)
+// Same arithmetic again (acc = b[col]; k ascending: acc = fma(W[col][k], in(row, k), acc)), bit-identical
+// to the kernels above.  128 x 64 output tile per 256-thread block; thread (tx, ty) owns rows ty + 16 i
+// (i < 8) and columns tx + 16 j (j < 4), 32 FP64 accumulators: per k, 8 + 4 conflict-free shared loads
+// (a warp reads 2 distinct A addresses and 16 consecutive W doubles) feed 32 DFMA.  K is staged 16 at a
+// time through double-buffered shared memory filled one chunk ahead from registers, one barrier per chunk.
+constexpr int SC2_TM = 128, SC2_TN = 64, SC2_KT = 16;
+__global__ void __launch_bounds__(256) score_layer_v2_kernel(const double* __restrict__ in, long long in_rs, long long in_cs,
+                                                             int n, int K, const double* __restrict__ W,
+                                                             const double* __restrict__ b, double* __restrict__ out,
+                                                             int N, int relu, int accumulate) {
+  __shared__ double As[2][SC2_KT][SC2_TM];   // [buf][k][row]
+  __shared__ double Bs[2][SC2_KT][SC2_TN];   // [buf][k][col]
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  const int row0 = blockIdx.y * SC2_TM, col0 = blockIdx.x * SC2_TN;
+  double acc[8][4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const int col = col0 + tx + 16 * j;
+    const double bj = col < N ? b[col] : 0.0;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i][j] = bj;
+  }
+  // per chunk: A tile 16 x 128 (8 per thread), W tile 16 x 64 (4 per thread)
+  double pa[8], pb[4];
+  auto load_chunk = [&](int k0) {
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int e = tid + q * 256;
+      int r, kk;
+      if (in_rs == 1) { r = e & 127; kk = e >> 7; } else { kk = e & 15; r = e >> 4; }
+      const int gr = row0 + r, gk = k0 + kk;
+      pa[q] = (gr < n && gk < K) ? in[static_cast<size_t>(gr) * in_rs + static_cast<size_t>(gk) * in_cs] : 0.0;
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int e = tid + q * 256;
+      const int c = e >> 4, kb = e & 15;
+      const int gc = col0 + c, gkb = k0 + kb;
+      pb[q] = (gc < N && gkb < K) ? W[static_cast<size_t>(gc) * K + gkb] : 0.0;
+    }
+  };
+  auto store_chunk = [&](int buf) {
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int e = tid + q * 256;
+      int r, kk;
+      if (in_rs == 1) { r = e & 127; kk = e >> 7; } else { kk = e & 15; r = e >> 4; }
+      As[buf][kk][r] = pa[q];
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int e = tid + q * 256;
+      Bs[buf][e & 15][e >> 4] = pb[q];
+    }
+  };
+  const int nk = (K + SC2_KT - 1) / SC2_KT;
+  load_chunk(0);
+  store_chunk(0);
+  __syncthreads();
+  for (int c = 0; c < nk; ++c) {
+    const int buf = c & 1;
+    if (c + 1 < nk) load_chunk((c + 1) * SC2_KT);
+    const int kmax = min(SC2_KT, K - c * SC2_KT);
+    if (kmax == SC2_KT) {
+#pragma unroll
+      for (int kk = 0; kk < SC2_KT; ++kk) {
+        double a[8], w[4];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) a[i] = As[buf][kk][ty + 16 * i];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) w[j] = Bs[buf][kk][tx + 16 * j];
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) acc[i][j] = fma(w[j], a[i], acc[i][j]);
+      }
+    } else {
+      for (int kk = 0; kk < kmax; ++kk) {
+        double a[8], w[4];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) a[i] = As[buf][kk][ty + 16 * i];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) w[j] = Bs[buf][kk][tx + 16 * j];
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) acc[i][j] = fma(w[j], a[i], acc[i][j]);
+      }
+    }
+    if (c + 1 < nk) store_chunk(buf ^ 1);   // the other buffer was last read in chunk c - 1 (barrier below)
+    __syncthreads();
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int r = row0 + ty + 16 * i;
+    if (r >= n) continue;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int col = col0 + tx + 16 * j;
+      if (col >= N) continue;
+      const double v = (relu && !(acc[i][j] > 0.0)) ? 0.0 : acc[i][j];
+      out[static_cast<size_t>(r) * N + col] = accumulate ? out[static_cast<size_t>(r) * N + col] + v : v;
+    }
+  }
+}
+
+// head layer (N = 1, row-major input [n][K]): thread per row, K staged 32 at a time through shared memory
+// (coalesced row segments), same fma order as above
+__global__ void __launch_bounds__(128) score_head_kernel(const double* __restrict__ in, int n, int K,
+                                                         const double* __restrict__ W, const double* __restrict__ b,
+                                                         double* __restrict__ out, int accumulate) {
+  __shared__ double Ts[128][33];
+  const int row0 = blockIdx.x * 128, t = threadIdx.x;
+  double acc = b[0];
+  for (int k0 = 0; k0 < K; k0 += 32) {
+    const int kw = min(32, K - k0);
+#pragma unroll 4
+    for (int q = 0; q < 32; ++q) {
+      const int e = t + q * 128, r = e >> 5, kk = e & 31;
+      const int gr = row0 + r;
+      Ts[r][kk] = (gr < n && kk < kw) ? in[static_cast<size_t>(gr) * K + k0 + kk] : 0.0;
+    }
+    __syncthreads();
+    for (int kk = 0; kk < kw; ++kk) acc = fma(W[k0 + kk], Ts[t][kk], acc);
+    __syncthreads();
+  }
+  const int r = row0 + t;
+  if (r < n) out[r] = accumulate ? out[r] + acc : acc;
+}
+
 // ---------------------------------------------------------------------------- K7 dedup + top-k
 // Each block owns a chunk of entries; k rounds of block argmax by (score desc, order key asc) over
 // alive entries, then every alive entry whose schedule equals the winner's is killed (dedup keeps

@@ -487,7 +487,30 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
   // candidate c is MLP row s * n + c.
   // NREP replicas of the PG groups per block, each on its own 32 candidates: warps running the same
   // cone's straight-line code share the SM's instruction fetches (the code is executed once per warp).
-  o << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd(const float* __restrict__ yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr) {\n"
+  // ADAM = 1 (felix_fwd_adam, split-cone searches): first apply Adam step s = *step_ctr - 1 (the reverse
+  // kernel of the previous step left its partial adjoints in part / pen) to this CTA's 32 candidates in
+  // place -- thread (wq, lane) owns vars j = wq + PG * jj, every load is issued before the first use --
+  // then evaluate the features at the new y.  Each CTA owns its candidates, so in-place is race-free.
+  // The arithmetic and its order are those of rev_body (sums over q = 0..P-1, seeds, Adam expression).
+  auto emit_autos = [&](const char* ind, const std::string& ysrc) {
+    for (int j = 0; j < M; ++j) o << ind << "const double y" << j << " = (double)" << ysrc << "[" << j << "]" << (ysrc == "sy" ? "[lane]" : "") << ";\n";
+    for (size_t q = 0; q < autos.size(); ++q) o << ind << "const double spa" << q << " = fmax(" << autos[q].val << ", 0.0);\n";
+    for (size_t q = 0; q < autos.size(); ++q) o << ind << "pen_ += spa" << q << " * spa" << q << ";\n";
+  };
+  auto emit_auto_grad_switch = [&](const char* ind) {
+    o << ind << "switch (j) {\n";
+    for (int j = 0; j < M; ++j) {
+      std::string terms;
+      for (size_t q = 0; q < autos.size(); ++q)
+        for (auto& tv : autos[q].terms)
+          if (tv.first == j) terms += std::string(tv.second > 0 ? " + " : " - ") + "spa" + std::to_string(q);
+      if (!terms.empty()) o << ind << "  case " << j << ": gd += 2.0 * dlam * (0.0" << terms << "); break;\n";
+    }
+    o << ind << "  default: break;\n" << ind << "}\n";
+  };
+  o << "template <int ADAM>\n__device__ __forceinline__ void fwd_body(float* yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr,\n"
+    << "    float* mv, float* vv, const double* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part,\n"
+    << "    int n_head_tiles, int ld_c, float head_b, float lam, float lr, float b1, float b2, float eps) {\n"
     << "  __shared__ float sphi_all[NREP][NS][32][K0P + 1];\n"
     << "  __shared__ double sx_all[NREP][NV][32];   // x = exp(y), computed once per replica and shared by its groups\n"
     << "  const int rep = threadIdx.x / (PG * 32), tid = threadIdx.x % (PG * 32);\n"
@@ -504,8 +527,59 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  TSTAMP(0, 0);\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");   // y is the previous step's output\n"
     << "  TSTAMP(0, 1);\n"
-    << "  if (blockIdx.x == 0 && threadIdx.x == 0 && step_ctr) *step_ctr += 1;\n"
-    << "  for (int e = tid; e < NV * 32; e += PG * 32) { const int l = e & 31; const int cl = c0 + l; sx[e >> 5][l] = exp((double)yv[(size_t)(e >> 5) * ldy + (cl < n ? cl : n - 1)]); }\n"
+    << "  if (!ADAM) {\n"
+    << "    if (blockIdx.x == 0 && threadIdx.x == 0 && step_ctr) *step_ctr += 1;\n"
+    << "    for (int e = tid; e < NV * 32; e += PG * 32) { const int l = e & 31; const int cl = c0 + l; sx[e >> 5][l] = exp((double)yv[(size_t)(e >> 5) * ldy + (cl < n ? cl : n - 1)]); }\n"
+    << "  } else {\n"
+    << "    __shared__ float sya_all[NREP][NV][32];\n"
+    << "    __shared__ unsigned sbad_all[NREP][PG];\n"
+    << "    float (&sy)[NV][32] = sya_all[rep];\n    unsigned* sbad = sbad_all[rep];\n"
+    << "    constexpr int NJ = (NV + PG - 1) / PG;\n"
+    << "    const int cl = c0 + lane;\n    const bool live = cl < n;\n    const int cc = live ? cl : n - 1;\n"
+    << "    float yl[NJ], ml[NJ], vl[NJ];\n    double gxa[NJ];\n"
+    << "#pragma unroll\n    for (int jj = 0; jj < NJ; ++jj) {\n"
+    << "      const int j = wq + PG * jj;\n      if (j >= NV) break;\n"
+    << "      yl[jj] = yv[(size_t)j * ldy + cc]; ml[jj] = mv[(size_t)j * n + cc]; vl[jj] = vv[(size_t)j * n + cc];\n"
+    << "      double a = 0.0;\n#pragma unroll\n      for (int q = 0; q < PG; ++q) a += part[((size_t)q * NV + j) * n + cc];\n"
+    << "      gxa[jj] = a;\n    }\n"
+    << "    const int s_ = *step_ctr - 1;   // Adam steps to apply: reverse kernels run so far (the counter starts at 1)\n"
+    << "#pragma unroll\n    for (int jj = 0; jj < NJ; ++jj) { const int j = wq + PG * jj; if (j >= NV) break; sy[j][lane] = yl[jj]; }\n"
+    << "    __syncthreads();\n"
+    << "    if (s_ <= 0) {\n"
+    << "#pragma unroll\n      for (int jj = 0; jj < NJ; ++jj) { const int j = wq + PG * jj; if (j >= NV) break; sx[j][lane] = exp((double)yl[jj]); }\n"
+    << "    } else {\n"
+    << "      const double dlam = (double)lam;\n"
+    << "      double pen_ = 0.0;\n"
+    << "#pragma unroll\n      for (int q = 0; q < PG; ++q) pen_ += pen[(size_t)q * n + cc];\n"
+    << "      float cst = head_b * NS;\n"
+    << "      for (int i = 0; i < NS * n_head_tiles; ++i) cst += c_part[(size_t)(i % n_head_tiles) * ld_c + (size_t)(i / n_head_tiles) * n + cc];\n";
+  emit_autos("      ", "sy");
+  o << "      const float loss = (float)(-(double)cst + dlam * pen_);\n"
+    << "      bool ok = isfinite(loss);\n"
+    << "      float gyv[NJ];\n"
+    << "#pragma unroll\n      for (int jj = 0; jj < NJ; ++jj) {\n"
+    << "        const int j = wq + PG * jj;\n        if (j >= NV) break;\n"
+    << "        double gd = exp((double)yl[jj]) * gxa[jj];\n";
+  emit_auto_grad_switch("        ");
+  o << "        gyv[jj] = (float)gd;\n        ok = ok && isfinite(gyv[jj]);\n      }\n"
+    << "      const unsigned bad = __ballot_sync(0xffffffffu, !ok);\n"
+    << "      if (lane == 0) sbad[wq] = bad;\n"
+    << "      __syncthreads();\n"
+    << "      unsigned anybad = 0;\n#pragma unroll\n      for (int q = 0; q < PG; ++q) anybad |= sbad[q];\n"
+    << "      const bool okall = !((anybad >> lane) & 1u);\n"
+    << "      const float bc1 = 1.f - powf(b1, (float)s_), bc2 = 1.f - powf(b2, (float)s_);\n"
+    << "      const float step = lr / bc1, rb = 1.f / sqrtf(bc2);\n"
+    << "#pragma unroll\n      for (int jj = 0; jj < NJ; ++jj) {\n"
+    << "        const int j = wq + PG * jj;\n        if (j >= NV) break;\n"
+    << "        float yy = yl[jj];\n"
+    << "        if (okall) {\n"
+    << "          float m = ml[jj], v = vl[jj];\n"
+    << "          m = b1 * m + (1.f - b1) * gyv[jj]; v = b2 * v + (1.f - b2) * gyv[jj] * gyv[jj];\n"
+    << "          yy = yl[jj] - step * m / (sqrtf(v) * rb + eps);\n"
+    << "          if (live) { mv[(size_t)j * n + cl] = m; vv[(size_t)j * n + cl] = v; yv[(size_t)j * ldy + cl] = yy; }\n"
+    << "        }\n"
+    << "        sx[j][lane] = exp((double)yy);\n      }\n"
+    << "    }\n  }\n"
     << "  for (int k = tid; k < NS * 32 * (K0P + 1); k += PG * 32) (&sphi[0][0][0])[k] = 0.f;\n"
     << "  BLOCK_SYNC();\n";
   for (int q = 0; q < P; ++q) {
@@ -545,7 +619,13 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "    }\n"
     << "    reinterpret_cast<uint4*>(phi_hi + row * K0P)[q8] = make_uint4(h[0], h[1], h[2], h[3]);\n"
     << "    reinterpret_cast<uint4*>(phi_lo + row * K0P)[q8] = make_uint4(l[0], l[1], l[2], l[3]);\n"
-    << "  }\n  TSTAMP(0, 3);\n}\n\n";
+    << "  }\n  TSTAMP(0, 3);\n}\n"
+    << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd(const float* __restrict__ yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr) {\n"
+    << "  fwd_body<0>(const_cast<float*>(yv), n, ldy, phi_hi, phi_lo, step_ctr, nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f);\n}\n"
+    << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd_adam(float* yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr,\n"
+    << "    float* mv, float* vv, const double* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part,\n"
+    << "    int n_head_tiles, int ld_c, float head_b, float lam, float lr, float b1, float b2, float eps) {\n"
+    << "  fwd_body<1>(yv, n, ldy, phi_hi, phi_lo, step_ctr, mv, vv, part, pen, c_part, n_head_tiles, ld_c, head_b, lam, lr, b1, b2, eps);\n}\n\n";
 
   // ---------------------------------------------------------------- felix_rev (template on mode)
   // smem: partial adjoints of x  spart[PG][NV][32], user-root penalties per group spen[PG][32],
@@ -710,6 +790,84 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
   o << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_eval(const float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
     << "    float* o_phi, float* o_g, float* o_cost, float* o_loss, float* o_grad) {\n"
     << "  rev_body<1>(nullptr, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, nullptr, nullptr, nullptr, 0.f, 0.f, 0.f, 0.f, o_phi, o_g, o_cost, o_loss, o_grad);\n}\n\n";
+
+  // ---------------------------------------------------------------- split-cone search kernels
+  // felix_rev_sc runs ONE cone per CTA (block-uniform q = blockIdx.x % PG) for W x 32 candidates, so the
+  // warps of an SM share one cone's straight-line code and instruction fetches (felix_rev_adam puts P
+  // different cones in one CTA and is instruction-fetch bound: 42 % of its stall samples are
+  // no_instructions).  Cone q's CTA writes its partial adjoints part[q][j][c] = dL/dx_j and its user-root
+  // penalty pen[q][c]; the cross-cone sums and Adam happen after the kernel boundary: in the next step's
+  // forward (felix_fwd_adam, whose CTAs own whole candidates) and, after the last step, in felix_adam_sc.
+  // Step counter: starts at 1, felix_rev_sc adds 1 (block 0, after griddepcontrol.wait; no CTA of the
+  // reverse kernel reads it), so the forward and the MLP chain of step t see t and Adam step t - 1 is due.
+  // Measured and dropped: Adam by the last of the P cone CTAs to arrive (+8 us at C2: a serial tail at
+  // 255 registers), and a split-cone forward (its 2-byte feature-column stores: 1.7x slower at C2).
+  o << "extern \"C\" __global__ void __launch_bounds__(256) felix_rev_sc(const float* __restrict__ yv, int n, int ldy, const float* __restrict__ dphi, int ld_dphi,\n"
+    << "    float lam, double* __restrict__ part, double* __restrict__ pen, int* step_ctr) {\n"
+    << "  const int cq_ = blockIdx.x % PG;\n"
+    << "  const int c = ((blockIdx.x / PG) * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32 + (threadIdx.x & 31);\n"
+    << "  const bool live = c < n;\n  const int ccw = live ? c : n - 1;\n"
+    << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
+    << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n"
+    << "  if (blockIdx.x == 0 && threadIdx.x == 0) *step_ctr += 1;\n"
+    << "  const double dlam = (double)lam;\n";
+  for (int q = 0; q < P; ++q) {
+    o << "  if (cq_ == " << q << ") {\n";
+    const auto used = vars_in(rcone[q]);
+    for (int j = 0; j < M; ++j)
+      if (used[j]) o << "    const double x" << j << " = exp((double)yv[(size_t)" << j << " * ldy + ccw]);\n";
+    g.emit_forward(rcone[q], 0, "x", "    ");
+    o << "    double pq = 0.0;\n";
+    for (int r : part.cons[q]) o << "    const double pr" << r << " = fmax(v" << d.croots[r] << ", 0.0); pq += pr" << r << " * pr" << r << ";\n";
+    const auto need = g.rev_live(rcone[q], rroots_g[q]);
+    g.emit_adj_decls(need, "    ");
+    for (int j = 0; j < M; ++j) o << "    ADJ_T gx" << j << " = 0;\n";
+    for (int k : part.feat[q]) {
+      const int r = d.froots[k];
+      o << "    " << g.adj(r) << " += (ADJ_T)((double)dphi[(size_t)" << fk(k) << " * ld_dphi + (size_t)" << fs(k)
+        << " * n + ccw] * slogp_(v" << r << "));\n";
+    }
+    for (int r : part.cons[q]) {
+      const int nd = d.croots[r];
+      if (g.depvar[nd]) o << "    " << g.adj(nd) << " += (ADJ_T)(2.0 * dlam * pr" << r << ");\n";
+    }
+    g.emit_reverse_body(need, "    ");
+    o << "    if (live) {\n      pen[(size_t)" << q << " * n + c] = pq;\n";
+    for (int j = 0; j < M; ++j) o << "      part[((size_t)" << q << " * NV + " << j << ") * n + c] = (double)gx" << j << ";\n";
+    o << "    }\n  }\n";
+  }
+  o << "}\n\n";
+  // felix_adam_sc: the last Adam step (thread per candidate, in place) + the final loss
+  o << "extern \"C\" __global__ void __launch_bounds__(128) felix_adam_sc(float* yv, int n, int ldy, float* mv, float* vv,\n"
+    << "    const double* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part, int n_head_tiles, int ld_c,\n"
+    << "    float head_b, float lam, float lr, float b1, float b2, float eps, const int* step_ctr, float* o_loss) {\n"
+    << "  const int c = blockIdx.x * blockDim.x + threadIdx.x;\n  if (c >= n) return;\n"
+    << "  const int s_ = *step_ctr - 1;\n  if (s_ <= 0) return;\n"
+    << "  const double dlam = (double)lam;\n"
+    << "  float syv[NV], ml[NV], vl[NV];\n  double gxa[NV];\n"
+    << "#pragma unroll\n  for (int j = 0; j < NV; ++j) {\n"
+    << "    syv[j] = yv[(size_t)j * ldy + c]; ml[j] = mv[(size_t)j * n + c]; vl[j] = vv[(size_t)j * n + c];\n"
+    << "    double a = 0.0;\n#pragma unroll\n    for (int q = 0; q < PG; ++q) a += part[((size_t)q * NV + j) * n + c];\n"
+    << "    gxa[j] = a;\n  }\n"
+    << "  double pen_ = 0.0;\n#pragma unroll\n  for (int q = 0; q < PG; ++q) pen_ += pen[(size_t)q * n + c];\n"
+    << "  float cst = head_b * NS;\n"
+    << "  for (int i = 0; i < NS * n_head_tiles; ++i) cst += c_part[(size_t)(i % n_head_tiles) * ld_c + (size_t)(i / n_head_tiles) * n + c];\n";
+  emit_autos("  ", "syv");
+  o << "  const float loss = (float)(-(double)cst + dlam * pen_);\n"
+    << "  if (o_loss) o_loss[c] = loss;\n"
+    << "  bool ok = isfinite(loss);\n  float gy[NV];\n"
+    << "#pragma unroll\n  for (int j = 0; j < NV; ++j) {\n"
+    << "    double gd = exp((double)syv[j]) * gxa[j];\n";
+  emit_auto_grad_switch("    ");
+  o << "    gy[j] = (float)gd;\n    ok = ok && isfinite(gy[j]);\n  }\n"
+    << "  if (!ok) return;\n"
+    << "  const float bc1 = 1.f - powf(b1, (float)s_), bc2 = 1.f - powf(b2, (float)s_);\n"
+    << "  const float step = lr / bc1, rb = 1.f / sqrtf(bc2);\n"
+    << "#pragma unroll\n  for (int j = 0; j < NV; ++j) {\n"
+    << "    float m = ml[j], v = vl[j];\n"
+    << "    m = b1 * m + (1.f - b1) * gy[j]; v = b2 * v + (1.f - b2) * gy[j] * gy[j];\n"
+    << "    mv[(size_t)j * n + c] = m; vv[(size_t)j * n + c] = v; yv[(size_t)j * ldy + c] = syv[j] - step * m / (sqrtf(v) * rb + eps);\n"
+    << "  }\n}\n\n";
 
   // ---------------------------------------------------------------- felix_hard (fp64 IEEE, integer points)
   std::vector<bool> all(g.n, true);

@@ -113,12 +113,17 @@ static CUtensorMap make_tmap(const void* base, int64_t rows, int64_t cols, int b
 }
 
 // ============================================================================ per-(space, model, n) plan
+static bool chain_exact() {
+  const char* e = std::getenv("FELIX_CHAIN_EXACT");
+  return !(e && std::atoi(e) == 0);
+}
 struct Plan {
   const CostModel* cm = nullptr;
   int64_t n = -1, n_pad = 0;
   DevBuf phi_hi, phi_lo;                                   // [n][K0p]
   std::vector<std::unique_ptr<DevBuf>> act_hi, act_lo, mask;  // per hidden layer l = 1..L-1
   DevBuf c_part, dphi, m, v, step_ctr;
+  DevBuf sc_part, sc_pen;                                // split-cone reverse: partial adjoints, penalties
   int n_head_tiles = 0;
   std::vector<GemmLaunch> gemms;           // per-layer kernels (FELIX_MLP=layers)
   ChainParams chain{};                     // persistent all-layer kernel
@@ -243,6 +248,7 @@ struct GroupCache {
   std::vector<int64_t> n, row_off;
   std::unique_ptr<Plan> plan;
   std::vector<std::unique_ptr<DevBuf>> m, v, step_ctr;
+  std::vector<std::unique_ptr<DevBuf>> sc_part, sc_pen;   // split-cone buffers per member (see Plan)
   std::vector<cudaStream_t> streams;
   cudaGraphExec_t graph = nullptr;
   std::vector<double> key;
@@ -266,6 +272,7 @@ struct felix_space {
   struct Module {
     cudaLibrary_t lib = nullptr;
     cudaKernel_t f_fwd = nullptr, f_rev_adam = nullptr, f_rev_eval = nullptr, f_hard = nullptr, f_init = nullptr;
+    cudaKernel_t f_rev_sc = nullptr, f_fwd_adam = nullptr, f_adam_sc = nullptr;   // split-cone search kernels
     int P = 1, R = 1, rev_smem = 0, regs_fwd = 0, regs_rev = 0;   // cone groups, replicas per block
     std::string source;
   };
@@ -441,7 +448,7 @@ static std::vector<char> nvrtc_compile(const std::string& source) {
 
 static felix_space::Module& get_module(felix_space* s, int P, int R = 1) {
   // the forward kernel stages NREP x NS x 32 x (K0P+1) floats + NREP x NV x 32 doubles statically
-  if (R > 1 && static_cast<int64_t>(R) * (s->desc.n_statements * 32 * (s->K0p + 1) * 4 + s->desc.n_vars * 32 * 8) > 48 * 1024)
+  if (R > 1 && static_cast<int64_t>(R) * (s->desc.n_statements * 32 * (s->K0p + 1) * 4 + s->desc.n_vars * 32 * (8 + 4) + 64) > 48 * 1024)
     R = 1;
   const int key = P + 64 * R;
   auto it = s->modules.find(key);
@@ -461,6 +468,9 @@ static felix_space::Module& get_module(felix_space* s, int P, int R = 1) {
   CUDA_OK(cudaLibraryGetKernel(&mod.f_rev_eval, mod.lib, "felix_rev_eval"));
   CUDA_OK(cudaLibraryGetKernel(&mod.f_hard, mod.lib, "felix_hard"));
   CUDA_OK(cudaLibraryGetKernel(&mod.f_init, mod.lib, "felix_init"));
+  CUDA_OK(cudaLibraryGetKernel(&mod.f_rev_sc, mod.lib, "felix_rev_sc"));
+  CUDA_OK(cudaLibraryGetKernel(&mod.f_fwd_adam, mod.lib, "felix_fwd_adam"));
+  CUDA_OK(cudaLibraryGetKernel(&mod.f_adam_sc, mod.lib, "felix_adam_sc"));
   for (cudaKernel_t k : {mod.f_rev_adam, mod.f_rev_eval})
     CUDA_OK(cudaFuncSetAttribute(reinterpret_cast<const void*>(k), cudaFuncAttributeMaxDynamicSharedMemorySize, mod.rev_smem));
   cudaFuncAttributes fa{};
@@ -560,6 +570,50 @@ static void launch_warp_per_item(cudaKernel_t f, int64_t n, void** args, cudaStr
 static void launch_flat(cudaKernel_t f, int64_t n, void** args, cudaStream_t st) {
   if (n <= 0) return;
   launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((n + 127) / 128)), dim3(128), 0, args, st, false);
+}
+
+// Split-cone reverse kernel (codegen.cpp felix_rev_sc): one cone per CTA for W x 32 candidates, partial
+// adjoints through global memory; the next step's forward (felix_fwd_adam) sums them and applies Adam,
+// felix_adam_sc after the last step.  Default for single-space searches; FELIX_SC=0 selects
+// felix_rev_adam, FELIX_SC=1 forces it in group searches too (measured there with an earlier variant:
+// C3 1.66e8 -> 1.65e8, C4 2.25e8 -> 2.08e8 cand-steps/s, so groups keep felix_rev_adam by default).
+// Not with history rounding (it rounds the caller's y before each step's forward, i.e. before Adam).
+static bool use_cpb();
+static bool use_sc(bool group = false) {
+  if (use_cpb()) return false;
+  const char* e = std::getenv("FELIX_SC");
+  const int v = e ? std::atoi(e) : -1;
+  if (v == 0) return false;
+  if (v == 1) return true;
+  return !group;
+}
+__global__ void set_int_kernel(int* p, int v) { *p = v; }
+// Split-cone searches: at least two cones (measured at the C5 shard, 131072 candidates: 2.53e8 at P = 1,
+// 2.72e8 at P = 2 cand-steps/s) and two replicas of the cone groups per felix_fwd_adam block (warps on the
+// same cone share instruction fetches; C2 forward 14.8 -> 12.8 us).  FELIX_P / FELIX_R override.
+static int choose_P_sc(int P) { return (P == 1 && !std::getenv("FELIX_P")) ? 2 : P; }
+static int choose_R_sc() {
+  if (const char* e = std::getenv("FELIX_R")) {
+    const int r = std::atoi(e);
+    if (r == 1 || r == 2 || r == 4) return r;
+  }
+  return 2;
+}
+// warps per split-cone CTA: about one CTA per SM (FELIX_SCW overrides)
+static int choose_scw(int64_t n, int P) {
+  if (const char* e = std::getenv("FELIX_SCW")) {
+    const int w = std::atoi(e);
+    if (w >= 1 && w <= 8) return w;
+  }
+  const int64_t groups = (n + 31) / 32;
+  int64_t w = (groups * P + 147) / 148;
+  return static_cast<int>(std::max<int64_t>(1, std::min<int64_t>(8, w)));
+}
+static int64_t sc_groups(int64_t n, int W) { return ((n + 31) / 32 + W - 1) / W; }
+static void launch_sc(cudaKernel_t f, int P, int W, int64_t n, void** args, cudaStream_t st, bool pdl) {
+  if (n <= 0) return;
+  launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>(sc_groups(n, W) * P)), dim3(32 * W), 0, args,
+             st, pdl);
 }
 
 // ============================================================================ plan
@@ -702,6 +756,16 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     L.a_hi = g.a_hi; L.a_lo = g.a_lo; L.c_hi = g.c_hi; L.c_lo = g.c_lo;
     L.b_hi = make_tmap(g.w_hi, N, g.args.K, bn);
     L.b_lo = make_tmap(g.w_lo, N, g.args.K, bn);
+    // the first backward layer takes the 0/1 mask of the head layer as its A operand and the head row
+    // folded into its weights (exact A: two MMA passes, no A lo loads); FELIX_CHAIN_EXACT=0 disables
+    L.a_exact = 0;
+    L.head_exact = 0;
+    if (i == static_cast<size_t>(cm->n_layers - 1) && i > 0 && chain_exact() && p->gemms[i - 1].epi == EPI_HEAD) {
+      L.a_exact = 1;
+      p->chain.layer[i - 1].head_exact = 1;
+      L.b_hi = make_tmap(cm->WTs_hi.p, N, g.args.K, bn);
+      L.b_lo = make_tmap(cm->WTs_lo.p, N, g.args.K, bn);
+    }
     if (g.epi == EPI_HEAD && use_chain()) p->n_head_tiles = 2 * (N / bn);   // chain: one partial per column half
     max_tiles = std::max(max_tiles, L.n_tiles);
   }
@@ -827,6 +891,7 @@ static void prof_mark(felix_space* s, int cls, cudaStream_t st, bool begin) {
 }
 
 // ============================================================================ step pieces
+static void run_mlp(felix_space* s, Plan& p, cudaStream_t st);
 static void run_forward_mlp(felix_space* s, Plan& p, const felix_space::Module& mod, const float* y, int64_t n,
                             int64_t ldy, cudaStream_t st, int* step_ctr) {
   int ni = static_cast<int>(n), ldi = static_cast<int>(ldy);
@@ -837,6 +902,10 @@ static void run_forward_mlp(felix_space* s, Plan& p, const felix_space::Module& 
   launch_grouped(mod.f_fwd, mod.P, mod.R, n, 0, args, st, true);
   prof_mark(s, 0, st, false);
   s->prof_launches[0] += 1;
+  run_mlp(s, p, st);
+}
+
+static void run_mlp(felix_space* s, Plan& p, cudaStream_t st) {
   prof_mark(s, 1, st, true);
   const MlpMode mode = static_cast<MlpMode>(p.mode);
   if (mode == MLP_TILE) {
@@ -1093,6 +1162,18 @@ felix_status felix_costmodel_load(int device, int32_t n_layers, const int32_t* d
   }
   const int Dh = dims[n_layers - 1];
   upload(m->head_w, std::vector<float>(W[n_layers - 1], W[n_layers - 1] + Dh));
+  if (n_layers >= 2) {
+    const int l = n_layers - 2, N = dims[l + 1], K = dims[l];
+    const int Kp = (l == 0) ? m->K0p : K;
+    std::vector<float> wt(static_cast<size_t>(Kp) * N, 0.f);
+    for (int r = 0; r < N; ++r)
+      for (int c = 0; c < K; ++c)
+        wt[static_cast<size_t>(c) * N + r] = -W[n_layers - 1][r] * W[l][static_cast<size_t>(r) * K + c];
+    std::vector<__half> thi, tlo;
+    split_half(wt, thi, tlo);
+    upload(m->WTs_hi, thi);
+    upload(m->WTs_lo, tlo);
+  }
   m->head_b = b[n_layers - 1][0];
   for (int l = 0; l < n_layers; ++l) {
     const int N = dims[l + 1], K = dims[l];
@@ -1132,7 +1213,10 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
   const int64_t n = p->n_seeds;
   Chunks& ch = get_chunks(s, s->search_chunks, m, n, choose_chunks(n));
   const int nck = static_cast<int>(ch.plans.size());
-  const felix_space::Module& mod = get_module(s, choose_P(ch.cnt[0]), choose_R(ch.cnt[0], choose_P(ch.cnt[0])));
+  const bool sc = use_sc() && !p->history;
+  const int P0 = choose_P(ch.cnt[0]);
+  const felix_space::Module& mod = sc ? get_module(s, choose_P_sc(P0), choose_R_sc()) : get_module(s, P0, choose_R(ch.cnt[0], P0));
+  const int scw = choose_scw(ch.cnt[0], mod.P);
   if (!p->init_from_y) {
     unsigned long long seed = p->rng_seed;
     long long ib = p->index_base;
@@ -1152,6 +1236,14 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     CUDA_OK(cudaMemsetAsync(pl->grid_bar.p, 0, pl->grid_bar.bytes, st));
     // dataflow flags count up with step_ctr (reset together; 8 * steps stays far below 2^32)
     CUDA_OK(cudaMemsetAsync(pl->chain_flags.p, 0, pl->chain_flags.bytes, st));
+    if (sc) {
+      const int64_t cnt = pl->n / s->desc.n_statements;
+      ensure(pl->sc_part, static_cast<size_t>(mod.P) * s->desc.n_vars * cnt * 8);
+      ensure(pl->sc_pen, static_cast<size_t>(mod.P) * cnt * 8);
+      set_int_kernel<<<1, 1, 0, st>>>(pl->step_ctr.as<int>(), 1);   // the reverse kernel counts from 1
+      CUDA_OK(cudaGetLastError());
+      s->prof_launches[3] += 1;
+    }
   }
   // varValuesHistory: a fresh pool for this search (worst case: every seed at every step is new)
   const int M = s->desc.n_vars;
@@ -1192,7 +1284,6 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     const int64_t o = ch.off[k], cnt = ch.cnt[k];
     float* yk = y + o;
     int* ctr = pl.step_ctr.as<int>();
-    run_forward_mlp(s, pl, mod, yk, cnt, n, cs, ctr);
     int ni = static_cast<int>(cnt), ldy = static_cast<int>(n);
     void* dphi = pl.dphi.p;
     void* cpart = pl.c_part.p;
@@ -1201,6 +1292,26 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     float hbv = hb, lam = lam0, lr = lr0, b1 = b10, b2 = b20, eps = eps0;
     void* mv = pl.m.p;
     void* vv = pl.v.p;
+    if (sc) {
+      // Adam step t-1 (in place) + features at y -> MLP -> split-cone reverse (partial adjoints)
+      void* phh = pl.phi_hi.p;
+      void* phl = pl.phi_lo.p;
+      void* part = pl.sc_part.p;
+      void* pen = pl.sc_pen.p;
+      void* fa[] = {&yk, &ni, &ldy, &phh, &phl, &ctr, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hbv, &lam, &lr, &b1, &b2, &eps};
+      prof_mark(s, 0, cs, true);
+      launch_grouped(mod.f_fwd_adam, mod.P, mod.R, cnt, 0, fa, cs, true);
+      prof_mark(s, 0, cs, false);
+      s->prof_launches[0] += 1;
+      run_mlp(s, pl, cs);
+      void* ra[] = {&yk, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr};
+      prof_mark(s, 2, cs, true);
+      launch_sc(mod.f_rev_sc, mod.P, scw, cnt, ra, cs, true);
+      prof_mark(s, 2, cs, false);
+      s->prof_launches[2] += 1;
+      return;
+    }
+    run_forward_mlp(s, pl, mod, yk, cnt, n, cs, ctr);
     float* lo = final_loss ? final_loss + o : nullptr;   // every step writes its loss; the last one stays
     void* args[] = {&yk, &ni, &ldy, &dphi, &ld, &cpart, &nht, &ld, &hbv, &lam, &mv, &vv, &ctr, &lr, &b1, &b2, &eps, &lo};
     prof_mark(s, 2, cs, true);
@@ -1222,7 +1333,9 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     // launched n_steps times with no per-step join, so one chunk's MLP overlaps another's DAG kernels
     // (a per-step fork/join would re-synchronise them every step).  Joined once at the end.
     auto ptr = [](const void* q) { return static_cast<double>(reinterpret_cast<uintptr_t>(q)); };
-    const std::vector<double> key = {static_cast<double>(mod.P), ptr(y), ptr(final_loss), lam0, lr0, b10, b20, eps0};
+    const std::vector<double> key = {static_cast<double>(mod.P), ptr(y), ptr(final_loss), lam0, lr0, b10, b20, eps0,
+                                     static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R),
+                                     ptr(ch.plans[0]->sc_part.p), ptr(ch.plans[0]->sc_pen.p)};
     while (static_cast<int>(ch.streams.size()) < nck) {
       cudaStream_t b;
       CUDA_OK(cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking));
@@ -1275,7 +1388,9 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     const std::vector<double> key = {static_cast<double>(mod.P), ptr(y), ptr(final_loss), lam0, lr0, b10, b20, eps0,
                                      static_cast<double>(s->h_valid), ptr(s->h_sched.p), ptr(s->h_last.p),
                                      ptr(s->h_slot_h.p), ptr(s->h_pool_sched.p), ptr(s->h_pool_key.p),
-                                     static_cast<double>(s->h_mask), static_cast<double>(s->h_cap)};
+                                     static_cast<double>(s->h_mask), static_cast<double>(s->h_cap),
+                                     static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R),
+                                     ptr(ch.plans[0]->sc_part.p), ptr(ch.plans[0]->sc_pen.p)};
     if (!ch.graph || ch.graph_key != key) {
       if (ch.graph) { cudaGraphExecDestroy(ch.graph); ch.graph = nullptr; }
       while (static_cast<int>(ch.streams.size()) < nck) {
@@ -1326,6 +1441,28 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
                            (ch.plans[0]->mode == MLP_LAYERS ? static_cast<int64_t>(ch.plans[0]->gemms.size()) : 1);
     s->prof_launches[2] += static_cast<int64_t>(p->n_steps) * nck;
   }
+  if (sc && p->n_steps > 0) {
+    // the last Adam step (the forward kernel of step t applies step t-1) and the final loss
+    for (int k = 0; k < nck; ++k) {
+      Plan& pl = *ch.plans[k];
+      const int64_t o = ch.off[k], cnt = ch.cnt[k];
+      float* yk = y + o;
+      int ni = static_cast<int>(cnt), ldy = static_cast<int>(n), ld = static_cast<int>(pl.n_pad), nht = pl.n_head_tiles;
+      void* mv = pl.m.p;
+      void* vv = pl.v.p;
+      void* part = pl.sc_part.p;
+      void* pen = pl.sc_pen.p;
+      void* cpart = pl.c_part.p;
+      void* ctr = pl.step_ctr.p;
+      float* lo = final_loss ? final_loss + o : nullptr;
+      float hbv = hb, lam = lam0, lr = lr0, b1 = b10, b2 = b20, eps = eps0;
+      void* aa[] = {&yk, &ni, &ldy, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hbv, &lam, &lr, &b1, &b2, &eps, &ctr, &lo};
+      prof_mark(s, 2, st, true);
+      launch_flat(mod.f_adam_sc, cnt, aa, st);
+      prof_mark(s, 2, st, false);
+      s->prof_launches[2] += 1;
+    }
+  }
   FELIX_API_END
 }
 
@@ -1372,6 +1509,7 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
       }
       gc->step_ctr.push_back(std::make_unique<DevBuf>());
       gc->step_ctr.back()->alloc(16);
+      for (auto* vec : {&gc->sc_part, &gc->sc_pen}) vec->push_back(std::make_unique<DevBuf>());
     }
     gc->plan = build_plan_rows(s0->device, m, rows, 0, 0);
     gc->plan->chain.epoch = gc->step_ctr[0]->as<int>();   // every member's forward bumps its counter once per step
@@ -1386,9 +1524,16 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
   Plan& pl = *gc.plan;
   // ---- per-search state: starting points, Adam state, counters, dataflow flags
   std::vector<const felix_space::Module*> mods(G);
+  const bool sc = use_sc(true);
+  std::vector<int> scws(G);
   for (int i = 0; i < G; ++i) {
     const int64_t n = params[i].n_seeds;
-    mods[i] = &get_module(spaces[i], choose_P(n), choose_R(n, choose_P(n)));
+    mods[i] = sc ? &get_module(spaces[i], choose_P_sc(choose_P(n)), choose_R_sc()) : &get_module(spaces[i], choose_P(n), choose_R(n, choose_P(n)));
+    scws[i] = choose_scw(n, mods[i]->P);
+    if (sc) {
+      ensure(*gc.sc_part[i], static_cast<size_t>(mods[i]->P) * spaces[i]->desc.n_vars * n * 8);
+      ensure(*gc.sc_pen[i], static_cast<size_t>(mods[i]->P) * n * 8);
+    }
     if (!params[i].init_from_y) {
       unsigned long long seed = params[i].rng_seed;
       long long ib = params[i].index_base;
@@ -1400,6 +1545,10 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
     CUDA_OK(cudaMemsetAsync(gc.m[i]->p, 0, gc.m[i]->bytes, st));
     CUDA_OK(cudaMemsetAsync(gc.v[i]->p, 0, gc.v[i]->bytes, st));
     CUDA_OK(cudaMemsetAsync(gc.step_ctr[i]->p, 0, 4, st));
+    if (sc) {
+      set_int_kernel<<<1, 1, 0, st>>>(gc.step_ctr[i]->as<int>(), 1);   // the split-cone reverse counts from 1
+      CUDA_OK(cudaGetLastError());
+    }
   }
   CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
   CUDA_OK(cudaMemsetAsync(pl.chain_flags.p, 0, pl.chain_flags.bytes, st));
@@ -1422,6 +1571,20 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
       void* phi_hi = pl.phi_hi.as<uint16_t>() + gc.row_off[i] * K0p;
       void* phi_lo = pl.phi_lo.as<uint16_t>() + gc.row_off[i] * K0p;
       int* ctr = gc.step_ctr[i]->as<int>();
+      if (sc) {
+        const felix_search_params& p = params[i];
+        float* ya = y[i];
+        void* mv = gc.m[i]->p;
+        void* vv = gc.v[i]->p;
+        void* part = gc.sc_part[i]->p;
+        void* pen = gc.sc_pen[i]->p;
+        void* cpart = pl.c_part.as<float>() + gc.row_off[i];
+        int ld = static_cast<int>(pl.n_pad), nht = pl.n_head_tiles;
+        float hbv = m->head_b, lam = p.lambda, lr = p.lr, b1 = p.beta1, b2 = p.beta2, eps = p.eps;
+        void* fa[] = {&ya, &ni, &ldi, &phi_hi, &phi_lo, &ctr, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hbv, &lam, &lr, &b1, &b2, &eps};
+        launch_grouped(mods[i]->f_fwd_adam, mods[i]->P, mods[i]->R, params[i].n_seeds, 0, fa, si, false);
+        continue;
+      }
       void* args[] = {&yi, &ni, &ldi, &phi_hi, &phi_lo, &ctr};
       launch_grouped(mods[i]->f_fwd, mods[i]->P, mods[i]->R, params[i].n_seeds, 0, args, si, false);
     }
@@ -1451,6 +1614,13 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
       void* vv = gc.v[i]->p;
       int* ctr = gc.step_ctr[i]->as<int>();
       float* lo = final_loss ? final_loss[i] : nullptr;
+      if (sc) {
+        void* part = gc.sc_part[i]->p;
+        void* pen = gc.sc_pen[i]->p;
+        void* ra[] = {&yi, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr};
+        launch_sc(mods[i]->f_rev_sc, mods[i]->P, scws[i], p.n_seeds, ra, si, false);
+        continue;
+      }
       void* args[] = {&yi, &ni, &ldy, &dphi, &ld, &cpart, &nht, &ld, &hbv, &lam, &mv, &vv, &ctr, &lr, &b1, &b2, &eps, &lo};
       launch_grouped(mods[i]->f_rev_adam, mods[i]->P, mods[i]->R, p.n_seeds, mods[i]->rev_smem, args, si, false);
     }
@@ -1459,12 +1629,32 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
       CUDA_OK(cudaStreamWaitEvent(main_st, ev[G + 1 + i], 0));
     }
   };
+  // the last Adam step of split-cone members (their forward kernel of step t applies step t-1)
+  auto final_adam = [&]() {
+    if (!sc) return;
+    for (int i = 0; i < G; ++i) {
+      const felix_search_params& p = params[i];
+      float* ya = y[i];
+      int ni = static_cast<int>(p.n_seeds), ldy = ni, ld = static_cast<int>(pl.n_pad), nht = pl.n_head_tiles;
+      void* mv = gc.m[i]->p;
+      void* vv = gc.v[i]->p;
+      void* part = gc.sc_part[i]->p;
+      void* pen = gc.sc_pen[i]->p;
+      void* cpart = pl.c_part.as<float>() + gc.row_off[i];
+      void* ctr = gc.step_ctr[i]->p;
+      float* lo = final_loss ? final_loss[i] : nullptr;
+      float hbv = m->head_b, lam = p.lambda, lr = p.lr, b1 = p.beta1, b2 = p.beta2, eps = p.eps;
+      void* aa[] = {&ya, &ni, &ldy, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hbv, &lam, &lr, &b1, &b2, &eps, &ctr, &lo};
+      launch_flat(mods[i]->f_adam_sc, p.n_seeds, aa, st);
+    }
+  };
   if (s0->profiling) {
     for (int t = 1; t <= T; ++t) {
       if (t % 100000 == 0) CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
       enqueue_step(st);
       s0->prof_launches[1] += 1;
     }
+    final_adam();
     return FELIX_OK;
   }
   auto ptr = [](const void* q) { return static_cast<double>(reinterpret_cast<uintptr_t>(q)); };
@@ -1472,7 +1662,9 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
   for (int i = 0; i < G; ++i) {
     const felix_search_params& p = params[i];
     key.insert(key.end(), {static_cast<double>(mods[i]->P), static_cast<double>(mods[i]->R), ptr(y[i]),
-                           ptr(final_loss ? final_loss[i] : nullptr), p.lambda, p.lr, p.beta1, p.beta2, p.eps});
+                           ptr(final_loss ? final_loss[i] : nullptr), p.lambda, p.lr, p.beta1, p.beta2, p.eps,
+                           static_cast<double>(sc), static_cast<double>(scws[i]), ptr(gc.sc_part[i]->p),
+                           ptr(gc.sc_pen[i]->p)});
   }
   if (!gc.graph || gc.key != key) {
     if (gc.graph) { cudaGraphExecDestroy(gc.graph); gc.graph = nullptr; }
@@ -1498,6 +1690,7 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
     if (t % 100000 == 0) CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
     CUDA_OK(cudaGraphLaunch(gc.graph, st));
   }
+  final_adam();
   FELIX_API_END
 }
 
@@ -1580,6 +1773,12 @@ static void do_hard(felix_space* s, const int32_t* sched, int64_t n, double* phi
   launch_flat(get_module(s, 1).f_hard, n, args, st);
 }
 
+// FELIX_SCORE=1 selects the previous 64 x 64 scoring kernels (same results)
+static bool score_v2() {
+  const char* e = std::getenv("FELIX_SCORE");
+  return !(e && std::atoi(e) == 1);
+}
+
 static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, int64_t n, double* score, cudaStream_t st) {
   // TenSet segment sum over statements: score = sum_s MLP(phi_s), phi64 = [S * K0][n] statement-major
   const int L = m->n_layers;
@@ -1595,11 +1794,19 @@ static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, in
       const int K = m->dims[l], N = m->dims[l + 1];
       const bool last = l == L - 1;
       double* out = last ? score : bufs[l & 1];
-      if (N >= 32) {   // register-blocked 64 x 64 tiles (bit-identical arithmetic)
+      if (N >= 32 && score_v2()) {   // register-blocked 128 x 64 tiles (bit-identical arithmetic)
+        const dim3 grid(static_cast<unsigned>((N + SC2_TN - 1) / SC2_TN), static_cast<unsigned>((n + SC2_TM - 1) / SC2_TM));
+        score_layer_v2_kernel<<<grid, 256, 0, st>>>(
+            in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
+            last ? 0 : 1, last && st_i > 0 ? 1 : 0);
+      } else if (N >= 32) {   // register-blocked 64 x 64 tiles (bit-identical arithmetic)
         const dim3 grid(static_cast<unsigned>((N + SCORE_T - 1) / SCORE_T), static_cast<unsigned>((n + SCORE_T - 1) / SCORE_T));
         score_layer_rb_kernel<<<grid, 256, 0, st>>>(
             in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
             last ? 0 : 1, last && st_i > 0 ? 1 : 0);
+      } else if (N == 1 && last && rs == K && cs == 1 && score_v2()) {
+        score_head_kernel<<<static_cast<unsigned>((n + 127) / 128), 128, 0, st>>>(
+            in, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, st_i > 0 ? 1 : 0);
       } else {
         const dim3 grid(static_cast<unsigned>((N + 31) / 32), static_cast<unsigned>((n + 31) / 32));
         score_layer_kernel<<<grid, dim3(32, 8), 0, st>>>(

@@ -94,6 +94,9 @@ struct CostModel {
   // per layer l = 0..L-2 (weights W_{l+1} in paper numbering): forward (N x Kp) and transposed
   std::vector<std::unique_ptr<DevBuf>> W_hi, W_lo, WT_hi, WT_lo, bias;
   DevBuf head_w;                 // last layer row [dims[L-1]] fp32
+  // first backward GEMM with the head row folded in: WTs[j][i] = -w_L[i] * W_{L-1}[i][j] (fp32 product, then
+  // split), so its A operand is the exact 0/1 mask [Z_{L-1} > 0] (chain: no A lo pass, no A lo bytes)
+  DevBuf WTs_hi, WTs_lo;
   float head_b = 0.f;
   std::vector<std::unique_ptr<DevBuf>> W64, b64;   // fp64 copies of every layer (scoring)
 };

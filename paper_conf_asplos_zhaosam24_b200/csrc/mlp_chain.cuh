@@ -55,7 +55,9 @@ struct ChainLayer {
   // chunks, still in its epilogue staging buffers in the A-operand layout (128-B swizzle, K-major), serve
   // as those K blocks (no TMA load; no wait for other CTAs), issued first.
   int reuse;
-  int _pad[2];
+  // a_exact: A is an exact 0/1 mask (fp16 hi exact, lo = 0): no A lo loads, no A lo MMA pass (the first
+  // backward layer, weights prescaled by the head row); head_exact: this HEAD layer writes that mask
+  int a_exact, head_exact;
 };
 
 struct ChainParams {
@@ -211,7 +213,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         }
         CHAIN_STAMP(l, 0);
         const int nkb = (L.args.K + GEMM_BK - 1) / GEMM_BK;
-        const uint32_t tx = 2 * CHAIN_A_BYTES + 2 * (L.bn * GEMM_BK * 2);
+        const uint32_t tx = (L.a_exact ? 1 : 2) * CHAIN_A_BYTES + 2 * (L.bn * GEMM_BK * 2);
         ChainTiles<CS> tiles(L.n_tiles_n, P.m_tiles);
         for (int tile = tiles.first(); tile >= 0; tile = tiles.next(tile)) {
           const int m0 = (tile / L.n_tiles_n) * GEMM_BM, n0 = (tile % L.n_tiles_n) * L.bn;
@@ -227,7 +229,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
               const bool own = i < nown;
               const int s = it % CHAIN_STAGES;
               if (it >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], ((it / CHAIN_STAGES) - 1) & 1);
-              ptx::mbar_arrive_expect_tx(&full_bar[s], own ? tx_b : tx);
+              ptx::mbar_arrive_expect_tx(&full_bar[s], own ? tx_b : tx);   // tx counts A lo only when loaded
               ptx::tma_load_2d(b_hi(s), &L.b_hi, kb * GEMM_BK, n0, &full_bar[s]);
               ptx::tma_load_2d(b_lo(s), &L.b_lo, kb * GEMM_BK, n0, &full_bar[s]);
               if (!own) {
@@ -237,7 +239,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
                   flag_ok = true;
                 }
                 ptx::tma_load_2d(a_hi(s), &L.a_hi, kb * GEMM_BK, m0, &full_bar[s]);
-                ptx::tma_load_2d(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, &full_bar[s]);
+                if (!L.a_exact) ptx::tma_load_2d(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, &full_bar[s]);
               }
             }
             continue;
@@ -258,7 +260,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             for (int kb = 0; kb < pre; ++kb) {
               const int s = (it + kb) % CHAIN_STAGES;
               ptx::tma_load_2d(a_hi(s), &L.a_hi, kb * GEMM_BK, m0, &full_bar[s]);
-              ptx::tma_load_2d(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, &full_bar[s]);
+              if (!L.a_exact) ptx::tma_load_2d(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, &full_bar[s]);
             }
             kb0 = pre;
             it += pre;
@@ -269,7 +271,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             ptx::mbar_arrive_expect_tx(&full_bar[s], tx);
             const int k0 = kb * GEMM_BK;
             ptx::tma_load_2d(a_hi(s), &L.a_hi, k0, m0, &full_bar[s]);
-            ptx::tma_load_2d(a_lo(s), &L.a_lo, k0, m0, &full_bar[s]);
+            if (!L.a_exact) ptx::tma_load_2d(a_lo(s), &L.a_lo, k0, m0, &full_bar[s]);
             ptx::tma_load_2d(b_hi(s), &L.b_hi, k0, n0, &full_bar[s]);
             ptx::tma_load_2d(b_lo(s), &L.b_lo, k0, n0, &full_bar[s]);
           }
@@ -291,6 +293,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
           ptx::tc_fence_after();
           const uint32_t d = tmem_base + acc * CHAIN_BN_MAX;
           const bool reuse = dataflow && l > 0 && L.reuse;
+          const bool a_exact = L.a_exact != 0;
           int own0 = 0, nown = 0;
           if (reuse) {
             const ChainLayer& Lp = P.layer[l - 1];
@@ -316,8 +319,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             for (int kk = 0; kk < GEMM_BK / GEMM_UMMA_K; ++kk) {
               const uint32_t off = kk * GEMM_UMMA_K * 2;
               const uint32_t acc0 = (i | kk) != 0;
-              ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(al + off), ptx::sdesc_k_sw128(bh + off), L.idesc, acc0);
-              ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bl + off), L.idesc, 1u);
+              if (!a_exact) ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(al + off), ptx::sdesc_k_sw128(bh + off), L.idesc, acc0);
+              ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bl + off), L.idesc, a_exact ? acc0 : 1u);
               ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bh + off), L.idesc, 1u);
             }
             ptx::mma_commit(&empty_bar[s]);
@@ -346,6 +349,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       // per-layer fields in registers once: read through the dynamically indexed param block, the
       // compiler otherwise re-fetches each pointer (LDC) before every element access
       const int epi = L.epi, bn = L.bn, ntn = L.n_tiles_n;
+      const bool hexact = L.head_exact != 0;   // HEAD: write the 0/1 mask (the next layer's weights carry -w)
       const int aM = L.args.M, aN = L.args.N, n_valid = L.args.n_valid, ld_f32 = L.args.ld_f32, ld_c = L.args.ld_c;
       const int ld_mask = L.args.ld_mask;
       const float* __restrict__ bias = L.args.bias;
@@ -451,7 +455,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
                   } else {
                     const float w = s_headw[n + i];
                     head_acc += (on ? z : 0.f) * w;
-                    v[i] = on ? -w : 0.f;        // delta_{L-1} = W_L^T (dL/dc = -1) (.) [Z > 0]
+                    v[i] = on ? (hexact ? 1.f : -w) : 0.f;   // delta_{L-1} = W_L^T (dL/dc = -1) (.) [Z > 0]
                   }
                 }
                 if (!head) s_mask[(ebuf * 2 + half) * GEMM_BM + r_tile] = bits;
@@ -481,7 +485,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             if (st0) CHAIN_STAMP2(l, 3);
             if (etid == 0) {
               ptx::tma_store_2d(tm_c_hi, n0 + c64, m0, epi_hi);
-              ptx::tma_store_2d(tm_c_lo, n0 + c64, m0, epi_lo);
+              if (!hexact) ptx::tma_store_2d(tm_c_lo, n0 + c64, m0, epi_lo);   // exact mask: lo = 0, never read
               if (epi == EPI_RELU) {   // the chunk's two mask-word columns (rows m0 .. m0+127; ld_mask >= padded rows)
                 ptx::bulk_s2g(mask_out + static_cast<size_t>((n0 + c64) / 32) * ld_mask + m0, s_mask + (ebuf * 2) * GEMM_BM, GEMM_BM * 4);
                 ptx::bulk_s2g(mask_out + static_cast<size_t>((n0 + c64) / 32 + 1) * ld_mask + m0, s_mask + (ebuf * 2 + 1) * GEMM_BM, GEMM_BM * 4);

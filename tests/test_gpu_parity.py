@@ -311,11 +311,13 @@ def test_shape_errors(fx):
 
 
 @pytest.mark.parametrize("mode,cg", [("chain", "1"), ("chain-cluster", "1"), ("chain-barrier", "1"), ("layers", "1"),
-                                     ("tile", "2")])
+                                     ("tile", "2"), ("chain-inexact", "1")])
 def test_mlp_execution_modes_agree(fx, mode, cg, monkeypatch):
     """The tile-local fused MLP (1-SM and 2-SM cta_group::2 variants), the persistent chain (dataflow
     flags, 4-CTA clusters, grid barriers) and the per-layer kernels compute the same split-fp16 products in the same K order: cost and gradient
-    agree to fp32 summation-order noise (the head partial sums are grouped differently)."""
+    agree to fp32 summation-order noise (the head partial sums are grouped differently).  The chain's
+    first backward layer takes the exact 0/1 mask with the head row folded into its weights (two MMA
+    passes); chain-inexact (FELIX_CHAIN_EXACT=0) is the three-pass form on -w (.) mask."""
     sp = fi.c2_space()
     mlp = fi.make_mlp(fi.DEFAULT_MLP)
     n = 2000
@@ -328,6 +330,7 @@ def test_mlp_execution_modes_agree(fx, mode, cg, monkeypatch):
     monkeypatch.setenv("FELIX_TILE_CG", cg)
     monkeypatch.setenv("FELIX_CHAIN_CS", "4" if mode == "chain-cluster" else "1")
     monkeypatch.setenv("FELIX_CHAIN_FLAGS", "0" if mode == "chain-barrier" else "1")
+    monkeypatch.setenv("FELIX_CHAIN_EXACT", "0" if mode == "chain-inexact" else "1")
     other = fx.Space(sp).eval(cm, y0, lam=1.0)
     for key in ("cost", "grad"):
         a, b = base[key].cpu().numpy(), other[key].cpu().numpy()
@@ -570,11 +573,14 @@ def _group_spaces():
 
 
 @pytest.mark.timeout(600)
-def test_search_group_equals_individual_searches(fx, monkeypatch):
+@pytest.mark.parametrize("sc", ["0", "1"])
+def test_search_group_equals_individual_searches(fx, sc, monkeypatch):
     """felix_search_group (one MLP pass per Adam step over the candidates of several spaces) computes
     every member's search exactly as felix_search does: with the tile kernel, whose per-row arithmetic
-    does not depend on the row's position, the final y and losses are bit-identical."""
+    does not depend on the row's position, the final y and losses are bit-identical (both with the
+    cone-group DAG kernels and with the split-cone ones, FELIX_SC)."""
     monkeypatch.setenv("FELIX_MLP", "tile")
+    monkeypatch.setenv("FELIX_SC", sc)
     mlp = fi.make_mlp(fi.DEFAULT_MLP)
     cm = fx.CostModel.from_weights(mlp)
     sps, ns = _group_spaces()
@@ -627,3 +633,69 @@ def test_search_group_errors(fx):
     y = torch.zeros((sp.n_vars, 64), device="cuda")
     with pytest.raises(fx.FelixError):
         fx.search_group([sp, sp], cm, [y, y.clone()], 2)          # a space twice
+
+
+@pytest.mark.parametrize("name,n,steps,P,W,chunks", [
+    ("C2", 1000, 7, "4", "", "1"), ("C2", 4096, 8, "4", "", "1"), ("C2", 1000, 5, "8", "3", "1"),
+    ("C2_2stmt", 700, 6, "4", "2", "1"), ("bmm", 257, 5, "2", "1", "1"), ("C2", 3000, 6, "4", "", "2"),
+    ("C5", 389, 9, "1", "", "1"), ("C5", 389, 8, "2", "", "1"), ("r50_conv1", 300, 4, "4", "1", "1"),
+    ("C2", 1000, 1, "4", "", "1")])
+def test_split_cone_kernels_match_cone_groups(fx, name, n, steps, P, W, chunks, monkeypatch):
+    """Split-cone reverse kernel (one cone per CTA, partial adjoints through global memory; the next
+    step's forward sums them and applies Adam in place, felix_adam_sc after the last step) against the
+    cone-group kernels over several Adam steps (ragged n, several chunks, P = 1..8): the same arithmetic
+    in the same order, so y and the final loss agree to fp32 rounding; the one-step result is also
+    checked against the oracle."""
+    make, dims, _ = CASES[name]
+    sp = make()
+    mlp = fi.make_mlp(dims)
+    cm = fx.CostModel.from_weights(mlp)
+    y0 = fi.make_y0(sp, n, seed=77)
+    monkeypatch.setenv("FELIX_P", P)
+    monkeypatch.setenv("FELIX_CHUNKS", chunks)
+    if W:
+        monkeypatch.setenv("FELIX_SCW", W)
+    out = {}
+    for sc in ("0", "1"):
+        monkeypatch.setenv("FELIX_SC", sc)
+        space = fx.Space(sp)
+        y = torch.from_numpy(y0).cuda()
+        loss = torch.empty(n, device="cuda")
+        space.search(cm, y, steps, init_from_y=True, final_loss=loss)
+        y1 = torch.from_numpy(y0).cuda()
+        space.search(cm, y1, 1, init_from_y=True)
+        out[sc] = (y.cpu().numpy(), loss.cpu().numpy(), y1.cpu().numpy())
+    (ya, la, y1a), (yb, lb, y1b) = out["0"], out["1"]
+    assert np.all(np.isfinite(yb)) and np.all(np.isfinite(lb))
+    same = np.mean(ya == yb)
+    print(f"{name} n={n} steps={steps} P={P}: exactly equal y {same:.4f}, max |dy| {np.max(np.abs(ya - yb)):.3e}")
+    assert np.max(np.abs(y1a - y1b)) <= 1e-5 * (1 + np.max(np.abs(y1a)))
+    assert np.mean(np.abs(ya - yb) <= 1e-4 * (1 + np.abs(ya))) >= 0.99
+    s = np.sqrt(np.mean(la.astype(np.float64) ** 2))
+    assert np.mean(np.abs(la - lb) <= 1e-4 * s) >= 0.99
+    ry, _, _, _ = fo.search(sp, mlp.W, mlp.b, y0, 1, lr=0.05, lam=1.0)
+    ob = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
+    exempt = (np.abs(ob.grad) < 1e-6) | (kink_margin(ob.zs) < 1e-4)[None, :]
+    assert not np.any((np.abs(y1b - ry) > 1e-4 * (1 + np.abs(ry))) & ~exempt)
+
+
+@pytest.mark.parametrize("name,n", [("C2", 4096), ("C1", 300), ("C2_2stmt", 700), ("r50_conv1", 129)])
+def test_scoring_kernels_bit_identical(fx, name, n, monkeypatch):
+    """FP64 scoring: the 128 x 64 register-blocked layer kernel and the row-staged head kernel run the
+    same fma sequence per output (bias first, k ascending) as the 64 x 64 kernels (FELIX_SCORE=1), so the
+    scores are bit-identical; both match the oracle to 1e-12."""
+    make, dims, _ = CASES[name]
+    sp = make()
+    mlp = fi.make_mlp(dims)
+    cm = fx.CostModel.from_weights(mlp)
+    space = fx.Space(sp)
+    rs = fo.round_schedules(sp, fi.make_y0(sp, n, seed=15))
+    sched = torch.from_numpy(rs).cuda()
+    monkeypatch.setenv("FELIX_SCORE", "1")
+    old = space.score(cm, sched).cpu().numpy()
+    monkeypatch.setenv("FELIX_SCORE", "0")
+    new = space.score(cm, sched).cpu().numpy()
+    assert np.array_equal(old, new, equal_nan=True)
+    ref = fo.score(sp, mlp.W, mlp.b, rs)
+    ok = np.isfinite(ref)
+    assert np.all(np.abs(new[ok] - ref[ok]) <= 1e-12 * np.maximum(np.abs(ref[ok]), 1e-3))

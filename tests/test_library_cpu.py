@@ -83,7 +83,8 @@ def test_validator_rejects(fx, case, status):
 def test_generated_kernels_compile_for_sm100a(fx, which):
     sp = {"paper": fi.paper_example_space, "C1": fi.c1_space, "C2": fi.c2_space}[which]()
     src = fx.codegen(sp, compile=True)
-    for k in ("felix_fwd", "felix_rev_adam", "felix_rev_eval", "felix_hard", "felix_init"):
+    for k in ("felix_fwd", "felix_rev_adam", "felix_rev_eval", "felix_hard", "felix_init", "felix_fwd_adam", "felix_rev_sc",
+              "felix_adam_sc"):
         assert re.search(r"__global__ void __launch_bounds__\([^)]*\) " + k + r"\(", src), k
 
 
