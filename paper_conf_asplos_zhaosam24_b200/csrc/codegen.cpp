@@ -803,16 +803,20 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
   // Measured and dropped: Adam by the last of the P cone CTAs to arrive (+8 us at C2: a serial tail at
   // 255 registers), and a split-cone forward (its 2-byte feature-column stores: 1.7x slower at C2).
   o << "extern \"C\" __global__ void __launch_bounds__(256) felix_rev_sc(const float* __restrict__ yv, int n, int ldy, const float* __restrict__ dphi, int ld_dphi,\n"
-    << "    float lam, double* __restrict__ part, double* __restrict__ pen, int* step_ctr) {\n"
+    << "    float lam, double* __restrict__ part, double* __restrict__ pen, int* step_ctr, int G) {\n"
     << "  const int cq_ = blockIdx.x % PG;\n"
-    << "  const int c = ((blockIdx.x / PG) * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32 + (threadIdx.x & 31);\n"
-    << "  const bool live = c < n;\n  const int ccw = live ? c : n - 1;\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n"
     << "  if (blockIdx.x == 0 && threadIdx.x == 0) *step_ctr += 1;\n"
     << "  const double dlam = (double)lam;\n";
+  // G groups of W x 32 candidates per CTA, one after the other: the second pass over the cone's
+  // straight-line code runs from the instruction caches the first one filled
   for (int q = 0; q < P; ++q) {
-    o << "  if (cq_ == " << q << ") {\n";
+    o << "  if (cq_ == " << q << ") {\n"
+      << "#pragma unroll 1\n"
+      << "  for (int g_ = 0; g_ < G; ++g_) {\n"
+      << "    const int c = (((blockIdx.x / PG) * G + g_) * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32 + (threadIdx.x & 31);\n"
+      << "    const bool live = c < n;\n    const int ccw = live ? c : n - 1;\n";
     const auto used = vars_in(rcone[q]);
     for (int j = 0; j < M; ++j)
       if (used[j]) o << "    const double x" << j << " = exp((double)yv[(size_t)" << j << " * ldy + ccw]);\n";
@@ -834,7 +838,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     g.emit_reverse_body(need, "    ");
     o << "    if (live) {\n      pen[(size_t)" << q << " * n + c] = pq;\n";
     for (int j = 0; j < M; ++j) o << "      part[((size_t)" << q << " * NV + " << j << ") * n + c] = (double)gx" << j << ";\n";
-    o << "    }\n  }\n";
+    o << "    }\n  }\n  }\n";
   }
   o << "}\n\n";
   // felix_adam_sc: the last Adam step (thread per candidate, in place) + the final loss

@@ -113,8 +113,8 @@ static CUtensorMap make_tmap(const void* base, int64_t rows, int64_t cols, int b
 }
 
 // ============================================================================ per-(space, model, n) plan
-static bool chain_exact() {
-  const char* e = std::getenv("FELIX_CHAIN_EXACT");
+static bool mask_exact() {
+  const char* e = std::getenv("FELIX_MASK_EXACT");
   return !(e && std::atoi(e) == 0);
 }
 struct Plan {
@@ -609,11 +609,19 @@ static int choose_scw(int64_t n, int P) {
   int64_t w = (groups * P + 147) / 148;
   return static_cast<int>(std::max<int64_t>(1, std::min<int64_t>(8, w)));
 }
+// groups of W x 32 candidates each split-cone CTA runs one after the other (FELIX_SCG overrides)
+static int choose_scg() {
+  if (const char* e = std::getenv("FELIX_SCG")) {
+    const int g = std::atoi(e);
+    if (g >= 1 && g <= 16) return g;
+  }
+  return 1;
+}
 static int64_t sc_groups(int64_t n, int W) { return ((n + 31) / 32 + W - 1) / W; }
-static void launch_sc(cudaKernel_t f, int P, int W, int64_t n, void** args, cudaStream_t st, bool pdl) {
+static void launch_sc(cudaKernel_t f, int P, int W, int G, int64_t n, void** args, cudaStream_t st, bool pdl) {
   if (n <= 0) return;
-  launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>(sc_groups(n, W) * P)), dim3(32 * W), 0, args,
-             st, pdl);
+  launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((sc_groups(n, W) + G - 1) / G * P)), dim3(32 * W),
+             0, args, st, pdl);
 }
 
 // ============================================================================ plan
@@ -757,10 +765,10 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     L.b_hi = make_tmap(g.w_hi, N, g.args.K, bn);
     L.b_lo = make_tmap(g.w_lo, N, g.args.K, bn);
     // the first backward layer takes the 0/1 mask of the head layer as its A operand and the head row
-    // folded into its weights (exact A: two MMA passes, no A lo loads); FELIX_CHAIN_EXACT=0 disables
+    // folded into its weights (exact A: two MMA passes, no A lo loads); FELIX_MASK_EXACT=0 disables
     L.a_exact = 0;
     L.head_exact = 0;
-    if (i == static_cast<size_t>(cm->n_layers - 1) && i > 0 && chain_exact() && p->gemms[i - 1].epi == EPI_HEAD) {
+    if (i == static_cast<size_t>(cm->n_layers - 1) && i > 0 && mask_exact() && p->gemms[i - 1].epi == EPI_HEAD) {
       L.a_exact = 1;
       p->chain.layer[i - 1].head_exact = 1;
       L.b_hi = make_tmap(cm->WTs_hi.p, N, g.args.K, bn);
@@ -815,8 +823,10 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     t.w2_lo = make_tmap(cm->W_lo[1]->p, d[2], d[1], 128);
     t.w3_hi = make_tmap(cm->W_hi[2]->p, d[3], d[2], 128);
     t.w3_lo = make_tmap(cm->W_lo[2]->p, d[3], d[2], 128);
-    t.w3t_hi = make_tmap(cm->WT_hi[2]->p, d[2], d[3], 128);
-    t.w3t_lo = make_tmap(cm->WT_lo[2]->p, d[2], d[3], 128);
+    // B1 on the exact mask with the head row folded into W3^T (as the chain's first backward layer)
+    t.d2_exact = mask_exact() ? 1 : 0;
+    t.w3t_hi = make_tmap(t.d2_exact ? cm->WTs_hi.p : cm->WT_hi[2]->p, d[2], d[3], 128);
+    t.w3t_lo = make_tmap(t.d2_exact ? cm->WTs_lo.p : cm->WT_lo[2]->p, d[2], d[3], 128);
     t.w2t_hi = make_tmap(cm->WT_hi[1]->p, d[1], d[2], 128 / cg);
     t.w2t_lo = make_tmap(cm->WT_lo[1]->p, d[1], d[2], 128 / cg);
     t.w1t_hi = make_tmap(cm->WT_hi[0]->p, K0p, d[1], K0p / cg);
@@ -1216,7 +1226,8 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
   const bool sc = use_sc() && !p->history;
   const int P0 = choose_P(ch.cnt[0]);
   const felix_space::Module& mod = sc ? get_module(s, choose_P_sc(P0), choose_R_sc()) : get_module(s, P0, choose_R(ch.cnt[0], P0));
-  const int scw = choose_scw(ch.cnt[0], mod.P);
+  const int scg = choose_scg();
+  const int scw = choose_scw((ch.cnt[0] + scg - 1) / scg, mod.P);
   if (!p->init_from_y) {
     unsigned long long seed = p->rng_seed;
     long long ib = p->index_base;
@@ -1304,9 +1315,10 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
       prof_mark(s, 0, cs, false);
       s->prof_launches[0] += 1;
       run_mlp(s, pl, cs);
-      void* ra[] = {&yk, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr};
+      int scg_ = scg;
+      void* ra[] = {&yk, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr, &scg_};
       prof_mark(s, 2, cs, true);
-      launch_sc(mod.f_rev_sc, mod.P, scw, cnt, ra, cs, true);
+      launch_sc(mod.f_rev_sc, mod.P, scw, scg, cnt, ra, cs, true);
       prof_mark(s, 2, cs, false);
       s->prof_launches[2] += 1;
       return;
@@ -1334,7 +1346,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     // (a per-step fork/join would re-synchronise them every step).  Joined once at the end.
     auto ptr = [](const void* q) { return static_cast<double>(reinterpret_cast<uintptr_t>(q)); };
     const std::vector<double> key = {static_cast<double>(mod.P), ptr(y), ptr(final_loss), lam0, lr0, b10, b20, eps0,
-                                     static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R),
+                                     static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R), static_cast<double>(scg),
                                      ptr(ch.plans[0]->sc_part.p), ptr(ch.plans[0]->sc_pen.p)};
     while (static_cast<int>(ch.streams.size()) < nck) {
       cudaStream_t b;
@@ -1389,7 +1401,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
                                      static_cast<double>(s->h_valid), ptr(s->h_sched.p), ptr(s->h_last.p),
                                      ptr(s->h_slot_h.p), ptr(s->h_pool_sched.p), ptr(s->h_pool_key.p),
                                      static_cast<double>(s->h_mask), static_cast<double>(s->h_cap),
-                                     static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R),
+                                     static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R), static_cast<double>(scg),
                                      ptr(ch.plans[0]->sc_part.p), ptr(ch.plans[0]->sc_pen.p)};
     if (!ch.graph || ch.graph_key != key) {
       if (ch.graph) { cudaGraphExecDestroy(ch.graph); ch.graph = nullptr; }
@@ -1617,8 +1629,9 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
       if (sc) {
         void* part = gc.sc_part[i]->p;
         void* pen = gc.sc_pen[i]->p;
-        void* ra[] = {&yi, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr};
-        launch_sc(mods[i]->f_rev_sc, mods[i]->P, scws[i], p.n_seeds, ra, si, false);
+        int scg = 1;
+        void* ra[] = {&yi, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr, &scg};
+        launch_sc(mods[i]->f_rev_sc, mods[i]->P, scws[i], 1, p.n_seeds, ra, si, false);
         continue;
       }
       void* args[] = {&yi, &ni, &ldy, &dphi, &ld, &cpart, &nht, &ld, &hbv, &lam, &mv, &vv, &ctr, &lr, &b1, &b2, &eps, &lo};

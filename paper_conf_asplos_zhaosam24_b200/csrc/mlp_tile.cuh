@@ -70,6 +70,7 @@ struct TileParams {
   int n_tiles;                         // 128-row tiles
   int k0p;                             // padded feature count (<= 128, multiple of 32)
   int n_valid;                         // real feature count
+  int d2_exact;                        // B1 takes the exact 0/1 mask [Z3 > 0] (w3t = W3^T diag(-w4)): 2 passes
   uint32_t idesc_128, idesc_256, idesc_k0p;   // M = 128*CG; N = 128 / 256 / K0p
   unsigned long long* trace;           // FELIX_TILE_TRACE builds only: [grid][32] timestamps
 };
@@ -109,13 +110,13 @@ __device__ __forceinline__ void arrive_leader(uint64_t* bar) {
 // 4 K-steps x 3 split passes of one 64-wide K block: D (+)= A[128 x 64] * B[N x 64]^T
 template <int CG>
 __device__ __forceinline__ void mma_kblock(uint32_t d, uint32_t a_hi, uint32_t a_lo, uint32_t b_hi, uint32_t b_lo,
-                                           uint32_t idesc, bool accumulate) {
+                                           uint32_t idesc, bool accumulate, bool a_exact = false) {
   const uint64_t dah = ptx::sdesc_k_sw128(a_hi), dal = ptx::sdesc_k_sw128(a_lo);
   const uint64_t dbh = ptx::sdesc_k_sw128(b_hi), dbl = ptx::sdesc_k_sw128(b_lo);
 #pragma unroll
   for (int kk = 0; kk < 4; ++kk) {           // +32 B along K = +2 in the descriptor's address field
-    mma<CG>(d, dal + 2 * kk, dbh + 2 * kk, idesc, (accumulate || kk) ? 1u : 0u);
-    mma<CG>(d, dah + 2 * kk, dbl + 2 * kk, idesc, 1u);
+    if (!a_exact) mma<CG>(d, dal + 2 * kk, dbh + 2 * kk, idesc, (accumulate || kk) ? 1u : 0u);   // A lo = 0 if exact
+    mma<CG>(d, dah + 2 * kk, dbl + 2 * kk, idesc, (!a_exact || accumulate || kk) ? 1u : 0u);
     mma<CG>(d, dah + 2 * kk, dbh + 2 * kk, idesc, 1u);
   }
 }
@@ -312,7 +313,7 @@ __global__ void __launch_bounds__(tile::THREADS, 1) mlp_tile_kernel(const __grid
       uint32_t it = 0;                                // ring entries consumed
       uint32_t hseq = 0, d1seq = 0, z1seq = 0, d1accseq = 0;
       // one logical GEMM step of width N into accumulator d (A = one 64-wide K block in smem)
-      auto step = [&](uint32_t d, uint8_t* a_chunk, int N, uint32_t idesc, bool accumulate) {
+      auto step = [&](uint32_t d, uint8_t* a_chunk, int N, uint32_t idesc, bool accumulate, bool a_exact = false) {
         const int per = N / CG;
         const int nsub = per <= 128 ? 1 : per / 128;
         const uint32_t ah = ptx::smem_u32(a_chunk), al = ah + HALF_BYTES;
@@ -321,7 +322,7 @@ __global__ void __launch_bounds__(tile::THREADS, 1) mlp_tile_kernel(const __grid
           wait_k<CG>(&ring_full[slot], it / RING);
           ptx::tc_fence_after();
           const uint32_t bh = ptx::smem_u32(ring_hi(slot));
-          mma_kblock<CG>(d + s * (N / nsub), ah, al, bh, bh + HALF_BYTES, idesc, accumulate);
+          mma_kblock<CG>(d + s * (N / nsub), ah, al, bh, bh + HALF_BYTES, idesc, accumulate, a_exact);
           commit<CG>(&ring_empty[slot]);
           ++it;
         }
@@ -333,11 +334,11 @@ __global__ void __launch_bounds__(tile::THREADS, 1) mlp_tile_kernel(const __grid
         wait_k<CG>(phi_full, t);
         TILE_STAMP(1);
         ptx::tc_fence_after();
-        auto consume_h = [&](uint32_t dacc, int N, uint32_t idesc, bool accumulate) {
+        auto consume_h = [&](uint32_t dacc, int N, uint32_t idesc, bool accumulate, bool a_exact = false) {
           const int b = hseq & 1;
           wait_k<CG>(&a_ready[b], hseq >> 1);
           ptx::tc_fence_after();
-          step(dacc, hbuf(b), N, idesc, accumulate);
+          step(dacc, hbuf(b), N, idesc, accumulate, a_exact);
           commit<CG>(&a_free[b]);
           ++hseq;
         };
@@ -361,7 +362,7 @@ __global__ void __launch_bounds__(tile::THREADS, 1) mlp_tile_kernel(const __grid
         TILE_STAMP(3);
         commit<CG>(z3_full);
         // ---- B1: D2 += delta3_j W3^T
-        for (int j = 0; j < D3 / 64; ++j) consume_h(tmem + T_D2, D2, id_n256, j > 0);
+        for (int j = 0; j < D3 / 64; ++j) consume_h(tmem + T_D2, D2, id_n256, j > 0, P.d2_exact != 0);
         TILE_STAMP(4);
         commit<CG>(d2_full);
         // ---- B3
@@ -474,7 +475,7 @@ __global__ void __launch_bounds__(tile::THREADS, 1) mlp_tile_kernel(const __grid
         float v[32];
         const int n0 = j * 64 + h * 32;
 #pragma unroll
-        for (int i = 0; i < 32; ++i) v[i] = ((m3w[j] >> i) & 1u) ? -__ldg(&P.w4[n0 + i]) : 0.f;
+        for (int i = 0; i < 32; ++i) v[i] = ((m3w[j] >> i) & 1u) ? (P.d2_exact ? 1.f : -__ldg(&P.w4[n0 + i])) : 0.f;
         tile::put_h<CG>(R0, a_free, a_ready, hseq, r, h, lane, v);
       }
       if (warp == 2 && lane == 0) TILE_STAMP(14);

@@ -311,13 +311,14 @@ def test_shape_errors(fx):
 
 
 @pytest.mark.parametrize("mode,cg", [("chain", "1"), ("chain-cluster", "1"), ("chain-barrier", "1"), ("layers", "1"),
-                                     ("tile", "2"), ("chain-inexact", "1")])
+                                     ("tile", "2"), ("chain-inexact", "1"), ("tile-inexact", "1")])
 def test_mlp_execution_modes_agree(fx, mode, cg, monkeypatch):
     """The tile-local fused MLP (1-SM and 2-SM cta_group::2 variants), the persistent chain (dataflow
     flags, 4-CTA clusters, grid barriers) and the per-layer kernels compute the same split-fp16 products in the same K order: cost and gradient
     agree to fp32 summation-order noise (the head partial sums are grouped differently).  The chain's
     first backward layer takes the exact 0/1 mask with the head row folded into its weights (two MMA
-    passes); chain-inexact (FELIX_CHAIN_EXACT=0) is the three-pass form on -w (.) mask."""
+    passes), and so does the tile kernel's B1 step; *-inexact (FELIX_MASK_EXACT=0) is the three-pass
+    form on -w (.) mask."""
     sp = fi.c2_space()
     mlp = fi.make_mlp(fi.DEFAULT_MLP)
     n = 2000
@@ -330,7 +331,7 @@ def test_mlp_execution_modes_agree(fx, mode, cg, monkeypatch):
     monkeypatch.setenv("FELIX_TILE_CG", cg)
     monkeypatch.setenv("FELIX_CHAIN_CS", "4" if mode == "chain-cluster" else "1")
     monkeypatch.setenv("FELIX_CHAIN_FLAGS", "0" if mode == "chain-barrier" else "1")
-    monkeypatch.setenv("FELIX_CHAIN_EXACT", "0" if mode == "chain-inexact" else "1")
+    monkeypatch.setenv("FELIX_MASK_EXACT", "0" if mode.endswith("inexact") else "1")
     other = fx.Space(sp).eval(cm, y0, lam=1.0)
     for key in ("cost", "grad"):
         a, b = base[key].cpu().numpy(), other[key].cpu().numpy()
@@ -639,7 +640,8 @@ def test_search_group_errors(fx):
     ("C2", 1000, 7, "4", "", "1"), ("C2", 4096, 8, "4", "", "1"), ("C2", 1000, 5, "8", "3", "1"),
     ("C2_2stmt", 700, 6, "4", "2", "1"), ("bmm", 257, 5, "2", "1", "1"), ("C2", 3000, 6, "4", "", "2"),
     ("C5", 389, 9, "1", "", "1"), ("C5", 389, 8, "2", "", "1"), ("r50_conv1", 300, 4, "4", "1", "1"),
-    ("C2", 1000, 1, "4", "", "1")])
+    ("C2", 1000, 1, "4", "", "1"), ("C2", 1000, 6, "8", "2:2", "1"), ("C2", 4096, 5, "8", "4:2", "1"),
+    ("C2_2stmt", 700, 5, "4", "1:3", "1")])
 def test_split_cone_kernels_match_cone_groups(fx, name, n, steps, P, W, chunks, monkeypatch):
     """Split-cone reverse kernel (one cone per CTA, partial adjoints through global memory; the next
     step's forward sums them and applies Adam in place, felix_adam_sc after the last step) against the
@@ -653,8 +655,9 @@ def test_split_cone_kernels_match_cone_groups(fx, name, n, steps, P, W, chunks, 
     y0 = fi.make_y0(sp, n, seed=77)
     monkeypatch.setenv("FELIX_P", P)
     monkeypatch.setenv("FELIX_CHUNKS", chunks)
-    if W:
-        monkeypatch.setenv("FELIX_SCW", W)
+    if W:   # "W" or "W:G" (G groups of W x 32 candidates per reverse CTA, one after the other)
+        monkeypatch.setenv("FELIX_SCW", W.split(":")[0])
+        monkeypatch.setenv("FELIX_SCG", W.split(":")[1] if ":" in W else "1")
     out = {}
     for sc in ("0", "1"):
         monkeypatch.setenv("FELIX_SC", sc)
