@@ -201,23 +201,23 @@ __global__ void __launch_bounds__(256) score_layer_kernel(const double* __restri
 
 // ---------------------------------------------------------------------------- K6 FP64 MLP scoring (v2)
 // Same arithmetic again (acc = b[col]; k ascending: acc = fma(W[col][k], in(row, k), acc)), bit-identical
-// to the kernels above.  128 x 64 output tile per 256-thread block; thread (tx, ty) owns rows ty + 16 i
-// (i < 8) and columns tx + 16 j (j < 4), 32 FP64 accumulators: per k, 8 + 4 conflict-free shared loads
-// (a warp reads 2 distinct A addresses and 16 consecutive W doubles) feed 32 DFMA.  K is staged 16 at a
+// to the kernels above.  128 x 64 output tile per 256-thread block; thread (tx, ty) owns rows ty * 8 + i
+// (i < 8) and 4 columns, 32 FP64 accumulators: per k, 4 + 2 16-byte shared loads (6 wavefronts per warp)
+// feed 32 DFMA.  K is staged 16 at a
 // time through double-buffered shared memory filled one chunk ahead from registers, one barrier per chunk.
 constexpr int SC2_TM = 128, SC2_TN = 64, SC2_KT = 16;
 __global__ void __launch_bounds__(256) score_layer_v2_kernel(const double* __restrict__ in, long long in_rs, long long in_cs,
                                                              int n, int K, const double* __restrict__ W,
                                                              const double* __restrict__ b, double* __restrict__ out,
                                                              int N, int relu, int accumulate) {
-  __shared__ double As[2][SC2_KT][SC2_TM];   // [buf][k][row]
-  __shared__ double Bs[2][SC2_KT][SC2_TN];   // [buf][k][col]
+  __shared__ __align__(16) double As[2][SC2_KT][SC2_TM];   // [buf][k][row]
+  __shared__ __align__(16) double Bs[2][SC2_KT][SC2_TN];   // [buf][k][col]
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
   const int row0 = blockIdx.y * SC2_TM, col0 = blockIdx.x * SC2_TN;
   double acc[8][4];
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
-    const int col = col0 + tx + 16 * j;
+    const int col = col0 + (j < 2 ? 2 * tx + j : 32 + 2 * tx + (j - 2));
     const double bj = col < N ? b[col] : 0.0;
 #pragma unroll
     for (int i = 0; i < 8; ++i) acc[i][j] = bj;
@@ -263,42 +263,39 @@ __global__ void __launch_bounds__(256) score_layer_v2_kernel(const double* __res
     const int buf = c & 1;
     if (c + 1 < nk) load_chunk((c + 1) * SC2_KT);
     const int kmax = min(SC2_KT, K - c * SC2_KT);
+    // thread (tx, ty): rows ty * 8 .. + 7 (4 x 16-B loads, two distinct addresses per warp: broadcast) and
+    // columns 2 tx, 2 tx + 1, 32 + 2 tx, 33 + 2 tx (2 x 16-B loads over 256 consecutive bytes: 2 wavefronts)
+    auto kstep = [&](int kk) {
+      double a[8], w[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const double2 v = *reinterpret_cast<const double2*>(&As[buf][kk][ty * 8 + 2 * i]);
+        a[2 * i] = v.x; a[2 * i + 1] = v.y;
+      }
+      const double2 w01 = *reinterpret_cast<const double2*>(&Bs[buf][kk][2 * tx]);
+      const double2 w23 = *reinterpret_cast<const double2*>(&Bs[buf][kk][32 + 2 * tx]);
+      w[0] = w01.x; w[1] = w01.y; w[2] = w23.x; w[3] = w23.y;
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fma(w[j], a[i], acc[i][j]);
+    };
     if (kmax == SC2_KT) {
 #pragma unroll
-      for (int kk = 0; kk < SC2_KT; ++kk) {
-        double a[8], w[4];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) a[i] = As[buf][kk][ty + 16 * i];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) w[j] = Bs[buf][kk][tx + 16 * j];
-#pragma unroll
-        for (int i = 0; i < 8; ++i)
-#pragma unroll
-          for (int j = 0; j < 4; ++j) acc[i][j] = fma(w[j], a[i], acc[i][j]);
-      }
+      for (int kk = 0; kk < SC2_KT; ++kk) kstep(kk);
     } else {
-      for (int kk = 0; kk < kmax; ++kk) {
-        double a[8], w[4];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) a[i] = As[buf][kk][ty + 16 * i];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) w[j] = Bs[buf][kk][tx + 16 * j];
-#pragma unroll
-        for (int i = 0; i < 8; ++i)
-#pragma unroll
-          for (int j = 0; j < 4; ++j) acc[i][j] = fma(w[j], a[i], acc[i][j]);
-      }
+      for (int kk = 0; kk < kmax; ++kk) kstep(kk);
     }
     if (c + 1 < nk) store_chunk(buf ^ 1);   // the other buffer was last read in chunk c - 1 (barrier below)
     __syncthreads();
   }
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
-    const int r = row0 + ty + 16 * i;
+    const int r = row0 + ty * 8 + i;
     if (r >= n) continue;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-      const int col = col0 + tx + 16 * j;
+      const int col = col0 + (j < 2 ? 2 * tx + j : 32 + 2 * tx + (j - 2));
       if (col >= N) continue;
       const double v = (relu && !(acc[i][j] > 0.0)) ? 0.0 : acc[i][j];
       out[static_cast<size_t>(r) * N + col] = accumulate ? out[static_cast<size_t>(r) * N + col] + v : v;

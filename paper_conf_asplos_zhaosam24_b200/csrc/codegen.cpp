@@ -542,17 +542,18 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "      yl[jj] = yv[(size_t)j * ldy + cc]; ml[jj] = mv[(size_t)j * n + cc]; vl[jj] = vv[(size_t)j * n + cc];\n"
     << "      double a = 0.0;\n#pragma unroll\n      for (int q = 0; q < PG; ++q) a += part[((size_t)q * NV + j) * n + cc];\n"
     << "      gxa[jj] = a;\n    }\n"
+    // the loss inputs are requested with the rest (one memory round trip before the first barrier)
+    << "    double pen_ = 0.0;\n"
+    << "#pragma unroll\n    for (int q = 0; q < PG; ++q) pen_ += pen[(size_t)q * n + cc];\n"
+    << "    float cst = head_b * NS;\n"
+    << "#pragma unroll 4\n    for (int i = 0; i < NS * n_head_tiles; ++i) cst += c_part[(size_t)(i % n_head_tiles) * ld_c + (size_t)(i / n_head_tiles) * n + cc];\n"
     << "    const int s_ = *step_ctr - 1;   // Adam steps to apply: reverse kernels run so far (the counter starts at 1)\n"
     << "#pragma unroll\n    for (int jj = 0; jj < NJ; ++jj) { const int j = wq + PG * jj; if (j >= NV) break; sy[j][lane] = yl[jj]; }\n"
     << "    __syncthreads();\n"
     << "    if (s_ <= 0) {\n"
     << "#pragma unroll\n      for (int jj = 0; jj < NJ; ++jj) { const int j = wq + PG * jj; if (j >= NV) break; sx[j][lane] = exp((double)yl[jj]); }\n"
     << "    } else {\n"
-    << "      const double dlam = (double)lam;\n"
-    << "      double pen_ = 0.0;\n"
-    << "#pragma unroll\n      for (int q = 0; q < PG; ++q) pen_ += pen[(size_t)q * n + cc];\n"
-    << "      float cst = head_b * NS;\n"
-    << "      for (int i = 0; i < NS * n_head_tiles; ++i) cst += c_part[(size_t)(i % n_head_tiles) * ld_c + (size_t)(i / n_head_tiles) * n + cc];\n";
+    << "      const double dlam = (double)lam;\n";
   emit_autos("      ", "sy");
   o << "      const float loss = (float)(-(double)cst + dlam * pen_);\n"
     << "      bool ok = isfinite(loss);\n"
