@@ -19,6 +19,9 @@
 //   felix_rev_eval   same, writing phi / g / cost / loss / grad instead of updating y
 //   felix_hard       hard semantics in FP64 (IEEE ops) at integer points -> slog features + validity
 //   felix_init       rejection sampler (FP64 decisions, counter-based RNG)
+//   felix_rev_sc     split-cone reverse (default search path): one cone per CTA, partial adjoints per cone
+//   felix_fwd_adam   felix_fwd preceded by Adam step t-1 from those partials (in place)
+//   felix_adam_sc    the last Adam step of a split-cone search
 #include <algorithm>
 #include <climits>
 #include <cmath>
