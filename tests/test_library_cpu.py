@@ -95,3 +95,47 @@ def test_device_calls_fail_loudly_without_gpu(fx):
     with pytest.raises(fx.FelixError) as e:
         fx.Space(fi.c1_space())
     assert e.value.status == 5
+
+
+def _kernel_body(src, name):
+    i = src.index(" " + name + "(")
+    j = src.find('extern "C" __global__', i + 1)
+    return src[i:j if j > 0 else len(src)]
+
+
+@pytest.mark.parametrize("P", ["1", "2", "4", "8"])
+def test_split_cone_codegen_partitions_every_seed_once(fx, P, monkeypatch):
+    """The generated split-cone reverse kernel has one branch per cone, seeds every variable-dependent
+    feature's adjoint from dL/dphi exactly once across the cones (the cone partition covers the roots
+    without overlap), and each cone writes a partial adjoint for every variable; the cone-group reverse
+    kernel (felix_rev_adam's body) seeds the same features once.  felix_fwd_adam applies step
+    *step_ctr - 1 (the reverse kernel advances the counter)."""
+    monkeypatch.setenv("FELIX_CODEGEN_P", P)
+    monkeypatch.setenv("FELIX_CODEGEN_R", "1")
+    sp = fi.c2_space()
+    src = fx.codegen(sp)
+    rev = _kernel_body(src, "felix_rev_sc")
+    assert len(re.findall(r"if \(cq_ == \d+\)", rev)) == int(P)
+    seeds = re.findall(r"dphi\[\(size_t\)(\d+) \* ld_dphi", rev)
+    n_dep = sum(1 for r in sp.feature_roots if _depends_on_var(sp, r))
+    assert sorted(int(k) for k in seeds) == sorted(set(int(k) for k in seeds)) and len(seeds) == n_dep
+    for q in range(int(P)):
+        for j in range(sp.n_vars):
+            assert f"part[((size_t){q} * NV + {j}) * n + c]" in rev
+    body = src[src.index("void rev_body("):src.index('extern "C" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_adam')]
+    assert sorted(re.findall(r"dphi\[\(size_t\)(\d+) \* ld_dphi", body)) == sorted(seeds)
+    assert "*step_ctr - 1" in src and "*step_ctr += 1" in rev
+
+
+def _depends_on_var(sp, root):
+    seen, stack = set(), [root]
+    while stack:
+        i = stack.pop()
+        if i in seen:
+            continue
+        seen.add(i)
+        op, a, b, c, _ = sp.nodes[i]
+        if op == fi.OP_VAR:
+            return True
+        stack.extend(x for x in (a, b, c) if x >= 0)
+    return False
