@@ -303,28 +303,18 @@ __global__ void __launch_bounds__(256) score_layer_v2_kernel(const double* __res
   }
 }
 
-// head layer (N = 1, row-major input [n][K]): thread per row, K staged 32 at a time through shared memory
-// (coalesced row segments), same fma order as above
-__global__ void __launch_bounds__(128) score_head_kernel(const double* __restrict__ in, int n, int K,
-                                                         const double* __restrict__ W, const double* __restrict__ b,
-                                                         double* __restrict__ out, int accumulate) {
-  __shared__ double Ts[128][33];
-  const int row0 = blockIdx.x * 128, t = threadIdx.x;
+// head layer (N = 1, row-major input [n][K]): thread per row streaming its own row (the L1 serves the
+// 16 doubles of each 128-B line), one-warp blocks so the rows spread over the SMs; same fma order as above
+__global__ void __launch_bounds__(32) score_head_kernel(const double* __restrict__ in, int n, int K,
+                                                        const double* __restrict__ W, const double* __restrict__ b,
+                                                        double* __restrict__ out, int accumulate) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= n) return;
+  const double* __restrict__ row = in + static_cast<size_t>(r) * K;
   double acc = b[0];
-  for (int k0 = 0; k0 < K; k0 += 32) {
-    const int kw = min(32, K - k0);
-#pragma unroll 4
-    for (int q = 0; q < 32; ++q) {
-      const int e = t + q * 128, r = e >> 5, kk = e & 31;
-      const int gr = row0 + r;
-      Ts[r][kk] = (gr < n && kk < kw) ? in[static_cast<size_t>(gr) * K + k0 + kk] : 0.0;
-    }
-    __syncthreads();
-    for (int kk = 0; kk < kw; ++kk) acc = fma(W[k0 + kk], Ts[t][kk], acc);
-    __syncthreads();
-  }
-  const int r = row0 + t;
-  if (r < n) out[r] = accumulate ? out[r] + acc : acc;
+#pragma unroll 8
+  for (int k = 0; k < K; ++k) acc = fma(W[k], row[k], acc);
+  out[r] = accumulate ? out[r] + acc : acc;
 }
 
 // ---------------------------------------------------------------------------- K7 dedup + top-k

@@ -1818,7 +1818,7 @@ static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, in
             in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
             last ? 0 : 1, last && st_i > 0 ? 1 : 0);
       } else if (N == 1 && last && rs == K && cs == 1 && score_v2()) {
-        score_head_kernel<<<static_cast<unsigned>((n + 127) / 128), 128, 0, st>>>(
+        score_head_kernel<<<static_cast<unsigned>((n + 31) / 32), 32, 0, st>>>(
             in, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, st_i > 0 ? 1 : 0);
       } else {
         const dim3 grid(static_cast<unsigned>((N + 31) / 32), static_cast<unsigned>((n + 31) / 32));
