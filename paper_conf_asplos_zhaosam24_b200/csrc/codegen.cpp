@@ -563,7 +563,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "      float gyv[NJ];\n"
     << "#pragma unroll\n      for (int jj = 0; jj < NJ; ++jj) {\n"
     << "        const int j = wq + PG * jj;\n        if (j >= NV) break;\n"
-    << "        double gd = exp((double)yl[jj]) * gxa[jj];\n";
+    << "        double gd = gxa[jj];   // the partials are dL/dy already (x_j folded in by felix_rev_sc)\n";
   emit_auto_grad_switch("        ");
   o << "        gyv[jj] = (float)gd;\n        ok = ok && isfinite(gyv[jj]);\n      }\n"
     << "      const unsigned bad = __ballot_sync(0xffffffffu, !ok);\n"
@@ -840,8 +840,10 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
       if (g.depvar[nd]) o << "    " << g.adj(nd) << " += (ADJ_T)(2.0 * dlam * pr" << r << ");\n";
     }
     g.emit_reverse_body(need, "    ");
+    // partial dL/dy_j = x_j * dL/dx_j of this cone (x_j is at hand here; the Adam prologue needs no exp)
     o << "    if (live) {\n      pen[(size_t)" << q << " * n + c] = pq;\n";
-    for (int j = 0; j < M; ++j) o << "      part[((size_t)" << q << " * NV + " << j << ") * n + c] = (double)gx" << j << ";\n";
+    for (int j = 0; j < M; ++j)
+      o << "      part[((size_t)" << q << " * NV + " << j << ") * n + c] = " << (used[j] ? "x" + std::to_string(j) + " * (double)gx" + std::to_string(j) : std::string("0.0")) << ";\n";
     o << "    }\n  }\n  }\n";
   }
   o << "}\n\n";
@@ -865,7 +867,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  if (o_loss) o_loss[c] = loss;\n"
     << "  bool ok = isfinite(loss);\n  float gy[NV];\n"
     << "#pragma unroll\n  for (int j = 0; j < NV; ++j) {\n"
-    << "    double gd = exp((double)syv[j]) * gxa[j];\n";
+    << "    double gd = gxa[j];\n";
   emit_auto_grad_switch("    ");
   o << "    gy[j] = (float)gd;\n    ok = ok && isfinite(gy[j]);\n  }\n"
     << "  if (!ok) return;\n"
