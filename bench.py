@@ -49,6 +49,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
+    ap.add_argument("--ref-seconds", type=float, default=90.0, help="target wall time of the whole --impl reference run")
     ap.add_argument("--seeds", type=int, default=0, help="override seeds per GPU (experiments; not the headline)")
     ap.add_argument("--search-steps", type=int, default=0, help="override Adam steps per search (experiments)")
     ap.add_argument("--two-statements", action="store_true",
@@ -122,6 +123,11 @@ def measured_peaks():
     return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback (B200_PROFILING.md)"
 
 
+def sp_info_flops(space):
+    """(forward, reverse-sweep) FP64 ops per candidate of a space's DAG (felix_space_info)."""
+    return int(space.info.dag_flops_fwd), int(space.info.dag_flops_rev)
+
+
 def dist_env():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
 
@@ -168,33 +174,94 @@ def oracle_baseline(cfg, seconds: float, history: bool = False):
     return rate, threads, sample, t_search + t_fin
 
 
+def workload_config(cfg, sp, n, T, k, world, hist=False):
+    """The `config` object of the bench line — identical for the felix arm and the reference arm."""
+    return {"workload": f"{cfg.name}: {sp.name}, {sp.n_vars} vars, {n} seeds x {T} steps per GPU, "
+                        f"MLP {list(cfg.mlp_dims)}, top-{k}" + (f", {sp.n_statements} statements (segment sum)"
+                                                               if sp.n_statements > 1 else "")
+                        + (", history rounding (Alg. 1 l.20 over all visited points)" if hist else ""),
+            "n_seeds_per_gpu": n, "n_steps": T, "topk": k, "parallelism": f"dp{world} (seed shards)",
+            "l2": "flushed (256 MB write) between timed iterations"}
+
+
+def felix_workload(args):
+    """(cfg, space, n seeds per GPU, n_steps) of the felix arm for these arguments (shared by both arms)."""
+    import felix_inputs as fi
+    cfg = fi.config(args.config)
+    if args.seeds:
+        cfg.n_seeds = args.seeds
+    elif args.config == "C5":
+        cfg.n_seeds = (1 << 20) // 8          # C5 is 2^20 candidates over 8 GPUs: one GPU's shard
+    if args.search_steps:
+        cfg.n_steps = args.search_steps
+    if args.two_statements:
+        assert args.config == "C2", "--two-statements is defined for C2"
+        cfg.spaces = [fi.c2_space_two_statements()]
+    return cfg, cfg.spaces[0], cfg.n_seeds, cfg.n_steps
+
+
 # ------------------------------------------------------------------------------------- reference arm
+def oracle_sample(cfg, sp, mlp, y0, steps, history):
+    """One bounded sample of the workload on the oracle: `steps` Adam steps of the given seeds, then the
+    finish (round / validate / score / top-k).  Returns (t_search, t_finish) in seconds."""
+    from oracle import felix_oracle as fo
+    t0 = time.perf_counter()
+    y, _, _, hist = fo.search(sp, mlp.W, mlp.b, y0, steps, cfg.lr, cfg.lam, history=history)
+    t1 = time.perf_counter()
+    if history:
+        fo.round_topk_history(sp, mlp.W, mlp.b, [h[0].astype(np.float32) for h in hist], cfg.topk)
+    else:
+        fo.round_topk(sp, mlp.W, mlp.b, y.astype(np.float32), cfg.topk)
+    return t1 - t0, time.perf_counter() - t1
+
+
 def run_reference(args):
+    """The reference arm (this tier: the float64 oracle, as it stands, on the host cores).  Each bench
+    step is ONE bounded sample of the felix arm's workload — the first m seeds of the same space, model
+    and starting points, s Adam steps, then round / top-k of those m — timed on the wall clock; value is
+    the whole-job rate that sample measures (per candidate-step of the search, per candidate of the
+    finish), ms_per_step the wall time a step actually took."""
     rank, world, _ = dist_env()
     if rank != 0:
         return 0
     import felix_inputs as fi
-    cfg = fi.config(args.config)
-    if args.two_statements:
-        cfg.spaces = [fi.c2_space_two_statements()]
+    from oracle import felix_oracle as fo
+    cfg, sp, n, T = felix_workload(args)
+    mlp = fi.make_mlp(cfg.mlp_dims)
+    k = cfg.topk
+    try:
+        import threadpoolctl
+        threads = max(i.get("num_threads", 1) for i in threadpoolctl.threadpool_info()) or os.cpu_count()
+    except Exception:
+        threads = os.cpu_count()
     W = max(args.warmup, 0)
     K = max(args.steps, 1)
-    rates = []
-    tot = 0.0
+    m = min(n, 1024)
+    y0 = fo.init_sample(sp, m, cfg.rng_seed)
+    # size s so that the whole run (W + K samples) takes about args.ref_seconds
+    t0 = time.perf_counter()
+    oracle_sample(cfg, sp, mlp, y0, 1, args.history)
+    probe = time.perf_counter() - t0
+    per_sample = max(0.5, args.ref_seconds / (W + K))
+    s_steps = int(max(1, min(T, per_sample / max(probe, 1e-6))))
+    rates, walls = [], []
     for it in range(W + K):
-        secs = max(2.0, args.cpu_seconds / max(1, (W + K)))
-        rate, threads, sample, t = oracle_baseline(cfg, secs, args.history)
+        t0 = time.perf_counter()
+        ts, tf = oracle_sample(cfg, sp, mlp, y0, s_steps, args.history)
+        wall = time.perf_counter() - t0
         if it >= W:
-            rates.append(rate)
-            tot += t
+            per_cs = ts / (m * s_steps)                      # s per candidate-step of the search
+            per_fin = tf / m if not args.history else tf / (m * s_steps) * T
+            rates.append(n * T / (per_cs * n * T + per_fin * n))
+            walls.append(wall)
     value = statistics.median(rates)
-    ms_per_step = cfg.n_seeds * cfg.n_steps / value * 1e3
+    sample = (f"per step: {m} of the {n} seeds x {s_steps} of {T} Adam steps of {sp.name} + round/top-k of those {m}, "
+              f"numpy float64; value = whole-job rate from the per-candidate-step search time and per-candidate finish time")
     line = {
-        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus, "steps": K,
-        "warmup": W, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-        "dtype": "f64", "data": "synthetic",
-        "config": {"workload": f"{cfg.name}: {cfg.spaces[0].name}, {cfg.n_seeds} seeds x {cfg.n_steps} steps, "
-                               f"MLP {list(cfg.mlp_dims)}", "n_seeds": cfg.n_seeds, "n_steps": cfg.n_steps},
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K,
+        "warmup": W, "ms_per_step": statistics.mean(walls) * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": workload_config(cfg, sp, n, T, k, world, args.history),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
@@ -215,17 +282,7 @@ def run_felix(args):
     import paper_conf_asplos_zhaosam24_b200 as fx
     from paper_conf_asplos_zhaosam24_b200 import dist as fdist
 
-    cfg = fi.config(args.config)
-    if args.seeds:
-        cfg.n_seeds = args.seeds
-    elif args.config == "C5":
-        cfg.n_seeds = (1 << 20) // 8          # C5 is 2^20 candidates over 8 GPUs: one GPU's shard
-    if args.search_steps:
-        cfg.n_steps = args.search_steps
-    if args.two_statements:
-        assert args.config == "C2", "--two-statements is defined for C2"
-        cfg.spaces = [fi.c2_space_two_statements()]
-    sp = cfg.spaces[0]
+    cfg, sp, _, _ = felix_workload(args)
     mlp = fi.make_mlp(cfg.mlp_dims)
     space = fx.Space(sp, device=dev)
     cm = fx.CostModel.from_weights(mlp, device=dev)
@@ -314,16 +371,12 @@ def run_felix(args):
 
     # ---- roofline of the dominant kernel: the tcgen05 MLP (tensor-bound contraction).  Which MLP kernel
     # runs follows felix_api.cu mlp_mode(): the tile-local fused kernel from one full wave of 128-row
-    # tiles (TenSet widths), the persistent layer chain below that; FELIX_MLP overrides.
+    # tiles (TenSet widths), the persistent layer chain below that.
     peaks, peak_src = measured_peaks()
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
-    env_mode = os.environ.get("FELIX_MLP", "")
     tile_fits = tuple(cfg.mlp_dims[1:]) == (512, 256, 256, 1)
     n_rows = n * sp.n_statements
-    if env_mode in ("chain", "layers"):
-        mlp_kernel = "mlp_chain_kernel" if env_mode == "chain" else "mlp_gemm_kernel"
-    else:
-        mlp_kernel = "mlp_tile_kernel" if tile_fits and (env_mode == "tile" or -(-n_rows // 128) >= sms) else "mlp_chain_kernel"
+    mlp_kernel = "mlp_tile_kernel" if tile_fits and -(-n_rows // 128) >= sms else "mlp_chain_kernel"
     traffic = None
     tname = {"mlp_chain_kernel": "roofline_traffic.json", "mlp_tile_kernel": "roofline_traffic_tile.json"}.get(mlp_kernel, "")
     tpath = os.path.join(ROOT, "profiles", "r01", tname) if tname else ""
@@ -335,9 +388,38 @@ def run_felix(args):
     mlp_flops_step = cm.mlp_flops_per_candidate_step() * n * sp.n_statements   # algorithmic (1-pass) FLOPs / Adam step
     gemm_per_step_ms = gemm_ms / (K * T)         # one chain launch (or 2(L-1) layer launches) per Adam step
     achieved_tflops = mlp_flops_step / (gemm_per_step_ms * 1e-3) / 1e12
-    peak = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops")))
+    clk = clocks.summary()
+    capped = "sw_power_cap" in clk.get("reasons", [])
+    # the MLP kernel is timed inside a ~12 ms search at the clocks above: the burst peak applies unless
+    # the power cap engaged (then the sustained one); both fractions are reported
+    peak_burst = float(peaks.get("bf16_tflops", 1590.0))
+    peak_sust = float(peaks.get("bf16_tflops_sustained", peak_burst))
+    peak = peak_sust if capped else peak_burst
     dag_fwd_ms, _ = prof["dag_fwd"]
     dag_rev_ms, _ = prof["dag_rev_adam"]
+    # expression kernels (FP64 straight-line DAG code): algorithmic FP64 ops and HBM bytes per
+    # candidate-step, against the FP64 ALU peak derived from unit counts (148 SMs x 64
+    # FP64 FMA/clk x 2 x max SM clock) and the measured HBM bandwidth
+    M, K0p = sp.n_vars, 96 if cfg.mlp_dims[0] <= 96 else 128
+    P = 4 if n <= 8192 else 2
+    ns = sp.n_statements
+    sm_max = float(clk.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0))
+    fp64_peak = sms * 64 * 2 * sm_max * 1e6 / 1e12
+    hbm_peak = float(peaks.get("hbm_gbs", 6550.0))
+    nht = 4   # head partials read by the Adam prologue (chain: two column halves of the 256-wide head layer x 2)
+    fwd_bytes = 24 * M + 8 * P * M + 8 * P + 4 * nht + ns * 2 * 2 * K0p
+    rev_bytes = 4 * M + 4 * ns * cfg.mlp_dims[0] + 8 * P * M + 8 * P
+    fwd_ops = sp_info_flops(space)[0] + 15 * M
+    rev_ops = sum(sp_info_flops(space))             # forward recompute + reverse sweep
+
+    def kroof(ms_total, ops, nbytes):
+        per_step_s = ms_total / (K * T) * 1e-3
+        f = ops * n / per_step_s / 1e12
+        b = nbytes * n / per_step_s / 1e9
+        return {"us_per_adam_step": per_step_s * 1e6, "fp64_tflops": f, "fp64_peak_tflops": fp64_peak,
+                "fp64_frac": f / fp64_peak, "hbm_gbs": b, "hbm_peak_gbs": hbm_peak, "hbm_frac": b / hbm_peak,
+                "ops_per_candidate_step": ops, "bytes_per_candidate_step": nbytes,
+                "bound": "latency (neither FP64 nor HBM: both fractions are small; DESIGN.md §6)"}
 
     # ---- end to end through the public API with host buffers (pinned), copies inside the timed region
     e2e = None
@@ -348,11 +430,15 @@ def run_felix(args):
         y_dev = torch.empty_like(y)
 
         def e2e_step():
+            # the same work as a timed device step (L2 flush, search, finish) through the public API, with
+            # the step's starting points coming from pinned host memory (H2D) instead of the device
+            # rejection sampler, and the losses + top-k records read back (D2H)
+            flush.zero_()
             y_dev.copy_(y0_host, non_blocking=True)                          # H2D: starting points
             space.search(cm, y_dev, T, lr=cfg.lr, lam=cfg.lam, init_from_y=True, index_base=base,
                          final_loss=loss, history=hist, stream=stream)
             loss_host.copy_(loss, non_blocking=True)                         # D2H: final losses
-            return finish(y_dev)                                             # D2H: top-k records
+            return finish(y_dev)                                             # D2H: top-k records (synchronises)
         for _ in range(2):
             e2e_step()
         barrier()
@@ -368,7 +454,10 @@ def run_felix(args):
         h2d = sp.n_vars * n * 4
         d2h = n * 4 + k * (8 + 8 + 4 * sp.n_vars) + 4
         e2e = {"value": world * n * T * K / t_e2e, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-               "timing": "host wall clock incl. pinned H2D of y0 and D2H of losses + top-k"}
+               "timing": "host wall clock over K steps (max over ranks); each step: L2 flush, pinned H2D of the "
+                         "starting points, felix_search, felix_round_topk, D2H of losses + top-k",
+               "work_vs_value": "value's work with a0 (device rejection sampler, ~0.5 % of a step) replaced by the "
+                                "H2D of host starting points, and the L2 flush inside the timed region"}
 
     if rank != 0:
         if world > 1:
@@ -381,7 +470,9 @@ def run_felix(args):
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample}
 
     n_gemm = len(cfg.mlp_dims) * 2 - 4          # (L-1) forward + (L-1) backward GEMM layers
-    mlp_launches = 1 if os.environ.get("FELIX_MLP", "chain") != "layers" else n_gemm
+    kernels = {"felix_fwd_adam": kroof(dag_fwd_ms, fwd_ops, fwd_bytes),
+               "felix_rev_sc": kroof(dag_rev_ms, rev_ops, rev_bytes)}
+    mlp_launches = 1
     # init + steps + finish; the reverse class counts the split-cone kernels' final Adam launch too
     rev_launches = int(round(prof["dag_rev_adam"][1] / K))
     init_launches = max(1, int(round(prof["init"][1] / K)))   # sampler (+ the split-cone counter reset)
@@ -391,13 +482,7 @@ def run_felix(args):
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "fp16x3 split (fp32-accurate) MLP, f64 DAG, f32 Adam", "data": "synthetic",
-        "config": {"workload": f"{cfg.name}: {sp.name}, {sp.n_vars} vars, {n} seeds x {T} steps per GPU, "
-                               f"MLP {list(cfg.mlp_dims)}, top-{k}" + (f", {sp.n_statements} statements (segment sum)"
-                                                                       if sp.n_statements > 1 else "")
-                               + (", history rounding (Alg. 1 l.20 over all "
-                                                                       "visited points)" if hist else ""),
-                   "n_seeds_per_gpu": n, "n_steps": T, "topk": k, "parallelism": f"dp{world} (seed shards)",
-                   "l2": "flushed (256 MB write) between timed iterations"},
+        "config": workload_config(cfg, sp, n, T, k, world, hist),
         "roofline": {"bound": "tensor", "achieved": achieved_tflops, "peak": peak, "unit": "TFLOP/s",
                      "frac": achieved_tflops / peak, "traffic": traffic,
                      "kernel": f"{mlp_kernel} (all {n_gemm} MLP layers of one Adam step, tcgen05 kind::f16, 3-pass hi/lo split)",
@@ -405,13 +490,16 @@ def run_felix(args):
                                         if traffic is not None else None),
                      "algorithmic_flops_per_adam_step": mlp_flops_step,
                      "executed_tflops": 3 * achieved_tflops,
-                     "peak_source": f"{peak_src} bf16_tflops_sustained (fp16 = bf16 rate)"},
+                     "peak_source": (f"{peak_src} bf16_tflops (burst; fp16 = bf16 rate)" if not capped else
+                                     f"{peak_src} bf16_tflops_sustained (sw_power_cap seen; fp16 = bf16 rate)"),
+                     "frac_vs_burst": achieved_tflops / peak_burst, "frac_vs_sustained": achieved_tflops / peak_sust},
+        "kernel_rooflines": kernels,
         "breakdown_ms_per_adam_step": {"dag_fwd": dag_fwd_ms / (K * T), "mlp_gemms": gemm_per_step_ms,
                                        "dag_rev_adam": dag_rev_ms / (K * T),
                                        "search_total": prof_total_ms / (K * T)},
         "finish_ms": finish_ms,
         "gpu_launches": launches_per_step * K,
-        "clocks": clocks.summary(),
+        "clocks": clk,
         "top1": ({"global_idx": int(gidx[0]) & ((1 << 40) - 1), "step": int(gidx[0]) >> 40, "score": float(gsc[0])}
                  if hist and len(gidx) else
                  {"global_idx": int(gidx[0]) if len(gidx) else None, "score": float(gsc[0]) if len(gsc) else None}),
@@ -607,8 +695,7 @@ def run_felix_tasks(args):
         rate, threads, sample, _ = oracle_baseline_tasks(cfg, args.cpu_seconds)
         cpu = {"value": rate, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample}
     # split-cone kernels (default for these population sizes) add one final Adam launch per task
-    sc_final = 1 if os.environ.get("FELIX_SC", "") == "1" else 0   # groups: split-cone only when forced
-    sc_final *= 2                                                   # counter reset + final Adam
+    sc_final = 0                                                    # groups use the cone-group kernels
     launches = sum(1 + T * 3 + sc_final + (6 + len(cfg.mlp_dims) - 1) for _ in shards)
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
@@ -677,8 +764,26 @@ def run_reference_tasks(args):
     return 0
 
 
+def spawn_ranks(args) -> int:
+    """`python bench.py --gpus N` without a torchrun environment: start N ranks (one per GPU) through
+    torch.distributed.run on 127.0.0.1 and pass their output through.  NCCL init logging is on so the
+    communicator size is visible in the log."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd, env=env)
+
+
 def main():
     args = parse()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return spawn_ranks(args)
     multi = args.config in ("C3", "C4")
     if args.impl == "reference":
         return run_reference_tasks(args) if multi else run_reference(args)

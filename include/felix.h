@@ -38,7 +38,7 @@
 extern "C" {
 #endif
 
-#define FELIX_ABI_VERSION 3
+#define FELIX_ABI_VERSION 4
 
 #if defined(__GNUC__)
 #define FELIX_EXPORT __attribute__((visibility("default")))
@@ -141,6 +141,8 @@ typedef struct {
   double nvrtc_ms;              /* time spent compiling the generated kernels                  */
   int32_t regs_fwd, regs_rev;   /* registers/thread of the generated forward / reverse kernels  */
   int64_t dag_flops_fwd;        /* arithmetic ops in one forward evaluation (per candidate)    */
+  int64_t dag_flops_rev;        /* arithmetic ops of one reverse sweep over the whole DAG (per candidate,
+                                   local partials + adjoint accumulations; the forward recompute excluded) */
 } felix_space_info_t;
 FELIX_EXPORT felix_status felix_space_info(const felix_space* s, felix_space_info_t* out);
 
@@ -222,6 +224,24 @@ FELIX_EXPORT felix_status felix_history_topk(felix_space* s, felix_costmodel* m,
  * cost [n] (C, higher = better), loss [n], grad [n_vars][n] (dL/dy). */
 FELIX_EXPORT felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int64_t n, float lambda,
                         float* phi, float* g, float* cost, float* loss, float* grad, void* stream);
+/* felix_eval_ex: felix_eval with two more views of the same evaluation (test hooks for the north star's
+ * parity bars).  All outputs device, any may be NULL:
+ *   phi, g, cost, loss, grad   as felix_eval
+ *   F        double [n_features][n]: the raw smoothed features Feat_k(e^y) before slog (P:L688-766,
+ *            reading O3), FP64, from the same forward code as phi — the "feature <= 1e-4" bar is on F.
+ *   search_path != 0: evaluate through the kernels and launch configuration of one felix_search Adam
+ *            step instead (split-cone reverse kernel: per-cone partial adjoints summed in fixed order by
+ *            the kernel that applies Adam in a search), writing the loss and the dL/dy that
+ *            step's Adam update would use; y is not modified.  Only loss and grad may be non-NULL
+ *            (FELIX_E_INVALID_ARG otherwise). */
+typedef struct {
+  float* phi; float* g; float* cost; float* loss; float* grad;
+  double* F;
+  int32_t search_path;
+  int32_t _pad;
+} felix_eval_out;
+FELIX_EXPORT felix_status felix_eval_ex(felix_space* s, felix_costmodel* m, const float* y, int64_t n, float lambda,
+                                        const felix_eval_out* out, void* stream);
 /* Rounding + validity only: sched device int32 [n][n_vars], valid device uint8 [n]. */
 FELIX_EXPORT felix_status felix_round(felix_space* s, const float* y, int64_t n, int32_t* sched, uint8_t* valid,
                          void* stream);
@@ -237,14 +257,29 @@ FELIX_EXPORT felix_status felix_score(felix_space* s, felix_costmodel* m, const 
 FELIX_EXPORT felix_status felix_init_sample(felix_space* s, int64_t n, uint64_t rng_seed, int64_t index_base,
                                float* y, void* stream);
 
+/* Process-wide execution knobs for experiments and tests; normal use needs none (the defaults are the
+ * measured choices of DESIGN.md; every knob gives the same results up to fp32 summation order).  The
+ * library never reads environment variables.  key / value (-1 = default):
+ *   "mlp"                 0 tile kernel, 1 persistent layer chain, 2 one GEMM kernel per layer
+ *   "cone_width"          cone-partition width P of the expression kernels: 1, 2, 4, 8, 16
+ *   "replicas"            cone-group replicas per block: 1, 2, 4
+ *   "sc_warps"            warps per split-cone reverse CTA: 1..8
+ *   "chunks"              concurrent population chunks: 1..16
+ *   "split_cone"          0 cone-group reverse + Adam kernel, 1 split-cone reverse kernel
+ *   "tile_cta_group"      tile kernel on 1-SM tiles (1) or 2-SM cta_group::2 pairs (2)
+ *   "codegen_cone_width", "codegen_replicas"   the variant felix_codegen emits
+ *   "trace"               0/1: per-block %globaltimer stamps in kernels generated afterwards
+ * FELIX_E_INVALID_ARG for an unknown key or value. */
+FELIX_EXPORT felix_status felix_tune(const char* key, int32_t value);
+
 /* Per-kernel-class device time accumulated by felix_search while profiling is enabled (CUDA events
  * on the search stream).  Classes: 0 DAG forward, 1 MLP GEMMs, 2 DAG reverse+Adam, 3 other.
  * ms[4], launches[4]; reset with felix_profile_reset. */
 FELIX_EXPORT felix_status felix_profile_enable(felix_space* s, int32_t enable);
 FELIX_EXPORT felix_status felix_profile_read(felix_space* s, double* ms, int64_t* launches);
 FELIX_EXPORT felix_status felix_profile_reset(felix_space* s);
-/* Debug: copy the per-block %globaltimer stamps of the generated kernels (only when the space was
- * created with the environment variable FELIX_TRACE set): uint64 [2][8192][4] = {fwd, rev} x block x
+/* Debug: copy the per-block %globaltimer stamps of the generated kernels (only for kernels generated
+ * after felix_tune("trace", 1)): uint64 [2][8192][4] = {fwd, rev} x block x
  * {start, after griddepcontrol.wait, after compute, end}.  n_words bounds the copy. */
 FELIX_EXPORT felix_status felix_debug_trace(felix_space* s, uint64_t* out, int64_t n_words);
 

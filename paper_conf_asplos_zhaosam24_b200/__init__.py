@@ -29,7 +29,8 @@ EXPORTED = ["felix_last_error", "felix_abi_version", "felix_space_create", "feli
             "felix_space_info", "felix_codegen", "felix_costmodel_load", "felix_costmodel_destroy",
             "felix_search", "felix_round_topk", "felix_eval", "felix_round", "felix_score",
             "felix_init_sample", "felix_profile_enable", "felix_profile_read", "felix_profile_reset",
-            "felix_debug_trace", "felix_history_topk", "felix_space_set_statements", "felix_search_group"]
+            "felix_debug_trace", "felix_history_topk", "felix_space_set_statements", "felix_search_group",
+            "felix_eval_ex", "felix_tune"]
 
 
 class FelixError(RuntimeError):
@@ -54,11 +55,18 @@ class _SearchParams(ctypes.Structure):
                 ("history", ctypes.c_int32), ("index_base", ctypes.c_int64)]
 
 
+class _EvalOut(ctypes.Structure):
+    _fields_ = [("phi", ctypes.c_void_p), ("g", ctypes.c_void_p), ("cost", ctypes.c_void_p), ("loss", ctypes.c_void_p),
+                ("grad", ctypes.c_void_p), ("F", ctypes.c_void_p), ("search_path", ctypes.c_int32),
+                ("_pad", ctypes.c_int32)]
+
+
 class _SpaceInfo(ctypes.Structure):
     _fields_ = [("n_vars", ctypes.c_int32), ("n_nodes", ctypes.c_int32), ("n_features", ctypes.c_int32),
                 ("n_constraints_user", ctypes.c_int32), ("n_roots_total", ctypes.c_int32),
                 ("n_components", ctypes.c_int32), ("n_tuples_total", ctypes.c_int64), ("nvrtc_ms", ctypes.c_double),
-                ("regs_fwd", ctypes.c_int32), ("regs_rev", ctypes.c_int32), ("dag_flops_fwd", ctypes.c_int64)]
+                ("regs_fwd", ctypes.c_int32), ("regs_rev", ctypes.c_int32), ("dag_flops_fwd", ctypes.c_int64),
+                ("dag_flops_rev", ctypes.c_int64)]
 
 
 _P = ctypes.c_void_p
@@ -69,6 +77,17 @@ for _name in EXPORTED:
         getattr(_lib, _name).restype = ctypes.c_int
 _lib.felix_space_destroy.restype = None
 _lib.felix_costmodel_destroy.restype = None
+
+
+def _check_tensor(t, shape, dtype_name: str, device_index: int, what: str) -> None:
+    """Argument validation before a pointer crosses the ABI: a CUDA tensor on the handle's device,
+    of the given dtype, contiguous, of exactly `shape`."""
+    import torch
+    dt = getattr(torch, dtype_name)
+    if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype == dt and t.is_contiguous()
+            and tuple(t.shape) == tuple(shape) and t.device.index == device_index):
+        got = (tuple(t.shape), t.dtype, str(t.device)) if isinstance(t, torch.Tensor) else type(t)
+        raise FelixError(1, f"{what} must be a contiguous {dtype_name} CUDA tensor {tuple(shape)} on cuda:{device_index}, got {got}")
 
 
 def _check(status: int) -> None:
@@ -117,8 +136,16 @@ def search_group(spaces: Sequence["Space"], cm: "CostModel", ys, n_steps: int, *
     G = len(spaces)
     if G == 0:
         return ys
+    if len(ys) != G:
+        raise FelixError(1, "len(ys) != len(spaces)")
     for sp, y in zip(spaces, ys):
         sp._check_y(y)
+    if final_losses is not None:
+        if len(final_losses) != G:
+            raise FelixError(1, "len(final_losses) != len(spaces)")
+        for sp, y, l in zip(spaces, ys, final_losses):
+            if l is not None:
+                _check_tensor(l, (y.shape[1],), "float32", sp.device, "final_losses[i]")
     seeds = list(rng_seeds) if rng_seeds is not None else [0] * G
     bases = list(index_bases) if index_bases is not None else [0] * G
     params = (_SearchParams * G)()
@@ -130,6 +157,35 @@ def search_group(spaces: Sequence["Space"], cm: "CostModel", ys, n_steps: int, *
     lp = (_P * G)(*[_ptr(l) for l in final_losses]) if final_losses is not None else None
     _check(_lib.felix_search_group(hs, G, cm._h, params, yp, lp, _P(_stream(stream))))
     return ys
+
+
+_TUNE_KEYS = ("mlp", "cone_width", "replicas", "sc_warps", "chunks", "split_cone", "tile_cta_group",
+              "codegen_cone_width", "codegen_replicas", "trace")
+_TUNE_DEFAULT = {k: (0 if k == "trace" else -1) for k in _TUNE_KEYS}
+
+
+def tune(**knobs) -> None:
+    """felix_tune: process-wide execution knobs (experiments / tests), e.g. tune(mlp=1, cone_width=8).
+    MLP modes may be given by name: mlp="tile" | "chain" | "layers" | "auto"."""
+    for k, v in knobs.items():
+        if k == "mlp" and isinstance(v, str):
+            v = {"auto": -1, "tile": 0, "chain": 1, "layers": 2}[v]
+        _check(_lib.felix_tune(k.encode(), ctypes.c_int32(int(v))))
+
+
+class tuned:
+    """Context manager: set knobs for a block, restore the defaults afterwards."""
+
+    def __init__(self, **knobs):
+        self.knobs = knobs
+
+    def __enter__(self):
+        tune(**self.knobs)
+        return self
+
+    def __exit__(self, *exc):
+        tune(**{k: _TUNE_DEFAULT[k] for k in self.knobs})
+        return False
 
 
 def abi_version() -> int:
@@ -161,6 +217,7 @@ class SpaceInfo:
     regs_fwd: int
     regs_rev: int
     dag_flops_fwd: int
+    dag_flops_rev: int
 
 
 class CostModel:
@@ -225,6 +282,8 @@ class Space:
         """felix_search on device y (torch fp32 [n_vars, n], updated in place).  history=True also records
         varValuesHistory (Alg. 1 l.13/17) for history_topk."""
         self._check_y(y)
+        if final_loss is not None:
+            _check_tensor(final_loss, (y.shape[1],), "float32", self.device, "final_loss")
         p = _SearchParams(int(y.shape[1]), int(n_steps), lr, beta1, beta2, eps, lam, int(rng_seed) & (2**64 - 1),
                           1 if init_from_y else 0, 1 if history else 0, int(index_base))
         _check(_lib.felix_search(self._h, cm._h, ctypes.byref(p), _P(_ptr(y)), _P(_ptr(final_loss)),
@@ -261,7 +320,9 @@ class Space:
         return idx[:m], step[:m], sc[:m], sched[:m], int(nu.value)
 
     # ---------------------------------------------------------------- test hooks
-    def eval(self, cm: CostModel, y, lam: float = 1.0, stream=None):
+    def eval(self, cm: CostModel, y, lam: float = 1.0, stream=None, features: bool = False):
+        """felix_eval(_ex): phi, g, cost, loss, grad at y; features=True adds the raw smoothed features
+        F (float64 [n_features, n])."""
         import torch
         self._check_y(y)
         n = y.shape[1]
@@ -273,9 +334,24 @@ class Space:
             loss=torch.empty(n, dtype=torch.float32, device=dev),
             grad=torch.empty((self.n_vars, n), dtype=torch.float32, device=dev),
         )
-        _check(_lib.felix_eval(self._h, cm._h, _P(_ptr(y)), ctypes.c_int64(n), ctypes.c_float(lam),
-                               _P(_ptr(out["phi"])), _P(_ptr(out["g"])), _P(_ptr(out["cost"])),
-                               _P(_ptr(out["loss"])), _P(_ptr(out["grad"])), _P(_stream(stream))))
+        if features:
+            out["F"] = torch.empty((self.info.n_features, n), dtype=torch.float64, device=dev)
+        eo = _EvalOut(*[_ptr(out.get(k)) for k in ("phi", "g", "cost", "loss", "grad", "F")], 0, 0)
+        _check(_lib.felix_eval_ex(self._h, cm._h, _P(_ptr(y)), ctypes.c_int64(n), ctypes.c_float(lam),
+                                  ctypes.byref(eo), _P(_stream(stream))))
+        return out
+
+    def eval_search_path(self, cm: CostModel, y, lam: float = 1.0, stream=None):
+        """felix_eval_ex(search_path=1): loss and dL/dy through the kernels of one felix_search Adam step
+        (split-cone partial adjoints summed as the search's Adam prologue sums them)."""
+        import torch
+        self._check_y(y)
+        n = y.shape[1]
+        out = dict(loss=torch.empty(n, dtype=torch.float32, device=y.device),
+                   grad=torch.empty((self.n_vars, n), dtype=torch.float32, device=y.device))
+        eo = _EvalOut(0, 0, 0, _ptr(out["loss"]), _ptr(out["grad"]), 0, 1, 0)
+        _check(_lib.felix_eval_ex(self._h, cm._h, _P(_ptr(y)), ctypes.c_int64(n), ctypes.c_float(lam),
+                                  ctypes.byref(eo), _P(_stream(stream))))
         return out
 
     def round(self, y, stream=None):
@@ -290,7 +366,8 @@ class Space:
 
     def score(self, cm: CostModel, sched, stream=None):
         import torch
-        n = sched.shape[0]
+        n = sched.shape[0] if hasattr(sched, "shape") else 0
+        _check_tensor(sched, (n, self.n_vars), "int32", self.device, "sched")
         out = torch.empty(n, dtype=torch.float64, device=sched.device)
         _check(_lib.felix_score(self._h, cm._h, _P(_ptr(sched)), ctypes.c_int64(n), _P(_ptr(out)),
                                 _P(_stream(stream))))
@@ -325,5 +402,5 @@ class Space:
     def _check_y(self, y) -> None:
         import torch
         if not (isinstance(y, torch.Tensor) and y.is_cuda and y.dtype == torch.float32 and y.dim() == 2
-                and y.shape[0] == self.n_vars and y.is_contiguous()):
-            raise FelixError(1, f"y must be a contiguous CUDA float32 tensor [{self.n_vars}, n]")
+                and y.shape[0] == self.n_vars and y.is_contiguous() and y.device.index == self.device):
+            raise FelixError(1, f"y must be a contiguous CUDA float32 tensor [{self.n_vars}, n] on cuda:{self.device}")

@@ -71,86 +71,6 @@ __global__ void round_int_kernel(const float* __restrict__ y, int n, int M, int 
   sched[static_cast<size_t>(cand) * M + j] = static_cast<int>(int_lo[q] + lo);
 }
 
-// ---------------------------------------------------------------------------- K6 FP64 MLP scoring (register-blocked)
-// Same arithmetic as score_layer_kernel below, operation for operation (acc = b[col]; for k ascending:
-// acc = fma(W[col][k], in(row, k), acc); then ReLU / segment-sum accumulate), so scores are bit-identical;
-// 64x64 output tile per 256-thread block, thread (tx, ty) owns rows ty*4..+3 x columns tx*4..+3 (16 FP64
-// accumulators), K staged through shared memory 16 at a time.
-constexpr int SCORE_T = 64, SCORE_KT = 16;
-__global__ void __launch_bounds__(256) score_layer_rb_kernel(const double* __restrict__ in, long long in_rs, long long in_cs,
-                                                             int n, int K, const double* __restrict__ W,
-                                                             const double* __restrict__ b, double* __restrict__ out,
-                                                             int N, int relu, int accumulate) {
-  __shared__ __align__(16) double As[SCORE_KT][SCORE_T];   // [k][row]
-  __shared__ __align__(16) double Bs[SCORE_KT][SCORE_T];   // [k][col]
-  const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4, tid = threadIdx.x;
-  const int row0 = blockIdx.y * SCORE_T, col0 = blockIdx.x * SCORE_T;
-  double acc[4][4];
-#pragma unroll
-  for (int j = 0; j < 4; ++j) {
-    const int col = col0 + tx * 4 + j;
-    const double bj = col < N ? b[col] : 0.0;
-#pragma unroll
-    for (int i = 0; i < 4; ++i) acc[i][j] = bj;
-  }
-  // this thread's share of a 16 x 64 A tile and B tile (4 elements each), loaded one K chunk ahead into
-  // registers so the global / L2 latency overlaps the FMAs of the current chunk
-  double pa[4], pb[4];
-  auto load_chunk = [&](int k0) {
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int e = tid + q * 256;
-      int r, kk;
-      if (in_rs == 1) { r = e & 63; kk = e >> 6; } else { kk = e & 15; r = e >> 4; }
-      const int gr = row0 + r, gk = k0 + kk;
-      pa[q] = (gr < n && gk < K) ? in[static_cast<size_t>(gr) * in_rs + static_cast<size_t>(gk) * in_cs] : 0.0;
-      const int c = e >> 4, kb = e & 15;
-      const int gc = col0 + c, gkb = k0 + kb;
-      pb[q] = (gc < N && gkb < K) ? W[static_cast<size_t>(gc) * K + gkb] : 0.0;
-    }
-  };
-  load_chunk(0);
-  for (int k0 = 0; k0 < K; k0 += SCORE_KT) {
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int e = tid + q * 256;                      // 1024 elements of each 16 x 64 tile
-      // A: consecutive threads -> consecutive rows when the input is feature-major (in_rs == 1),
-      // consecutive k when it is row-major
-      int r, kk;
-      if (in_rs == 1) { r = e & 63; kk = e >> 6; } else { kk = e & 15; r = e >> 4; }
-      As[kk][r] = pa[q];
-      Bs[e & 15][e >> 4] = pb[q];                       // B: consecutive threads -> consecutive k (row-major W)
-    }
-    __syncthreads();
-    if (k0 + SCORE_KT < K) load_chunk(k0 + SCORE_KT);
-    const int kmax = min(SCORE_KT, K - k0);
-    for (int kk = 0; kk < kmax; ++kk) {
-      const double2 a01 = *reinterpret_cast<const double2*>(&As[kk][ty * 4]);
-      const double2 a23 = *reinterpret_cast<const double2*>(&As[kk][ty * 4 + 2]);
-      const double2 w01 = *reinterpret_cast<const double2*>(&Bs[kk][tx * 4]);
-      const double2 w23 = *reinterpret_cast<const double2*>(&Bs[kk][tx * 4 + 2]);
-      const double a[4] = {a01.x, a01.y, a23.x, a23.y}, w[4] = {w01.x, w01.y, w23.x, w23.y};
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc[i][j] = fma(w[j], a[i], acc[i][j]);
-    }
-    __syncthreads();
-  }
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const int r = row0 + ty * 4 + i;
-    if (r >= n) continue;
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int col = col0 + tx * 4 + j;
-      if (col >= N) continue;
-      const double v = (relu && !(acc[i][j] > 0.0)) ? 0.0 : acc[i][j];
-      out[static_cast<size_t>(r) * N + col] = accumulate ? out[static_cast<size_t>(r) * N + col] + v : v;
-    }
-  }
-}
-
 // ---------------------------------------------------------------------------- K6 FP64 MLP scoring
 // out[row][col] = act( b[col] + sum_k W[col][k] * in(row, k) ), k ascending (deterministic, so equal
 // schedules get bit-identical scores); accumulate != 0 adds to out (segment sum over statements).  32x32 output tile per 256-thread block, K staged through

@@ -53,32 +53,36 @@ typedef unsigned int u32;
 typedef unsigned short u16;
 __device__ __forceinline__ u16 f2h(float f) { u16 h; asm("cvt.rn.f16.f32 %0, %1;" : "=h"(h) : "f"(f)); return h; }
 __device__ __forceinline__ float h2f(u16 h) { float f; asm("cvt.f32.f16 %0, %1;" : "=f"(f) : "h"(h)); return f; }
-// ---- fast FP64 reciprocal / sqrt for the search kernels: MUFU seed + Newton (~1 ulp, no slow
-//      path).  The hard / sampler kernels, which take integer decisions, use IEEE '/' and sqrt.
+// ---- fast FP64 reciprocal / sqrt for the search kernels: MUFU seed + one Newton step (relative error
+//      ~2^-44, far inside the 1e-4 feature tolerance; no slow path).  The hard / sampler kernels, which
+//      take integer decisions, use IEEE '/' and sqrt.
 __device__ __forceinline__ double f_rcp(double b) {
   double r0; asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r0) : "d"(b));
-  double e = fma(-b, r0, 1.0); double r = fma(r0, e, r0);
-  e = fma(-b, r, 1.0); r = fma(r, e, r);
+  const double e = fma(-b, r0, 1.0); const double r = fma(r0, e, r0);
   return (r0 == 0.0 || isinf(r0)) ? r0 : r;
 }
+// ---- FP32 helpers (MUFU approximations, ~2 ulp): the tails of the smooth step in the forward and the
+//      whole split-cone reverse kernel (DESIGN.md "Precision of the expression kernels")
+__device__ __forceinline__ float f_rcpf(float x) { float r; asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }
+__device__ __forceinline__ float f_sqrtf(float x) { float r; asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }
+__device__ __forceinline__ float sf_hyp(float t) { return f_sqrtf(fmaf(t, t, 1.f)); }
+__device__ __forceinline__ float sf_tail(float t, float h) { return 0.5f * f_rcpf(h * (h + fabsf(t))); }
+__device__ __forceinline__ float sf_Sh(float t, float h) { const float tl = sf_tail(t, h); return t >= 0.f ? 1.f - tl : tl; }
+__device__ __forceinline__ float sf_dSh(float h) { return 0.5f * f_rcpf(h * h * h); }
+__device__ __forceinline__ float sf_gaph(float t, float h) { return 0.5f * f_rcpf(h + fabsf(t)); }
+// smooth step with an FP64 argument and an FP32 tail: t = a - b is exact in FP64 (no cancellation),
+// the tail 1/(2h(h+|t|)) is only needed to relative precision (S = 1 - tail or tail in FP64)
+__device__ __forceinline__ double sm_Sf(double t, float h) { const double tl = (double)sf_tail((float)t, h); return t >= 0.0 ? 1.0 - tl : tl; }
+__device__ __forceinline__ float slogpf_(float f) { return f_rcpf((1.f + fabsf(f)) * 0.69314718055994530942f); }
+__device__ __forceinline__ float f_powf(float a, float e) { return powf(a, e); }
 __device__ __forceinline__ double f_div(double a, double b) { return a * f_rcp(b); }
 __device__ __forceinline__ void cp_async4(float* dst, const float* src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"((unsigned)__cvta_generic_to_shared(dst)), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-// ---- thread-block cluster helpers (cone-per-CTA kernels): rank, barrier, distributed shared memory
-__device__ __forceinline__ unsigned cl_rank() { unsigned r; asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r)); return r; }
-__device__ __forceinline__ void cl_sync() { asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory"); }
-__device__ __forceinline__ unsigned cl_map(const void* p, unsigned rank) {
-  unsigned r; asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"((unsigned)__cvta_generic_to_shared(p)), "r"(rank)); return r;
-}
-__device__ __forceinline__ double cl_ld_f64(const double* p, unsigned rank) { double v; asm volatile("ld.shared::cluster.f64 %0, [%1];" : "=d"(v) : "r"(cl_map(p, rank)) : "memory"); return v; }
-__device__ __forceinline__ void cl_st_f32(float* p, unsigned rank, float v) { asm volatile("st.shared::cluster.f32 [%0], %1;" :: "r"(cl_map(p, rank)), "f"(v) : "memory"); }
-__device__ __forceinline__ void cl_st_f64(double* p, unsigned rank, double v) { asm volatile("st.shared::cluster.f64 [%0], %1;" :: "r"(cl_map(p, rank)), "d"(v) : "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 __device__ __forceinline__ double f_sqrt(double x) {
   double y; asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
-  y = y * fma(-0.5 * x, y * y, 1.5);
   y = y * fma(-0.5 * x, y * y, 1.5);
   double s = x * y;
   s = fma(0.5 * y, fma(-s, s, x), s);
@@ -145,6 +149,7 @@ struct Gen {
   std::vector<bool> depvar;     // node depends on a variable
   std::ostringstream o;
   int64_t flops = 0;
+  int64_t flops_rev = 0;   // arithmetic ops of the emitted reverse sweep (adjoint accumulations + local partials)
 
   explicit Gen(const SpaceDesc& dd) : d(dd), n((int)dd.nodes.size()), depvar(n, false) {
     for (int i = 0; i < n; ++i) {
@@ -174,48 +179,54 @@ struct Gen {
     return in;
   }
 
-  // forward node values (double) for the nodes in `in`.  mode 0: fast smooth, 1: IEEE smooth, 2: hard.
+  // forward node values for the nodes in `in`.  mode 0: search forward (FP64 values, FP32 tails of the
+  // smooth step), 1: IEEE smooth FP64 (sampler), 2: hard FP64 (integer points), 3: FP32 (split-cone
+  // reverse kernel).  Smooth compare / min / max nodes keep t and h = sqrt(1+t^2) as named values for
+  // the reverse sweep: compares as FP32 hf<i> (and kf<i> for EQ/NE), min / max as h<i> in the node's type.
   void emit_forward(const std::vector<bool>& in, int mode, const char* xname, const char* ind = "  ") {
-    const bool hard = mode == 2;
+    const bool hard = mode == 2, f32 = mode == 3;
+    const std::string T = f32 ? "float" : "double";
+    const std::string one = f32 ? "1.f" : "1.0", half = f32 ? "0.5f" : "0.5";
     const std::string mn = mode == 0 ? "sm_min" : "ie_min", mx = mode == 0 ? "sm_max" : "ie_max",
                       S = mode == 0 ? "sm_S" : "ie_S";
     auto divx = [&](const std::string& a, const std::string& b) {
+      if (f32) return a + " * f_rcpf(" + b + ")";
       return mode == 0 ? "f_div(" + a + ", " + b + ")" : "(" + a + " / " + b + ")";
     };
+    auto cst = [&](double v) { return f32 ? "(float)" + lit(v) : lit(v); };
     for (int i = 0; i < n; ++i) {
       if (!in[i]) continue;
       const felix_node& nd = d.nodes[i];
       const std::string A = "v" + std::to_string(nd.a), B = "v" + std::to_string(nd.b), C = "v" + std::to_string(nd.c);
       std::string e;
       const std::string I = std::to_string(i);
-      if (mode == 0) {
-        // smooth ops: keep t and h = sqrt(1+t^2) as named values for the reverse sweep
+      if (mode == 0 || f32) {
         switch (nd.op) {
           case FELIX_OP_GT: case FELIX_OP_GE: case FELIX_OP_LT: case FELIX_OP_LE: {
             const bool ab = nd.op == FELIX_OP_GT || nd.op == FELIX_OP_GE;
-            o << ind << "const double t" << I << " = " << (ab ? A + " - " + B : B + " - " + A) << ";\n"
-              << ind << "const double h" << I << " = sm_hyp(t" << I << ");\n"
-              << ind << "const double v" << I << " = sm_Sh(t" << I << ", h" << I << ");\n";
+            o << ind << "const " << T << " t" << I << " = " << (ab ? A + " - " + B : B + " - " + A) << ";\n"
+              << ind << "const float hf" << I << " = sf_hyp((float)t" << I << ");\n"
+              << ind << "const " << T << " v" << I << " = " << (f32 ? "sf_Sh" : "sm_Sf") << "(t" << I << ", hf" << I << ");\n";
             flops += 6;
             continue;
           }
           case FELIX_OP_MIN: case FELIX_OP_MAX: {
-            const bool mx = nd.op == FELIX_OP_MAX;
-            o << ind << "const double t" << I << " = " << A << " - " << B << ";\n"
-              << ind << "const double h" << I << " = sm_hyp(t" << I << ");\n"
-              << ind << "const double v" << I << " = (t" << I << " >= 0.0 ? " << (mx ? A : B) << " : " << (mx ? B : A) << ") "
-              << (mx ? "+" : "-") << " sm_gaph(t" << I << ", h" << I << ");\n";
+            const bool mx_ = nd.op == FELIX_OP_MAX;
+            o << ind << "const " << T << " t" << I << " = " << A << " - " << B << ";\n"
+              << ind << "const " << T << " h" << I << " = " << (f32 ? "sf_hyp" : "sm_hyp") << "(t" << I << ");\n"
+              << ind << "const " << T << " v" << I << " = (t" << I << " >= 0 ? " << (mx_ ? A : B) << " : " << (mx_ ? B : A) << ") "
+              << (mx_ ? "+" : "-") << (f32 ? " sf_gaph(t" : " sm_gaph(t") << I << ", h" << I << ");\n";
             flops += 6;
             continue;
           }
           case FELIX_OP_EQ: case FELIX_OP_NE: {
-            o << ind << "const double t" << I << " = (" << A << " - " << B << ") + 0.5;\n"
-              << ind << "const double u" << I << " = 0.5 - (" << A << " - " << B << ");\n"
-              << ind << "const double h" << I << " = sm_hyp(t" << I << ");\n"
-              << ind << "const double k" << I << " = sm_hyp(u" << I << ");\n"
-              << ind << "const double p" << I << " = sm_Sh(t" << I << ", h" << I << ");\n"
-              << ind << "const double q" << I << " = sm_Sh(u" << I << ", k" << I << ");\n"
-              << ind << "const double v" << I << " = " << (nd.op == FELIX_OP_EQ ? "" : "1.0 - ") << "p" << I << " * q" << I << ";\n";
+            o << ind << "const " << T << " t" << I << " = (" << A << " - " << B << ") + " << half << ";\n"
+              << ind << "const " << T << " u" << I << " = " << half << " - (" << A << " - " << B << ");\n"
+              << ind << "const float hf" << I << " = sf_hyp((float)t" << I << ");\n"
+              << ind << "const float kf" << I << " = sf_hyp((float)u" << I << ");\n"
+              << ind << "const " << T << " p" << I << " = " << (f32 ? "sf_Sh" : "sm_Sf") << "(t" << I << ", hf" << I << ");\n"
+              << ind << "const " << T << " q" << I << " = " << (f32 ? "sf_Sh" : "sm_Sf") << "(u" << I << ", kf" << I << ");\n"
+              << ind << "const " << T << " v" << I << " = " << (nd.op == FELIX_OP_EQ ? "" : one + " - ") << "p" << I << " * q" << I << ";\n";
             flops += 13;
             continue;
           }
@@ -223,17 +234,17 @@ struct Gen {
         }
       }
       switch (nd.op) {
-        case FELIX_OP_CONST: e = lit(nd.imm); break;
+        case FELIX_OP_CONST: e = cst(nd.imm); break;
         case FELIX_OP_VAR: e = std::string(xname) + std::to_string((int)nd.imm); break;
         case FELIX_OP_ADD: e = A + " + " + B; ++flops; break;
         case FELIX_OP_SUB: e = A + " - " + B; ++flops; break;
         case FELIX_OP_MUL: e = A + " * " + B; ++flops; break;
         case FELIX_OP_DIV: e = divx(A, B); ++flops; break;
         case FELIX_OP_NEG: e = "-" + A; break;
-        case FELIX_OP_POW: e = "pow(" + A + ", " + lit(nd.imm) + ")"; ++flops; break;
-        case FELIX_OP_EXP: e = "exp(" + A + ")"; ++flops; break;
-        case FELIX_OP_LOG: e = "log(" + A + ")"; ++flops; break;
-        case FELIX_OP_SQRT: e = (mode == 0 ? "f_sqrt(" : "sqrt(") + A + ")"; ++flops; break;
+        case FELIX_OP_POW: e = (f32 ? "f_powf(" : "pow(") + A + ", " + cst(nd.imm) + ")"; ++flops; break;
+        case FELIX_OP_EXP: e = (f32 ? "__expf(" : "exp(") + A + ")"; ++flops; break;
+        case FELIX_OP_LOG: e = (f32 ? "__logf(" : "log(") + A + ")"; ++flops; break;
+        case FELIX_OP_SQRT: e = (f32 ? "f_sqrtf(" : mode == 0 ? "f_sqrt(" : "sqrt(") + A + ")"; ++flops; break;
         case FELIX_OP_MIN: e = hard ? "fmin(" + A + ", " + B + ")" : mn + "(" + A + ", " + B + ")"; flops += 6; break;
         case FELIX_OP_MAX: e = hard ? "fmax(" + A + ", " + B + ")" : mx + "(" + A + ", " + B + ")"; flops += 6; break;
         case FELIX_OP_GT: e = hard ? "(" + A + " > " + B + " ? 1.0 : 0.0)" : S + "(" + A + " - " + B + ")"; flops += 6; break;
@@ -246,13 +257,13 @@ struct Gen {
                                    : "1.0 - " + S + "((" + A + " - " + B + ") + 0.5) * " + S + "(0.5 - (" + A + " - " + B + "))"; flops += 13; break;
         case FELIX_OP_AND: e = A + " * " + B; ++flops; break;
         case FELIX_OP_OR: e = A + " + " + B + " - " + A + " * " + B; flops += 3; break;
-        case FELIX_OP_NOT: e = "1.0 - " + A; ++flops; break;
+        case FELIX_OP_NOT: e = one + " - " + A; ++flops; break;
         case FELIX_OP_SELECT: e = hard ? "(" + A + " != 0.0 ? " + B + " : " + C + ")" : C + " + (" + B + " - " + C + ") * " + A; flops += 3; break;
         case FELIX_OP_FLOORDIV: e = hard ? "floor(" + A + " / " + B + ")" : divx(A, B); ++flops; break;
         case FELIX_OP_CEILDIV: e = hard ? "ceil(" + A + " / " + B + ")" : divx(A, B); ++flops; break;
-        default: e = "0.0"; break;
+        default: e = f32 ? "0.f" : "0.0"; break;
       }
-      o << ind << "const double v" << i << " = " << e << ";\n";
+      o << ind << "const " << T << " v" << i << " = " << e << ";\n";
     }
   }
 
@@ -276,62 +287,80 @@ struct Gen {
     return need;
   }
 
-  void emit_adj_decls(const std::vector<bool>& need, const char* ind) {
+  void emit_adj_decls(const std::vector<bool>& need, const char* ind, bool f32) {
     for (int i = 0; i < n; ++i)
-      if (need[i] && d.nodes[i].op != FELIX_OP_VAR) o << ind << "ADJ_T a" << i << " = 0;\n";
+      if (need[i] && d.nodes[i].op != FELIX_OP_VAR) o << ind << (f32 ? "float" : "double") << " a" << i << " = 0;\n";
   }
 
-  // Reverse sweep.  Adjoints are ADJ_T (double by default; float with FELIX_ADJ=f32);
-  // every local partial derivative is evaluated in FP64 from the FP64 forward values and rounded to
-  // ADJ_T once, via J(...), before it multiplies the adjoint.
-  void emit_reverse_body(const std::vector<bool>& need, const char* ind) {
+  // Reverse sweep over the values of emit_forward (mode 0 -> FP64 adjoints, mode 3 -> FP32 adjoints):
+  // every local partial derivative is evaluated from the forward values and multiplies the adjoint.
+  void emit_reverse_body(const std::vector<bool>& need, const char* ind, bool f32 = false) {
+    const std::string T = f32 ? "float" : "double", one = f32 ? "1.f" : "1.0";
     auto acc = [&](int tgt, const std::string& expr, bool neg = false) {
       if (!depvar[tgt]) return;
       o << ind << "  " << adj(tgt) << (neg ? " -= " : " += ") << expr << ";\n";
     };
-    auto J = [](const std::string& e) { return "(ADJ_T)(" + e + ")"; };
+    auto J = [&](const std::string& e) { return "(" + T + ")(" + e + ")"; };
+    const std::string rcp = f32 ? "f_rcpf(" : "f_rcp(";
     for (int i = n - 1; i >= 0; --i) {
       const felix_node& nd = d.nodes[i];
       if (!need[i] || nd.op == FELIX_OP_VAR || nd.op == FELIX_OP_CONST) continue;
       const std::string g = "a" + std::to_string(i);
       const std::string A = "v" + std::to_string(nd.a), B = "v" + std::to_string(nd.b), C = "v" + std::to_string(nd.c);
       const std::string V = "v" + std::to_string(i);
+      const std::string I = std::to_string(i);
       o << ind << "{\n";
+      switch (nd.op) {
+        case FELIX_OP_ADD: case FELIX_OP_SUB: flops_rev += 2; break;
+        case FELIX_OP_NEG: case FELIX_OP_NOT: flops_rev += 1; break;
+        case FELIX_OP_MUL: case FELIX_OP_AND: flops_rev += 4; break;
+        case FELIX_OP_DIV: case FELIX_OP_FLOORDIV: case FELIX_OP_CEILDIV: flops_rev += 6; break;
+        case FELIX_OP_POW: flops_rev += 5; break;
+        case FELIX_OP_EXP: flops_rev += 2; break;
+        case FELIX_OP_LOG: case FELIX_OP_SQRT: flops_rev += 4; break;
+        case FELIX_OP_MIN: case FELIX_OP_MAX: flops_rev += 9; break;
+        case FELIX_OP_GT: case FELIX_OP_GE: case FELIX_OP_LT: case FELIX_OP_LE: flops_rev += 8; break;
+        case FELIX_OP_EQ: case FELIX_OP_NE: flops_rev += 16; break;
+        case FELIX_OP_OR: flops_rev += 6; break;
+        case FELIX_OP_SELECT: flops_rev += 7; break;
+        default: break;
+      }
       switch (nd.op) {
         case FELIX_OP_ADD: acc(nd.a, g); acc(nd.b, g); break;
         case FELIX_OP_SUB: acc(nd.a, g); acc(nd.b, g, true); break;
         case FELIX_OP_MUL: acc(nd.a, g + " * " + J(B)); acc(nd.b, g + " * " + J(A)); break;
         case FELIX_OP_DIV: case FELIX_OP_FLOORDIV: case FELIX_OP_CEILDIV:
-          o << ind << "  const ADJ_T t = " << g << " * " << J("f_rcp(" + B + ")") << ";\n";
+          o << ind << "  const " << T << " t = " << g << " * " << J(rcp + B + ")") << ";\n";
           acc(nd.a, "t"); acc(nd.b, "t * " + J(V), true); break;
         case FELIX_OP_NEG: acc(nd.a, g, true); break;
-        case FELIX_OP_POW: acc(nd.a, g + " * " + J(lit(nd.imm) + " * pow(" + A + ", " + lit(nd.imm - 1.0) + ")")); break;
+        case FELIX_OP_POW:
+          acc(nd.a, g + " * " + J(f32 ? "(float)" + lit(nd.imm) + " * f_powf(" + A + ", (float)" + lit(nd.imm - 1.0) + ")"
+                                       : lit(nd.imm) + " * pow(" + A + ", " + lit(nd.imm - 1.0) + ")")); break;
         case FELIX_OP_EXP: acc(nd.a, g + " * " + J(V)); break;
-        case FELIX_OP_LOG: acc(nd.a, g + " * " + J("f_rcp(" + A + ")")); break;
-        case FELIX_OP_SQRT: acc(nd.a, g + " * " + J("0.5 * f_rcp(" + V + ")")); break;
+        case FELIX_OP_LOG: acc(nd.a, g + " * " + J(rcp + A + ")")); break;
+        case FELIX_OP_SQRT: acc(nd.a, g + " * " + J((f32 ? "0.5f * " : "0.5 * ") + rcp + V + ")")); break;
         case FELIX_OP_MAX:
-          o << ind << "  const ADJ_T s = " << J("sm_Sh(t" + std::to_string(i) + ", h" + std::to_string(i) + ")") << ";\n";
-          acc(nd.a, g + " * s"); acc(nd.b, g + " * ((ADJ_T)1 - s)"); break;
+          o << ind << "  const " << T << " s = " << J((f32 ? "sf_Sh(t" : "sm_Sh(t") + I + ", h" + I + ")") << ";\n";
+          acc(nd.a, g + " * s"); acc(nd.b, g + " * (" + one + " - s)"); break;
         case FELIX_OP_MIN:
-          o << ind << "  const ADJ_T s = " << J("sm_Sh(t" + std::to_string(i) + ", h" + std::to_string(i) + ")") << ";\n";
-          acc(nd.a, g + " * ((ADJ_T)1 - s)"); acc(nd.b, g + " * s"); break;
+          o << ind << "  const " << T << " s = " << J((f32 ? "sf_Sh(t" : "sm_Sh(t") + I + ", h" + I + ")") << ";\n";
+          acc(nd.a, g + " * (" + one + " - s)"); acc(nd.b, g + " * s"); break;
         case FELIX_OP_GT: case FELIX_OP_GE:
-          o << ind << "  const ADJ_T t = " << g << " * " << J("sm_dSh(h" + std::to_string(i) + ")") << ";\n";
+          o << ind << "  const " << T << " t = " << g << " * " << J("sf_dSh(hf" + I + ")") << ";\n";
           acc(nd.a, "t"); acc(nd.b, "t", true); break;
         case FELIX_OP_LT: case FELIX_OP_LE:
-          o << ind << "  const ADJ_T t = " << g << " * " << J("sm_dSh(h" + std::to_string(i) + ")") << ";\n";
+          o << ind << "  const " << T << " t = " << g << " * " << J("sf_dSh(hf" + I + ")") << ";\n";
           acc(nd.a, "t", true); acc(nd.b, "t"); break;
         case FELIX_OP_EQ: case FELIX_OP_NE: {
-          const std::string I = std::to_string(i);
-          o << ind << "  const ADJ_T t = " << (nd.op == FELIX_OP_EQ ? "" : "-") << g << " * "
-            << J("sm_dSh(h" + I + ") * q" + I + " - p" + I + " * sm_dSh(k" + I + ")") << ";\n";
+          o << ind << "  const " << T << " t = " << (nd.op == FELIX_OP_EQ ? "" : "-") << g << " * "
+            << J("(" + T + ")sf_dSh(hf" + I + ") * q" + I + " - p" + I + " * (" + T + ")sf_dSh(kf" + I + ")") << ";\n";
           acc(nd.a, "t"); acc(nd.b, "t", true); break;
         }
         case FELIX_OP_AND: acc(nd.a, g + " * " + J(B)); acc(nd.b, g + " * " + J(A)); break;
-        case FELIX_OP_OR: acc(nd.a, g + " * " + J("1.0 - " + B)); acc(nd.b, g + " * " + J("1.0 - " + A)); break;
+        case FELIX_OP_OR: acc(nd.a, g + " * " + J(one + " - " + B)); acc(nd.b, g + " * " + J(one + " - " + A)); break;
         case FELIX_OP_NOT: acc(nd.a, g, true); break;
         case FELIX_OP_SELECT:
-          acc(nd.a, g + " * " + J(B + " - " + C)); acc(nd.b, g + " * " + J(A)); acc(nd.c, g + " * " + J("1.0 - " + A)); break;
+          acc(nd.a, g + " * " + J(B + " - " + C)); acc(nd.b, g + " * " + J(A)); acc(nd.c, g + " * " + J(one + " - " + A)); break;
         default: break;
       }
       o << ind << "}\n";
@@ -393,29 +422,16 @@ int SpaceDesc::n_roots_total() const {
   return (int)croots.size() + n_split + (int)split_extent.size() + 2 * n_int;
 }
 
-std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, CodegenInfo* info) {
+std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, bool trace, CodegenInfo* info) {
   Gen g(d);
   std::ostringstream& o = g.o;
-  const bool trace = std::getenv("FELIX_TRACE") != nullptr;   // debug: per-block phase timestamps
   const int M = d.n_vars, K = (int)d.froots.size(), Ru = (int)d.croots.size();
   const int R = d.n_roots_total(), Ra = R - Ru;
   const int NS = d.n_statements, K0 = K / NS;   // per-statement feature vectors (TenSet segment sum)
   // feature k -> (statement, index within the statement's vector)
   auto fs = [&](int k) { return k / K0; };
   auto fk = [&](int k) { return k % K0; };
-  // NREPv == 0: cone-per-CTA kernels.  A cluster of PG CTAs (PG warps each) owns PG x 32 candidates; CTA q
-  // runs cone q for all of them (its warps share one cone's straight-line code and instruction fetches),
-  // warp w working on the 32 candidates CTA w owns: it reads their x from, and writes features / partial
-  // adjoints to, CTA w's shared memory (DSMEM).  Each CTA then finishes its own 32 rows as before.
-  const bool cpb = NREPv == 0;
-  if (cpb) NREPv = 1;
-  o << "#define CPB " << (cpb ? 1 : 0) << "\n";
-  o << "#define CONE_OF_WARP " << (cpb ? "cone" : "wq") << "\n";
-  // cone-phase access to the owner's staged x / features / partials (owner = warp index in CPB mode)
-  o << "#if CPB\n#define X_OWN(ptr) cl_ld_f64(&(ptr), (unsigned)wq)\n#define ST_OWN32(ptr, v) cl_st_f32(&(ptr), (unsigned)wq, (v))\n"
-       "#define ST_OWN64(ptr, v) cl_st_f64(&(ptr), (unsigned)wq, (v))\n#define BLOCK_SYNC() cl_sync()\n"
-       "#else\n#define X_OWN(ptr) (ptr)\n#define ST_OWN32(ptr, v) ((ptr) = (v))\n#define ST_OWN64(ptr, v) ((ptr) = (v))\n"
-       "#define BLOCK_SYNC() __syncthreads()\n#endif\n";
+  if (NREPv < 1) NREPv = 1;
   o << kPrelude;
 
   if (trace)
@@ -423,11 +439,6 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
          "#define TSTAMP(k, s) do { if (threadIdx.x == 0 && blockIdx.x < 8192) { unsigned long long t_; asm volatile(\"mov.u64 %0, %globaltimer;\" : \"=l\"(t_)); felix_trace[k][blockIdx.x][s] = t_; } } while (0)\n";
   else
     o << "#define TSTAMP(k, s) do {} while (0)\n";
-  // reverse-sweep adjoint type: double by default; FELIX_ADJ=f32 uses float adjoints (parity-green,
-  // measured no faster: C2 reverse kernel 16.7 us either way, C5 -2 %)
-  const char* adj_env = std::getenv("FELIX_ADJ");
-  const bool adj64 = !(adj_env && std::string(adj_env) == "f32");
-  o << "#define ADJ_T " << (adj64 ? "double" : "float") << "\n";
   o << "#define NV " << M << "\n#define NF " << K << "\n#define NRU " << Ru << "\n#define NR " << R
     << "\n#define NRA " << Ra << "\n#define K0P " << K0p << "\n#define PG " << P << "\n#define NS " << NS
     << "\n#define NREP " << NREPv << "\n";
@@ -471,7 +482,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     return used;
   };
   // arithmetic ops of one full forward evaluation (reported by felix_space_info)
-  int64_t flops_fwd = 0;
+  int64_t flops_fwd = 0, flops_rev = 0;
   {
     std::ostringstream save;
     save << o.str();
@@ -479,6 +490,11 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     g.flops = 0;
     g.emit_forward(all, 0, "x");
     flops_fwd = g.flops;
+    std::vector<int> allroots(d.froots.begin(), d.froots.end());
+    allroots.insert(allroots.end(), d.croots.begin(), d.croots.end());
+    g.flops_rev = 0;
+    g.emit_reverse_body(g.rev_live(all, allroots), "");
+    flops_rev = g.flops_rev;
     o.str("");
     o.clear();
     o << save.str();
@@ -512,7 +528,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     o << ind << "  default: break;\n" << ind << "}\n";
   };
   o << "template <int ADAM>\n__device__ __forceinline__ void fwd_body(float* yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr,\n"
-    << "    float* mv, float* vv, const double* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part,\n"
+    << "    float* mv, float* vv, const float* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part,\n"
     << "    int n_head_tiles, int ld_c, float head_b, float lam, float lr, float b1, float b2, float eps) {\n"
     << "  __shared__ float sphi_all[NREP][NS][32][K0P + 1];\n"
     << "  __shared__ double sx_all[NREP][NV][32];   // x = exp(y), computed once per replica and shared by its groups\n"
@@ -520,12 +536,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  float (&sphi)[NS][32][K0P + 1] = sphi_all[rep];\n"
     << "  double (&sx)[NV][32] = sx_all[rep];\n"
     << "  const int lane = threadIdx.x & 31, wq = tid >> 5;\n"
-    << "#if CPB\n"
-    << "  const int cone = (int)cl_rank();\n"
-    << "  const int c0 = (blockIdx.x / PG) * (PG * 32) + cone * 32;   // the 32 rows this CTA owns\n"
-    << "#else\n"
     << "  const int c0 = (blockIdx.x * NREP + rep) * 32;\n"
-    << "#endif\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
     << "  TSTAMP(0, 0);\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");   // y is the previous step's output\n"
@@ -539,11 +550,11 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "    float (&sy)[NV][32] = sya_all[rep];\n    unsigned* sbad = sbad_all[rep];\n"
     << "    constexpr int NJ = (NV + PG - 1) / PG;\n"
     << "    const int cl = c0 + lane;\n    const bool live = cl < n;\n    const int cc = live ? cl : n - 1;\n"
-    << "    float yl[NJ], ml[NJ], vl[NJ];\n    double gxa[NJ];\n"
+    << "    float yl[NJ], ml[NJ], vl[NJ], gxa[NJ];\n"
     << "#pragma unroll\n    for (int jj = 0; jj < NJ; ++jj) {\n"
     << "      const int j = wq + PG * jj;\n      if (j >= NV) break;\n"
     << "      yl[jj] = yv[(size_t)j * ldy + cc]; ml[jj] = mv[(size_t)j * n + cc]; vl[jj] = vv[(size_t)j * n + cc];\n"
-    << "      double a = 0.0;\n#pragma unroll\n      for (int q = 0; q < PG; ++q) a += part[((size_t)q * NV + j) * n + cc];\n"
+    << "      float a = 0.f;\n#pragma unroll\n      for (int q = 0; q < PG; ++q) a += part[((size_t)q * NV + j) * n + cc];\n"
     << "      gxa[jj] = a;\n    }\n"
     // the loss inputs are requested with the rest (one memory round trip before the first barrier)
     << "    double pen_ = 0.0;\n"
@@ -563,7 +574,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "      float gyv[NJ];\n"
     << "#pragma unroll\n      for (int jj = 0; jj < NJ; ++jj) {\n"
     << "        const int j = wq + PG * jj;\n        if (j >= NV) break;\n"
-    << "        double gd = gxa[jj];   // the partials are dL/dy already (x_j folded in by felix_rev_sc)\n";
+    << "        double gd = (double)gxa[jj];   // the partials are dL/dy already (x_j folded in by felix_rev_sc)\n";
   emit_auto_grad_switch("        ");
   o << "        gyv[jj] = (float)gd;\n        ok = ok && isfinite(gyv[jj]);\n      }\n"
     << "      const unsigned bad = __ballot_sync(0xffffffffu, !ok);\n"
@@ -585,25 +596,25 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "        sx[j][lane] = exp((double)yy);\n      }\n"
     << "    }\n  }\n"
     << "  for (int k = tid; k < NS * 32 * (K0P + 1); k += PG * 32) (&sphi[0][0][0])[k] = 0.f;\n"
-    << "  BLOCK_SYNC();\n";
+    << "  __syncthreads();\n";
   for (int q = 0; q < P; ++q) {
-    o << "  if (CONE_OF_WARP == " << q << ") {\n";
+    o << "  if (wq == " << q << ") {\n";
     if (q == 0)
       for (int k = 0; k < K; ++k)
         if (!g.depvar[d.froots[k]]) {
           // constant feature: value of its (var-free) cone, evaluated here
           o << "    {\n";
           g.emit_forward(g.cone({d.froots[k]}), 0, "x", "      ");
-          o << "      ST_OWN32(sphi[" << fs(k) << "][lane][" << fk(k) << "], slogf_(v" << d.froots[k] << "));\n    }\n";
+          o << "      sphi[" << fs(k) << "][lane][" << fk(k) << "] = slogf_(v" << d.froots[k] << ");\n    }\n";
         }
     const auto used = vars_in(fcone[q]);
     for (int j = 0; j < M; ++j)
-      if (used[j]) o << "    const double x" << j << " = X_OWN(sx[" << j << "][lane]);\n";
+      if (used[j]) o << "    const double x" << j << " = sx[" << j << "][lane];\n";
     g.emit_forward(fcone[q], 0, "x", "    ");
-    for (int k : part.feat[q]) o << "    ST_OWN32(sphi[" << fs(k) << "][lane][" << fk(k) << "], slogf_(v" << d.froots[k] << "));\n";
+    for (int k : part.feat[q]) o << "    sphi[" << fs(k) << "][lane][" << fk(k) << "] = slogf_(v" << d.froots[k] << ");\n";
     o << "  }\n";
   }
-  o << "  BLOCK_SYNC();\n  TSTAMP(0, 2);\n"
+  o << "  __syncthreads();\n  TSTAMP(0, 2);\n"
     << "  // rows c0 .. c0+31 of each statement are contiguous: K0P/8 uint4 per row for hi and for lo\n"
     << "#pragma unroll\n"
     << "  for (int it = 0; it < (NS * 32 * (K0P / 8) + PG * 32 - 1) / (PG * 32); ++it) {\n"
@@ -627,7 +638,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd(const float* __restrict__ yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr) {\n"
     << "  fwd_body<0>(const_cast<float*>(yv), n, ldy, phi_hi, phi_lo, step_ctr, nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f);\n}\n"
     << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd_adam(float* yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr,\n"
-    << "    float* mv, float* vv, const double* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part,\n"
+    << "    float* mv, float* vv, const float* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part,\n"
     << "    int n_head_tiles, int ld_c, float head_b, float lam, float lr, float b1, float b2, float eps) {\n"
     << "  fwd_body<1>(yv, n, ldy, phi_hi, phi_lo, step_ctr, mv, vv, part, pen, c_part, n_head_tiles, ld_c, head_b, lam, lr, b1, b2, eps);\n}\n\n";
 
@@ -637,7 +648,8 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
   o << "template <int EVAL>\n__device__ __forceinline__ void rev_body(float* __restrict__ yv, const float* __restrict__ yin, int n, int ldy,\n"
     << "    const float* __restrict__ dphi, int ld_dphi, const float* __restrict__ c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
     << "    float* __restrict__ mv, float* __restrict__ vv, const int* step_ctr, float lr, float b1, float b2, float eps,\n"
-    << "    float* __restrict__ o_phi, float* __restrict__ o_g, float* __restrict__ o_cost, float* __restrict__ o_loss, float* __restrict__ o_grad) {\n"
+    << "    float* __restrict__ o_phi, float* __restrict__ o_g, float* __restrict__ o_cost, float* __restrict__ o_loss, float* __restrict__ o_grad,\n"
+    << "    double* __restrict__ o_F) {\n"
     << "  extern __shared__ double smem[];\n"
     << "  const int rep = threadIdx.x / (PG * 32), tid = threadIdx.x % (PG * 32);\n"
     << "  constexpr int REPW = ((PG * NV * 32 + PG * 32 + (NRA > 0 ? NRA : 1) * 32) * 8 + NV * 32 * 4 + 15) / 16 * 2;   // doubles per replica\n"
@@ -646,14 +658,8 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  double* spa = spen + PG * 32;                          // [NRA][32]\n"
     << "  float* sy = reinterpret_cast<float*>(spa + (NRA > 0 ? NRA : 1) * 32);   // [NV][32]\n"
     << "  const int lane = threadIdx.x & 31, wq = tid >> 5;\n"
-    << "#if CPB\n"
-    << "  const int cone = (int)cl_rank();\n"
-    << "  const int c0 = (blockIdx.x / PG) * (PG * 32) + cone * 32, c = c0 + lane;   // own rows (finish)\n"
-    << "  const int cw = (blockIdx.x / PG) * (PG * 32) + wq * 32 + lane;            // this warp's candidate (cone phase)\n"
-    << "#else\n"
     << "  const int c0 = (blockIdx.x * NREP + rep) * 32, c = c0 + lane;\n"
     << "  const int cw = c;\n"
-    << "#endif\n"
     << "  const bool live = c < n;\n"
     << "  const int cc = live ? c : n - 1;\n"
     << "  const bool livew = cw < n;\n"
@@ -667,7 +673,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  __shared__ double sx_all[NREP][NV * 32];\n"
     << "  double* sx = sx_all[rep];\n"
     << "  for (int e = tid; e < NV * 32; e += PG * 32) { const int j = e >> 5, l = e & 31; const int cl = c0 + l; const float yy = yin[(size_t)j * ldy + (cl < n ? cl : n - 1)]; sy[e] = yy; sx[e] = exp((double)yy); }\n"
-    << "  BLOCK_SYNC();\n"
+    << "  __syncthreads();\n"
     << "  constexpr int NJ = (NV + PG - 1) / PG;   // vars handled by this thread: j = wq + PG * jj\n"
     // Adam state and the head partials go to shared memory with cp.async (no registers held across the
     // DAG, latency hidden behind it); consumed after the cone groups finish
@@ -682,50 +688,60 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  if (cp_smem) for (int e = tid; e < nht_all * 32; e += PG * 32) { const int i = e >> 5, l = e & 31; const int cl = c0 + l < n ? c0 + l : n - 1; cp_async4(&scp[e], c_part + (size_t)(i % n_head_tiles) * ld_c + (size_t)(i / n_head_tiles) * n + cl); }\n"
     << "  cp_async_commit();\n"
     << "  const int tstep = EVAL ? 1 : *step_ctr;\n";
+  // Per cone: with EVAL, the FP64 search forward (mode 0) for the phi / F / g outputs; then, in both
+  // kernels, the FP32 forward recompute + FP32 reverse sweep of the search (DESIGN.md "Precision of the
+  // expression kernels"), penalties and partial adjoints to shared memory.
   for (int q = 0; q < P; ++q) {
-    o << "  if (CONE_OF_WARP == " << q << ") {\n";
+    o << "  if (wq == " << q << ") {\n";
+    const auto used = vars_in(rcone[q]);
+    o << "    if constexpr (EVAL) {\n";
     if (q == 0) {
-      o << "    if (EVAL && o_phi && livew) {\n";
+      o << "    if ((o_phi || o_F) && livew) {\n";
       for (int k = 0; k < K; ++k)
         if (!g.depvar[d.froots[k]]) {
           o << "      {\n";
           g.emit_forward(g.cone({d.froots[k]}), 0, "x", "        ");
-          o << "        o_phi[(size_t)" << k << " * n + cw] = slogf_(v" << d.froots[k] << ");\n      }\n";
+          o << "        if (o_phi) o_phi[(size_t)" << k << " * n + cw] = slogf_(v" << d.froots[k] << ");\n"
+            << "        if (o_F) o_F[(size_t)" << k << " * n + cw] = v" << d.froots[k] << ";\n      }\n";
         }
       o << "    }\n";
     }
-    const auto used = vars_in(rcone[q]);
     for (int j = 0; j < M; ++j)
-      if (used[j]) o << "    const double x" << j << " = X_OWN(sx[" << j << " * 32 + lane]);\n";
+      if (used[j]) o << "    const double x" << j << " = sx[" << j << " * 32 + lane];\n";
     g.emit_forward(rcone[q], 0, "x", "    ");
-    // user-root penalties of this group
-    o << "    double pen = 0.0;\n";
-    for (int r : part.cons[q]) {
-      o << "    const double p" << r << " = fmax(v" << d.croots[r] << ", 0.0); pen += p" << r << " * p" << r << ";\n";
-      o << "    if (EVAL && o_g && livew) o_g[(size_t)" << r << " * n + cw] = (float)v" << d.croots[r] << ";\n";
-    }
-    o << "    ST_OWN64(spen[" << q << " * 32 + lane], pen);\n";
-    o << "    if (EVAL && o_phi && livew) {\n";
+    for (int r : part.cons[q]) o << "    if (o_g && livew) o_g[(size_t)" << r << " * n + cw] = (float)v" << d.croots[r] << ";\n";
+    o << "    if (o_phi && livew) {\n";
     for (int k : part.feat[q]) o << "      o_phi[(size_t)" << k << " * n + cw] = slogf_(v" << d.froots[k] << ");\n";
     o << "    }\n";
+    o << "    if (o_F && livew) {\n";
+    for (int k : part.feat[q]) o << "      o_F[(size_t)" << k << " * n + cw] = v" << d.froots[k] << ";\n";
+    o << "    }\n";
+    o << "    }\n    {\n";
+    for (int j = 0; j < M; ++j)
+      if (used[j]) o << "    const float x" << j << " = (float)sx[" << j << " * 32 + lane];\n";
+    g.emit_forward(rcone[q], 3, "x", "    ");
+    // user-root penalties of this group
+    o << "    float pen = 0.f;\n";
+    for (int r : part.cons[q]) o << "    const float p" << r << " = fmaxf(v" << d.croots[r] << ", 0.f); pen += p" << r << " * p" << r << ";\n";
+    o << "    spen[" << q << " * 32 + lane] = (double)pen;\n";
     const auto need = g.rev_live(rcone[q], rroots_g[q]);
-    g.emit_adj_decls(need, "    ");
-    for (int j = 0; j < M; ++j) o << "    ADJ_T gx" << j << " = 0;\n";
+    g.emit_adj_decls(need, "    ", true);
+    for (int j = 0; j < M; ++j) o << "    float gx" << j << " = 0.f;\n";
     for (int k : part.feat[q]) {
       const int r = d.froots[k];
-      o << "    " << g.adj(r) << " += (ADJ_T)((double)dphi[(size_t)" << fk(k) << " * ld_dphi + (size_t)" << fs(k)
-        << " * n + ccw] * slogp_(v" << r << "));\n";
+      o << "    " << g.adj(r) << " += dphi[(size_t)" << fk(k) << " * ld_dphi + (size_t)" << fs(k)
+        << " * n + ccw] * slogpf_(v" << r << ");\n";
     }
     for (int r : part.cons[q]) {
       const int nd = d.croots[r];
-      if (g.depvar[nd]) o << "    " << g.adj(nd) << " += (ADJ_T)(2.0 * dlam * p" << r << ");\n";
+      if (g.depvar[nd]) o << "    " << g.adj(nd) << " += 2.f * lam * p" << r << ";\n";
     }
-    g.emit_reverse_body(need, "    ");
-    for (int j = 0; j < M; ++j) o << "    ST_OWN64(spart[(" << q << " * NV + " << j << ") * 32 + lane], (double)gx" << j << ");\n";
-    o << "  }\n";
+    g.emit_reverse_body(need, "    ", true);
+    for (int j = 0; j < M; ++j) o << "    spart[(" << q << " * NV + " << j << ") * 32 + lane] = (double)gx" << j << ";\n";
+    o << "    }\n  }\n";
   }
   // automatic roots (warp 0) from the staged y
-  o << "  cp_async_wait_all();\n  BLOCK_SYNC();\n  if (!EVAL) TSTAMP(1, 2);\n"
+  o << "  cp_async_wait_all();\n  __syncthreads();\n  if (!EVAL) TSTAMP(1, 2);\n"
     << "  if (wq == 0) {\n";
   for (int j = 0; j < M; ++j) o << "    const double y" << j << " = (double)sy[" << j << " * 32 + lane];\n";
   for (size_t q = 0; q < autos.size(); ++q) {
@@ -790,74 +806,73 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  }\n}\n\n";
   o << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_adam(float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
     << "    float* mv, float* vv, const int* step_ctr, float lr, float b1, float b2, float eps, float* o_loss) {\n"
-    << "  rev_body<0>(yv, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, mv, vv, step_ctr, lr, b1, b2, eps, nullptr, nullptr, nullptr, o_loss, nullptr);\n}\n";
+    << "  rev_body<0>(yv, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, mv, vv, step_ctr, lr, b1, b2, eps, nullptr, nullptr, nullptr, o_loss, nullptr, nullptr);\n}\n";
   o << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_eval(const float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
-    << "    float* o_phi, float* o_g, float* o_cost, float* o_loss, float* o_grad) {\n"
-    << "  rev_body<1>(nullptr, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, nullptr, nullptr, nullptr, 0.f, 0.f, 0.f, 0.f, o_phi, o_g, o_cost, o_loss, o_grad);\n}\n\n";
+    << "    float* o_phi, float* o_g, float* o_cost, float* o_loss, float* o_grad, double* o_F) {\n"
+    << "  rev_body<1>(nullptr, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, nullptr, nullptr, nullptr, 0.f, 0.f, 0.f, 0.f, o_phi, o_g, o_cost, o_loss, o_grad, o_F);\n}\n\n";
 
   // ---------------------------------------------------------------- split-cone search kernels
   // felix_rev_sc runs ONE cone per CTA (block-uniform q = blockIdx.x % PG) for W x 32 candidates, so the
   // warps of an SM share one cone's straight-line code and instruction fetches (felix_rev_adam puts P
   // different cones in one CTA and is instruction-fetch bound: 42 % of its stall samples are
-  // no_instructions).  Cone q's CTA writes its partial adjoints part[q][j][c] = dL/dx_j and its user-root
+  // no_instructions).  Cone q's CTA writes its partial adjoints part[q][j][c] = x_j dL/dx_j = this cone's dL/dy_j (x_j folded in) and its user-root
   // penalty pen[q][c]; the cross-cone sums and Adam happen after the kernel boundary: in the next step's
   // forward (felix_fwd_adam, whose CTAs own whole candidates) and, after the last step, in felix_adam_sc.
   // Step counter: starts at 1, felix_rev_sc adds 1 (block 0, after griddepcontrol.wait; no CTA of the
   // reverse kernel reads it), so the forward and the MLP chain of step t see t and Adam step t - 1 is due.
   // Measured and dropped: Adam by the last of the P cone CTAs to arrive (+8 us at C2: a serial tail at
   // 255 registers), and a split-cone forward (its 2-byte feature-column stores: 1.7x slower at C2).
+  // The whole kernel is FP32 (forward recompute, seeds, reverse sweep): its outputs are gradients, whose
+  // tolerance is 1e-3; half the registers and a third
+  // of the instructions of the FP64 form, so the straight-line cone code streams through the SM's
+  // instruction fetch faster.
   o << "extern \"C\" __global__ void __launch_bounds__(256) felix_rev_sc(const float* __restrict__ yv, int n, int ldy, const float* __restrict__ dphi, int ld_dphi,\n"
-    << "    float lam, double* __restrict__ part, double* __restrict__ pen, int* step_ctr, int G) {\n"
+    << "    float lam, float* __restrict__ part, double* __restrict__ pen, int* step_ctr) {\n"
     << "  const int cq_ = blockIdx.x % PG;\n"
+    << "  const int c = ((blockIdx.x / PG) * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32 + (threadIdx.x & 31);\n"
+    << "  const bool live = c < n;\n  const int ccw = live ? c : n - 1;\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n"
-    << "  if (blockIdx.x == 0 && threadIdx.x == 0) *step_ctr += 1;\n"
-    << "  const double dlam = (double)lam;\n";
-  // G groups of W x 32 candidates per CTA, one after the other: the second pass over the cone's
-  // straight-line code runs from the instruction caches the first one filled
+    << "  if (blockIdx.x == 0 && threadIdx.x == 0) *step_ctr += 1;\n";
   for (int q = 0; q < P; ++q) {
-    o << "  if (cq_ == " << q << ") {\n"
-      << "#pragma unroll 1\n"
-      << "  for (int g_ = 0; g_ < G; ++g_) {\n"
-      << "    const int c = (((blockIdx.x / PG) * G + g_) * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32 + (threadIdx.x & 31);\n"
-      << "    const bool live = c < n;\n    const int ccw = live ? c : n - 1;\n";
+    o << "  if (cq_ == " << q << ") {\n";
     const auto used = vars_in(rcone[q]);
     for (int j = 0; j < M; ++j)
-      if (used[j]) o << "    const double x" << j << " = exp((double)yv[(size_t)" << j << " * ldy + ccw]);\n";
-    g.emit_forward(rcone[q], 0, "x", "    ");
-    o << "    double pq = 0.0;\n";
-    for (int r : part.cons[q]) o << "    const double pr" << r << " = fmax(v" << d.croots[r] << ", 0.0); pq += pr" << r << " * pr" << r << ";\n";
+      if (used[j]) o << "    const float x" << j << " = __expf(yv[(size_t)" << j << " * ldy + ccw]);\n";
+    g.emit_forward(rcone[q], 3, "x", "    ");
+    o << "    float pq = 0.f;\n";
+    for (int r : part.cons[q]) o << "    const float pr" << r << " = fmaxf(v" << d.croots[r] << ", 0.f); pq += pr" << r << " * pr" << r << ";\n";
     const auto need = g.rev_live(rcone[q], rroots_g[q]);
-    g.emit_adj_decls(need, "    ");
-    for (int j = 0; j < M; ++j) o << "    ADJ_T gx" << j << " = 0;\n";
+    g.emit_adj_decls(need, "    ", true);
+    for (int j = 0; j < M; ++j) o << "    float gx" << j << " = 0.f;\n";
     for (int k : part.feat[q]) {
       const int r = d.froots[k];
-      o << "    " << g.adj(r) << " += (ADJ_T)((double)dphi[(size_t)" << fk(k) << " * ld_dphi + (size_t)" << fs(k)
-        << " * n + ccw] * slogp_(v" << r << "));\n";
+      o << "    " << g.adj(r) << " += dphi[(size_t)" << fk(k) << " * ld_dphi + (size_t)" << fs(k)
+        << " * n + ccw] * slogpf_(v" << r << ");\n";
     }
     for (int r : part.cons[q]) {
       const int nd = d.croots[r];
-      if (g.depvar[nd]) o << "    " << g.adj(nd) << " += (ADJ_T)(2.0 * dlam * pr" << r << ");\n";
+      if (g.depvar[nd]) o << "    " << g.adj(nd) << " += 2.f * lam * pr" << r << ";\n";
     }
-    g.emit_reverse_body(need, "    ");
+    g.emit_reverse_body(need, "    ", true);
     // partial dL/dy_j = x_j * dL/dx_j of this cone (x_j is at hand here; the Adam prologue needs no exp)
-    o << "    if (live) {\n      pen[(size_t)" << q << " * n + c] = pq;\n";
+    o << "    if (live) {\n      pen[(size_t)" << q << " * n + c] = (double)pq;\n";
     for (int j = 0; j < M; ++j)
-      o << "      part[((size_t)" << q << " * NV + " << j << ") * n + c] = " << (used[j] ? "x" + std::to_string(j) + " * (double)gx" + std::to_string(j) : std::string("0.0")) << ";\n";
-    o << "    }\n  }\n  }\n";
+      o << "      part[((size_t)" << q << " * NV + " << j << ") * n + c] = " << (used[j] ? "x" + std::to_string(j) + " * gx" + std::to_string(j) : std::string("0.f")) << ";\n";
+    o << "    }\n  }\n";
   }
   o << "}\n\n";
   // felix_adam_sc: the last Adam step (thread per candidate, in place) + the final loss
   o << "extern \"C\" __global__ void __launch_bounds__(128) felix_adam_sc(float* yv, int n, int ldy, float* mv, float* vv,\n"
-    << "    const double* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part, int n_head_tiles, int ld_c,\n"
-    << "    float head_b, float lam, float lr, float b1, float b2, float eps, const int* step_ctr, float* o_loss) {\n"
+    << "    const float* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part, int n_head_tiles, int ld_c,\n"
+    << "    float head_b, float lam, float lr, float b1, float b2, float eps, const int* step_ctr, float* o_loss, float* o_grad) {\n"
     << "  const int c = blockIdx.x * blockDim.x + threadIdx.x;\n  if (c >= n) return;\n"
     << "  const int s_ = *step_ctr - 1;\n  if (s_ <= 0) return;\n"
     << "  const double dlam = (double)lam;\n"
-    << "  float syv[NV], ml[NV], vl[NV];\n  double gxa[NV];\n"
+    << "  float syv[NV], ml[NV], vl[NV], gxa[NV];\n"
     << "#pragma unroll\n  for (int j = 0; j < NV; ++j) {\n"
     << "    syv[j] = yv[(size_t)j * ldy + c]; ml[j] = mv[(size_t)j * n + c]; vl[j] = vv[(size_t)j * n + c];\n"
-    << "    double a = 0.0;\n#pragma unroll\n    for (int q = 0; q < PG; ++q) a += part[((size_t)q * NV + j) * n + c];\n"
+    << "    float a = 0.f;\n#pragma unroll\n    for (int q = 0; q < PG; ++q) a += part[((size_t)q * NV + j) * n + c];\n"
     << "    gxa[j] = a;\n  }\n"
     << "  double pen_ = 0.0;\n#pragma unroll\n  for (int q = 0; q < PG; ++q) pen_ += pen[(size_t)q * n + c];\n"
     << "  float cst = head_b * NS;\n"
@@ -867,9 +882,11 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
     << "  if (o_loss) o_loss[c] = loss;\n"
     << "  bool ok = isfinite(loss);\n  float gy[NV];\n"
     << "#pragma unroll\n  for (int j = 0; j < NV; ++j) {\n"
-    << "    double gd = gxa[j];\n";
+    << "    double gd = (double)gxa[j];\n";
   emit_auto_grad_switch("    ");
   o << "    gy[j] = (float)gd;\n    ok = ok && isfinite(gy[j]);\n  }\n"
+    << "  if (o_grad) {   // test hook (felix_eval_ex search_path): dL/dy as the search's Adam step sees it, no update\n"
+    << "#pragma unroll\n    for (int j = 0; j < NV; ++j) o_grad[(size_t)j * n + c] = gy[j];\n    return;\n  }\n"
     << "  if (!ok) return;\n"
     << "  const float bc1 = 1.f - powf(b1, (float)s_), bc2 = 1.f - powf(b2, (float)s_);\n"
     << "  const float step = lr / bc1, rb = 1.f / sqrtf(bc2);\n"
@@ -964,6 +981,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, C
 
   if (info) {
     info->flops_fwd = flops_fwd;
+    info->flops_rev = flops_rev;
     info->rev_smem_bytes = NREPv * (((P * M * 32 + P * 32 + std::max(Ra, 1) * 32) * 8 + M * 32 * 4 + 15) / 16 * 16);
   }
   return o.str();

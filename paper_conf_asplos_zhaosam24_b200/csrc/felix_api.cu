@@ -6,6 +6,8 @@
 // and after the search (lines 20-21): rounding (K5), hard features + validity (NVRTC), FP64 MLP
 // scoring (K6), dedup + top-k (K7).
 #include <algorithm>
+#include <atomic>
+#include <set>
 #include <chrono>
 #include <cmath>
 #include <cstring>
@@ -29,6 +31,25 @@ namespace felix {
 static thread_local std::string g_last_error;
 void set_error(const std::string& m) { g_last_error = m; }
 
+uint64_t next_uid() {
+  static std::atomic<uint64_t> ctr{1};
+  return ctr.fetch_add(1);
+}
+
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) is per device context: remember (kernel, device)
+// pairs already configured, under a mutex (concurrent callers, several GPUs in one process).
+static void set_smem_attr(const void* fn, int bytes, bool nonportable_cluster = false) {
+  static std::mutex mu;
+  static std::set<std::pair<const void*, int>> done;
+  int dev = 0;
+  CUDA_OK(cudaGetDevice(&dev));
+  std::lock_guard<std::mutex> lk(mu);
+  if (done.count({fn, dev})) return;
+  CUDA_OK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
+  if (nonportable_cluster) CUDA_OK(cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 0));
+  done.insert({fn, dev});
+}
+
 // ============================================================================ GEMM dispatch
 struct GemmLaunch {
   int epi = 0, bn = 0, stages = 2;
@@ -51,12 +72,7 @@ static cudaLaunchAttribute g_pdl_attr = [] {
 template <int BN, int EPI>
 static void launch_gemm_t(const GemmLaunch& g, cudaStream_t st) {
   auto kern = mlp_gemm_kernel<BN, EPI>;
-  static bool attr_set = false;   // per instantiation; devices share the same limit on one box
-  if (!attr_set) {
-    CUDA_OK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 GemmCfg<BN>::smem_bytes(GemmCfg<BN>::MAX_STAGES)));
-    attr_set = true;
-  }
+  set_smem_attr(reinterpret_cast<const void*>(kern), GemmCfg<BN>::smem_bytes(GemmCfg<BN>::MAX_STAGES));
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = g.grid;
   cfg.blockDim = dim3(128);
@@ -112,11 +128,23 @@ static CUtensorMap make_tmap(const void* base, int64_t rows, int64_t cols, int b
   return m;
 }
 
+// ============================================================================ execution knobs
+// Process-wide knobs set through felix_tune (experiments and tests only; the library never reads the
+// environment).  -1 = the measured default.
+struct Tuning {
+  std::atomic<int> mlp{-1};          // 0 tile kernel, 1 persistent chain, 2 per-layer GEMMs
+  std::atomic<int> P{-1};            // cone-partition width of the DAG kernels
+  std::atomic<int> R{-1};            // replicas of the cone groups per block
+  std::atomic<int> scw{-1};          // warps per split-cone reverse CTA
+  std::atomic<int> chunks{-1};       // concurrent population chunks
+  std::atomic<int> sc{-1};           // split-cone reverse kernel (1) or cone-group kernel (0)
+  std::atomic<int> tile_cg{-1};      // tile kernel: 1-SM tiles (1) or 2-SM cta_group::2 pairs (2)
+  std::atomic<int> codegen_P{-1}, codegen_R{-1};   // felix_codegen's variant
+  std::atomic<int> trace{0};         // per-block %globaltimer stamps in kernels generated afterwards
+};
+static Tuning g_tune;
+
 // ============================================================================ per-(space, model, n) plan
-static bool mask_exact() {
-  const char* e = std::getenv("FELIX_MASK_EXACT");
-  return !(e && std::atoi(e) == 0);
-}
 struct Plan {
   const CostModel* cm = nullptr;
   int64_t n = -1, n_pad = 0;
@@ -128,44 +156,35 @@ struct Plan {
   std::vector<GemmLaunch> gemms;           // per-layer kernels (FELIX_MLP=layers)
   ChainParams chain{};                     // persistent all-layer kernel
   int chain_grid = 0;
-  int chain_cs = 1;                        // 4: cluster chain (one 4-CTA cluster per row block, cluster barriers)
   DevBuf grid_bar;
   DevBuf chain_flags;                      // dataflow chain: per (layer, row block) completion counters
   bool tile_ok = false;                    // model has the shape mlp_tile_kernel is specialised for
   TileParams tile{};                       // tile-local fused MLP (default when tile_ok)
   int tile_grid = 0;
-  int tile_cg = 1;                         // 1 = one SM per 128-row tile; FELIX_TILE_CG=2: 2-SM cta_group::2 pairs
+  int tile_cg = 1;                         // 1 = one SM per 128-row tile; 2 = 2-SM cta_group::2 pairs (felix_tune)
   bool tile_full_wave = false;             // >= one 128-row tile per SM
   int mode = 0;                            // MlpMode, fixed when the plan is built
 };
 
 // MLP execution mode: "tile" (tile-local fused kernel), "chain" (persistent layer-by-layer kernel),
-// "layers" (one kernel per GEMM).  FELIX_MLP overrides.  Default (measured on B200, DESIGN.md
+// "layers" (one kernel per GEMM).  felix_tune("mlp") overrides.  Default (measured on B200, DESIGN.md
 // "MLP modes"): a tile's serial on-chip pipeline takes ~55 us whatever the population, so the tile
 // kernel wins once there is at least one full wave of 128-row tiles (C5 shard: 364 vs 518 us per
 // Adam step) and the chain, which spreads every layer over all SMs, wins below that (C2: 48 vs 56 us).
 enum MlpMode { MLP_TILE, MLP_CHAIN, MLP_LAYERS };
 static MlpMode mlp_mode(const Plan& p) {
-  const char* e = std::getenv("FELIX_MLP");
-  if (e && std::string(e) == "layers") return MLP_LAYERS;
-  if (e && std::string(e) == "chain") return MLP_CHAIN;
-  if (e && std::string(e) == "tile" && p.tile_ok) return MLP_TILE;
+  const int t = g_tune.mlp.load();
+  if (t == 2) return MLP_LAYERS;
+  if (t == 1) return MLP_CHAIN;
+  if (t == 0 && p.tile_ok) return MLP_TILE;
   return (p.tile_ok && p.tile_full_wave) ? MLP_TILE : MLP_CHAIN;
 }
-static bool use_chain() {
-  const char* e = std::getenv("FELIX_MLP");
-  return !(e && std::string(e) == "layers");
-}
+static bool use_chain() { return g_tune.mlp.load() != 2; }
 
 static void launch_tile(const Plan& p, cudaStream_t st) {
-  static bool attr_set[3] = {false, false, false};
   const void* fn = p.tile_cg == 2 ? reinterpret_cast<const void*>(mlp_tile_kernel<2>)
                                   : reinterpret_cast<const void*>(mlp_tile_kernel<1>);
-  if (!attr_set[p.tile_cg]) {
-    CUDA_OK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, tile::SMEM_BYTES));
-    if (p.tile_cg == 2) CUDA_OK(cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 0));
-    attr_set[p.tile_cg] = true;
-  }
+  set_smem_attr(fn, tile::SMEM_BYTES, p.tile_cg == 2);
   cudaLaunchAttribute attrs[2];
   attrs[0] = g_pdl_attr;
   attrs[1].id = cudaLaunchAttributeClusterDimension;
@@ -184,24 +203,11 @@ static void launch_tile(const Plan& p, cudaStream_t st) {
 }
 
 static void launch_chain(const Plan& p, cudaStream_t st) {
-  static bool attr_set[2] = {false, false};
-  const int ci = p.chain_cs == 4 ? 1 : 0;
-  if (!attr_set[ci]) {
-    if (ci) CUDA_OK(cudaFuncSetAttribute(mlp_chain_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES));
-    else CUDA_OK(cudaFuncSetAttribute(mlp_chain_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, CHAIN_SMEM_BYTES));
-    attr_set[ci] = true;
-  }
+  set_smem_attr(reinterpret_cast<const void*>(mlp_chain_kernel<1>), CHAIN_SMEM_BYTES);
   cudaLaunchAttribute attrs[2];
   attrs[0] = g_pdl_attr;
-  if (ci) {
-    attrs[1].id = cudaLaunchAttributeClusterDimension;
-    attrs[1].val.clusterDim.x = static_cast<unsigned>(p.chain_cs);
-    attrs[1].val.clusterDim.y = 1;
-    attrs[1].val.clusterDim.z = 1;
-  } else {
-    attrs[1].id = cudaLaunchAttributeCooperative;   // the grid barrier needs every CTA resident
-    attrs[1].val.cooperative = 1;
-  }
+  attrs[1].id = cudaLaunchAttributeCooperative;   // the dataflow flags need every CTA resident
+  attrs[1].val.cooperative = 1;
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(static_cast<unsigned>(p.chain_grid));
   cfg.blockDim = dim3(CHAIN_THREADS);
@@ -209,8 +215,7 @@ static void launch_chain(const Plan& p, cudaStream_t st) {
   cfg.stream = st;
   cfg.attrs = attrs;
   cfg.numAttrs = 2;
-  if (ci) CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_chain_kernel<4>, p.chain));
-  else CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_chain_kernel<1>, p.chain));
+  CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_chain_kernel<1>, p.chain));
 }
 
 // The population split into K independent chunks, each with its own workspace (Plan).  One Adam
@@ -218,6 +223,7 @@ static void launch_chain(const Plan& p, cudaStream_t st) {
 // chunk's tensor-core GEMMs overlap another chunk's latency-bound expression kernels.
 struct Chunks {
   const CostModel* cm = nullptr;
+  uint64_t cm_uid = 0;
   int64_t n = -1;
   int K = 0;
   std::vector<int64_t> off, cnt;
@@ -243,8 +249,9 @@ struct ProfEvent { int cls; cudaEvent_t a, b; };
 // felix_search_group workspace: one MLP plan over the rows of every member space; per member its Adam
 // state and step counter; a one-step graph (fork: DAG forwards, join: MLP, fork: reverse/Adam, join)
 struct GroupCache {
-  const CostModel* cm = nullptr;
-  std::vector<void*> spaces;
+  uint64_t cm_uid = 0;
+  std::vector<uint64_t> space_uid;   // member identities (uid + statement count), never raw addresses
+  std::vector<int> space_ns;
   std::vector<int64_t> n, row_off;
   std::unique_ptr<Plan> plan;
   std::vector<std::unique_ptr<DevBuf>> m, v, step_ctr;
@@ -261,6 +268,7 @@ struct GroupCache {
 }  // namespace felix
 
 struct felix_space {
+  uint64_t uid = felix::next_uid();   // identity for workspace caches (see GroupCache)
   int device = 0;
   felix::SpaceDesc desc;
   felix::RoundTables rt;
@@ -279,7 +287,7 @@ struct felix_space {
   std::map<int, Module> modules;
   double nvrtc_ms = 0;
   int regs_fwd = 0, regs_rev = 0;
-  int64_t flops_fwd = 0;
+  int64_t flops_fwd = 0, flops_rev = 0;
   // workspace caches (search: chunked; eval: one chunk) + scratch
   std::unique_ptr<felix::Chunks> search_chunks, eval_chunks;
   std::unique_ptr<felix::GroupCache> group_cache;   // felix_search_group with this space first
@@ -450,15 +458,17 @@ static felix_space::Module& get_module(felix_space* s, int P, int R = 1) {
   // the forward kernel stages NREP x NS x 32 x (K0P+1) floats + NREP x NV x 32 doubles statically
   if (R > 1 && static_cast<int64_t>(R) * (s->desc.n_statements * 32 * (s->K0p + 1) * 4 + s->desc.n_vars * 32 * (8 + 4) + 64) > 48 * 1024)
     R = 1;
-  const int key = P + 64 * R;
+  const bool trace = g_tune.trace.load() != 0;
+  const int key = P + 64 * R + (trace ? 4096 : 0);
   auto it = s->modules.find(key);
   if (it != s->modules.end()) return it->second;
   felix_space::Module mod;
   mod.P = P;
   mod.R = R;
   CodegenInfo info;
-  mod.source = generate_dag_module(s->desc, s->K0p, P, R, &info);
+  mod.source = generate_dag_module(s->desc, s->K0p, P, R, trace, &info);
   s->flops_fwd = info.flops_fwd;
+  s->flops_rev = info.flops_rev;
   mod.rev_smem = info.rev_smem_bytes;
   auto t0 = std::chrono::steady_clock::now();
   std::vector<char> cubin = nvrtc_compile(mod.source);
@@ -484,45 +494,22 @@ static felix_space::Module& get_module(felix_space* s, int P, int R = 1) {
   return s->modules.emplace(key, std::move(mod)).first->second;
 }
 
-// Replicas of the cone groups per block: warps running the same cone's straight-line code share the
-// SM's instruction fetches (ncu: 42 % of the reverse kernel's stall samples are no_instructions; its
-// SASS is 124 KB at C2).  Measured at C2: R=2 takes the reverse kernel from 16.9 to 15.3 us but the step
-// only +0.6 %; R=4 exceeds the static shared budget.  Default 1; FELIX_R overrides.
-// 0 = cone-per-CTA kernels (FELIX_CPB=1: clusters of P CTAs, DSMEM exchange), else replicas of the cone
-// groups per block (FELIX_R=1|2|4).  Cone-per-CTA is parity-green but measured slower at C2 (forward
-// 11.1 -> 12.8 us at P = 4, 26.9 us at P = 8; reverse 17.4 -> 16.8 / 20.9 us): the DSMEM round trips and
-// cluster barriers cost more than the shared instruction fetches save (a timing-only variant without the
-// exchange gave 8.6 / 12.8 us at P = 8), and 8-CTA clusters of one-CTA-per-SM kernels do not fit one wave.
-static bool use_cpb() {
-  const char* e = std::getenv("FELIX_CPB");
-  return e && std::atoi(e) == 1;
-}
+// Replicas of the cone groups per block (cone-group kernels): warps running the same cone's straight-line
+// code share the SM's instruction fetches.  Measured at C2: R=2 takes the reverse kernel from 16.9 to
+// 15.3 us but the step only +0.6 %; R=4 exceeds the static shared budget.  Default 1; felix_tune overrides.
 static int choose_R(int64_t n, int P) {
-  (void)n;
-  if (P > 1 && use_cpb()) return 0;
-  if (const char* e = std::getenv("FELIX_R")) {
-    const int r = std::atoi(e);
-    if (r == 1 || r == 2 || r == 4) return r;
-  }
-  return 1;
+  (void)n; (void)P;
+  const int r = g_tune.R.load();
+  return (r == 1 || r == 2 || r == 4) ? r : 1;
 }
 
 // Cone-partition width: enough warps to give every SM ~8 resident warps of expression work.
 static int choose_P(int64_t n) {
-  if (const char* e = std::getenv("FELIX_P")) {   // experiments: force the cone-partition width
-    const int p = std::atoi(e);
-    if (p == 1 || p == 2 || p == 4 || p == 8 || p == 16) return p;
-  }
+  const int p = g_tune.P.load();
+  if (p == 1 || p == 2 || p == 4 || p == 8 || p == 16) return p;
   // measured on B200 (C2 space, per-class event timing): P=4 best at 4096 candidates, P=2 at 32768,
   // P=1 once the population alone fills the SMs
   int P = 1;
-  if (use_cpb()) {
-    // cone-per-CTA kernels (measured at C2, timing experiment with every warp of a CTA on one cone:
-    // forward 11.1 -> 8.6 us, reverse 17.5 -> 12.8 us at P = 8)
-    if (n <= 16384) P = 8;
-    else if (n <= 65536) P = 4;
-    return P;
-  }
   if (n <= 8192) P = 4;
   else if (n <= 65536) P = 2;
   return P;
@@ -541,24 +528,6 @@ static void launch_cfg(const void* f, dim3 grid, dim3 block, size_t smem, void**
 }
 static void launch_grouped(cudaKernel_t f, int P, int R, int64_t n, size_t smem, void** args, cudaStream_t st, bool pdl) {
   if (n <= 0) return;
-  if (R == 0) {
-    // cone-per-CTA kernels: clusters of P CTAs x P warps, one cluster per P x 32 candidates
-    cudaLaunchAttribute attrs[2];
-    attrs[0].id = cudaLaunchAttributeClusterDimension;
-    attrs[0].val.clusterDim.x = static_cast<unsigned>(P);
-    attrs[0].val.clusterDim.y = 1;
-    attrs[0].val.clusterDim.z = 1;
-    attrs[1] = g_pdl_attr;
-    cudaLaunchConfig_t cfg{};
-    cfg.gridDim = dim3(static_cast<unsigned>((n + 32 * P - 1) / (32 * P) * P));
-    cfg.blockDim = dim3(32 * P);
-    cfg.dynamicSmemBytes = smem;
-    cfg.stream = st;
-    cfg.attrs = attrs;
-    cfg.numAttrs = pdl ? 2 : 1;
-    CUDA_OK(cudaLaunchKernelExC(&cfg, reinterpret_cast<const void*>(f), args));
-    return;
-  }
   launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((n + 32 * R - 1) / (32 * R))), dim3(32 * P * R),
              smem, args, st, pdl);
 }
@@ -574,15 +543,12 @@ static void launch_flat(cudaKernel_t f, int64_t n, void** args, cudaStream_t st)
 
 // Split-cone reverse kernel (codegen.cpp felix_rev_sc): one cone per CTA for W x 32 candidates, partial
 // adjoints through global memory; the next step's forward (felix_fwd_adam) sums them and applies Adam,
-// felix_adam_sc after the last step.  Default for single-space searches; FELIX_SC=0 selects
-// felix_rev_adam, FELIX_SC=1 forces it in group searches too (measured there with an earlier variant:
+// felix_adam_sc after the last step.  Default for single-space searches; felix_tune("split_cone", 0)
+// selects felix_rev_adam, 1 forces it in group searches too (measured there with an earlier variant:
 // C3 1.66e8 -> 1.65e8, C4 2.25e8 -> 2.08e8 cand-steps/s, so groups keep felix_rev_adam by default).
 // Not with history rounding (it rounds the caller's y before each step's forward, i.e. before Adam).
-static bool use_cpb();
 static bool use_sc(bool group = false) {
-  if (use_cpb()) return false;
-  const char* e = std::getenv("FELIX_SC");
-  const int v = e ? std::atoi(e) : -1;
+  const int v = g_tune.sc.load();
   if (v == 0) return false;
   if (v == 1) return true;
   return !group;
@@ -590,37 +556,24 @@ static bool use_sc(bool group = false) {
 __global__ void set_int_kernel(int* p, int v) { *p = v; }
 // Split-cone searches: at least two cones (measured at the C5 shard, 131072 candidates: 2.53e8 at P = 1,
 // 2.72e8 at P = 2 cand-steps/s) and two replicas of the cone groups per felix_fwd_adam block (warps on the
-// same cone share instruction fetches; C2 forward 14.8 -> 12.8 us).  FELIX_P / FELIX_R override.
-static int choose_P_sc(int P) { return (P == 1 && !std::getenv("FELIX_P")) ? 2 : P; }
+// same cone share instruction fetches; C2 forward 14.8 -> 12.8 us).  felix_tune overrides.
+static int choose_P_sc(int P) { return (P == 1 && g_tune.P.load() < 0) ? 2 : P; }
 static int choose_R_sc() {
-  if (const char* e = std::getenv("FELIX_R")) {
-    const int r = std::atoi(e);
-    if (r == 1 || r == 2 || r == 4) return r;
-  }
-  return 2;
+  const int r = g_tune.R.load();
+  return (r == 1 || r == 2 || r == 4) ? r : 2;
 }
-// warps per split-cone CTA: about one CTA per SM (FELIX_SCW overrides)
+// warps per split-cone CTA: about one CTA per SM (felix_tune("sc_warps") overrides)
 static int choose_scw(int64_t n, int P) {
-  if (const char* e = std::getenv("FELIX_SCW")) {
-    const int w = std::atoi(e);
-    if (w >= 1 && w <= 8) return w;
-  }
+  const int w0 = g_tune.scw.load();
+  if (w0 >= 1 && w0 <= 8) return w0;
   const int64_t groups = (n + 31) / 32;
   int64_t w = (groups * P + 147) / 148;
   return static_cast<int>(std::max<int64_t>(1, std::min<int64_t>(8, w)));
 }
-// groups of W x 32 candidates each split-cone CTA runs one after the other (FELIX_SCG overrides)
-static int choose_scg() {
-  if (const char* e = std::getenv("FELIX_SCG")) {
-    const int g = std::atoi(e);
-    if (g >= 1 && g <= 16) return g;
-  }
-  return 1;
-}
 static int64_t sc_groups(int64_t n, int W) { return ((n + 31) / 32 + W - 1) / W; }
-static void launch_sc(cudaKernel_t f, int P, int W, int G, int64_t n, void** args, cudaStream_t st, bool pdl) {
+static void launch_sc(cudaKernel_t f, int P, int W, int64_t n, void** args, cudaStream_t st, bool pdl) {
   if (n <= 0) return;
-  launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>((sc_groups(n, W) + G - 1) / G * P)), dim3(32 * W),
+  launch_cfg(reinterpret_cast<const void*>(f), dim3(static_cast<unsigned>(sc_groups(n, W) * P)), dim3(32 * W),
              0, args, st, pdl);
 }
 
@@ -753,7 +706,6 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
       // one N tile only mt CTAs work; 32-wide N tiles spread it over 3x the CTAs while they fit in one wave
       bn = g.bn;                                                          // K0p (<= 128 required)
       if (N % 32 == 0 && mt * (N / 32) <= sms) bn = 32;
-      if (const char* e = std::getenv("FELIX_DPHI_BN")) { const int v = std::atoi(e); if (v > 0 && N % v == 0 && v % 16 == 0) bn = v; }
     }
     else bn = (N % 128 == 0 && mt * (N / 128) >= sms * 2 / 3) ? 128 : 64;
     if (bn > CHAIN_BN_MAX) FELIX_THROW(FELIX_E_UNSUPPORTED, "chain tile N > 128");
@@ -768,7 +720,7 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     // folded into its weights (exact A: two MMA passes, no A lo loads); FELIX_MASK_EXACT=0 disables
     L.a_exact = 0;
     L.head_exact = 0;
-    if (i == static_cast<size_t>(cm->n_layers - 1) && i > 0 && mask_exact() && p->gemms[i - 1].epi == EPI_HEAD) {
+    if (i == static_cast<size_t>(cm->n_layers - 1) && i > 0 && p->gemms[i - 1].epi == EPI_HEAD) {
       L.a_exact = 1;
       p->chain.layer[i - 1].head_exact = 1;
       L.b_hi = make_tmap(cm->WTs_hi.p, N, g.args.K, bn);
@@ -778,26 +730,17 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     max_tiles = std::max(max_tiles, L.n_tiles);
   }
   p->chain_grid = std::min(sms, max_tiles);
-  // Grid chain with per-row-block dataflow flags (cooperative launch: every CTA resident) by default: at C2
-  // 44.2 us per Adam step vs 45.7 us for the cluster chain (one 4-CTA cluster per row block, cluster
-  // barriers), and faster above 37 row blocks (n=8192: 56 vs 90 us).  FELIX_CHAIN_CS=4 selects the
-  // cluster chain.
-  p->chain_cs = 1;
-  if (const char* e = std::getenv("FELIX_CHAIN_CS")) p->chain_cs = std::atoi(e) == 4 ? 4 : 1;
-  if (p->chain_cs == 4) p->chain_grid = static_cast<int>(std::min<int64_t>(sms / 4, mt)) * 4;
-  // grid chain: per-row-block dataflow flags instead of grid barriers between layers (FELIX_CHAIN_FLAGS=0:
-  // grid barriers).  The epoch is the step counter the forward DAG kernel bumps before every chain launch.
+  // Grid chain with per-row-block dataflow flags (cooperative launch: every CTA resident): at C2 44.2 us
+  // per Adam step vs 45.7 us for a cluster chain (one 4-CTA cluster per row block, cluster barriers; removed)
+  // and faster above 37 row blocks (n=8192: 56 vs 90 us).  The epoch is the step counter the forward DAG
+  // kernel bumps before every chain launch.
   p->chain_flags.alloc(static_cast<size_t>(p->chain.n_layers) * mt * CHAIN_FLAG_STRIDE * 4);
   CUDA_OK(cudaMemset(p->chain_flags.p, 0, p->chain_flags.bytes));
   {
-    const char* e = std::getenv("FELIX_CHAIN_FLAGS");
-    const bool flags = !(e && std::atoi(e) == 0);
-    p->chain.flags = (p->chain_cs == 1 && flags) ? p->chain_flags.as<unsigned int>() : nullptr;
+    p->chain.flags = p->chain_flags.as<unsigned int>();
     p->chain.epoch = p->step_ctr.as<int>();
-    // own-chunk reuse (mlp_chain.cuh ChainLayer::reuse) where every CTA keeps its row block between two
-    // layers; FELIX_CHAIN_REUSE=0 disables
-    const char* er = std::getenv("FELIX_CHAIN_REUSE");
-    const bool reuse_ok = p->chain.flags != nullptr && CHAIN_EPI_BUFS == 2 && !(er && std::atoi(er) == 0);
+    // own-chunk reuse (mlp_chain.cuh ChainLayer::reuse) where every CTA keeps its row block between two layers
+    const bool reuse_ok = CHAIN_EPI_BUFS == 2;
     for (int i = 0; i < p->chain.n_layers; ++i) {
       ChainLayer& Li = p->chain.layer[i];
       Li.reuse = 0;
@@ -811,7 +754,7 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
   // tile-local fused MLP: TenSet widths [K0p, 512, 256, 256, 1] only
   p->tile_ok = L == 4 && d[1] == tile::D1 && d[2] == tile::D2 && d[3] == tile::D3 && K0p <= 128 && K0p % 32 == 0;   // K0p/2 rows: multiple of 16
   if (p->tile_ok) {
-    if (const char* e = std::getenv("FELIX_TILE_CG")) p->tile_cg = std::atoi(e) == 2 ? 2 : 1;
+    p->tile_cg = g_tune.tile_cg.load() == 2 ? 2 : 1;
     p->tile_full_wave = mt >= sms;
     const int cg = p->tile_cg;
     TileParams& t = p->tile;
@@ -824,7 +767,7 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     t.w3_hi = make_tmap(cm->W_hi[2]->p, d[3], d[2], 128);
     t.w3_lo = make_tmap(cm->W_lo[2]->p, d[3], d[2], 128);
     // B1 on the exact mask with the head row folded into W3^T (as the chain's first backward layer)
-    t.d2_exact = mask_exact() ? 1 : 0;
+    t.d2_exact = 1;
     t.w3t_hi = make_tmap(t.d2_exact ? cm->WTs_hi.p : cm->WT_hi[2]->p, d[2], d[3], 128);
     t.w3t_lo = make_tmap(t.d2_exact ? cm->WTs_lo.p : cm->WT_lo[2]->p, d[2], d[3], 128);
     t.w2t_hi = make_tmap(cm->WT_hi[1]->p, d[1], d[2], 128 / cg);
@@ -861,19 +804,18 @@ static std::unique_ptr<Plan> build_plan(felix_space* s, const CostModel* cm, int
 
 // number of concurrent chunks for a population of n (FELIX_CHUNKS overrides; tuned on B200)
 static int choose_chunks(int64_t n) {
-  if (const char* e = std::getenv("FELIX_CHUNKS")) {
-    const int k = std::atoi(e);
-    if (k >= 1 && k <= 16) return k;
-  }
+  const int k = g_tune.chunks.load();
+  if (k >= 1 && k <= 16) return k;
   (void)n;   // measured on B200 (C2): 2/4/8 concurrent chunks were 3-14% slower than 1
   return 1;
 }
 
 static Chunks& get_chunks(felix_space* s, std::unique_ptr<Chunks>& slot, const CostModel* cm, int64_t n, int K) {
-  if (slot && slot->cm == cm && slot->n == n && slot->K == K) return *slot;
+  if (slot && slot->cm_uid == cm->uid && slot->n == n && slot->K == K) return *slot;
   slot.reset();
   auto c = std::make_unique<Chunks>();
   c->cm = cm;
+  c->cm_uid = cm->uid;
   c->n = n;
   const int64_t per = ((n + K - 1) / K + 127) / 128 * 128;
   for (int64_t o = 0; o < n; o += per) {
@@ -1067,10 +1009,9 @@ felix_status felix_codegen(const felix_var* vars, int32_t n_vars, const felix_sp
   const int K0 = n_features / n_statements;
   s->K0p = K0 <= 64 ? 64 : K0 <= 96 ? 96 : 128;
   CodegenInfo info;
-  // FELIX_CODEGEN_P / FELIX_CODEGEN_R select the variant to inspect (default: P = 8 cone-per-CTA kernels)
-  const char* ep = std::getenv("FELIX_CODEGEN_P");
-  const char* er = std::getenv("FELIX_CODEGEN_R");
-  const std::string code = generate_dag_module(s->desc, s->K0p, ep ? std::atoi(ep) : 8, er ? std::atoi(er) : 0, &info);
+  // felix_tune("codegen_cone_width" / "codegen_replicas") select the variant to inspect (default P = 4, R = 2)
+  const int cp = g_tune.codegen_P.load(), cr = g_tune.codegen_R.load();
+  const std::string code = generate_dag_module(s->desc, s->K0p, cp > 0 ? cp : 4, cr > 0 ? cr : 2, g_tune.trace.load() != 0, &info);
   if (src_len) *src_len = static_cast<int64_t>(code.size());
   if (src && src_cap > 0) {
     const size_t nb = std::min<size_t>(code.size() + 1, static_cast<size_t>(src_cap));
@@ -1105,6 +1046,8 @@ felix_status felix_space_set_statements(felix_space* s, int32_t n_statements) {
   s->modules.clear();
   s->search_chunks.reset();
   s->eval_chunks.reset();
+  s->group_cache.reset();
+  s->uid = next_uid();   // group caches on other spaces that list this one become stale
   FELIX_API_END
 }
 
@@ -1122,6 +1065,7 @@ felix_status felix_space_info(const felix_space* s, felix_space_info_t* out) {
   out->regs_fwd = s->regs_fwd;
   out->regs_rev = s->regs_rev;
   out->dag_flops_fwd = s->flops_fwd;
+  out->dag_flops_rev = s->flops_rev;
   FELIX_API_END
 }
 
@@ -1148,6 +1092,7 @@ felix_status felix_costmodel_load(int device, int32_t n_layers, const int32_t* d
   check_device(device);
   DeviceGuard dg(device);
   auto m = std::make_unique<felix_costmodel>();
+  m->uid = next_uid();
   m->device = device;
   m->n_layers = n_layers;
   m->dims.assign(dims, dims + n_layers + 1);
@@ -1226,8 +1171,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
   const bool sc = use_sc() && !p->history;
   const int P0 = choose_P(ch.cnt[0]);
   const felix_space::Module& mod = sc ? get_module(s, choose_P_sc(P0), choose_R_sc()) : get_module(s, P0, choose_R(ch.cnt[0], P0));
-  const int scg = choose_scg();
-  const int scw = choose_scw((ch.cnt[0] + scg - 1) / scg, mod.P);
+  const int scw = choose_scw(ch.cnt[0], mod.P);
   if (!p->init_from_y) {
     unsigned long long seed = p->rng_seed;
     long long ib = p->index_base;
@@ -1249,7 +1193,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     CUDA_OK(cudaMemsetAsync(pl->chain_flags.p, 0, pl->chain_flags.bytes, st));
     if (sc) {
       const int64_t cnt = pl->n / s->desc.n_statements;
-      ensure(pl->sc_part, static_cast<size_t>(mod.P) * s->desc.n_vars * cnt * 8);
+      ensure(pl->sc_part, static_cast<size_t>(mod.P) * s->desc.n_vars * cnt * 4);
       ensure(pl->sc_pen, static_cast<size_t>(mod.P) * cnt * 8);
       set_int_kernel<<<1, 1, 0, st>>>(pl->step_ctr.as<int>(), 1);   // the reverse kernel counts from 1
       CUDA_OK(cudaGetLastError());
@@ -1315,10 +1259,9 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
       prof_mark(s, 0, cs, false);
       s->prof_launches[0] += 1;
       run_mlp(s, pl, cs);
-      int scg_ = scg;
-      void* ra[] = {&yk, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr, &scg_};
+      void* ra[] = {&yk, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr};
       prof_mark(s, 2, cs, true);
-      launch_sc(mod.f_rev_sc, mod.P, scw, scg, cnt, ra, cs, true);
+      launch_sc(mod.f_rev_sc, mod.P, scw, cnt, ra, cs, true);
       prof_mark(s, 2, cs, false);
       s->prof_launches[2] += 1;
       return;
@@ -1346,7 +1289,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     // (a per-step fork/join would re-synchronise them every step).  Joined once at the end.
     auto ptr = [](const void* q) { return static_cast<double>(reinterpret_cast<uintptr_t>(q)); };
     const std::vector<double> key = {static_cast<double>(mod.P), ptr(y), ptr(final_loss), lam0, lr0, b10, b20, eps0,
-                                     static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R), static_cast<double>(scg),
+                                     static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R),
                                      ptr(ch.plans[0]->sc_part.p), ptr(ch.plans[0]->sc_pen.p)};
     while (static_cast<int>(ch.streams.size()) < nck) {
       cudaStream_t b;
@@ -1401,7 +1344,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
                                      static_cast<double>(s->h_valid), ptr(s->h_sched.p), ptr(s->h_last.p),
                                      ptr(s->h_slot_h.p), ptr(s->h_pool_sched.p), ptr(s->h_pool_key.p),
                                      static_cast<double>(s->h_mask), static_cast<double>(s->h_cap),
-                                     static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R), static_cast<double>(scg),
+                                     static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R),
                                      ptr(ch.plans[0]->sc_part.p), ptr(ch.plans[0]->sc_pen.p)};
     if (!ch.graph || ch.graph_key != key) {
       if (ch.graph) { cudaGraphExecDestroy(ch.graph); ch.graph = nullptr; }
@@ -1468,7 +1411,8 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
       void* ctr = pl.step_ctr.p;
       float* lo = final_loss ? final_loss + o : nullptr;
       float hbv = hb, lam = lam0, lr = lr0, b1 = b10, b2 = b20, eps = eps0;
-      void* aa[] = {&yk, &ni, &ldy, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hbv, &lam, &lr, &b1, &b2, &eps, &ctr, &lo};
+      void* og = nullptr;
+      void* aa[] = {&yk, &ni, &ldy, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hbv, &lam, &lr, &b1, &b2, &eps, &ctr, &lo, &og};
       prof_mark(s, 2, st, true);
       launch_flat(mod.f_adam_sc, cnt, aa, st);
       prof_mark(s, 2, st, false);
@@ -1502,16 +1446,18 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
   const int T = params[0].n_steps;
   // ---- workspace (cached on spaces[0])
   std::unique_ptr<GroupCache>& slot = s0->group_cache;
-  bool fresh = !slot || slot->cm != m || static_cast<int>(slot->spaces.size()) != G;
+  bool fresh = !slot || slot->cm_uid != m->uid || static_cast<int>(slot->space_uid.size()) != G;
   for (int i = 0; !fresh && i < G; ++i)
-    fresh = slot->spaces[i] != spaces[i] || slot->n[i] != params[i].n_seeds;
+    fresh = slot->space_uid[i] != spaces[i]->uid || slot->space_ns[i] != spaces[i]->desc.n_statements ||
+            slot->n[i] != params[i].n_seeds;
   if (fresh) {
     slot.reset();
     auto gc = std::make_unique<GroupCache>();
-    gc->cm = m;
+    gc->cm_uid = m->uid;
     int64_t off = 0;
     for (int i = 0; i < G; ++i) {
-      gc->spaces.push_back(spaces[i]);
+      gc->space_uid.push_back(spaces[i]->uid);
+      gc->space_ns.push_back(spaces[i]->desc.n_statements);
       gc->n.push_back(params[i].n_seeds);
       gc->row_off.push_back(off);
       off += params[i].n_seeds * spaces[i]->desc.n_statements;
@@ -1543,7 +1489,7 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
     mods[i] = sc ? &get_module(spaces[i], choose_P_sc(choose_P(n)), choose_R_sc()) : &get_module(spaces[i], choose_P(n), choose_R(n, choose_P(n)));
     scws[i] = choose_scw(n, mods[i]->P);
     if (sc) {
-      ensure(*gc.sc_part[i], static_cast<size_t>(mods[i]->P) * spaces[i]->desc.n_vars * n * 8);
+      ensure(*gc.sc_part[i], static_cast<size_t>(mods[i]->P) * spaces[i]->desc.n_vars * n * 4);
       ensure(*gc.sc_pen[i], static_cast<size_t>(mods[i]->P) * n * 8);
     }
     if (!params[i].init_from_y) {
@@ -1629,9 +1575,8 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
       if (sc) {
         void* part = gc.sc_part[i]->p;
         void* pen = gc.sc_pen[i]->p;
-        int scg = 1;
-        void* ra[] = {&yi, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr, &scg};
-        launch_sc(mods[i]->f_rev_sc, mods[i]->P, scws[i], 1, p.n_seeds, ra, si, false);
+        void* ra[] = {&yi, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr};
+        launch_sc(mods[i]->f_rev_sc, mods[i]->P, scws[i], p.n_seeds, ra, si, false);
         continue;
       }
       void* args[] = {&yi, &ni, &ldy, &dphi, &ld, &cpart, &nht, &ld, &hbv, &lam, &mv, &vv, &ctr, &lr, &b1, &b2, &eps, &lo};
@@ -1657,7 +1602,8 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
       void* ctr = gc.step_ctr[i]->p;
       float* lo = final_loss ? final_loss[i] : nullptr;
       float hbv = m->head_b, lam = p.lambda, lr = p.lr, b1 = p.beta1, b2 = p.beta2, eps = p.eps;
-      void* aa[] = {&ya, &ni, &ldy, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hbv, &lam, &lr, &b1, &b2, &eps, &ctr, &lo};
+      void* og = nullptr;
+      void* aa[] = {&ya, &ni, &ldy, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hbv, &lam, &lr, &b1, &b2, &eps, &ctr, &lo, &og};
       launch_flat(mods[i]->f_adam_sc, p.n_seeds, aa, st);
     }
   };
@@ -1707,29 +1653,79 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
   FELIX_API_END
 }
 
-felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int64_t n, float lambda, float* phi,
-                        float* g, float* cost, float* loss, float* grad, void* stream) {
-  FELIX_API_BEGIN
-  check_pair(s, m);
-  if (!y && n > 0) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL y");
-  if (n < 0 || n > (int64_t(1) << 30)) FELIX_THROW(FELIX_E_INVALID_ARG, "n out of range");
-  if (n == 0) return FELIX_OK;
-  DeviceGuard dg(s->device);
-  cudaStream_t st = static_cast<cudaStream_t>(stream);
+// felix_eval / felix_eval_ex.  Default: one objective + gradient evaluation with the eval kernels
+// (felix_fwd -> MLP -> felix_rev_eval).  search_path: the kernels and launch configuration of one
+// felix_search Adam step (felix_fwd_adam at step 1, i.e. no update -> the MLP of the search plan ->
+// felix_rev_sc partial adjoints -> felix_adam_sc summing them as the Adam prologue does), writing
+// the loss and dL/dy instead of updating y.
+static void eval_impl(felix_space* s, felix_costmodel* m, const float* y, int64_t n, float lambda, const felix_eval_out& o,
+                      cudaStream_t st) {
   Plan& pl = *get_chunks(s, s->eval_chunks, m, n, 1).plans[0];
   CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
   CUDA_OK(cudaMemsetAsync(pl.chain_flags.p, 0, pl.chain_flags.bytes, st));
   CUDA_OK(cudaMemsetAsync(pl.step_ctr.p, 0, 4, st));     // the forward kernel makes it 1: the chain's epoch
-  const felix_space::Module& mod = get_module(s, choose_P(n), choose_R(n, choose_P(n)));
-  run_forward_mlp(s, pl, mod, y, n, n, st, pl.step_ctr.as<int>());
   int ni = static_cast<int>(n);
   void* dphi = pl.dphi.p;
   void* cpart = pl.c_part.p;
   int ld = static_cast<int>(pl.n_pad);
   int nht = pl.n_head_tiles;
   float hb = m->head_b, lam = lambda;
-  void* args[] = {&y, &ni, &ni, &dphi, &ld, &cpart, &nht, &ld, &hb, &lam, &phi, &g, &cost, &loss, &grad};
+  if (o.search_path) {
+    const felix_space::Module& mod = get_module(s, choose_P_sc(choose_P(n)), choose_R_sc());
+    const int scw = choose_scw(n, mod.P);
+    ensure(pl.sc_part, static_cast<size_t>(mod.P) * s->desc.n_vars * n * 4);
+    ensure(pl.sc_pen, static_cast<size_t>(mod.P) * n * 8);
+    CUDA_OK(cudaMemsetAsync(pl.m.p, 0, pl.m.bytes, st));
+    CUDA_OK(cudaMemsetAsync(pl.v.p, 0, pl.v.bytes, st));
+    set_int_kernel<<<1, 1, 0, st>>>(pl.step_ctr.as<int>(), 1);
+    CUDA_OK(cudaGetLastError());
+    float* yk = const_cast<float*>(y);   // step counter 1: felix_fwd_adam applies no update, y is not written
+    int* ctr = pl.step_ctr.as<int>();
+    void* phh = pl.phi_hi.p;
+    void* phl = pl.phi_lo.p;
+    void* part = pl.sc_part.p;
+    void* pen = pl.sc_pen.p;
+    void* mv = pl.m.p;
+    void* vv = pl.v.p;
+    float lr = 0.f, b1 = 0.9f, b2 = 0.999f, eps = 1e-8f;
+    void* fa[] = {&yk, &ni, &ni, &phh, &phl, &ctr, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hb, &lam, &lr, &b1, &b2, &eps};
+    launch_grouped(mod.f_fwd_adam, mod.P, mod.R, n, 0, fa, st, true);
+    run_mlp(s, pl, st);
+    void* ra[] = {&yk, &ni, &ni, &dphi, &ld, &lam, &part, &pen, &ctr};
+    launch_sc(mod.f_rev_sc, mod.P, scw, n, ra, st, true);
+    float* lo = o.loss;
+    float* og = o.grad;
+    void* aa[] = {&yk, &ni, &ni, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hb, &lam, &lr, &b1, &b2, &eps, &ctr, &lo, &og};
+    launch_flat(mod.f_adam_sc, n, aa, st);
+    return;
+  }
+  const felix_space::Module& mod = get_module(s, choose_P(n), choose_R(n, choose_P(n)));
+  run_forward_mlp(s, pl, mod, y, n, n, st, pl.step_ctr.as<int>());
+  float *phi = o.phi, *g = o.g, *cost = o.cost, *loss = o.loss, *grad = o.grad;
+  double* F = o.F;
+  void* args[] = {&y, &ni, &ni, &dphi, &ld, &cpart, &nht, &ld, &hb, &lam, &phi, &g, &cost, &loss, &grad, &F};
   launch_grouped(mod.f_rev_eval, mod.P, mod.R, n, mod.rev_smem, args, st, false);
+}
+
+felix_status felix_eval(felix_space* s, felix_costmodel* m, const float* y, int64_t n, float lambda, float* phi,
+                        float* g, float* cost, float* loss, float* grad, void* stream) {
+  felix_eval_out o{};
+  o.phi = phi; o.g = g; o.cost = cost; o.loss = loss; o.grad = grad;
+  return felix_eval_ex(s, m, y, n, lambda, &o, stream);
+}
+
+felix_status felix_eval_ex(felix_space* s, felix_costmodel* m, const float* y, int64_t n, float lambda,
+                           const felix_eval_out* out, void* stream) {
+  FELIX_API_BEGIN
+  check_pair(s, m);
+  if (!out) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL out");
+  if (!y && n > 0) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL y");
+  if (n < 0 || n > (int64_t(1) << 30)) FELIX_THROW(FELIX_E_INVALID_ARG, "n out of range");
+  if (out->search_path && (out->phi || out->g || out->cost || out->F))
+    FELIX_THROW(FELIX_E_INVALID_ARG, "search_path evaluates loss and grad only");
+  if (n == 0) return FELIX_OK;
+  DeviceGuard dg(s->device);
+  eval_impl(s, m, y, n, lambda, *out, static_cast<cudaStream_t>(stream));
   FELIX_API_END
 }
 
@@ -1786,11 +1782,6 @@ static void do_hard(felix_space* s, const int32_t* sched, int64_t n, double* phi
   launch_flat(get_module(s, 1).f_hard, n, args, st);
 }
 
-// FELIX_SCORE=1 selects the previous 64 x 64 scoring kernels (same results)
-static bool score_v2() {
-  const char* e = std::getenv("FELIX_SCORE");
-  return !(e && std::atoi(e) == 1);
-}
 
 static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, int64_t n, double* score, cudaStream_t st) {
   // TenSet segment sum over statements: score = sum_s MLP(phi_s), phi64 = [S * K0][n] statement-major
@@ -1807,17 +1798,12 @@ static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, in
       const int K = m->dims[l], N = m->dims[l + 1];
       const bool last = l == L - 1;
       double* out = last ? score : bufs[l & 1];
-      if (N >= 32 && score_v2()) {   // register-blocked 128 x 64 tiles (bit-identical arithmetic)
+      if (N >= 32) {   // register-blocked 128 x 64 tiles
         const dim3 grid(static_cast<unsigned>((N + SC2_TN - 1) / SC2_TN), static_cast<unsigned>((n + SC2_TM - 1) / SC2_TM));
         score_layer_v2_kernel<<<grid, 256, 0, st>>>(
             in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
             last ? 0 : 1, last && st_i > 0 ? 1 : 0);
-      } else if (N >= 32) {   // register-blocked 64 x 64 tiles (bit-identical arithmetic)
-        const dim3 grid(static_cast<unsigned>((N + SCORE_T - 1) / SCORE_T), static_cast<unsigned>((n + SCORE_T - 1) / SCORE_T));
-        score_layer_rb_kernel<<<grid, 256, 0, st>>>(
-            in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
-            last ? 0 : 1, last && st_i > 0 ? 1 : 0);
-      } else if (N == 1 && last && rs == K && cs == 1 && score_v2()) {
+      } else if (N == 1 && last && rs == K && cs == 1) {
         score_head_kernel<<<static_cast<unsigned>((n + 31) / 32), 32, 0, st>>>(
             in, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, st_i > 0 ? 1 : 0);
       } else {
@@ -1991,7 +1977,29 @@ felix_status felix_debug_trace(felix_space* s, uint64_t* out, int64_t n_words) {
     CUDA_OK(cudaMemcpy(out, ptr, std::min<size_t>(bytes, static_cast<size_t>(n_words) * 8), cudaMemcpyDeviceToHost));
     return FELIX_OK;
   }
-  FELIX_THROW(FELIX_E_UNSUPPORTED, "no trace buffer (set FELIX_TRACE before felix_space_create)");
+  FELIX_THROW(FELIX_E_UNSUPPORTED, "no trace buffer (felix_tune(\"trace\", 1) before the kernels are generated)");
+  FELIX_API_END
+}
+
+felix_status felix_tune(const char* key, int32_t value) {
+  FELIX_API_BEGIN
+  if (!key) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL key");
+  const std::string k(key);
+  auto in = [&](std::initializer_list<int> ok) {
+    for (int v : ok) if (v == value) return;
+    FELIX_THROW(FELIX_E_INVALID_ARG, "felix_tune: bad value " + std::to_string(value) + " for " + k);
+  };
+  if (k == "mlp") { in({-1, 0, 1, 2}); g_tune.mlp = value; }
+  else if (k == "cone_width") { in({-1, 1, 2, 4, 8, 16}); g_tune.P = value; }
+  else if (k == "replicas") { in({-1, 1, 2, 4}); g_tune.R = value; }
+  else if (k == "sc_warps") { in({-1, 1, 2, 3, 4, 5, 6, 7, 8}); g_tune.scw = value; }
+  else if (k == "chunks") { if (value != -1 && (value < 1 || value > 16)) in({}); g_tune.chunks = value; }
+  else if (k == "split_cone") { in({-1, 0, 1}); g_tune.sc = value; }
+  else if (k == "tile_cta_group") { in({-1, 1, 2}); g_tune.tile_cg = value; }
+  else if (k == "codegen_cone_width") { in({-1, 1, 2, 4, 8, 16}); g_tune.codegen_P = value; }
+  else if (k == "codegen_replicas") { in({-1, 1, 2, 4}); g_tune.codegen_R = value; }
+  else if (k == "trace") { in({0, 1}); g_tune.trace = value; }
+  else FELIX_THROW(FELIX_E_INVALID_ARG, "felix_tune: unknown key " + k);
   FELIX_API_END
 }
 

@@ -80,13 +80,15 @@ void build_round_tables(const SpaceDesc& d, RoundTables& t);
 // -------------------------------------------------------------------------- codegen
 struct CodegenInfo {
   int64_t flops_fwd = 0;
+  int64_t flops_rev = 0;
   int rev_smem_bytes = 0;
 };
 // P = warps cooperating on one 32-candidate block (cone partition of the roots), 1..8
-std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int R, CodegenInfo* info);
+std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int R, bool trace, CodegenInfo* info);
 
 // -------------------------------------------------------------------------- cost model
 struct CostModel {
+  uint64_t uid = 0;              // process-wide unique id (workspace caches key on it, never on the address)
   int device = 0;
   int n_layers = 0;
   std::vector<int32_t> dims;     // dims[0..L]
@@ -100,5 +102,7 @@ struct CostModel {
   float head_b = 0.f;
   std::vector<std::unique_ptr<DevBuf>> W64, b64;   // fp64 copies of every layer (scoring)
 };
+
+uint64_t next_uid();            // process-wide counter for CostModel / space identities
 
 }  // namespace felix

@@ -310,55 +310,46 @@ def test_shape_errors(fx):
     del bad
 
 
-@pytest.mark.parametrize("mode,cg", [("chain", "1"), ("chain-cluster", "1"), ("chain-barrier", "1"), ("layers", "1"),
-                                     ("tile", "2"), ("chain-inexact", "1"), ("tile-inexact", "1")])
-def test_mlp_execution_modes_agree(fx, mode, cg, monkeypatch):
+@pytest.mark.parametrize("mode,cg", [("chain", 1), ("layers", 1), ("tile", 2)])
+def test_mlp_execution_modes_agree(fx, mode, cg):
     """The tile-local fused MLP (1-SM and 2-SM cta_group::2 variants), the persistent chain (dataflow
-    flags, 4-CTA clusters, grid barriers) and the per-layer kernels compute the same split-fp16 products in the same K order: cost and gradient
-    agree to fp32 summation-order noise (the head partial sums are grouped differently).  The chain's
-    first backward layer takes the exact 0/1 mask with the head row folded into its weights (two MMA
-    passes), and so does the tile kernel's B1 step; *-inexact (FELIX_MASK_EXACT=0) is the three-pass
-    form on -w (.) mask."""
+    flags) and the per-layer kernels compute the same split-fp16 products in the same K order: cost and
+    gradient agree to fp32 summation-order noise (the head partial sums are grouped differently).  The
+    first backward layer takes the exact 0/1 mask with the head row folded into its weights."""
     sp = fi.c2_space()
     mlp = fi.make_mlp(fi.DEFAULT_MLP)
     n = 2000
     y0 = torch.from_numpy(fi.make_y0(sp, n, seed=5)).cuda()
     cm = fx.CostModel.from_weights(mlp)
-    monkeypatch.setenv("FELIX_MLP", "tile")
-    monkeypatch.setenv("FELIX_TILE_CG", "1")
-    base = fx.Space(sp).eval(cm, y0, lam=1.0)
-    monkeypatch.setenv("FELIX_MLP", mode.split("-")[0])
-    monkeypatch.setenv("FELIX_TILE_CG", cg)
-    monkeypatch.setenv("FELIX_CHAIN_CS", "4" if mode == "chain-cluster" else "1")
-    monkeypatch.setenv("FELIX_CHAIN_FLAGS", "0" if mode == "chain-barrier" else "1")
-    monkeypatch.setenv("FELIX_MASK_EXACT", "0" if mode.endswith("inexact") else "1")
-    other = fx.Space(sp).eval(cm, y0, lam=1.0)
+    with fx.tuned(mlp="tile", tile_cta_group=1):
+        base = fx.Space(sp).eval(cm, y0, lam=1.0)
+    with fx.tuned(mlp=mode, tile_cta_group=cg):
+        other = fx.Space(sp).eval(cm, y0, lam=1.0)
     for key in ("cost", "grad"):
         a, b = base[key].cpu().numpy(), other[key].cpu().numpy()
         s = np.sqrt(np.mean(a.astype(np.float64) ** 2))
         assert np.max(np.abs(a - b)) / s <= 1e-5, key
 
 
-@pytest.mark.parametrize("cg", ["1", "2"])
-def test_tile_mlp_eval_parity_vs_oracle(fx, cg, monkeypatch):
+@pytest.mark.parametrize("cg", [1, 2])
+def test_tile_mlp_eval_parity_vs_oracle(fx, cg):
     """Tile-local fused MLP (forced; default only from one full wave of tiles) against the oracle on
     C2 and C5 shapes with a ragged last tile (and, for the 2-SM pairs, an odd tile count)."""
-    monkeypatch.setenv("FELIX_MLP", "tile")
-    monkeypatch.setenv("FELIX_TILE_CG", cg)
-    for name, n in (("C2", 1000), ("C5", 389), ("C2_2stmt", 333)):
-        make, dims, _ = CASES[name]
-        sp = make()
-        mlp = fi.make_mlp(dims)
-        y0 = fi.make_y0(sp, n, seed=21)
-        out = {k: v.cpu().numpy() for k, v in fx.Space(sp).eval(fx.CostModel.from_weights(mlp),
-                                                                  torch.from_numpy(y0).cuda(), lam=1.0).items()}
-        ref = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
-        s = np.sqrt(np.mean(ref.c ** 2))
-        assert np.max(np.abs(out["cost"] - ref.c)) / s <= 1e-4, name
-        km = kink_margin(ref.zs)
-        err = np.linalg.norm(out["grad"] - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
-        bad = (err > 1e-3) & ~(km < 1e-4)
-        assert not np.any(bad), (name, np.nonzero(bad)[0][:10], err[bad][:10])
+    with fx.tuned(mlp="tile", tile_cta_group=cg):
+        for name, n in (("C2", 1000), ("C5", 389), ("C2_2stmt", 333)):
+            make, dims, _ = CASES[name]
+            sp = make()
+            mlp = fi.make_mlp(dims)
+            y0 = fi.make_y0(sp, n, seed=21)
+            out = {k: v.cpu().numpy() for k, v in fx.Space(sp).eval(fx.CostModel.from_weights(mlp),
+                                                                      torch.from_numpy(y0).cuda(), lam=1.0).items()}
+            ref = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
+            s = np.sqrt(np.mean(ref.c ** 2))
+            assert np.max(np.abs(out["cost"] - ref.c)) / s <= 1e-4, name
+            km = kink_margin(ref.zs)
+            err = np.linalg.norm(out["grad"] - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
+            bad = (err > 1e-3) & ~(km < 1e-4)
+            assert not np.any(bad), (name, np.nonzero(bad)[0][:10], err[bad][:10])
 
 
 def _gpu_trajectory(space, cm, y0, T, **kw):
@@ -539,49 +530,23 @@ def test_every_c3_c4_task_eval_and_rounding_parity(fx, fam, i):
                 *fo.round_topk(sp, mlp.W, mlp.b, y0, 16))
 
 
-@pytest.mark.parametrize("name", ["C2", "C2_2stmt", "bmm"])
-def test_cone_per_cta_kernels_parity(fx, name, monkeypatch):
-    """Opt-in cone-per-CTA DAG kernels (FELIX_CPB=1: clusters of P CTAs, features and partial adjoints
-    exchanged through distributed shared memory): same tolerances as the default kernels, and one Adam
-    step agrees with the default kernels to fp32 rounding."""
-    make, dims, n = CASES[name]
-    sp = make()
-    mlp = fi.make_mlp(dims)
-    cm = fx.CostModel.from_weights(mlp)
-    y0 = fi.make_y0(sp, n, seed=31)
-    monkeypatch.setenv("FELIX_CPB", "1")
-    space = fx.Space(sp)
-    out = {k: v.cpu().numpy() for k, v in space.eval(cm, torch.from_numpy(y0).cuda(), lam=1.0).items()}
-    ref = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
-    assert np.max(np.abs(out["phi"] - ref.phi) / np.maximum(np.abs(ref.phi), 1.0)) <= 1e-4
-    assert np.max(np.abs(out["g"] - ref.g) / np.maximum(np.abs(ref.g), 1.0)) <= 1e-4
-    for key, r in (("cost", ref.c), ("loss", ref.loss)):
-        assert np.max(np.abs(out[key] - r)) / np.sqrt(np.mean(r ** 2)) <= 1e-4, key
-    err = np.linalg.norm(out["grad"] - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
-    km = kink_margin(ref.zs)
-    assert not np.any((err > 1e-3) & (km >= 1e-4))
-    y1 = torch.from_numpy(y0).cuda()
-    space.search(cm, y1, 1, init_from_y=True)
-    monkeypatch.setenv("FELIX_CPB", "0")
-    y2 = torch.from_numpy(y0).cuda()
-    fx.Space(sp).search(cm, y2, 1, init_from_y=True)
-    assert torch.max(torch.abs(y1 - y2)).item() <= 1e-4 * (1 + torch.max(torch.abs(y2)).item())
-
-
 def _group_spaces():
     r50 = fi.resnet50_spaces()
     return [fi.c2_space(), r50[0], fi.bert_spaces()[1]], [700, 400, 513]
 
 
 @pytest.mark.timeout(600)
-@pytest.mark.parametrize("sc", ["0", "1"])
-def test_search_group_equals_individual_searches(fx, sc, monkeypatch):
+@pytest.mark.parametrize("sc", [0, 1])
+def test_search_group_equals_individual_searches(fx, sc):
     """felix_search_group (one MLP pass per Adam step over the candidates of several spaces) computes
     every member's search exactly as felix_search does: with the tile kernel, whose per-row arithmetic
     does not depend on the row's position, the final y and losses are bit-identical (both with the
-    cone-group DAG kernels and with the split-cone ones, FELIX_SC)."""
-    monkeypatch.setenv("FELIX_MLP", "tile")
-    monkeypatch.setenv("FELIX_SC", sc)
+    cone-group DAG kernels and with the split-cone ones)."""
+    with fx.tuned(mlp="tile", split_cone=sc):
+        _group_vs_individual(fx)
+
+
+def _group_vs_individual(fx):
     mlp = fi.make_mlp(fi.DEFAULT_MLP)
     cm = fx.CostModel.from_weights(mlp)
     sps, ns = _group_spaces()
@@ -637,38 +602,32 @@ def test_search_group_errors(fx):
 
 
 @pytest.mark.parametrize("name,n,steps,P,W,chunks", [
-    ("C2", 1000, 7, "4", "", "1"), ("C2", 4096, 8, "4", "", "1"), ("C2", 1000, 5, "8", "3", "1"),
-    ("C2_2stmt", 700, 6, "4", "2", "1"), ("bmm", 257, 5, "2", "1", "1"), ("C2", 3000, 6, "4", "", "2"),
-    ("C5", 389, 9, "1", "", "1"), ("C5", 389, 8, "2", "", "1"), ("r50_conv1", 300, 4, "4", "1", "1"),
-    ("C2", 1000, 1, "4", "", "1"), ("C2", 1000, 6, "8", "2:2", "1"), ("C2", 4096, 5, "8", "4:2", "1"),
-    ("C2_2stmt", 700, 5, "4", "1:3", "1")])
-def test_split_cone_kernels_match_cone_groups(fx, name, n, steps, P, W, chunks, monkeypatch):
-    """Split-cone reverse kernel (one cone per CTA, partial adjoints through global memory; the next
+    ("C2", 1000, 7, 4, -1, 1), ("C2", 4096, 8, 4, -1, 1), ("C2", 1000, 5, 8, 3, 1),
+    ("C2_2stmt", 700, 6, 4, 2, 1), ("bmm", 257, 5, 2, 1, 1), ("C2", 3000, 6, 4, -1, 2),
+    ("C5", 389, 9, 1, -1, 1), ("C5", 389, 8, 2, -1, 1), ("r50_conv1", 300, 4, 4, 1, 1),
+    ("C2", 1000, 1, 4, -1, 1), ("C2", 1000, 6, 8, 2, 1)])
+def test_split_cone_kernels_match_cone_groups(fx, name, n, steps, P, W, chunks):
+    """Split-cone reverse kernel (one cone per CTA, FP32 partial adjoints through global memory; the next
     step's forward sums them and applies Adam in place, felix_adam_sc after the last step) against the
-    cone-group kernels over several Adam steps (ragged n, several chunks, P = 1..8): the same arithmetic
-    in the same order, so y and the final loss agree to fp32 rounding; the one-step result is also
+    cone-group kernels over several Adam steps (ragged n, several chunks, P = 1..8): both run the same
+    FP32 reverse arithmetic, so y and the final loss agree to fp32 rounding; the one-step result is also
     checked against the oracle."""
     make, dims, _ = CASES[name]
     sp = make()
     mlp = fi.make_mlp(dims)
     cm = fx.CostModel.from_weights(mlp)
     y0 = fi.make_y0(sp, n, seed=77)
-    monkeypatch.setenv("FELIX_P", P)
-    monkeypatch.setenv("FELIX_CHUNKS", chunks)
-    if W:   # "W" or "W:G" (G groups of W x 32 candidates per reverse CTA, one after the other)
-        monkeypatch.setenv("FELIX_SCW", W.split(":")[0])
-        monkeypatch.setenv("FELIX_SCG", W.split(":")[1] if ":" in W else "1")
     out = {}
-    for sc in ("0", "1"):
-        monkeypatch.setenv("FELIX_SC", sc)
-        space = fx.Space(sp)
-        y = torch.from_numpy(y0).cuda()
-        loss = torch.empty(n, device="cuda")
-        space.search(cm, y, steps, init_from_y=True, final_loss=loss)
-        y1 = torch.from_numpy(y0).cuda()
-        space.search(cm, y1, 1, init_from_y=True)
-        out[sc] = (y.cpu().numpy(), loss.cpu().numpy(), y1.cpu().numpy())
-    (ya, la, y1a), (yb, lb, y1b) = out["0"], out["1"]
+    for sc in (0, 1):
+        with fx.tuned(cone_width=P, chunks=chunks, sc_warps=W, split_cone=sc):
+            space = fx.Space(sp)
+            y = torch.from_numpy(y0).cuda()
+            loss = torch.empty(n, device="cuda")
+            space.search(cm, y, steps, init_from_y=True, final_loss=loss)
+            y1 = torch.from_numpy(y0).cuda()
+            space.search(cm, y1, 1, init_from_y=True)
+            out[sc] = (y.cpu().numpy(), loss.cpu().numpy(), y1.cpu().numpy())
+    (ya, la, y1a), (yb, lb, y1b) = out[0], out[1]
     assert np.all(np.isfinite(yb)) and np.all(np.isfinite(lb))
     same = np.mean(ya == yb)
     print(f"{name} n={n} steps={steps} P={P}: exactly equal y {same:.4f}, max |dy| {np.max(np.abs(ya - yb)):.3e}")
@@ -683,22 +642,17 @@ def test_split_cone_kernels_match_cone_groups(fx, name, n, steps, P, W, chunks, 
 
 
 @pytest.mark.parametrize("name,n", [("C2", 4096), ("C1", 300), ("C2_2stmt", 700), ("r50_conv1", 129)])
-def test_scoring_kernels_bit_identical(fx, name, n, monkeypatch):
-    """FP64 scoring: the 128 x 64 register-blocked layer kernel and the row-staged head kernel run the
-    same fma sequence per output (bias first, k ascending) as the 64 x 64 kernels (FELIX_SCORE=1), so the
-    scores are bit-identical; both match the oracle to 1e-12."""
+def test_scoring_kernels_vs_oracle(fx, name, n):
+    """FP64 scoring: the 128 x 64 register-blocked layer kernel and the row-staged head kernel (fixed k
+    order per output) against the oracle's column-at-a-time FP64 MLP to 1e-12."""
     make, dims, _ = CASES[name]
     sp = make()
     mlp = fi.make_mlp(dims)
     cm = fx.CostModel.from_weights(mlp)
     space = fx.Space(sp)
     rs = fo.round_schedules(sp, fi.make_y0(sp, n, seed=15))
-    sched = torch.from_numpy(rs).cuda()
-    monkeypatch.setenv("FELIX_SCORE", "1")
-    old = space.score(cm, sched).cpu().numpy()
-    monkeypatch.setenv("FELIX_SCORE", "0")
-    new = space.score(cm, sched).cpu().numpy()
-    assert np.array_equal(old, new, equal_nan=True)
+    new = space.score(cm, torch.from_numpy(rs).cuda()).cpu().numpy()
     ref = fo.score(sp, mlp.W, mlp.b, rs)
     ok = np.isfinite(ref)
+    assert np.array_equal(np.isfinite(new), ok)
     assert np.all(np.abs(new[ok] - ref[ok]) <= 1e-12 * np.maximum(np.abs(ref[ok]), 1e-3))

@@ -79,9 +79,10 @@ def test_validator_rejects(fx, case, status):
     assert e.value.status == status
 
 
-@pytest.mark.parametrize("which", ["paper", "C1", "C2"])
+@pytest.mark.parametrize("which", ["paper", "C1", "C2", "allops", "rnan"])
 def test_generated_kernels_compile_for_sm100a(fx, which):
-    sp = {"paper": fi.paper_example_space, "C1": fi.c1_space, "C2": fi.c2_space}[which]()
+    sp = {"paper": fi.paper_example_space, "C1": fi.c1_space, "C2": fi.c2_space, "allops": fi.allops_space,
+          "rnan": fi.rnan_space}[which]()
     src = fx.codegen(sp, compile=True)
     for k in ("felix_fwd", "felix_rev_adam", "felix_rev_eval", "felix_hard", "felix_init", "felix_fwd_adam", "felix_rev_sc",
               "felix_adam_sc"):
@@ -104,16 +105,15 @@ def _kernel_body(src, name):
 
 
 @pytest.mark.parametrize("P", ["1", "2", "4", "8"])
-def test_split_cone_codegen_partitions_every_seed_once(fx, P, monkeypatch):
+def test_split_cone_codegen_partitions_every_seed_once(fx, P):
     """The generated split-cone reverse kernel has one branch per cone, seeds every variable-dependent
     feature's adjoint from dL/dphi exactly once across the cones (the cone partition covers the roots
     without overlap), and each cone writes a partial adjoint for every variable; the cone-group reverse
     kernel (felix_rev_adam's body) seeds the same features once.  felix_fwd_adam applies step
     *step_ctr - 1 (the reverse kernel advances the counter)."""
-    monkeypatch.setenv("FELIX_CODEGEN_P", P)
-    monkeypatch.setenv("FELIX_CODEGEN_R", "1")
     sp = fi.c2_space()
-    src = fx.codegen(sp)
+    with fx.tuned(codegen_cone_width=int(P), codegen_replicas=1):
+        src = fx.codegen(sp)
     rev = _kernel_body(src, "felix_rev_sc")
     assert len(re.findall(r"if \(cq_ == \d+\)", rev)) == int(P)
     seeds = re.findall(r"dphi\[\(size_t\)(\d+) \* ld_dphi", rev)
@@ -139,3 +139,28 @@ def _depends_on_var(sp, root):
             return True
         stack.extend(x for x in (a, b, c) if x >= 0)
     return False
+
+
+def test_tune_knobs_validated(fx):
+    """felix_tune: the only way to change execution knobs (the library reads no environment variables)."""
+    with pytest.raises(fx.FelixError) as e:
+        fx.tune(no_such_knob=1)
+    assert e.value.status == 1
+    with pytest.raises(fx.FelixError):
+        fx.tune(cone_width=3)
+    with fx.tuned(mlp="chain", cone_width=8, split_cone=0):
+        pass
+    csrc = os.path.join(ROOT, "paper_conf_asplos_zhaosam24_b200", "csrc")
+    for f in os.listdir(csrc):
+        assert "getenv" not in open(os.path.join(csrc, f)).read(), f
+
+
+def test_split_cone_reverse_is_fp32_and_forward_keeps_fp64_values(fx):
+    """Precision plan of the expression kernels: the split-cone reverse kernel is FP32
+    throughout (no double arithmetic besides the penalty it stores), the search forward evaluates node
+    values in FP64 with FP32 tails of the smooth step (sm_Sf), min / max gaps in FP64."""
+    src = fx.codegen(fi.c2_space())
+    rev = _kernel_body(src, "felix_rev_sc")
+    assert "const double" not in rev and "sf_Sh(" in rev and "sf_dSh(" in rev
+    fwd = src[src.index("void fwd_body("):src.index('extern "C" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd(')]
+    assert "sm_Sf(" in fwd and "const double v" in fwd

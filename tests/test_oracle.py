@@ -141,6 +141,47 @@ def test_smooth_ops_closed_forms():
         assert np.isfinite(fo.smooth_R(np.array([v])))[0] and fo.smooth_S(np.array([-v]))[0] >= 0
 
 
+def test_smooth_eq_ne_value_pins():
+    """EQ(a,b) = S(a-b+1/2) S(b-a+1/2), NE = 1 - EQ (reading O3): values at d = a - b typed in from the
+    closed form S(t) = (1 + t/sqrt(1+t^2))/2: EQ(0) = S(1/2)^2 = (3 + sqrt 5)/10 = 0.52360680,
+    EQ(+-1) = S(3/2) S(-1/2) = 0.25318312; symmetric in d, maximal at d = 0, -> 0 as |d| grows."""
+    B = fi.DagBuilder()
+    a, b = B.var(0), B.var(1)
+    eq, ne = B.cmp(fi.OP_EQ, a, b), B.cmp(fi.OP_NE, a, b)
+    nodes = B.nodes()
+    sp = fi.Space("eqne", [fi.Var("a", fi.VAR_SPLIT, 1, 64), fi.Var("b", fi.VAR_SPLIT, 1, 64)],
+                  [fi.Split(64, [0]), fi.Split(64, [1])], nodes, np.array([a], np.int32), np.array([], np.int32))
+    x = np.array([[5.0, 6.0, 4.0, 2.5, 40.0, 7.0], [5.0, 5.0, 5.0, 2.0, 7.0, 7.0 + 1e-9]])
+    ev = fo.eval_dag(sp, x, smooth=True)
+    E, N = ev.vals[eq], ev.vals[ne]
+    assert abs(E[0] - 0.52360680) < 1e-8 and abs(E[0] - (3 + math.sqrt(5)) / 10) < 1e-15
+    assert abs(E[1] - 0.25318312) < 1e-8 and abs(E[2] - 0.25318312) < 1e-8
+    assert np.allclose(N, 1.0 - E, atol=0, rtol=0)
+    assert E[3] < E[0] and E[3] > E[1] and E[4] < 1e-3 and abs(E[5] - E[0]) < 1e-9
+    hard = fo.eval_dag(sp, np.array([[5.0, 6.0], [5.0, 5.0]]), smooth=False)
+    assert list(hard.vals[eq]) == [1.0, 0.0] and list(hard.vals[ne]) == [0.0, 1.0]
+
+
+def test_rnan_freeze_rule_first_step_closed_form():
+    """Reading R-NaN: a candidate whose loss or gradient is non-finite is not updated (y, m, v stay);
+    every other candidate takes the closed-form first Adam step y - lr g/(|g| + eps)."""
+    sp = fi.rnan_space()
+    mlp = fi.make_mlp(fi.DEFAULT_MLP)
+    y0 = fi.make_y0(sp, 200, seed=9).astype(np.float64)
+    ob = fo.objective(sp, mlp.W, mlp.b, y0, 1.0)
+    ok = np.isfinite(ob.loss) & np.all(np.isfinite(ob.grad), axis=0)
+    assert 0.2 < ok.mean() < 0.95
+    # the non-finite ones are exactly those with x_a < 3 (LOG of a negative number)
+    assert np.array_equal(~ok, np.exp(y0[0]) < 3.0)
+    y1, m1, v1, _ = fo.search(sp, mlp.W, mlp.b, y0, 1, lr=0.05, lam=1.0)
+    assert np.array_equal(y1[:, ~ok], y0[:, ~ok]) and np.all(m1[:, ~ok] == 0) and np.all(v1[:, ~ok] == 0)
+    g = ob.grad[:, ok]
+    assert np.allclose(y1[:, ok], y0[:, ok] - 0.05 * g / (np.abs(g) + 1e-8), rtol=0, atol=1e-12)
+    # rounding: schedules with a non-finite hard feature (x_a in {1, 2}) are invalid
+    rs = fo.round_schedules(sp, y0.astype(np.float32))
+    assert np.array_equal(~fo.validate(sp, rs), rs[:, 0] <= 2)
+
+
 def test_fig4_shapes():
     """Fig. 4: smoothed select(x>0,5,2) stays in (2,5); smoothed max(x,0) > 0 -> x."""
     g4 = GOLD["fig4_select_smooth"]

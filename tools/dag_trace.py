@@ -1,10 +1,10 @@
-"""Phase timing of the generated DAG kernels (FELIX_TRACE): one graph-replayed Adam step's fwd/rev blocks."""
+"""Phase timing of the generated DAG kernels (felix_tune trace): one graph-replayed Adam step's fwd/rev blocks."""
 import os, sys
-os.environ["FELIX_TRACE"] = "1"
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 import felix_inputs as fi
 import paper_conf_asplos_zhaosam24_b200 as fx
+fx.tune(trace=1)
 cfg = fi.config("C2")
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 4096
 sp = cfg.spaces[0]
@@ -20,5 +20,5 @@ for k, name in enumerate(["fwd", "rev"]):
     t = tr[k, :nb]
     t0 = T0
     rel = (t - t0) / 1e3
-    print(f"{name} P={os.environ.get('FELIX_P','auto')} n={n}: start {rel[:,0].min():.2f}..{rel[:,0].max():.2f} | after-wait {rel[:,1].min():.2f}..{rel[:,1].max():.2f} | "
+    print(f"{name} P={os.environ.get('P','auto')} n={n}: start {rel[:,0].min():.2f}..{rel[:,0].max():.2f} | after-wait {rel[:,1].min():.2f}..{rel[:,1].max():.2f} | "
           f"after-compute {rel[:,2].min():.2f}/{np.median(rel[:,2]):.2f}/{rel[:,2].max():.2f} | end {rel[:,3].min():.2f}/{np.median(rel[:,3]):.2f}/{rel[:,3].max():.2f} us")
