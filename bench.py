@@ -704,7 +704,9 @@ def run_felix_tasks(args):
         "config": {"workload": f"{cfg.name}: {len(cfg.spaces)} tasks x {cfg.n_seeds} seeds x {T} steps, "
                                f"MLP {list(cfg.mlp_dims)}, top-{k} per task",
                    "tasks": [sp.name for sp in cfg.spaces], "n_seeds_per_task": cfg.n_seeds, "n_steps": T,
-                   "parallelism": (f"dp{world}: subgraphs by LPT" if mode == "task" else f"dp{world}: seed shards of every task"),
+                   "parallelism": {"task": f"dp{world}: subgraphs by LPT",
+                                   "hybrid": f"dp{world}: seed-split LPT over task chunks (tasks.hybrid_assign)"}.get(
+                                       mode, f"dp{world}: seed shards of every task"),
                    "rank0_tasks": [s.task for s in shards], "rank0_cand_steps_per_bench_step": local_cs,
                    "batching": ("felix_search_group: per Adam step every task's DAG kernels on its own stream, one "
                                 "tensor-core MLP pass over all tasks' candidates" if batched else

@@ -72,7 +72,7 @@ def test_task_plan_uses_est_cost():
     p = ft.plan(3, 8192, 2, "task", costs)
     assert [s.task for s in p[0]] == [1] and [s.task for s in p[1]] == [0, 2]
     assert all(s.seed_lo == 0 and s.n == 8192 for r in p for s in r)
-    assert ft.config_mode("C3") == "task" and ft.config_mode("C4") == "seeds"
+    assert ft.config_mode("C3") == "hybrid" and ft.config_mode("C4") == "seeds"
 
 
 def test_pack_merge_roundtrip_single_rank():
@@ -119,7 +119,7 @@ def _worker(rank, world, port, mode, ys, k, out):
 
 
 @pytest.mark.timeout(300)
-@pytest.mark.parametrize("mode", ["task", "seeds"])
+@pytest.mark.parametrize("mode", ["task", "seeds", "hybrid"])
 def test_gloo_world2_per_task_topk_equals_single_process(mode):
     spaces, mlp = _tasks()
     k = 12
@@ -145,3 +145,49 @@ def test_gloo_world2_per_task_topk_equals_single_process(mode):
             assert gidx == list(ridx)
             assert np.array_equal(np.array(gsc), rsc)
             assert gsched == rsched.tolist()
+
+
+# ----------------------------------------------------------------------------- hybrid (seed-split LPT)
+def _check_partition(plan, n_tasks, n):
+    for t in range(n_tasks):
+        rng = sorted((s.seed_lo, s.seed_lo + s.n) for sh in plan for s in sh if s.task == t)
+        assert rng[0][0] == 0 and rng[-1][1] == n
+        assert all(a[1] == b[0] for a, b in zip(rng, rng[1:]))          # contiguous, disjoint cover
+    for sh in plan:
+        assert len({s.task for s in sh}) == len(sh)                      # one shard per (rank, task)
+
+
+def test_hybrid_plan_partitions_every_task_and_balances_c3():
+    """C3 (21 nearly equal ResNet-50 tasks) on 8 ranks: task-mode LPT gives 3 tasks vs a mean of 2.625
+    (0.875); the seed-split plan is within 5 % of the lower bound total / world."""
+    costs = [ft.est_cost(8192, 200, 955392, nn) for nn in np.linspace(150, 260, 21).astype(int)]
+    for world in (1, 2, 4, 8):
+        p = ft.plan(21, 8192, world, "hybrid", costs)
+        _check_partition(p, 21, 8192)
+        eff = (sum(costs) / world) / ft.makespan(p, costs, 8192)
+        assert eff >= 0.95, (world, eff)
+    lpt = ft.plan(21, 8192, 8, "task", costs)
+    assert (sum(costs) / 8) / ft.makespan(lpt, costs, 8192) <= 0.88
+
+
+def test_hybrid_makespan_vs_brute_force_optimum():
+    """Small instances: the plan's makespan against the brute-force optimum over all assignments of the
+    same chunks to ranks (the plan is LPT over the chunks: within Graham's 4/3 bound of it), and against
+    the fractional lower bound max(total / world, largest chunk)."""
+    rng = np.random.default_rng(11)
+    for world in (2, 3):
+        for _ in range(4):
+            costs = list(rng.integers(1, 40, size=4).astype(float))
+            n = 12
+            p = ft.hybrid_assign(costs, n, world, chunks_per_rank=1)
+            _check_partition(p, 4, n)
+            total = sum(costs)
+            target = total / world
+            nch = [max(1, min(n, int(np.ceil(c / target - 1e-9)))) for c in costs]
+            chunks = [costs[t] * (ft.seed_range(n, i, nch[t])[1] - ft.seed_range(n, i, nch[t])[0]) / n
+                      for t in range(4) for i in range(nch[t])]
+            opt = min(max(sum(c for c, r in zip(chunks, asg) if r == q) for q in range(world))
+                      for asg in itertools.product(range(world), repeat=len(chunks)))
+            ms = ft.makespan(p, costs, n)
+            assert ms <= (4 / 3 - 1 / (3 * world)) * opt + 1e-9
+            assert ms >= max(total / world, max(chunks)) - 1e-9
