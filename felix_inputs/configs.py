@@ -18,7 +18,7 @@ from typing import Dict, List, Sequence, Tuple
 import numpy as np
 
 from .dag import Space, VAR_INT, VAR_SPLIT
-from .programs import build_space, conv2d_spec, dense_spec, paper_dense_add_s1
+from .programs import build_space, conv2d_spec, dense_spec, layernorm_spec, paper_dense_add_s1, softmax_spec
 
 MASK64 = (1 << 64) - 1
 DEFAULT_MLP = (82, 512, 256, 256, 1)
@@ -136,7 +136,9 @@ def c5_space() -> Space:
 
 
 def bert_spaces() -> List[Space]:
-    """BERT-base seq 128 dense / bmm subgraphs (C4; softmax/layernorm sketches are NEXT)."""
+    """BERT-base seq 128 subgraphs (C4, BASELINE.json configs[3] "batched matmul/softmax"): QKV / output /
+    FFN dense layers, the two attention bmms, the attention softmax (12 heads x 128 x 128) and a layernorm
+    (128 x 768)."""
     return [
         build_space(dense_spec("bert_qkv_128x2304x768", 128, 2304, 768, i_levels="vti", j_levels="vti", k_vars=2)),
         build_space(dense_spec("bert_bmm_qk_12x128x128x64", 128, 128, 64, batch=12, i_levels="ti", j_levels="vti", k_vars=1, bias=False)),
@@ -144,6 +146,8 @@ def bert_spaces() -> List[Space]:
         build_space(dense_spec("bert_proj_128x768x768", 128, 768, 768, i_levels="vti", j_levels="vti", k_vars=2)),
         build_space(dense_spec("bert_ffn1_128x3072x768", 128, 3072, 768, i_levels="vti", j_levels="vti", k_vars=2, gelu=True)),
         build_space(dense_spec("bert_ffn2_128x768x3072", 128, 768, 3072, i_levels="vti", j_levels="vti", k_vars=2)),
+        build_space(softmax_spec("bert_softmax_12x128x128", 12, 128, 128, i_levels="vti", j_vars=1)),
+        build_space(layernorm_spec("bert_layernorm_128x768", 128, 768, i_levels="vti", j_vars=2)),
     ]
 
 

@@ -43,6 +43,14 @@ import numpy as np
 from .dag import (DagBuilder, Space, Split, Var, VAR_INT, VAR_SPLIT, prune)
 
 N_FEATURES = 82          # "a total of 82 distinct features"
+# Arithmetic of one reduction-statement instance (op-count features and flop counts):
+#   "mad"      O[s] += A * B                    contraction (dense, bmm, conv)
+#   "exp_sum"  O[s] += exp(A)                   softmax's exp-sum stage (Fig. 9 operator mix)
+#   "sum_sq"   O1[s] += A; O2[s] += A * A       layernorm's mean / variance statistics
+STMT_OPS = {"mad": {"mad": 1, "addsub": 0, "math": 0},
+            "exp_sum": {"mad": 0, "addsub": 1, "math": 1},
+            "sum_sq": {"mad": 1, "addsub": 1, "math": 0}}
+STMT_FLOPS = {"mad": 2.0, "exp_sum": 2.0, "sum_sq": 3.0}
 UNROLL_MAX = 1024        # Unroll(max_step=UNROLL0), Fig. 3 L584 / L599; search range [1, 1024]
 
 
@@ -81,6 +89,7 @@ class ProgramSpec:
     thread_limit: int = 1024
     local_limit: int = 256
     vthread_limit: int = 64
+    stmt: str = "mad"          # reduction statement kind (STMT_OPS)
 
     def axis_extent(self, name: str) -> int:
         for a in self.spatial:
@@ -331,10 +340,12 @@ def build_space(spec: ProgramSpec, statements: int = 1) -> Space:
 
     # -- op counts / GPU mapping / loop structure
     epi_in_main = statements == 1
-    feats.append(("float_mad", b.const(nmac)))
-    feats.append(("float_addsub", b.const(prodE if spec.bias and epi_in_main else 0.0)))
+    ops = STMT_OPS[spec.stmt]
+    fpi = STMT_FLOPS[spec.stmt]
+    feats.append(("float_mad", b.const(nmac * ops["mad"])))
+    feats.append(("float_addsub", b.const((prodE if spec.bias and epi_in_main else 0.0) + nmac * ops["addsub"])))
     feats.append(("float_cmp", b.const(prodE if spec.relu and epi_in_main else 0.0)))
-    feats.append(("float_math", b.const(prodE if spec.gelu and epi_in_main else 0.0)))
+    feats.append(("float_math", b.const((prodE if spec.gelu and epi_in_main else 0.0) + nmac * ops["math"])))
     feats.append(("blockIdx_len", NB))
     feats.append(("vthread_len", NV))
     feats.append(("threadIdx_len", NT))
@@ -393,8 +404,8 @@ def build_space(spec: ProgramSpec, statements: int = 1) -> Space:
         ("out.stores", b.const(prodE)),
         ("shared_bytes_total", smem_bytes),
         ("local_bytes", b.mul(b.const(4.0), out_per_thread)),
-        ("flops_per_global_byte", b.div(b.const(2.0 * nmac), b.add(b.sum(gbytes), b.const(4.0 * prodE)))),
-        ("flops_per_thread", b.mul(b.const(2.0), stmts_per_thread)),
+        ("flops_per_global_byte", b.div(b.const(fpi * nmac), b.add(b.sum(gbytes), b.const(4.0 * prodE)))),
+        ("flops_per_thread", b.mul(b.const(fpi), stmts_per_thread)),
         ("global_bytes_per_block", b.div(b.sum(gbytes), NB)),
     ]
     assert len(feats) <= N_FEATURES
@@ -448,6 +459,21 @@ def conv2d_spec(name: str, C: int, H: int, W: int, K: int, R: int, S: int, strid
     inp = Buffer("In", [[("rc", 1)], [("h", stride), ("rh", 1)], [("w", stride), ("rw", 1)]])
     wt = Buffer("Wt", [[("co", 1)], [("rc", 1)], [("rh", 1)], [("rw", 1)]])
     return ProgramSpec(name, spatial, red, [inp, wt], bias=bias, relu=relu, bias_axis="co")
+
+
+def softmax_spec(name: str, B: int, N: int, M: int, *, i_levels="vti", j_vars=1) -> ProgramSpec:
+    """Softmax's reduction stage over the last axis, O[b, i] += exp(A[b, i, j]) (BERT attention scores,
+    batch x heads folded into b; the operator mix of Fig. 9).  The normalisation stage is an
+    elementwise pass without schedule variables of its own."""
+    spatial = [SAxis("b", B, "t"), SAxis("i", N, i_levels)]
+    return ProgramSpec(name, spatial, [RAxis("j", M, j_vars)], [Buffer("A", [[("b", 1)], [("i", 1)], [("j", 1)]])],
+                       bias=False, stmt="exp_sum")
+
+
+def layernorm_spec(name: str, N: int, D: int, *, i_levels="vti", j_vars=2) -> ProgramSpec:
+    """LayerNorm's statistics stage, O1[i] += A[i, j], O2[i] += A[i, j]^2 (BERT hidden states)."""
+    return ProgramSpec(name, [SAxis("i", N, i_levels)], [RAxis("j", D, j_vars)], [Buffer("A", [[("i", 1)], [("j", 1)]])],
+                       bias=False, stmt="sum_sq")
 
 
 def paper_dense_add_s1(N: int = 64, M: int = 64, K: int = 64) -> Space:

@@ -110,10 +110,13 @@ def simulate(spec, x: Dict[str, int]) -> Dict[str, float]:
     for s in sp:
         out_lin = out_lin * s["E"] + idx[s["name"]]
     assert len(np.unique(out_lin)) == E
-    f["float_mad"] = n
-    f["float_addsub"] = E if spec.bias else 0
+    # one reduction-statement instance does: "mad" 1 multiply-add; "exp_sum" 1 exp + 1 add;
+    # "sum_sq" 1 add + 1 multiply-add (written out here independently of the feature DAG)
+    k_mad, k_add, k_math, k_flops = {"mad": (1, 0, 0, 2), "exp_sum": (0, 1, 1, 2), "sum_sq": (1, 1, 0, 3)}[spec.stmt]
+    f["float_mad"] = n * k_mad
+    f["float_addsub"] = (E if spec.bias else 0) + n * k_add
     f["float_cmp"] = E if spec.relu else 0
-    f["float_math"] = E if spec.gelu else 0
+    f["float_math"] = (E if spec.gelu else 0) + n * k_math
     NB = len(np.unique(blk))
     NT = len(np.unique(thr))
     f["blockIdx_len"] = NB
@@ -186,8 +189,8 @@ def simulate(spec, x: Dict[str, int]) -> Dict[str, float]:
     f["out.stores"] = E
     f["shared_bytes_total"] = smem_total
     f["local_bytes"] = 4 * f["outputs_per_thread"]
-    f["flops_per_global_byte"] = 2.0 * n / (gbytes_total + 4 * E)
-    f["flops_per_thread"] = 2.0 * f["stmts_per_thread"]
+    f["flops_per_global_byte"] = k_flops * n / (gbytes_total + 4 * E)
+    f["flops_per_thread"] = k_flops * f["stmts_per_thread"]
     f["global_bytes_per_block"] = gbytes_total / NB
     # constraint quantities
     f["_threads"] = NT
