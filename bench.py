@@ -57,6 +57,8 @@ def parse():
                          "(SURVEY 8(f) row 3; not the headline)")
     ap.add_argument("--unbatched", action="store_true",
                     help="C3/C4: one felix_search per task on its own stream instead of felix_search_group")
+    ap.add_argument("--tune", action="append", default=[],
+                    help="experiments: felix_tune knob key=value (repeatable; the headline uses the defaults)")
     ap.add_argument("--history", action="store_true",
                     help="paper-faithful Alg. 1: round every visited point (varValuesHistory, l.13/17/20) "
                          "instead of the final point only (SURVEY 8(f) row 1; not the headline)")
@@ -121,6 +123,12 @@ def measured_peaks():
         with open(path) as f:
             return json.load(f), "measured"
     return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback (B200_PROFILING.md)"
+
+
+def apply_tune(fx, args):
+    for kv in args.tune:
+        k, v = kv.split("=")
+        fx.tune(**{k: (v if k == "mlp" and not v.lstrip("-").isdigit() else int(v))})
 
 
 def sp_info_flops(space):
@@ -281,6 +289,7 @@ def run_felix(args):
     import felix_inputs as fi
     import paper_conf_asplos_zhaosam24_b200 as fx
     from paper_conf_asplos_zhaosam24_b200 import dist as fdist
+    apply_tune(fx, args)
 
     cfg, sp, _, _ = felix_workload(args)
     mlp = fi.make_mlp(cfg.mlp_dims)
@@ -508,6 +517,8 @@ def run_felix(args):
         line["e2e"] = e2e
     if cpu is not None:
         line["cpu_baseline"] = cpu
+    if args.tune:
+        line["tune"] = args.tune
     print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
@@ -568,6 +579,7 @@ def run_felix_tasks(args):
     dev = torch.cuda.current_device()
     import felix_inputs as fi
     import paper_conf_asplos_zhaosam24_b200 as fx
+    apply_tune(fx, args)
     tasks = _tasks_module()
 
     cfg = fi.config(args.config)

@@ -279,8 +279,10 @@ FELIX_EXPORT felix_status felix_profile_enable(felix_space* s, int32_t enable);
 FELIX_EXPORT felix_status felix_profile_read(felix_space* s, double* ms, int64_t* launches);
 FELIX_EXPORT felix_status felix_profile_reset(felix_space* s);
 /* Debug: copy the per-block %globaltimer stamps of the generated kernels (only for kernels generated
- * after felix_tune("trace", 1)): uint64 [2][8192][4] = {fwd, rev} x block x
- * {start, after griddepcontrol.wait, after compute, end}.  n_words bounds the copy. */
+ * after felix_tune("trace", 1)): uint64 [2][8192][8] = {forward, reverse} x block x stamp.  Forward
+ * (felix_fwd / felix_fwd_adam): start, after griddepcontrol.wait, after the Adam prologue, after the cone
+ * compute, end.  Split-cone reverse: start, after wait, after compute, end; cone-group reverse: slots
+ * 4..7.  Only the last launch's stamps survive.  n_words bounds the copy. */
 FELIX_EXPORT felix_status felix_debug_trace(felix_space* s, uint64_t* out, int64_t n_words);
 
 #ifdef __cplusplus

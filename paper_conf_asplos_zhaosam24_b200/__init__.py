@@ -394,8 +394,8 @@ class Space:
         _check(_lib.felix_profile_reset(self._h))
 
     def debug_trace(self) -> np.ndarray:
-        """uint64 [2][8192][4] globaltimer stamps (space created with FELIX_TRACE set)."""
-        out = np.zeros((2, 8192, 4), dtype=np.uint64)
+        """uint64 [2][8192][8] globaltimer stamps (kernels generated after tune(trace=1))."""
+        out = np.zeros((2, 8192, 8), dtype=np.uint64)
         _check(_lib.felix_debug_trace(self._h, out.ctypes.data_as(_P), ctypes.c_int64(out.size)))
         return out
 

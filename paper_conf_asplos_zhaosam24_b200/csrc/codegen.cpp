@@ -242,8 +242,8 @@ struct Gen {
         case FELIX_OP_DIV: e = divx(A, B); ++flops; break;
         case FELIX_OP_NEG: e = "-" + A; break;
         case FELIX_OP_POW: e = (f32 ? "f_powf(" : "pow(") + A + ", " + cst(nd.imm) + ")"; ++flops; break;
-        case FELIX_OP_EXP: e = (f32 ? "__expf(" : "exp(") + A + ")"; ++flops; break;
-        case FELIX_OP_LOG: e = (f32 ? "__logf(" : "log(") + A + ")"; ++flops; break;
+        case FELIX_OP_EXP: e = (f32 ? "expf(" : "exp(") + A + ")"; ++flops; break;
+        case FELIX_OP_LOG: e = (f32 ? "logf(" : "log(") + A + ")"; ++flops; break;
         case FELIX_OP_SQRT: e = (f32 ? "f_sqrtf(" : mode == 0 ? "f_sqrt(" : "sqrt(") + A + ")"; ++flops; break;
         case FELIX_OP_MIN: e = hard ? "fmin(" + A + ", " + B + ")" : mn + "(" + A + ", " + B + ")"; flops += 6; break;
         case FELIX_OP_MAX: e = hard ? "fmax(" + A + ", " + B + ")" : mx + "(" + A + ", " + B + ")"; flops += 6; break;
@@ -435,7 +435,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
   o << kPrelude;
 
   if (trace)
-    o << "__device__ unsigned long long felix_trace[2][8192][4];\n"
+    o << "__device__ unsigned long long felix_trace[2][8192][8];\n"
          "#define TSTAMP(k, s) do { if (threadIdx.x == 0 && blockIdx.x < 8192) { unsigned long long t_; asm volatile(\"mov.u64 %0, %globaltimer;\" : \"=l\"(t_)); felix_trace[k][blockIdx.x][s] = t_; } } while (0)\n";
   else
     o << "#define TSTAMP(k, s) do {} while (0)\n";
@@ -596,7 +596,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "        sx[j][lane] = exp((double)yy);\n      }\n"
     << "    }\n  }\n"
     << "  for (int k = tid; k < NS * 32 * (K0P + 1); k += PG * 32) (&sphi[0][0][0])[k] = 0.f;\n"
-    << "  __syncthreads();\n";
+    << "  __syncthreads();\n  TSTAMP(0, 2);\n";
   for (int q = 0; q < P; ++q) {
     o << "  if (wq == " << q << ") {\n";
     if (q == 0)
@@ -614,7 +614,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     for (int k : part.feat[q]) o << "    sphi[" << fs(k) << "][lane][" << fk(k) << "] = slogf_(v" << d.froots[k] << ");\n";
     o << "  }\n";
   }
-  o << "  __syncthreads();\n  TSTAMP(0, 2);\n"
+  o << "  __syncthreads();\n  TSTAMP(0, 3);\n"
     << "  // rows c0 .. c0+31 of each statement are contiguous: K0P/8 uint4 per row for hi and for lo\n"
     << "#pragma unroll\n"
     << "  for (int it = 0; it < (NS * 32 * (K0P / 8) + PG * 32 - 1) / (PG * 32); ++it) {\n"
@@ -634,7 +634,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "    }\n"
     << "    reinterpret_cast<uint4*>(phi_hi + row * K0P)[q8] = make_uint4(h[0], h[1], h[2], h[3]);\n"
     << "    reinterpret_cast<uint4*>(phi_lo + row * K0P)[q8] = make_uint4(l[0], l[1], l[2], l[3]);\n"
-    << "  }\n  TSTAMP(0, 3);\n}\n"
+    << "  }\n  TSTAMP(0, 4);\n}\n"
     << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd(const float* __restrict__ yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr) {\n"
     << "  fwd_body<0>(const_cast<float*>(yv), n, ldy, phi_hi, phi_lo, step_ctr, nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f);\n}\n"
     << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd_adam(float* yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr,\n"
@@ -665,9 +665,9 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "  const bool livew = cw < n;\n"
     << "  const int ccw = livew ? cw : n - 1;\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
-    << "  if (!EVAL) TSTAMP(1, 0);\n"
+    << "  if (!EVAL) TSTAMP(1, 4);\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n"
-    << "  if (!EVAL) TSTAMP(1, 1);\n"
+    << "  if (!EVAL) TSTAMP(1, 5);\n"
     << "  const double dlam = (double)lam;\n"
     // everything the epilogue needs from memory is requested now, so its latency overlaps the DAG
     << "  __shared__ double sx_all[NREP][NV * 32];\n"
@@ -718,7 +718,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     o << "    }\n";
     o << "    }\n    {\n";
     for (int j = 0; j < M; ++j)
-      if (used[j]) o << "    const float x" << j << " = (float)sx[" << j << " * 32 + lane];\n";
+      if (used[j]) o << "    const float x" << j << " = expf(sy[" << j << " * 32 + lane]);\n";
     g.emit_forward(rcone[q], 3, "x", "    ");
     // user-root penalties of this group
     o << "    float pen = 0.f;\n";
@@ -741,7 +741,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     o << "    }\n  }\n";
   }
   // automatic roots (warp 0) from the staged y
-  o << "  cp_async_wait_all();\n  __syncthreads();\n  if (!EVAL) TSTAMP(1, 2);\n"
+  o << "  cp_async_wait_all();\n  __syncthreads();\n  if (!EVAL) TSTAMP(1, 6);\n"
     << "  if (wq == 0) {\n";
   for (int j = 0; j < M; ++j) o << "    const double y" << j << " = (double)sy[" << j << " * 32 + lane];\n";
   for (size_t q = 0; q < autos.size(); ++q) {
@@ -802,7 +802,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "        mv[o_] = m; vv[o_] = v; yv[(size_t)j * ldy + c] = sy[j * 32 + lane] - step * m / (sqrtf(v) * rb + eps);\n"
     << "      }\n"
     << "    }\n"
-    << "    TSTAMP(1, 3);\n"
+    << "    TSTAMP(1, 7);\n"
     << "  }\n}\n\n";
   o << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_adam(float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
     << "    float* mv, float* vv, const int* step_ctr, float lr, float b1, float b2, float eps, float* o_loss) {\n"
@@ -832,13 +832,15 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "  const int c = ((blockIdx.x / PG) * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32 + (threadIdx.x & 31);\n"
     << "  const bool live = c < n;\n  const int ccw = live ? c : n - 1;\n"
     << "  asm volatile(\"griddepcontrol.launch_dependents;\" ::: \"memory\");\n"
+    << "  TSTAMP(1, 0);\n"
     << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n"
+    << "  TSTAMP(1, 1);\n"
     << "  if (blockIdx.x == 0 && threadIdx.x == 0) *step_ctr += 1;\n";
   for (int q = 0; q < P; ++q) {
     o << "  if (cq_ == " << q << ") {\n";
     const auto used = vars_in(rcone[q]);
     for (int j = 0; j < M; ++j)
-      if (used[j]) o << "    const float x" << j << " = __expf(yv[(size_t)" << j << " * ldy + ccw]);\n";
+      if (used[j]) o << "    const float x" << j << " = expf(yv[(size_t)" << j << " * ldy + ccw]);\n";
     g.emit_forward(rcone[q], 3, "x", "    ");
     o << "    float pq = 0.f;\n";
     for (int r : part.cons[q]) o << "    const float pr" << r << " = fmaxf(v" << d.croots[r] << ", 0.f); pq += pr" << r << " * pr" << r << ";\n";
@@ -855,11 +857,12 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
       if (g.depvar[nd]) o << "    " << g.adj(nd) << " += 2.f * lam * pr" << r << ";\n";
     }
     g.emit_reverse_body(need, "    ", true);
+    o << "    TSTAMP(1, 2);\n";
     // partial dL/dy_j = x_j * dL/dx_j of this cone (x_j is at hand here; the Adam prologue needs no exp)
     o << "    if (live) {\n      pen[(size_t)" << q << " * n + c] = (double)pq;\n";
     for (int j = 0; j < M; ++j)
       o << "      part[((size_t)" << q << " * NV + " << j << ") * n + c] = " << (used[j] ? "x" + std::to_string(j) + " * gx" + std::to_string(j) : std::string("0.f")) << ";\n";
-    o << "    }\n  }\n";
+    o << "    }\n    TSTAMP(1, 3);\n  }\n";
   }
   o << "}\n\n";
   // felix_adam_sc: the last Adam step (thread per candidate, in place) + the final loss

@@ -1,24 +1,38 @@
-"""Phase timing of the generated DAG kernels (felix_tune trace): one graph-replayed Adam step's fwd/rev blocks."""
-import os, sys
+"""Phase timing of the generated DAG kernels inside the graph-replayed search (felix_tune trace=1):
+per-block %globaltimer stamps of the last Adam step's felix_fwd_adam (start, after griddepcontrol.wait,
+after the Adam prologue, after the cone compute, end) and felix_rev_sc (start, after wait, after
+compute, end), relative to the first forward block's start.  Usage: python tools/dag_trace.py [C2|C5] [n]"""
+import json
+import os
+import sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-import numpy as np, torch
+import numpy as np
+import torch
 import felix_inputs as fi
 import paper_conf_asplos_zhaosam24_b200 as fx
+
 fx.tune(trace=1)
-cfg = fi.config("C2")
-n = int(sys.argv[1]) if len(sys.argv) > 1 else 4096
+cfg = fi.config(sys.argv[1] if len(sys.argv) > 1 else "C2")
+n = int(sys.argv[2]) if len(sys.argv) > 2 else cfg.n_seeds
 sp = cfg.spaces[0]
 space = fx.Space(sp)
 cm = fx.CostModel.from_weights(fi.make_mlp(cfg.mlp_dims))
 y = torch.empty((sp.n_vars, n), device="cuda")
-space.search(cm, y, 10, rng_seed=cfg.rng_seed, init_from_y=False)
+for _ in range(3):
+    space.search(cm, y, 20, rng_seed=cfg.rng_seed, init_from_y=False)
 torch.cuda.synchronize()
 tr = space.debug_trace().astype(np.int64)
-nb = (n + 31) // 32
-T0 = tr[0, :nb, 1].min()          # common origin: the forward kernel's first block past griddepcontrol.wait
-for k, name in enumerate(["fwd", "rev"]):
-    t = tr[k, :nb]
-    t0 = T0
-    rel = (t - t0) / 1e3
-    print(f"{name} P={os.environ.get('P','auto')} n={n}: start {rel[:,0].min():.2f}..{rel[:,0].max():.2f} | after-wait {rel[:,1].min():.2f}..{rel[:,1].max():.2f} | "
-          f"after-compute {rel[:,2].min():.2f}/{np.median(rel[:,2]):.2f}/{rel[:,2].max():.2f} | end {rel[:,3].min():.2f}/{np.median(rel[:,3]):.2f}/{rel[:,3].max():.2f} us")
+f = tr[0][tr[0, :, 0] > 0]
+r = tr[1][tr[1, :, 0] > 0]
+t0 = f[:, 0].min()
+q = lambda a: [round(float(np.min(a)) / 1e3, 2), round(float(np.median(a)) / 1e3, 2), round(float(np.max(a)) / 1e3, 2)]
+out = {"config": cfg.name, "n": n, "fwd_blocks": len(f), "rev_blocks": len(r),
+       "fwd_us_rel_min_med_max": {"start": q(f[:, 0] - t0), "after_wait": q(f[:, 1] - t0), "after_adam": q(f[:, 2] - t0),
+                                  "after_compute": q(f[:, 3] - t0), "end": q(f[:, 4] - t0)},
+       "fwd_phase_us_med": {"wait": q(f[:, 1] - f[:, 0])[1], "adam_prologue": q(f[:, 2] - f[:, 1])[1],
+                            "cones": q(f[:, 3] - f[:, 2])[1], "phi_store": q(f[:, 4] - f[:, 3])[1]},
+       "rev_us_rel_min_med_max": {"start": q(r[:, 0] - t0), "after_wait": q(r[:, 1] - t0), "after_compute": q(r[:, 2] - t0),
+                                  "end": q(r[:, 3] - t0)},
+       "rev_phase_us_med": {"wait": q(r[:, 1] - r[:, 0])[1], "cone": q(r[:, 2] - r[:, 1])[1], "store": q(r[:, 3] - r[:, 2])[1]},
+       "span_us": round((max(f[:, 4].max(), r[:, 3].max()) - t0) / 1e3, 2)}
+print(json.dumps(out))
