@@ -40,7 +40,7 @@ from typing import Dict, List, Optional, Sequence, Tuple
 
 import numpy as np
 
-from .dag import (DagBuilder, Space, Split, Var, VAR_INT, VAR_SPLIT, prune)
+from .dag import (DagBuilder, Space, Split, Var, VAR_INT, VAR_SPLIT, OP_EQ, prune)
 
 N_FEATURES = 82          # "a total of 82 distinct features"
 # Arithmetic of one reduction-statement instance (op-count features and flop counts):
@@ -235,6 +235,82 @@ def _dim_footprint(ctx: _Ctx, dim: List[Tuple[str, int]], scope: str) -> int:
     return b.sub(b.mul(V, L), b.mul(b.sub(V, b.const(1.0)), overlap))
 
 
+def _dim_bbox(ctx: _Ctx, dim: List[Tuple[str, int]]) -> int:
+    """Bounding-box extent (max - min + 1) of one index dim over block 0's first outer-reduction tile:
+    the shared-memory tile a block allocates for it (row-major over the dims' boxes)."""
+    b, spec = ctx.b, ctx.spec
+    if not dim:
+        return b.const(1.0)
+    sp = [(a, c) for a, c in dim if spec.is_spatial(a)]
+    rd = [(a, c) for a, c in dim if not spec.is_spatial(a)]
+    if not sp:
+        (a, _), = rd
+        return ctx.Rt(next(x for x in spec.reduction if x.name == a))
+    (sa, c), = sp
+    ax = next(x for x in spec.spatial if x.name == sa)
+    if not rd:
+        return ctx.Tb(ax)
+    (ra, _), = rd
+    R = next(x for x in spec.reduction if x.name == ra).extent
+    return b.add(b.mul(b.const(c), b.sub(ctx.Tb(ax), b.const(1.0))), b.const(R))
+
+
+def _smem_stride(ctx: _Ctx, buf: Buffer, loops) -> int:
+    """Shared-memory address delta (elements, row-major over the dims' bounding boxes) along the innermost
+    non-trivial loop of L; 0 when that loop is an outer-reduction loop (each ro tile reuses the buffer)."""
+    b = ctx.b
+    boxes = [_dim_bbox(ctx, d) for d in buf.dims]
+    pitch = []
+    for d in range(len(buf.dims)):
+        pitch.append(b.prod(boxes[d + 1:]))
+    stride = b.const(0.0)
+    for kind, ext, axn, step in loops:
+        coef = [c for d, dim in enumerate(buf.dims) for a, c in dim if a == axn]
+        dpos = [d for d, dim in enumerate(buf.dims) for a, c in dim if a == axn]
+        if kind == "ro" or not coef:
+            delta = b.const(0.0)
+        else:
+            delta = b.sum([b.mul(b.mul(step, b.const(float(c))), pitch[d]) for c, d in zip(coef, dpos)])
+        stride = b.select(b.gt(ext, b.const(1.0)), delta, stride)
+    return stride, b.prod(boxes)
+
+
+def _out_stride(spec: ProgramSpec, loops) -> float:
+    """(per loop) output linear-index delta: spatial axes row-major in spec.spatial order."""
+    E = [ax.extent for ax in spec.spatial]
+    pitch = {ax.name: float(np.prod(E[i + 1:])) for i, ax in enumerate(spec.spatial)}
+    return pitch
+
+
+def _loop_shape_feats(ctx: _Ctx, loops, NB, NT) -> List[Tuple[str, int]]:
+    """GPU-mapping / loop-structure features shared by both statements."""
+    b = ctx.b
+    inner_len, outer_len = b.const(1.0), b.const(1.0)
+    for _, ext, _, _ in loops:                   # outer -> inner: the innermost non-trivial loop wins
+        inner_len = b.select(b.gt(ext, b.const(1.0)), ext, inner_len)
+    for _, ext, _, _ in reversed(loops):         # inner -> outer: the outermost non-trivial loop wins
+        outer_len = b.select(b.gt(ext, b.const(1.0)), ext, outer_len)
+    mx = b.const(1.0)
+    for _, ext, _, _ in loops:
+        mx = b.max(mx, ext)
+    return [("total_threads", b.mul(NB, NT)), ("innermost_len", inner_len), ("outermost_len", outer_len),
+            ("max_loop_extent", mx)]
+
+
+def _out_feats(ctx: _Ctx, loops) -> List[Tuple[str, int]]:
+    """Output-buffer slot: store stride along the innermost non-trivial loop (reduction loops do not
+    move the output), its vectorizability, and the outputs a block writes."""
+    b, spec = ctx.b, ctx.spec
+    pitch = _out_stride(spec, loops)
+    stride = b.const(0.0)
+    for kind, ext, axn, step in loops:
+        d = b.mul(step, b.const(pitch[axn])) if axn in pitch else b.const(0.0)
+        stride = b.select(b.gt(ext, b.const(1.0)), d, stride)
+    vec = b.select(b.cmp(OP_EQ, stride, b.const(1.0)), b.const(1.0), b.const(0.0))
+    return [("out.innermost_stride", stride), ("out.vectorizable", vec),
+            ("out.block_footprint", b.prod([ctx.Tb(ax) for ax in spec.spatial]))]
+
+
 def _linear_stride(spec: ProgramSpec, buf: Buffer, axis: str) -> int:
     """Address delta (elements, row-major buffer) when `axis` index increases by 1."""
     shape = spec.buffer_shape(buf)
@@ -296,12 +372,16 @@ def _epilogue_feats(spec: ProgramSpec, ctx: "_Ctx") -> List[Tuple[str, int]]:
             for kind, ext, axn, step in loops:
                 d = b.mul(step, b.const(float(_linear_stride(spec, buf, axn))))
                 stride = b.select(b.gt(ext, b.const(1.0)), d, stride)
+            sstride, bbox = _smem_stride(ctx, buf, loops)
             vals = [blk, gl, gb, b.ceildiv(blk, NT), thr, b.div(opt, thr), b.div(b.mul(opt, NT), blk),
-                    b.div(b.const(E), gl), stride, b.mul(b.const(4.0), blk)]
+                    b.div(b.const(E), gl), stride, b.mul(b.const(4.0), blk),
+                    b.select(b.cmp(OP_EQ, stride, b.const(1.0)), b.const(1.0), b.const(0.0)),
+                    b.div(gl, b.const(float(np.prod(spec.buffer_shape(buf))))), sstride, bbox, b.div(blk, bbox)]
         else:
-            vals = [b.const(0.0)] * 10
+            vals = [b.const(0.0)] * 15
         names = ["block_footprint", "global_load_elems", "global_bytes", "coop_loads_per_thread", "thread_footprint",
-                 "thread_reuse", "block_reuse", "global_reuse", "innermost_stride", "shared_bytes"]
+                 "thread_reuse", "block_reuse", "global_reuse", "innermost_stride", "shared_bytes",
+                 "vectorizable", "load_ratio", "smem_inner_stride", "smem_tile_elems", "smem_tile_util"]
         f += [(f"in{slot}.{nm}", v) for nm, v in zip(names, vals)]
     gsum = b.sum(gbytes) if gbytes else b.const(0.0)
     f += [
@@ -312,6 +392,8 @@ def _epilogue_feats(spec: ProgramSpec, ctx: "_Ctx") -> List[Tuple[str, int]]:
         ("flops_per_thread", b.mul(b.const(n_ops), opt)),
         ("global_bytes_per_block", b.div(gsum, NB)),
     ]
+    f += _out_feats(ctx, loops)
+    f += _loop_shape_feats(ctx, loops, NB, NT)
     return f
 
 
@@ -387,6 +469,7 @@ def build_space(spec: ProgramSpec, statements: int = 1) -> Space:
             s = _linear_stride(spec, buf, axn)
             d = b.mul(step, b.const(float(s)))
             stride = b.select(b.gt(ext, b.const(1.0)), d, stride)
+        sstride, bbox = _smem_stride(ctx, buf, loops)
         feats += [
             (f"{buf.name}.block_footprint", blk),
             (f"{buf.name}.global_load_elems", gl),
@@ -398,6 +481,12 @@ def build_space(spec: ProgramSpec, statements: int = 1) -> Space:
             (f"{buf.name}.global_reuse", b.div(b.const(nmac), gl)),
             (f"{buf.name}.innermost_stride", stride),
             (f"{buf.name}.shared_bytes", b.mul(b.const(4.0), blk)),
+            # global-side vectorizability and re-fetch ratio, shared-memory tile (bounding box) layout
+            (f"{buf.name}.vectorizable", b.select(b.cmp(OP_EQ, stride, b.const(1.0)), b.const(1.0), b.const(0.0))),
+            (f"{buf.name}.load_ratio", b.div(gl, b.const(float(np.prod(spec.buffer_shape(buf)))))),
+            (f"{buf.name}.smem_inner_stride", sstride),
+            (f"{buf.name}.smem_tile_elems", bbox),
+            (f"{buf.name}.smem_tile_util", b.div(blk, bbox)),
         ]
     smem_bytes = b.mul(b.const(4.0), b.sum(smem_elems))
     feats += [
@@ -408,6 +497,8 @@ def build_space(spec: ProgramSpec, statements: int = 1) -> Space:
         ("flops_per_thread", b.mul(b.const(fpi), stmts_per_thread)),
         ("global_bytes_per_block", b.div(b.sum(gbytes), NB)),
     ]
+    feats += _out_feats(ctx, loops)
+    feats += _loop_shape_feats(ctx, loops, NB, NT)
     assert len(feats) <= N_FEATURES
     n_used = len(feats)
     zero = b.const(0.0)

@@ -77,12 +77,26 @@ def allops_space() -> Space:
 
 
 def rnan_space() -> Space:
-    B = DagBuilder()
-    a, b = B.var(0), B.var(1)
-    f = [a, b, B.mul(a, b), B.log(B.sub(a, B.const(3.0))), B.div(b, B.sub(a, B.const(2.0))),
-         B.min(a, B.mul(b, B.const(2.0))), B.sqrt(B.add(a, b))]
-    f += [B.const(0.0)] * (82 - len(f))
-    nodes = B.nodes()
-    return Space("rnan", [Var("a", VAR_SPLIT, 1, 64), Var("b", VAR_SPLIT, 1, 64)],
-                 [Split(64, [0]), Split(64, [1])], nodes, np.array(f, dtype=np.int32), np.array([], dtype=np.int32),
-                 feature_names=[f"f{i}" for i in range(82)])
+    """C1's dense 64x64x64 space (6 variables, its 58 features) with two reserved feature slots replaced by
+    LOG(x_0 - 3) and x_1 / (x_0 - 2): a real, well-conditioned feature set in which candidates with
+    x_0 < 3 have a non-finite smooth feature and schedules with x_0 in {1, 2} a non-finite hard one."""
+    from .configs import c1_space
+    base = c1_space()
+    nodes = list(base.nodes.tolist())
+    def add(op, a=-1, b=-1, c=-1, imm=0.0):
+        nodes.append((op, a, b, c, imm))
+        return len(nodes) - 1
+    from .dag import OP_CONST, OP_VAR, OP_SUB, OP_LOG, OP_DIV
+    x0, x1 = add(OP_VAR, imm=0.0), add(OP_VAR, imm=1.0)
+    f_log = add(OP_LOG, add(OP_SUB, x0, add(OP_CONST, imm=3.0)))
+    f_div = add(OP_DIV, x1, add(OP_SUB, x0, add(OP_CONST, imm=2.0)))
+    arr = np.zeros(len(nodes), dtype=base.nodes.dtype)
+    for i, r in enumerate(nodes):
+        arr[i] = r
+    froots = base.feature_roots.copy()
+    names = list(base.feature_names)
+    free = [k for k, nm in enumerate(names) if nm.startswith("reserved")]
+    froots[free[0]], froots[free[1]] = f_log, f_div
+    names[free[0]], names[free[1]] = "log(x0-3)", "x1/(x0-2)"
+    return Space("rnan", base.vars, base.splits, arr, froots, base.constraint_roots.copy(), names,
+                 list(base.constraint_names), None)

@@ -151,7 +151,14 @@ struct Gen {
   int64_t flops = 0;
   int64_t flops_rev = 0;   // arithmetic ops of the emitted reverse sweep (adjoint accumulations + local partials)
 
-  explicit Gen(const SpaceDesc& dd) : d(dd), n((int)dd.nodes.size()), depvar(n, false) {
+  std::vector<bool> isbool;     // comparison / logic node (FP32 mode keeps its complement c<i> = 1 - v<i>)
+
+  explicit Gen(const SpaceDesc& dd) : d(dd), n((int)dd.nodes.size()), depvar(n, false), isbool(n, false) {
+    for (int i = 0; i < n; ++i) {
+      const int op_ = dd.nodes[i].op;
+      isbool[i] = op_ == FELIX_OP_GT || op_ == FELIX_OP_GE || op_ == FELIX_OP_LT || op_ == FELIX_OP_LE || op_ == FELIX_OP_EQ ||
+                  op_ == FELIX_OP_NE || op_ == FELIX_OP_AND || op_ == FELIX_OP_OR || op_ == FELIX_OP_NOT;
+    }
     for (int i = 0; i < n; ++i) {
       const felix_node& nd = d.nodes[i];
       if (nd.op == FELIX_OP_VAR) { depvar[i] = true; continue; }
@@ -183,6 +190,72 @@ struct Gen {
   // smooth step), 1: IEEE smooth FP64 (sampler), 2: hard FP64 (integer points), 3: FP32 (split-cone
   // reverse kernel).  Smooth compare / min / max nodes keep t and h = sqrt(1+t^2) as named values for
   // the reverse sweep: compares as FP32 hf<i> (and kf<i> for EQ/NE), min / max as h<i> in the node's type.
+  // complement 1 - v of a BOOL operand in FP32 mode (a CONST used as a condition has none stored)
+  std::string cmp_of(int j) const {
+    return isbool[j] ? "c" + std::to_string(j) : "(1.f - v" + std::to_string(j) + ")";
+  }
+
+  // FP32 forward of the BOOL / SELECT nodes with complements: a smooth step near 1 keeps its tail in
+  // c<i> (1 - S rounded to 1.f would lose it), and a SELECT uses the complement of its condition on the
+  // side where the condition is near 1, so  select(c, a, b) = a + (b - a) (1 - c)  with (1 - c) exact to
+  // FP32 relative precision (e.g. b = 5e9, 1 - c = 1.9e-8: the value 98 that b + (a - b) c loses in FP32).
+  bool emit_f32_bool(int i, const char* ind) {
+    const felix_node& nd = d.nodes[i];
+    const std::string A = "v" + std::to_string(nd.a), B = "v" + std::to_string(nd.b), C = "v" + std::to_string(nd.c);
+    const std::string I = std::to_string(i);
+    switch (nd.op) {
+      case FELIX_OP_GT: case FELIX_OP_GE: case FELIX_OP_LT: case FELIX_OP_LE: {
+        const bool ab = nd.op == FELIX_OP_GT || nd.op == FELIX_OP_GE;
+        o << ind << "const float t" << I << " = " << (ab ? A + " - " + B : B + " - " + A) << ";\n"
+          << ind << "const float hf" << I << " = sf_hyp(t" << I << ");\n"
+          << ind << "const float tl" << I << " = sf_tail(t" << I << ", hf" << I << ");\n"
+          << ind << "const float v" << I << " = t" << I << " >= 0.f ? 1.f - tl" << I << " : tl" << I << ";\n"
+          << ind << "const float c" << I << " = t" << I << " >= 0.f ? tl" << I << " : 1.f - tl" << I << ";\n";
+        flops += 6;
+        return true;
+      }
+      case FELIX_OP_EQ: case FELIX_OP_NE: {
+        o << ind << "const float d" << I << " = " << A << " - " << B << ";\n"
+          << ind << "const float t" << I << " = d" << I << " + 0.5f;\n"
+          << ind << "const float u" << I << " = 0.5f - d" << I << ";\n"
+          << ind << "const float hf" << I << " = sf_hyp(t" << I << ");\n"
+          << ind << "const float kf" << I << " = sf_hyp(u" << I << ");\n"
+          << ind << "const float ta" << I << " = sf_tail(t" << I << ", hf" << I << "), tb" << I << " = sf_tail(u" << I << ", kf" << I << ");\n"
+          << ind << "const float pa" << I << " = t" << I << " >= 0.f ? 1.f - ta" << I << " : ta" << I << ";\n"
+          << ind << "const float qa" << I << " = t" << I << " >= 0.f ? ta" << I << " : 1.f - ta" << I << ";\n"
+          << ind << "const float pb" << I << " = u" << I << " >= 0.f ? 1.f - tb" << I << " : tb" << I << ";\n"
+          << ind << "const float qb" << I << " = u" << I << " >= 0.f ? tb" << I << " : 1.f - tb" << I << ";\n"
+          << ind << "const float e" << I << " = pa" << I << " * pb" << I << ";\n"
+          << ind << "const float ce" << I << " = qa" << I << " + qb" << I << " - qa" << I << " * qb" << I << ";\n"
+          << ind << "const float v" << I << " = " << (nd.op == FELIX_OP_EQ ? "e" : "ce") << I << ";\n"
+          << ind << "const float c" << I << " = " << (nd.op == FELIX_OP_EQ ? "ce" : "e") << I << ";\n";
+        flops += 16;
+        return true;
+      }
+      case FELIX_OP_AND:
+        o << ind << "const float v" << I << " = " << A << " * " << B << ";\n"
+          << ind << "const float c" << I << " = " << cmp_of(nd.a) << " + " << cmp_of(nd.b) << " - " << cmp_of(nd.a) << " * " << cmp_of(nd.b) << ";\n";
+        flops += 4;
+        return true;
+      case FELIX_OP_OR:
+        o << ind << "const float v" << I << " = " << A << " + " << B << " - " << A << " * " << B << ";\n"
+          << ind << "const float c" << I << " = " << cmp_of(nd.a) << " * " << cmp_of(nd.b) << ";\n";
+        flops += 4;
+        return true;
+      case FELIX_OP_NOT:
+        o << ind << "const float v" << I << " = " << cmp_of(nd.a) << ";\n"
+          << ind << "const float c" << I << " = " << A << ";\n";
+        return true;
+      case FELIX_OP_SELECT:
+        o << ind << "const float v" << I << " = " << A << " >= 0.5f ? " << B << " + (" << C << " - " << B << ") * " << cmp_of(nd.a)
+          << " : " << C << " + (" << B << " - " << C << ") * " << A << ";\n";
+        flops += 3;
+        return true;
+      default:
+        return false;
+    }
+  }
+
   void emit_forward(const std::vector<bool>& in, int mode, const char* xname, const char* ind = "  ") {
     const bool hard = mode == 2, f32 = mode == 3;
     const std::string T = f32 ? "float" : "double";
@@ -200,6 +273,7 @@ struct Gen {
       const std::string A = "v" + std::to_string(nd.a), B = "v" + std::to_string(nd.b), C = "v" + std::to_string(nd.c);
       std::string e;
       const std::string I = std::to_string(i);
+      if (f32 && emit_f32_bool(i, ind)) continue;
       if (mode == 0 || f32) {
         switch (nd.op) {
           case FELIX_OP_GT: case FELIX_OP_GE: case FELIX_OP_LT: case FELIX_OP_LE: {
@@ -339,12 +413,16 @@ struct Gen {
         case FELIX_OP_EXP: acc(nd.a, g + " * " + J(V)); break;
         case FELIX_OP_LOG: acc(nd.a, g + " * " + J(rcp + A + ")")); break;
         case FELIX_OP_SQRT: acc(nd.a, g + " * " + J((f32 ? "0.5f * " : "0.5 * ") + rcp + V + ")")); break;
-        case FELIX_OP_MAX:
-          o << ind << "  const " << T << " s = " << J((f32 ? "sf_Sh(t" : "sm_Sh(t") + I + ", h" + I + ")") << ";\n";
-          acc(nd.a, g + " * s"); acc(nd.b, g + " * (" + one + " - s)"); break;
-        case FELIX_OP_MIN:
-          o << ind << "  const " << T << " s = " << J((f32 ? "sf_Sh(t" : "sm_Sh(t") + I + ", h" + I + ")") << ";\n";
-          acc(nd.a, g + " * (" + one + " - s)"); acc(nd.b, g + " * s"); break;
+        case FELIX_OP_MAX: case FELIX_OP_MIN:
+          if (f32) {   // S(t) and 1 - S(t) both from the tail
+            o << ind << "  const float tl = sf_tail(t" << I << ", h" << I << ");\n"
+              << ind << "  const float s = t" << I << " >= 0.f ? 1.f - tl : tl, cs = t" << I << " >= 0.f ? tl : 1.f - tl;\n";
+          } else {
+            o << ind << "  const double s = sm_Sh(t" << I << ", h" << I << "), cs = 1.0 - s;\n";
+          }
+          if (nd.op == FELIX_OP_MAX) { acc(nd.a, g + " * s"); acc(nd.b, g + " * cs"); }
+          else { acc(nd.a, g + " * cs"); acc(nd.b, g + " * s"); }
+          break;
         case FELIX_OP_GT: case FELIX_OP_GE:
           o << ind << "  const " << T << " t = " << g << " * " << J("sf_dSh(hf" + I + ")") << ";\n";
           acc(nd.a, "t"); acc(nd.b, "t", true); break;
@@ -352,15 +430,28 @@ struct Gen {
           o << ind << "  const " << T << " t = " << g << " * " << J("sf_dSh(hf" + I + ")") << ";\n";
           acc(nd.a, "t", true); acc(nd.b, "t"); break;
         case FELIX_OP_EQ: case FELIX_OP_NE: {
-          o << ind << "  const " << T << " t = " << (nd.op == FELIX_OP_EQ ? "" : "-") << g << " * "
-            << J("(" + T + ")sf_dSh(hf" + I + ") * q" + I + " - p" + I + " * (" + T + ")sf_dSh(kf" + I + ")") << ";\n";
+          if (f32) {
+            // d/dd [S(d+1/2) S(1/2-d)] without the cancellation of S'(a) S(b) - S(a) S'(b) near d = 0:
+            // -d/2 [(ha^2 + ha hb + hb^2)/(ha + hb) + 1 + a^2 + ab + b^2] / (ha^3 hb^3), a = d+1/2, b = 1/2-d
+            o << ind << "  const float ha = hf" << I << ", hb = kf" << I << ", a_ = t" << I << ", b_ = u" << I << ";\n"
+              << ind << "  const float der = -0.5f * d" << I << " * ((ha * ha + ha * hb + hb * hb) * f_rcpf(ha + hb) + 1.f + a_ * a_ + a_ * b_ + b_ * b_)"
+              << " * f_rcpf(ha * ha * ha * hb * hb * hb);\n"
+              << ind << "  const float t = " << (nd.op == FELIX_OP_EQ ? "" : "-") << g << " * der;\n";
+          } else {
+            o << ind << "  const double t = " << (nd.op == FELIX_OP_EQ ? "" : "-") << g << " * "
+              << "((double)sf_dSh(hf" << I << ") * q" << I << " - p" << I << " * (double)sf_dSh(kf" << I << "));\n";
+          }
           acc(nd.a, "t"); acc(nd.b, "t", true); break;
         }
         case FELIX_OP_AND: acc(nd.a, g + " * " + J(B)); acc(nd.b, g + " * " + J(A)); break;
-        case FELIX_OP_OR: acc(nd.a, g + " * " + J(one + " - " + B)); acc(nd.b, g + " * " + J(one + " - " + A)); break;
+        case FELIX_OP_OR:
+          if (f32) { acc(nd.a, g + " * " + cmp_of(nd.b)); acc(nd.b, g + " * " + cmp_of(nd.a)); }
+          else { acc(nd.a, g + " * " + J(one + " - " + B)); acc(nd.b, g + " * " + J(one + " - " + A)); }
+          break;
         case FELIX_OP_NOT: acc(nd.a, g, true); break;
         case FELIX_OP_SELECT:
-          acc(nd.a, g + " * " + J(B + " - " + C)); acc(nd.b, g + " * " + J(A)); acc(nd.c, g + " * " + J(one + " - " + A)); break;
+          acc(nd.a, g + " * " + J(B + " - " + C)); acc(nd.b, g + " * " + J(A));
+          acc(nd.c, g + " * " + (f32 ? cmp_of(nd.a) : J(one + " - " + A))); break;
         default: break;
       }
       o << ind << "}\n";

@@ -99,6 +99,30 @@ def _buffer_index(spec, buf, idx) -> np.ndarray:
     return lin
 
 
+def _dim_values(spec, buf, idx):
+    """Per index dim of `buf`: its value for every instance."""
+    n = len(next(iter(idx.values())))
+    return [sum(c * idx[a] for a, c in dim) if dim else np.zeros(n, dtype=np.int64) for dim in buf.dims]
+
+
+def _smem_layout(dims, sel):
+    """Bounding box (max - min + 1 per dim) of the instances `sel` and the row-major local index of every
+    instance inside it (the block's shared-memory tile)."""
+    lo = [int(d[sel].min()) for d in dims]
+    box = [int(d[sel].max()) - l + 1 for d, l in zip(dims, lo)]
+    local = np.zeros_like(dims[0])
+    for d, l, e in zip(dims, lo, box):
+        local = local * e + (d - l)
+    return box, local
+
+
+def _shape_feats(L, NB, NT):
+    ext = [e for _, _, e in L]
+    nontriv = [e for e in ext if e > 1]
+    return {"total_threads": NB * NT, "innermost_len": nontriv[-1] if nontriv else 1,
+            "outermost_len": nontriv[0] if nontriv else 1, "max_loop_extent": max([1] + ext)}
+
+
 def simulate(spec, x: Dict[str, int]) -> Dict[str, float]:
     sp, rd = _levels(spec, x)
     L, blk, thr, ro, idx, lvec = _instances(spec, sp, rd)
@@ -153,9 +177,21 @@ def simulate(spec, x: Dict[str, int]) -> Dict[str, float]:
         if L[pos][2] > 1:
             inner = pos
             break
+    if inner is None:
+        sel0 = sel1 = None
+    else:
+        sel0 = t0 & np.all(lvec == 0, axis=1)
+        one = np.zeros(len(L), dtype=np.int64)
+        one[inner] = 1
+        sel1 = t0 & np.all(lvec == one[None, :], axis=1)
     for buf in spec.inputs:
         lin = _buffer_index(spec, buf, idx)
         blk_fp = len(np.unique(lin[b0r0]))
+        box, local = _smem_layout(_dim_values(spec, buf, idx), b0r0)
+        if inner is None or L[inner][0] == "ro":
+            sstride = 0                                # no loop, or a new tile per outer-reduction step
+        else:
+            sstride = int(local[sel1][0] - local[sel0][0])
         # per (block, ro) distinct counts
         key = blk * (ro.max() + 1) + ro
         order = np.lexsort((lin, key))
@@ -184,6 +220,11 @@ def simulate(spec, x: Dict[str, int]) -> Dict[str, float]:
         f[f"{buf.name}.global_reuse"] = n / gl
         f[f"{buf.name}.innermost_stride"] = stride
         f[f"{buf.name}.shared_bytes"] = 4 * blk_fp
+        f[f"{buf.name}.vectorizable"] = 1 if stride == 1 else 0
+        f[f"{buf.name}.load_ratio"] = gl / int(np.prod(spec.buffer_shape(buf)))
+        f[f"{buf.name}.smem_inner_stride"] = sstride
+        f[f"{buf.name}.smem_tile_elems"] = int(np.prod(box))
+        f[f"{buf.name}.smem_tile_util"] = blk_fp / int(np.prod(box))
         gbytes_total += 4 * gl
         smem_total += 4 * blk_fp
     f["out.stores"] = E
@@ -192,6 +233,11 @@ def simulate(spec, x: Dict[str, int]) -> Dict[str, float]:
     f["flops_per_global_byte"] = k_flops * n / (gbytes_total + 4 * E)
     f["flops_per_thread"] = k_flops * f["stmts_per_thread"]
     f["global_bytes_per_block"] = gbytes_total / NB
+    ostride = 0 if inner is None else int(out_lin[sel1][0] - out_lin[sel0][0])
+    f["out.innermost_stride"] = ostride
+    f["out.vectorizable"] = 1 if ostride == 1 else 0
+    f["out.block_footprint"] = len(np.unique(out_lin[blk == 0]))
+    f.update(_shape_feats(L, NB, NT))
     # constraint quantities
     f["_threads"] = NT
     f["_smem"] = smem_total
@@ -285,7 +331,18 @@ def simulate_epilogue(spec, x: Dict[str, int]) -> Dict[str, float]:
             inner = pos
             break
     names = ["block_footprint", "global_load_elems", "global_bytes", "coop_loads_per_thread", "thread_footprint",
-             "thread_reuse", "block_reuse", "global_reuse", "innermost_stride", "shared_bytes"]
+             "thread_reuse", "block_reuse", "global_reuse", "innermost_stride", "shared_bytes",
+             "vectorizable", "load_ratio", "smem_inner_stride", "smem_tile_elems", "smem_tile_util"]
+    if inner is None:
+        sel0 = sel1 = None
+    else:
+        sel0 = t0 & np.all(lvec == 0, axis=1)
+        one = np.zeros(len(L), dtype=np.int64)
+        one[inner] = 1
+        sel1 = t0 & np.all(lvec == one[None, :], axis=1)
+    out_lin = np.zeros(n, dtype=np.int64)
+    for s in sp:
+        out_lin = out_lin * s["E"] + idx[s["name"]]
     gsum = smem = 0
     for slot in range(len(spec.inputs)):
         if slot == 0 and spec.bias:
@@ -295,20 +352,16 @@ def simulate_epilogue(spec, x: Dict[str, int]) -> Dict[str, float]:
             gl = int(sum(len(np.unique(lin[blk == bb])) for bb in range(NB)))
             thr_fp = len(np.unique(lin[t0]))
             pt = np.bincount(np.arange(blk_fp) % NT, minlength=NT)
-            if inner is None:
-                stride = 0
-            else:
-                sel0 = t0 & np.all(lvec == 0, axis=1)
-                one = np.zeros(len(L), dtype=np.int64)
-                one[inner] = 1
-                sel1 = t0 & np.all(lvec == one[None, :], axis=1)
-                stride = int(lin[sel1][0] - lin[sel0][0])
+            stride = 0 if inner is None else int(lin[sel1][0] - lin[sel0][0])
+            box, local = _smem_layout([lin], b0)
+            sstride = 0 if inner is None else int(local[sel1][0] - local[sel0][0])
+            size = spec.axis_extent(spec.bias_axis)
             vals = [blk_fp, gl, 4 * gl, int(pt.max()), thr_fp, per_thread / thr_fp, int(b0.sum()) / blk_fp, n / gl,
-                    stride, 4 * blk_fp]
+                    stride, 4 * blk_fp, 1 if stride == 1 else 0, gl / size, sstride, box[0], blk_fp / box[0]]
             gsum += 4 * gl
             smem += 4 * blk_fp
         else:
-            vals = [0] * 10
+            vals = [0] * 15
         for nm, v in zip(names, vals):
             f[f"in{slot}.{nm}"] = v
     n_ops = int(spec.bias) + int(spec.relu) + int(spec.gelu)
@@ -318,4 +371,9 @@ def simulate_epilogue(spec, x: Dict[str, int]) -> Dict[str, float]:
     f["flops_per_global_byte"] = n_ops * E / (gsum + 4 * E)
     f["flops_per_thread"] = n_ops * per_thread
     f["global_bytes_per_block"] = gsum / NB
+    ostride = 0 if inner is None else int(out_lin[sel1][0] - out_lin[sel0][0])
+    f["out.innermost_stride"] = ostride
+    f["out.vectorizable"] = 1 if ostride == 1 else 0
+    f["out.block_footprint"] = len(np.unique(out_lin[blk == 0]))
+    f.update(_shape_feats(L, NB, NT))
     return f

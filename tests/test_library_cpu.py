@@ -157,10 +157,11 @@ def test_tune_knobs_validated(fx):
 
 def test_split_cone_reverse_is_fp32_and_forward_keeps_fp64_values(fx):
     """Precision plan of the expression kernels: the split-cone reverse kernel is FP32
-    throughout (no double arithmetic besides the penalty it stores), the search forward evaluates node
+    throughout (no double arithmetic besides the penalty it stores; comparison / logic nodes carry their
+    complements c = 1 - v), the search forward evaluates node
     values in FP64 with FP32 tails of the smooth step (sm_Sf), min / max gaps in FP64."""
     src = fx.codegen(fi.c2_space())
     rev = _kernel_body(src, "felix_rev_sc")
-    assert "const double" not in rev and "sf_Sh(" in rev and "sf_dSh(" in rev
+    assert "const double" not in rev and "sf_tail(" in rev and "sf_dSh(" in rev and "const float c" in rev
     fwd = src[src.index("void fwd_body("):src.index('extern "C" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd(')]
     assert "sm_Sf(" in fwd and "const double v" in fwd

@@ -5,7 +5,7 @@
 #include <algorithm>
 #include <cuda.h>
 #include <cuda_runtime.h>
-#include "../paper_conf_asplos_zhaosam24_b200/csrc/mlp_chain.cuh"
+#include "../../paper_conf_asplos_zhaosam24_b200/csrc/mlp_chain.cuh"
 using namespace felix;
 static CUtensorMap mk(const void* p, int rows, int cols, int box) {
   CUtensorMap m; cuuint64_t d[2] = {(cuuint64_t)cols, (cuuint64_t)rows}; cuuint64_t st[1] = {(cuuint64_t)cols * 2};
@@ -38,7 +38,7 @@ int main(int argc, char** argv) {
   add(2, EPI_HEAD, 256, 256, act[2], W[2], act[3], bnB);
   add(3, EPI_MASK, 256, 256, act[3], WT[2], act[2], bnB);
   add(4, EPI_MASK, 512, 256, act[2], WT[1], act[1], bnA);
-  add(5, EPI_F32T, 96, 512, act[1], WT[0], act[0], 96);
+  add(5, EPI_F32T, 96, 512, act[1], WT[0], act[0], argc > 7 ? atoi(argv[7]) : 32);
   P.n_layers = 6; P.m_tiles = mt;
   P.grid_bar = (unsigned int*)dz(64);
   int grid = std::min(148, mt * 512 / bnA);

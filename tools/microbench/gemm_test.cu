@@ -7,7 +7,7 @@
 #include <algorithm>
 #include <cuda.h>
 #include <cuda_runtime.h>
-#include "../paper_conf_asplos_zhaosam24_b200/csrc/mlp_gemm.cuh"
+#include "../../paper_conf_asplos_zhaosam24_b200/csrc/mlp_gemm.cuh"
 
 using namespace felix;
 #define CK(x) do { cudaError_t e = (x); if (e != cudaSuccess) { printf("CUDA %s at %d: %s\n", #x, __LINE__, cudaGetErrorString(e)); exit(1);} } while (0)

@@ -1,7 +1,7 @@
 // tcgen05.mma kind::f16 SS-mode issue-rate microbenchmark (scratch): cycles per MMA (M=128, K=16)
 #include <cstdio>
 #include <cuda_runtime.h>
-#include "../paper_conf_asplos_zhaosam24_b200/csrc/sm100_ptx.cuh"
+#include "../../paper_conf_asplos_zhaosam24_b200/csrc/sm100_ptx.cuh"
 using namespace felix;
 __global__ void __launch_bounds__(128, 1) k_rate(int N, int iters, int sts, unsigned long long* out) {
   extern __shared__ uint8_t smem_raw[];

@@ -1,7 +1,7 @@
 // tcgen05.mma SS-mode: which feature of the tile kernel's MMA stream costs throughput (scratch)
 #include <cstdio>
 #include <cuda_runtime.h>
-#include "../paper_conf_asplos_zhaosam24_b200/csrc/sm100_ptx.cuh"
+#include "../../paper_conf_asplos_zhaosam24_b200/csrc/sm100_ptx.cuh"
 using namespace felix;
 // mode bits: 1 = 3-pass hi/lo addresses, 2 = alternate accumulator halves every 12, 4 = F1 mix (24 x N=64 then 24 x N=128),
 //            8 = commit every 12, 16 = accumulate=0 at each block start

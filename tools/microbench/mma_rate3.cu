@@ -1,7 +1,7 @@
 // tcgen05.mma issue-cost variants (scratch): 3-pass 64-wide K block = 12 MMAs, N=64 (TC floor 48 cyc/MMA)
 #include <cstdio>
 #include <cuda_runtime.h>
-#include "../paper_conf_asplos_zhaosam24_b200/csrc/sm100_ptx.cuh"
+#include "../../paper_conf_asplos_zhaosam24_b200/csrc/sm100_ptx.cuh"
 using namespace felix;
 
 __device__ __forceinline__ void mma_elect(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {

@@ -5,7 +5,7 @@
 #include <algorithm>
 #include <cuda.h>
 #include <cuda_runtime.h>
-#include "../paper_conf_asplos_zhaosam24_b200/csrc/mlp_tile.cuh"
+#include "../../paper_conf_asplos_zhaosam24_b200/csrc/mlp_tile.cuh"
 using namespace felix;
 static CUtensorMap mk(const void* p, int rows, int cols, int box) {
   CUtensorMap m; cuuint64_t d[2] = {(cuuint64_t)cols, (cuuint64_t)rows}; cuuint64_t st[1] = {(cuuint64_t)cols * 2};
