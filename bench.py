@@ -798,7 +798,7 @@ def main():
     args = parse()
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         return spawn_ranks(args)
-    multi = args.config in ("C3", "C4")
+    multi = args.config in ("C3", "C4", "MBV2")
     if args.impl == "reference":
         return run_reference_tasks(args) if multi else run_reference(args)
     return run_felix_tasks(args) if multi else run_felix(args)

@@ -18,7 +18,8 @@ from typing import Dict, List, Sequence, Tuple
 import numpy as np
 
 from .dag import Space, VAR_INT, VAR_SPLIT
-from .programs import build_space, conv2d_spec, dense_spec, layernorm_spec, paper_dense_add_s1, softmax_spec
+from .programs import (build_space, conv2d_spec, dense_spec, depthwise_conv2d_spec, layernorm_spec, paper_dense_add_s1,
+                       softmax_spec)
 
 MASK64 = (1 << 64) - 1
 DEFAULT_MLP = (82, 512, 256, 256, 1)
@@ -170,6 +171,17 @@ def resnet50_spaces() -> List[Space]:
     return S
 
 
+def mobilenet_v2_spaces() -> List[Space]:
+    """MobileNet-v2 @224 (the north star's "ResNet/MobileNet convs"): its depthwise 3x3 convs
+    (stride 1 and 2) and representative pointwise 1x1 expansion / projection convs, batch 1."""
+    dws = [(32, 112, 112, 1), (96, 56, 56, 2), (144, 56, 56, 1), (144, 28, 28, 2), (192, 28, 28, 1),
+           (384, 14, 14, 1), (576, 7, 7, 2), (960, 7, 7, 1)]          # (C, H_out, W_out, stride)
+    out = [build_space(depthwise_conv2d_spec(f"mbv2_dw_c{C}_h{H}_s{st}", C, H, W, 3, 3, st)) for C, H, W, st in dws]
+    pws = [(16, 112, 112, 96), (24, 56, 56, 144), (144, 28, 28, 32), (384, 14, 14, 96), (960, 7, 7, 320)]
+    out += [build_space(conv2d_spec(f"mbv2_pw_c{C}_h{H}_k{K}", C, H, W, K, 1, 1, 1)) for C, H, W, K in pws]
+    return out
+
+
 def config(name: str) -> Config:
     if name == "C1":
         return Config("C1", [c1_space()], C1_MLP, 64, 20, 0x5EED0001)
@@ -179,6 +191,8 @@ def config(name: str) -> Config:
         return Config("C3", resnet50_spaces(), DEFAULT_MLP, 8192, 200, 0x5EED0003)
     if name == "C4":
         return Config("C4", bert_spaces(), DEFAULT_MLP, 16384, 500, 0x5EED0004)
+    if name == "MBV2":      # not a BASELINE config: MobileNet-v2 task set, searched like C3
+        return Config("MBV2", mobilenet_v2_spaces(), DEFAULT_MLP, 8192, 200, 0x5EED0006)
     if name == "C5":
         return Config("C5", [c5_space()], DEFAULT_MLP, 1 << 20, 200, 0x5EED0005, topk=64)
     raise KeyError(name)

@@ -552,6 +552,18 @@ def conv2d_spec(name: str, C: int, H: int, W: int, K: int, R: int, S: int, strid
     return ProgramSpec(name, spatial, red, [inp, wt], bias=bias, relu=relu, bias_axis="co")
 
 
+def depthwise_conv2d_spec(name: str, C: int, H: int, W: int, R: int, S: int, stride: int = 1, *,
+                          c_levels="vti", h_levels="vti", w_levels="vti", bias=True, relu=True) -> ProgramSpec:
+    """Depthwise conv (MobileNet-v2): O[c, h, w] += In[c, stride*h + rh, stride*w + rw] * Wt[c, rh, rw]
+    (batch 1, pre-padded input; no reduction over channels, so the only reduction axes are the unsplit
+    kernel window rh, rw)."""
+    spatial = [SAxis("c", C, c_levels), SAxis("h", H, h_levels), SAxis("w", W, w_levels)]
+    red = [RAxis("rh", R, 0), RAxis("rw", S, 0)]
+    inp = Buffer("In", [[("c", 1)], [("h", stride), ("rh", 1)], [("w", stride), ("rw", 1)]])
+    wt = Buffer("Wt", [[("c", 1)], [("rh", 1)], [("rw", 1)]])
+    return ProgramSpec(name, spatial, red, [inp, wt], bias=bias, relu=relu, bias_axis="c")
+
+
 def softmax_spec(name: str, B: int, N: int, M: int, *, i_levels="vti", j_vars=1) -> ProgramSpec:
     """Softmax's reduction stage over the last axis, O[b, i] += exp(A[b, i, j]) (BERT attention scores,
     batch x heads folded into b; the operator mix of Fig. 9).  The normalisation stage is an

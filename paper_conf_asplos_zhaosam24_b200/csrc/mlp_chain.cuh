@@ -330,7 +330,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
           if (L.epi != EPI_F32T) {          // the epilogue will stage this tile's bn / 64 chunks
             prev_chunk_base = chunk_count;
             chunk_count += L.bn / 64;
-            ++staged_tiles;
+            // own_bar completes one phase per tile whose chunks the NEXT layer reuses (every arrive is waited on)
+            if (dataflow && l + 1 < P.n_layers && P.layer[l + 1].reuse) ++staged_tiles;
           }
         }
       }
@@ -360,6 +361,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       float* __restrict__ out_f32 = L.args.out_f32;
       const CUtensorMap* tm_c_hi = &L.c_hi;
       const CUtensorMap* tm_c_lo = &L.c_lo;
+      const bool next_reuse = dataflow && l + 1 < P.n_layers && P.layer[l + 1].reuse;
       // stage this layer's bias / head row in smem while the MMA warp works (previous layer's
       // readers are past the layer-end barrier, so the buffer is free)
       if (epi == EPI_RELU || epi == EPI_HEAD) {
@@ -491,7 +493,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
                 ptx::bulk_s2g(mask_out + static_cast<size_t>((n0 + c64) / 32 + 1) * ld_mask + m0, s_mask + (ebuf * 2 + 1) * GEMM_BM, GEMM_BM * 4);
               }
               ptx::bulk_commit();
-              if (c64 + 64 >= bn) ptx::mbar_arrive(own_bar);   // all chunks of the tile staged (reuse, next layer)
+              if (c64 + 64 >= bn && next_reuse) ptx::mbar_arrive(own_bar);   // all chunks staged, the next layer reuses them
             }
           }
         }

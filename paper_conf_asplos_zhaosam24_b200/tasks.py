@@ -136,7 +136,7 @@ def plan(n_tasks: int, n_seeds: int, world: int, mode: str, costs: Sequence[floa
 
 def config_mode(name: str) -> str:
     """C3 shards by subgraph with seed-split LPT (hybrid), C4 shards every task's seeds."""
-    return {"C3": "hybrid", "C4": "seeds"}.get(name, "seeds")
+    return {"C3": "hybrid", "MBV2": "hybrid", "C4": "seeds"}.get(name, "seeds")
 
 
 # ----------------------------------------------------------------------------- top-k records

@@ -12,7 +12,7 @@ import pytest
 import torch
 
 import felix_inputs as fi
-from felix_inputs.programs import build_space, conv2d_spec, dense_spec, layernorm_spec, softmax_spec
+from felix_inputs.programs import build_space, conv2d_spec, dense_spec, depthwise_conv2d_spec, layernorm_spec, softmax_spec
 from oracle import felix_oracle as fo
 from tests.sim.loopnest import enumerate_valid, simulate, simulate_epilogue
 
@@ -26,6 +26,7 @@ TINY_SPECS = [
     conv2d_spec("tiny_conv3x3_s2", 2, 3, 3, 2, 3, 3, 2, rc_vars=1),
     softmax_spec("tiny_softmax", 2, 4, 8, j_vars=1),
     layernorm_spec("tiny_layernorm", 4, 8, j_vars=2),
+    depthwise_conv2d_spec("tiny_dwconv3x3_s2", 4, 3, 3, 3, 3, 2),
 ]
 
 
