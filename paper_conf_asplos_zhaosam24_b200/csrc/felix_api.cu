@@ -139,6 +139,7 @@ struct Tuning {
   std::atomic<int> chunks{-1};       // concurrent population chunks
   std::atomic<int> sc{-1};           // split-cone reverse kernel (1) or cone-group kernel (0)
   std::atomic<int> tile_cg{-1};      // tile kernel: 1-SM tiles (1) or 2-SM cta_group::2 pairs (2)
+  std::atomic<int> chain_cg{-1};     // layer chain: 1-SM tiles (1) or 2-SM cta_group::2 pairs (2)
   std::atomic<int> codegen_P{-1}, codegen_R{-1};   // felix_codegen's variant
   std::atomic<int> trace{0};         // per-block %globaltimer stamps in kernels generated afterwards
 };
@@ -156,6 +157,7 @@ struct Plan {
   std::vector<GemmLaunch> gemms;           // per-layer kernels (FELIX_MLP=layers)
   ChainParams chain{};                     // persistent all-layer kernel
   int chain_grid = 0;
+  int chain_cg = 1;                        // 2: 2-SM cta_group::2 pairs (256-row tiles, weights split along N)
   DevBuf grid_bar;
   DevBuf chain_flags;                      // dataflow chain: per (layer, row block) completion counters
   bool tile_ok = false;                    // model has the shape mlp_tile_kernel is specialised for
@@ -203,19 +205,26 @@ static void launch_tile(const Plan& p, cudaStream_t st) {
 }
 
 static void launch_chain(const Plan& p, cudaStream_t st) {
-  set_smem_attr(reinterpret_cast<const void*>(mlp_chain_kernel<1>), CHAIN_SMEM_BYTES);
-  cudaLaunchAttribute attrs[2];
+  const bool cg2 = p.chain_cg == 2;
+  set_smem_attr(cg2 ? reinterpret_cast<const void*>(mlp_chain_kernel<2>) : reinterpret_cast<const void*>(mlp_chain_kernel<1>),
+                CHAIN_SMEM_BYTES);
+  cudaLaunchAttribute attrs[3];
   attrs[0] = g_pdl_attr;
   attrs[1].id = cudaLaunchAttributeCooperative;   // the dataflow flags need every CTA resident
   attrs[1].val.cooperative = 1;
+  attrs[2].id = cudaLaunchAttributeClusterDimension;
+  attrs[2].val.clusterDim.x = 2;
+  attrs[2].val.clusterDim.y = 1;
+  attrs[2].val.clusterDim.z = 1;
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(static_cast<unsigned>(p.chain_grid));
   cfg.blockDim = dim3(CHAIN_THREADS);
   cfg.dynamicSmemBytes = CHAIN_SMEM_BYTES;
   cfg.stream = st;
   cfg.attrs = attrs;
-  cfg.numAttrs = 2;
-  CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_chain_kernel<1>, p.chain));
+  cfg.numAttrs = cg2 ? 3 : 2;
+  if (cg2) CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_chain_kernel<2>, p.chain));
+  else CUDA_OK(cudaLaunchKernelEx(&cfg, mlp_chain_kernel<1>, p.chain));
 }
 
 // The population split into K independent chunks, each with its own workspace (Plan).  One Adam
@@ -590,7 +599,10 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
   auto p = std::make_unique<Plan>();
   p->cm = cm;
   p->n = n;
-  p->n_pad = (n + 127) / 128 * 128;
+  // 2-SM chain pairs: rows padded to whole 256-row pairs (the OOB rows are zero-filled by TMA and
+  // clipped on store; every row-block flag exists)
+  p->chain_cg = g_tune.chain_cg.load() == 2 ? 2 : 1;
+  p->n_pad = (n + 128 * p->chain_cg - 1) / (128 * p->chain_cg) * (128 * p->chain_cg);
   const int L = cm->n_layers;
   const auto& d = cm->dims;
   const int64_t np = p->n_pad;
@@ -712,10 +724,11 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     L.bn = bn;
     L.n_tiles_n = N / bn;
     L.n_tiles = static_cast<int>(mt) * L.n_tiles_n;
-    L.idesc = ptx::idesc_f16_f32(GEMM_BM, static_cast<uint32_t>(bn));
+    const int ccg = p->chain_cg;
+    L.idesc = ptx::idesc_f16_f32(GEMM_BM * ccg, static_cast<uint32_t>(bn));
     L.a_hi = g.a_hi; L.a_lo = g.a_lo; L.c_hi = g.c_hi; L.c_lo = g.c_lo;
-    L.b_hi = make_tmap(g.w_hi, N, g.args.K, bn);
-    L.b_lo = make_tmap(g.w_lo, N, g.args.K, bn);
+    L.b_hi = make_tmap(g.w_hi, N, g.args.K, bn / ccg);     // CG = 2: each CTA loads half of the tile's weight rows
+    L.b_lo = make_tmap(g.w_lo, N, g.args.K, bn / ccg);
     // the first backward layer takes the 0/1 mask of the head layer as its A operand and the head row
     // folded into its weights (exact A: two MMA passes, no A lo loads); FELIX_MASK_EXACT=0 disables
     L.a_exact = 0;
@@ -723,13 +736,13 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     if (i == static_cast<size_t>(cm->n_layers - 1) && i > 0 && p->gemms[i - 1].epi == EPI_HEAD) {
       L.a_exact = 1;
       p->chain.layer[i - 1].head_exact = 1;
-      L.b_hi = make_tmap(cm->WTs_hi.p, N, g.args.K, bn);
-      L.b_lo = make_tmap(cm->WTs_lo.p, N, g.args.K, bn);
+      L.b_hi = make_tmap(cm->WTs_hi.p, N, g.args.K, bn / ccg);
+      L.b_lo = make_tmap(cm->WTs_lo.p, N, g.args.K, bn / ccg);
     }
     if (g.epi == EPI_HEAD && use_chain()) p->n_head_tiles = 2 * (N / bn);   // chain: one partial per column half
-    max_tiles = std::max(max_tiles, L.n_tiles);
+    max_tiles = std::max(max_tiles, static_cast<int>((mt + ccg - 1) / ccg) * L.n_tiles_n * ccg);   // CTAs the layer can use
   }
-  p->chain_grid = std::min(sms, max_tiles);
+  p->chain_grid = std::min(sms / p->chain_cg * p->chain_cg, max_tiles);
   // Grid chain with per-row-block dataflow flags (cooperative launch: every CTA resident): at C2 44.2 us
   // per Adam step vs 45.7 us for a cluster chain (one 4-CTA cluster per row block, cluster barriers; removed)
   // and faster above 37 row blocks (n=8192: 56 vs 90 us).  The epoch is the step counter the forward DAG
@@ -746,7 +759,10 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
       Li.reuse = 0;
       if (!reuse_ok || i == 0) continue;
       const ChainLayer& Lp = p->chain.layer[i - 1];
-      if (Lp.epi != EPI_F32T && Lp.n_tiles <= p->chain_grid && Li.n_tiles <= p->chain_grid &&
+      // every CTA (pair) has at most one tile of each of the two layers and the same N tile in both
+      const int64_t units_p = (mt + p->chain_cg - 1) / p->chain_cg * Lp.n_tiles_n, units_i = (mt + p->chain_cg - 1) / p->chain_cg * Li.n_tiles_n;
+      const int64_t clusters = p->chain_grid / p->chain_cg;
+      if (Lp.epi != EPI_F32T && units_p <= clusters && units_i <= clusters &&
           Lp.n_tiles_n == Li.n_tiles_n && Lp.bn % GEMM_BK == 0)
         Li.reuse = 1;
     }
@@ -1996,6 +2012,7 @@ felix_status felix_tune(const char* key, int32_t value) {
   else if (k == "chunks") { if (value != -1 && (value < 1 || value > 16)) in({}); g_tune.chunks = value; }
   else if (k == "split_cone") { in({-1, 0, 1}); g_tune.sc = value; }
   else if (k == "tile_cta_group") { in({-1, 1, 2}); g_tune.tile_cg = value; }
+  else if (k == "chain_cta_group") { in({-1, 1, 2}); g_tune.chain_cg = value; }
   else if (k == "codegen_cone_width") { in({-1, 1, 2, 4, 8, 16}); g_tune.codegen_P = value; }
   else if (k == "codegen_replicas") { in({-1, 1, 2, 4}); g_tune.codegen_R = value; }
   else if (k == "trace") { in({0, 1}); g_tune.trace = value; }

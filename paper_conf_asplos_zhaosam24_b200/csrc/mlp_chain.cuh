@@ -14,6 +14,16 @@
 // 64-column chunk into two 32-column halves (two warps per SM sub-partition hide the latency of
 // the convert/split chains).  TMEM holds two 128-column accumulators so the epilogue of tile i
 // overlaps the MMAs of tile i+1.
+//
+// CG = 2 (2-SM pairs, tcgen05 cta_group::2): a cluster of two CTAs computes 256-row x bn tiles (rows
+// 256p + 128 rank ...); each CTA loads its own 128 A rows and HALF of the tile's weight rows (B split
+// along N), the leader issues M=256 MMAs that read A and B from both CTAs' shared memory, and each
+// CTA's TMEM receives the 128 x bn accumulator of its own rows.  Per SM the weight bytes of a tile
+// halve (C2: 1376 -> 1128 KB ingested per Adam step); every epilogue, flag and own-chunk reuse stays
+// per CTA (its own 128-row block), exactly as with CG = 1.  TMA loads of both CTAs complete on the
+// leader's full barrier (armed by the leader with both CTAs' bytes); MMA commits are multicast to both
+// CTAs' empty / accumulator-ready barriers; the epilogues of both CTAs arrive on the leader's
+// accumulator-drained and own-chunk barriers.
 #pragma once
 #include <cstdint>
 #include <cuda_fp16.h>
@@ -66,7 +76,7 @@ struct ChainParams {
   int m_tiles;
   unsigned int* grid_bar;              // monotonic arrival counter (never reset)
   unsigned long long* trace;           // debug: [grid][layers][8] globaltimer stamps (FELIX_CHAIN_TRACE)
-  // Dataflow mode (CS == 1, flags != nullptr): no grid barrier.  flags[(l * m_tiles + m) * 8] counts the
+  // Dataflow mode (flags != nullptr): no grid barrier.  flags[(l * m_tiles + m) * 8] counts the
   // layer-l tiles of row block m whose outputs are complete (release); a layer-(l+1) tile of row block m
   // waits (acquire) until it reaches epoch * n_tiles_n(l).  Counters only grow during a search; *epoch
   // is the launch's 1-based sequence number (the forward DAG kernel's step counter, or 1 after a reset).
@@ -109,46 +119,21 @@ __device__ __forceinline__ void grid_barrier(unsigned int* ctr, unsigned int nbl
   asm volatile("fence.proxy.async.global;" ::: "memory");
 }
 
-// Tiles of one layer owned by this CTA.  CS == 1: tile = blockIdx.x, +gridDim.x, ... over all
-// (row block, N tile) pairs, layers separated by a grid-wide barrier.  CS > 1 (cluster chain): CTA rank
-// r of cluster c computes N tiles r, r+CS, ... of row blocks c, c+#clusters, ..., so every dependency
-// between consecutive layers stays inside the cluster and the layer barrier is a cluster barrier.
-template <int CS>
+// Tiles of one layer owned by this CTA (pair): tile = cluster, +#clusters, ... over all (row block
+// [pair], N tile) pairs, N fastest.  CG = 1: a "pair" is one 128-row block.
+template <int CG>
 struct ChainTiles {
-  int t0, tstep, m, mstep, nt0, nt, ntn, mt;
-  __device__ ChainTiles(int n_tiles_n, int m_tiles) : ntn(n_tiles_n), mt(m_tiles) {
-    if (CS == 1) { t0 = blockIdx.x; tstep = gridDim.x; }
-    else { m = blockIdx.x / CS; mstep = gridDim.x / CS; nt0 = blockIdx.x % CS; nt = nt0; }
+  int t0, tstep, ntn, units;
+  __device__ ChainTiles(int n_tiles_n, int m_tiles) : ntn(n_tiles_n) {
+    t0 = blockIdx.x / CG;
+    tstep = gridDim.x / CG;
+    units = ((m_tiles + CG - 1) / CG) * ntn;
   }
-  // first tile (or -1), then next(tile)
-  __device__ int first() {
-    if (CS == 1) return t0 < ntn * mt ? t0 : -1;
-    nt = nt0;
-    return (m < mt && nt < ntn) ? m * ntn + nt : -1;
-  }
-  __device__ int next(int tile) {
-    if (CS == 1) { tile += tstep; return tile < ntn * mt ? tile : -1; }
-    int mm = tile / ntn;
-    nt += CS;
-    if (nt >= ntn) { nt = nt0; mm += mstep; }
-    return (mm < mt && nt < ntn) ? mm * ntn + nt : -1;
-  }
+  __device__ int first() const { return t0 < units ? t0 : -1; }
+  __device__ int next(int tile) const { tile += tstep; return tile < units ? tile : -1; }
 };
 
-// cluster barrier for one thread per CTA: arrive (release, cluster scope) on every CTA's layer
-// barrier, then wait on this CTA's (acquire, cluster scope); global writes of the async proxy
-// (TMA stores, completed by bulk_wait) are ordered around it with fence.proxy.async.global
-template <int CS>
-__device__ __forceinline__ void cluster_layer_barrier(uint64_t* bar, uint32_t phase) {
-  asm volatile("fence.proxy.async.global;" ::: "memory");
-  const uint32_t a = ptx::smem_u32(bar);
-#pragma unroll
-  for (int r = 0; r < CS; ++r) ptx::mbar_arrive_cluster(ptx::mapa_shared(a, r));
-  ptx::mbar_wait_cluster(bar, phase & 1u);
-  asm volatile("fence.proxy.async.global;" ::: "memory");
-}
-
-template <int CS>
+template <int CG>
 __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __grid_constant__ ChainParams P) {
   extern __shared__ uint8_t smem_raw[];
   // 1024-B alignment by offsetting the shared array itself (a round trip through uintptr_t would turn
@@ -165,11 +150,11 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
   uint64_t* tempty = tfull + 2;                    // [2] accumulator drained
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
   uint32_t* gen_slot = tmem_slot + 1;              // layers completed grid-wide (producer handshake)
-  uint64_t* cl_bar = tempty + 3;                   // cluster layer barrier (CS > 1), 8-byte aligned
   uint64_t* own_bar = tempty + 4;                  // epilogue -> MMA: a tile's output chunks are staged
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned int G = gridDim.x;
+  const uint32_t rank = CG == 2 ? ptx::cluster_ctarank() : 0u;
 
   auto a_hi = [&](int s) { return smem + s * CHAIN_STAGE_BYTES; };
   auto a_lo = [&](int s) { return smem + s * CHAIN_STAGE_BYTES + CHAIN_A_BYTES; };
@@ -178,28 +163,49 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
 
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < CHAIN_STAGES; ++s) { ptx::mbar_init(&full_bar[s], 1); ptx::mbar_init(&empty_bar[s], 1); }
-    for (int a = 0; a < 2; ++a) { ptx::mbar_init(&tfull[a], 1); ptx::mbar_init(&tempty[a], CHAIN_EPI_WARPS); }
-    if (CS > 1) ptx::mbar_init(cl_bar, CS);
-    ptx::mbar_init(own_bar, 1);
+    for (int a = 0; a < 2; ++a) { ptx::mbar_init(&tfull[a], 1); ptx::mbar_init(&tempty[a], CHAIN_EPI_WARPS * CG); }
+    ptx::mbar_init(own_bar, CG);
     *gen_slot = 0;
     ptx::fence_barrier_init();
   }
-  if (warp == 1) ptx::tmem_alloc(tmem_slot, 2 * CHAIN_BN_MAX);
+  if (warp == 1) {
+    if constexpr (CG == 2) ptx::tmem_alloc_cg2(tmem_slot, 2 * CHAIN_BN_MAX);
+    else ptx::tmem_alloc(tmem_slot, 2 * CHAIN_BN_MAX);
+  }
   ptx::tc_fence_before();
-  if constexpr (CS > 1) ptx::cluster_sync();
+  if constexpr (CG == 2) ptx::cluster_sync();
   else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
   ptx::pdl_launch_dependents();
   ptx::pdl_wait();                                  // phi (layer-1 A operand) comes from the DAG kernel
-  const bool dataflow = CS == 1 && P.flags != nullptr;
+  const bool dataflow = P.flags != nullptr;
   const unsigned int epoch = dataflow ? static_cast<unsigned int>(*reinterpret_cast<const volatile int*>(P.epoch)) : 0u;
   auto flag_of = [&](int l, int m) { return P.flags + (static_cast<size_t>(l) * P.m_tiles + m) * CHAIN_FLAG_STRIDE; };
+  // leader-CTA copies of the barriers that receive arrivals from both CTAs (CG = 2)
+  auto leader_addr = [&](const void* p) { return ptx::mapa_shared(ptx::smem_u32(p), 0); };
+  auto arrive_leader = [&](uint64_t* bar) {
+    if constexpr (CG == 2) ptx::mbar_arrive_cluster(leader_addr(bar));
+    else ptx::mbar_arrive(bar);
+  };
+  auto wait_in = [&](uint64_t* bar, uint32_t parity) {   // barriers that receive arrivals from the peer
+    if constexpr (CG == 2) ptx::mbar_wait_cluster(bar, parity);
+    else ptx::mbar_wait(bar, parity);
+  };
+  // this CTA's 128-row block of pair tile `tile`
+  auto row_block = [&](int tile, int ntn) { return (tile / ntn) * CG + static_cast<int>(rank); };
 
   if (warp == 0) {
     if (lane == 0) {
-      // ------------------------------------------------------------ TMA producer
+      // ------------------------------------------------------------ TMA producer (both CTAs)
       int it = 0;                                   // running k-block counter (ring position)
+      auto load = [&](void* dst, const CUtensorMap* m, int c0, int c1, int s) {
+        if constexpr (CG == 2) ptx::tma_load_2d_cg2(dst, m, c0, c1, leader_addr(&full_bar[s]));
+        else ptx::tma_load_2d(dst, m, c0, c1, &full_bar[s]);
+      };
+      auto arm = [&](int s, uint32_t bytes_per_cta) {   // the leader expects both CTAs' bytes
+        if (rank == 0) ptx::mbar_arrive_expect_tx(&full_bar[s], bytes_per_cta * CG);
+      };
       for (int l = 0; l < P.n_layers; ++l) {
         const ChainLayer& L = P.layer[l];
         if (l > 0 && !dataflow) {
@@ -213,33 +219,35 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         }
         CHAIN_STAMP(l, 0);
         const int nkb = (L.args.K + GEMM_BK - 1) / GEMM_BK;
-        const uint32_t tx = (L.a_exact ? 1 : 2) * CHAIN_A_BYTES + 2 * (L.bn * GEMM_BK * 2);
-        ChainTiles<CS> tiles(L.n_tiles_n, P.m_tiles);
+        const int bnc = L.bn / CG;                                  // weight rows this CTA loads per tile
+        const uint32_t tx_b = 2 * (bnc * GEMM_BK * 2);
+        const uint32_t tx = (L.a_exact ? 1 : 2) * CHAIN_A_BYTES + tx_b;
+        ChainTiles<CG> tiles(L.n_tiles_n, P.m_tiles);
         for (int tile = tiles.first(); tile >= 0; tile = tiles.next(tile)) {
-          const int m0 = (tile / L.n_tiles_n) * GEMM_BM, n0 = (tile % L.n_tiles_n) * L.bn;
+          const int mb = row_block(tile, L.n_tiles_n);
+          const int m0 = mb * GEMM_BM, n0 = (tile % L.n_tiles_n) * L.bn, nb = n0 + static_cast<int>(rank) * bnc;
           int kb0 = 0;
           if (dataflow && l > 0 && L.reuse) {
             // own K blocks (B only) first, then the others (B, row-block flag once, A)
             const ChainLayer& Lp = P.layer[l - 1];
             const int own0 = (tile % Lp.n_tiles_n) * Lp.bn / GEMM_BK, nown = Lp.bn / GEMM_BK;
-            const uint32_t tx_b = 2 * (L.bn * GEMM_BK * 2);
             bool flag_ok = false;
             for (int i = 0; i < nkb; ++i, ++it) {
               const int kb = i < nown ? own0 + i : (i - nown < own0 ? i - nown : i);
               const bool own = i < nown;
               const int s = it % CHAIN_STAGES;
               if (it >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], ((it / CHAIN_STAGES) - 1) & 1);
-              ptx::mbar_arrive_expect_tx(&full_bar[s], own ? tx_b : tx);   // tx counts A lo only when loaded
-              ptx::tma_load_2d(b_hi(s), &L.b_hi, kb * GEMM_BK, n0, &full_bar[s]);
-              ptx::tma_load_2d(b_lo(s), &L.b_lo, kb * GEMM_BK, n0, &full_bar[s]);
+              arm(s, own ? tx_b : tx);
+              load(b_hi(s), &L.b_hi, kb * GEMM_BK, nb, s);
+              load(b_lo(s), &L.b_lo, kb * GEMM_BK, nb, s);
               if (!own) {
                 if (!flag_ok) {
-                  flag_wait(flag_of(l - 1, m0 / GEMM_BM), epoch * static_cast<unsigned int>(Lp.n_tiles_n));
+                  flag_wait(flag_of(l - 1, mb), epoch * static_cast<unsigned int>(Lp.n_tiles_n));
                   asm volatile("fence.proxy.async.global;" ::: "memory");
                   flag_ok = true;
                 }
-                ptx::tma_load_2d(a_hi(s), &L.a_hi, kb * GEMM_BK, m0, &full_bar[s]);
-                if (!L.a_exact) ptx::tma_load_2d(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, &full_bar[s]);
+                load(a_hi(s), &L.a_hi, kb * GEMM_BK, m0, s);
+                if (!L.a_exact) load(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, s);
               }
             }
             continue;
@@ -251,16 +259,16 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             for (int kb = 0; kb < pre; ++kb) {
               const int s = (it + kb) % CHAIN_STAGES;
               if (it + kb >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], (((it + kb) / CHAIN_STAGES) - 1) & 1);
-              ptx::mbar_arrive_expect_tx(&full_bar[s], tx);
-              ptx::tma_load_2d(b_hi(s), &L.b_hi, kb * GEMM_BK, n0, &full_bar[s]);
-              ptx::tma_load_2d(b_lo(s), &L.b_lo, kb * GEMM_BK, n0, &full_bar[s]);
+              arm(s, tx);
+              load(b_hi(s), &L.b_hi, kb * GEMM_BK, nb, s);
+              load(b_lo(s), &L.b_lo, kb * GEMM_BK, nb, s);
             }
-            flag_wait(flag_of(l - 1, m0 / GEMM_BM), epoch * static_cast<unsigned int>(P.layer[l - 1].n_tiles_n));
+            flag_wait(flag_of(l - 1, mb), epoch * static_cast<unsigned int>(P.layer[l - 1].n_tiles_n));
             asm volatile("fence.proxy.async.global;" ::: "memory");
             for (int kb = 0; kb < pre; ++kb) {
               const int s = (it + kb) % CHAIN_STAGES;
-              ptx::tma_load_2d(a_hi(s), &L.a_hi, kb * GEMM_BK, m0, &full_bar[s]);
-              if (!L.a_exact) ptx::tma_load_2d(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, &full_bar[s]);
+              load(a_hi(s), &L.a_hi, kb * GEMM_BK, m0, s);
+              if (!L.a_exact) load(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, s);
             }
             kb0 = pre;
             it += pre;
@@ -268,28 +276,28 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
           for (int kb = kb0; kb < nkb; ++kb, ++it) {
             const int s = it % CHAIN_STAGES;
             if (it >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], ((it / CHAIN_STAGES) - 1) & 1);
-            ptx::mbar_arrive_expect_tx(&full_bar[s], tx);
+            arm(s, tx);
             const int k0 = kb * GEMM_BK;
-            ptx::tma_load_2d(a_hi(s), &L.a_hi, k0, m0, &full_bar[s]);
-            if (!L.a_exact) ptx::tma_load_2d(a_lo(s), &L.a_lo, k0, m0, &full_bar[s]);
-            ptx::tma_load_2d(b_hi(s), &L.b_hi, k0, n0, &full_bar[s]);
-            ptx::tma_load_2d(b_lo(s), &L.b_lo, k0, n0, &full_bar[s]);
+            load(a_hi(s), &L.a_hi, k0, m0, s);
+            if (!L.a_exact) load(a_lo(s), &L.a_lo, k0, m0, s);
+            load(b_hi(s), &L.b_hi, k0, nb, s);
+            load(b_lo(s), &L.b_lo, k0, nb, s);
           }
         }
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
-      // ------------------------------------------------------------ MMA issuer
+    if (lane == 0 && rank == 0) {
+      // ------------------------------------------------------------ MMA issuer (leader CTA)
       int it = 0, tcount = 0;
       int staged_tiles = 0, chunk_count = 0, prev_chunk_base = 0;   // mirror of the epilogue's staging sequence
       for (int l = 0; l < P.n_layers; ++l) {
         const ChainLayer& L = P.layer[l];
         const int nkb = (L.args.K + GEMM_BK - 1) / GEMM_BK;
-        ChainTiles<CS> tiles(L.n_tiles_n, P.m_tiles);
+        ChainTiles<CG> tiles(L.n_tiles_n, P.m_tiles);
         for (int tile = tiles.first(); tile >= 0; tile = tiles.next(tile), ++tcount) {
           const int acc = tcount & 1;
-          if (tcount >= 2) ptx::mbar_wait(&tempty[acc], ((tcount >> 1) - 1) & 1);
+          if (tcount >= 2) wait_in(&tempty[acc], ((tcount >> 1) - 1) & 1);
           ptx::tc_fence_after();
           const uint32_t d = tmem_base + acc * CHAIN_BN_MAX;
           const bool reuse = dataflow && l > 0 && L.reuse;
@@ -299,13 +307,14 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             const ChainLayer& Lp = P.layer[l - 1];
             own0 = (tile % Lp.n_tiles_n) * Lp.bn / GEMM_BK;
             nown = Lp.bn / GEMM_BK;
-            // the previous tile's chunks are staged and fenced for the async proxy
-            ptx::mbar_wait(own_bar, (staged_tiles - 1) & 1);
+            // the previous tile's chunks are staged (in both CTAs) and fenced for the async proxy
+            wait_in(own_bar, (staged_tiles - 1) & 1);
           }
           for (int i = 0; i < nkb; ++i, ++it) {
             const int kb = !reuse ? i : (i < nown ? own0 + i : (i - nown < own0 ? i - nown : i));
+            (void)kb;
             const int s = it % CHAIN_STAGES;
-            ptx::mbar_wait(&full_bar[s], (it / CHAIN_STAGES) & 1);
+            wait_in(&full_bar[s], (it / CHAIN_STAGES) & 1);
             if (i == 0 && tcount == 0) CHAIN_STAMP(l, 1);
             ptx::tc_fence_after();
             uint32_t ah = ptx::smem_u32(a_hi(s)), al = ptx::smem_u32(a_lo(s));
@@ -319,13 +328,21 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             for (int kk = 0; kk < GEMM_BK / GEMM_UMMA_K; ++kk) {
               const uint32_t off = kk * GEMM_UMMA_K * 2;
               const uint32_t acc0 = (i | kk) != 0;
-              if (!a_exact) ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(al + off), ptx::sdesc_k_sw128(bh + off), L.idesc, acc0);
-              ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bl + off), L.idesc, a_exact ? acc0 : 1u);
-              ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bh + off), L.idesc, 1u);
+              if constexpr (CG == 2) {
+                if (!a_exact) ptx::mma_f16_ss_cg2(d, ptx::sdesc_k_sw128(al + off), ptx::sdesc_k_sw128(bh + off), L.idesc, acc0);
+                ptx::mma_f16_ss_cg2(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bl + off), L.idesc, a_exact ? acc0 : 1u);
+                ptx::mma_f16_ss_cg2(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bh + off), L.idesc, 1u);
+              } else {
+                if (!a_exact) ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(al + off), ptx::sdesc_k_sw128(bh + off), L.idesc, acc0);
+                ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bl + off), L.idesc, a_exact ? acc0 : 1u);
+                ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bh + off), L.idesc, 1u);
+              }
             }
-            ptx::mma_commit(&empty_bar[s]);
+            if constexpr (CG == 2) ptx::mma_commit_mc(&empty_bar[s], 0x3);
+            else ptx::mma_commit(&empty_bar[s]);
           }
-          ptx::mma_commit(&tfull[acc]);
+          if constexpr (CG == 2) ptx::mma_commit_mc(&tfull[acc], 0x3);
+          else ptx::mma_commit(&tfull[acc]);
           CHAIN_STAMP(l, 2);
           if (L.epi != EPI_F32T) {          // the epilogue will stage this tile's bn / 64 chunks
             prev_chunk_base = chunk_count;
@@ -337,7 +354,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       }
     }
   } else {
-    // ------------------------------------------------------------ epilogue warps 2..9
+    // ------------------------------------------------------------ epilogue warps 2..9 (both CTAs)
     const int q = warp & 3;                          // TMEM lane quadrant this warp may access
     const int half = (warp - 2) >> 2;                // which 32-column half of each 64-column chunk
     const int r_tile = q * 32 + lane;
@@ -351,7 +368,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       // compiler otherwise re-fetches each pointer (LDC) before every element access
       const int epi = L.epi, bn = L.bn, ntn = L.n_tiles_n;
       const bool hexact = L.head_exact != 0;   // HEAD: write the 0/1 mask (the next layer's weights carry -w)
-      const int aM = L.args.M, aN = L.args.N, n_valid = L.args.n_valid, ld_f32 = L.args.ld_f32, ld_c = L.args.ld_c;
+      const int aM = L.args.M, n_valid = L.args.n_valid, ld_f32 = L.args.ld_f32, ld_c = L.args.ld_c;
+      const int aN = L.args.N;
       const int ld_mask = L.args.ld_mask;
       const float* __restrict__ bias = L.args.bias;
       const float* __restrict__ head_w = L.args.head_w;
@@ -371,11 +389,12 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         }
       }
       ptx::named_bar_sync(1, NEPI);
-      ChainTiles<CS> tiles(ntn, P.m_tiles);
-      int first_tile = tiles.first();
+      ChainTiles<CG> tiles(ntn, P.m_tiles);
+      const int first_tile = tiles.first();
       for (int tile = first_tile; tile >= 0; tile = tiles.next(tile), ++tcount) {
         const int acc = tcount & 1;
-        const int m0 = (tile / ntn) * GEMM_BM, n0 = (tile % ntn) * bn;
+        const int mb = row_block(tile, ntn);
+        const int m0 = mb * GEMM_BM, n0 = (tile % ntn) * bn;
         const int row = m0 + r_tile;
         const bool row_ok = row < aM;
         // this thread's mask words for the tile (<= 2 chunks of 64 columns), requested before the wait
@@ -383,7 +402,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         if (dataflow && epi == EPI_MASK) {
           // the mask words come from an earlier layer of this row block (other CTAs): acquire the
           // row block's flag of the previous layer first (the epilogue warps are idle in the mainloop)
-          if (etid == 0) flag_wait(flag_of(l - 1, m0 / GEMM_BM), epoch * static_cast<unsigned int>(P.layer[l - 1].n_tiles_n));
+          if (etid == 0) flag_wait(flag_of(l - 1, mb), epoch * static_cast<unsigned int>(P.layer[l - 1].n_tiles_n));
           ptx::named_bar_sync(1, NEPI);
         }
         if (epi == EPI_MASK && row_ok) {
@@ -493,7 +512,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
                 ptx::bulk_s2g(mask_out + static_cast<size_t>((n0 + c64) / 32 + 1) * ld_mask + m0, s_mask + (ebuf * 2 + 1) * GEMM_BM, GEMM_BM * 4);
               }
               ptx::bulk_commit();
-              if (c64 + 64 >= bn && next_reuse) ptx::mbar_arrive(own_bar);   // all chunks staged, the next layer reuses them
+              if (c64 + 64 >= bn && next_reuse) arrive_leader(own_bar);   // all chunks staged, the next layer reuses them
             }
           }
         }
@@ -511,16 +530,16 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             ptx::bulk_commit();
           }
         }
-        // accumulator drained: let the MMA warp reuse it
+        // accumulator drained: let the (leader's) MMA warp reuse it
         ptx::tc_fence_before();
         __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
+        if (lane == 0) arrive_leader(&tempty[acc]);
         if (dataflow && l + 1 < P.n_layers && etid == 0) {
           // every global write of this tile (activations, mask words, head partials) was a bulk copy issued
           // by this thread: complete them, then count the tile (release)
           ptx::bulk_wait<0>();
           asm volatile("fence.proxy.async.global;" ::: "memory");
-          asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(flag_of(l, m0 / GEMM_BM)) : "memory");
+          asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(flag_of(l, mb)) : "memory");
         }
       }
       // ---- layer end: all of this CTA's outputs complete + visible, then the grid barrier
@@ -531,8 +550,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         ptx::named_bar_sync(1, NEPI);
         if (etid == 0) {
           CHAIN_STAMP(l, 5);
-          if constexpr (CS > 1) cluster_layer_barrier<CS>(cl_bar, static_cast<uint32_t>(l));
-          else grid_barrier(P.grid_bar, G);
+          grid_barrier(P.grid_bar, G);
           CHAIN_STAMP(l, 6);
           // publish "layer l done everywhere" to the producer warp of this CTA
           asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" :: "r"(ptx::smem_u32(gen_slot)), "r"(static_cast<unsigned int>(l + 1)) : "memory");
@@ -542,9 +560,12 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
     if (etid == 0) ptx::bulk_wait<0>();
   }
   ptx::tc_fence_before();
-  if constexpr (CS > 1) ptx::cluster_sync();
+  if constexpr (CG == 2) ptx::cluster_sync();
   else __syncthreads();
-  if (warp == 1) ptx::tmem_dealloc(tmem_base, 2 * CHAIN_BN_MAX);
+  if (warp == 1) {
+    if constexpr (CG == 2) ptx::tmem_dealloc_cg2(tmem_base, 2 * CHAIN_BN_MAX);
+    else ptx::tmem_dealloc(tmem_base, 2 * CHAIN_BN_MAX);
+  }
 }
 
 }  // namespace felix

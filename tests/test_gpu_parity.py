@@ -310,7 +310,7 @@ def test_shape_errors(fx):
     del bad
 
 
-@pytest.mark.parametrize("mode,cg", [("chain", 1), ("layers", 1), ("tile", 2)])
+@pytest.mark.parametrize("mode,cg", [("chain", 1), ("chain", 2), ("layers", 1), ("tile", 2)])
 def test_mlp_execution_modes_agree(fx, mode, cg):
     """The tile-local fused MLP (1-SM and 2-SM cta_group::2 variants), the persistent chain (dataflow
     flags) and the per-layer kernels compute the same split-fp16 products in the same K order: cost and
@@ -323,7 +323,7 @@ def test_mlp_execution_modes_agree(fx, mode, cg):
     cm = fx.CostModel.from_weights(mlp)
     with fx.tuned(mlp="tile", tile_cta_group=1):
         base = fx.Space(sp).eval(cm, y0, lam=1.0)
-    with fx.tuned(mlp=mode, tile_cta_group=cg):
+    with fx.tuned(mlp=mode, tile_cta_group=cg, chain_cta_group=cg):
         other = fx.Space(sp).eval(cm, y0, lam=1.0)
     for key in ("cost", "grad"):
         a, b = base[key].cpu().numpy(), other[key].cpu().numpy()
