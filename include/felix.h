@@ -283,7 +283,8 @@ FELIX_EXPORT felix_status felix_profile_reset(felix_space* s);
  * after felix_tune("trace", 1)): uint64 [2][8192][8] = {forward, reverse} x block x stamp.  Forward
  * (felix_fwd / felix_fwd_adam): start, after griddepcontrol.wait, after the Adam prologue, after the cone
  * compute, end.  Split-cone reverse: start, after wait, after compute, end; cone-group reverse: slots
- * 4..7.  Only the last launch's stamps survive.  n_words bounds the copy. */
+ * 4..7.  If n_words exceeds 2 * 8192 * 8, the forward kernel's per-warp cone-end stamps [8192][16] follow.
+ * Only the last launch's stamps survive.  n_words bounds the copy. */
 FELIX_EXPORT felix_status felix_debug_trace(felix_space* s, uint64_t* out, int64_t n_words);
 
 #ifdef __cplusplus

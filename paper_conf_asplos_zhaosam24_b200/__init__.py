@@ -393,11 +393,13 @@ class Space:
     def profile_reset(self) -> None:
         _check(_lib.felix_profile_reset(self._h))
 
-    def debug_trace(self) -> np.ndarray:
-        """uint64 [2][8192][8] globaltimer stamps (kernels generated after tune(trace=1))."""
-        out = np.zeros((2, 8192, 8), dtype=np.uint64)
+    def debug_trace(self, warps: bool = False):
+        """uint64 [2][8192][8] globaltimer stamps (kernels generated after tune(trace=1)); warps=True also
+        returns the forward kernel's per-warp cone-end stamps [8192][16]."""
+        out = np.zeros(2 * 8192 * 8 + (8192 * 16 if warps else 0), dtype=np.uint64)
         _check(_lib.felix_debug_trace(self._h, out.ctypes.data_as(_P), ctypes.c_int64(out.size)))
-        return out
+        tr = out[:2 * 8192 * 8].reshape(2, 8192, 8)
+        return (tr, out[2 * 8192 * 8:].reshape(8192, 16)) if warps else tr
 
     def _check_y(self, y) -> None:
         import torch

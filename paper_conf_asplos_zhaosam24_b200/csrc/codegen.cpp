@@ -131,17 +131,24 @@ int arity(int op) {
   }
 }
 
-// relative cost of a node in the fast-math forward + reverse (balances the cone partition)
+// relative cost of a node in the search forward (FP64 values, FP32 smooth-step tails; SASS instructions of
+// the emitted code, which is what the warps of a cone-group block wait on at their barrier): balances
+// the cone partition.  A feature root adds kSlogCost (slog + shared-memory store).
 int node_cost(int op) {
   switch (op) {
     case FELIX_OP_CONST: case FELIX_OP_VAR: return 0;
-    case FELIX_OP_MIN: case FELIX_OP_MAX: case FELIX_OP_GT: case FELIX_OP_GE: case FELIX_OP_LT: case FELIX_OP_LE: return 14;
-    case FELIX_OP_EQ: case FELIX_OP_NE: return 28;
-    case FELIX_OP_DIV: case FELIX_OP_FLOORDIV: case FELIX_OP_CEILDIV: return 8;
-    case FELIX_OP_EXP: case FELIX_OP_LOG: case FELIX_OP_POW: case FELIX_OP_SQRT: return 24;
-    default: return 2;
+    case FELIX_OP_GT: case FELIX_OP_GE: case FELIX_OP_LT: case FELIX_OP_LE: return 12;
+    case FELIX_OP_EQ: case FELIX_OP_NE: return 26;
+    case FELIX_OP_MIN: case FELIX_OP_MAX: return 18;
+    case FELIX_OP_DIV: case FELIX_OP_FLOORDIV: case FELIX_OP_CEILDIV: return 7;
+    case FELIX_OP_SQRT: return 8;
+    case FELIX_OP_EXP: case FELIX_OP_LOG: return 40;
+    case FELIX_OP_POW: return 80;
+    case FELIX_OP_SELECT: case FELIX_OP_OR: return 3;
+    default: return 1;
   }
 }
+constexpr int kSlogCost = 10;
 
 struct Gen {
   const SpaceDesc& d;
@@ -478,7 +485,7 @@ Partition partition_roots(const Gen& g, const SpaceDesc& d, int P) {
   for (int k = 0; k < K; ++k) {
     const int r = d.froots[k];
     if (!g.depvar[r]) continue;      // constant features: group 0 writes them, no compute
-    items.push_back({true, k, r, cone_cost(r)});
+    items.push_back({true, k, r, cone_cost(r) + kSlogCost});
   }
   for (int r = 0; r < Ru; ++r) items.push_back({false, r, d.croots[r], cone_cost(d.croots[r])});
   std::stable_sort(items.begin(), items.end(), [](const Item& a, const Item& b) { return a.cost > b.cost; });
@@ -492,7 +499,7 @@ Partition partition_roots(const Gen& g, const SpaceDesc& d, int P) {
     int best = 0;
     int64_t best_total = INT64_MAX;
     for (int q = 0; q < P; ++q) {
-      int64_t add = 0;
+      int64_t add = it.is_feat ? kSlogCost : 0;
       for (int i = 0; i < g.n; ++i) if (c[i] && !in[q][i]) add += node_cost(d.nodes[i].op);
       if (gcost[q] + add < best_total) { best_total = gcost[q] + add; best = q; }
     }
@@ -527,9 +534,11 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
 
   if (trace)
     o << "__device__ unsigned long long felix_trace[2][8192][8];\n"
+         "__device__ unsigned long long felix_wtrace[8192][16];\n"
+         "#define TWSTAMP() do { if ((threadIdx.x & 31) == 0 && blockIdx.x < 8192 && (threadIdx.x >> 5) < 16) { unsigned long long t_; asm volatile(\"mov.u64 %0, %globaltimer;\" : \"=l\"(t_)); felix_wtrace[blockIdx.x][threadIdx.x >> 5] = t_; } } while (0)\n"
          "#define TSTAMP(k, s) do { if (threadIdx.x == 0 && blockIdx.x < 8192) { unsigned long long t_; asm volatile(\"mov.u64 %0, %globaltimer;\" : \"=l\"(t_)); felix_trace[k][blockIdx.x][s] = t_; } } while (0)\n";
   else
-    o << "#define TSTAMP(k, s) do {} while (0)\n";
+    o << "#define TSTAMP(k, s) do {} while (0)\n#define TWSTAMP() do {} while (0)\n";
   o << "#define NV " << M << "\n#define NF " << K << "\n#define NRU " << Ru << "\n#define NR " << R
     << "\n#define NRA " << Ra << "\n#define K0P " << K0p << "\n#define PG " << P << "\n#define NS " << NS
     << "\n#define NREP " << NREPv << "\n";
@@ -703,7 +712,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
       if (used[j]) o << "    const double x" << j << " = sx[" << j << "][lane];\n";
     g.emit_forward(fcone[q], 0, "x", "    ");
     for (int k : part.feat[q]) o << "    sphi[" << fs(k) << "][lane][" << fk(k) << "] = slogf_(v" << d.froots[k] << ");\n";
-    o << "  }\n";
+    o << "    TWSTAMP();\n  }\n";
   }
   o << "  __syncthreads();\n  TSTAMP(0, 3);\n"
     << "  // rows c0 .. c0+31 of each statement are contiguous: K0P/8 uint4 per row for hi and for lo\n"

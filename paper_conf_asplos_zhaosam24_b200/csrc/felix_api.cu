@@ -556,11 +556,13 @@ static void launch_flat(cudaKernel_t f, int64_t n, void** args, cudaStream_t st)
 // selects felix_rev_adam, 1 forces it in group searches too (measured there with an earlier variant:
 // C3 1.66e8 -> 1.65e8, C4 2.25e8 -> 2.08e8 cand-steps/s, so groups keep felix_rev_adam by default).
 // Not with history rounding (it rounds the caller's y before each step's forward, i.e. before Adam).
-static bool use_sc(bool group = false) {
+static bool use_sc(bool group = false, int64_t min_member_n = 0) {
   const int v = g_tune.sc.load();
   if (v == 0) return false;
   if (v == 1) return true;
-  return !group;
+  // groups: split-cone once every member has >= 2048 candidates (measured, FP32 reverse: C4 shards of
+  // 2048 / 4096 seeds per task +7 % / +13 %, C3 with 1024 per task -8 %)
+  return !group || min_member_n >= 2048;
 }
 __global__ void set_int_kernel(int* p, int v) { *p = v; }
 // Split-cone searches: at least two cones (measured at the C5 shard, 131072 candidates: 2.53e8 at P = 1,
@@ -771,7 +773,10 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
   p->tile_ok = L == 4 && d[1] == tile::D1 && d[2] == tile::D2 && d[3] == tile::D3 && K0p <= 128 && K0p % 32 == 0;   // K0p/2 rows: multiple of 16
   if (p->tile_ok) {
     p->tile_cg = g_tune.tile_cg.load() == 2 ? 2 : 1;
-    p->tile_full_wave = mt >= sms;
+    // measured on B200 (C2 space, default MLP): the chain wins at 64 row blocks (8192 rows: 1.24e8 vs
+    // 1.14e8 cand-steps/s), the tile kernel at 128 (16384 rows: 2.09e8 vs 1.66e8) -> tile kernel from
+    // ~56 % of a wave of 128-row tiles
+    p->tile_full_wave = mt * 16 >= static_cast<int64_t>(sms) * 9;
     const int cg = p->tile_cg;
     TileParams& t = p->tile;
     t.phi_hi = make_tmap(p->phi_hi.p, n, K0p, 128);
@@ -1498,7 +1503,9 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
   Plan& pl = *gc.plan;
   // ---- per-search state: starting points, Adam state, counters, dataflow flags
   std::vector<const felix_space::Module*> mods(G);
-  const bool sc = use_sc(true);
+  int64_t min_n = INT64_MAX;
+  for (int i = 0; i < G; ++i) min_n = std::min<int64_t>(min_n, params[i].n_seeds);
+  const bool sc = use_sc(true, min_n);
   std::vector<int> scws(G);
   for (int i = 0; i < G; ++i) {
     const int64_t n = params[i].n_seeds;
@@ -1990,7 +1997,15 @@ felix_status felix_debug_trace(felix_space* s, uint64_t* out, int64_t n_words) {
       cudaGetLastError();
       continue;
     }
-    CUDA_OK(cudaMemcpy(out, ptr, std::min<size_t>(bytes, static_cast<size_t>(n_words) * 8), cudaMemcpyDeviceToHost));
+    const size_t nb = std::min<size_t>(bytes, static_cast<size_t>(n_words) * 8);
+    CUDA_OK(cudaMemcpy(out, ptr, nb, cudaMemcpyDeviceToHost));
+    // then the per-warp cone-end stamps of the forward kernel, [8192][16], if the caller asked for them
+    void* wptr = nullptr;
+    size_t wbytes = 0;
+    if (static_cast<size_t>(n_words) * 8 > nb && cudaLibraryGetGlobal(&wptr, &wbytes, kv.second.lib, "felix_wtrace") == cudaSuccess)
+      CUDA_OK(cudaMemcpy(reinterpret_cast<char*>(out) + nb, wptr, std::min<size_t>(wbytes, static_cast<size_t>(n_words) * 8 - nb),
+                         cudaMemcpyDeviceToHost));
+    cudaGetLastError();
     return FELIX_OK;
   }
   FELIX_THROW(FELIX_E_UNSUPPORTED, "no trace buffer (felix_tune(\"trace\", 1) before the kernels are generated)");

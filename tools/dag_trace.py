@@ -21,7 +21,8 @@ y = torch.empty((sp.n_vars, n), device="cuda")
 for _ in range(3):
     space.search(cm, y, 20, rng_seed=cfg.rng_seed, init_from_y=False)
 torch.cuda.synchronize()
-tr = space.debug_trace().astype(np.int64)
+tr, wt = space.debug_trace(warps=True)
+tr, wt = tr.astype(np.int64), wt.astype(np.int64)
 f = tr[0][tr[0, :, 0] > 0]
 r = tr[1][tr[1, :, 0] > 0]
 t0 = f[:, 0].min()
@@ -35,4 +36,10 @@ out = {"config": cfg.name, "n": n, "fwd_blocks": len(f), "rev_blocks": len(r),
                                   "end": q(r[:, 3] - t0)},
        "rev_phase_us_med": {"wait": q(r[:, 1] - r[:, 0])[1], "cone": q(r[:, 2] - r[:, 1])[1], "store": q(r[:, 3] - r[:, 2])[1]},
        "span_us": round((max(f[:, 4].max(), r[:, 3].max()) - t0) / 1e3, 2)}
+# cone imbalance of the forward: per warp (cone q = warp % P of its replica), cone end - after-Adam stamp
+nb = len(f)
+w = wt[:nb]
+rel = np.where(w > 0, w - tr[0, :nb, 2][:, None], 0)
+nw = int((w[0] > 0).sum())
+out["fwd_cone_end_us_med_per_warp"] = [round(float(np.median(rel[:, k])) / 1e3, 2) for k in range(nw)]
 print(json.dumps(out))
