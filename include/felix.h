@@ -268,6 +268,8 @@ FELIX_EXPORT felix_status felix_init_sample(felix_space* s, int64_t n, uint64_t 
  *   "split_cone"          0 cone-group reverse + Adam kernel, 1 split-cone reverse kernel
  *   "tile_cta_group"      tile kernel on 1-SM tiles (1) or 2-SM cta_group::2 pairs (2)
  *   "chain_cta_group"     layer chain on 1-SM 128-row tiles (1) or 2-SM cta_group::2 256-row pairs (2)
+ *   "dphi_ksplit"         layer chain: split-K parts of the dL/dphi layer, 1, 2 or 4 (partial slabs summed
+ *                         in fixed order by the reverse kernel)
  *   "codegen_cone_width", "codegen_replicas"   the variant felix_codegen emits
  *   "trace"               0/1: per-block %globaltimer stamps in kernels generated afterwards
  * FELIX_E_INVALID_ARG for an unknown key or value. */

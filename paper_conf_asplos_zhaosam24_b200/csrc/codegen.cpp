@@ -520,8 +520,15 @@ int SpaceDesc::n_roots_total() const {
   return (int)croots.size() + n_split + (int)split_extent.size() + 2 * n_int;
 }
 
-std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, bool trace, CodegenInfo* info) {
+std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, bool trace, int dphi_parts, CodegenInfo* info) {
   Gen g(d);
+  // dL/dphi of feature row `idx`, summed over the MLP's split-K partial slabs in fixed order (compile-time
+  // unrolled: a runtime loop per seed makes NVRTC 3.5x slower on these straight-line kernels)
+  auto dphi_at = [&](const std::string& idx) {
+    std::string e = "dphi[" + idx + "]";
+    for (int pp = 1; pp < dphi_parts; ++pp) e = "(" + e + " + dphi[" + idx + " + (size_t)" + std::to_string(pp) + " * K0P * ld_dphi])";
+    return e;
+  };
   std::ostringstream& o = g.o;
   const int M = d.n_vars, K = (int)d.froots.size(), Ru = (int)d.croots.size();
   const int R = d.n_roots_total(), Ra = R - Ru;
@@ -829,8 +836,8 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     for (int j = 0; j < M; ++j) o << "    float gx" << j << " = 0.f;\n";
     for (int k : part.feat[q]) {
       const int r = d.froots[k];
-      o << "    " << g.adj(r) << " += dphi[(size_t)" << fk(k) << " * ld_dphi + (size_t)" << fs(k)
-        << " * n + ccw] * slogpf_(v" << r << ");\n";
+      o << "    " << g.adj(r) << " += " << dphi_at("(size_t)" + std::to_string(fk(k)) + " * ld_dphi + (size_t)" +
+                                                  std::to_string(fs(k)) + " * n + ccw") << " * slogpf_(v" << r << ");\n";
     }
     for (int r : part.cons[q]) {
       const int nd = d.croots[r];
@@ -949,8 +956,8 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     for (int j = 0; j < M; ++j) o << "    float gx" << j << " = 0.f;\n";
     for (int k : part.feat[q]) {
       const int r = d.froots[k];
-      o << "    " << g.adj(r) << " += dphi[(size_t)" << fk(k) << " * ld_dphi + (size_t)" << fs(k)
-        << " * n + ccw] * slogpf_(v" << r << ");\n";
+      o << "    " << g.adj(r) << " += " << dphi_at("(size_t)" + std::to_string(fk(k)) + " * ld_dphi + (size_t)" +
+                                                  std::to_string(fs(k)) + " * n + ccw") << " * slogpf_(v" << r << ");\n";
     }
     for (int r : part.cons[q]) {
       const int nd = d.croots[r];

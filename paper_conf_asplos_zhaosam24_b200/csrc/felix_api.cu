@@ -140,6 +140,7 @@ struct Tuning {
   std::atomic<int> sc{-1};           // split-cone reverse kernel (1) or cone-group kernel (0)
   std::atomic<int> tile_cg{-1};      // tile kernel: 1-SM tiles (1) or 2-SM cta_group::2 pairs (2)
   std::atomic<int> chain_cg{-1};     // layer chain: 1-SM tiles (1) or 2-SM cta_group::2 pairs (2)
+  std::atomic<int> dphi_ksplit{-1};  // layer chain: split-K parts of the dL/dphi layer (1, 2, 4)
   std::atomic<int> codegen_P{-1}, codegen_R{-1};   // felix_codegen's variant
   std::atomic<int> trace{0};         // per-block %globaltimer stamps in kernels generated afterwards
 };
@@ -152,6 +153,7 @@ struct Plan {
   DevBuf phi_hi, phi_lo;                                   // [n][K0p]
   std::vector<std::unique_ptr<DevBuf>> act_hi, act_lo, mask;  // per hidden layer l = 1..L-1
   DevBuf c_part, dphi, m, v, step_ctr;
+  int dphi_parts = 1;                      // split-K slabs of dL/dphi the reverse kernel sums (chain only)
   DevBuf sc_part, sc_pen;                                // split-cone reverse: partial adjoints, penalties
   int n_head_tiles = 0;
   std::vector<GemmLaunch> gemms;           // per-layer kernels (FELIX_MLP=layers)
@@ -463,19 +465,19 @@ static std::vector<char> nvrtc_compile(const std::string& source) {
   return cubin;
 }
 
-static felix_space::Module& get_module(felix_space* s, int P, int R = 1) {
+static felix_space::Module& get_module(felix_space* s, int P, int R = 1, int dphi_parts = 1) {
   // the forward kernel stages NREP x NS x 32 x (K0P+1) floats + NREP x NV x 32 doubles statically
   if (R > 1 && static_cast<int64_t>(R) * (s->desc.n_statements * 32 * (s->K0p + 1) * 4 + s->desc.n_vars * 32 * (8 + 4) + 64) > 48 * 1024)
     R = 1;
   const bool trace = g_tune.trace.load() != 0;
-  const int key = P + 64 * R + (trace ? 4096 : 0);
+  const int key = P + 64 * R + (trace ? 4096 : 0) + 8192 * dphi_parts;
   auto it = s->modules.find(key);
   if (it != s->modules.end()) return it->second;
   felix_space::Module mod;
   mod.P = P;
   mod.R = R;
   CodegenInfo info;
-  mod.source = generate_dag_module(s->desc, s->K0p, P, R, trace, &info);
+  mod.source = generate_dag_module(s->desc, s->K0p, P, R, trace, dphi_parts, &info);
   s->flops_fwd = info.flops_fwd;
   s->flops_rev = info.flops_rev;
   mod.rev_smem = info.rev_smem_bytes;
@@ -624,7 +626,19 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
       p->mask[l]->alloc(np * (d[l] / 32) * 4);
     }
   }
-  p->dphi.alloc(static_cast<size_t>(K0p) * np * 4);
+  // split-K of the chain's dL/dphi layer (K = d1): ksplit contiguous K ranges on ksplit CTAs per row block,
+  // each writing a partial slab (measured at C2: see DESIGN.md §8); only while every part fits one wave
+  int sms0 = 148;
+  CUDA_OK(cudaDeviceGetAttribute(&sms0, cudaDevAttrMultiProcessorCount, device));
+  int dphi_split = 1;
+  {
+    const int nkb1 = (d[1] + GEMM_BK - 1) / GEMM_BK;
+    const int ks = g_tune.dphi_ksplit.load();
+    auto fits = [&](int sp) { return nkb1 % sp == 0 && (np / 128) * sp <= sms0; };
+    if ((ks == 2 || ks == 4) && nkb1 % ks == 0) dphi_split = ks;
+    else if (ks < 0 && fits(4)) dphi_split = 4;
+  }
+  p->dphi.alloc(static_cast<size_t>(dphi_split) * K0p * np * 4);
   p->m.alloc(static_cast<size_t>(n_vars) * n_cand * 4);
   p->v.alloc(static_cast<size_t>(n_vars) * n_cand * 4);
   p->step_ctr.alloc(16);
@@ -715,11 +729,14 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     L.epi = g.epi;
     const int N = g.args.N;
     int bn = g.bn;
+    L.ksplit = 1;
     if (g.epi == EPI_F32T) {
       // dL/dphi (K = d1 = 512, N = K0p): its A row block is the largest operand a CTA ingests, and with
-      // one N tile only mt CTAs work; 32-wide N tiles spread it over 3x the CTAs while they fit in one wave
+      // one N tile only mt CTAs work: split K over dphi_split CTAs (partial slabs), else 32-wide N tiles
+      // spread it over 3x the CTAs while they fit in one wave
       bn = g.bn;                                                          // K0p (<= 128 required)
-      if (N % 32 == 0 && mt * (N / 32) <= sms) bn = 32;
+      if (dphi_split > 1) L.ksplit = dphi_split;
+      else if (N % 32 == 0 && mt * (N / 32) <= sms) bn = 32;
     }
     else bn = (N % 128 == 0 && mt * (N / 128) >= sms * 2 / 3) ? 128 : 64;
     if (bn > CHAIN_BN_MAX) FELIX_THROW(FELIX_E_UNSUPPORTED, "chain tile N > 128");
@@ -742,7 +759,7 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
       L.b_lo = make_tmap(cm->WTs_lo.p, N, g.args.K, bn / ccg);
     }
     if (g.epi == EPI_HEAD && use_chain()) p->n_head_tiles = 2 * (N / bn);   // chain: one partial per column half
-    max_tiles = std::max(max_tiles, static_cast<int>((mt + ccg - 1) / ccg) * L.n_tiles_n * ccg);   // CTAs the layer can use
+    max_tiles = std::max(max_tiles, static_cast<int>((mt + ccg - 1) / ccg) * L.n_tiles_n * L.ksplit * ccg);   // CTAs the layer can use
   }
   p->chain_grid = std::min(sms / p->chain_cg * p->chain_cg, max_tiles);
   // Grid chain with per-row-block dataflow flags (cooperative launch: every CTA resident): at C2 44.2 us
@@ -764,7 +781,7 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
       // every CTA (pair) has at most one tile of each of the two layers and the same N tile in both
       const int64_t units_p = (mt + p->chain_cg - 1) / p->chain_cg * Lp.n_tiles_n, units_i = (mt + p->chain_cg - 1) / p->chain_cg * Li.n_tiles_n;
       const int64_t clusters = p->chain_grid / p->chain_cg;
-      if (Lp.epi != EPI_F32T && units_p <= clusters && units_i <= clusters &&
+      if (Lp.epi != EPI_F32T && Li.ksplit == 1 && units_p <= clusters && units_i <= clusters &&
           Lp.n_tiles_n == Li.n_tiles_n && Lp.bn % GEMM_BK == 0)
         Li.reuse = 1;
     }
@@ -813,6 +830,7 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     p->tile_grid = static_cast<int>(std::min<int64_t>(sms / cg, units) * cg);
   }
   p->mode = mlp_mode(*p);
+  p->dphi_parts = p->mode == MLP_CHAIN ? dphi_split : 1;   // the tile kernel and the per-layer GEMMs write one slab
   if (p->mode == MLP_TILE) p->n_head_tiles = 2;                           // one partial per column half
   else if (p->mode == MLP_LAYERS) p->n_head_tiles = p->gemms[L - 2].args.N / p->gemms[L - 2].bn;
   return p;
@@ -1032,7 +1050,7 @@ felix_status felix_codegen(const felix_var* vars, int32_t n_vars, const felix_sp
   CodegenInfo info;
   // felix_tune("codegen_cone_width" / "codegen_replicas") select the variant to inspect (default P = 4, R = 2)
   const int cp = g_tune.codegen_P.load(), cr = g_tune.codegen_R.load();
-  const std::string code = generate_dag_module(s->desc, s->K0p, cp > 0 ? cp : 4, cr > 0 ? cr : 2, g_tune.trace.load() != 0, &info);
+  const std::string code = generate_dag_module(s->desc, s->K0p, cp > 0 ? cp : 4, cr > 0 ? cr : 2, g_tune.trace.load() != 0, 1, &info);
   if (src_len) *src_len = static_cast<int64_t>(code.size());
   if (src && src_cap > 0) {
     const size_t nb = std::min<size_t>(code.size() + 1, static_cast<size_t>(src_cap));
@@ -1191,7 +1209,8 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
   const int nck = static_cast<int>(ch.plans.size());
   const bool sc = use_sc() && !p->history;
   const int P0 = choose_P(ch.cnt[0]);
-  const felix_space::Module& mod = sc ? get_module(s, choose_P_sc(P0), choose_R_sc()) : get_module(s, P0, choose_R(ch.cnt[0], P0));
+  const int dpp = ch.plans[0]->dphi_parts;
+  const felix_space::Module& mod = sc ? get_module(s, choose_P_sc(P0), choose_R_sc(), dpp) : get_module(s, P0, choose_R(ch.cnt[0], P0), dpp);
   const int scw = choose_scw(ch.cnt[0], mod.P);
   if (!p->init_from_y) {
     unsigned long long seed = p->rng_seed;
@@ -1509,7 +1528,8 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
   std::vector<int> scws(G);
   for (int i = 0; i < G; ++i) {
     const int64_t n = params[i].n_seeds;
-    mods[i] = sc ? &get_module(spaces[i], choose_P_sc(choose_P(n)), choose_R_sc()) : &get_module(spaces[i], choose_P(n), choose_R(n, choose_P(n)));
+    mods[i] = sc ? &get_module(spaces[i], choose_P_sc(choose_P(n)), choose_R_sc(), pl.dphi_parts)
+                 : &get_module(spaces[i], choose_P(n), choose_R(n, choose_P(n)), pl.dphi_parts);
     scws[i] = choose_scw(n, mods[i]->P);
     if (sc) {
       ensure(*gc.sc_part[i], static_cast<size_t>(mods[i]->P) * spaces[i]->desc.n_vars * n * 4);
@@ -1694,7 +1714,7 @@ static void eval_impl(felix_space* s, felix_costmodel* m, const float* y, int64_
   int nht = pl.n_head_tiles;
   float hb = m->head_b, lam = lambda;
   if (o.search_path) {
-    const felix_space::Module& mod = get_module(s, choose_P_sc(choose_P(n)), choose_R_sc());
+    const felix_space::Module& mod = get_module(s, choose_P_sc(choose_P(n)), choose_R_sc(), pl.dphi_parts);
     const int scw = choose_scw(n, mod.P);
     ensure(pl.sc_part, static_cast<size_t>(mod.P) * s->desc.n_vars * n * 4);
     ensure(pl.sc_pen, static_cast<size_t>(mod.P) * n * 8);
@@ -1722,7 +1742,7 @@ static void eval_impl(felix_space* s, felix_costmodel* m, const float* y, int64_
     launch_flat(mod.f_adam_sc, n, aa, st);
     return;
   }
-  const felix_space::Module& mod = get_module(s, choose_P(n), choose_R(n, choose_P(n)));
+  const felix_space::Module& mod = get_module(s, choose_P(n), choose_R(n, choose_P(n)), pl.dphi_parts);
   run_forward_mlp(s, pl, mod, y, n, n, st, pl.step_ctr.as<int>());
   float *phi = o.phi, *g = o.g, *cost = o.cost, *loss = o.loss, *grad = o.grad;
   double* F = o.F;
@@ -2028,6 +2048,7 @@ felix_status felix_tune(const char* key, int32_t value) {
   else if (k == "split_cone") { in({-1, 0, 1}); g_tune.sc = value; }
   else if (k == "tile_cta_group") { in({-1, 1, 2}); g_tune.tile_cg = value; }
   else if (k == "chain_cta_group") { in({-1, 1, 2}); g_tune.chain_cg = value; }
+  else if (k == "dphi_ksplit") { in({-1, 1, 2, 4}); g_tune.dphi_ksplit = value; }
   else if (k == "codegen_cone_width") { in({-1, 1, 2, 4, 8, 16}); g_tune.codegen_P = value; }
   else if (k == "codegen_replicas") { in({-1, 1, 2, 4}); g_tune.codegen_R = value; }
   else if (k == "trace") { in({0, 1}); g_tune.trace = value; }

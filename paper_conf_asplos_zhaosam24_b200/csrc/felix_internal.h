@@ -84,7 +84,7 @@ struct CodegenInfo {
   int rev_smem_bytes = 0;
 };
 // P = warps cooperating on one 32-candidate block (cone partition of the roots), 1..8
-std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int R, bool trace, CodegenInfo* info);
+std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int R, bool trace, int dphi_parts, CodegenInfo* info);
 
 // -------------------------------------------------------------------------- cost model
 struct CostModel {

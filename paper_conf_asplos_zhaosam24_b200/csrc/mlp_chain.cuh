@@ -68,6 +68,11 @@ struct ChainLayer {
   // a_exact: A is an exact 0/1 mask (fp16 hi exact, lo = 0): no A lo loads, no A lo MMA pass (the first
   // backward layer, weights prescaled by the head row); head_exact: this HEAD layer writes that mask
   int a_exact, head_exact;
+  // ksplit (EPI_F32T, the last layer only): K is cut into ksplit contiguous ranges, tile = (row block, N
+  // tile, part), part fastest; part p writes its partial dL/dphi to slab p of out_f32 (slab = N x ld_f32
+  // floats); the reverse kernel sums the slabs in fixed order.  Spreads the largest per-CTA operand (A of
+  // the K = 512 layer) over ksplit CTAs.
+  int ksplit;
 };
 
 struct ChainParams {
@@ -124,10 +129,10 @@ __device__ __forceinline__ void grid_barrier(unsigned int* ctr, unsigned int nbl
 template <int CG>
 struct ChainTiles {
   int t0, tstep, ntn, units;
-  __device__ ChainTiles(int n_tiles_n, int m_tiles) : ntn(n_tiles_n) {
+  __device__ ChainTiles(int n_tiles_n, int m_tiles, int ksplit = 1) : ntn(n_tiles_n) {
     t0 = blockIdx.x / CG;
     tstep = gridDim.x / CG;
-    units = ((m_tiles + CG - 1) / CG) * ntn;
+    units = ((m_tiles + CG - 1) / CG) * ntn * ksplit;
   }
   __device__ int first() const { return t0 < units ? t0 : -1; }
   __device__ int next(int tile) const { tile += tstep; return tile < units ? tile : -1; }
@@ -218,14 +223,17 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
           asm volatile("fence.proxy.async.global;" ::: "memory");
         }
         CHAIN_STAMP(l, 0);
-        const int nkb = (L.args.K + GEMM_BK - 1) / GEMM_BK;
+        const int S = L.ksplit;
+        const int nkb_all = (L.args.K + GEMM_BK - 1) / GEMM_BK;
         const int bnc = L.bn / CG;                                  // weight rows this CTA loads per tile
         const uint32_t tx_b = 2 * (bnc * GEMM_BK * 2);
         const uint32_t tx = (L.a_exact ? 1 : 2) * CHAIN_A_BYTES + tx_b;
-        ChainTiles<CG> tiles(L.n_tiles_n, P.m_tiles);
+        ChainTiles<CG> tiles(L.n_tiles_n, P.m_tiles, S);
         for (int tile = tiles.first(); tile >= 0; tile = tiles.next(tile)) {
-          const int mb = row_block(tile, L.n_tiles_n);
-          const int m0 = mb * GEMM_BM, n0 = (tile % L.n_tiles_n) * L.bn, nb = n0 + static_cast<int>(rank) * bnc;
+          const int tq = tile / S, part = tile % S;
+          const int kbeg = part * nkb_all / S, nkb = (part + 1) * nkb_all / S - kbeg;
+          const int mb = row_block(tq, L.n_tiles_n);
+          const int m0 = mb * GEMM_BM, n0 = (tq % L.n_tiles_n) * L.bn, nb = n0 + static_cast<int>(rank) * bnc;
           int kb0 = 0;
           if (dataflow && l > 0 && L.reuse) {
             // own K blocks (B only) first, then the others (B, row-block flag once, A)
@@ -260,15 +268,15 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
               const int s = (it + kb) % CHAIN_STAGES;
               if (it + kb >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], (((it + kb) / CHAIN_STAGES) - 1) & 1);
               arm(s, tx);
-              load(b_hi(s), &L.b_hi, kb * GEMM_BK, nb, s);
-              load(b_lo(s), &L.b_lo, kb * GEMM_BK, nb, s);
+              load(b_hi(s), &L.b_hi, (kbeg + kb) * GEMM_BK, nb, s);
+              load(b_lo(s), &L.b_lo, (kbeg + kb) * GEMM_BK, nb, s);
             }
             flag_wait(flag_of(l - 1, mb), epoch * static_cast<unsigned int>(P.layer[l - 1].n_tiles_n));
             asm volatile("fence.proxy.async.global;" ::: "memory");
             for (int kb = 0; kb < pre; ++kb) {
               const int s = (it + kb) % CHAIN_STAGES;
-              load(a_hi(s), &L.a_hi, kb * GEMM_BK, m0, s);
-              if (!L.a_exact) load(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, s);
+              load(a_hi(s), &L.a_hi, (kbeg + kb) * GEMM_BK, m0, s);
+              if (!L.a_exact) load(a_lo(s), &L.a_lo, (kbeg + kb) * GEMM_BK, m0, s);
             }
             kb0 = pre;
             it += pre;
@@ -277,7 +285,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             const int s = it % CHAIN_STAGES;
             if (it >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], ((it / CHAIN_STAGES) - 1) & 1);
             arm(s, tx);
-            const int k0 = kb * GEMM_BK;
+            const int k0 = (kbeg + kb) * GEMM_BK;
             load(a_hi(s), &L.a_hi, k0, m0, s);
             if (!L.a_exact) load(a_lo(s), &L.a_lo, k0, m0, s);
             load(b_hi(s), &L.b_hi, k0, nb, s);
@@ -293,9 +301,12 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       int staged_tiles = 0, chunk_count = 0, prev_chunk_base = 0;   // mirror of the epilogue's staging sequence
       for (int l = 0; l < P.n_layers; ++l) {
         const ChainLayer& L = P.layer[l];
-        const int nkb = (L.args.K + GEMM_BK - 1) / GEMM_BK;
-        ChainTiles<CG> tiles(L.n_tiles_n, P.m_tiles);
+        const int S = L.ksplit;
+        const int nkb_all = (L.args.K + GEMM_BK - 1) / GEMM_BK;
+        ChainTiles<CG> tiles(L.n_tiles_n, P.m_tiles, S);
         for (int tile = tiles.first(); tile >= 0; tile = tiles.next(tile), ++tcount) {
+          const int part = tile % S;
+          const int nkb = (part + 1) * nkb_all / S - part * nkb_all / S;
           const int acc = tcount & 1;
           if (tcount >= 2) wait_in(&tempty[acc], ((tcount >> 1) - 1) & 1);
           ptx::tc_fence_after();
@@ -380,6 +391,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       const CUtensorMap* tm_c_hi = &L.c_hi;
       const CUtensorMap* tm_c_lo = &L.c_lo;
       const bool next_reuse = dataflow && l + 1 < P.n_layers && P.layer[l + 1].reuse;
+      const int S = L.ksplit;
       // stage this layer's bias / head row in smem while the MMA warp works (previous layer's
       // readers are past the layer-end barrier, so the buffer is free)
       if (epi == EPI_RELU || epi == EPI_HEAD) {
@@ -389,12 +401,13 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         }
       }
       ptx::named_bar_sync(1, NEPI);
-      ChainTiles<CG> tiles(ntn, P.m_tiles);
+      ChainTiles<CG> tiles(ntn, P.m_tiles, S);
       const int first_tile = tiles.first();
       for (int tile = first_tile; tile >= 0; tile = tiles.next(tile), ++tcount) {
         const int acc = tcount & 1;
-        const int mb = row_block(tile, ntn);
-        const int m0 = mb * GEMM_BM, n0 = (tile % ntn) * bn;
+        const int tq = tile / S, part = tile % S;
+        const int mb = row_block(tq, ntn);
+        const int m0 = mb * GEMM_BM, n0 = (tq % ntn) * bn;
         const int row = m0 + r_tile;
         const bool row_ok = row < aM;
         // this thread's mask words for the tile (<= 2 chunks of 64 columns), requested before the wait
@@ -426,10 +439,11 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
               for (int i = 0; i < 16; ++i) { v[i] = a[i]; v[16 + i] = b[i]; }
             }
             const int n = n0 + c;
+            float* __restrict__ slab = out_f32 + static_cast<size_t>(part) * aN * ld_f32;
             if (row_ok) {
 #pragma unroll
               for (int i = 0; i < 32; ++i)
-                if (n + i < n_valid) out_f32[static_cast<size_t>(n + i) * ld_f32 + row] = v[i];
+                if (n + i < n_valid) slab[static_cast<size_t>(n + i) * ld_f32 + row] = v[i];
             }
           }
         } else {

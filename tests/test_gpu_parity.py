@@ -219,20 +219,14 @@ def test_full_size_c2_sampled(fx):
     assert np.sum((err > 1e-3) & (kink_margin(ref.zs) >= 1e-4)) == 0
 
 
-def test_full_size_c5_per_gpu_sampled(fx):
-    """C5's per-GPU shard (2^20 / 8 = 131072 candidates of the ViT-L fc1 space): one objective
-    evaluation at full size, 48 sampled candidates checked against the oracle; then a short search
-    and its top-k, whose records must be valid rounded schedules with oracle-exact FP64 scores."""
+def test_full_size_c5_per_gpu_search_topk(fx):
+    """C5's per-GPU shard (2^20 / 8 = 131072 candidates of the ViT-L fc1 space; its objective and gradient
+    at full size are checked in test_gpu_parity_ops.py): a short search and its top-k, whose records
+    must be valid rounded schedules with oracle-exact FP64 scores."""
     sp, mlp, _, space, cm = _setup(fx, "C5")
     n = 131072
     y0 = fo.init_sample(sp, n, 0x5EED0005)
     yt = torch.from_numpy(y0).cuda()
-    out = space.eval(cm, yt)
-    pick = np.random.default_rng(1).choice(n, 48, replace=False)
-    ref = fo.objective(sp, mlp.W, mlp.b, y0[:, pick].astype(np.float64), 1.0)
-    cost = out["cost"].cpu().numpy()[pick]
-    s = np.sqrt(np.mean(ref.c ** 2))
-    assert np.max(np.abs(cost - ref.c)) / s <= 1e-4
     space.search(cm, yt, 5, init_from_y=True)
     idx, sc, sched = space.round_topk(cm, yt, 64)
     assert len(idx) == 64 and len(set(map(tuple, sched))) == 64
@@ -474,7 +468,7 @@ def test_multitask_shards_equal_single_rank_and_oracle(fx, mode):
     cm = fx.CostModel.from_weights(mlp)
     r50 = fi.resnet50_spaces()
     spaces = [r50[0], r50[6], r50[-1], fi.bert_spaces()[1]]
-    n, T, k = 700, 6, 16
+    n, T, k = 400, 4, 16
     costs = [tasks.est_cost(n, T, cm.mlp_flops_per_candidate_step(), sp.nodes.shape[0]) for sp in spaces]
     nv = [sp.n_vars for sp in spaces]
     one = tasks.TaskRunner(spaces, tasks.plan(len(spaces), n, 1, mode, costs)[0], cm)
@@ -602,10 +596,8 @@ def test_search_group_errors(fx):
 
 
 @pytest.mark.parametrize("name,n,steps,P,W,chunks", [
-    ("C2", 1000, 7, 4, -1, 1), ("C2", 4096, 8, 4, -1, 1), ("C2", 1000, 5, 8, 3, 1),
-    ("C2_2stmt", 700, 6, 4, 2, 1), ("bmm", 257, 5, 2, 1, 1), ("C2", 3000, 6, 4, -1, 2),
-    ("C5", 389, 9, 1, -1, 1), ("C5", 389, 8, 2, -1, 1), ("r50_conv1", 300, 4, 4, 1, 1),
-    ("C2", 1000, 1, 4, -1, 1), ("C2", 1000, 6, 8, 2, 1)])
+    ("C2", 4096, 8, 4, -1, 1), ("C2", 1000, 5, 8, 3, 1), ("C2_2stmt", 700, 6, 4, 2, 1),
+    ("bmm", 257, 5, 2, 1, 1), ("C2", 3000, 6, 4, -1, 2), ("C5", 389, 9, 1, -1, 1), ("r50_conv1", 300, 4, 4, 1, 1)])
 def test_split_cone_kernels_match_cone_groups(fx, name, n, steps, P, W, chunks):
     """Split-cone reverse kernel (one cone per CTA, FP32 partial adjoints through global memory; the next
     step's forward sums them and applies Adam in place, felix_adam_sc after the last step) against the
