@@ -116,14 +116,14 @@ def test_split_cone_codegen_partitions_every_seed_once(fx, P):
         src = fx.codegen(sp)
     rev = _kernel_body(src, "felix_rev_sc")
     assert len(re.findall(r"if \(cq_ == \d+\)", rev)) == int(P)
-    seeds = re.findall(r"dphi_sum\(dphi, \(size_t\)(\d+) \* ld_dphi", rev)
+    seeds = re.findall(r"dphi\[\(size_t\)(\d+) \* ld_dphi", rev)
     n_dep = sum(1 for r in sp.feature_roots if _depends_on_var(sp, r))
     assert sorted(int(k) for k in seeds) == sorted(set(int(k) for k in seeds)) and len(seeds) == n_dep
     for q in range(int(P)):
         for j in range(sp.n_vars):
             assert f"part[((size_t){q} * NV + {j}) * n + c]" in rev
     body = src[src.index("void rev_body("):src.index('extern "C" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_adam')]
-    assert sorted(re.findall(r"dphi_sum\(dphi, \(size_t\)(\d+) \* ld_dphi", body)) == sorted(seeds)
+    assert sorted(re.findall(r"dphi\[\(size_t\)(\d+) \* ld_dphi", body)) == sorted(seeds)
     assert "*step_ctr - 1" in src and "*step_ctr += 1" in rev
 
 
