@@ -388,7 +388,7 @@ def run_felix(args):
     mlp_kernel = "mlp_tile_kernel" if tile_fits and -(-n_rows // 128) >= sms else "mlp_chain_kernel"
     traffic = None
     tname = {"mlp_chain_kernel": "roofline_traffic.json", "mlp_tile_kernel": "roofline_traffic_tile.json"}.get(mlp_kernel, "")
-    tpath = os.path.join(ROOT, "profiles", "r01", tname) if tname else ""
+    tpath = os.path.join(ROOT, "profiles", "r02", tname) if tname else ""
     if tname and os.path.exists(tpath):
         with open(tpath) as f:
             tj = json.load(f)
@@ -495,7 +495,7 @@ def run_felix(args):
         "roofline": {"bound": "tensor", "achieved": achieved_tflops, "peak": peak, "unit": "TFLOP/s",
                      "frac": achieved_tflops / peak, "traffic": traffic,
                      "kernel": f"{mlp_kernel} (all {n_gemm} MLP layers of one Adam step, tcgen05 kind::f16, 3-pass hi/lo split)",
-                     "traffic_source": (f"profiles/r01/{tname} (ncu --set full, DRAM bytes per launch)"
+                     "traffic_source": (f"profiles/r02/{tname} (ncu --set full, DRAM bytes per launch)"
                                         if traffic is not None else None),
                      "algorithmic_flops_per_adam_step": mlp_flops_step,
                      "executed_tflops": 3 * achieved_tflops,
