@@ -4,4 +4,4 @@ from .configs import (Config, MLPWeights, config, make_mlp, make_y0, var_upper_b
                       c1_space, c2_space, c2_space_two_statements, c2_sketches, c5_space, bert_spaces, resnet50_spaces, paper_example_space,
                       mobilenet_v2_spaces,
                       DEFAULT_MLP, C1_MLP)
-from .testspaces import allops_space, rnan_space  # noqa: F401
+from .testspaces import allops_space, composite_space, rnan_space  # noqa: F401

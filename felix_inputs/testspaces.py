@@ -100,3 +100,35 @@ def rnan_space() -> Space:
     names[free[0]], names[free[1]] = "log(x0-3)", "x1/(x0-2)"
     return Space("rnan", base.vars, base.splits, arr, froots, base.constraint_roots.copy(), names,
                  list(base.constraint_names), None)
+
+
+def composite_space(n_tile_vars: int = 4, extent: int = 720720) -> Space:
+    """Highly composite split extents for the rounding search (SURVEY §7c hard part 7; "N is
+    ... typically smaller than 10^6"): `extent` = 720720 = 2^4 3^2 5 7 11 13 (240 divisors) tiled by
+    `n_tile_vars` variables (4: 6.6e5 divisor tuples; 8: 1.5e8), a second component in which one
+    variable sits in two splits (5040 and 2520), and an INT variable; 82 feature roots over all of them
+    (products, ratios, logs) so a cost model of the default dims scores the schedules."""
+    B = DagBuilder()
+    nt = n_tile_vars
+    xs = [B.var(j) for j in range(nt + 4)]
+    f = []
+    for a in range(len(xs)):
+        f += [xs[a], B.log(B.add(xs[a], B.const(1.0)))]
+    for a in range(len(xs)):
+        for b in range(a + 1, len(xs)):
+            f += [B.mul(xs[a], xs[b]), B.div(xs[a], B.add(xs[b], B.const(1.0)))]
+            if len(f) >= 82:
+                break
+        if len(f) >= 82:
+            break
+    while len(f) < 82:
+        f.append(B.add(f[len(f) % 7], B.const(float(len(f)))))
+    con = B.sub(B.mul(xs[0], xs[1]), B.const(4096.0))
+    nodes = B.nodes()
+    vars_ = [Var(f"t{j}", VAR_SPLIT, 1, extent) for j in range(nt)]
+    vars_ += [Var("s0", VAR_SPLIT, 1, 2520), Var("s1", VAR_SPLIT, 1, 5040), Var("s2", VAR_SPLIT, 1, 2520),
+              Var("u", VAR_INT, 1, 100)]
+    splits = [Split(extent, list(range(nt))), Split(5040, [nt, nt + 1]), Split(2520, [nt, nt + 2])]
+    return Space(f"composite{nt}", vars_, splits, nodes, np.array(f[:82], dtype=np.int32),
+                 np.array([con], dtype=np.int32), feature_names=[f"f{i}" for i in range(82)],
+                 constraint_names=["t0t1"])

@@ -102,8 +102,11 @@ typedef struct felix_costmodel felix_costmodel;
  * The library appends the automatic log-space validity roots (reading O2), in this order
  * after the user roots:  -y_j for every SPLIT var;  sum_{j in s} y_j - ln(extent_s) per split;
  * ln(lo_j) - y_j and y_j - ln(hi_j) per INT var.  R = total number of roots (felix_space_info).
- * Builds the divisor-tuple tables of every split component, generates straight-line CUDA for the
- * DAG (forward, reverse, hard, sampler) and compiles it for sm_100a with NVRTC. */
+ * Builds the divisor-tuple tables of every split component with at most 65536 tuples (larger ones —
+ * highly composite extents — are rounded by a branch-and-bound search over per-variable divisor lists,
+ * same result; a component may hold at most 8 variables and touch at most 16 splits, else
+ * FELIX_E_UNSUPPORTED), generates straight-line CUDA for the DAG (forward, reverse, hard, sampler) and
+ * compiles it for sm_100a with NVRTC. */
 FELIX_EXPORT felix_status felix_space_create(int device,
                                 const felix_var* vars, int32_t n_vars,
                                 const felix_split* splits, int32_t n_splits,
@@ -137,7 +140,7 @@ FELIX_EXPORT felix_status felix_codegen(const felix_var* vars, int32_t n_vars,
 
 typedef struct {
   int32_t n_vars, n_nodes, n_features, n_constraints_user, n_roots_total, n_components;
-  int64_t n_tuples_total;       /* rows of the divisor-tuple tables                            */
+  int64_t n_tuples_total;       /* rows of the divisor-tuple tables (branch-and-bound components: 0) */
   double nvrtc_ms;              /* time spent compiling the generated kernels                  */
   int32_t regs_fwd, regs_rev;   /* registers/thread of the generated forward / reverse kernels  */
   int64_t dag_flops_fwd;        /* arithmetic ops in one forward evaluation (per candidate)    */
@@ -272,6 +275,8 @@ FELIX_EXPORT felix_status felix_init_sample(felix_space* s, int64_t n, uint64_t 
  *                         in fixed order by the reverse kernel)
  *   "codegen_cone_width", "codegen_replicas"   the variant felix_codegen emits
  *   "trace"               0/1: per-block %globaltimer stamps in kernels generated afterwards
+ *   "round_bnb"           0/1: 1 = every split component is rounded by the branch-and-bound kernel
+ *                         (default 0: only components with more than 65536 divisor tuples are)
  * FELIX_E_INVALID_ARG for an unknown key or value. */
 FELIX_EXPORT felix_status felix_tune(const char* key, int32_t value);
 

@@ -27,6 +27,7 @@ __global__ void __launch_bounds__(256) round_split_kernel(
 #pragma unroll
   for (int k = 0; k < 8; ++k) yv[k] = k < nv ? static_cast<double>(y[static_cast<size_t>(vars[k]) * n + cand]) : 0.0;
   const long long eoff = comp_eoff[comp], T = comp_tcount[comp];
+  if (T < 0) return;                               // no table: round_bnb_kernel searches this component
   double best = DBL_MAX;
   long long bi = -1;
   for (long long t = lane; t < T; t += 32) {
@@ -50,6 +51,113 @@ __global__ void __launch_bounds__(256) round_split_kernel(
     const int* tp = tuples + eoff + bi * nv;
     for (int k = 0; k < nv; ++k) sched[static_cast<size_t>(cand) * M + vars[k]] = tp[k];
   }
+}
+
+// ---------------------------------------------------------------------------- K5a' branch and bound
+// The same argmin as round_split_kernel (sum_j (y_j - ln f_j)^2 over the divisor-respecting tuples,
+// FP64 in var order, explicitly rounded, ties -> lexicographically smallest tuple) for components whose
+// tuple table would be too large (highly composite extents, SURVEY §7c hard part 7; N is
+// "typically smaller than 10^6", and 720720 split four ways has 6.6e5 tuples, eight ways 1.5e8).
+// One thread per (candidate, component): depth-first over the component's vars in order; at depth k
+// the divisors of the var's gcd extent are visited outward from y_k (nearest first), a divisor is
+// taken only if it divides every remaining split extent the var belongs to, and a direction stops
+// as soon as partial + (y_k - ln d)^2 > best: the remaining terms are >= 0 and FP64 addition is
+// monotone, so every pruned tuple costs strictly more than the best found.  Leaves replace the best
+// on a smaller cost or on an equal cost and a lexicographically smaller tuple, so the result is the
+// exhaustive scan's bit for bit.  Non-finite y anywhere in the component: every tuple costs inf / NaN
+// and the scan returns its first tuple, all ones; so does this kernel.
+__global__ void __launch_bounds__(128) round_bnb_kernel(
+    const float* __restrict__ y, int n, int M, int n_sel, const int* __restrict__ sel_comp,
+    const int* __restrict__ comp_nvars, const int* __restrict__ comp_var0, const int* __restrict__ comp_vars,
+    const int* __restrict__ comp_ns, const int* __restrict__ comp_s0, const long long* __restrict__ comp_sext,
+    const unsigned* __restrict__ var_smask, const long long* __restrict__ var_doff, const int* __restrict__ var_dcnt,
+    const long long* __restrict__ dval, const double* __restrict__ dln, int* __restrict__ sched) {
+  const long long g = static_cast<long long>(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (g >= static_cast<long long>(n) * n_sel) return;
+  const int cand = static_cast<int>(g / n_sel), comp = sel_comp[g % n_sel];
+  const int nv = comp_nvars[comp], v0 = comp_var0[comp], ns = comp_ns[comp];
+  const int* vars = comp_vars + v0;
+  double yv[8];
+  bool finite = true;
+  for (int k = 0; k < nv; ++k) {
+    yv[k] = static_cast<double>(y[static_cast<size_t>(vars[k]) * n + cand]);
+    finite = finite && isfinite(yv[k]);
+  }
+  long long bt[8];
+  for (int k = 0; k < nv; ++k) bt[k] = 1;
+  if (finite) {
+    long long rem[16];
+    for (int q = 0; q < ns; ++q) rem[q] = comp_sext[comp_s0[comp] + q];
+    int lo[8], hi[8];
+    double acc[9];
+    long long cur[8];
+    double best = DBL_MAX;
+    bool found = false;
+    // position of y_k among the ascending ln d of var k: lo = last index with ln d < y, hi = lo + 1
+    auto start = [&](int k) {
+      const double* L = dln + var_doff[v0 + k];
+      int a = 0, b = var_dcnt[v0 + k];
+      while (a < b) { const int m = (a + b) >> 1; if (L[m] < yv[k]) a = m + 1; else b = m; }
+      lo[k] = a - 1; hi[k] = a;
+    };
+    acc[0] = 0.0;
+    int k = 0;
+    start(0);
+    while (k >= 0) {
+      const double* L = dln + var_doff[v0 + k];
+      const long long* D = dval + var_doff[v0 + k];
+      const int cnt = var_dcnt[v0 + k];
+      double elo = DBL_MAX, ehi = DBL_MAX;
+      bool olo = false, ohi = false;
+      if (lo[k] >= 0) {
+        const double d = __dsub_rn(yv[k], L[lo[k]]);
+        elo = __dadd_rn(acc[k], __dmul_rn(d, d));
+        olo = !(elo > best);
+      }
+      if (hi[k] < cnt) {
+        const double d = __dsub_rn(yv[k], L[hi[k]]);
+        ehi = __dadd_rn(acc[k], __dmul_rn(d, d));
+        ohi = !(ehi > best);
+      }
+      if (!olo && !ohi) {                       // level exhausted: back up, restoring the extents
+        --k;
+        if (k >= 0) {
+          const unsigned msk = var_smask[v0 + k];
+          for (int q = 0; q < ns; ++q) if (msk >> q & 1u) rem[q] *= cur[k];
+        }
+        continue;
+      }
+      const bool take_lo = olo && (!ohi || elo <= ehi);
+      const int idx = take_lo ? lo[k]-- : hi[k]++;
+      const double e = take_lo ? elo : ehi;
+      const long long dv = D[idx];
+      const unsigned msk = var_smask[v0 + k];
+      bool ok = true;
+      for (int q = 0; q < ns; ++q) if ((msk >> q & 1u) && rem[q] % dv != 0) ok = false;
+      if (!ok) continue;
+      if (k == nv - 1) {                        // leaf
+        bool better = !found || e < best;
+        if (!better && e == best) {
+          cur[k] = dv;
+          int q = 0;
+          while (q < nv && cur[q] == bt[q]) ++q;
+          better = q < nv && cur[q] < bt[q];
+        }
+        if (better) {
+          best = e; found = true;
+          cur[k] = dv;
+          for (int q = 0; q < nv; ++q) bt[q] = cur[q];
+        }
+        continue;
+      }
+      cur[k] = dv;
+      for (int q = 0; q < ns; ++q) if (msk >> q & 1u) rem[q] /= dv;
+      acc[k + 1] = e;
+      ++k;
+      start(k);
+    }
+  }
+  for (int k = 0; k < nv; ++k) sched[static_cast<size_t>(cand) * M + vars[k]] = static_cast<int>(bt[k]);
 }
 
 // ---------------------------------------------------------------------------- K5b INT rounding

@@ -742,12 +742,14 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "    reinterpret_cast<uint4*>(phi_hi + row * K0P)[q8] = make_uint4(h[0], h[1], h[2], h[3]);\n"
     << "    reinterpret_cast<uint4*>(phi_lo + row * K0P)[q8] = make_uint4(l[0], l[1], l[2], l[3]);\n"
     << "  }\n  TSTAMP(0, 4);\n}\n"
+    << "#if !defined(FELIX_PART) || FELIX_PART == 1\n"
     << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd(const float* __restrict__ yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr) {\n"
-    << "  fwd_body<0>(const_cast<float*>(yv), n, ldy, phi_hi, phi_lo, step_ctr, nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f);\n}\n"
+    << "  fwd_body<0>(const_cast<float*>(yv), n, ldy, phi_hi, phi_lo, step_ctr, nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f);\n}\n#endif\n"
+    << "#if !defined(FELIX_PART) || FELIX_PART == 2\n"
     << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd_adam(float* yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr,\n"
     << "    float* mv, float* vv, const float* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part,\n"
     << "    int n_head_tiles, int ld_c, float head_b, float lam, float lr, float b1, float b2, float eps) {\n"
-    << "  fwd_body<1>(yv, n, ldy, phi_hi, phi_lo, step_ctr, mv, vv, part, pen, c_part, n_head_tiles, ld_c, head_b, lam, lr, b1, b2, eps);\n}\n\n";
+    << "  fwd_body<1>(yv, n, ldy, phi_hi, phi_lo, step_ctr, mv, vv, part, pen, c_part, n_head_tiles, ld_c, head_b, lam, lr, b1, b2, eps);\n}\n#endif\n\n";
 
   // ---------------------------------------------------------------- felix_rev (template on mode)
   // smem: partial adjoints of x  spart[PG][NV][32], user-root penalties per group spen[PG][32],
@@ -911,12 +913,12 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "    }\n"
     << "    TSTAMP(1, 7);\n"
     << "  }\n}\n\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_adam(float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
+  o << "#if !defined(FELIX_PART) || FELIX_PART == 3\n" "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_adam(float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
     << "    float* mv, float* vv, const int* step_ctr, float lr, float b1, float b2, float eps, float* o_loss) {\n"
-    << "  rev_body<0>(yv, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, mv, vv, step_ctr, lr, b1, b2, eps, nullptr, nullptr, nullptr, o_loss, nullptr, nullptr);\n}\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_eval(const float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
+    << "  rev_body<0>(yv, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, mv, vv, step_ctr, lr, b1, b2, eps, nullptr, nullptr, nullptr, o_loss, nullptr, nullptr);\n}\n#endif\n";
+  o << "#if !defined(FELIX_PART) || FELIX_PART == 4\n" "extern \"C\" __global__ void __launch_bounds__(PG * 32 * NREP) felix_rev_eval(const float* yv, int n, int ldy, const float* dphi, int ld_dphi, const float* c_part, int n_head_tiles, int ld_c, float head_b, float lam,\n"
     << "    float* o_phi, float* o_g, float* o_cost, float* o_loss, float* o_grad, double* o_F) {\n"
-    << "  rev_body<1>(nullptr, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, nullptr, nullptr, nullptr, 0.f, 0.f, 0.f, 0.f, o_phi, o_g, o_cost, o_loss, o_grad, o_F);\n}\n\n";
+    << "  rev_body<1>(nullptr, yv, n, ldy, dphi, ld_dphi, c_part, n_head_tiles, ld_c, head_b, lam, nullptr, nullptr, nullptr, 0.f, 0.f, 0.f, 0.f, o_phi, o_g, o_cost, o_loss, o_grad, o_F);\n}\n#endif\n\n";
 
   // ---------------------------------------------------------------- split-cone search kernels
   // felix_rev_sc runs ONE cone per CTA (block-uniform q = blockIdx.x % PG) for W x 32 candidates, so the
@@ -933,7 +935,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
   // tolerance is 1e-3; half the registers and a third
   // of the instructions of the FP64 form, so the straight-line cone code streams through the SM's
   // instruction fetch faster.
-  o << "extern \"C\" __global__ void __launch_bounds__(256) felix_rev_sc(const float* __restrict__ yv, int n, int ldy, const float* __restrict__ dphi, int ld_dphi,\n"
+  o << "#if !defined(FELIX_PART) || FELIX_PART == 5\n" "extern \"C\" __global__ void __launch_bounds__(256) felix_rev_sc(const float* __restrict__ yv, int n, int ldy, const float* __restrict__ dphi, int ld_dphi,\n"
     << "    float lam, float* __restrict__ part, double* __restrict__ pen, int* step_ctr) {\n"
     << "  const int cq_ = blockIdx.x % PG;\n"
     << "  const int c = ((blockIdx.x / PG) * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32 + (threadIdx.x & 31);\n"
@@ -971,9 +973,9 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
       o << "      part[((size_t)" << q << " * NV + " << j << ") * n + c] = " << (used[j] ? "x" + std::to_string(j) + " * gx" + std::to_string(j) : std::string("0.f")) << ";\n";
     o << "    }\n    TSTAMP(1, 3);\n  }\n";
   }
-  o << "}\n\n";
+  o << "}\n#endif\n\n";
   // felix_adam_sc: the last Adam step (thread per candidate, in place) + the final loss
-  o << "extern \"C\" __global__ void __launch_bounds__(128) felix_adam_sc(float* yv, int n, int ldy, float* mv, float* vv,\n"
+  o << "#if !defined(FELIX_PART) || FELIX_PART == 6\n" "extern \"C\" __global__ void __launch_bounds__(128) felix_adam_sc(float* yv, int n, int ldy, float* mv, float* vv,\n"
     << "    const float* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part, int n_head_tiles, int ld_c,\n"
     << "    float head_b, float lam, float lr, float b1, float b2, float eps, const int* step_ctr, float* o_loss, float* o_grad) {\n"
     << "  const int c = blockIdx.x * blockDim.x + threadIdx.x;\n  if (c >= n) return;\n"
@@ -1004,11 +1006,11 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "    float m = ml[j], v = vl[j];\n"
     << "    m = b1 * m + (1.f - b1) * gy[j]; v = b2 * v + (1.f - b2) * gy[j] * gy[j];\n"
     << "    mv[(size_t)j * n + c] = m; vv[(size_t)j * n + c] = v; yv[(size_t)j * ldy + c] = syv[j] - step * m / (sqrtf(v) * rb + eps);\n"
-    << "  }\n}\n\n";
+    << "  }\n}\n#endif\n\n";
 
   // ---------------------------------------------------------------- felix_hard (fp64 IEEE, integer points)
   std::vector<bool> all(g.n, true);
-  o << "extern \"C\" __global__ void __launch_bounds__(128) felix_hard(const int* __restrict__ sched, int n, double* __restrict__ phi64, unsigned char* __restrict__ valid) {\n"
+  o << "#if !defined(FELIX_PART) || FELIX_PART == 7\n" "extern \"C\" __global__ void __launch_bounds__(128) felix_hard(const int* __restrict__ sched, int n, double* __restrict__ phi64, unsigned char* __restrict__ valid) {\n"
     << "  const int i = blockIdx.x * blockDim.x + threadIdx.x;\n  if (i >= n) return;\n";
   for (int j = 0; j < M; ++j) o << "  const double h" << j << " = (double)sched[(size_t)i * NV + " << j << "];\n";
   g.emit_forward(all, 2, "h");
@@ -1016,7 +1018,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
   for (int k = 0; k < K; ++k)
     o << "  ok = ok && isfinite(v" << d.froots[k] << "); phi64[(size_t)" << k << " * n + i] = slogd_(v" << d.froots[k] << ");\n";
   for (int r = 0; r < Ru; ++r) o << "  ok = ok && isfinite(v" << d.croots[r] << ") && (v" << d.croots[r] << " <= 1e-9);\n";
-  o << "  valid[i] = ok ? 1 : 0;\n}\n\n";
+  o << "  valid[i] = ok ? 1 : 0;\n}\n#endif\n\n";
 
   // ---------------------------------------------------------------- felix_init (rejection sampler)
   std::vector<int> parent(M);
@@ -1036,7 +1038,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
   // one warp per candidate: lane L evaluates outer attempt a2 = base + L (a pure function of a2), the
   // first accepted attempt in attempt order wins (ballot) and its y is broadcast: the same starting point
   // as the serial rejection loop of the spec, with the serial chain of attempts replaced by 32 in flight
-  o << "extern \"C\" __global__ void __launch_bounds__(128) felix_init(u64 seed, int n, long long index_base, float* __restrict__ yout) {\n"
+  o << "#if !defined(FELIX_PART) || FELIX_PART == 8\n" "extern \"C\" __global__ void __launch_bounds__(128) felix_init(u64 seed, int n, long long index_base, float* __restrict__ yout) {\n"
     << "  const int lane = threadIdx.x & 31;\n"
     << "  const int i = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5);\n  if (i >= n) return;\n"
     << "  const u64 cand = (u64)(index_base + i);\n";
@@ -1087,7 +1089,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     o << "    y" << j << " = " << (d.vars[j].kind == FELIX_VAR_INT ? lit(std::log((double)d.vars[j].lo)) : "0.0") << ";\n";
   o << "  }\n";
   for (int j = 0; j < M; ++j) o << "  if (lane == " << (j % 32) << ") yout[(size_t)" << j << " * n + i] = (float)y" << j << ";\n";
-  o << "}\n\n";
+  o << "}\n#endif\n\n";
 
   if (info) {
     info->flops_fwd = flops_fwd;

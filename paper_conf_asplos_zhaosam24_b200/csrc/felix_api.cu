@@ -17,6 +17,8 @@
 #include <mutex>
 #include <numeric>
 #include <string>
+#include <thread>
+#include <memory>
 #include <vector>
 #include <nvrtc.h>
 #include <cudaTypedefs.h>
@@ -143,6 +145,7 @@ struct Tuning {
   std::atomic<int> dphi_ksplit{-1};  // layer chain: split-K parts of the dL/dphi layer (1, 2, 4)
   std::atomic<int> codegen_P{-1}, codegen_R{-1};   // felix_codegen's variant
   std::atomic<int> trace{0};         // per-block %globaltimer stamps in kernels generated afterwards
+  std::atomic<int> round_bnb{0};     // 1: every split component rounds by branch and bound (test hook)
 };
 static Tuning g_tune;
 
@@ -278,6 +281,8 @@ struct GroupCache {
 
 }  // namespace felix
 
+static constexpr int kModuleParts = 8;   // kernels of a generated module (codegen.cpp FELIX_PART)
+
 struct felix_space {
   uint64_t uid = felix::next_uid();   // identity for workspace caches (see GroupCache)
   int device = 0;
@@ -287,9 +292,10 @@ struct felix_space {
   // device copies of the rounding tables
   felix::DevBuf d_comp_nvars, d_comp_var0, d_comp_vars, d_comp_eoff, d_comp_tcount, d_tuples, d_lnf;
   felix::DevBuf d_int_vars, d_int_lo, d_int_cnt, d_int_toff, d_int_thr;
+  felix::DevBuf d_comp_ns, d_comp_s0, d_comp_sext, d_var_smask, d_var_doff, d_var_dcnt, d_dval, d_dln, d_bnb_sel, d_all_sel;
   // NVRTC modules, one per cone-partition width P (compiled on first use)
   struct Module {
-    cudaLibrary_t lib = nullptr;
+    cudaLibrary_t libs[kModuleParts] = {};   // one library per generated kernel (compiled in parallel)
     cudaKernel_t f_fwd = nullptr, f_rev_adam = nullptr, f_rev_eval = nullptr, f_hard = nullptr, f_init = nullptr;
     cudaKernel_t f_rev_sc = nullptr, f_fwd_adam = nullptr, f_adam_sc = nullptr;   // split-cone search kernels
     int P = 1, R = 1, rev_smem = 0, regs_fwd = 0, regs_rev = 0;   // cone groups, replicas per block
@@ -316,7 +322,8 @@ struct felix_space {
   int64_t prof_launches[4] = {0, 0, 0, 0};
   ~felix_space() {
     for (auto& e : prof) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
-    for (auto& kv : modules) if (kv.second.lib) cudaLibraryUnload(kv.second.lib);
+    for (auto& kv : modules)
+      for (cudaLibrary_t l : kv.second.libs) if (l) cudaLibraryUnload(l);
   }
 };
 
@@ -391,46 +398,76 @@ void build_round_tables(const SpaceDesc& d, RoundTables& t) {
     if (root_of[r] < 0) { root_of[r] = (int)comps.size(); comps.push_back({}); }
     comps[root_of[r]].push_back(j);
   }
-  const int64_t kMaxTuples = int64_t(1) << 22;
   for (auto& comp : comps) {
     if (comp.size() > 8) FELIX_THROW(FELIX_E_UNSUPPORTED, "split component with more than 8 variables");
     std::vector<int> sp;   // splits touching the component
     for (size_t s = 0; s < d.split_vars.size(); ++s)
       for (int v : d.split_vars[s]) if (std::find(comp.begin(), comp.end(), v) != comp.end()) { sp.push_back((int)s); break; }
+    if (sp.size() > static_cast<size_t>(kRoundMaxSplits))
+      FELIX_THROW(FELIX_E_UNSUPPORTED, "split component touching more than 16 splits");
+    auto in_split = [&](int q, int j) {
+      return std::find(d.split_vars[sp[q]].begin(), d.split_vars[sp[q]].end(), j) != d.split_vars[sp[q]].end();
+    };
     const int nv = (int)comp.size();
+    const int ci = (int)t.comp_nvars.size();
     t.comp_nvars.push_back(nv);
     t.comp_var0.push_back((int)t.comp_vars.size());
     for (int j : comp) t.comp_vars.push_back(j);
+    // branch-and-bound data (always built: felix_tune("round_bnb", 1) searches every component that way)
+    t.comp_ns.push_back((int)sp.size());
+    t.comp_s0.push_back((int)t.comp_sext.size());
+    for (int q : sp) t.comp_sext.push_back(d.split_extent[q]);
+    for (int j : comp) {
+      uint32_t mask = 0;
+      int64_t g = 0;
+      for (size_t q = 0; q < sp.size(); ++q)
+        if (in_split((int)q, j)) { mask |= 1u << q; g = std::gcd(g, d.split_extent[sp[q]]); }
+      t.var_smask.push_back(mask);
+      t.var_doff.push_back((int64_t)t.dval.size());
+      const auto dv = divisors(g);
+      t.var_dcnt.push_back((int32_t)dv.size());
+      for (int64_t x : dv) { t.dval.push_back(x); t.dln.push_back(std::log((double)x)); }
+    }
+    // the tuple table, in lexicographic order, unless it exceeds kRoundTableMax rows
     t.comp_toff.push_back(t.n_tuples_total);
     t.comp_eoff.push_back((int64_t)t.tuples.size());
+    const size_t tup0 = t.tuples.size();
     int64_t count = 0;
+    bool overflow = false;
     std::vector<int64_t> rem(sp.size());
     for (size_t q = 0; q < sp.size(); ++q) rem[q] = d.split_extent[sp[q]];
     std::vector<int32_t> cur(nv);
     std::function<void(int)> rec = [&](int k) {
+      if (overflow) return;
       if (k == nv) {
-        if (++count > kMaxTuples) FELIX_THROW(FELIX_E_UNSUPPORTED, "divisor-tuple table exceeds 2^22 rows");
+        if (++count > kRoundTableMax) { overflow = true; return; }
         for (int q = 0; q < nv; ++q) { t.tuples.push_back(cur[q]); t.lnf.push_back(std::log((double)cur[q])); }
         return;
       }
       const int j = comp[k];
       int64_t g = 0;
       for (size_t q = 0; q < sp.size(); ++q)
-        if (std::find(d.split_vars[sp[q]].begin(), d.split_vars[sp[q]].end(), j) != d.split_vars[sp[q]].end())
-          g = std::gcd(g, rem[q]);
+        if (in_split((int)q, j)) g = std::gcd(g, rem[q]);
       for (int64_t dv : divisors(g)) {
+        if (overflow) return;
         std::vector<int64_t> save = rem;
         for (size_t q = 0; q < sp.size(); ++q)
-          if (std::find(d.split_vars[sp[q]].begin(), d.split_vars[sp[q]].end(), j) != d.split_vars[sp[q]].end())
-            rem[q] /= dv;
+          if (in_split((int)q, j)) rem[q] /= dv;
         cur[k] = (int32_t)dv;
         rec(k + 1);
         rem = save;
       }
     };
     rec(0);
-    t.comp_tcount.push_back(count);
-    t.n_tuples_total += count;
+    if (overflow) {
+      t.tuples.resize(tup0);
+      t.lnf.resize(tup0);
+      t.comp_tcount.push_back(-1);
+      t.bnb_comps.push_back(ci);
+    } else {
+      t.comp_tcount.push_back(count);
+      t.n_tuples_total += count;
+    }
   }
   for (int j = 0; j < M; ++j) {
     if (d.vars[j].kind != FELIX_VAR_INT) continue;
@@ -443,12 +480,13 @@ void build_round_tables(const SpaceDesc& d, RoundTables& t) {
 }
 
 // ============================================================================ NVRTC
-static std::vector<char> nvrtc_compile(const std::string& source) {
+static std::vector<char> nvrtc_compile(const std::string& source, int part = 0) {
   nvrtcProgram prog;
   if (nvrtcCreateProgram(&prog, source.c_str(), "felix_space.cu", 0, nullptr, nullptr) != NVRTC_SUCCESS)
     FELIX_THROW(FELIX_E_NVRTC, "nvrtcCreateProgram failed");
-  const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "--fmad=true"};
-  nvrtcResult rc = nvrtcCompileProgram(prog, 4, opts);
+  const std::string def = "-DFELIX_PART=" + std::to_string(part);
+  const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "--fmad=true", def.c_str()};
+  nvrtcResult rc = nvrtcCompileProgram(prog, part > 0 ? 5 : 4, opts);
   if (rc != NVRTC_SUCCESS) {
     size_t ls = 0;
     nvrtcGetProgramLogSize(prog, &ls);
@@ -463,6 +501,45 @@ static std::vector<char> nvrtc_compile(const std::string& source) {
   nvrtcGetCUBIN(prog, cubin.data());
   nvrtcDestroyProgram(&prog);
   return cubin;
+}
+
+// The generated module's kernels, one NVRTC program each (codegen.cpp guards every kernel with
+// FELIX_PART == k): the eight compile on parallel host threads, ~3x faster than one program at C2
+// (7.5 s -> 2.7 s on 8 cores), and ptxas sees one kernel's straight-line code at a time.
+static const char* const kModuleKernels[kModuleParts] = {"felix_fwd", "felix_fwd_adam", "felix_rev_adam", "felix_rev_eval",
+                                                          "felix_rev_sc", "felix_adam_sc", "felix_hard", "felix_init"};
+
+// Process-wide cubin cache keyed by the generated source: spaces with the same expression DAG and
+// launch shape (a re-created space, the same subgraph in another task list) load the compiled kernels
+// instead of recompiling them.  Bounded; cleared wholesale when full.
+static std::mutex g_cubin_mu;
+static std::map<std::string, std::shared_ptr<const std::vector<std::vector<char>>>> g_cubins;
+
+static std::shared_ptr<const std::vector<std::vector<char>>> compile_module_parts(const std::string& source) {
+  {
+    std::lock_guard<std::mutex> lk(g_cubin_mu);
+    auto it = g_cubins.find(source);
+    if (it != g_cubins.end()) return it->second;
+  }
+  auto parts = std::make_shared<std::vector<std::vector<char>>>(kModuleParts);
+  std::vector<std::string> err(kModuleParts);
+  std::atomic<int> next{0};
+  auto worker = [&]() {
+    for (int k; (k = next.fetch_add(1)) < kModuleParts;) {
+      try { (*parts)[k] = nvrtc_compile(source, k + 1); } catch (const std::exception& e) { err[k] = e.what(); }
+    }
+  };
+  const int nt = std::max(1, std::min<int>(kModuleParts, static_cast<int>(std::thread::hardware_concurrency())));
+  std::vector<std::thread> th;
+  for (int t = 1; t < nt; ++t) th.emplace_back(worker);
+  worker();
+  for (auto& t : th) t.join();
+  for (int k = 0; k < kModuleParts; ++k)
+    if (!err[k].empty()) FELIX_THROW(FELIX_E_NVRTC, std::string(kModuleKernels[k]) + ": " + err[k]);
+  std::lock_guard<std::mutex> lk(g_cubin_mu);
+  if (g_cubins.size() >= 64) g_cubins.clear();
+  g_cubins.emplace(source, parts);
+  return parts;
 }
 
 static felix_space::Module& get_module(felix_space* s, int P, int R = 1, int dphi_parts = 1) {
@@ -482,16 +559,13 @@ static felix_space::Module& get_module(felix_space* s, int P, int R = 1, int dph
   s->flops_rev = info.flops_rev;
   mod.rev_smem = info.rev_smem_bytes;
   auto t0 = std::chrono::steady_clock::now();
-  std::vector<char> cubin = nvrtc_compile(mod.source);
-  CUDA_OK(cudaLibraryLoadData(&mod.lib, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0));
-  CUDA_OK(cudaLibraryGetKernel(&mod.f_fwd, mod.lib, "felix_fwd"));
-  CUDA_OK(cudaLibraryGetKernel(&mod.f_rev_adam, mod.lib, "felix_rev_adam"));
-  CUDA_OK(cudaLibraryGetKernel(&mod.f_rev_eval, mod.lib, "felix_rev_eval"));
-  CUDA_OK(cudaLibraryGetKernel(&mod.f_hard, mod.lib, "felix_hard"));
-  CUDA_OK(cudaLibraryGetKernel(&mod.f_init, mod.lib, "felix_init"));
-  CUDA_OK(cudaLibraryGetKernel(&mod.f_rev_sc, mod.lib, "felix_rev_sc"));
-  CUDA_OK(cudaLibraryGetKernel(&mod.f_fwd_adam, mod.lib, "felix_fwd_adam"));
-  CUDA_OK(cudaLibraryGetKernel(&mod.f_adam_sc, mod.lib, "felix_adam_sc"));
+  const auto cubins = compile_module_parts(mod.source);
+  cudaKernel_t* slots[kModuleParts] = {&mod.f_fwd, &mod.f_fwd_adam, &mod.f_rev_adam, &mod.f_rev_eval,
+                                       &mod.f_rev_sc, &mod.f_adam_sc, &mod.f_hard, &mod.f_init};
+  for (int k = 0; k < kModuleParts; ++k) {
+    CUDA_OK(cudaLibraryLoadData(&mod.libs[k], (*cubins)[k].data(), nullptr, nullptr, 0, nullptr, nullptr, 0));
+    CUDA_OK(cudaLibraryGetKernel(slots[k], mod.libs[k], kModuleKernels[k]));
+  }
   for (cudaKernel_t k : {mod.f_rev_adam, mod.f_rev_eval})
     CUDA_OK(cudaFuncSetAttribute(reinterpret_cast<const void*>(k), cudaFuncAttributeMaxDynamicSharedMemorySize, mod.rev_smem));
   cudaFuncAttributes fa{};
@@ -1029,6 +1103,12 @@ felix_status felix_space_create(int device, const felix_var* vars, int32_t n_var
   for (size_t q = 0; q < t.int_vars.size(); ++q) icnt.push_back(t.int_hi[q] - t.int_lo[q]);
   upload(s->d_int_vars, iv); upload(s->d_int_lo, t.int_lo); upload(s->d_int_cnt, icnt);
   upload(s->d_int_toff, t.int_toff); upload(s->d_int_thr, t.int_thr);
+  upload(s->d_comp_ns, t.comp_ns); upload(s->d_comp_s0, t.comp_s0); upload(s->d_comp_sext, t.comp_sext);
+  upload(s->d_var_smask, t.var_smask); upload(s->d_var_doff, t.var_doff); upload(s->d_var_dcnt, t.var_dcnt);
+  upload(s->d_dval, t.dval); upload(s->d_dln, t.dln); upload(s->d_bnb_sel, t.bnb_comps);
+  std::vector<int32_t> all_sel(t.comp_nvars.size());
+  std::iota(all_sel.begin(), all_sel.end(), 0);
+  upload(s->d_all_sel, all_sel);
   get_module(s.get(), 1);
   *out = s.release();
   FELIX_API_END
@@ -1056,7 +1136,7 @@ felix_status felix_codegen(const felix_var* vars, int32_t n_vars, const felix_sp
     const size_t nb = std::min<size_t>(code.size() + 1, static_cast<size_t>(src_cap));
     std::memcpy(src, code.c_str(), nb);
   }
-  if (compile) (void)nvrtc_compile(code);
+  if (compile) (void)compile_module_parts(code);
   FELIX_API_END
 }
 
@@ -1081,7 +1161,8 @@ felix_status felix_space_set_statements(felix_space* s, int32_t n_statements) {
   CUDA_OK(cudaDeviceSynchronize());
   s->desc.n_statements = n_statements;
   s->K0p = K0 <= 64 ? 64 : K0 <= 96 ? 96 : 128;
-  for (auto& kv : s->modules) if (kv.second.lib) cudaLibraryUnload(kv.second.lib);
+  for (auto& kv : s->modules)
+    for (cudaLibrary_t l : kv.second.libs) if (l) cudaLibraryUnload(l);
   s->modules.clear();
   s->search_chunks.reset();
   s->eval_chunks.reset();
@@ -1790,13 +1871,24 @@ static void do_round(felix_space* s, const float* y, int64_t n, int32_t* sched, 
   const int M = s->desc.n_vars;
   const int nc = static_cast<int>(s->rt.comp_nvars.size());
   const int ni = static_cast<int>(n);
-  if (nc > 0) {
+  const bool force_bnb = g_tune.round_bnb.load() != 0;
+  if (nc > 0 && !force_bnb) {
     const long long warps = static_cast<long long>(n) * nc;
     const unsigned grid = static_cast<unsigned>((warps * 32 + 255) / 256);
     round_split_kernel<<<grid, 256, 0, st>>>(y, ni, M, nc, s->d_comp_nvars.as<int>(), s->d_comp_var0.as<int>(),
                                              s->d_comp_vars.as<int>(), s->d_comp_eoff.as<long long>(),
                                              s->d_comp_tcount.as<long long>(), s->d_tuples.as<int>(),
                                              s->d_lnf.as<double>(), sched);
+    CUDA_OK(cudaGetLastError());
+  }
+  const int nb = force_bnb ? nc : static_cast<int>(s->rt.bnb_comps.size());
+  if (nb > 0) {
+    const long long tot = static_cast<long long>(n) * nb;
+    round_bnb_kernel<<<static_cast<unsigned>((tot + 127) / 128), 128, 0, st>>>(
+        y, ni, M, nb, (force_bnb ? s->d_all_sel : s->d_bnb_sel).as<int>(), s->d_comp_nvars.as<int>(),
+        s->d_comp_var0.as<int>(), s->d_comp_vars.as<int>(), s->d_comp_ns.as<int>(), s->d_comp_s0.as<int>(),
+        s->d_comp_sext.as<long long>(), s->d_var_smask.as<unsigned>(), s->d_var_doff.as<long long>(),
+        s->d_var_dcnt.as<int>(), s->d_dval.as<long long>(), s->d_dln.as<double>(), sched);
     CUDA_OK(cudaGetLastError());
   }
   const int nint = static_cast<int>(s->rt.int_vars.size());
@@ -2009,23 +2101,29 @@ felix_status felix_debug_trace(felix_space* s, uint64_t* out, int64_t n_words) {
   FELIX_API_BEGIN
   if (!s || !out) FELIX_THROW(FELIX_E_INVALID_ARG, "NULL argument");
   DeviceGuard dg(s->device);
-  for (auto it = s->modules.rbegin(); it != s->modules.rend(); ++it) {   // widest P first (the search's)
-    auto& kv = *it;
-    void* ptr = nullptr;
-    size_t bytes = 0;
-    if (cudaLibraryGetGlobal(&ptr, &bytes, kv.second.lib, "felix_trace") != cudaSuccess) {
-      cudaGetLastError();
-      continue;
+  // every kernel of a module is its own library with its own copy of the stamp arrays: read them all and
+  // take the elementwise max (%globaltimer is monotonic; a kernel leaves the other kernels' slots at 0)
+  auto read_max = [&](const felix_space::Module& m, const char* name, uint64_t* dst, size_t words) {
+    bool found = false;
+    std::vector<uint64_t> tmp(words);
+    std::fill(dst, dst + words, uint64_t(0));
+    for (cudaLibrary_t l : m.libs) {
+      void* ptr = nullptr;
+      size_t bytes = 0;
+      if (!l || cudaLibraryGetGlobal(&ptr, &bytes, l, name) != cudaSuccess) { cudaGetLastError(); continue; }
+      const size_t nw = std::min(words, bytes / 8);
+      CUDA_OK(cudaMemcpy(tmp.data(), ptr, nw * 8, cudaMemcpyDeviceToHost));
+      for (size_t i = 0; i < nw; ++i) dst[i] = std::max(dst[i], tmp[i]);
+      found = true;
     }
-    const size_t nb = std::min<size_t>(bytes, static_cast<size_t>(n_words) * 8);
-    CUDA_OK(cudaMemcpy(out, ptr, nb, cudaMemcpyDeviceToHost));
+    return found;
+  };
+  for (auto it = s->modules.rbegin(); it != s->modules.rend(); ++it) {   // widest P first (the search's)
+    const size_t tw = std::min<size_t>(2 * 8192 * 8, static_cast<size_t>(n_words));
+    if (!read_max(it->second, "felix_trace", out, tw)) continue;
     // then the per-warp cone-end stamps of the forward kernel, [8192][16], if the caller asked for them
-    void* wptr = nullptr;
-    size_t wbytes = 0;
-    if (static_cast<size_t>(n_words) * 8 > nb && cudaLibraryGetGlobal(&wptr, &wbytes, kv.second.lib, "felix_wtrace") == cudaSuccess)
-      CUDA_OK(cudaMemcpy(reinterpret_cast<char*>(out) + nb, wptr, std::min<size_t>(wbytes, static_cast<size_t>(n_words) * 8 - nb),
-                         cudaMemcpyDeviceToHost));
-    cudaGetLastError();
+    if (static_cast<size_t>(n_words) > tw)
+      read_max(it->second, "felix_wtrace", out + tw, std::min<size_t>(8192 * 16, static_cast<size_t>(n_words) - tw));
     return FELIX_OK;
   }
   FELIX_THROW(FELIX_E_UNSUPPORTED, "no trace buffer (felix_tune(\"trace\", 1) before the kernels are generated)");
@@ -2052,6 +2150,7 @@ felix_status felix_tune(const char* key, int32_t value) {
   else if (k == "codegen_cone_width") { in({-1, 1, 2, 4, 8, 16}); g_tune.codegen_P = value; }
   else if (k == "codegen_replicas") { in({-1, 1, 2, 4}); g_tune.codegen_R = value; }
   else if (k == "trace") { in({0, 1}); g_tune.trace = value; }
+  else if (k == "round_bnb") { in({0, 1}); g_tune.round_bnb = value; }
   else FELIX_THROW(FELIX_E_INVALID_ARG, "felix_tune: unknown key " + k);
   FELIX_API_END
 }

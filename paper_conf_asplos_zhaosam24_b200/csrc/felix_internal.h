@@ -73,8 +73,21 @@ struct RoundTables {
   std::vector<int32_t> int_vars;                  // INT variables
   std::vector<int64_t> int_lo, int_hi, int_toff;  // thresholds ln(k + 1/2), k in [lo, hi)
   std::vector<double> int_thr;
-  int64_t n_tuples_total = 0;
+  int64_t n_tuples_total = 0;                     // rows of the tuple tables (components searched by scan)
+  // branch-and-bound search (components with more than kRoundTableMax tuples, or all of them under
+  // felix_tune("round_bnb", 1)): per component its splits, per component var its split mask and the
+  // ascending divisors of the gcd of its splits' extents
+  std::vector<int32_t> comp_ns, comp_s0;          // per component: #splits touching it, offset into comp_sext
+  std::vector<int64_t> comp_sext;                 // extents of those splits
+  std::vector<uint32_t> var_smask;                // per comp_vars entry: bit q <=> var is in the component's split q
+  std::vector<int64_t> var_doff;                  // per comp_vars entry: offset of its divisor list
+  std::vector<int32_t> var_dcnt;
+  std::vector<int64_t> dval;                      // divisors (ascending) ...
+  std::vector<double> dln;                        // ... and their ln (host libm, as the tables)
+  std::vector<int32_t> bnb_comps;                 // components without a tuple table
 };
+constexpr int64_t kRoundTableMax = int64_t(1) << 16;   // larger components use the branch-and-bound kernel
+constexpr int kRoundMaxSplits = 16;                      // splits touching one component (B&B register state)
 void build_round_tables(const SpaceDesc& d, RoundTables& t);
 
 // -------------------------------------------------------------------------- codegen

@@ -242,3 +242,15 @@ def test_rnan_rounding_validity_topk(fx):
     idx, sc, sch = space.round_topk(cm, yt, 16)
     ridx, rsc, rsch = fo.round_topk(sp, mlp.W, mlp.b, y0, 16)
     assert np.array_equal(idx, ridx) and np.array_equal(sch, rsch) and np.all(sch[:, 0] >= 4)
+
+
+def test_module_cache_reuses_compiled_kernels(fx):
+    """A second space with the same DAG loads the process-wide cubin cache (felix_api.cu
+    compile_module_parts) instead of recompiling, and its kernels give bit-identical results."""
+    sp, mlp, space, cm = _setup(fx, "C1", lambda: fi.config("C1").spaces[0])
+    again = fx.Space(sp)
+    assert again.info.nvrtc_ms < 1000.0
+    y0 = torch.from_numpy(fi.make_y0(sp, 300, seed=5)).cuda()
+    a, b = space.eval(cm, y0, lam=1.0), again.eval(cm, y0, lam=1.0)
+    for key in ("phi", "cost", "loss", "grad"):
+        assert torch.equal(a[key], b[key]), key
