@@ -62,18 +62,42 @@ __global__ void __launch_bounds__(256) round_split_kernel(
 // the divisors of the var's gcd extent are visited outward from y_k (nearest first), a divisor is
 // taken only if it divides every remaining split extent the var belongs to, and a direction stops
 // as soon as partial + (y_k - ln d)^2 > best: the remaining terms are >= 0 and FP64 addition is
-// monotone, so every pruned tuple costs strictly more than the best found.  Leaves replace the best
+// monotone, so every pruned tuple costs strictly more than the best found.  A child is also skipped
+// when partial + LB > best, LB a lower bound of the remaining vars' cost under the product constraint
+// (ln f_j >= 0 and sum_{j in split q} ln f_j <= ln rem_q): per var (y_j < 0: y_j^2; y_j > ln rem: the
+// excess squared), and per split (sum of the positive y_j - ln rem_q)^2 / (their count) by Cauchy-Schwarz;
+// compared with a 1e-9 relative margin, far above the FP64 rounding of the leaf sums (~1e-15), so a
+// skipped subtree never holds a tuple that ties or beats the best.  Without it an eight-way split of
+// 720720 visits most of its 1.5e8 tuples.  Leaves replace the best
 // on a smaller cost or on an equal cost and a lexicographically smaller tuple, so the result is the
 // exhaustive scan's bit for bit.  Non-finite y anywhere in the component: every tuple costs inf / NaN
 // and the scan returns its first tuple, all ones; so does this kernel.
+// Exact lower bound for single-split components (every var tiles the same extent E): one warp per
+// (candidate, component) first fills V[k][r] = min over f | r of (y_k - ln f)^2 + V[k+1][r / f] (V[nv] = 0,
+// r over the divisors of E: the cost of vars k .. nv-1 when their product must divide r, a dynamic
+// programme over the remaining extent) in shared memory, lanes over r.  Lane 0 then takes the DP's own
+// argmin path as the first incumbent and runs the search above with the child test
+// (partial + (y_k - ln d)^2 + V[k+1][rem / d]) * (1 - 1e-12) > best: V is the exact optimum of the
+// remaining vars up to FP64 rounding (~1e-15 relative), so only near-ties of the best are visited and the
+// leaves -- summed left to right exactly as the table scan sums them -- decide, bit for bit.
+// Components touching several splits (or whose table would not fit) use the weaker bound above.
+__device__ __forceinline__ int bnb_div_index(const long long* __restrict__ D, int cnt, long long x) {
+  int a = 0, b = cnt - 1;
+  while (a < b) { const int m = (a + b) >> 1; if (D[m] < x) a = m + 1; else b = m; }
+  return a;
+}
+
 __global__ void __launch_bounds__(128) round_bnb_kernel(
     const float* __restrict__ y, int n, int M, int n_sel, const int* __restrict__ sel_comp,
     const int* __restrict__ comp_nvars, const int* __restrict__ comp_var0, const int* __restrict__ comp_vars,
     const int* __restrict__ comp_ns, const int* __restrict__ comp_s0, const long long* __restrict__ comp_sext,
     const unsigned* __restrict__ var_smask, const long long* __restrict__ var_doff, const int* __restrict__ var_dcnt,
-    const long long* __restrict__ dval, const double* __restrict__ dln, int* __restrict__ sched) {
-  const long long g = static_cast<long long>(blockIdx.x) * blockDim.x + threadIdx.x;
+    const long long* __restrict__ dval, const double* __restrict__ dln, int* __restrict__ sched, int dp_cap) {
+  extern __shared__ double bnb_smem[];
+  const long long g = (static_cast<long long>(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;   // warp per item
+  const int lane = threadIdx.x & 31;
   if (g >= static_cast<long long>(n) * n_sel) return;
+  double* V = bnb_smem + (threadIdx.x >> 5) * (dp_cap / 8);
   const int cand = static_cast<int>(g / n_sel), comp = sel_comp[g % n_sel];
   const int nv = comp_nvars[comp], v0 = comp_var0[comp], ns = comp_ns[comp];
   const int* vars = comp_vars + v0;
@@ -83,6 +107,29 @@ __global__ void __launch_bounds__(128) round_bnb_kernel(
     yv[k] = static_cast<double>(y[static_cast<size_t>(vars[k]) * n + cand]);
     finite = finite && isfinite(yv[k]);
   }
+  // the DP bound: one split, every var's divisor list = the divisors of E
+  const int nd = var_dcnt[v0];
+  const bool dp = finite && ns == 1 && (nv + 1) * nd * 8 <= dp_cap;
+  const long long* DE = dval + var_doff[v0];
+  const double* LE = dln + var_doff[v0];
+  if (dp) {
+    for (int i = lane; i < nd; i += 32) V[nv * nd + i] = 0.0;
+    __syncwarp();
+    for (int k = nv - 1; k >= 0; --k) {
+      for (int i = lane; i < nd; i += 32) {
+        const long long r = DE[i];
+        double m = DBL_MAX;
+        for (int j = 0; j <= i; ++j) {
+          if (r % DE[j] != 0) continue;
+          const double d = yv[k] - LE[j];
+          m = fmin(m, d * d + V[(k + 1) * nd + bnb_div_index(DE, nd, r / DE[j])]);
+        }
+        V[k * nd + i] = m;
+      }
+      __syncwarp();
+    }
+  }
+  if (lane != 0) return;
   long long bt[8];
   for (int k = 0; k < nv; ++k) bt[k] = 1;
   if (finite) {
@@ -93,6 +140,30 @@ __global__ void __launch_bounds__(128) round_bnb_kernel(
     long long cur[8];
     double best = DBL_MAX;
     bool found = false;
+    if (dp) {
+      // incumbent: the DP's argmin path (ties -> smallest divisor), its cost summed as the leaves are
+      long long r = rem[0];
+      double c = 0.0;
+      for (int k = 0; k < nv; ++k) {
+        const int ir = bnb_div_index(DE, nd, r);
+        double m = DBL_MAX;
+        long long fb = 1;
+        for (int j = 0; j <= ir; ++j) {
+          if (r % DE[j] != 0) continue;
+          const double d = yv[k] - LE[j];
+          const double v = d * d + V[(k + 1) * nd + bnb_div_index(DE, nd, r / DE[j])];
+          if (v < m) { m = v; fb = DE[j]; }
+        }
+        bt[k] = fb;
+        r /= fb;
+      }
+      for (int k = 0; k < nv; ++k) {
+        const double d = __dsub_rn(yv[k], LE[bnb_div_index(DE, nd, bt[k])]);
+        c = __dadd_rn(c, __dmul_rn(d, d));
+      }
+      best = c;
+      found = true;
+    }
     // position of y_k among the ascending ln d of var k: lo = last index with ln d < y, hi = lo + 1
     auto start = [&](int k) {
       const double* L = dln + var_doff[v0 + k];
@@ -152,6 +223,36 @@ __global__ void __launch_bounds__(128) round_bnb_kernel(
       }
       cur[k] = dv;
       for (int q = 0; q < ns; ++q) if (msk >> q & 1u) rem[q] /= dv;
+      double lb;
+      if (dp) {
+        lb = V[(k + 1) * nd + bnb_div_index(DE, nd, rem[0])];
+      } else {
+        // lower bound of the cost of vars k+1 .. nv-1 under the remaining extents
+        double lnr[16];
+        for (int q = 0; q < ns; ++q) lnr[q] = log(static_cast<double>(rem[q]));
+        double lb_var = 0.0, lb_neg = 0.0, lb_split = 0.0;
+        double psum[16];
+        int pcnt[16];
+        for (int q = 0; q < ns; ++q) { psum[q] = 0.0; pcnt[q] = 0; }
+        for (int j = k + 1; j < nv; ++j) {
+          const unsigned mj = var_smask[v0 + j];
+          const double yj = yv[j];
+          if (yj < 0.0) { lb_neg += yj * yj; continue; }
+          double cap = DBL_MAX;
+          for (int q = 0; q < ns; ++q)
+            if (mj >> q & 1u) { cap = fmin(cap, lnr[q]); psum[q] += yj; pcnt[q] += 1; }
+          if (yj > cap) lb_var += (yj - cap) * (yj - cap);
+        }
+        for (int q = 0; q < ns; ++q) {
+          const double ex = psum[q] - lnr[q];
+          if (pcnt[q] > 0 && ex > 0.0) lb_split = fmax(lb_split, ex * ex / pcnt[q]);
+        }
+        lb = fmax(lb_neg + lb_var, lb_neg + lb_split);
+      }
+      if ((e + lb) * (1.0 - 1e-9) > best) {     // nothing below this child can tie or beat the best
+        for (int q = 0; q < ns; ++q) if (msk >> q & 1u) rem[q] *= dv;
+        continue;
+      }
       acc[k + 1] = e;
       ++k;
       start(k);

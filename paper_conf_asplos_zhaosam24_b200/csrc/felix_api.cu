@@ -743,7 +743,7 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     if (head) {
       a.head_w = cm->head_w.as<float>();
       p->n_head_tiles = N / g.bn;
-      p->c_part.alloc(static_cast<size_t>(N / 32) * np * 4);      // room for any partial width >= 32
+      p->c_part.alloc(static_cast<size_t>(N / 16) * np * 4);      // room for any partial width >= 16
       a.c_part = p->c_part.as<float>();
       a.ld_c = static_cast<int>(np);
     } else {
@@ -819,6 +819,7 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     L.n_tiles = static_cast<int>(mt) * L.n_tiles_n;
     const int ccg = p->chain_cg;
     L.idesc = ptx::idesc_f16_f32(GEMM_BM * ccg, static_cast<uint32_t>(bn));
+    L.idesc_cat = ptx::idesc_f16_f32(GEMM_BM, static_cast<uint32_t>(2 * bn));   // [B_hi ; B_lo] (FELIX_CHAIN_NCAT, CG = 1)
     L.a_hi = g.a_hi; L.a_lo = g.a_lo; L.c_hi = g.c_hi; L.c_lo = g.c_lo;
     L.b_hi = make_tmap(g.w_hi, N, g.args.K, bn / ccg);     // CG = 2: each CTA loads half of the tile's weight rows
     L.b_lo = make_tmap(g.w_lo, N, g.args.K, bn / ccg);
@@ -832,7 +833,7 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
       L.b_hi = make_tmap(cm->WTs_hi.p, N, g.args.K, bn / ccg);
       L.b_lo = make_tmap(cm->WTs_lo.p, N, g.args.K, bn / ccg);
     }
-    if (g.epi == EPI_HEAD && use_chain()) p->n_head_tiles = 2 * (N / bn);   // chain: one partial per column half
+    if (g.epi == EPI_HEAD && use_chain()) p->n_head_tiles = CHAIN_EPI_NQ * (N / bn);   // chain: one partial per column slice
     max_tiles = std::max(max_tiles, static_cast<int>((mt + ccg - 1) / ccg) * L.n_tiles_n * L.ksplit * ccg);   // CTAs the layer can use
   }
   p->chain_grid = std::min(sms / p->chain_cg * p->chain_cg, max_tiles);
@@ -1883,12 +1884,23 @@ static void do_round(felix_space* s, const float* y, int64_t n, int32_t* sched, 
   }
   const int nb = force_bnb ? nc : static_cast<int>(s->rt.bnb_comps.size());
   if (nb > 0) {
-    const long long tot = static_cast<long long>(n) * nb;
-    round_bnb_kernel<<<static_cast<unsigned>((tot + 127) / 128), 128, 0, st>>>(
+    // warp per (candidate, component); the DP bound table of a single-split component ((nv + 1) x #divisors
+    // doubles) sits in shared memory, up to 24 KB per warp (components above that use the weaker bound)
+    int dp_cap = 0;
+    for (int i = 0; i < nb; ++i) {
+      const int c = force_bnb ? i : s->rt.bnb_comps[i];
+      if (s->rt.comp_ns[c] != 1) continue;
+      const int need = (s->rt.comp_nvars[c] + 1) * s->rt.var_dcnt[s->rt.comp_var0[c]] * 8;
+      if (need <= 24576) dp_cap = std::max(dp_cap, need);
+    }
+    dp_cap = (dp_cap + 15) / 16 * 16;
+    if (dp_cap * 4 > 48 * 1024) set_smem_attr(reinterpret_cast<const void*>(round_bnb_kernel), dp_cap * 4);
+    const long long tot = static_cast<long long>(n) * nb * 32;
+    round_bnb_kernel<<<static_cast<unsigned>((tot + 127) / 128), 128, dp_cap * 4, st>>>(
         y, ni, M, nb, (force_bnb ? s->d_all_sel : s->d_bnb_sel).as<int>(), s->d_comp_nvars.as<int>(),
         s->d_comp_var0.as<int>(), s->d_comp_vars.as<int>(), s->d_comp_ns.as<int>(), s->d_comp_s0.as<int>(),
         s->d_comp_sext.as<long long>(), s->d_var_smask.as<unsigned>(), s->d_var_doff.as<long long>(),
-        s->d_var_dcnt.as<int>(), s->d_dval.as<long long>(), s->d_dln.as<double>(), sched);
+        s->d_var_dcnt.as<int>(), s->d_dval.as<long long>(), s->d_dln.as<double>(), sched, dp_cap);
     CUDA_OK(cudaGetLastError());
   }
   const int nint = static_cast<int>(s->rt.int_vars.size());

@@ -39,8 +39,26 @@ constexpr int CHAIN_BN_MAX = 128;
 #endif
 constexpr int CHAIN_STAGES = FELIX_CHAIN_STAGES;
 constexpr int CHAIN_EPI_BUFS = CHAIN_STAGES >= 3 ? 1 : 2;   // epilogue staging buffers (double-buffered when smem allows)
-constexpr int CHAIN_THREADS = 320;
-constexpr int CHAIN_EPI_WARPS = 8;
+// Epilogue warps: 8 = two warps per TMEM lane quadrant, each draining a 32-column half of every 64-column
+// chunk (16 = four warps, 16-column slices).  Measured at C2 (tools/microbench/chain_trace.cu): 16 warps are
+// no faster (37.3 vs 37.4 us per chain): the chunk epilogue is bound by the SM sub-partitions' issue slots
+// (~8 instructions per element), not by per-warp latency.
+#ifndef FELIX_CHAIN_EPI_WARPS
+#define FELIX_CHAIN_EPI_WARPS 8
+#endif
+// NCAT = 1: the B tile of a stage is [B_hi ; B_lo] (2bn rows, contiguous), and the split product takes
+// two MMAs per K step instead of three: A_hi x [B_hi ; B_lo] (N = 2bn, accumulator columns [0, 2bn)) and
+// A_lo x B_hi (N = bn, accumulated into [0, bn)); the epilogue adds the two halves.  Shared-memory
+// operand reads per K step fall from 3(128 + bn) to (128 + 2bn) + (128 + bn) rows: the mainloop is bound
+// by the SM's shared-memory port (TMA writes + MMA operand reads), measured in tools/microbench/tma_ingest.cu.
+#ifndef FELIX_CHAIN_NCAT
+#define FELIX_CHAIN_NCAT 1
+#endif
+constexpr int CHAIN_EPI_WARPS = FELIX_CHAIN_EPI_WARPS;
+constexpr int CHAIN_THREADS = 64 + 32 * CHAIN_EPI_WARPS;
+constexpr int CHAIN_EPI_NQ = CHAIN_EPI_WARPS / 4;            // epilogue warps per TMEM lane quadrant
+constexpr int CHAIN_EPI_CPW = 64 / CHAIN_EPI_NQ;             // columns of each 64-column chunk per warp (16 or 32)
+static_assert(CHAIN_EPI_CPW == 16 || CHAIN_EPI_CPW == 32, "8 or 16 epilogue warps");
 constexpr int CHAIN_A_BYTES = GEMM_BM * GEMM_BK * 2;                 // 16 KB (one of hi / lo)
 #ifndef FELIX_CHAIN_STAGE_BN
 #define FELIX_CHAIN_STAGE_BN CHAIN_BN_MAX
@@ -50,9 +68,9 @@ constexpr int CHAIN_STAGE_BYTES = 2 * CHAIN_A_BYTES + 2 * CHAIN_B_BYTES;
 constexpr int CHAIN_EPI_BYTES = CHAIN_EPI_BUFS * 2 * GEMM_BM * 64 * 2;   // hi + lo staging of 64-col chunks
 constexpr int CHAIN_MAX_N = 1024;                                  // widest layer staged in smem (bias / head row)
 constexpr int CHAIN_PARAM_BYTES = 2 * CHAIN_MAX_N * 4;
-// ReLU mask words [buf][half][128 rows] and head partials [half][128 rows], staged for 1-D bulk copies so
+// ReLU mask words [buf][word][128 rows] and head partials [slice][128 rows], staged for 1-D bulk copies so
 // every global write of a tile goes through the async proxy (one bulk_wait before the row-block flag)
-constexpr int CHAIN_AUX_BYTES = CHAIN_EPI_BUFS * 2 * GEMM_BM * 4 + 2 * GEMM_BM * 4;
+constexpr int CHAIN_AUX_BYTES = CHAIN_EPI_BUFS * 2 * GEMM_BM * 4 + CHAIN_EPI_NQ * GEMM_BM * 4;
 constexpr int CHAIN_SMEM_BYTES = 1024 + CHAIN_STAGES * CHAIN_STAGE_BYTES + CHAIN_EPI_BYTES + CHAIN_PARAM_BYTES + CHAIN_AUX_BYTES + 256;
 
 struct ChainLayer {
@@ -60,6 +78,7 @@ struct ChainLayer {
   GemmArgs args;
   int epi, bn, n_tiles_n, n_tiles;     // tiles = m_tiles * n_tiles_n (n fastest)
   uint32_t idesc;
+  uint32_t idesc_cat;                  // M x 2bn (FELIX_CHAIN_NCAT, CG = 1)
   // reuse: this layer's A row block is the previous layer's output and every CTA keeps its row block from
   // one layer to the next (one tile per CTA in both, same N-tile count): the CTA's own previous output
   // chunks, still in its epilogue staging buffers in the A-operand layout (128-B swizzle, K-major), serve
@@ -148,7 +167,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
   float* s_bias = reinterpret_cast<float*>(epi_base + CHAIN_EPI_BYTES);   // [CHAIN_MAX_N] this layer's bias
   float* s_headw = s_bias + CHAIN_MAX_N;                                   // [CHAIN_MAX_N] head row (HEAD layer)
   uint32_t* s_mask = reinterpret_cast<uint32_t*>(epi_base + CHAIN_EPI_BYTES + CHAIN_PARAM_BYTES);   // [EPI_BUFS][2][128]
-  float* s_cpart = reinterpret_cast<float*>(s_mask + CHAIN_EPI_BUFS * 2 * GEMM_BM);                  // [2][128]
+  float* s_cpart = reinterpret_cast<float*>(s_mask + CHAIN_EPI_BUFS * 2 * GEMM_BM);                  // [NQ][128]
   uint64_t* full_bar = reinterpret_cast<uint64_t*>(epi_base + CHAIN_EPI_BYTES + CHAIN_PARAM_BYTES + CHAIN_AUX_BYTES);
   uint64_t* empty_bar = full_bar + CHAIN_STAGES;
   uint64_t* tfull = empty_bar + CHAIN_STAGES;      // [2] accumulator ready
@@ -159,6 +178,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const unsigned int G = gridDim.x;
+  constexpr bool ncat = FELIX_CHAIN_NCAT && CG == 1;
+  constexpr uint32_t ACC = ncat ? 2 * CHAIN_BN_MAX : CHAIN_BN_MAX;   // TMEM columns per accumulator buffer
   const uint32_t rank = CG == 2 ? ptx::cluster_ctarank() : 0u;
 
   auto a_hi = [&](int s) { return smem + s * CHAIN_STAGE_BYTES; };
@@ -174,8 +195,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
     ptx::fence_barrier_init();
   }
   if (warp == 1) {
-    if constexpr (CG == 2) ptx::tmem_alloc_cg2(tmem_slot, 2 * CHAIN_BN_MAX);
-    else ptx::tmem_alloc(tmem_slot, 2 * CHAIN_BN_MAX);
+    if constexpr (CG == 2) ptx::tmem_alloc_cg2(tmem_slot, 2 * ACC);
+    else ptx::tmem_alloc(tmem_slot, 2 * ACC);
   }
   ptx::tc_fence_before();
   if constexpr (CG == 2) ptx::cluster_sync();
@@ -226,6 +247,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         const int S = L.ksplit;
         const int nkb_all = (L.args.K + GEMM_BK - 1) / GEMM_BK;
         const int bnc = L.bn / CG;                                  // weight rows this CTA loads per tile
+        // NCAT: B lo rows follow the B hi rows ([B_hi ; B_lo] is one 2bn-row operand)
+        auto blo = [&](int s) { return ncat ? b_hi(s) + bnc * GEMM_BK * 2 : b_lo(s); };
         const uint32_t tx_b = 2 * (bnc * GEMM_BK * 2);
         const uint32_t tx = (L.a_exact ? 1 : 2) * CHAIN_A_BYTES + tx_b;
         ChainTiles<CG> tiles(L.n_tiles_n, P.m_tiles, S);
@@ -247,12 +270,13 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
               if (it >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], ((it / CHAIN_STAGES) - 1) & 1);
               arm(s, own ? tx_b : tx);
               load(b_hi(s), &L.b_hi, kb * GEMM_BK, nb, s);
-              load(b_lo(s), &L.b_lo, kb * GEMM_BK, nb, s);
+              load(blo(s), &L.b_lo, kb * GEMM_BK, nb, s);
               if (!own) {
                 if (!flag_ok) {
                   flag_wait(flag_of(l - 1, mb), epoch * static_cast<unsigned int>(Lp.n_tiles_n));
                   asm volatile("fence.proxy.async.global;" ::: "memory");
                   flag_ok = true;
+                  if (tile == tiles.first()) CHAIN_STAMP(l, 5);
                 }
                 load(a_hi(s), &L.a_hi, kb * GEMM_BK, m0, s);
                 if (!L.a_exact) load(a_lo(s), &L.a_lo, kb * GEMM_BK, m0, s);
@@ -269,10 +293,11 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
               if (it + kb >= CHAIN_STAGES) ptx::mbar_wait(&empty_bar[s], (((it + kb) / CHAIN_STAGES) - 1) & 1);
               arm(s, tx);
               load(b_hi(s), &L.b_hi, (kbeg + kb) * GEMM_BK, nb, s);
-              load(b_lo(s), &L.b_lo, (kbeg + kb) * GEMM_BK, nb, s);
+              load(blo(s), &L.b_lo, (kbeg + kb) * GEMM_BK, nb, s);
             }
             flag_wait(flag_of(l - 1, mb), epoch * static_cast<unsigned int>(P.layer[l - 1].n_tiles_n));
             asm volatile("fence.proxy.async.global;" ::: "memory");
+            if (tile == tiles.first()) CHAIN_STAMP(l, 5);
             for (int kb = 0; kb < pre; ++kb) {
               const int s = (it + kb) % CHAIN_STAGES;
               load(a_hi(s), &L.a_hi, (kbeg + kb) * GEMM_BK, m0, s);
@@ -289,7 +314,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             load(a_hi(s), &L.a_hi, k0, m0, s);
             if (!L.a_exact) load(a_lo(s), &L.a_lo, k0, m0, s);
             load(b_hi(s), &L.b_hi, k0, nb, s);
-            load(b_lo(s), &L.b_lo, k0, nb, s);
+            load(blo(s), &L.b_lo, k0, nb, s);
           }
         }
       }
@@ -310,7 +335,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
           const int acc = tcount & 1;
           if (tcount >= 2) wait_in(&tempty[acc], ((tcount >> 1) - 1) & 1);
           ptx::tc_fence_after();
-          const uint32_t d = tmem_base + acc * CHAIN_BN_MAX;
+          const uint32_t d = tmem_base + acc * ACC;
           const bool reuse = dataflow && l > 0 && L.reuse;
           const bool a_exact = L.a_exact != 0;
           int own0 = 0, nown = 0;
@@ -339,7 +364,11 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             for (int kk = 0; kk < GEMM_BK / GEMM_UMMA_K; ++kk) {
               const uint32_t off = kk * GEMM_UMMA_K * 2;
               const uint32_t acc0 = (i | kk) != 0;
-              if constexpr (CG == 2) {
+              if constexpr (ncat) {
+                // [A_hi x B_hi | A_hi x B_lo] in columns [0, 2bn), then A_lo x B_hi into [0, bn)
+                ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bh + off), L.idesc_cat, acc0);
+                if (!a_exact) ptx::mma_f16_ss(d, ptx::sdesc_k_sw128(al + off), ptx::sdesc_k_sw128(bh + off), L.idesc, 1u);
+              } else if constexpr (CG == 2) {
                 if (!a_exact) ptx::mma_f16_ss_cg2(d, ptx::sdesc_k_sw128(al + off), ptx::sdesc_k_sw128(bh + off), L.idesc, acc0);
                 ptx::mma_f16_ss_cg2(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bl + off), L.idesc, a_exact ? acc0 : 1u);
                 ptx::mma_f16_ss_cg2(d, ptx::sdesc_k_sw128(ah + off), ptx::sdesc_k_sw128(bh + off), L.idesc, 1u);
@@ -365,14 +394,38 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
       }
     }
   } else {
-    // ------------------------------------------------------------ epilogue warps 2..9 (both CTAs)
+    // ------------------------------------------------------------ epilogue warps 2.. (both CTAs)
+    constexpr int CPW = CHAIN_EPI_CPW, NQ = CHAIN_EPI_NQ;
     const int q = warp & 3;                          // TMEM lane quadrant this warp may access
-    const int half = (warp - 2) >> 2;                // which 32-column half of each 64-column chunk
+    const int sub = (warp - 2) >> 2;                 // which CPW-column slice of each 64-column chunk
+    const int cs = sub * CPW;
     const int r_tile = q * 32 + lane;
-    const int etid = threadIdx.x - 64;               // 0..255
+    const int etid = threadIdx.x - 64;
     int epi_count = 0;                               // 64-column chunks staged so far (buffer parity)
     constexpr int NEPI = CHAIN_EPI_WARPS * 32;
     int tcount = 0;
+    // CPW accumulator columns c .. c+CPW-1 of this thread's row (NCAT: the two halves summed)
+    auto acc_cols = [&](uint32_t t_row, int c, int bn, float (&v)[CPW]) {
+      if constexpr (ncat) {
+#pragma unroll
+        for (int h = 0; h < CPW; h += 16) {
+          float t[32];
+          ptx::tmem_ld2x16(t_row + c + h, t_row + bn + c + h, t);
+#pragma unroll
+          for (int i = 0; i < 16; ++i) v[h + i] = t[i] + t[16 + i];
+        }
+      } else if constexpr (CPW == 32) {
+        float t[32];
+        ptx::tmem_ld2x16(t_row + c, t_row + c + 16, t);
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = t[i];
+      } else {
+        float t[16];
+        ptx::tmem_ld16(t_row + c, t);
+#pragma unroll
+        for (int i = 0; i < 16; ++i) v[i] = t[i];
+      }
+    };
     for (int l = 0; l < P.n_layers; ++l) {
       const ChainLayer& L = P.layer[l];
       // per-layer fields in registers once: read through the dynamically indexed param block, the
@@ -410,7 +463,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         const int m0 = mb * GEMM_BM, n0 = (tq % ntn) * bn;
         const int row = m0 + r_tile;
         const bool row_ok = row < aM;
-        // this thread's mask words for the tile (<= 2 chunks of 64 columns), requested before the wait
+        // this thread's mask bits for the tile (<= 2 chunks of 64 columns), requested before the wait
         uint32_t mwords[CHAIN_BN_MAX / 64] = {0u};
         if (dataflow && epi == EPI_MASK) {
           // the mask words come from an earlier layer of this row block (other CTAs): acquire the
@@ -419,30 +472,25 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
           ptx::named_bar_sync(1, NEPI);
         }
         if (epi == EPI_MASK && row_ok) {
+          // written earlier in this launch by other CTAs: coherent L2 load, not the .nc path
 #pragma unroll
           for (int q64 = 0; q64 < CHAIN_BN_MAX / 64; ++q64)
-            if (q64 * 64 < bn) mwords[q64] = __ldcg(&mask_in[static_cast<size_t>((n0 + q64 * 64 + half * 32) / 32) * ld_mask + row]);
+            if (q64 * 64 < bn) mwords[q64] = __ldcg(&mask_in[static_cast<size_t>((n0 + q64 * 64 + cs) / 32) * ld_mask + row]) >> (cs & 31);
         }
         ptx::mbar_wait(&tfull[acc], (tcount >> 1) & 1);
         if (etid == 0 && tile == first_tile) CHAIN_STAMP(l, 3);
         ptx::tc_fence_after();
-        const uint32_t t_row = tmem_base + acc * CHAIN_BN_MAX + (static_cast<uint32_t>(q * 32) << 16);
+        const uint32_t t_row = tmem_base + acc * ACC + (static_cast<uint32_t>(q * 32) << 16);
         float head_acc = 0.f;
         if (epi == EPI_F32T) {
-          for (int c = half * 32; c < bn; c += 64) {
-            float v[32];
-            {
-              float a[16], b[16];
-              ptx::tmem_ld16(t_row + c, a);
-              ptx::tmem_ld16(t_row + c + 16, b);
-#pragma unroll
-              for (int i = 0; i < 16; ++i) { v[i] = a[i]; v[16 + i] = b[i]; }
-            }
+          for (int c = cs; c < bn; c += 64) {
+            float v[CPW];
+            acc_cols(t_row, c, bn, v);
             const int n = n0 + c;
             float* __restrict__ slab = out_f32 + static_cast<size_t>(part) * aN * ld_f32;
             if (row_ok) {
 #pragma unroll
-              for (int i = 0; i < 32; ++i)
+              for (int i = 0; i < CPW; ++i)
                 if (n + i < n_valid) slab[static_cast<size_t>(n + i) * ld_f32 + row] = v[i];
             }
           }
@@ -460,43 +508,49 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             const bool st0 = etid == 0 && c64 == 0 && tile == first_tile;
             if (st0) CHAIN_STAMP2(l, 0);
             {
-              const int c32 = half * 32;
-              const int c = c64 + c32;
-              float v[32];
-              {
-                float a[16], b[16];
-                ptx::tmem_ld16(t_row + c, a);
-                ptx::tmem_ld16(t_row + c + 16, b);
-#pragma unroll
-                for (int i = 0; i < 16; ++i) { v[i] = a[i]; v[16 + i] = b[i]; }
-              }
+              const int c = c64 + cs;
+              float v[CPW];
+              acc_cols(t_row, c, bn, v);
               if (st0) CHAIN_STAMP2(l, 1);
               const int n = n0 + c;
               if (epi == EPI_MASK) {
-                // written earlier in this launch by other CTAs: coherent L2 load, not the .nc path
                 const uint32_t bits = c64 == 0 ? mwords[0] : mwords[CHAIN_BN_MAX / 64 - 1];
 #pragma unroll
-                for (int i = 0; i < 32; ++i) v[i] = ((bits >> i) & 1u) ? v[i] : 0.f;
+                for (int i = 0; i < CPW; ++i) v[i] = ((bits >> i) & 1u) ? v[i] : 0.f;
               } else {
                 uint32_t bits = 0;
                 const bool head = epi == EPI_HEAD;
 #pragma unroll
-                for (int i = 0; i < 32; ++i) {
-                  const float z = v[i] + s_bias[n + i];
-                  const bool on = z > 0.f;
-                  bits |= (on ? 1u : 0u) << i;
-                  if (!head) {
-                    v[i] = on ? z : 0.f;
-                  } else {
-                    const float w = s_headw[n + i];
-                    head_acc += (on ? z : 0.f) * w;
-                    v[i] = on ? (hexact ? 1.f : -w) : 0.f;   // delta_{L-1} = W_L^T (dL/dc = -1) (.) [Z > 0]
+                for (int i4 = 0; i4 < CPW; i4 += 4) {
+                  const float4 b4 = *reinterpret_cast<const float4*>(s_bias + n + i4);
+                  const float bb[4] = {b4.x, b4.y, b4.z, b4.w};
+                  float ww[4] = {0.f, 0.f, 0.f, 0.f};
+                  if (head) {
+                    const float4 w4 = *reinterpret_cast<const float4*>(s_headw + n + i4);
+                    ww[0] = w4.x; ww[1] = w4.y; ww[2] = w4.z; ww[3] = w4.w;
+                  }
+#pragma unroll
+                  for (int u = 0; u < 4; ++u) {
+                    const int i = i4 + u;
+                    const float z = v[i] + bb[u];
+                    const bool on = z > 0.f;
+                    bits |= (on ? 1u : 0u) << i;
+                    if (!head) {
+                      v[i] = on ? z : 0.f;
+                    } else {
+                      head_acc += (on ? z : 0.f) * ww[u];
+                      v[i] = on ? (hexact ? 1.f : -ww[u]) : 0.f;   // delta_{L-1} = W_L^T (dL/dc = -1) (.) [Z > 0]
+                    }
                   }
                 }
-                if (!head) s_mask[(ebuf * 2 + half) * GEMM_BM + r_tile] = bits;
+                if (!head) {
+                  uint32_t* mw = s_mask + (ebuf * 2 + cs / 32) * GEMM_BM + r_tile;   // word (n0 + c64 + cs) / 32 of the row
+                  if constexpr (CPW == 32) *mw = bits;
+                  else reinterpret_cast<uint16_t*>(mw)[(cs >> 4) & 1] = static_cast<uint16_t>(bits);
+                }
               }
 #pragma unroll
-              for (int qq = 0; qq < 4; ++qq) {
+              for (int qq = 0; qq < CPW / 8; ++qq) {
                 // split 8 values into fp16 hi / lo with packed f16x2 converts
                 uint32_t h[4], lo[4];
 #pragma unroll
@@ -508,10 +562,10 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
                   h[u] = *reinterpret_cast<const uint32_t*>(&hh);
                   lo[u] = *reinterpret_cast<const uint32_t*>(&ll);
                 }
-                const int q16 = c32 / 8 + qq;
+                const int q16 = cs / 8 + qq;
                 const uint32_t off = r_tile * 128 + ((q16 ^ (r_tile & 7)) << 4);
                 *reinterpret_cast<uint4*>(epi_hi + off) = make_uint4(h[0], h[1], h[2], h[3]);
-                *reinterpret_cast<uint4*>(epi_lo + off) = make_uint4(lo[0], lo[1], lo[2], lo[3]);
+                if (!hexact) *reinterpret_cast<uint4*>(epi_lo + off) = make_uint4(lo[0], lo[1], lo[2], lo[3]);
               }
             }
             if (st0) CHAIN_STAMP2(l, 2);
@@ -530,17 +584,18 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
             }
           }
         }
-        // head partial per (N tile, column half); the reverse kernel sums all 2 * N / bn partials.  Staged in
+        // head partial per (N tile, column slice); the reverse kernel sums all NQ * N / bn partials.  Staged in
         // shared memory and bulk-copied (rows m0 .. m0+127; c_part has padded rows)
         if (epi == EPI_HEAD) {
           if (etid == 0) ptx::bulk_wait_read<0>();          // the previous tile's copy has read s_cpart
           ptx::named_bar_sync(1, NEPI);
-          s_cpart[half * GEMM_BM + r_tile] = head_acc;
+          s_cpart[sub * GEMM_BM + r_tile] = head_acc;
           ptx::fence_proxy_async_smem();
           ptx::named_bar_sync(1, NEPI);
           if (etid == 0) {
-            ptx::bulk_s2g(c_part + static_cast<size_t>(2 * (n0 / bn)) * ld_c + m0, s_cpart, GEMM_BM * 4);
-            ptx::bulk_s2g(c_part + static_cast<size_t>(2 * (n0 / bn) + 1) * ld_c + m0, s_cpart + GEMM_BM, GEMM_BM * 4);
+#pragma unroll
+            for (int j = 0; j < NQ; ++j)
+              ptx::bulk_s2g(c_part + static_cast<size_t>(NQ * (n0 / bn) + j) * ld_c + m0, s_cpart + j * GEMM_BM, GEMM_BM * 4);
             ptx::bulk_commit();
           }
         }
@@ -554,6 +609,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
           ptx::bulk_wait<0>();
           asm volatile("fence.proxy.async.global;" ::: "memory");
           asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(flag_of(l, mb)) : "memory");
+          if (tile == first_tile) CHAIN_STAMP(l, 6);
         }
       }
       // ---- layer end: all of this CTA's outputs complete + visible, then the grid barrier
@@ -577,8 +633,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
   if constexpr (CG == 2) ptx::cluster_sync();
   else __syncthreads();
   if (warp == 1) {
-    if constexpr (CG == 2) ptx::tmem_dealloc_cg2(tmem_base, 2 * CHAIN_BN_MAX);
-    else ptx::tmem_dealloc(tmem_base, 2 * CHAIN_BN_MAX);
+    if constexpr (CG == 2) ptx::tmem_dealloc_cg2(tmem_base, 2 * ACC);
+    else ptx::tmem_dealloc(tmem_base, 2 * ACC);
   }
 }
 
