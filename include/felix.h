@@ -221,6 +221,20 @@ FELIX_EXPORT felix_status felix_history_topk(felix_space* s, felix_costmodel* m,
                                 int32_t* step_out, double* score_out, int32_t* sched_out, int32_t* n_out,
                                 int64_t* n_unique_out, void* stream);
 
+/* Multi-GPU exchange: candidates shard across ranks with no per-step communication
+ * (Eq. 4 is a sum over seeds, Adam is elementwise); each rank's local top-k
+ * records are all-gathered once and merged identically on every rank with this call.  Inputs are HOST
+ * arrays of n_rows gathered records: key[n_rows] (the order key: global candidate index for
+ * felix_round_topk, step * 2^40 + global index for felix_history_topk; < 0 marks an empty row),
+ * score[n_rows] (FP64), sched[n_rows][n_vars] (int32).  Output: the best k distinct schedules by
+ * (score desc, key asc), a schedule held by several rows kept once with its first row in that order
+ * (a NaN score orders last) -- for any sharding, the single-process top-k of the union.  key_out[k],
+ * score_out[k], sched_out[k][n_vars] HOST, caller-owned; *n_out = rows written (<= k).  Host only (no
+ * device, no stream).  FELIX_E_INVALID_ARG on NULL pointers with n_rows > 0, n_vars < 1 or k < 0. */
+FELIX_EXPORT felix_status felix_merge_topk(const int64_t* key, const double* score, const int32_t* sched,
+                              int64_t n_rows, int32_t n_vars, int32_t k, int64_t* key_out, double* score_out,
+                              int32_t* sched_out, int32_t* n_out);
+
 /* ---------------------------------------------------------------- test hooks (same kernels)
  * felix_eval: one objective + gradient evaluation, no Adam.  y device [n_vars][n].  Outputs (device,
  * any may be NULL): phi [n_features][n] (slog features), g [R][n] (user roots then automatic roots),

@@ -30,7 +30,7 @@ EXPORTED = ["felix_last_error", "felix_abi_version", "felix_space_create", "feli
             "felix_search", "felix_round_topk", "felix_eval", "felix_round", "felix_score",
             "felix_init_sample", "felix_profile_enable", "felix_profile_read", "felix_profile_reset",
             "felix_debug_trace", "felix_history_topk", "felix_space_set_statements", "felix_search_group",
-            "felix_eval_ex", "felix_tune"]
+            "felix_eval_ex", "felix_tune", "felix_merge_topk"]
 
 
 class FelixError(RuntimeError):
@@ -162,6 +162,26 @@ def search_group(spaces: Sequence["Space"], cm: "CostModel", ys, n_steps: int, *
 _TUNE_KEYS = ("mlp", "cone_width", "replicas", "sc_warps", "chunks", "split_cone", "tile_cta_group", "chain_cta_group", "dphi_ksplit",
               "codegen_cone_width", "codegen_replicas", "trace", "round_bnb")
 _TUNE_DEFAULT = {k: (0 if k in ("trace", "round_bnb") else -1) for k in _TUNE_KEYS}
+
+
+def merge_topk(key, score, sched, k: int):
+    """felix_merge_topk: deterministic merge of gathered top-k records (host arrays; rows with key < 0
+    are empty).  Returns (key int64 [m], score float64 [m], sched int32 [m, n_vars]), m <= k."""
+    import numpy as np
+    key = np.ascontiguousarray(key, dtype=np.int64)
+    score = np.ascontiguousarray(score, dtype=np.float64)
+    sched = np.ascontiguousarray(sched, dtype=np.int32)
+    if sched.ndim != 2 or key.shape != (sched.shape[0],) or score.shape != key.shape:
+        raise FelixError(1, "merge_topk: key [R], score [R], sched [R, n_vars] expected")
+    n_vars = max(int(sched.shape[1]), 1)
+    ko = np.zeros(k, np.int64)
+    so = np.zeros(k, np.float64)
+    xo = np.zeros((k, n_vars), np.int32)
+    m = ctypes.c_int32(0)
+    _check(_lib.felix_merge_topk(key.ctypes.data_as(_P), score.ctypes.data_as(_P), sched.ctypes.data_as(_P),
+                                 ctypes.c_int64(key.shape[0]), ctypes.c_int32(n_vars), ctypes.c_int32(k),
+                                 ko.ctypes.data_as(_P), so.ctypes.data_as(_P), xo.ctypes.data_as(_P), ctypes.byref(m)))
+    return ko[:m.value], so[:m.value], xo[:m.value]
 
 
 def tune(**knobs) -> None:

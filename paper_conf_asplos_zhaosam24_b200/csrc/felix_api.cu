@@ -1081,6 +1081,37 @@ static std::unique_ptr<felix_space> parse_space(const felix_var* vars, int32_t n
 extern "C" {
 
 const char* felix_last_error(void) { return g_last_error.c_str(); }
+
+felix_status felix_merge_topk(const int64_t* key, const double* score, const int32_t* sched, int64_t n_rows,
+                              int32_t n_vars, int32_t k, int64_t* key_out, double* score_out, int32_t* sched_out,
+                              int32_t* n_out) {
+  FELIX_API_BEGIN
+  if (n_vars < 1 || k < 0 || n_rows < 0 || !n_out) FELIX_THROW(FELIX_E_INVALID_ARG, "felix_merge_topk: bad sizes");
+  if (n_rows > 0 && (!key || !score || !sched)) FELIX_THROW(FELIX_E_INVALID_ARG, "felix_merge_topk: NULL input");
+  if (k > 0 && (!key_out || !score_out || !sched_out)) FELIX_THROW(FELIX_E_INVALID_ARG, "felix_merge_topk: NULL output");
+  std::vector<int64_t> rows;
+  for (int64_t r = 0; r < n_rows; ++r) if (key[r] >= 0) rows.push_back(r);
+  // (score desc, key asc); NaN scores after every number
+  std::sort(rows.begin(), rows.end(), [&](int64_t a, int64_t b) {
+    const bool na = std::isnan(score[a]), nb = std::isnan(score[b]);
+    if (na != nb) return nb;
+    if (!na && score[a] != score[b]) return score[a] > score[b];
+    return key[a] < key[b];
+  });
+  std::set<std::vector<int32_t>> seen;
+  int32_t m = 0;
+  for (int64_t r : rows) {
+    if (m >= k) break;
+    std::vector<int32_t> sv(sched + r * n_vars, sched + (r + 1) * n_vars);
+    if (!seen.insert(sv).second) continue;
+    key_out[m] = key[r];
+    score_out[m] = score[r];
+    std::copy(sv.begin(), sv.end(), sched_out + static_cast<int64_t>(m) * n_vars);
+    ++m;
+  }
+  *n_out = m;
+  FELIX_API_END
+}
 int32_t felix_abi_version(void) { return FELIX_ABI_VERSION; }
 
 felix_status felix_space_create(int device, const felix_var* vars, int32_t n_vars, const felix_split* splits,

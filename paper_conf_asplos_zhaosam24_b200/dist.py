@@ -10,7 +10,7 @@ each schedule's smallest index, the merged list equals the single-GPU top-k of t
 """
 from __future__ import annotations
 
-from typing import List, Tuple
+from typing import Tuple
 
 import numpy as np
 
@@ -27,21 +27,10 @@ def pack_records(idx: np.ndarray, score: np.ndarray, sched: np.ndarray, k: int, 
 
 
 def merge_records(rows: np.ndarray, k: int) -> Tuple[np.ndarray, np.ndarray, np.ndarray]:
-    """Deterministic host merge of gathered records [R, 2 + n_vars]."""
-    rows = rows[rows[:, 0] >= 0]
-    order = sorted(range(len(rows)), key=lambda r: (-rows[r, 1], rows[r, 0]))
-    seen = {}
-    keep: List[int] = []
-    for r in order:
-        key = rows[r, 2:].astype(np.int64).tobytes()
-        if key in seen:
-            continue
-        seen[key] = r
-        keep.append(r)
-        if len(keep) == k:
-            break
-    sel = rows[keep]
-    return sel[:, 0].astype(np.int64), sel[:, 1], sel[:, 2:].astype(np.int32)
+    """Deterministic merge of gathered records [R, 2 + n_vars] through the C ABI (felix_merge_topk):
+    dedup by schedule, order (score desc, global index asc), best k."""
+    from . import merge_topk
+    return merge_topk(rows[:, 0].astype(np.int64), rows[:, 1], rows[:, 2:].astype(np.int32), k)
 
 
 def allgather_topk(idx, score, sched, k: int, n_vars: int, group=None, device=None):

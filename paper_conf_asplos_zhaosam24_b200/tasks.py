@@ -161,22 +161,10 @@ def merge_task_records(gathered: np.ndarray, n_tasks: int, k: int, n_vars: Seque
     world = gathered.shape[0] // (n_tasks * k)
     g = gathered.reshape(world, n_tasks, k, -1)
     out = {}
+    from . import merge_topk
     for t in range(n_tasks):
         rows = g[:, t].reshape(world * k, -1)
-        rows = rows[rows[:, 0] >= 0]
-        order = sorted(range(len(rows)), key=lambda r: (-rows[r, 1], rows[r, 0]))
-        seen = set()
-        keep: List[int] = []
-        for r in order:
-            key = rows[r, 2:2 + n_vars[t]].astype(np.int64).tobytes()
-            if key in seen:
-                continue
-            seen.add(key)
-            keep.append(r)
-            if len(keep) == k:
-                break
-        sel = rows[keep]
-        out[t] = (sel[:, 0].astype(np.int64), sel[:, 1], sel[:, 2:2 + n_vars[t]].astype(np.int32))
+        out[t] = merge_topk(rows[:, 0].astype(np.int64), rows[:, 1], rows[:, 2:2 + n_vars[t]].astype(np.int32), k)
     return out
 
 

@@ -22,14 +22,11 @@ def _free_port() -> int:
 
 
 def _load_dist_module():
-    """paper_conf_asplos_zhaosam24_b200/dist.py without importing the package (no .so needed)."""
-    import importlib.util
-    spec = importlib.util.spec_from_file_location(
-        "felix_dist", os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
-                                   "paper_conf_asplos_zhaosam24_b200", "dist.py"))
-    m = importlib.util.module_from_spec(spec)
-    spec.loader.exec_module(m)
-    return m
+    """paper_conf_asplos_zhaosam24_b200.dist (the merge runs in libfelix's host code: felix_merge_topk)."""
+    import __graft_entry__
+    __graft_entry__.build()
+    from paper_conf_asplos_zhaosam24_b200 import dist
+    return dist
 
 
 def _worker(rank, world, port, y_all, k, out):

@@ -165,3 +165,30 @@ def test_split_cone_reverse_is_fp32_and_forward_keeps_fp64_values(fx):
     assert "const double" not in rev and "sf_tail(" in rev and "sf_dSh(" in rev and "const float c" in rev
     fwd = src[src.index("void fwd_body("):src.index('extern "C" __global__ void __launch_bounds__(PG * 32 * NREP) felix_fwd(')]
     assert "sm_Sf(" in fwd and "const double v" in fwd
+
+
+def test_merge_topk_host_call_against_brute_force(fx):
+    """felix_merge_topk (the multi-GPU exchange's merge, host code in libfelix) against a brute-force
+    reference: rank every row by (score desc, key asc; NaN last), keep the first row of each schedule."""
+    rng = np.random.default_rng(5)
+    for trial in range(20):
+        R, nv, k = int(rng.integers(0, 40)), int(rng.integers(1, 5)), int(rng.integers(0, 12))
+        key = rng.permutation(1000)[:R].astype(np.int64)
+        key[rng.random(R) < 0.15] = -1                                   # empty rows
+        sched = rng.integers(1, 3, size=(R, nv)).astype(np.int32)        # many duplicate schedules
+        score = np.round(rng.normal(size=R), 1)                          # many equal scores
+        score[rng.random(R) < 0.1] = np.nan
+        rows = [r for r in range(R) if key[r] >= 0]
+        rows.sort(key=lambda r: (np.isnan(score[r]), -score[r] if not np.isnan(score[r]) else 0.0, key[r]))
+        seen, ref = set(), []
+        for r in rows:
+            t = tuple(sched[r])
+            if t in seen:
+                continue
+            seen.add(t)
+            ref.append(r)
+        ref = ref[:k]
+        ko, so, xo = fx.merge_topk(key, score, sched.reshape(R, nv), k)
+        assert list(ko) == [key[r] for r in ref]
+        assert np.array_equal(so, score[ref], equal_nan=True)
+        assert np.array_equal(xo, sched[ref].reshape(len(ref), nv))

@@ -16,15 +16,11 @@ from oracle import felix_oracle as fo
 
 
 def _load_tasks_module():
-    """paper_conf_asplos_zhaosam24_b200/tasks.py without importing the package (no .so needed)."""
-    import importlib.util
-    spec = importlib.util.spec_from_file_location(
-        "felix_tasks", os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
-                                    "paper_conf_asplos_zhaosam24_b200", "tasks.py"))
-    m = importlib.util.module_from_spec(spec)
-    sys.modules["felix_tasks"] = m               # dataclasses resolve annotations through sys.modules
-    spec.loader.exec_module(m)
-    return m
+    """paper_conf_asplos_zhaosam24_b200.tasks (its per-task merge runs in libfelix: felix_merge_topk)."""
+    import __graft_entry__
+    __graft_entry__.build()
+    from paper_conf_asplos_zhaosam24_b200 import tasks
+    return tasks
 
 
 ft = _load_tasks_module()
