@@ -634,6 +634,19 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     }
     o << ind << "  default: break;\n" << ind << "}\n";
   };
+  // the automatic-root terms of dL/dy_j computed inside var j's case (felix_fwd_adam: a thread needs only
+  // the autos of its own vars; the loss itself is not formed there, only its finiteness matters)
+  auto emit_auto_grad_switch_inline = [&](const char* ind) {
+    o << ind << "switch (j) {\n";
+    for (int j = 0; j < M; ++j) {
+      std::string terms;
+      for (size_t q = 0; q < autos.size(); ++q)
+        for (auto& tv : autos[q].terms)
+          if (tv.first == j) terms += std::string(tv.second > 0 ? " + " : " - ") + "fmax(" + autos[q].val + ", 0.0)";
+      if (!terms.empty()) o << ind << "  case " << j << ": gd += 2.0 * dlam * (0.0" << terms << "); break;\n";
+    }
+    o << ind << "  default: break;\n" << ind << "}\n";
+  };
   o << "template <int ADAM>\n__device__ __forceinline__ void fwd_body(float* yv, int n, int ldy, u16* __restrict__ phi_hi, u16* __restrict__ phi_lo, int* step_ctr,\n"
     << "    float* mv, float* vv, const float* __restrict__ part, const double* __restrict__ pen, const float* __restrict__ c_part,\n"
     << "    int n_head_tiles, int ld_c, float head_b, float lam, float lr, float b1, float b2, float eps) {\n"
@@ -670,23 +683,24 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "#pragma unroll 4\n    for (int i = 0; i < NS * n_head_tiles; ++i) cst += c_part[(size_t)(i % n_head_tiles) * ld_c + (size_t)(i / n_head_tiles) * n + cc];\n"
     << "    const int s_ = *step_ctr - 1;   // Adam steps to apply: reverse kernels run so far (the counter starts at 1)\n"
     << "#pragma unroll\n    for (int jj = 0; jj < NJ; ++jj) { const int j = wq + PG * jj; if (j >= NV) break; sy[j][lane] = yl[jj]; }\n"
-    << "    __syncthreads();\n"
+    << "    __syncthreads();\n    TSTAMP(0, 5);\n"
     << "    if (s_ <= 0) {\n"
     << "#pragma unroll\n      for (int jj = 0; jj < NJ; ++jj) { const int j = wq + PG * jj; if (j >= NV) break; sx[j][lane] = exp((double)yl[jj]); }\n"
     << "    } else {\n"
     << "      const double dlam = (double)lam;\n";
-  emit_autos("      ", "sy");
-  o << "      const float loss = (float)(-(double)cst + dlam * pen_);\n"
-    << "      bool ok = isfinite(loss);\n"
+  // the loss -C + lam (user penalties + auto penalties) is finite iff C and the user penalties are (the
+  // auto penalties are finite for finite y; a non-finite y makes its own gradient non-finite)
+  for (int j = 0; j < M; ++j) o << "      const double y" << j << " = (double)sy[" << j << "][lane];\n";
+  o << "      bool ok = isfinite(cst) && isfinite(pen_);\n"
     << "      float gyv[NJ];\n"
     << "#pragma unroll\n      for (int jj = 0; jj < NJ; ++jj) {\n"
     << "        const int j = wq + PG * jj;\n        if (j >= NV) break;\n"
     << "        double gd = (double)gxa[jj];   // the partials are dL/dy already (x_j folded in by felix_rev_sc)\n";
-  emit_auto_grad_switch("        ");
+  emit_auto_grad_switch_inline("        ");
   o << "        gyv[jj] = (float)gd;\n        ok = ok && isfinite(gyv[jj]);\n      }\n"
     << "      const unsigned bad = __ballot_sync(0xffffffffu, !ok);\n"
     << "      if (lane == 0) sbad[wq] = bad;\n"
-    << "      __syncthreads();\n"
+    << "      __syncthreads();\n      TSTAMP(0, 6);\n"
     << "      unsigned anybad = 0;\n#pragma unroll\n      for (int q = 0; q < PG; ++q) anybad |= sbad[q];\n"
     << "      const bool okall = !((anybad >> lane) & 1u);\n"
     << "      const float bc1 = 1.f - powf(b1, (float)s_), bc2 = 1.f - powf(b2, (float)s_);\n"
@@ -702,7 +716,7 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "        }\n"
     << "        sx[j][lane] = exp((double)yy);\n      }\n"
     << "    }\n  }\n"
-    << "  for (int k = tid; k < NS * 32 * (K0P + 1); k += PG * 32) (&sphi[0][0][0])[k] = 0.f;\n"
+    << "  TSTAMP(0, 7);\n  for (int k = tid; k < NS * 32 * (K0P + 1); k += PG * 32) (&sphi[0][0][0])[k] = 0.f;\n"
     << "  __syncthreads();\n  TSTAMP(0, 2);\n";
   for (int q = 0; q < P; ++q) {
     o << "  if (wq == " << q << ") {\n";

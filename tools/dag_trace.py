@@ -30,6 +30,8 @@ q = lambda a: [round(float(np.min(a)) / 1e3, 2), round(float(np.median(a)) / 1e3
 out = {"config": cfg.name, "n": n, "fwd_blocks": len(f), "rev_blocks": len(r),
        "fwd_us_rel_min_med_max": {"start": q(f[:, 0] - t0), "after_wait": q(f[:, 1] - t0), "after_adam": q(f[:, 2] - t0),
                                   "after_compute": q(f[:, 3] - t0), "end": q(f[:, 4] - t0)},
+       "fwd_adam_parts_us_med": {"loads_to_sync1": q(f[:, 5] - f[:, 1])[1], "loss_ballot_sync2": q(f[:, 6] - f[:, 5])[1],
+                                 "adam_exp": q(f[:, 7] - f[:, 6])[1], "zero_phi_sync3": q(f[:, 2] - f[:, 7])[1]},
        "fwd_phase_us_med": {"wait": q(f[:, 1] - f[:, 0])[1], "adam_prologue": q(f[:, 2] - f[:, 1])[1],
                             "cones": q(f[:, 3] - f[:, 2])[1], "phi_store": q(f[:, 4] - f[:, 3])[1]},
        "rev_us_rel_min_med_max": {"start": q(r[:, 0] - t0), "after_wait": q(r[:, 1] - t0), "after_compute": q(r[:, 2] - t0),
