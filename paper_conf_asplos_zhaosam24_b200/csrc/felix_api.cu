@@ -826,7 +826,7 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     L.b_hi = make_tmap(g.w_hi, N, g.args.K, bn / ccg);     // CG = 2: each CTA loads half of the tile's weight rows
     L.b_lo = make_tmap(g.w_lo, N, g.args.K, bn / ccg);
     // the first backward layer takes the 0/1 mask of the head layer as its A operand and the head row
-    // folded into its weights (exact A: two MMA passes, no A lo loads); FELIX_MASK_EXACT=0 disables
+    // folded into its weights (exact A: no A lo loads, one N-concatenated MMA per K step)
     L.a_exact = 0;
     L.head_exact = 0;
     if (i == static_cast<size_t>(cm->n_layers - 1) && i > 0 && p->gemms[i - 1].epi == EPI_HEAD) {

@@ -520,24 +520,33 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
               } else {
                 uint32_t bits = 0;
                 const bool head = epi == EPI_HEAD;
+                // two separate loops: a runtime `head` inside one loop is if-converted, so ReLU layers would
+                // execute the head arithmetic too (~16 instead of ~8 instructions per element)
+                if (!head) {
 #pragma unroll
-                for (int i4 = 0; i4 < CPW; i4 += 4) {
-                  const float4 b4 = *reinterpret_cast<const float4*>(s_bias + n + i4);
-                  const float bb[4] = {b4.x, b4.y, b4.z, b4.w};
-                  float ww[4] = {0.f, 0.f, 0.f, 0.f};
-                  if (head) {
-                    const float4 w4 = *reinterpret_cast<const float4*>(s_headw + n + i4);
-                    ww[0] = w4.x; ww[1] = w4.y; ww[2] = w4.z; ww[3] = w4.w;
-                  }
+                  for (int i4 = 0; i4 < CPW; i4 += 4) {
+                    const float4 b4 = *reinterpret_cast<const float4*>(s_bias + n + i4);
+                    const float bb[4] = {b4.x, b4.y, b4.z, b4.w};
 #pragma unroll
-                  for (int u = 0; u < 4; ++u) {
-                    const int i = i4 + u;
-                    const float z = v[i] + bb[u];
-                    const bool on = z > 0.f;
-                    bits |= (on ? 1u : 0u) << i;
-                    if (!head) {
+                    for (int u = 0; u < 4; ++u) {
+                      const int i = i4 + u;
+                      const float z = v[i] + bb[u];
+                      const bool on = z > 0.f;
+                      bits |= (on ? 1u : 0u) << i;
                       v[i] = on ? z : 0.f;
-                    } else {
+                    }
+                  }
+                } else {
+#pragma unroll
+                  for (int i4 = 0; i4 < CPW; i4 += 4) {
+                    const float4 b4 = *reinterpret_cast<const float4*>(s_bias + n + i4);
+                    const float4 w4 = *reinterpret_cast<const float4*>(s_headw + n + i4);
+                    const float bb[4] = {b4.x, b4.y, b4.z, b4.w}, ww[4] = {w4.x, w4.y, w4.z, w4.w};
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                      const int i = i4 + u;
+                      const float z = v[i] + bb[u];
+                      const bool on = z > 0.f;
                       head_acc += (on ? z : 0.f) * ww[u];
                       v[i] = on ? (hexact ? 1.f : -ww[u]) : 0.f;   // delta_{L-1} = W_L^T (dL/dc = -1) (.) [Z > 0]
                     }
