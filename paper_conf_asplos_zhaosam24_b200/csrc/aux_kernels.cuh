@@ -522,6 +522,85 @@ __global__ void __launch_bounds__(1024) topk_select_kernel(
   }
 }
 
+// The same selection with the block's entries (score, order key, candidate, alive, schedule) staged in
+// shared memory once: the k rounds then touch no global memory (each round of the kernel above pays
+// dependent L2 round trips for the scores and the winner's schedule compare).  Identical results.
+__global__ void __launch_bounds__(1024) topk_select_smem_kernel(
+    long long n_entries, long long chunk, const int* __restrict__ cand_of, const long long* __restrict__ okey,
+    const double* __restrict__ score, const unsigned char* __restrict__ valid, const int* __restrict__ sched, int M,
+    int k, int* __restrict__ out_cand, int* __restrict__ out_cnt) {
+  extern __shared__ double tk_smem[];
+  __shared__ TopkKey red[32];
+  __shared__ TopkKey win;
+  const long long c0 = static_cast<long long>(blockIdx.x) * chunk;
+  const int ne = static_cast<int>(min(n_entries, c0 + chunk) - c0);
+  double* s_sc = tk_smem;                                            // [chunk]
+  long long* s_ok = reinterpret_cast<long long*>(s_sc + chunk);      // [chunk]
+  int* s_c = reinterpret_cast<int*>(s_ok + chunk);                   // [chunk]
+  int* s_sched = s_c + chunk;                                        // [chunk][M]
+  unsigned char* s_alive = reinterpret_cast<unsigned char*>(s_sched + chunk * M);   // [chunk]
+  for (int e = threadIdx.x; e < ne; e += blockDim.x) {
+    const int c = cand_of ? cand_of[c0 + e] : static_cast<int>(c0 + e);
+    const bool live = c >= 0 && valid[c] && isfinite(score[c]);
+    s_alive[e] = live ? 1 : 0;
+    s_c[e] = c;
+    s_sc[e] = live ? score[c] : 0.0;
+    s_ok[e] = live ? (okey ? okey[c] : static_cast<long long>(c)) : 0;
+    for (int j = 0; j < M; ++j) s_sched[e * M + j] = live ? sched[static_cast<size_t>(c) * M + j] : 0;
+  }
+  __syncthreads();
+  int r = 0;
+  for (; r < k; ++r) {
+    TopkKey best{0.0, 0, -1};
+    int bestE = -1;
+    for (int e = threadIdx.x; e < ne; e += blockDim.x) {
+      if (!s_alive[e]) continue;
+      const TopkKey t{s_sc[e], s_ok[e], s_c[e]};
+      if (topk_better(t, best)) { best = t; bestE = e; }
+    }
+    // carry the entry index in the key's candidate slot's shadow: reduce on (score, order key) as above
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      const TopkKey o = topk_shfl(best, off);
+      const int oe = __shfl_xor_sync(0xffffffffu, bestE, off);
+      if (topk_better(o, best)) { best = o; bestE = oe; }
+    }
+    __shared__ int redE[32];
+    __shared__ int winE;
+    if ((threadIdx.x & 31) == 0) { red[threadIdx.x >> 5] = best; redE[threadIdx.x >> 5] = bestE; }
+    __syncthreads();
+    if (threadIdx.x < 32) {
+      const bool has = threadIdx.x < (blockDim.x + 31) / 32;
+      TopkKey b = has ? red[threadIdx.x] : TopkKey{0.0, 0, -1};
+      int be = has ? redE[threadIdx.x] : -1;
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) {
+        const TopkKey o = topk_shfl(b, off);
+        const int oe = __shfl_xor_sync(0xffffffffu, be, off);
+        if (topk_better(o, b)) { b = o; be = oe; }
+      }
+      if (threadIdx.x == 0) { win = b; winE = be; }
+    }
+    __syncthreads();
+    const TopkKey w = win;
+    if (w.c < 0) break;
+    if (threadIdx.x == 0) out_cand[blockIdx.x * static_cast<long long>(k) + r] = w.c;
+    const int* ws = s_sched + winE * M;
+    for (int e = threadIdx.x; e < ne; e += blockDim.x) {
+      if (!s_alive[e]) continue;
+      const int* cs = s_sched + e * M;
+      bool same = true;
+      for (int j = 0; j < M; ++j) same = same && (cs[j] == ws[j]);
+      if (same) s_alive[e] = 0;
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    out_cnt[blockIdx.x] = r;
+    for (int q = r; q < k; ++q) out_cand[blockIdx.x * static_cast<long long>(k) + q] = -1;
+  }
+}
+
 // ---------------------------------------------------------------------------- K8 history (Alg. 1 l.13/17/20)
 // One thread per seed, run on the rounded point sigma_x_i at which step i's objective is evaluated
 // (before the fwd kernel bumps step_ctr to i+1).  A seed whose rounded schedule equals its previous

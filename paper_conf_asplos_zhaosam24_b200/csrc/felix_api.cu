@@ -309,6 +309,9 @@ struct felix_space {
   std::unique_ptr<felix::Chunks> search_chunks, eval_chunks;
   std::unique_ptr<felix::GroupCache> group_cache;   // felix_search_group with this space first
   felix::DevBuf sched, valid, phi64, score, act64a, act64b, alive, rec_cand, rec_cnt, fin_cand, fin_cnt, o_idx, o_score, o_sched;
+  felix::DevBuf o_pack;                       // felix_round_topk outputs, one contiguous block: [count | idx | score | sched]
+  void* h_pack = nullptr;                     // pinned host copy of o_pack (one D2H copy per call)
+  size_t h_pack_bytes = 0;
   // varValuesHistory (Alg. 1 l.13/17) of the last search run with history != 0: per-step rounded points,
   // each seed's previous schedule, the schedule hash set and the pool of distinct schedules
   felix::DevBuf h_sched, h_last, h_slot_h, h_slot_i, h_pool_sched, h_pool_key, h_cnt, o_step;   // h_cnt: count, overflow
@@ -321,6 +324,7 @@ struct felix_space {
   double prof_ms[4] = {0, 0, 0, 0};
   int64_t prof_launches[4] = {0, 0, 0, 0};
   ~felix_space() {
+    if (h_pack) cudaFreeHost(h_pack);
     for (auto& e : prof) { cudaEventDestroy(e.a); cudaEventDestroy(e.b); }
     for (auto& kv : modules)
       for (cudaLibrary_t l : kv.second.libs) if (l) cudaLibraryUnload(l);
@@ -1950,6 +1954,24 @@ static void do_round(felix_space* s, const float* y, int64_t n, int32_t* sched, 
 // (k rounds of block argmax + dedup), the second phase merges the blocks' lists.  Enough blocks to run
 // the rounds in parallel (C2: 8 blocks of 512 instead of one of 4096), few enough that the single-block
 // merge stays short.
+// one top-k selection phase: the shared-memory kernel when the block's entries fit (<= 96 KB), else the
+// global-memory one (identical results)
+static void launch_topk_select(long long nblk, long long n_entries, long long chunk, const int* cand_of,
+                               const long long* okey, const double* score, const uint8_t* valid, const int32_t* sched,
+                               int M, int k, uint8_t* alive, int* out_cand, int* out_cnt, cudaStream_t st) {
+  const long long bytes = chunk * (8 + 8 + 4 + 4LL * M + 1);
+  if (bytes <= 96 * 1024) {
+    const int b = static_cast<int>((bytes + 15) / 16 * 16);
+    if (b > 48 * 1024) set_smem_attr(reinterpret_cast<const void*>(topk_select_smem_kernel), 96 * 1024);
+    topk_select_smem_kernel<<<static_cast<unsigned>(nblk), 1024, b, st>>>(n_entries, chunk, cand_of, okey, score, valid,
+                                                                            sched, M, k, out_cand, out_cnt);
+  } else {
+    topk_select_kernel<<<static_cast<unsigned>(nblk), 1024, 0, st>>>(n_entries, chunk, cand_of, okey, score, valid,
+                                                                       sched, M, k, alive, out_cand, out_cnt);
+  }
+  CUDA_OK(cudaGetLastError());
+}
+
 static long long topk_chunk(long long n) {
   long long c = (n + 63) / 64;
   c = (c + 255) / 256 * 256;
@@ -2056,28 +2078,37 @@ felix_status felix_round_topk(felix_space* s, felix_costmodel* m, const float* y
   ensure(s->rec_cand, static_cast<size_t>(nblk) * k * 4);
   ensure(s->rec_cnt, static_cast<size_t>(nblk) * 4);
   ensure(s->fin_cand, static_cast<size_t>(k) * 4);
-  ensure(s->fin_cnt, 4);
-  topk_select_kernel<<<static_cast<unsigned>(nblk), 1024, 0, st>>>(
-      n, chunk, nullptr, nullptr, s->score.as<double>(), s->valid.as<uint8_t>(), s->sched.as<int32_t>(), M, k,
-      s->alive.as<uint8_t>(), s->rec_cand.as<int>(), s->rec_cnt.as<int>());
-  CUDA_OK(cudaGetLastError());
-  topk_select_kernel<<<1, 1024, 0, st>>>(
-      nblk * k, nblk * k, s->rec_cand.as<int>(), nullptr, s->score.as<double>(), s->valid.as<uint8_t>(), s->sched.as<int32_t>(),
-      M, k, s->alive.as<uint8_t>(), s->fin_cand.as<int>(), s->fin_cnt.as<int>());
-  CUDA_OK(cudaGetLastError());
-  ensure(s->o_idx, static_cast<size_t>(k) * 8);
-  ensure(s->o_score, static_cast<size_t>(k) * 8);
-  ensure(s->o_sched, static_cast<size_t>(k) * M * 4);
+  // outputs packed in one device block and read back with a single copy into pinned memory:
+  // [count (8 B) | idx k x 8 | score k x 8 | sched k x M x 4]
+  const size_t pack_bytes = 8 + static_cast<size_t>(k) * 16 + static_cast<size_t>(k) * M * 4;
+  ensure(s->o_pack, pack_bytes);
+  if (s->h_pack_bytes < pack_bytes) {
+    if (s->h_pack) cudaFreeHost(s->h_pack);
+    s->h_pack = nullptr;
+    s->h_pack_bytes = 0;
+    CUDA_OK(cudaHostAlloc(&s->h_pack, pack_bytes, cudaHostAllocDefault));
+    s->h_pack_bytes = pack_bytes;
+  }
+  uint8_t* pk = s->o_pack.as<uint8_t>();
+  int* p_cnt = reinterpret_cast<int*>(pk);
+  long long* p_idx = reinterpret_cast<long long*>(pk + 8);
+  double* p_score = reinterpret_cast<double*>(pk + 8 + static_cast<size_t>(k) * 8);
+  int32_t* p_sched = reinterpret_cast<int32_t*>(pk + 8 + static_cast<size_t>(k) * 16);
+  launch_topk_select(nblk, n, chunk, nullptr, nullptr, s->score.as<double>(), s->valid.as<uint8_t>(), s->sched.as<int32_t>(),
+                     M, k, s->alive.as<uint8_t>(), s->rec_cand.as<int>(), s->rec_cnt.as<int>(), st);
+  launch_topk_select(1, nblk * k, nblk * k, s->rec_cand.as<int>(), nullptr, s->score.as<double>(), s->valid.as<uint8_t>(),
+                     s->sched.as<int32_t>(), M, k, s->alive.as<uint8_t>(), s->fin_cand.as<int>(), p_cnt, st);
   topk_gather_kernel<<<1, std::max(32, (k + 31) / 32 * 32), 0, st>>>(
-      s->fin_cand.as<int>(), s->fin_cnt.as<int>(), k, s->score.as<double>(), s->sched.as<int32_t>(), M, index_base,
-      s->o_idx.as<long long>(), s->o_score.as<double>(), s->o_sched.as<int32_t>());
+      s->fin_cand.as<int>(), p_cnt, k, s->score.as<double>(), s->sched.as<int32_t>(), M, index_base,
+      p_idx, p_score, p_sched);
   CUDA_OK(cudaGetLastError());
-  int cnt = 0;
-  CUDA_OK(cudaMemcpyAsync(&cnt, s->fin_cnt.p, 4, cudaMemcpyDeviceToHost, st));
-  CUDA_OK(cudaMemcpyAsync(idx_out, s->o_idx.p, static_cast<size_t>(k) * 8, cudaMemcpyDeviceToHost, st));
-  CUDA_OK(cudaMemcpyAsync(score_out, s->o_score.p, static_cast<size_t>(k) * 8, cudaMemcpyDeviceToHost, st));
-  CUDA_OK(cudaMemcpyAsync(sched_out, s->o_sched.p, static_cast<size_t>(k) * M * 4, cudaMemcpyDeviceToHost, st));
+  CUDA_OK(cudaMemcpyAsync(s->h_pack, pk, pack_bytes, cudaMemcpyDeviceToHost, st));
   CUDA_OK(cudaStreamSynchronize(st));
+  const uint8_t* hp = static_cast<const uint8_t*>(s->h_pack);
+  const int cnt = *reinterpret_cast<const int*>(hp);
+  std::memcpy(idx_out, hp + 8, static_cast<size_t>(k) * 8);
+  std::memcpy(score_out, hp + 8 + static_cast<size_t>(k) * 8, static_cast<size_t>(k) * 8);
+  std::memcpy(sched_out, hp + 8 + static_cast<size_t>(k) * 16, static_cast<size_t>(k) * M * 4);
   *n_out = cnt;
   FELIX_API_END
 }
@@ -2115,14 +2146,10 @@ felix_status felix_history_topk(felix_space* s, felix_costmodel* m, int32_t k, i
   ensure(s->fin_cand, static_cast<size_t>(k) * 4);
   ensure(s->fin_cnt, 4);
   const long long* key = s->h_pool_key.as<long long>();
-  topk_select_kernel<<<static_cast<unsigned>(nblk), 1024, 0, st>>>(
-      n, chunk, nullptr, key, s->score.as<double>(), s->valid.as<uint8_t>(), sched, M, k,
-      s->alive.as<uint8_t>(), s->rec_cand.as<int>(), s->rec_cnt.as<int>());
-  CUDA_OK(cudaGetLastError());
-  topk_select_kernel<<<1, 1024, 0, st>>>(
-      nblk * k, nblk * k, s->rec_cand.as<int>(), key, s->score.as<double>(), s->valid.as<uint8_t>(), sched,
-      M, k, s->alive.as<uint8_t>(), s->fin_cand.as<int>(), s->fin_cnt.as<int>());
-  CUDA_OK(cudaGetLastError());
+  launch_topk_select(nblk, n, chunk, nullptr, key, s->score.as<double>(), s->valid.as<uint8_t>(), sched, M, k,
+                     s->alive.as<uint8_t>(), s->rec_cand.as<int>(), s->rec_cnt.as<int>(), st);
+  launch_topk_select(1, nblk * k, nblk * k, s->rec_cand.as<int>(), key, s->score.as<double>(), s->valid.as<uint8_t>(), sched,
+                     M, k, s->alive.as<uint8_t>(), s->fin_cand.as<int>(), s->fin_cnt.as<int>(), st);
   ensure(s->o_idx, static_cast<size_t>(k) * 8);
   ensure(s->o_step, static_cast<size_t>(k) * 4);
   ensure(s->o_score, static_cast<size_t>(k) * 8);
