@@ -291,6 +291,7 @@ FELIX_EXPORT felix_status felix_init_sample(felix_space* s, int64_t n, uint64_t 
  *   "trace"               0/1: per-block %globaltimer stamps in kernels generated afterwards
  *   "round_bnb"           0/1: 1 = every split component is rounded by the branch-and-bound kernel
  *                         (default 0: only components with more than 65536 divisor tuples are)
+ *   "graph_steps"         Adam steps captured per search graph: 1..1000 (default 20)
  * FELIX_E_INVALID_ARG for an unknown key or value. */
 FELIX_EXPORT felix_status felix_tune(const char* key, int32_t value);
 

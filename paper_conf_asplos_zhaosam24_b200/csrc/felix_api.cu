@@ -145,7 +145,8 @@ struct Tuning {
   std::atomic<int> dphi_ksplit{-1};  // layer chain: split-K parts of the dL/dphi layer (1, 2, 4)
   std::atomic<int> codegen_P{-1}, codegen_R{-1};   // felix_codegen's variant
   std::atomic<int> trace{0};         // per-block %globaltimer stamps in kernels generated afterwards
-  std::atomic<int> round_bnb{0};     // 1: every split component rounds by branch and bound (test hook)
+  std::atomic<int> round_bnb{0};
+  std::atomic<int> graph_steps{-1};  // Adam steps per search graph (-1: kGraphSteps)     // 1: every split component rounds by branch and bound (test hook)
 };
 static Tuning g_tune;
 
@@ -235,6 +236,7 @@ static void launch_chain(const Plan& p, cudaStream_t st) {
 // The population split into K independent chunks, each with its own workspace (Plan).  One Adam
 // step of all chunks is captured as ONE CUDA graph with K parallel branches (fork/join), so one
 // chunk's tensor-core GEMMs overlap another chunk's latency-bound expression kernels.
+constexpr int kGraphSteps = 20;   // Adam steps captured per search graph (see felix_search)
 struct Chunks {
   const CostModel* cm = nullptr;
   uint64_t cm_uid = 0;
@@ -243,7 +245,9 @@ struct Chunks {
   std::vector<int64_t> off, cnt;
   std::vector<std::unique_ptr<Plan>> plans;
   std::vector<cudaStream_t> streams;       // capture-time branch streams / per-chunk launch streams
-  cudaGraphExec_t graph = nullptr;
+  cudaGraphExec_t graph = nullptr;            // kGraphSteps Adam steps per launch
+  cudaGraphExec_t graph_tail = nullptr;       // the remainder (n_steps % kGraphSteps steps)
+  int graph_tail_steps = 0;
   std::vector<double> graph_key;
   std::vector<cudaGraphExec_t> chunk_graphs;   // independent per-chunk step graphs (no per-step join)
   std::vector<double> chunk_key;
@@ -251,6 +255,7 @@ struct Chunks {
   std::vector<cudaEvent_t> ev_join;
   ~Chunks() {
     if (graph) cudaGraphExecDestroy(graph);
+    if (graph_tail) cudaGraphExecDestroy(graph_tail);
     for (auto g : chunk_graphs) if (g) cudaGraphExecDestroy(g);
     if (ev_fork) cudaEventDestroy(ev_fork);
     for (auto e : ev_join) cudaEventDestroy(e);
@@ -1414,7 +1419,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
       void* pen = pl.sc_pen.p;
       void* fa[] = {&yk, &ni, &ldy, &phh, &phl, &ctr, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hbv, &lam, &lr, &b1, &b2, &eps};
       prof_mark(s, 0, cs, true);
-      launch_grouped(mod.f_fwd_adam, mod.P, mod.R, cnt, 0, fa, cs, true);
+      launch_grouped(mod.f_fwd_adam, mod.P, mod.R, cnt, 0, fa, cs, false);   // no PDL edge from the previous step's reverse (measured slower)
       prof_mark(s, 0, cs, false);
       s->prof_launches[0] += 1;
       run_mlp(s, pl, cs);
@@ -1505,14 +1510,17 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
                                      static_cast<double>(s->h_mask), static_cast<double>(s->h_cap),
                                      static_cast<double>(sc), static_cast<double>(scw), static_cast<double>(mod.R),
                                      ptr(ch.plans[0]->sc_part.p), ptr(ch.plans[0]->sc_pen.p)};
-    if (!ch.graph || ch.graph_key != key) {
-      if (ch.graph) { cudaGraphExecDestroy(ch.graph); ch.graph = nullptr; }
+    // Several Adam steps per graph: inside one graph the programmatic (PDL) edges also link step t's
+    // reverse kernel to step t+1's forward, and the graph launch cost is paid once per kGraphSteps steps
+    // (between graph launches the next step waits for the whole previous graph).
+    auto build = [&](int steps) {
       while (static_cast<int>(ch.streams.size()) < nck) {
         cudaStream_t b;
         CUDA_OK(cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking));
         ch.streams.push_back(b);
       }
       cudaGraph_t graph = nullptr;
+      cudaGraphExec_t exec = nullptr;
       cudaEvent_t fork, join[16];
       CUDA_OK(cudaEventCreateWithFlags(&fork, cudaEventDisableTiming));
       for (int k = 0; k < nck; ++k) CUDA_OK(cudaEventCreateWithFlags(&join[k], cudaEventDisableTiming));
@@ -1521,13 +1529,17 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
       int64_t saved[4];
       std::copy(s->prof_launches, s->prof_launches + 4, saved);
       try {
-        if (s->h_valid) history_step(cap);
-        CUDA_OK(cudaEventRecord(fork, cap));
-        for (int k = 1; k < nck; ++k) CUDA_OK(cudaStreamWaitEvent(ch.streams[k], fork, 0));
-        for (int k = 0; k < nck; ++k) chunk_step(k, ch.streams[k]);
-        for (int k = 1; k < nck; ++k) {
-          CUDA_OK(cudaEventRecord(join[k], ch.streams[k]));
-          CUDA_OK(cudaStreamWaitEvent(cap, join[k], 0));
+        for (int i = 0; i < steps; ++i) {
+          if (s->h_valid) history_step(cap);
+          if (nck > 1) {
+            CUDA_OK(cudaEventRecord(fork, cap));
+            for (int k = 1; k < nck; ++k) CUDA_OK(cudaStreamWaitEvent(ch.streams[k], fork, 0));
+          }
+          for (int k = 0; k < nck; ++k) chunk_step(k, ch.streams[k]);
+          for (int k = 1; k < nck; ++k) {
+            CUDA_OK(cudaEventRecord(join[k], ch.streams[k]));
+            CUDA_OK(cudaStreamWaitEvent(cap, join[k], 0));
+          }
         }
         std::copy(saved, saved + 4, s->prof_launches);
       } catch (...) {
@@ -1538,18 +1550,36 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
         throw;
       }
       CUDA_OK(cudaStreamEndCapture(cap, &graph));
-      cudaError_t ie = cudaGraphInstantiate(&ch.graph, graph, 0);
+      cudaError_t ie = cudaGraphInstantiate(&exec, graph, 0);
       cudaGraphDestroy(graph);
       cudaEventDestroy(fork);
       for (int k = 0; k < nck; ++k) cudaEventDestroy(join[k]);
       CUDA_OK(ie);
-      ch.graph_key = key;
+      return exec;
+    };
+    const int gs_t = g_tune.graph_steps.load();
+    const int gs = static_cast<int>(std::min<int64_t>(gs_t >= 1 ? gs_t : kGraphSteps, p->n_steps));
+    const int tail = static_cast<int>(p->n_steps % gs);
+    std::vector<double> key_s = key;
+    key_s.push_back(static_cast<double>(gs));
+    if (!ch.graph || ch.graph_key != key_s) {
+      if (ch.graph) { cudaGraphExecDestroy(ch.graph); ch.graph = nullptr; }
+      if (ch.graph_tail) { cudaGraphExecDestroy(ch.graph_tail); ch.graph_tail = nullptr; }
+      ch.graph_tail_steps = 0;
+      ch.graph = build(gs);
+      ch.graph_key = key_s;
     }
-    for (int t = 1; t <= p->n_steps; ++t) {
-      if (t % 100000 == 0)   // keep the grid-barrier counter far from 2^32 on very long searches
+    if (tail > 0 && ch.graph_tail_steps != tail) {
+      if (ch.graph_tail) { cudaGraphExecDestroy(ch.graph_tail); ch.graph_tail = nullptr; }
+      ch.graph_tail = build(tail);
+      ch.graph_tail_steps = tail;
+    }
+    for (int64_t t = 0; t + gs <= p->n_steps; t += gs) {
+      if (t % 100000 < gs && t > 0)   // keep the grid-barrier counter far from 2^32 on very long searches
         for (auto& pl : ch.plans) CUDA_OK(cudaMemsetAsync(pl->grid_bar.p, 0, pl->grid_bar.bytes, st));
       CUDA_OK(cudaGraphLaunch(ch.graph, st));
     }
+    if (tail > 0) CUDA_OK(cudaGraphLaunch(ch.graph_tail, st));
     s->prof_launches[0] += static_cast<int64_t>(p->n_steps) * nck;
     s->prof_launches[1] += static_cast<int64_t>(p->n_steps) * nck *
                            (ch.plans[0]->mode == MLP_LAYERS ? static_cast<int64_t>(ch.plans[0]->gemms.size()) : 1);
@@ -2223,6 +2253,7 @@ felix_status felix_tune(const char* key, int32_t value) {
   else if (k == "codegen_replicas") { in({-1, 1, 2, 4}); g_tune.codegen_R = value; }
   else if (k == "trace") { in({0, 1}); g_tune.trace = value; }
   else if (k == "round_bnb") { in({0, 1}); g_tune.round_bnb = value; }
+  else if (k == "graph_steps") { if (value != -1 && (value < 1 || value > 1000)) in({}); g_tune.graph_steps = value; }
   else FELIX_THROW(FELIX_E_INVALID_ARG, "felix_tune: unknown key " + k);
   FELIX_API_END
 }

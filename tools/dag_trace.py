@@ -44,4 +44,9 @@ w = wt[:nb]
 rel = np.where(w > 0, w - tr[0, :nb, 2][:, None], 0)
 nw = int((w[0] > 0).sum())
 out["fwd_cone_end_us_med_per_warp"] = [round(float(np.median(rel[:, k])) / 1e3, 2) for k in range(nw)]
+# reverse: per cone q (block % P, P = argv[3], default 4), median of (after compute - after wait)
+P = int(sys.argv[3]) if len(sys.argv) > 3 else 4
+rb = np.nonzero(tr[1, :, 0] > 0)[0]
+out["rev_cone_us_med_per_q"] = [round(float(np.median((tr[1, rb[rb % P == q], 2] - tr[1, rb[rb % P == q], 1]))) / 1e3, 2)
+                                for q in range(P)]
 print(json.dumps(out))
