@@ -71,6 +71,8 @@ static cudaLaunchAttribute g_pdl_attr = [] {
   return a;
 }();
 
+static int pdl_mask();   // felix_tune("pdl") below
+
 template <int BN, int EPI>
 static void launch_gemm_t(const GemmLaunch& g, cudaStream_t st) {
   auto kern = mlp_gemm_kernel<BN, EPI>;
@@ -81,7 +83,7 @@ static void launch_gemm_t(const GemmLaunch& g, cudaStream_t st) {
   cfg.dynamicSmemBytes = GemmCfg<BN>::smem_bytes(g.stages);
   cfg.stream = st;
   cfg.attrs = &g_pdl_attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = (pdl_mask() & 2) ? 1 : 0;
   CUDA_OK(cudaLaunchKernelEx(&cfg, kern, g.a_hi, g.a_lo, g.b_hi, g.b_lo, g.c_hi, g.c_lo, g.args, g.stages));
 }
 
@@ -146,7 +148,8 @@ struct Tuning {
   std::atomic<int> codegen_P{-1}, codegen_R{-1};   // felix_codegen's variant
   std::atomic<int> trace{0};         // per-block %globaltimer stamps in kernels generated afterwards
   std::atomic<int> round_bnb{0};
-  std::atomic<int> graph_steps{-1};  // Adam steps per search graph (-1: kGraphSteps)     // 1: every split component rounds by branch and bound (test hook)
+  std::atomic<int> graph_steps{-1};  // Adam steps per search graph (-1: kGraphSteps)
+  std::atomic<int> pdl{-1};          // PDL edges: bit 0 forward, 1 MLP kernels, 2 reverse / other (-1: none)     // 1: every split component rounds by branch and bound (test hook)
 };
 static Tuning g_tune;
 
@@ -188,6 +191,11 @@ static MlpMode mlp_mode(const Plan& p) {
   return (p.tile_ok && p.tile_full_wave) ? MLP_TILE : MLP_CHAIN;
 }
 static bool use_chain() { return g_tune.mlp.load() != 2; }
+// Programmatic dependent launch edges (felix_tune "pdl", bit mask: 1 forward DAG kernel, 2 MLP kernels,
+// 4 reverse / other kernels).  Default none: measured at C2 (profiles/r02/bench_pdl.log), every edge costs
+// more than the prologue overlap it buys -- the early-resident dependent CTAs slow the running kernel
+// (no PDL 8.75e7 cand-steps/s; chain + reverse edges 8.22e7; all edges 7.74e7).
+static int pdl_mask() { const int m = g_tune.pdl.load(); return m >= 0 ? m : 0; }
 
 static void launch_tile(const Plan& p, cudaStream_t st) {
   const void* fn = p.tile_cg == 2 ? reinterpret_cast<const void*>(mlp_tile_kernel<2>)
@@ -195,6 +203,7 @@ static void launch_tile(const Plan& p, cudaStream_t st) {
   set_smem_attr(fn, tile::SMEM_BYTES, p.tile_cg == 2);
   cudaLaunchAttribute attrs[2];
   attrs[0] = g_pdl_attr;
+  if (!(pdl_mask() & 2)) attrs[0].val.programmaticStreamSerializationAllowed = 0;
   attrs[1].id = cudaLaunchAttributeClusterDimension;
   attrs[1].val.clusterDim.x = static_cast<unsigned>(p.tile_cg);
   attrs[1].val.clusterDim.y = 1;
@@ -216,6 +225,7 @@ static void launch_chain(const Plan& p, cudaStream_t st) {
                 CHAIN_SMEM_BYTES);
   cudaLaunchAttribute attrs[3];
   attrs[0] = g_pdl_attr;
+  if (!(pdl_mask() & 2)) attrs[0].val.programmaticStreamSerializationAllowed = 0;
   attrs[1].id = cudaLaunchAttributeCooperative;   // the dataflow flags need every CTA resident
   attrs[1].val.cooperative = 1;
   attrs[2].id = cudaLaunchAttributeClusterDimension;
@@ -617,7 +627,7 @@ static void launch_cfg(const void* f, dim3 grid, dim3 block, size_t smem, void**
   cfg.blockDim = block;
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  if (pdl) { cfg.attrs = &g_pdl_attr; cfg.numAttrs = 1; }
+  if (pdl && pdl_mask()) { cfg.attrs = &g_pdl_attr; cfg.numAttrs = 1; }
   CUDA_OK(cudaLaunchKernelExC(&cfg, f, args));
 }
 static void launch_grouped(cudaKernel_t f, int P, int R, int64_t n, size_t smem, void** args, cudaStream_t st, bool pdl) {
@@ -1419,13 +1429,13 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
       void* pen = pl.sc_pen.p;
       void* fa[] = {&yk, &ni, &ldy, &phh, &phl, &ctr, &mv, &vv, &part, &pen, &cpart, &nht, &ld, &hbv, &lam, &lr, &b1, &b2, &eps};
       prof_mark(s, 0, cs, true);
-      launch_grouped(mod.f_fwd_adam, mod.P, mod.R, cnt, 0, fa, cs, false);   // no PDL edge from the previous step's reverse (measured slower)
+      launch_grouped(mod.f_fwd_adam, mod.P, mod.R, cnt, 0, fa, cs, pdl_mask() & 1);   // default: no PDL edge from the previous step's reverse (measured slower)
       prof_mark(s, 0, cs, false);
       s->prof_launches[0] += 1;
       run_mlp(s, pl, cs);
       void* ra[] = {&yk, &ni, &ldy, &dphi, &ld, &lam, &part, &pen, &ctr};
       prof_mark(s, 2, cs, true);
-      launch_sc(mod.f_rev_sc, mod.P, scw, cnt, ra, cs, true);
+      launch_sc(mod.f_rev_sc, mod.P, scw, cnt, ra, cs, (pdl_mask() & 4) != 0);
       prof_mark(s, 2, cs, false);
       s->prof_launches[2] += 1;
       return;
@@ -1562,6 +1572,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
     const int tail = static_cast<int>(p->n_steps % gs);
     std::vector<double> key_s = key;
     key_s.push_back(static_cast<double>(gs));
+    key_s.push_back(static_cast<double>(pdl_mask()));
     if (!ch.graph || ch.graph_key != key_s) {
       if (ch.graph) { cudaGraphExecDestroy(ch.graph); ch.graph = nullptr; }
       if (ch.graph_tail) { cudaGraphExecDestroy(ch.graph_tail); ch.graph_tail = nullptr; }
@@ -1569,7 +1580,7 @@ felix_status felix_search(felix_space* s, felix_costmodel* m, const felix_search
       ch.graph = build(gs);
       ch.graph_key = key_s;
     }
-    if (tail > 0 && ch.graph_tail_steps != tail) {
+    if (tail > 0 && (ch.graph_tail_steps != tail || !ch.graph_tail)) {
       if (ch.graph_tail) { cudaGraphExecDestroy(ch.graph_tail); ch.graph_tail = nullptr; }
       ch.graph_tail = build(tail);
       ch.graph_tail_steps = tail;
@@ -2253,6 +2264,7 @@ felix_status felix_tune(const char* key, int32_t value) {
   else if (k == "codegen_replicas") { in({-1, 1, 2, 4}); g_tune.codegen_R = value; }
   else if (k == "trace") { in({0, 1}); g_tune.trace = value; }
   else if (k == "round_bnb") { in({0, 1}); g_tune.round_bnb = value; }
+  else if (k == "pdl") { if (value != -1 && (value < 0 || value > 7)) in({}); g_tune.pdl = value; }
   else if (k == "graph_steps") { if (value != -1 && (value < 1 || value > 1000)) in({}); g_tune.graph_steps = value; }
   else FELIX_THROW(FELIX_E_INVALID_ARG, "felix_tune: unknown key " + k);
   FELIX_API_END
