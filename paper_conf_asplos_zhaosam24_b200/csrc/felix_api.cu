@@ -668,14 +668,15 @@ static int choose_R_sc() {
   const int r = g_tune.R.load();
   return (r == 1 || r == 2 || r == 4) ? r : 2;
 }
-// warps per split-cone CTA: about two CTAs per SM (felix_tune("sc_warps") overrides).  Measured at C2
-// (P = 4, 128 candidate groups; profiles/r02/sc_warps.log): W = 2 (256 CTAs) 8.20e7 cand-steps/s, W = 3
-// 8.20e7, W = 4 (one CTA per SM) 8.00e7, W = 8 8.17e7, W = 1 8.05e7.
+// warps per split-cone CTA: about one CTA per SM (felix_tune("sc_warps") overrides).  Measured at C2
+// (P = 4, 128 candidate groups) without PDL edges (profiles/r02/sc_warps_nopdl.log): W = 4 (128 CTAs)
+// 9.13e7 cand-steps/s, W = 8 9.04e7, W = 6 9.03e7, W = 2 8.95e7.  (With PDL edges W = 2 had measured
+// best, profiles/r02/sc_warps.log: the early-resident next kernel then competed with fewer, larger CTAs.)
 static int choose_scw(int64_t n, int P) {
   const int w0 = g_tune.scw.load();
   if (w0 >= 1 && w0 <= 8) return w0;
   const int64_t groups = (n + 31) / 32;
-  int64_t w = (groups * P + 2 * 148 - 1) / (2 * 148);
+  int64_t w = (groups * P + 147) / 148;
   return static_cast<int>(std::max<int64_t>(1, std::min<int64_t>(8, w)));
 }
 static int64_t sc_groups(int64_t n, int W) { return ((n + 31) / 32 + W - 1) / W; }
