@@ -687,7 +687,10 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "    if (s_ <= 0) {\n"
     << "#pragma unroll\n      for (int jj = 0; jj < NJ; ++jj) { const int j = wq + PG * jj; if (j >= NV) break; sx[j][lane] = exp((double)yl[jj]); }\n"
     << "    } else {\n"
-    << "      const double dlam = (double)lam;\n";
+    << "      const double dlam = (double)lam;\n"
+    // bias corrections first: independent of the loads and the barrier below, so they overlap them
+    << "      const float bc1 = 1.f - powf(b1, (float)s_), bc2 = 1.f - powf(b2, (float)s_);\n"
+    << "      const float step = lr / bc1, rb = 1.f / sqrtf(bc2);\n";
   // the loss -C + lam (user penalties + auto penalties) is finite iff C and the user penalties are (the
   // auto penalties are finite for finite y; a non-finite y makes its own gradient non-finite)
   for (int j = 0; j < M; ++j) o << "      const double y" << j << " = (double)sy[" << j << "][lane];\n";
@@ -703,8 +706,6 @@ std::string generate_dag_module(const SpaceDesc& d, int K0p, int P, int NREPv, b
     << "      __syncthreads();\n      TSTAMP(0, 6);\n"
     << "      unsigned anybad = 0;\n#pragma unroll\n      for (int q = 0; q < PG; ++q) anybad |= sbad[q];\n"
     << "      const bool okall = !((anybad >> lane) & 1u);\n"
-    << "      const float bc1 = 1.f - powf(b1, (float)s_), bc2 = 1.f - powf(b2, (float)s_);\n"
-    << "      const float step = lr / bc1, rb = 1.f / sqrtf(bc2);\n"
     << "#pragma unroll\n      for (int jj = 0; jj < NJ; ++jj) {\n"
     << "        const int j = wq + PG * jj;\n        if (j >= NV) break;\n"
     << "        float yy = yl[jj];\n"
