@@ -432,6 +432,108 @@ __global__ void __launch_bounds__(256) score_layer_v2_kernel(const double* __res
   }
 }
 
+// The same layer on the FP64 tensor cores (mma.sync m8n8k4 f64): 128 x 64 tiles, 8 warps of 32 x 32 (4 x 4
+// MMAs of 8 x 8 per K step of 4, 32 accumulators per thread), K staged 16 at a time through double-buffered
+// shared memory (rows padded so a fragment load of 4 k x 8 doubles takes the minimum two wavefronts).  Each
+// thread's fragment loads feed 2 MMAs per load instead of the CUDA-core kernel's 32 DFMA per 6 loads at one
+// CTA per SM; FP64 throughout, products summed by the MMA unit (differences to the CUDA-core order are at
+// the 1e-16 level, far inside the 1e-12 score tolerance).
+constexpr int SCD_TM = 128, SCD_TN = 64, SCD_KT = 16, SCD_AP = SCD_TM + 4, SCD_BP = SCD_TN + 4;
+constexpr int SCD_SMEM = 2 * SCD_KT * (SCD_AP + SCD_BP) * 8;   // dynamic shared memory (51 KB, opt-in)
+__global__ void __launch_bounds__(256) score_layer_dmma_kernel(const double* __restrict__ in, long long in_rs, long long in_cs,
+                                                               int n, int K, const double* __restrict__ W,
+                                                               const double* __restrict__ b, double* __restrict__ out,
+                                                               int N, int relu, int accumulate) {
+  extern __shared__ __align__(16) double scd_smem[];
+  double (*As)[SCD_KT][SCD_AP] = reinterpret_cast<double (*)[SCD_KT][SCD_AP]>(scd_smem);                      // [buf][k][row]
+  double (*Bs)[SCD_KT][SCD_BP] = reinterpret_cast<double (*)[SCD_KT][SCD_BP]>(scd_smem + 2 * SCD_KT * SCD_AP);  // [buf][k][col]
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int gid = lane >> 2, tig = lane & 3;
+  const int wr = (warp & 3) * 32, wc = (warp >> 2) * 32;    // warp tile origin inside the block tile
+  const int row0 = blockIdx.y * SCD_TM, col0 = blockIdx.x * SCD_TN;
+  double acc[4][4][2];
+#pragma unroll
+  for (int nj = 0; nj < 4; ++nj) {
+    const int c = col0 + wc + nj * 8 + 2 * tig;
+    const double b0 = c < N ? b[c] : 0.0, b1 = c + 1 < N ? b[c + 1] : 0.0;
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) { acc[mi][nj][0] = b0; acc[mi][nj][1] = b1; }
+  }
+  double pa[8], pb[4];
+  auto load_chunk = [&](int k0) {
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int e = tid + q * 256;
+      int r, kk;
+      if (in_rs == 1) { r = e & 127; kk = e >> 7; } else { kk = e & 15; r = e >> 4; }
+      const int gr = row0 + r, gk = k0 + kk;
+      pa[q] = (gr < n && gk < K) ? in[static_cast<size_t>(gr) * in_rs + static_cast<size_t>(gk) * in_cs] : 0.0;
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int e = tid + q * 256;
+      const int c = e >> 4, kb = e & 15;
+      const int gc = col0 + c, gkb = k0 + kb;
+      pb[q] = (gc < N && gkb < K) ? W[static_cast<size_t>(gc) * K + gkb] : 0.0;
+    }
+  };
+  auto store_chunk = [&](int buf) {
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int e = tid + q * 256;
+      int r, kk;
+      if (in_rs == 1) { r = e & 127; kk = e >> 7; } else { kk = e & 15; r = e >> 4; }
+      As[buf][kk][r] = pa[q];
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int e = tid + q * 256;
+      Bs[buf][e & 15][e >> 4] = pb[q];
+    }
+  };
+  const int nk = (K + SCD_KT - 1) / SCD_KT;
+  load_chunk(0);
+  store_chunk(0);
+  __syncthreads();
+  for (int c = 0; c < nk; ++c) {
+    const int buf = c & 1;
+    if (c + 1 < nk) load_chunk((c + 1) * SCD_KT);
+    // zero-padded K: the chunk's k beyond K are 0 in both operands, so all 4 K steps run
+#pragma unroll
+    for (int k4 = 0; k4 < SCD_KT; k4 += 4) {
+      double af[4], bf[4];
+#pragma unroll
+      for (int mi = 0; mi < 4; ++mi) af[mi] = As[buf][k4 + tig][wr + mi * 8 + gid];
+#pragma unroll
+      for (int nj = 0; nj < 4; ++nj) bf[nj] = Bs[buf][k4 + tig][wc + nj * 8 + gid];
+#pragma unroll
+      for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+        for (int nj = 0; nj < 4; ++nj)
+          asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
+                       : "+d"(acc[mi][nj][0]), "+d"(acc[mi][nj][1]) : "d"(af[mi]), "d"(bf[nj]));
+    }
+    if (c + 1 < nk) store_chunk(buf ^ 1);   // the other buffer was last read in chunk c - 1 (barrier below)
+    __syncthreads();
+  }
+#pragma unroll
+  for (int mi = 0; mi < 4; ++mi) {
+    const int r = row0 + wr + mi * 8 + gid;
+    if (r >= n) continue;
+#pragma unroll
+    for (int nj = 0; nj < 4; ++nj) {
+      const int col = col0 + wc + nj * 8 + 2 * tig;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        if (col + h >= N) continue;
+        const double v = (relu && !(acc[mi][nj][h] > 0.0)) ? 0.0 : acc[mi][nj][h];
+        double* o = out + static_cast<size_t>(r) * N + col + h;
+        *o = accumulate ? *o + v : v;
+      }
+    }
+  }
+}
+
 // head layer (N = 1, row-major input [n][K]): thread per row streaming its own row (the L1 serves the
 // 16 doubles of each 128-B line), one-warp blocks so the rows spread over the SMs; same fma order as above
 __global__ void __launch_bounds__(32) score_head_kernel(const double* __restrict__ in, int n, int K,

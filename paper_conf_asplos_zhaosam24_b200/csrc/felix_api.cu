@@ -149,6 +149,7 @@ struct Tuning {
   std::atomic<int> trace{0};         // per-block %globaltimer stamps in kernels generated afterwards
   std::atomic<int> round_bnb{0};
   std::atomic<int> graph_steps{-1};  // Adam steps per search graph (-1: kGraphSteps)
+  std::atomic<int> score_dmma{-1};  // FP64 scoring layers on the FP64 tensor cores (0: CUDA-core kernel; -1 = 1)
   std::atomic<int> pdl{-1};          // PDL edges: bit 0 forward, 1 MLP kernels, 2 reverse / other (-1: none)     // 1: every split component rounds by branch and bound (test hook)
 };
 static Tuning g_tune;
@@ -2042,7 +2043,13 @@ static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, in
       const int K = m->dims[l], N = m->dims[l + 1];
       const bool last = l == L - 1;
       double* out = last ? score : bufs[l & 1];
-      if (N >= 32) {   // register-blocked 128 x 64 tiles
+      if (N >= 32 && g_tune.score_dmma.load() != 0) {   // FP64 tensor cores, 128 x 64 tiles
+        const dim3 grid(static_cast<unsigned>((N + SCD_TN - 1) / SCD_TN), static_cast<unsigned>((n + SCD_TM - 1) / SCD_TM));
+        set_smem_attr(reinterpret_cast<const void*>(score_layer_dmma_kernel), SCD_SMEM);
+        score_layer_dmma_kernel<<<grid, 256, SCD_SMEM, st>>>(
+            in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
+            last ? 0 : 1, last && st_i > 0 ? 1 : 0);
+      } else if (N >= 32) {   // register-blocked 128 x 64 tiles on the CUDA cores
         const dim3 grid(static_cast<unsigned>((N + SC2_TN - 1) / SC2_TN), static_cast<unsigned>((n + SC2_TM - 1) / SC2_TM));
         score_layer_v2_kernel<<<grid, 256, 0, st>>>(
             in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
@@ -2265,6 +2272,7 @@ felix_status felix_tune(const char* key, int32_t value) {
   else if (k == "codegen_replicas") { in({-1, 1, 2, 4}); g_tune.codegen_R = value; }
   else if (k == "trace") { in({0, 1}); g_tune.trace = value; }
   else if (k == "round_bnb") { in({0, 1}); g_tune.round_bnb = value; }
+  else if (k == "score_dmma") { in({-1, 0, 1}); g_tune.score_dmma = value; }
   else if (k == "pdl") { if (value != -1 && (value < 0 || value > 7)) in({}); g_tune.pdl = value; }
   else if (k == "graph_steps") { if (value != -1 && (value < 1 || value > 1000)) in({}); g_tune.graph_steps = value; }
   else FELIX_THROW(FELIX_E_INVALID_ARG, "felix_tune: unknown key " + k);
