@@ -287,10 +287,13 @@ struct GroupCache {
   std::vector<std::unique_ptr<DevBuf>> m, v, step_ctr;
   std::vector<std::unique_ptr<DevBuf>> sc_part, sc_pen;   // split-cone buffers per member (see Plan)
   std::vector<cudaStream_t> streams;
-  cudaGraphExec_t graph = nullptr;
+  cudaGraphExec_t graph = nullptr;            // graph_steps Adam steps per launch (see felix_search)
+  cudaGraphExec_t graph_tail = nullptr;
+  int graph_tail_steps = 0;
   std::vector<double> key;
   ~GroupCache() {
     if (graph) cudaGraphExecDestroy(graph);
+    if (graph_tail) cudaGraphExecDestroy(graph_tail);
     for (auto st : streams) cudaStreamDestroy(st);
   }
 };
@@ -1830,30 +1833,49 @@ felix_status felix_search_group(felix_space* const* spaces, int32_t n_spaces, fe
                            static_cast<double>(sc), static_cast<double>(scws[i]), ptr(gc.sc_part[i]->p),
                            ptr(gc.sc_pen[i]->p)});
   }
-  if (!gc.graph || gc.key != key) {
-    if (gc.graph) { cudaGraphExecDestroy(gc.graph); gc.graph = nullptr; }
+  // several Adam steps per graph launch, as in felix_search
+  auto build = [&](int steps) {
     cudaGraph_t graph = nullptr;
+    cudaGraphExec_t exec = nullptr;
     cudaStream_t cap;
     CUDA_OK(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
     struct StGuard { cudaStream_t s; ~StGuard() { cudaStreamDestroy(s); } } capg{cap};
     CUDA_OK(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
     try {
-      enqueue_step(cap);
+      for (int i = 0; i < steps; ++i) enqueue_step(cap);
     } catch (...) {
       cudaStreamEndCapture(cap, &graph);
       if (graph) cudaGraphDestroy(graph);
       throw;
     }
     CUDA_OK(cudaStreamEndCapture(cap, &graph));
-    cudaError_t ie = cudaGraphInstantiate(&gc.graph, graph, 0);
+    cudaError_t ie = cudaGraphInstantiate(&exec, graph, 0);
     cudaGraphDestroy(graph);
     CUDA_OK(ie);
+    return exec;
+  };
+  const int gs_t = g_tune.graph_steps.load();
+  const int gs = std::max(1, std::min(gs_t >= 1 ? gs_t : kGraphSteps, T));
+  const int tail = T > 0 ? T % gs : 0;
+  key.push_back(static_cast<double>(gs));
+  key.push_back(static_cast<double>(pdl_mask()));
+  if (!gc.graph || gc.key != key) {
+    if (gc.graph) { cudaGraphExecDestroy(gc.graph); gc.graph = nullptr; }
+    if (gc.graph_tail) { cudaGraphExecDestroy(gc.graph_tail); gc.graph_tail = nullptr; }
+    gc.graph_tail_steps = 0;
+    gc.graph = build(gs);
     gc.key = key;
   }
-  for (int t = 1; t <= T; ++t) {
-    if (t % 100000 == 0) CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
+  if (tail > 0 && (gc.graph_tail_steps != tail || !gc.graph_tail)) {
+    if (gc.graph_tail) { cudaGraphExecDestroy(gc.graph_tail); gc.graph_tail = nullptr; }
+    gc.graph_tail = build(tail);
+    gc.graph_tail_steps = tail;
+  }
+  for (int t = 0; t + gs <= T; t += gs) {
+    if (t % 100000 < gs && t > 0) CUDA_OK(cudaMemsetAsync(pl.grid_bar.p, 0, pl.grid_bar.bytes, st));
     CUDA_OK(cudaGraphLaunch(gc.graph, st));
   }
+  if (tail > 0) CUDA_OK(cudaGraphLaunch(gc.graph_tail, st));
   final_adam();
   FELIX_API_END
 }
