@@ -328,7 +328,8 @@ struct felix_space {
   std::unique_ptr<felix::Chunks> search_chunks, eval_chunks;
   std::unique_ptr<felix::GroupCache> group_cache;   // felix_search_group with this space first
   felix::DevBuf sched, valid, phi64, score, act64a, act64b, alive, rec_cand, rec_cnt, fin_cand, fin_cnt, o_idx, o_score, o_sched;
-  felix::DevBuf o_pack;                       // felix_round_topk outputs, one contiguous block: [count | idx | score | sched]
+  felix::DevBuf o_pack;
+  felix::DevBuf rec_cand2, rec_cnt2;         // multi-phase top-k: records of the odd phases                       // felix_round_topk outputs, one contiguous block: [count | idx | score | sched]
   void* h_pack = nullptr;                     // pinned host copy of o_pack (one D2H copy per call)
   size_t h_pack_bytes = 0;
   // varValuesHistory (Alg. 1 l.13/17) of the last search run with history != 0: per-step rounded points,
@@ -2037,10 +2038,60 @@ static void launch_topk_select(long long nblk, long long n_entries, long long ch
   CUDA_OK(cudaGetLastError());
 }
 
+// Dedup + top-k of n entries in phases: each phase cuts its entries into blocks whose (score, key,
+// candidate, schedule) fit shared memory and keeps each block's k best records; the records of one phase
+// are the entries of the next, until one block remains.  Every phase is the same selection (score desc,
+// key asc, dedup by schedule keeping the best), so the result equals a single pass over all entries.
+static void run_topk(felix_space* s, int64_t n, const long long* okey, const int32_t* sched, int M, int k,
+                     int* out_cand, int* out_cnt, cudaStream_t st);
+
 static long long topk_chunk(long long n) {
   long long c = (n + 63) / 64;
   c = (c + 255) / 256 * 256;
   return std::max(512LL, std::min(4096LL, c));
+}
+
+static void run_topk(felix_space* s, int64_t n, const long long* okey, const int32_t* sched, int M, int k,
+                     int* out_cand, int* out_cnt, cudaStream_t st) {
+  const double* score = s->score.as<double>();
+  const uint8_t* valid = s->valid.as<uint8_t>();
+  long long chunk = 1;
+  while (chunk * 2 * (8 + 8 + 4 + 4LL * M + 1) <= 96 * 1024) chunk *= 2;
+  if (chunk < 2LL * k) {   // schedules too long for a shared-memory block of 2k entries: the global-memory kernel
+    const long long ch = topk_chunk(n), nblk = (n + ch - 1) / ch;
+    ensure(s->alive, static_cast<size_t>(std::max<long long>(n, nblk * k)));
+    ensure(s->rec_cand, static_cast<size_t>(nblk) * k * 4);
+    ensure(s->rec_cnt, static_cast<size_t>(nblk) * 4);
+    launch_topk_select(nblk, n, ch, nullptr, okey, score, valid, sched, M, k, s->alive.as<uint8_t>(),
+                       s->rec_cand.as<int>(), s->rec_cnt.as<int>(), st);
+    launch_topk_select(1, nblk * k, nblk * k, s->rec_cand.as<int>(), okey, score, valid, sched, M, k,
+                       s->alive.as<uint8_t>(), out_cand, out_cnt, st);
+    return;
+  }
+  long long entries = n;
+  const int* cand_of = nullptr;
+  int phase = 0;
+  while (true) {
+    const long long nblk = (entries + chunk - 1) / chunk;
+    int* oc;
+    int* on;
+    if (nblk == 1) {
+      oc = out_cand;
+      on = out_cnt;
+    } else {
+      felix::DevBuf& rc = (phase & 1) ? s->rec_cand2 : s->rec_cand;
+      felix::DevBuf& rn = (phase & 1) ? s->rec_cnt2 : s->rec_cnt;
+      ensure(rc, static_cast<size_t>(nblk) * k * 4);
+      ensure(rn, static_cast<size_t>(nblk) * 4);
+      oc = rc.as<int>();
+      on = rn.as<int>();
+    }
+    launch_topk_select(nblk, entries, chunk, cand_of, okey, score, valid, sched, M, k, nullptr, oc, on, st);
+    if (nblk == 1) return;
+    cand_of = oc;
+    entries = nblk * k;
+    ++phase;
+  }
 }
 
 static void do_hard(felix_space* s, const int32_t* sched, int64_t n, double* phi64, uint8_t* valid, cudaStream_t st) {
@@ -2143,11 +2194,6 @@ felix_status felix_round_topk(felix_space* s, felix_costmodel* m, const float* y
   do_round(s, y, n, s->sched.as<int32_t>(), st);
   do_hard(s, s->sched.as<int32_t>(), n, s->phi64.as<double>(), s->valid.as<uint8_t>(), st);
   do_score(s, m, s->phi64.as<double>(), n, s->score.as<double>(), st);
-  const long long chunk = topk_chunk(n);
-  const long long nblk = (n + chunk - 1) / chunk;
-  ensure(s->alive, static_cast<size_t>(std::max<long long>(n, nblk * k)));
-  ensure(s->rec_cand, static_cast<size_t>(nblk) * k * 4);
-  ensure(s->rec_cnt, static_cast<size_t>(nblk) * 4);
   ensure(s->fin_cand, static_cast<size_t>(k) * 4);
   // outputs packed in one device block and read back with a single copy into pinned memory:
   // [count (8 B) | idx k x 8 | score k x 8 | sched k x M x 4]
@@ -2165,10 +2211,7 @@ felix_status felix_round_topk(felix_space* s, felix_costmodel* m, const float* y
   long long* p_idx = reinterpret_cast<long long*>(pk + 8);
   double* p_score = reinterpret_cast<double*>(pk + 8 + static_cast<size_t>(k) * 8);
   int32_t* p_sched = reinterpret_cast<int32_t*>(pk + 8 + static_cast<size_t>(k) * 16);
-  launch_topk_select(nblk, n, chunk, nullptr, nullptr, s->score.as<double>(), s->valid.as<uint8_t>(), s->sched.as<int32_t>(),
-                     M, k, s->alive.as<uint8_t>(), s->rec_cand.as<int>(), s->rec_cnt.as<int>(), st);
-  launch_topk_select(1, nblk * k, nblk * k, s->rec_cand.as<int>(), nullptr, s->score.as<double>(), s->valid.as<uint8_t>(),
-                     s->sched.as<int32_t>(), M, k, s->alive.as<uint8_t>(), s->fin_cand.as<int>(), p_cnt, st);
+  run_topk(s, n, nullptr, s->sched.as<int32_t>(), M, k, s->fin_cand.as<int>(), p_cnt, st);
   topk_gather_kernel<<<1, std::max(32, (k + 31) / 32 * 32), 0, st>>>(
       s->fin_cand.as<int>(), p_cnt, k, s->score.as<double>(), s->sched.as<int32_t>(), M, index_base,
       p_idx, p_score, p_sched);
@@ -2209,18 +2252,10 @@ felix_status felix_history_topk(felix_space* s, felix_costmodel* m, int32_t k, i
   ensure(s->score, static_cast<size_t>(n) * 8);
   do_hard(s, sched, n, s->phi64.as<double>(), s->valid.as<uint8_t>(), st);
   do_score(s, m, s->phi64.as<double>(), n, s->score.as<double>(), st);
-  const long long chunk = topk_chunk(n);
-  const long long nblk = (n + chunk - 1) / chunk;
-  ensure(s->alive, static_cast<size_t>(std::max<long long>(n, nblk * k)));
-  ensure(s->rec_cand, static_cast<size_t>(nblk) * k * 4);
-  ensure(s->rec_cnt, static_cast<size_t>(nblk) * 4);
   ensure(s->fin_cand, static_cast<size_t>(k) * 4);
   ensure(s->fin_cnt, 4);
   const long long* key = s->h_pool_key.as<long long>();
-  launch_topk_select(nblk, n, chunk, nullptr, key, s->score.as<double>(), s->valid.as<uint8_t>(), sched, M, k,
-                     s->alive.as<uint8_t>(), s->rec_cand.as<int>(), s->rec_cnt.as<int>(), st);
-  launch_topk_select(1, nblk * k, nblk * k, s->rec_cand.as<int>(), key, s->score.as<double>(), s->valid.as<uint8_t>(), sched,
-                     M, k, s->alive.as<uint8_t>(), s->fin_cand.as<int>(), s->fin_cnt.as<int>(), st);
+  run_topk(s, n, key, sched, M, k, s->fin_cand.as<int>(), s->fin_cnt.as<int>(), st);
   ensure(s->o_idx, static_cast<size_t>(k) * 8);
   ensure(s->o_step, static_cast<size_t>(k) * 4);
   ensure(s->o_score, static_cast<size_t>(k) * 8);
