@@ -149,6 +149,25 @@ def test_score_fp64(fx, name):
     assert np.all(np.abs(got[ok] - ref[ok]) <= 1e-12 * np.maximum(np.abs(ref[ok]), 1e-3))
 
 
+@pytest.mark.parametrize("name", ["C2", "C5"])
+def test_score_tensor_core_and_cuda_core_kernels_agree(fx, name):
+    """FP64 scoring layers on the FP64 tensor cores (default) and on the CUDA cores (score_dmma=0): both
+    within 1e-12 of the oracle, and within 1e-13 of each other (only the summation order differs)."""
+    sp, mlp, n, space, cm = _setup(fx, name)
+    y0 = fi.make_y0(sp, n, seed=15)
+    rs = fo.round_schedules(sp, y0)
+    st = torch.from_numpy(rs).cuda()
+    tc = space.score(cm, st).cpu().numpy()
+    with fx.tuned(score_dmma=0):
+        cc = space.score(cm, st).cpu().numpy()
+    ref = fo.score(sp, mlp.W, mlp.b, rs)
+    ok = np.isfinite(ref)
+    assert np.array_equal(np.isfinite(tc), ok) and np.array_equal(np.isfinite(cc), ok)
+    for got in (tc, cc):
+        assert np.all(np.abs(got[ok] - ref[ok]) <= 1e-12 * np.maximum(np.abs(ref[ok]), 1e-3))
+    assert np.all(np.abs(tc[ok] - cc[ok]) <= 1e-13 * np.maximum(np.abs(ref[ok]), 1e-3))
+
+
 def _topk_equal(idx, sc, sched, ridx, rsc, rsched):
     assert len(idx) == len(ridx)
     assert np.all(np.abs(sc - rsc) <= 1e-12 * np.maximum(np.abs(rsc), 1e-3))
