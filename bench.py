@@ -490,7 +490,7 @@ def run_felix(args):
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-        "dtype": "fp16x3 split (fp32-accurate) MLP, f64 DAG, f32 Adam", "data": "synthetic",
+        "dtype": "fp16 hi/lo split (fp32-accurate) MLP, f64 DAG forward, f32 DAG reverse, f32 Adam, f64 scoring", "data": "synthetic",
         "config": workload_config(cfg, sp, n, T, k, world, hist),
         "roofline": {"bound": "tensor", "achieved": achieved_tflops, "peak": peak, "unit": "TFLOP/s",
                      "frac": achieved_tflops / peak, "traffic": traffic,
@@ -712,7 +712,7 @@ def run_felix_tasks(args):
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
         "ms_per_step": t_max / K, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
-        "dtype": "fp16x3 split (fp32-accurate) MLP, f64 DAG, f32 Adam", "data": "synthetic",
+        "dtype": "fp16 hi/lo split (fp32-accurate) MLP, f64 DAG forward, f32 DAG reverse, f32 Adam, f64 scoring", "data": "synthetic",
         "config": {"workload": f"{cfg.name}: {len(cfg.spaces)} tasks x {cfg.n_seeds} seeds x {T} steps, "
                                f"MLP {list(cfg.mlp_dims)}, top-{k} per task",
                    "tasks": [sp.name for sp in cfg.spaces], "n_seeds_per_task": cfg.n_seeds, "n_steps": T,
