@@ -438,34 +438,42 @@ __global__ void __launch_bounds__(256) score_layer_v2_kernel(const double* __res
 // thread's fragment loads feed 2 MMAs per load instead of the CUDA-core kernel's 32 DFMA per 6 loads at one
 // CTA per SM; FP64 throughout, products summed by the MMA unit (differences to the CUDA-core order are at
 // the 1e-16 level, far inside the 1e-12 score tolerance).
-constexpr int SCD_TM = 128, SCD_TN = 64, SCD_KT = 16, SCD_AP = SCD_TM + 4, SCD_BP = SCD_TN + 4;
-constexpr int SCD_SMEM = 2 * SCD_KT * (SCD_AP + SCD_BP) * 8;   // dynamic shared memory (51 KB, opt-in)
-__global__ void __launch_bounds__(256) score_layer_dmma_kernel(const double* __restrict__ in, long long in_rs, long long in_cs,
+// MI = 8-row MMA blocks per warp tile: 4 (128 x 64 block tiles, 32 x 32 warp tiles) or 8 (256 x 64 block
+// tiles, 64 x 32 warp tiles: 12 fragment loads per 32 MMAs instead of 8 per 16; used when the population
+// gives at least two such tiles per SM).
+constexpr int SCD_TN = 64, SCD_KT = 16, SCD_BP = SCD_TN + 4;
+template <int MI> __host__ __device__ constexpr int scd_tm() { return 32 * MI; }
+template <int MI> __host__ __device__ constexpr int scd_ap() { return 32 * MI + 4; }
+template <int MI> __host__ __device__ constexpr int scd_smem() { return 2 * SCD_KT * (scd_ap<MI>() + SCD_BP) * 8; }   // dynamic, opt-in
+template <int MI>
+__global__ void __launch_bounds__(256, 1) score_layer_dmma_kernel(const double* __restrict__ in, long long in_rs, long long in_cs,
                                                                int n, int K, const double* __restrict__ W,
                                                                const double* __restrict__ b, double* __restrict__ out,
                                                                int N, int relu, int accumulate) {
   extern __shared__ __align__(16) double scd_smem[];
-  double (*As)[SCD_KT][SCD_AP] = reinterpret_cast<double (*)[SCD_KT][SCD_AP]>(scd_smem);                      // [buf][k][row]
-  double (*Bs)[SCD_KT][SCD_BP] = reinterpret_cast<double (*)[SCD_KT][SCD_BP]>(scd_smem + 2 * SCD_KT * SCD_AP);  // [buf][k][col]
+  constexpr int TM = scd_tm<MI>(), AP = scd_ap<MI>();
+  double (*As)[SCD_KT][AP] = reinterpret_cast<double (*)[SCD_KT][AP]>(scd_smem);                      // [buf][k][row]
+  double (*Bs)[SCD_KT][SCD_BP] = reinterpret_cast<double (*)[SCD_KT][SCD_BP]>(scd_smem + 2 * SCD_KT * AP);  // [buf][k][col]
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int gid = lane >> 2, tig = lane & 3;
-  const int wr = (warp & 3) * 32, wc = (warp >> 2) * 32;    // warp tile origin inside the block tile
-  const int row0 = blockIdx.y * SCD_TM, col0 = blockIdx.x * SCD_TN;
-  double acc[4][4][2];
+  const int wr = (warp & 3) * (8 * MI), wc = (warp >> 2) * 32;    // warp tile origin inside the block tile
+  const int row0 = blockIdx.y * TM, col0 = blockIdx.x * SCD_TN;
+  double acc[MI][4][2];
 #pragma unroll
   for (int nj = 0; nj < 4; ++nj) {
     const int c = col0 + wc + nj * 8 + 2 * tig;
     const double b0 = c < N ? b[c] : 0.0, b1 = c + 1 < N ? b[c + 1] : 0.0;
 #pragma unroll
-    for (int mi = 0; mi < 4; ++mi) { acc[mi][nj][0] = b0; acc[mi][nj][1] = b1; }
+    for (int mi = 0; mi < MI; ++mi) { acc[mi][nj][0] = b0; acc[mi][nj][1] = b1; }
   }
-  double pa[8], pb[4];
+  constexpr int QA = TM * SCD_KT / 256;   // A elements per thread per chunk
+  double pa[QA], pb[4];
   auto load_chunk = [&](int k0) {
 #pragma unroll
-    for (int q = 0; q < 8; ++q) {
+    for (int q = 0; q < QA; ++q) {
       const int e = tid + q * 256;
       int r, kk;
-      if (in_rs == 1) { r = e & 127; kk = e >> 7; } else { kk = e & 15; r = e >> 4; }
+      if (in_rs == 1) { r = e % TM; kk = e / TM; } else { kk = e & 15; r = e >> 4; }
       const int gr = row0 + r, gk = k0 + kk;
       pa[q] = (gr < n && gk < K) ? in[static_cast<size_t>(gr) * in_rs + static_cast<size_t>(gk) * in_cs] : 0.0;
     }
@@ -479,10 +487,10 @@ __global__ void __launch_bounds__(256) score_layer_dmma_kernel(const double* __r
   };
   auto store_chunk = [&](int buf) {
 #pragma unroll
-    for (int q = 0; q < 8; ++q) {
+    for (int q = 0; q < QA; ++q) {
       const int e = tid + q * 256;
       int r, kk;
-      if (in_rs == 1) { r = e & 127; kk = e >> 7; } else { kk = e & 15; r = e >> 4; }
+      if (in_rs == 1) { r = e % TM; kk = e / TM; } else { kk = e & 15; r = e >> 4; }
       As[buf][kk][r] = pa[q];
     }
 #pragma unroll
@@ -501,13 +509,13 @@ __global__ void __launch_bounds__(256) score_layer_dmma_kernel(const double* __r
     // zero-padded K: the chunk's k beyond K are 0 in both operands, so all 4 K steps run
 #pragma unroll
     for (int k4 = 0; k4 < SCD_KT; k4 += 4) {
-      double af[4], bf[4];
+      double af[MI], bf[4];
 #pragma unroll
-      for (int mi = 0; mi < 4; ++mi) af[mi] = As[buf][k4 + tig][wr + mi * 8 + gid];
+      for (int mi = 0; mi < MI; ++mi) af[mi] = As[buf][k4 + tig][wr + mi * 8 + gid];
 #pragma unroll
       for (int nj = 0; nj < 4; ++nj) bf[nj] = Bs[buf][k4 + tig][wc + nj * 8 + gid];
 #pragma unroll
-      for (int mi = 0; mi < 4; ++mi)
+      for (int mi = 0; mi < MI; ++mi)
 #pragma unroll
         for (int nj = 0; nj < 4; ++nj)
           asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
@@ -517,7 +525,7 @@ __global__ void __launch_bounds__(256) score_layer_dmma_kernel(const double* __r
     __syncthreads();
   }
 #pragma unroll
-  for (int mi = 0; mi < 4; ++mi) {
+  for (int mi = 0; mi < MI; ++mi) {
     const int r = row0 + wr + mi * 8 + gid;
     if (r >= n) continue;
 #pragma unroll

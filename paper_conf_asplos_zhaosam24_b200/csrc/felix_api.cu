@@ -2117,11 +2117,20 @@ static void do_score(felix_space* s, felix_costmodel* m, const double* phi64, in
       const bool last = l == L - 1;
       double* out = last ? score : bufs[l & 1];
       if (N >= 32 && g_tune.score_dmma.load() != 0) {   // FP64 tensor cores, 128 x 64 tiles
-        const dim3 grid(static_cast<unsigned>((N + SCD_TN - 1) / SCD_TN), static_cast<unsigned>((n + SCD_TM - 1) / SCD_TM));
-        set_smem_attr(reinterpret_cast<const void*>(score_layer_dmma_kernel), SCD_SMEM);
-        score_layer_dmma_kernel<<<grid, 256, SCD_SMEM, st>>>(
-            in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
-            last ? 0 : 1, last && st_i > 0 ? 1 : 0);
+        const long long big_tiles = ((N + SCD_TN - 1) / SCD_TN) * ((n + scd_tm<8>() - 1) / scd_tm<8>());
+        if (big_tiles >= 2 * 148) {   // 256 x 64 tiles while they still give two per SM
+          const dim3 grid(static_cast<unsigned>((N + SCD_TN - 1) / SCD_TN), static_cast<unsigned>((n + scd_tm<8>() - 1) / scd_tm<8>()));
+          set_smem_attr(reinterpret_cast<const void*>(score_layer_dmma_kernel<8>), scd_smem<8>());
+          score_layer_dmma_kernel<8><<<grid, 256, scd_smem<8>(), st>>>(
+              in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
+              last ? 0 : 1, last && st_i > 0 ? 1 : 0);
+        } else {
+          const dim3 grid(static_cast<unsigned>((N + SCD_TN - 1) / SCD_TN), static_cast<unsigned>((n + scd_tm<4>() - 1) / scd_tm<4>()));
+          set_smem_attr(reinterpret_cast<const void*>(score_layer_dmma_kernel<4>), scd_smem<4>());
+          score_layer_dmma_kernel<4><<<grid, 256, scd_smem<4>(), st>>>(
+              in, rs, cs, static_cast<int>(n), K, m->W64[l]->as<double>(), m->b64[l]->as<double>(), out, N,
+              last ? 0 : 1, last && st_i > 0 ? 1 : 0);
+        }
       } else if (N >= 32) {   // register-blocked 128 x 64 tiles on the CUDA cores
         const dim3 grid(static_cast<unsigned>((N + SC2_TN - 1) / SC2_TN), static_cast<unsigned>((n + SC2_TM - 1) / SC2_TM));
         score_layer_v2_kernel<<<grid, 256, 0, st>>>(
