@@ -446,7 +446,7 @@ template <int MI> __host__ __device__ constexpr int scd_tm() { return 32 * MI; }
 template <int MI> __host__ __device__ constexpr int scd_ap() { return 32 * MI + 4; }
 template <int MI> __host__ __device__ constexpr int scd_smem() { return 2 * SCD_KT * (scd_ap<MI>() + SCD_BP) * 8; }   // dynamic, opt-in
 template <int MI>
-__global__ void __launch_bounds__(256, 1) score_layer_dmma_kernel(const double* __restrict__ in, long long in_rs, long long in_cs,
+__global__ void __launch_bounds__(256, MI == 4 ? 2 : 1) score_layer_dmma_kernel(const double* __restrict__ in, long long in_rs, long long in_cs,
                                                                int n, int K, const double* __restrict__ W,
                                                                const double* __restrict__ b, double* __restrict__ out,
                                                                int N, int relu, int accumulate) {
