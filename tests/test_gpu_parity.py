@@ -667,3 +667,29 @@ def test_scoring_kernels_vs_oracle(fx, name, n):
     ok = np.isfinite(ref)
     assert np.array_equal(np.isfinite(new), ok)
     assert np.all(np.abs(new[ok] - ref[ok]) <= 1e-12 * np.maximum(np.abs(ref[ok]), 1e-3))
+
+
+@pytest.mark.parametrize("history", [False, True])
+def test_multi_step_graphs_equal_single_step_graphs(fx, history):
+    """felix_search captures graph_steps Adam steps per CUDA graph (default 20) plus a tail graph: 25 steps as
+    20 + 5 give bit-for-bit the y, final loss and top-k of 25 one-step graph launches (the same kernels in
+    the same order; only the launch grouping differs)."""
+    sp, mlp, n, space, cm = _setup(fx, "C2")
+    n = 1000
+    y0 = torch.from_numpy(fi.make_y0(sp, n, seed=21)).cuda()
+    out = []
+    for gs in (-1, 1):
+        with fx.tuned(graph_steps=gs):
+            y = y0.clone()
+            loss = torch.empty(n, dtype=torch.float32, device="cuda")
+            space.search(cm, y, 25, init_from_y=True, final_loss=loss, history=history)
+            if history:
+                rec = space.history_topk(cm, 16)
+            else:
+                rec = space.round_topk(cm, y, 16)
+            torch.cuda.synchronize()
+            out.append((y.cpu().numpy(), loss.cpu().numpy(), rec))
+    (ya, la, ra), (yb, lb, rb) = out
+    assert np.array_equal(ya, yb) and np.array_equal(la, lb, equal_nan=True)
+    for a, b in zip(ra, rb):
+        assert np.array_equal(np.asarray(a), np.asarray(b))
