@@ -292,6 +292,7 @@ FELIX_EXPORT felix_status felix_init_sample(felix_space* s, int64_t n, uint64_t 
  *   "round_bnb"           0/1: 1 = every split component is rounded by the branch-and-bound kernel
  *                         (default 0: only components with more than 65536 divisor tuples are)
  *   "graph_steps"         Adam steps captured per search graph: 1..1000 (default 20)
+ *   "dphi_tma"            layer chain: the dL/dphi tile written by one TMA store (1, default) or per-thread stores (0)
  *   "score_dmma"          FP64 scoring layers on the FP64 tensor cores (1, default) or the CUDA cores (0)
  *   "pdl"                 programmatic-dependent-launch edges, bit mask: 1 forward DAG kernel, 2 MLP kernels,
  *                         4 reverse and other kernels (default 0: none, measured faster)

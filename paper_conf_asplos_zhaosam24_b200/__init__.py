@@ -160,7 +160,7 @@ def search_group(spaces: Sequence["Space"], cm: "CostModel", ys, n_steps: int, *
 
 
 _TUNE_KEYS = ("mlp", "cone_width", "replicas", "sc_warps", "chunks", "split_cone", "tile_cta_group", "chain_cta_group", "dphi_ksplit",
-              "codegen_cone_width", "codegen_replicas", "trace", "round_bnb", "graph_steps", "pdl", "score_dmma")
+              "codegen_cone_width", "codegen_replicas", "trace", "round_bnb", "graph_steps", "pdl", "score_dmma", "dphi_tma")
 _TUNE_DEFAULT = {k: (0 if k in ("trace", "round_bnb") else -1) for k in _TUNE_KEYS}
 
 

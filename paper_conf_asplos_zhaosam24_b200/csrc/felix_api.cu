@@ -132,6 +132,19 @@ static CUtensorMap make_tmap(const void* base, int64_t rows, int64_t cols, int b
   return m;
 }
 
+// fp32 [rows][cols] row-major (cols contiguous), no swizzle, box {box_cols (inner), box_rows}
+static CUtensorMap make_tmap_f32(const void* base, int64_t rows, int64_t cols, int box_cols, int box_rows) {
+  CUtensorMap m;
+  cuuint64_t dims[2] = {static_cast<cuuint64_t>(cols), static_cast<cuuint64_t>(rows)};
+  cuuint64_t strides[1] = {static_cast<cuuint64_t>(cols) * 4};
+  cuuint32_t box[2] = {static_cast<cuuint32_t>(box_cols), static_cast<cuuint32_t>(box_rows)};
+  cuuint32_t es[2] = {1, 1};
+  CU_OK(encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void*>(base), dims, strides, box, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE));
+  return m;
+}
+
 // ============================================================================ execution knobs
 // Process-wide knobs set through felix_tune (experiments and tests only; the library never reads the
 // environment).  -1 = the measured default.
@@ -150,6 +163,7 @@ struct Tuning {
   std::atomic<int> round_bnb{0};
   std::atomic<int> graph_steps{-1};  // Adam steps per search graph (-1: kGraphSteps)
   std::atomic<int> score_dmma{-1};  // FP64 scoring layers on the FP64 tensor cores (0: CUDA-core kernel; -1 = 1)
+  std::atomic<int> dphi_tma{-1};     // chain dL/dphi epilogue: one TMA store per tile (1, default) or per-thread stores (0)
   std::atomic<int> pdl{-1};          // PDL edges: bit 0 forward, 1 MLP kernels, 2 reverse / other (-1: none)     // 1: every split component rounds by branch and bound (test hook)
 };
 static Tuning g_tune;
@@ -843,6 +857,12 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     if (bn > CHAIN_BN_MAX) FELIX_THROW(FELIX_E_UNSUPPORTED, "chain tile N > 128");
     L.bn = bn;
     L.n_tiles_n = N / bn;
+    L.f32t_tma = 0;
+    if (g.epi == EPI_F32T && bn <= CHAIN_BN_MAX && g_tune.dphi_tma.load() != 0) {
+      // the dL/dphi slabs [ksplit * N][n_pad] fp32 through one TMA store per tile (mlp_chain.cuh)
+      L.c_f32 = make_tmap_f32(g.args.out_f32, static_cast<int64_t>(L.ksplit) * N, g.args.ld_f32, GEMM_BM, bn);
+      L.f32t_tma = 1;
+    }
     L.n_tiles = static_cast<int>(mt) * L.n_tiles_n;
     const int ccg = p->chain_cg;
     L.idesc = ptx::idesc_f16_f32(GEMM_BM * ccg, static_cast<uint32_t>(bn));
@@ -2339,6 +2359,7 @@ felix_status felix_tune(const char* key, int32_t value) {
   else if (k == "trace") { in({0, 1}); g_tune.trace = value; }
   else if (k == "round_bnb") { in({0, 1}); g_tune.round_bnb = value; }
   else if (k == "score_dmma") { in({-1, 0, 1}); g_tune.score_dmma = value; }
+  else if (k == "dphi_tma") { in({-1, 0, 1}); g_tune.dphi_tma = value; }
   else if (k == "pdl") { if (value != -1 && (value < 0 || value > 7)) in({}); g_tune.pdl = value; }
   else if (k == "graph_steps") { if (value != -1 && (value < 1 || value > 1000)) in({}); g_tune.graph_steps = value; }
   else FELIX_THROW(FELIX_E_INVALID_ARG, "felix_tune: unknown key " + k);

@@ -75,6 +75,11 @@ constexpr int CHAIN_SMEM_BYTES = 1024 + CHAIN_STAGES * CHAIN_STAGE_BYTES + CHAIN
 
 struct ChainLayer {
   CUtensorMap a_hi, a_lo, b_hi, b_lo, c_hi, c_lo;
+  // EPI_F32T: fp32 dL/dphi slabs as one 2-D map [ksplit * N rows (slab-major)][ld_f32 candidates], box
+  // {128 candidates, bn features}: the tile is staged transposed in shared memory and written by one TMA
+  // store (f32t_tma = 1; else per-thread stores)
+  CUtensorMap c_f32;
+  int f32t_tma;
   GemmArgs args;
   int epi, bn, n_tiles_n, n_tiles;     // tiles = m_tiles * n_tiles_n (n fastest)
   uint32_t idesc;
@@ -482,7 +487,27 @@ __global__ void __launch_bounds__(CHAIN_THREADS, 1) mlp_chain_kernel(const __gri
         ptx::tc_fence_after();
         const uint32_t t_row = tmem_base + acc * ACC + (static_cast<uint32_t>(q * 32) << 16);
         float head_acc = 0.f;
-        if (epi == EPI_F32T) {
+        if (epi == EPI_F32T && L.f32t_tma) {
+          // stage [bn features][128 rows] fp32 (48 KB at bn = 96, in the epilogue staging buffers: the last
+          // layer, nothing reuses them), then one TMA store of the tile into slab `part`
+          float* stg = reinterpret_cast<float*>(epi_base);
+          if (etid == 0) ptx::bulk_wait_read<0>();          // a previous tile's store has read the staging
+          ptx::named_bar_sync(1, NEPI);
+          for (int c = cs; c < bn; c += 64) {
+            float v[CPW];
+            acc_cols(t_row, c, bn, v);
+#pragma unroll
+            for (int i = 0; i < CPW; ++i)
+              if (c + i < bn) stg[(c + i) * GEMM_BM + r_tile] = v[i];
+          }
+          ptx::fence_proxy_async_smem();
+          ptx::named_bar_sync(1, NEPI);
+          if (etid == 0) {
+            asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];"
+                         :: "l"(reinterpret_cast<uint64_t>(&L.c_f32)), "r"(m0), "r"(part * aN + n0), "r"(ptx::smem_u32(stg)) : "memory");
+            ptx::bulk_commit();
+          }
+        } else if (epi == EPI_F32T) {
           for (int c = cs; c < bn; c += 64) {
             float v[CPW];
             acc_cols(t_row, c, bn, v);

@@ -42,6 +42,14 @@ int main(int argc, char** argv) {
   // production settings at C2 (felix_api.cu build_plan): exact-mask first backward layer, split-K dL/dphi
   P.layer[2].head_exact = 1; P.layer[3].a_exact = 1;
   P.layer[5].ksplit = argc > 8 ? atoi(argv[8]) : 4;
+  {
+    const int f32tma = argc > 9 ? atoi(argv[9]) : 1;
+    CUtensorMap m; cuuint64_t d[2] = {(cuuint64_t)M, (cuuint64_t)(P.layer[5].ksplit * 96)}; cuuint64_t st[1] = {(cuuint64_t)M * 4};
+    cuuint32_t b[2] = {128, (cuuint32_t)P.layer[5].bn}; cuuint32_t e[2] = {1, 1};
+    cuTensorMapEncodeTiled(&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, dphi, d, st, b, e, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                           CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    P.layer[5].c_f32 = m; P.layer[5].f32t_tma = f32tma;
+  }
   P.n_layers = 6; P.m_tiles = mt;
   P.grid_bar = (unsigned int*)dz(64);
   int grid = std::min(148, mt * 512 / bnA);
