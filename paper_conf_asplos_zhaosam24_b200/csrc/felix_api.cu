@@ -941,6 +941,8 @@ static std::unique_ptr<Plan> build_plan_rows(int device, const CostModel* cm, in
     t.c_part = p->c_part.as<float>();
     t.dphi = p->dphi.as<float>();
     t.ld = static_cast<int>(np);
+    t.dphi_tma = g_tune.dphi_tma.load() != 0 ? 1 : 0;
+    if (t.dphi_tma) t.dphi_map = make_tmap_f32(p->dphi.p, K0p, np, 128, K0p);
     t.n = static_cast<int>(n);
     t.n_tiles = static_cast<int>(mt);
     t.k0p = K0p;

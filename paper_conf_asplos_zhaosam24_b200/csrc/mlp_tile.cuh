@@ -65,6 +65,8 @@ struct TileParams {
   const float* w4;
   float* c_part;                       // [2][ld] head partials (one per column half)
   float* dphi;                         // [K0p][ld]
+  CUtensorMap dphi_map;                // fp32 [K0p][ld], box {128 rows, K0p}: B4 as one TMA store per tile
+  int dphi_tma;                        // 1: B4 staged in shared memory + TMA store; 0: per-thread stores
   int ld;
   int n;                               // rows (candidates)
   int n_tiles;                         // 128-row tiles
@@ -403,6 +405,11 @@ __global__ void __launch_bounds__(tile::THREADS, 1) mlp_tile_kernel(const __grid
       const int m0 = (unit * CG + static_cast<int>(rank)) * 128;
       const int row = m0 + r;
       const bool row_ok = row < P.n;
+      if (t > 0 && P.dphi_tma) {
+        // the previous tile's dL/dphi store has read its staging (the H buffers written again below)
+        if (warp == 2 && lane == 0) ptx::bulk_wait_read<0>();
+        ptx::named_bar_sync(1, EPI_WARPS * 32);
+      }
       uint32_t m1w[D1 / 64], m2w[D2 / 64], m3w[D3 / 64];
       float head = 0.f;
       // ---- F1: drain Z1_c (128 columns) -> H1 chunks 2c, 2c+1
@@ -517,18 +524,40 @@ __global__ void __launch_bounds__(tile::THREADS, 1) mlp_tile_kernel(const __grid
       wait_k<1>(dphi_full, t);
       if (warp == 2 && lane == 0) TILE_STAMP(26);
       ptx::tc_fence_after();
-      for (int c = h * 32; c < P.k0p; c += 64) {
-        float v[32];
-        tile::tmem_ld32(tmem + lane_base + T_DPHI + c, v);
-        if (row_ok) {
+      if (P.dphi_tma) {
+        // staged [K0p][128 rows] fp32 in the H buffers (free here: every MMA reading them has completed
+        // before dphi_full) and written by one TMA store (per-thread fp32 stores took ~2.4 us per tile)
+        float* stg = reinterpret_cast<float*>(R0 + 2 * CHUNK_BYTES);
+        for (int c = h * 32; c < P.k0p; c += 64) {
+          float v[32];
+          tile::tmem_ld32(tmem + lane_base + T_DPHI + c, v);
 #pragma unroll
           for (int i = 0; i < 32; ++i)
-            if (c + i < P.n_valid) P.dphi[static_cast<size_t>(c + i) * P.ld + row] = v[i];
+            if (c + i < P.k0p) stg[(c + i) * 128 + r] = v[i];
         }
+        ptx::tc_fence_before();
+        ptx::fence_proxy_async_smem();
+        ptx::named_bar_sync(1, EPI_WARPS * 32);
+        if (warp == 2 && lane == 0) {
+          asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];"
+                       :: "l"(reinterpret_cast<uint64_t>(&P.dphi_map)), "r"(m0), "r"(0), "r"(ptx::smem_u32(stg)) : "memory");
+          ptx::bulk_commit();
+        }
+      } else {
+        for (int c = h * 32; c < P.k0p; c += 64) {
+          float v[32];
+          tile::tmem_ld32(tmem + lane_base + T_DPHI + c, v);
+          if (row_ok) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i)
+              if (c + i < P.n_valid) P.dphi[static_cast<size_t>(c + i) * P.ld + row] = v[i];
+          }
+        }
+        ptx::tc_fence_before();
       }
-      ptx::tc_fence_before();
       if (warp == 2 && lane == 0) TILE_STAMP(27);
     }
+    if (warp == 2 && lane == 0) ptx::bulk_wait<0>();   // the last dL/dphi store complete before exit
   }
   ptx::tc_fence_before();
   if constexpr (CG == 2) ptx::cluster_sync();
