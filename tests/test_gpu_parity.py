@@ -693,3 +693,19 @@ def test_multi_step_graphs_equal_single_step_graphs(fx, history):
     assert np.array_equal(ya, yb) and np.array_equal(la, lb, equal_nan=True)
     for a, b in zip(ra, rb):
         assert np.array_equal(np.asarray(a), np.asarray(b))
+
+
+@pytest.mark.parametrize("n,ksplit", [(5120, -1), (4096, 2), (4096, 1)])
+def test_chain_dphi_layer_variants_search_path_gradient(fx, n, ksplit):
+    """The chain's dL/dphi layer in its other shapes -- 32-wide N tiles without split-K (n = 5120: 40 row
+    blocks), split-K 2 and no split at 4096 -- all written by the staged TMA store: the search path's dL/dy
+    against the oracle (normwise 1e-3 per candidate, R-kink exemption < 1 %)."""
+    sp, mlp, _, space, cm = _setup(fx, "C2")
+    y0 = fi.make_y0(sp, n, seed=5)
+    with fx.tuned(mlp="chain", dphi_ksplit=ksplit):
+        out = space.eval_search_path(cm, torch.from_numpy(y0).cuda())
+        torch.cuda.synchronize()
+    ref = fo.objective(sp, mlp.W, mlp.b, y0.astype(np.float64), 1.0)
+    g = out["grad"].cpu().numpy()
+    err = np.linalg.norm(g - ref.grad, axis=0) / np.maximum(np.linalg.norm(ref.grad, axis=0), 1e-12)
+    assert np.mean(err > 1e-3) < 0.01
